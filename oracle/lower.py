@@ -1,0 +1,221 @@
+"""ORACLE — test infrastructure only (tests/, __graft_entry__.smoke(), bench.py cpu_baseline).
+
+Plain-Python lowering of CUDA / CUDA-aware-MPI calls to happens-before primitives (method step a0),
+written directly from the paper's CuSan runtime description and SURVEY.md §8(b)'s table.  It shares no
+code with the product library (``paper_conf_sc_huckzsjb24_b200/csrc/lower.cpp``).
+
+Fibers (§IV-A(a)): 0 = host thread H, 1 = legacy default stream S0 (always
+tracked), user streams in creation order, then MPI-request fibers from a pool.
+Sync keys: K(stream fiber f) = 1<<56 | f, K(event e) = 2<<56 | e, K(request r) = 3<<56 | r.
+"""
+from __future__ import annotations
+
+import bisect
+
+import numpy as np
+
+from tracegen.program import (ARG_DTYPE, CPY_D2H, CPY_H2D, CPY_H2H, EVENT_DTYPE, EV_ACCESS, EV_ACQUIRE,
+                              EV_FORK, EV_RELEASE, EV_RELEASE_STORE, MEM_PINNED, MODE_R, OP_DEVICE_SYNC,
+                              OP_DTYPE, OP_EVENT_RECORD, OP_EVENT_SYNC, OP_FREE, OP_HOST_ACCESS, OP_KERNEL,
+                              OP_MALLOC, OP_MEMCPY, OP_MEMCPY_ASYNC, OP_MEMSET, OP_MEMSET_ASYNC,
+                              OP_MPI_IRECV, OP_MPI_ISEND, OP_MPI_RECV, OP_MPI_SEND, OP_MPI_TEST,
+                              OP_MPI_WAIT, OP_STREAM_CREATE, OP_STREAM_QUERY, OP_STREAM_SYNC,
+                              OP_STREAM_WAIT_EVENT, READ, STREAM_NONBLOCKING, WRITE)
+
+H, S0 = 0, 1
+
+
+def K_stream(f):
+    return (1 << 56) | f
+
+
+def K_event(e):
+    return (2 << 56) | e
+
+
+def K_req(r):
+    return (3 << 56) | r
+
+
+class Lowering:
+    """CuSan per-device context: stream → fiber table with a non-blocking flag,
+    event handles, memory-attribute table (allocation registry), host
+    fiber, plus MUST's request → fiber map."""
+
+    def __init__(self):
+        self.ev: list[tuple] = []            # (kind, fiber, a, b, mode)
+        self.stream_fiber = {0: S0}
+        self.blocking_user: list[int] = []   # fibers of blocking user streams, creation order
+        self.all_streams: list[int] = [S0]   # S0 then user streams, creation order
+        self.next_fiber = 2
+        self.free_mpi: list[int] = []        # pool of returned MPI fibers
+        self.req_fiber: dict[int, int] = {}
+        self.alloc_base: list[int] = []      # sorted bases
+        self.alloc: dict[int, tuple[int, int]] = {}   # base -> (size, kind)
+
+    # -- primitives (TSan API) ---------------------------------------------
+    def access(self, f, mode, addr, n):
+        self.ev.append((EV_ACCESS, f, addr, n, mode))
+
+    def release(self, f, key):
+        self.ev.append((EV_RELEASE, f, key, 0, 0))
+
+    def release_store(self, f, key):
+        self.ev.append((EV_RELEASE_STORE, f, key, 0, 0))
+
+    def acquire(self, f, key):
+        self.ev.append((EV_ACQUIRE, f, key, 0, 0))
+
+    def fork(self, src, dst):
+        self.ev.append((EV_FORK, dst, src, 0, 0))
+
+    # -- helpers -------------------------------------------------------------------------------
+    def find_alloc(self, p):
+        """Allocation containing pointer p (TypeART extent lookup)."""
+        i = bisect.bisect_right(self.alloc_base, p) - 1
+        if i < 0:
+            return None
+        base = self.alloc_base[i]
+        size, kind = self.alloc[base]
+        if base <= p < base + size:
+            return base, size, kind
+        return None
+
+    def prologue(self, f):
+        """Issue edge H → stream and the legacy default-stream barriers (Fig. 3,
+        PAPER.md:356-364)."""
+        self.fork(H, f)
+        if f in self.blocking_user:
+            self.acquire(f, K_stream(S0))
+        if f == S0:
+            for u in self.blocking_user:
+                self.acquire(S0, K_stream(u))
+
+    def epilogue(self, f):
+        """AnnotateHappensBefore on the stream after each operation."""
+        self.release(f, K_stream(f))
+
+    def sync_stream_host(self, f):
+        """cudaStreamSynchronize; on S0 it also covers every blocking
+        stream."""
+        self.acquire(H, K_stream(f))
+        if f == S0:
+            for u in self.blocking_user:
+                self.acquire(H, K_stream(u))
+
+    def sync_device_host(self):
+        """cudaDeviceSynchronize: acquire on every stream."""
+        for f in self.all_streams:
+            self.acquire(H, K_stream(f))
+
+    def tracked_range(self, p, n):
+        return n > 0 and self.find_alloc(p) is not None
+
+    # -- one API call --------------------------------------------------------------------------
+    def call(self, op, args):
+        kind = int(op["op"])
+        x, a, b, c, s = int(op["x"]), int(op["a"]), int(op["b"]), int(op["c"]), int(op["s"])
+        if kind == OP_MALLOC:
+            bisect.insort(self.alloc_base, a)
+            self.alloc[a] = (b, x)
+        elif kind == OP_FREE:
+            self.sync_device_host()
+        elif kind == OP_STREAM_CREATE:
+            f = self.next_fiber
+            self.next_fiber += 1
+            self.stream_fiber[s] = f
+            self.all_streams.append(f)
+            if not (x & STREAM_NONBLOCKING):
+                self.blocking_user.append(f)
+        elif kind == OP_KERNEL:
+            f = self.stream_fiber[s]
+            self.prologue(f)
+            for j in range(b, b + x):
+                al = self.find_alloc(int(args[j]["ptr"]))
+                if al is None:
+                    continue
+                mode = READ if int(args[j]["mode"]) == MODE_R else WRITE   # RW → WRITE (A10)
+                self.access(f, mode, al[0], al[1])         # whole allocation
+            self.epilogue(f)
+        elif kind in (OP_STREAM_SYNC,):
+            self.sync_stream_host(self.stream_fiber[s])
+        elif kind == OP_STREAM_QUERY:
+            if x:                                          # only a successful query syncs (A9)
+                self.sync_stream_host(self.stream_fiber[s])
+        elif kind == OP_DEVICE_SYNC:
+            self.sync_device_host()
+        elif kind == OP_EVENT_RECORD:
+            f = self.stream_fiber[s]
+            self.prologue(f)
+            self.release_store(f, K_event(c))             # re-record replaces the capture (A4)
+        elif kind == OP_EVENT_SYNC:
+            self.acquire(H, K_event(c))
+        elif kind == OP_STREAM_WAIT_EVENT:
+            f = self.stream_fiber[s]
+            self.prologue(f)
+            self.acquire(f, K_event(c))
+        elif kind in (OP_MEMCPY, OP_MEMCPY_ASYNC):
+            f = S0 if kind == OP_MEMCPY else self.stream_fiber[s]
+            self.prologue(f)
+            if self.tracked_range(a, c):
+                self.access(f, WRITE, a, c)
+            if self.tracked_range(b, c):
+                self.access(f, READ, b, c)
+            self.epilogue(f)
+            if kind == OP_MEMCPY and x in (CPY_H2H, CPY_H2D, CPY_D2H):   # PAPER.md:433-436 (A6)
+                self.acquire(H, K_stream(S0))
+        elif kind in (OP_MEMSET, OP_MEMSET_ASYNC):
+            f = S0 if kind == OP_MEMSET else self.stream_fiber[s]
+            self.prologue(f)
+            al = self.find_alloc(a)
+            if self.tracked_range(a, c):
+                self.access(f, WRITE, a, c)
+            self.epilogue(f)
+            if kind == OP_MEMSET and al is not None and al[2] == MEM_PINNED:  # PAPER.md:463-466 (A7)
+                self.acquire(H, K_stream(S0))
+        elif kind == OP_HOST_ACCESS:
+            self.access(H, WRITE if x else READ, a, c)
+        elif kind in (OP_MPI_ISEND, OP_MPI_IRECV):
+            if self.free_mpi:
+                m = min(self.free_mpi)
+                self.free_mpi.remove(m)
+            else:
+                m = self.next_fiber
+                self.next_fiber += 1
+            self.req_fiber[b] = m
+            self.fork(H, m)
+            self.access(m, READ if kind == OP_MPI_ISEND else WRITE, a, c)
+            self.release(m, K_req(b))
+        elif kind in (OP_MPI_WAIT, OP_MPI_TEST):
+            if kind == OP_MPI_WAIT or x:
+                self.acquire(H, K_req(b))
+                m = self.req_fiber.pop(b, None)
+                if m is not None:
+                    self.free_mpi.append(m)
+        elif kind == OP_MPI_SEND:
+            self.access(H, READ, a, c)
+        elif kind == OP_MPI_RECV:
+            self.access(H, WRITE, a, c)
+        else:
+            raise ValueError(f"unknown op {kind}")
+
+    def events(self) -> np.ndarray:
+        out = np.zeros(len(self.ev), EVENT_DTYPE)
+        if self.ev:
+            arr = np.array(self.ev, dtype=object)
+            out["kind"] = arr[:, 0].astype(np.uint8)
+            out["fiber"] = arr[:, 1].astype(np.uint32)
+            out["a"] = np.array([int(v) for v in arr[:, 2]], dtype=np.uint64)
+            out["b"] = np.array([int(v) for v in arr[:, 3]], dtype=np.uint64)
+            out["mode"] = arr[:, 4].astype(np.uint8)
+        return out
+
+
+def lower(ops: np.ndarray, args: np.ndarray) -> tuple[np.ndarray, int]:
+    """API program → (primitive events, number of fibers used)."""
+    L = Lowering()
+    ops = np.asarray(ops, OP_DTYPE)
+    args = np.asarray(args, ARG_DTYPE)
+    for op in ops:
+        L.call(op, args)
+    return L.events(), L.next_fiber

@@ -1,0 +1,293 @@
+"""Pins for the oracle (oracle/): paper listings, brute-force graph HB, invariants, closed forms.
+
+None of these compare the oracle with itself: expected values come from the paper's stated
+classifications (tests/golden/listings.txt), from an explicit-graph transitive closure (tests/brute.py)
+or from the mathematics of the definitions (subset / emptiness / relabelling / sync insertion).
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import oracle
+from oracle.lower import Lowering, lower
+from tracegen import configs, fuzz
+from tracegen.program import (EVENT_DTYPE, EV_ACCESS, EV_ACQUIRE, EV_FORK, EV_RELEASE, OP_DTYPE,
+                              OP_KERNEL, OP_MEMCPY, OP_MEMCPY_ASYNC, OP_MEMSET, OP_MEMSET_ASYNC)
+
+import brute
+import listing_dsl
+
+
+def oracle_lower_with_offsets(ops, args):
+    L = Lowering()
+    first = []
+    for op in np.asarray(ops, OP_DTYPE):
+        first.append(len(L.ev))
+        L.call(op, args)
+    return L.events(), L.next_fiber, first
+
+
+# ------------------------------------------------------------------------------------------------
+# paper listings (racy / fixed pairs with the paper's classification)
+# ------------------------------------------------------------------------------------------------
+LISTINGS = listing_dsl.parse()
+
+
+@pytest.mark.parametrize("lst", LISTINGS, ids=[l.name for l in LISTINGS])
+def test_listing_classification(lst):
+    ops, args = lst.program.arrays()
+    ev, nf, first = oracle_lower_with_offsets(ops, args)
+    rep = oracle.check_events(ev, nf, threads=1)
+    labels = listing_dsl.label_events(lst, ev, first)
+    got = listing_dsl.observed_pairs(rep["runs"], labels)
+    want = {(a, b): n for a, b, n in lst.expect}
+    assert set(got) == set(want), (lst.name, got, want)
+    for k, n in want.items():
+        if n is not None:
+            assert got[k] == n, (lst.name, k, got[k], n)
+    # and the brute-force graph checker agrees on the full triple set
+    assert brute.runs_to_triples(rep["runs"]) == brute.per_fiber_race_set(ev)
+
+
+def test_listing_pairs_are_paired():
+    names = {l.name for l in LISTINGS}
+    for n in names:
+        if n.endswith("_racy"):
+            assert n[:-5] + "_fixed" in names
+
+
+# ------------------------------------------------------------------------------------------------
+# brute force on tiny random traces
+# ------------------------------------------------------------------------------------------------
+def _fuzz_cases(n, seed, **kw):
+    rng = np.random.default_rng(seed)
+    for _ in range(n):
+        ne = int(rng.integers(2, 64))
+        nf = int(rng.integers(2, 6))
+        yield fuzz.random_primitive_trace(rng, ne, nf, n_keys=int(rng.integers(1, 4)),
+                                          n_granules=int(rng.integers(1, 17)), **kw), nf
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_oracle_equals_graph_hb_bruteforce(seed):
+    """RS(oracle, vector clocks) == RS(per-fiber definition over explicit-graph HB)."""
+    for ev, nf in _fuzz_cases(60, 100 + seed, unaligned=bool(seed % 2)):
+        rep = oracle.check_events(ev, nf, threads=1 + seed % 3)
+        got = brute.runs_to_triples(rep["runs"])
+        reach = brute.hb_closure(ev)
+        want = brute.per_fiber_race_set(ev, reach)
+        assert got == want
+        assert rep["n_race_granules"] == len(want)
+        allp = brute.all_pairs_race_set(ev, reach)
+        assert got <= allp                                    # RS ⊆ all racy pairs
+        for g in {t[0] for t in allp} | {t[0] for t in got}:  # per-granule emptiness equivalence
+            assert any(t[0] == g for t in got) == any(t[0] == g for t in allp)
+            first_later = min(t[2] for t in allp if t[0] == g)  # first racy access is reported
+            assert any(t[0] == g and t[2] == first_later for t in got)
+
+
+def test_runs_are_canonical_and_roundtrip():
+    for ev, nf in _fuzz_cases(80, 7):
+        rep = oracle.check_events(ev, nf, threads=2)
+        runs = rep["runs"]
+        keys = [(int(r["later"]), int(r["earlier"]), int(r["g_begin"])) for r in runs]
+        assert keys == sorted(keys) and len(set(keys)) == len(keys)
+        assert rep["n_race_granules"] == int(np.sum(runs["g_end"] - runs["g_begin"]))
+        # maximality: no two runs with equal (earlier, later) abut
+        for a, b in zip(runs[:-1], runs[1:]):
+            if a["later"] == b["later"] and a["earlier"] == b["earlier"]:
+                assert a["g_end"] < b["g_begin"]
+        # round trip: expand → re-merge gives the same runs
+        trip = sorted(brute.runs_to_triples(runs), key=lambda t: (t[2], t[1], t[0]))
+        merged = []
+        for g, e, l in trip:
+            if merged and merged[-1][2] == e and merged[-1][3] == l and merged[-1][1] == g:
+                merged[-1][1] += 1
+            else:
+                merged.append([g, g + 1, e, l])
+        assert merged == [[int(r["g_begin"]), int(r["g_end"]), int(r["earlier"]), int(r["later"])]
+                          for r in runs]
+
+
+# ------------------------------------------------------------------------------------------------
+# invariants
+# ------------------------------------------------------------------------------------------------
+def test_fully_synchronised_programs_are_race_free():
+    """DeviceSynchronize + completion of every request after each call orders everything."""
+    rng = np.random.default_rng(11)
+    for _ in range(40):
+        p = fuzz.random_program(rng, int(rng.integers(5, 40)))
+        ops, args = p.arrays()
+        from tracegen.program import Program, OP_MPI_ISEND, OP_MPI_IRECV, OP_MPI_WAIT, OP_MPI_TEST
+        q = Program()
+        q.args = p.args
+        waited = set()
+        for op in ops:
+            if int(op["op"]) in (OP_MPI_WAIT, OP_MPI_TEST) and int(op["b"]) in waited:
+                continue
+            q.ops.append(tuple(int(v) for v in op))
+            if int(op["op"]) in (OP_MPI_ISEND, OP_MPI_IRECV):
+                q.wait(int(op["b"]))
+                waited.add(int(op["b"]))
+            q.device_sync()
+        o2, a2 = q.arrays()
+        rep = oracle.check_program(o2, a2, threads=1)
+        assert rep["n_race_granules"] == 0 and rep["n_runs"] == 0
+
+
+def _insert(ev, pos, rows):
+    rows = np.array(rows, EVENT_DTYPE)
+    return np.concatenate([ev[:pos], rows, ev[pos:]])
+
+
+def test_sync_insertion_removes_exactly_newly_ordered_candidates():
+    rng = np.random.default_rng(5)
+    checked = 0
+    for ev, nf in _fuzz_cases(150, 23):
+        n = len(ev)
+        p = int(rng.integers(0, n + 1))
+        q = int(rng.integers(p, n + 1))
+        f1, f2 = int(rng.integers(nf)), int(rng.integers(nf))
+        key = 999_999
+        # RELEASE at p, ACQUIRE at q (after the shift): ids ≥ p shift by 1, ids ≥ q (orig) by 2
+        ev2 = _insert(ev, q, [(EV_ACQUIRE, 0, 0, f2, key, 0)])
+        ev2 = _insert(ev2, p, [(EV_RELEASE, 0, 0, f1, key, 0)])
+
+        def remap(i):
+            return i + (1 if i >= p else 0) + (1 if i >= q else 0)
+
+        r1 = brute.runs_to_triples(oracle.check_events(ev, nf, threads=1)["runs"])
+        r2 = brute.runs_to_triples(oracle.check_events(ev2, nf, threads=1)["runs"])
+        r1m = {(g, remap(a), remap(b)) for g, a, b in r1}
+        assert r2 <= r1m
+        reach2 = brute.hb_closure(ev2)
+        for g, a, b in r1m - r2:
+            assert (reach2[a] >> b) & 1          # removed ⇒ newly ordered
+        for g, a, b in r2:
+            assert not (reach2[a] >> b) & 1      # kept ⇒ still unordered
+        checked += len(r1m - r2)
+    assert checked > 0
+
+
+def test_fiber_relabelling_invariance():
+    rng = np.random.default_rng(9)
+    for ev, nf in _fuzz_cases(40, 31):
+        perm = rng.permutation(nf)
+        ev2 = ev.copy()
+        ev2["fiber"] = perm[ev["fiber"]]
+        fork = ev["kind"] == EV_FORK
+        ev2["a"][fork] = perm[ev["a"][fork].astype(np.int64)]
+        r1 = oracle.check_events(ev, nf, threads=1)
+        r2 = oracle.check_events(ev2, nf, threads=1)
+        assert np.array_equal(r1["runs"], r2["runs"])
+
+
+def test_thread_count_invariance_and_sampling():
+    w = configs.make(5, "small")
+    ops, args = w.arrays(True)
+    ev, nf = lower(ops, args)
+    r1 = oracle.check_events(ev, nf, threads=1)
+    r8 = oracle.check_events(ev, nf, threads=8)
+    assert np.array_equal(r1["runs"], r8["runs"]) and r1["n_race_granules"] == r8["n_race_granules"]
+    # sampled granules give exactly the full result restricted to the sample
+    full = brute.runs_to_triples(r1["runs"])
+    gs = sorted({g for g, _, _ in full})
+    rng = np.random.default_rng(0)
+    acc = ev[ev["kind"] == EV_ACCESS]
+    lo, hi = int(acc["a"].min()) >> 3, (int((acc["a"] + acc["b"]).max()) + 7) >> 3
+    sample = np.unique(np.concatenate([rng.choice(gs, 200), rng.integers(lo, hi, 200)]).astype(np.uint64))
+    rs = oracle.check_events(ev, nf, threads=3, sample=sample)
+    sset = set(int(x) for x in sample)
+    assert brute.runs_to_triples(rs["runs"]) == {t for t in full if t[0] in sset}
+
+
+# ------------------------------------------------------------------------------------------------
+# closed forms and the paper's counters
+# ------------------------------------------------------------------------------------------------
+def test_config1_closed_form():
+    """Racy listing: exactly one run over the 4 KiB buffer (512 granules), earlier = the compute
+    kernel's RW access, later = the MPI_Isend read; the fixed twin is race-free."""
+    w = configs.make(1)
+    ops, args = w.arrays(True)
+    ev, nf, first = oracle_lower_with_offsets(ops, args)
+    rep = oracle.check_events(ev, nf)
+    assert len(ev) == 14
+    assert rep["n_runs"] == 1 and rep["n_race_granules"] == 512
+    r = rep["runs"][0]
+    d = w.meta["buffer"]
+    assert int(r["g_begin"]) == d >> 3 and int(r["g_end"]) == (d + 4096) >> 3
+    e, l = ev[int(r["earlier"])], ev[int(r["later"])]
+    assert (int(e["kind"]), int(e["mode"]), int(e["fiber"])) == (EV_ACCESS, 1, 2)   # kernel on s
+    assert (int(l["kind"]), int(l["mode"]), int(l["fiber"])) == (EV_ACCESS, 0, 3)   # MPI fiber
+    ops, args = w.arrays(False)
+    ev, nf = lower(ops, args)
+    assert len(ev) == 15
+    assert oracle.check_events(ev, nf)["n_race_granules"] == 0
+
+
+def test_table1_release_identity():
+    """Table I: HappensBefore = kernels + memcpys + memsets (1200+602+2=1804);
+    our lowering emits exactly one stream-key release per kernel / memcpy / memset."""
+    for c in (2, 3):
+        w = configs.make(c, "small")
+        ops, args = w.arrays(False)
+        ev, _ = lower(ops, args)
+        n_ops = int(np.isin(ops["op"], [OP_KERNEL, OP_MEMCPY, OP_MEMCPY_ASYNC, OP_MEMSET,
+                                        OP_MEMSET_ASYNC]).sum())
+        stream_rel = int(((ev["kind"] == EV_RELEASE) & ((ev["a"] >> np.uint64(56)) == 1)).sum())
+        assert stream_rel == n_ops
+
+
+@pytest.mark.parametrize("c", [2, 3, 4, 5])
+def test_small_configs_clean_and_racy(c):
+    w = configs.make(c, "small")
+    ops, args = w.arrays(False)
+    rep = oracle.check_program(ops, args)
+    assert rep["n_race_granules"] == 0
+    acc = rep["events"][rep["events"]["kind"] == EV_ACCESS]
+    assert rep["tracked_bytes"] == int(np.sum(((acc["a"] + acc["b"] + np.uint64(7)) >> np.uint64(3))
+                                              - (acc["a"] >> np.uint64(3)))) * 8
+    ops, args = w.arrays(True)
+    rep = oracle.check_program(ops, args)
+    assert rep["n_race_granules"] > 0
+
+
+def _listing_failures(mutate):
+    """Number of listings whose paper classification a mutated lowering gets wrong."""
+    bad = 0
+    for lst in LISTINGS:
+        ops, args = lst.program.arrays()
+        L = Lowering()
+        mutate(L)
+        first = []
+        for op in np.asarray(ops, OP_DTYPE):
+            first.append(len(L.ev))
+            L.call(op, args)
+        ev = L.events()
+        rep = oracle.check_events(ev, L.next_fiber, threads=1)
+        got = set(listing_dsl.observed_pairs(rep["runs"], listing_dsl.label_events(lst, ev, first)))
+        bad += got != {(a, b) for a, b, _ in lst.expect}
+    return bad
+
+
+def test_listings_reject_counterfactual_readings():
+    """without the issue edge (FORK H→stream), or with a stream→host edge on return,
+    or without the legacy default-stream barriers, some paper listing is misclassified."""
+    def no_fork(L):
+        L.fork = lambda src, dst: None
+
+    def back_edge(L):
+        orig = L.epilogue
+
+        def epi(f):
+            orig(f)
+            L.acquire(0, (1 << 56) | f)
+        L.epilogue = epi
+
+    def no_legacy(L):
+        L.prologue = lambda f: L.fork(0, f)
+
+    assert _listing_failures(no_fork) > 0
+    assert _listing_failures(back_edge) > 0
+    assert _listing_failures(no_legacy) > 0
