@@ -1,0 +1,364 @@
+#!/usr/bin/env python
+"""bench.py — race-checked GB/s of the B200 happens-before race check (DESIGN.md §"Measurement").
+
+One step = one pass of the whole hot path over the workload: the shadow-check kernels (a3) with
+in-warp run compaction (a4), the run download, the canonical merge and the report (a5), with the
+event / clock / interval tables (a1, a2) already resident in HBM.  `e2e` repeats the metric
+through the public C ABI from host buffers: lowering of the recorded CUDA/MPI call program (a0),
+planning (a1, a2), table upload, check and report, every step.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+    torchrun --nproc-per-node N bench.py --gpus N ...      (one rank per GPU, shards by granule range)
+
+Workload: BASELINE.json config 5 (scaling sweep: 64 GiB of log-uniform allocations, 64 fibers,
+~100k primitive events; the largest trace, the one the metric is quoted on at 1/2/4/8 GPUs), racy
+twin, online (windowed) mode: the shadow lives in HBM between windows of 4096 accesses.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "tracked bytes checked/sec (race-checked GB/s) at 1/2/4/8 B200 vs HBM peak"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", type=int, default=5)
+    ap.add_argument("--size", default="full", choices=["full", "small"])
+    ap.add_argument("--window", type=int, default=4096, help="access events per shadow window")
+    ap.add_argument("--clean", action="store_true", help="race-free twin instead of the racy twin")
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle sample time")
+    return ap.parse_args()
+
+
+def measured_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+def ncu_traffic():
+    """dram read+write bytes per launch of the shadow-check kernel from the committed ncu capture."""
+    p = os.path.join(ROOT, "profiles", "ncu_k1_summary.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get("dram_bytes_per_launch"), d
+    except Exception:
+        return None, None
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+
+    def __init__(self, index: int):
+        self.f = tempfile.NamedTemporaryFile("w+", suffix=".csv", delete=False)
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                       "-lms", "200", "-i", str(index)], stdout=self.f, stderr=subprocess.DEVNULL)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        self.p.wait()
+        self.f.seek(0)
+        sm, smax, reasons = [], [], set()
+        for line in self.f:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                smax.append(float(parts[2]))
+            except ValueError:
+                continue
+            for name, v in zip(self.NAMES, parts[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(name)
+        os.unlink(self.f.name)
+        loaded = [s for s in sm if s > 500] or sm
+        return {"sm_mhz": statistics.median(loaded) if loaded else None,
+                "sm_max_mhz": max(smax) if smax else None, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def workload(args):
+    from tracegen import configs
+    w = configs.make(args.config, args.size)
+    ops, args_ = w.arrays(not args.clean)
+    name = {1: "config1 racy listing", 2: "config2 Jacobi halo exchange 4096x4096 fp32, 100 iterations",
+            3: "config3 multi-stream event DAG, 8 streams, 1 GiB, 10k launches",
+            4: "config4 large tracked memory, 16 x 1 GiB annotated per launch, 1k launches",
+            5: "config5 scaling sweep, 64 GiB log-uniform allocations, 64 fibers, ~100k events"}[args.config]
+    return w, ops, args_, f"{name} ({'clean' if args.clean else 'racy'} twin, {args.size} size)"
+
+
+# ------------------------------------------------------------------------------------------------
+# CPU baseline: the oracle (as it stands) on a bounded contiguous granule sample of the same trace
+# ------------------------------------------------------------------------------------------------
+def oracle_sample(events, max_fibers, target_s, threads):
+    import numpy as np
+    import oracle
+    acc = events[events["kind"] == 0]
+    g0 = (acc["a"] >> np.uint64(3)).astype(np.int64)
+    g1 = ((acc["a"] + acc["b"] + np.uint64(7)) >> np.uint64(3)).astype(np.int64)
+    lo, hi = int(g0.min()), int(g1.max())
+
+    def checked(a, b):
+        return int(8 * np.sum(np.clip(np.minimum(g1, b) - np.maximum(g0, a), 0, None)))
+
+    span = max(1, (hi - lo) // 4096)         # calibration slice
+    r = oracle.check_events(events, max_fibers, threads=threads, granule_range=(lo, lo + span))
+    rate = checked(lo, lo + span) / max(r["seconds"], 1e-3)
+    for _ in range(4):                       # grow the slice until the oracle takes ~target_s
+        want = target_s * rate
+        b = lo + span
+        # extend the range until it holds `want` checked bytes (binary search over the end)
+        l2, h2 = lo + 1, hi
+        while l2 < h2:
+            m = (l2 + h2) // 2
+            if checked(lo, m) < want:
+                l2 = m + 1
+            else:
+                h2 = m
+        b = max(l2, lo + 1)
+        r = oracle.check_events(events, max_fibers, threads=threads, granule_range=(lo, b))
+        cb = checked(lo, b)
+        rate = cb / max(r["seconds"], 1e-3)
+        if r["seconds"] >= 0.5 * target_s or b >= hi:
+            break
+        span = b - lo
+    return dict(checked_bytes=cb, seconds=r["seconds"], granules=b - lo, range=(lo, b),
+                race_granules=r["n_race_granules"], rate_gbs=cb / r["seconds"] / 1e9)
+
+
+def run_reference(args):
+    """--impl reference: the oracle timed on the host cores, K bounded-sample steps (rank 0)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    from oracle.lower import lower
+    w, ops, args_, wname = workload(args)
+    ev, nf = lower(ops, args_)
+    threads = os.cpu_count() or 1
+    per_step = max(1.0, min(20.0, 150.0 / max(1, args.steps + args.warmup)))
+    s = oracle_sample(ev, nf, per_step, threads)
+    for _ in range(args.warmup):
+        oracle_sample_step(ev, nf, s, threads)
+    tot_b, tot_s = 0, 0.0
+    for _ in range(args.steps):
+        b, secs = oracle_sample_step(ev, nf, s, threads)
+        tot_b += b
+        tot_s += secs
+    value = tot_b / tot_s / 1e9
+    sample = (f"granules [{s['range'][0]}, {s['range'][1]}) = {s['granules']} granules, "
+              f"{s['checked_bytes'] / 1e9:.1f} GB checked per step")
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot_s / args.steps,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
+        "data": "synthetic", "config": {"workload": wname, "window_events": None},
+        "cpu_baseline": {"value": value, "unit": "GB/s", "cores": threads, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }))
+
+
+def oracle_sample_step(ev, nf, s, threads):
+    import oracle
+    r = oracle.check_events(ev, nf, threads=threads, granule_range=s["range"])
+    return s["checked_bytes"], r["seconds"]
+
+
+# ------------------------------------------------------------------------------------------------
+# our arm
+# ------------------------------------------------------------------------------------------------
+def run_ours(args):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sc_huckzsjb24_b200 as cs
+    from paper_conf_sc_huckzsjb24_b200.dist import ShardedPlan, gather_runs
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    stream = torch.cuda.current_stream(dev)
+
+    w, ops, args_, wname = workload(args)
+    tr = cs.Trace(255)
+    cs.Lowering(tr).cusan_lower_program(ops, args_)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    def max_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    kw = dict(window_events=args.window, device=local, stream=stream.cuda_stream)
+    if world > 1:
+        plan = ShardedPlan(tr, comm_device=dev, **kw)
+        run = plan.run
+    else:
+        plan = cs.Plan(tr, **kw)
+        run = plan.run
+    for _ in range(args.warmup):
+        rep = run()
+    # ---- timed region: K steps, CUDA events on the plan's stream, max over ranks ------------------
+    clocks = Clocks(local)
+    barrier()
+    torch.cuda.synchronize(dev)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    kernel_ms, reps = [], []
+    for _ in range(args.steps):
+        rep = run()
+        shard = plan.last_shard_report if world > 1 else rep
+        kernel_ms.append(shard.counters["kernel_ms"])
+        reps.append(rep)
+    e1.record(stream)
+    torch.cuda.synchronize(dev)
+    barrier()
+    clk = clocks.stop()
+    elapsed_s = max_over_ranks(e0.elapsed_time(e1) / 1e3)
+    shard = plan.last_shard_report if world > 1 else rep
+    ctr = shard.counters
+    launches = int(ctr["kernel_launches"]) * args.steps
+    final = reps[-1]
+    plan.close()
+    del plan
+
+    tracked = ctr["tracked_bytes"]                       # whole trace (every rank's shard together)
+    value = tracked * args.steps / elapsed_s / 1e9
+    k_ms = statistics.mean(kernel_ms)
+    cell_bytes = ctr["shadow_cell_bytes"]
+    peak, peak_src = measured_peaks()
+    achieved = cell_bytes / (k_ms / 1e3) / 1e9 if k_ms > 0 else 0.0
+    nl = max(1, int(ctr["kernel_launches"]))
+    traffic, _ = ncu_traffic()
+
+    # ---- e2e: public C ABI from host buffers, every step: lower + plan + upload + check + report ----
+    e2e_s, h2d, d2h = [], 0, 0
+    for _ in range(max(1, args.e2e_steps)):
+        barrier()
+        torch.cuda.synchronize(dev)
+        t0 = time.perf_counter()
+        t2 = cs.Trace(255)
+        cs.Lowering(t2).cusan_lower_program(ops, args_)
+        if world > 1:
+            p2 = ShardedPlan(t2, comm_device=dev, **kw)
+            r2 = p2.run()
+            c2 = p2.last_shard_report.counters
+            p2.close()
+        else:
+            r2 = cs.check(t2, **kw)
+            c2 = r2.counters
+        torch.cuda.synchronize(dev)
+        e2e_s.append(max_over_ranks(time.perf_counter() - t0))
+        h2d, d2h = int(c2["h2d_bytes"]), int(c2["d2h_bytes"])
+        if rank == 0:
+            assert r2.n_race_granules == final.n_race_granules and np.array_equal(r2.runs, final.runs)
+    e2e_value = tracked / statistics.mean(e2e_s) / 1e9
+
+    # ---- post-mortem variant (extra, for context): one window, no shadow traffic --------------------
+    pm = None
+    if world == 1:
+        p3 = cs.Plan(tr, window_events=0, device=local, stream=stream.cuda_stream)
+        p3.run()
+        torch.cuda.synchronize(dev)
+        t0 = time.perf_counter()
+        r3 = p3.run()
+        pm_s = time.perf_counter() - t0
+        assert r3.n_race_granules == final.n_race_granules and np.array_equal(r3.runs, final.runs)
+        pm = {"value": tracked / pm_s / 1e9, "unit": "GB/s", "ms_per_step": pm_s * 1e3,
+              "kernel_ms": r3.counters["kernel_ms"], "window_events": "all (one window)"}
+        p3.close()
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        ev = tr.cusan_trace_read()
+        s = oracle_sample(ev, 255, args.cpu_seconds, os.cpu_count() or 1)
+        cpu = {"value": s["rate_gbs"], "unit": "GB/s", "cores": os.cpu_count() or 1, "kind": "oracle",
+               "sample": (f"contiguous granule range [{s['range'][0]}, {s['range'][1]}) of the same trace: "
+                          f"{s['granules']} granules, {s['checked_bytes'] / 1e9:.1f} GB checked in "
+                          f"{s['seconds']:.1f} s")}
+    d_cov = tracked / 8 / max(1, ctr["n_windows"]) / max(1, ctr["shard_granules"]) if world == 1 else None
+    line = {
+        "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": 1e3 * elapsed_s / args.steps, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+        "config": {"workload": wname, "window_events": args.window, "windows": int(ctr["n_windows"]),
+                   "events": int(ctr["n_events"]), "accesses": int(ctr["n_access"]), "fibers": 64,
+                   "tracked_bytes": int(tracked), "shadow_bytes_per_gpu": int(ctr["shadow_bytes"]),
+                   "granules_per_gpu": int(ctr["shard_granules"]), "coverage_per_window": d_cov,
+                   "race_granules": int(final.n_race_granules), "race_runs": int(final.n_runs),
+                   "parallelism": f"granule-range shards x{world}",
+                   "l2": "inputs larger than L2 (shadow 128 GiB / n_gpus, streamed every window)"},
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                     "kernel": "shadow_check_window", "kernel_ms_per_step": k_ms, "launches_per_step": nl,
+                     "algorithmic_bytes_per_launch": cell_bytes / nl},
+        "cpu_baseline": cpu,
+        "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                "ms_per_step": 1e3 * statistics.mean(e2e_s)},
+        "gpu_launches": launches,
+        "clocks": clk,
+        "postmortem": pm,
+    }
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

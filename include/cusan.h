@@ -1,0 +1,173 @@
+/*
+ * cusan.h — C ABI of the B200-native happens-before race check over device memory
+ * (CuSan, Hück et al., SC-W 2024; /root/reference/PAPER.md).
+ *
+ * The library is the data-parallel hot path of CuSan's method: a trace of range accesses and
+ * release / acquire / fork edges goes in (the TSan primitives CuSan and MUST emit,
+ * PAPER.md:164-186, §II-A), an exact per-8-byte-granule race set comes out.
+ *
+ *   a0  append primitives (this header) or lower CUDA / MPI calls to them (cusan_lower.h)
+ *   a1  vector-clock / segment pass (host)                             — cusan_plan_create
+ *   a2  range → granule expansion, interval compaction, shard clip, windows (host) + upload
+ *   a3  shadow check, one sm_100a kernel launch per window (device)    — cusan_plan_run
+ *   a4  race-hit compaction into runs (kernel epilogue) + canonical merge (host)
+ *   a5  report                                                          — cusan_report_*
+ *
+ * Conventions for every function:
+ *   - returns CUSAN_OK (0) or a negative CUSAN_E* status; cusan_last_error() then returns a
+ *     thread-local message describing the failure.  No function aborts the process.
+ *   - pointers are host pointers unless stated; the library never retains caller pointers beyond
+ *     the call except the trace passed to cusan_plan_create (which must outlive the plan).
+ *   - objects are not thread-safe: one host thread per trace / plan.
+ *   - there is no CPU fallback: without a usable CUDA device the check returns CUSAN_ECUDA.
+ */
+#ifndef CUSAN_H
+#define CUSAN_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define CUSAN_OK 0
+#define CUSAN_EINVAL (-1)  /* null pointer, fiber >= max_fibers, bad enum, bad option            */
+#define CUSAN_ERANGE (-2)  /* > 2^24-2 events (24-bit event index), addr + nbytes overflows      */
+#define CUSAN_ENOMEM (-3)  /* host or device allocation failed / workspace too small             */
+#define CUSAN_ECUDA (-4)   /* CUDA runtime error (includes: no device)                           */
+#define CUSAN_ESTATE (-5)  /* object used in the wrong state                                     */
+
+#define CUSAN_MAX_FIBERS 255u          /* fiber id is 8 bits in a shadow slot; 0xFF tags a spill record */
+#define CUSAN_MAX_EVENTS ((1u << 24) - 2u) /* event index + 1 is 24 bits in a shadow slot   */
+
+typedef struct cusan_trace cusan_trace;   /* opaque; caller owns (create / destroy)            */
+typedef struct cusan_plan cusan_plan;     /* opaque; caller owns (create / destroy)            */
+typedef struct cusan_report cusan_report; /* library-allocated; free with cusan_report_free    */
+typedef struct cusan_counters cusan_counters; /* defined below (report section)                */
+
+/* Access mode of a range annotation (tsan_read_range / tsan_write_range).
+ * A kernel argument the analysis marks RW is passed as CUSAN_WRITE. */
+enum cusan_mode { CUSAN_READ = 0, CUSAN_WRITE = 1 };
+
+/* Synchronisation primitives (TSan annotation API; fibers PAPER.md:178-186). */
+enum cusan_sync {
+    CUSAN_RELEASE = 0,       /* AnnotateHappensBefore(key): SC_key := SC_key ⊔ C_fiber             */
+    CUSAN_RELEASE_STORE = 1, /* SC_key := C_fiber (a re-recorded CUDA event replaces its capture)    */
+    CUSAN_ACQUIRE = 2,       /* AnnotateHappensAfter(key): C_fiber := C_fiber ⊔ SC_key             */
+    CUSAN_FORK = 3           /* issue edge src -> dst: `fiber` = dst, `key_or_src_fiber` = src;
+                                an event of src's program order; C_dst := C_dst ⊔ C_src          */
+};
+
+/* Event kinds of the bulk record format (cusan_event.kind). */
+enum cusan_event_kind {
+    CUSAN_EV_ACCESS = 0, CUSAN_EV_RELEASE = 1, CUSAN_EV_RELEASE_STORE = 2,
+    CUSAN_EV_ACQUIRE = 3, CUSAN_EV_FORK = 4
+};
+
+/* 24-byte primitive record, little-endian (same layout as tracegen.EVENT_DTYPE).
+ * ACCESS: a = address, b = nbytes, mode = cusan_mode.  RELEASE / RELEASE_STORE / ACQUIRE:
+ * a = key.  FORK: fiber = dst, a = src fiber.  The event id of a record is its trace position. */
+typedef struct cusan_event {
+    uint8_t kind, mode;
+    uint16_t pad;
+    uint32_t fiber;
+    uint64_t a, b;
+} cusan_event;
+
+/* A maximal run of consecutive granules [g_begin, g_end) (granule = address >> 3) on which the
+ * access event `earlier` races with the later access event `later` (event ids = trace positions). */
+typedef struct cusan_race_run {
+    uint64_t g_begin, g_end;
+    uint32_t earlier, later;
+} cusan_race_run;
+
+/* ---- trace (step a0) ------------------------------------------------------------------------ */
+/* max_fibers in [1, 255]; reserve_events is a capacity hint. */
+int cusan_trace_create(uint32_t max_fibers, uint64_t reserve_events, cusan_trace** out);
+int cusan_trace_destroy(cusan_trace* t);
+/* tsan_{read,write}_range(addr, nbytes) on `fiber`.  nbytes = 0 covers no
+ * granule.  event_id (nullable) receives the trace position. */
+int cusan_trace_append_access(cusan_trace* t, uint32_t fiber, enum cusan_mode mode, uint64_t addr,
+                              uint64_t nbytes, uint32_t* event_id);
+int cusan_trace_append_sync(cusan_trace* t, enum cusan_sync kind, uint32_t fiber,
+                            uint64_t key_or_src_fiber, uint32_t* event_id);
+/* Bulk append of n records; validated as the single-record calls; all-or-nothing. */
+int cusan_trace_append_events(cusan_trace* t, const cusan_event* events, uint64_t n);
+int cusan_trace_size(const cusan_trace* t, uint64_t* n_events, uint32_t* max_fibers);
+/* Copies events [first, first + n) into out (host buffer of n records). */
+int cusan_trace_read(const cusan_trace* t, uint64_t first, uint64_t n, cusan_event* out);
+
+/* ---- check (steps a1-a5) ---------------------------------------------------------------------- */
+typedef struct cusan_check_opts {
+    int nshards;          /* granule-range shards of the shadow space (1 = whole space); one per GPU */
+    int shard;            /* shard this call checks, 0 <= shard < nshards                        */
+    int device;           /* CUDA device ordinal                                                   */
+    int window_events;    /* access events per shadow window; 0 = library default (one window)    */
+    int persist_shadow;   /* 1: store every window's final cells (shadow left valid after the run) */
+    int flags;            /* CUSAN_CHECK_* diagnostics flags (0 for normal use)                    */
+    uint64_t max_runs;    /* runs kept in the report (0 = all); counts stay exact when truncated   */
+    void* stream;         /* cudaStream_t to run on (NULL = the legacy default stream)             */
+    void* workspace;      /* optional caller-owned device memory (e.g. a torch tensor); NULL = the
+                             library allocates with cudaMalloc                                     */
+    uint64_t workspace_bytes;
+} cusan_check_opts;
+
+/* Diagnostics: disable the equal-cells range path so every granule takes the lane-parallel
+ * per-granule path (used by the parity tests to exercise both paths; results are identical). */
+#define CUSAN_CHECK_FORCE_LANES 1
+
+/* Defaults: nshards 1, shard 0, device 0, window_events 0, persist 0, max_runs 0, all NULL. */
+void cusan_check_opts_init(cusan_check_opts* o);
+
+/* Whole check: plan_create + plan_run + plan_destroy.  The trace is not mutated. */
+int cusan_check(const cusan_trace* t, const cusan_check_opts* o, cusan_report** out);
+
+/* Host preparation (a1, a2) and upload of the event / clock / interval tables to the device.
+ * The trace must stay alive and unmodified while the plan exists. */
+int cusan_plan_create(const cusan_trace* t, const cusan_check_opts* o, cusan_plan** out);
+/* Device bytes the plan needs (tables + shadow + ext slots + run buffer). */
+int cusan_plan_workspace_bytes(const cusan_plan* p, uint64_t* bytes);
+/* Device part (a3, a4) and the report (a5).  May be called repeatedly (each run starts from an
+ * empty shadow); asynchronous work is complete when it returns. */
+int cusan_plan_run(cusan_plan* p, cusan_report** out);
+int cusan_plan_destroy(cusan_plan* p);
+/* Host steps a1 and a2 only (no device needed): fills the trace / plan counters the same
+ * plan_create would compute (shard clip, intervals, segments, windows, spill records). */
+int cusan_plan_describe(const cusan_trace* t, const cusan_check_opts* o, cusan_counters* out);
+
+/* ---- report (a5) ------------------------------------------------------------------------------ */
+typedef struct cusan_counters {
+    /* trace counters, cf. CuSan's Table I */
+    uint64_t n_events, n_access, n_read, n_write, n_release, n_release_store, n_acquire, n_fork;
+    uint64_t tracked_bytes;        /* Σ over accesses of 8 × granules covered (the metric)        */
+    uint64_t tracked_bytes_shard;  /* the part of it inside this report's shard                    */
+    uint64_t bytes_read, bytes_written;
+    /* plan */
+    uint64_t n_fibers, n_segments, n_intervals, n_incidences, n_windows, n_spans;
+    uint64_t shard_granules, spill_heap_bytes, spill_spans; /* spill records: > 3 reader fibers */
+    uint64_t shadow_bytes, workspace_bytes, raw_runs;
+    /* device timings of the last run, CUDA events on the plan's stream, milliseconds */
+    double kernel_ms;              /* all shadow-check launches                                  */
+    double run_ms;                 /* whole cusan_plan_run incl. run download and merge          */
+    uint64_t kernel_launches;
+    uint64_t shadow_cell_bytes;    /* algorithmic shadow bytes moved by the check kernels          */
+    uint64_t h2d_bytes;            /* host -> device bytes: plan tables (create) + counters (run)  */
+    uint64_t d2h_bytes;            /* device -> host bytes of the last run (counters + runs)       */
+} cusan_counters;
+
+int cusan_report_get(const cusan_report* r, uint64_t* n_race_granules, uint64_t* n_runs,
+                     const cusan_race_run** runs, int* truncated);
+int cusan_report_counters(const cusan_report* r, cusan_counters* out);
+/* Report from explicit parts (e.g. runs gathered from the shards of a multi-GPU check):
+ * concatenates, sorts canonically by (later, earlier, g_begin) and merges abutting runs. */
+int cusan_report_merge(const cusan_race_run* runs, uint64_t n_runs, uint64_t n_race_granules,
+                       uint64_t max_runs, cusan_report** out);
+int cusan_report_free(cusan_report* r);
+
+const char* cusan_last_error(void);
+const char* cusan_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* CUSAN_H */

@@ -45,8 +45,10 @@ def read_report(path: str) -> dict:
 
 
 def check_events(events: np.ndarray, max_fibers: int = 0, threads: int | None = None,
-                 sample: np.ndarray | None = None) -> dict:
-    """Run the C oracle on a primitive trace; returns the canonical report."""
+                 sample: np.ndarray | None = None, granule_range: tuple[int, int] | None = None) -> dict:
+    """Run the C oracle on a primitive trace; returns the canonical report (plus the wall time of
+    the oracle process in ``seconds``)."""
+    import time
     build()
     threads = threads or os.cpu_count() or 1
     with tempfile.TemporaryDirectory() as d:
@@ -57,9 +59,14 @@ def check_events(events: np.ndarray, max_fibers: int = 0, threads: int | None = 
             sp = os.path.join(d, "s.bin")
             np.ascontiguousarray(np.unique(np.asarray(sample, np.uint64))).tofile(sp)
             cmd += ["--sample", sp]
+        if granule_range is not None:
+            cmd += ["--range", str(int(granule_range[0])), str(int(granule_range[1]))]
+        t0 = time.perf_counter()
         subprocess.check_call(cmd)
+        secs = time.perf_counter() - t0
         rep = read_report(rp)
     rep["threads"] = threads
+    rep["seconds"] = secs
     return rep
 
 

@@ -34,6 +34,7 @@
  *             u32 later}
  *   GRANULES: optional file of sorted u64 absolute granule numbers; only those granules are checked
  *             (sampled parity at full sizes).
+ *   --range LO HI: only granules in [LO, HI) are checked (a bounded contiguous sample).
  */
 #define _GNU_SOURCE
 #include <pthread.h>
@@ -364,6 +365,7 @@ static void check_range(worker_t* w, uint64_t t, uint64_t gb, uint64_t ge) {
 static uint64_t* sample;
 static uint64_t n_sample;
 static uint64_t next_item;
+static uint64_t range_lo = 0, range_hi = UINT64_MAX;   /* --range: bounded sample of granules */
 static pthread_mutex_t mu = PTHREAD_MUTEX_INITIALIZER;
 
 static void* worker_main(void* arg) {
@@ -379,7 +381,9 @@ static void* worker_main(void* arg) {
             if (t < n_tiles && tile_b[t] <= g) check_range(w, t, g, g + 1);
         } else {
             if (it >= n_tiles) break;
-            check_range(w, it, tile_b[it], tile_e[it]);
+            uint64_t gb = tile_b[it] > range_lo ? tile_b[it] : range_lo;
+            uint64_t ge = tile_e[it] < range_hi ? tile_e[it] : range_hi;
+            if (gb < ge) check_range(w, it, gb, ge);
         }
     }
     merge_triples(&w->trip, &w->runs);
@@ -393,6 +397,10 @@ int main(int argc, char** argv) {
     for (int i = 3; i < argc; i++) {
         if (!strcmp(argv[i], "--threads") && i + 1 < argc) threads = atoi(argv[++i]);
         else if (!strcmp(argv[i], "--sample") && i + 1 < argc) sample_path = argv[++i];
+        else if (!strcmp(argv[i], "--range") && i + 2 < argc) {
+            range_lo = strtoull(argv[++i], NULL, 0);
+            range_hi = strtoull(argv[++i], NULL, 0);
+        }
         else die("bad argument");
     }
     if (threads < 1) threads = 1;

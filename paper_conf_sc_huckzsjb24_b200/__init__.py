@@ -1,0 +1,224 @@
+"""paper_conf_sc_huckzsjb24_b200 — B200-native happens-before race check over device memory.
+
+Thin Python binding of ``libcusan.so`` (C ABI in ``include/cusan.h`` and ``include/cusan_lower.h``).
+Function and method names follow the C names; everything here is argument marshalling — every step
+of the check runs in the library (host C++ for a0-a2, sm_100a kernels for a3/a4).  Importing this
+module fails if the library is missing; there is no CPU fallback.
+
+    tr = Trace(max_fibers=8)
+    low = Lowering(tr); low.cusan_lower_program(ops, args)    # or tr.cusan_trace_append_*
+    rep = check(tr)                                            # K1 on cuda:0
+    rep.n_race_granules, rep.runs                              # canonical race runs
+"""
+from __future__ import annotations
+
+import ctypes as C
+
+import numpy as np
+
+from ._lib import (CusanError, check as _ck, cusan_check_opts, cusan_counters, cusan_race_run, lib)
+
+RUN_DTYPE = np.dtype([("g_begin", "<u8"), ("g_end", "<u8"), ("earlier", "<u4"), ("later", "<u4")])
+EVENT_DTYPE = np.dtype([("kind", "u1"), ("mode", "u1"), ("pad", "<u2"), ("fiber", "<u4"),
+                        ("a", "<u8"), ("b", "<u8")])
+OP_DTYPE = np.dtype([("op", "<u4"), ("x", "<u4"), ("a", "<u8"), ("b", "<u8"), ("c", "<u8"), ("s", "<u8")])
+ARG_DTYPE = np.dtype([("ptr", "<u8"), ("mode", "<u4"), ("pad", "<u4")])
+
+CUSAN_READ, CUSAN_WRITE = 0, 1
+CUSAN_RELEASE, CUSAN_RELEASE_STORE, CUSAN_ACQUIRE, CUSAN_FORK = 0, 1, 2, 3
+__all__ = ["Trace", "Lowering", "Plan", "Report", "check", "report_merge", "CusanError", "version",
+           "RUN_DTYPE", "EVENT_DTYPE"]
+
+
+def version() -> str:
+    return lib.cusan_version().decode()
+
+
+def _ptr(a: np.ndarray) -> C.c_void_p:
+    return C.c_void_p(a.ctypes.data) if a.size else C.c_void_p(0)
+
+
+class Trace:
+    """cusan_trace: the primitive event trace (step a0)."""
+
+    def __init__(self, max_fibers: int = 255, reserve_events: int = 0):
+        h = C.c_void_p()
+        _ck(lib.cusan_trace_create(max_fibers, reserve_events, C.byref(h)))
+        self.h = h
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            lib.cusan_trace_destroy(self.h)
+            self.h = None
+
+    def cusan_trace_append_access(self, fiber: int, mode: int, addr: int, nbytes: int) -> int:
+        ev = C.c_uint32()
+        _ck(lib.cusan_trace_append_access(self.h, fiber, mode, addr, nbytes, C.byref(ev)))
+        return ev.value
+
+    def cusan_trace_append_sync(self, kind: int, fiber: int, key_or_src: int) -> int:
+        ev = C.c_uint32()
+        _ck(lib.cusan_trace_append_sync(self.h, kind, fiber, key_or_src, C.byref(ev)))
+        return ev.value
+
+    def cusan_trace_append_events(self, events: np.ndarray):
+        ev = np.ascontiguousarray(events, EVENT_DTYPE)
+        _ck(lib.cusan_trace_append_events(self.h, _ptr(ev), len(ev)))
+
+    def cusan_trace_size(self) -> tuple[int, int]:
+        n, f = C.c_uint64(), C.c_uint32()
+        _ck(lib.cusan_trace_size(self.h, C.byref(n), C.byref(f)))
+        return n.value, f.value
+
+    def cusan_trace_read(self, first: int = 0, n: int | None = None) -> np.ndarray:
+        total, _ = self.cusan_trace_size()
+        n = total - first if n is None else n
+        out = np.zeros(n, EVENT_DTYPE)
+        _ck(lib.cusan_trace_read(self.h, first, n, _ptr(out)))
+        return out
+
+    def __len__(self):
+        return self.cusan_trace_size()[0]
+
+
+class Lowering:
+    """cusan_lowering: CUDA / MPI call -> primitive lowering (CuSan's per-device context)."""
+
+    def __init__(self, trace: Trace):
+        h = C.c_void_p()
+        _ck(lib.cusan_lowering_create(trace.h, C.byref(h)))
+        self.h = h
+        self.trace = trace
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            lib.cusan_lowering_destroy(self.h)
+            self.h = None
+
+    def cusan_lowering_fibers(self) -> int:
+        n = C.c_uint32()
+        _ck(lib.cusan_lowering_fibers(self.h, C.byref(n)))
+        return n.value
+
+    def cusan_lower_program(self, ops: np.ndarray, args: np.ndarray) -> np.ndarray:
+        """Lower a recorded API program; returns the first event id of every call."""
+        ops = np.ascontiguousarray(ops, OP_DTYPE)
+        args = np.ascontiguousarray(args, ARG_DTYPE)
+        first = np.zeros(len(ops), np.uint32)
+        _ck(lib.cusan_lower_program(self.h, _ptr(ops), len(ops), _ptr(args), len(args),
+                                    first.ctypes.data_as(C.POINTER(C.c_uint32))))
+        return first
+
+    def __getattr__(self, name):
+        """cusan_on_*(...) → the C call with this lowering as first argument."""
+        if name.startswith("cusan_on_"):
+            fn = getattr(lib, name)
+
+            def call(*a):
+                if name == "cusan_on_kernel":
+                    stream, ptrs, modes = a
+                    p = (C.c_uint64 * len(ptrs))(*ptrs)
+                    m = (C.c_uint32 * len(modes))(*modes)
+                    _ck(fn(self.h, stream, len(ptrs), p, m))
+                else:
+                    _ck(fn(self.h, *a))
+            return call
+        raise AttributeError(name)
+
+
+class Report:
+    """cusan_report: race count, canonical runs, counters."""
+
+    def __init__(self, h: C.c_void_p, max_runs: int = 0):
+        self.h = h
+        ng, nr, tr = C.c_uint64(), C.c_uint64(), C.c_int()
+        rp = C.POINTER(cusan_race_run)()
+        _ck(lib.cusan_report_get(h, C.byref(ng), C.byref(nr), C.byref(rp), C.byref(tr)))
+        self.n_race_granules = ng.value
+        self.n_runs = nr.value
+        self.truncated = bool(tr.value)
+        kept = nr.value if not tr.value else min(nr.value, max_runs)
+        ctr = cusan_counters()
+        _ck(lib.cusan_report_counters(h, C.byref(ctr)))
+        self.counters = {n: getattr(ctr, n) for n, _ in cusan_counters._fields_}
+        if kept:
+            buf = (C.c_char * (kept * RUN_DTYPE.itemsize)).from_address(C.addressof(rp.contents))
+            self.runs = np.frombuffer(bytes(buf), RUN_DTYPE).copy()
+        else:
+            self.runs = np.zeros(0, RUN_DTYPE)
+
+    def __del__(self):
+        if getattr(self, "h", None):
+            lib.cusan_report_free(self.h)
+            self.h = None
+
+
+CUSAN_CHECK_FORCE_LANES = 1
+
+
+def _opts(nshards=1, shard=0, device=0, window_events=0, persist_shadow=False, max_runs=0, stream=None,
+          flags=0):
+    o = cusan_check_opts()
+    lib.cusan_check_opts_init(C.byref(o))
+    o.nshards, o.shard, o.device, o.flags = nshards, shard, device, flags
+    o.window_events, o.persist_shadow, o.max_runs = window_events, int(persist_shadow), max_runs
+    o.stream = stream
+    return o
+
+
+def _report(h, max_runs):
+    return Report(h, max_runs)
+
+
+class Plan:
+    """cusan_plan: host preparation (a1, a2) + device tables; run() does a3-a5 on the GPU."""
+
+    def __init__(self, trace: Trace, **kw):
+        self.trace = trace            # must outlive the plan
+        self.max_runs = kw.get("max_runs", 0)
+        o = _opts(**kw)
+        h = C.c_void_p()
+        _ck(lib.cusan_plan_create(trace.h, C.byref(o), C.byref(h)))
+        self.h = h
+
+    def workspace_bytes(self) -> int:
+        b = C.c_uint64()
+        _ck(lib.cusan_plan_workspace_bytes(self.h, C.byref(b)))
+        return b.value
+
+    def run(self) -> Report:
+        h = C.c_void_p()
+        _ck(lib.cusan_plan_run(self.h, C.byref(h)))
+        return _report(h, self.max_runs)
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib.cusan_plan_destroy(self.h)
+            self.h = None
+
+    __del__ = close
+
+
+def describe(trace: Trace, **kw) -> dict:
+    """cusan_plan_describe: the host steps a1/a2 only (no GPU) — plan counters of a shard."""
+    o = _opts(**kw)
+    ctr = cusan_counters()
+    _ck(lib.cusan_plan_describe(trace.h, C.byref(o), C.byref(ctr)))
+    return {n: getattr(ctr, n) for n, _ in cusan_counters._fields_}
+
+
+def check(trace: Trace, **kw) -> Report:
+    """cusan_check: plan + run + destroy.  kw: nshards, shard, device, window_events,
+    persist_shadow, max_runs, stream (a cudaStream_t as int, e.g. torch's current stream)."""
+    o = _opts(**kw)
+    h = C.c_void_p()
+    _ck(lib.cusan_check(trace.h, C.byref(o), C.byref(h)))
+    return _report(h, kw.get("max_runs", 0))
+
+
+def report_merge(runs: np.ndarray, n_race_granules: int, max_runs: int = 0) -> Report:
+    """cusan_report_merge: canonical report from runs gathered from several shards."""
+    runs = np.ascontiguousarray(runs, RUN_DTYPE)
+    h = C.c_void_p()
+    _ck(lib.cusan_report_merge(_ptr(runs), len(runs), n_race_granules, max_runs, C.byref(h)))
+    return _report(h, max_runs)

@@ -1,0 +1,732 @@
+// Device part of the check (steps a3, a4) and the plan / check C ABI.
+//
+// K1 shadow_check_window — one launch per window of consecutive access events.
+//   Shadow cell: 16 B per 8-byte granule {W, R0, R1, R2}, each u32 = fiber:8 | (event id + 1):24,
+//   0 = empty.  When more than three fibers have read since the last write,
+//   R2 holds SPILL_TAG | r: the readers beyond R0, R1 live in an immutable spill record r of the
+//   device heap ({n, epoch_1..epoch_n}), so the read set stays exact with a fixed 16-B cell.
+//   The per-granule rule is the FastTrack-style check of SURVEY.md §8(c) step 3:
+//       any access b:      W ≠ ∅ ∧ ¬HB(W, b)            → race (W, b)
+//       write b:           ∀ read r ≠ ∅ ∧ ¬HB(r, b)     → race (r, b);   W := b, R := ∅
+//       read b on fiber f: R[f] := b
+//   with HB(e = (g, i+1), b in segment s of fiber f) ⇔ g = f ∨ i+1 ≤ segvc[s][g].
+//   Work unit = a warp range: consecutive granules of one elementary interval, all covered by the
+//   same accesses of the window.  Warps own contiguous runs of ranges (coverage-weighted).
+//   Per range:
+//     pass 1  stream the cells in (coalesced 128-bit loads, 8 in flight per lane) and vote whether
+//             they are all equal (skipped in the interval's first window: known empty);
+//     pass 2  equal cells evolve identically under the same accesses, so the warp applies the
+//             window's accesses once to the common cell (spilled readers in shared memory); each
+//             hit is a run over the whole range;
+//     pass 3  stream the final cell out (128-bit stores; skipped when no later window needs it).
+//   Ranges whose cells differ take the exact lane-parallel path: 32 lanes × 4 consecutive granules
+//   per step, each lane its own cell and spill record (copy-on-write), hits compacted in the warp
+//   (__ballot_sync over hit lanes, __shfl_up_sync comparison with the left neighbour, run heads
+//   sized from the continuation mask).  Both paths feed a 32-entry per-warp run cache (one entry
+//   per lane) that extends runs across steps and ranges before appending them to global memory.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "common.h"
+
+using namespace cusan;
+
+namespace {
+
+constexpr int U = 4;                    // 32-granule chunks per lane-parallel step
+constexpr int CHUNK = 32 * U;           // granules per lane-parallel step
+constexpr int UL = 8;                   // 16-B loads / stores in flight per lane when streaming
+constexpr int WARPS = 8;                // warps per block
+constexpr int THREADS = 32 * WARPS;
+constexpr int MAXS = 256;               // shared-memory spill list per warp (≥ 255 − 2 readers)
+constexpr unsigned FULL = 0xffffffffu;
+
+// counters[]: 0 race granules, 1 raw runs, 2 heap top (record units), 3 heap overflow flag
+enum { C_RACE = 0, C_RUNS = 1, C_HEAP = 2, C_HEAP_OVF = 3, N_COUNTERS = 4 };
+
+// A window's work on one elementary interval, cut into warp ranges of `rsize` granules.
+struct DSpan {
+    uint64_t abs_begin, dense_begin, len;
+    uint64_t tile0, weight0;     // prefix of ranges / of range weights over the window's spans
+    uint32_t rsize, rweight;     // granules per range (multiple of CHUNK), weight of one range
+    uint32_t list_off, list_cnt, flags, rec, rec_units, pad;
+};
+static_assert(sizeof(DSpan) == 72, "DSpan layout");
+
+struct Ctx {                     // kernel-wide pointers
+    const AccRec* __restrict__ inc;
+    const uint32_t* __restrict__ segvc;
+    uint32_t F;
+    uint4* __restrict__ shadow;
+    uint32_t* __restrict__ heap;
+    unsigned long long heap_cap;  // record units
+    cusan_race_run* __restrict__ runs;
+    unsigned long long* __restrict__ counters;
+    unsigned long long run_cap;
+};
+
+struct RunCache {
+    uint32_t e, l;       // earlier / later event id
+    uint64_t gb, ge;     // [gb, ge), empty when ge == gb
+    uint32_t rr;         // round-robin victim lane (warp-uniform)
+    unsigned long long nrace;
+};
+
+__device__ __forceinline__ bool is_spill(uint32_t v) { return (v >> 24) == 0xFFu; }
+__device__ __forceinline__ uint32_t* rec_ptr(const Ctx& k, uint32_t v) {
+    return k.heap + (uint64_t)(v & 0xffffffu) * REC_WORDS;
+}
+
+__device__ __forceinline__ void flush_entry(const RunCache& c, const Ctx& k) {
+    unsigned long long idx = atomicAdd(&k.counters[C_RUNS], 1ull);
+    if (idx < k.run_cap) {
+        cusan_race_run r;
+        r.g_begin = c.gb;
+        r.g_end = c.ge;
+        r.earlier = c.e;
+        r.later = c.l;
+        k.runs[idx] = r;
+    }
+}
+
+// Warp-collective: add run [rgb, rge) of (re, rl) to the per-warp run cache (one entry per lane):
+// extend an entry that ends where the run begins, else evict the round-robin victim.
+__device__ __forceinline__ void cache_insert(uint32_t re, uint32_t rl, uint64_t rgb, uint64_t rge, int lane,
+                                             RunCache& rc, const Ctx& k) {
+    const unsigned mm = __ballot_sync(FULL, rc.ge > rc.gb && rc.e == re && rc.l == rl && rc.ge == rgb);
+    if (mm) {
+        if (lane == __ffs(mm) - 1) rc.ge = rge;
+    } else {
+        if (lane == (int)rc.rr) {
+            if (rc.ge > rc.gb) flush_entry(rc, k);
+            rc.e = re;
+            rc.l = rl;
+            rc.gb = rgb;
+            rc.ge = rge;
+        }
+        rc.rr = (rc.rr + 1) & 31u;
+    }
+}
+
+// Warp-collective, lane-parallel granules: every lane passes its own hit flag (false for lanes
+// without a granule).  Lanes hold consecutive granules g.
+__device__ __forceinline__ void emit(bool hit, uint32_t earlier_epoch, uint32_t later_id, uint64_t g,
+                                     int lane, RunCache& rc, const Ctx& k) {
+    const unsigned m = __ballot_sync(FULL, hit);
+    if (!m) return;
+    rc.nrace += __popc(m);
+    const uint32_t e_id = (earlier_epoch & 0xffffffu) - 1u;
+    const uint32_t prev = __shfl_up_sync(FULL, e_id, 1);
+    const bool cont = hit && lane > 0 && ((m >> (lane - 1)) & 1u) && prev == e_id;
+    const unsigned cm = __ballot_sync(FULL, cont);
+    unsigned heads = m & ~cm;
+    uint32_t len = 0;
+    if (hit && !cont) {
+        const unsigned long long rest = (unsigned long long)cm >> (lane + 1);
+        len = (uint32_t)__ffsll((long long)~rest);   // 1 + number of continuing lanes
+    }
+    while (heads) {
+        const int h = __ffs(heads) - 1;
+        heads &= heads - 1;
+        const uint32_t re = __shfl_sync(FULL, e_id, h);
+        const uint64_t rgb = __shfl_sync(FULL, g, h);
+        const uint32_t rl = __shfl_sync(FULL, len, h);
+        cache_insert(re, later_id, rgb, rgb + rl, lane, rc, k);
+    }
+}
+
+// Warp-uniform: one hit covering every granule of [gb, ge).
+__device__ __forceinline__ void emit_range(bool hit, uint32_t earlier_epoch, uint32_t later_id, uint64_t gb,
+                                           uint64_t ge, int lane, RunCache& rc, const Ctx& k) {
+    if (!hit) return;
+    rc.nrace += ge - gb;
+    cache_insert((earlier_epoch & 0xffffffu) - 1u, later_id, gb, ge, lane, rc, k);
+}
+
+// ¬HB(earlier epoch e, later access of fiber f whose segment row is `row`)
+__device__ __forceinline__ bool unordered(uint32_t e, uint32_t f, const uint32_t* __restrict__ row) {
+    if (!e) return false;
+    const uint32_t g = e >> 24;
+    return g != f && (e & 0xffffffu) > __ldg(row + g);
+}
+
+__device__ __forceinline__ bool same(const uint4& a, const uint4& b) {
+    return ((a.x ^ b.x) | (a.y ^ b.y) | (a.z ^ b.z) | (a.w ^ b.w)) == 0u;
+}
+
+// ---- lane path: per-lane spill records, copy-on-write ------------------------------------------
+// allocate a record of n entries; returns the tagged slot value, or 0 on heap overflow (flagged)
+__device__ __forceinline__ uint32_t rec_alloc(const Ctx& k, uint32_t n, uint32_t** out) {
+    const uint32_t units = (n + 1 + REC_WORDS - 1) / REC_WORDS;
+    const unsigned long long at = atomicAdd(&k.counters[C_HEAP], (unsigned long long)units);
+    if (at + units > k.heap_cap) {
+        k.counters[C_HEAP_OVF] = 1ull;
+        *out = nullptr;
+        return 0;
+    }
+    *out = k.heap + at * REC_WORDS;
+    (*out)[0] = n;
+    return SPILL_TAG | (uint32_t)at;
+}
+
+// R[f] := ep on one lane's cell
+__device__ void lane_read_update(uint4& c, uint32_t ep, uint32_t f, const Ctx& k) {
+    if (c.y && (c.y >> 24) == f) { c.y = ep; return; }
+    if (c.z && (c.z >> 24) == f) { c.z = ep; return; }
+    if (c.w && !is_spill(c.w) && (c.w >> 24) == f) { c.w = ep; return; }
+    if (!c.y) { c.y = ep; return; }
+    if (!c.z) { c.z = ep; return; }
+    if (!c.w) { c.w = ep; return; }
+    uint32_t* dst;
+    if (!is_spill(c.w)) {                      // fourth reader: record {R2, ep}
+        const uint32_t v = rec_alloc(k, 2, &dst);
+        if (dst) { dst[1] = c.w; dst[2] = ep; }
+        c.w = v;
+        return;
+    }
+    const uint32_t* src = rec_ptr(k, c.w);
+    const uint32_t n = src[0];
+    int pos = -1;
+    for (uint32_t j = 0; j < n; j++)
+        if ((src[1 + j] >> 24) == f) { pos = (int)j; break; }
+    if (pos >= 0 && src[1 + pos] == ep) return;
+    const uint32_t v = rec_alloc(k, pos >= 0 ? n : n + 1, &dst);   // copy-on-write
+    if (dst) {
+        for (uint32_t j = 0; j < n; j++) dst[1 + j] = src[1 + j];
+        if (pos >= 0) dst[1 + pos] = ep; else dst[1 + n] = ep;
+    }
+    c.w = v;
+}
+
+// Lane-parallel exact path for granules [x0, x0 + n) of span sp (each lane its own cells).
+__device__ void check_lanes(const DSpan& sp, uint64_t x0, uint64_t n, int lane, RunCache& rc, const Ctx& k) {
+    for (uint64_t xc = x0; xc < x0 + n; xc += CHUNK) {
+        uint4 cell[U];
+        bool valid[U];
+#pragma unroll
+        for (int c = 0; c < U; c++) {
+            const uint64_t x = xc + c * 32 + lane;
+            valid[c] = x < x0 + n;
+            cell[c] = make_uint4(0, 0, 0, 0);
+            if (valid[c] && (sp.flags & SPAN_LOAD)) cell[c] = __ldcs(k.shadow + sp.dense_begin + x);
+        }
+        const uint32_t qe = sp.list_off + sp.list_cnt;
+        for (uint32_t q = sp.list_off; q < qe; q++) {
+            const AccRec r = k.inc[q];
+            const uint32_t f = r.epoch >> 24;
+            const uint32_t later = (r.epoch & 0xffffffu) - 1u;
+            const uint32_t* row = k.segvc + (uint64_t)(r.segm & 0x7fffffffu) * k.F;
+            const bool wr = r.segm >> 31;
+#pragma unroll
+            for (int c = 0; c < U; c++) {
+                const uint64_t g = sp.abs_begin + xc + c * 32 + lane;
+                emit(valid[c] && unordered(cell[c].x, f, row), cell[c].x, later, g, lane, rc, k);
+                if (wr) {
+                    emit(valid[c] && unordered(cell[c].y, f, row), cell[c].y, later, g, lane, rc, k);
+                    emit(valid[c] && unordered(cell[c].z, f, row), cell[c].z, later, g, lane, rc, k);
+                    const bool sp_w = valid[c] && is_spill(cell[c].w);
+                    emit(valid[c] && !sp_w && unordered(cell[c].w, f, row), cell[c].w, later, g, lane, rc, k);
+                    const uint32_t* rp = sp_w ? rec_ptr(k, cell[c].w) : nullptr;
+                    const uint32_t nr = sp_w ? rp[0] : 0u;
+                    const uint32_t nmax = __reduce_max_sync(FULL, nr);
+                    for (uint32_t j = 0; j < nmax; j++) {
+                        const uint32_t v = j < nr ? rp[1 + j] : 0u;
+                        emit(unordered(v, f, row), v, later, g, lane, rc, k);
+                    }
+                    cell[c] = make_uint4(r.epoch, 0, 0, 0);
+                } else if (valid[c]) {
+                    lane_read_update(cell[c], r.epoch, f, k);
+                }
+            }
+        }
+        if (sp.flags & SPAN_STORE) {
+#pragma unroll
+            for (int c = 0; c < U; c++) {
+                const uint64_t x = xc + c * 32 + lane;
+                if (valid[c]) __stcs(k.shadow + sp.dense_begin + x, cell[c]);
+            }
+        }
+    }
+}
+
+__device__ __forceinline__ uint32_t find_span_by_tile(const DSpan* __restrict__ sp, uint32_t n, uint64_t t) {
+    uint32_t lo = 0, hi = n;        // last span with tile0 <= t
+    while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (sp[mid].tile0 <= t) lo = mid; else hi = mid;
+    }
+    return lo;
+}
+
+// first range whose start weight is >= pos
+__device__ __forceinline__ uint64_t tile_at_weight(const DSpan* __restrict__ sp, uint32_t n,
+                                                   uint64_t pos, uint64_t total_w, uint64_t total_t) {
+    if (pos >= total_w) return total_t;
+    uint32_t lo = 0, hi = n;
+    while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (sp[mid].weight0 <= pos) lo = mid; else hi = mid;
+    }
+    const uint64_t w = sp[lo].rweight;
+    return sp[lo].tile0 + (pos - sp[lo].weight0 + w - 1) / w;
+}
+
+__global__ void __launch_bounds__(THREADS, 3)
+shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t total_tiles,
+                    uint64_t total_weight, Ctx k, int force_lanes) {
+    __shared__ uint32_t s_list[WARPS][MAXS];
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    uint32_t* lst = s_list[warp];
+    const uint64_t nwarps = (uint64_t)gridDim.x * WARPS;
+    const uint64_t wid = (uint64_t)blockIdx.x * WARPS + warp;
+    const uint64_t t0 = tile_at_weight(spans, nspans, (uint64_t)((unsigned __int128)total_weight * wid / nwarps),
+                                       total_weight, total_tiles);
+    const uint64_t t1 = tile_at_weight(spans, nspans, (uint64_t)((unsigned __int128)total_weight * (wid + 1) / nwarps),
+                                       total_weight, total_tiles);
+    RunCache rc;
+    rc.e = rc.l = 0;
+    rc.gb = rc.ge = 0;
+    rc.rr = 0;
+    rc.nrace = 0;
+    if (t0 < t1) {
+        uint32_t s = find_span_by_tile(spans, nspans, t0);
+        for (uint64_t t = t0; t < t1; t++) {
+            while (t >= spans[s + 1].tile0) s++;   // spans[nspans] is a sentinel
+            const DSpan sp = spans[s];
+            const uint64_t x0 = (t - sp.tile0) * sp.rsize;
+            const uint64_t n = min((uint64_t)sp.rsize, sp.len - x0);
+            uint4* cells = k.shadow + sp.dense_begin + x0;
+            // ---- pass 1: stream the range's cells in and vote that they are all equal ----------
+            uint4 c = make_uint4(0, 0, 0, 0);      // first window of the interval: known empty
+            bool uniform = !force_lanes;
+            if (uniform && (sp.flags & SPAN_LOAD)) {
+                c = cells[0];
+                bool ok = true;
+                for (uint64_t i = lane; i < n; i += 32 * UL) {
+                    uint4 v[UL];
+#pragma unroll
+                    for (int u = 0; u < UL; u++) v[u] = (i + u * 32 < n) ? __ldcs(cells + i + u * 32) : c;
+#pragma unroll
+                    for (int u = 0; u < UL; u++) ok &= same(v[u], c);
+                }
+                uniform = __all_sync(FULL, ok);
+            }
+            if (!uniform) {
+                check_lanes(sp, x0, n, lane, rc, k);
+                continue;
+            }
+            // ---- pass 2: all cells of the range equal `c`: apply the window's accesses once -----
+            // readers beyond R0, R1 are kept as a list in shared memory (ns entries)
+            uint32_t ns = 0;
+            if (c.w) {
+                if (is_spill(c.w)) {
+                    const uint32_t* rp = rec_ptr(k, c.w);
+                    ns = rp[0];
+                    for (uint32_t j = lane; j < ns; j += 32) lst[j] = rp[1 + j];
+                } else {
+                    if (lane == 0) lst[0] = c.w;
+                    ns = 1;
+                }
+                c.w = 0;
+                __syncwarp();
+            }
+            const uint64_t gb = sp.abs_begin + x0, ge = gb + n;
+            const uint32_t qe = sp.list_off + sp.list_cnt;
+            AccRec nxt = k.inc[sp.list_off];
+            for (uint32_t q = sp.list_off; q < qe; q++) {
+                const AccRec r = nxt;
+                if (q + 1 < qe) nxt = k.inc[q + 1];
+                const uint32_t f = r.epoch >> 24;
+                const uint32_t later = (r.epoch & 0xffffffu) - 1u;
+                const uint32_t* row = k.segvc + (uint64_t)(r.segm & 0x7fffffffu) * k.F;
+                emit_range(unordered(c.x, f, row), c.x, later, gb, ge, lane, rc, k);
+                if (r.segm >> 31) {
+                    emit_range(unordered(c.y, f, row), c.y, later, gb, ge, lane, rc, k);
+                    emit_range(unordered(c.z, f, row), c.z, later, gb, ge, lane, rc, k);
+                    for (uint32_t j = 0; j < ns; j++) {
+                        const uint32_t v = lst[j];
+                        emit_range(unordered(v, f, row), v, later, gb, ge, lane, rc, k);
+                    }
+                    c = make_uint4(r.epoch, 0, 0, 0);
+                    ns = 0;
+                } else if (c.y && (c.y >> 24) == f) {
+                    c.y = r.epoch;
+                } else if (c.z && (c.z >> 24) == f) {
+                    c.z = r.epoch;
+                } else {
+                    int pos = -1;
+                    for (uint32_t b = 0; b < ns; b += 32) {
+                        const uint32_t j = b + lane;
+                        const unsigned m = __ballot_sync(FULL, j < ns && (lst[j] >> 24) == f);
+                        if (m) { pos = (int)(b + __ffs(m) - 1); break; }
+                    }
+                    if (pos >= 0) { if (lane == 0) lst[pos] = r.epoch; }
+                    else if (!c.y) c.y = r.epoch;
+                    else if (!c.z) c.z = r.epoch;
+                    else { if (lane == 0) lst[ns] = r.epoch; ns++; }
+                    __syncwarp();
+                }
+            }
+            // ---- pass 3: stream the final cell out -----------------------------------------------
+            if (sp.flags & SPAN_STORE) {
+                if (ns == 1) {
+                    c.w = lst[0];
+                } else if (ns > 1) {
+                    uint32_t* dst = nullptr;
+                    uint32_t v = 0;
+                    if (ns + 1 <= sp.rec_units * REC_WORDS) {      // the span's pre-assigned record
+                        v = SPILL_TAG | sp.rec;
+                        dst = k.heap + (uint64_t)sp.rec * REC_WORDS;
+                    } else {
+                        if (lane == 0) v = rec_alloc(k, ns, &dst);
+                        v = __shfl_sync(FULL, v, 0);
+                        dst = v ? rec_ptr(k, v) : nullptr;
+                    }
+                    if (dst) {
+                        if (lane == 0) dst[0] = ns;
+                        for (uint32_t j = lane; j < ns; j += 32) dst[1 + j] = lst[j];
+                    }
+                    c.w = v;
+                }
+                for (uint64_t i = lane; i < n; i += 32 * UL) {
+#pragma unroll
+                    for (int u = 0; u < UL; u++)
+                        if (i + u * 32 < n) __stcs(cells + i + u * 32, c);
+                }
+            }
+            __syncwarp();
+        }
+    }
+    if (rc.ge > rc.gb) flush_entry(rc, k);
+    if (lane == 0 && rc.nrace) atomicAdd(&k.counters[C_RACE], rc.nrace);
+}
+
+int cuda_fail(cudaError_t e, const char* what) {
+    return fail(CUSAN_ECUDA, std::string(what) + ": " + cudaGetErrorString(e));
+}
+#define CK(call)                                        \
+    do {                                                \
+        cudaError_t _e = (call);                        \
+        if (_e != cudaSuccess) return cuda_fail(_e, #call); \
+    } while (0)
+
+constexpr uint64_t ALIGN = 256;
+inline uint64_t align_up(uint64_t x) { return (x + ALIGN - 1) / ALIGN * ALIGN; }
+
+struct Window {
+    uint64_t span_off;      // into d_spans (window-local array incl. sentinel)
+    uint32_t nspans;
+    uint64_t tiles, weight;
+    uint32_t grid;
+};
+
+}  // namespace
+
+struct cusan_plan {
+    const cusan_trace* trace = nullptr;
+    HostPlan hp;
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    int max_blocks = 0;
+    // device memory
+    char* own = nullptr;          // library-allocated workspace (null when the caller's is used)
+    char* ws = nullptr;
+    uint64_t ws_bytes = 0;
+    AccRec* d_inc = nullptr;
+    uint32_t* d_segvc = nullptr;
+    DSpan* d_spans = nullptr;
+    unsigned long long* d_counters = nullptr;
+    uint4* d_shadow = nullptr;
+    uint32_t* d_heap = nullptr;
+    uint64_t heap_cap = 0;                  // record units
+    uint32_t* d_heap_own = nullptr;         // grown heap after an overflow
+    cusan_race_run* d_runs = nullptr;
+    cusan_race_run* d_runs_own = nullptr;   // grown run buffer after an overflow
+    uint64_t run_cap = 0;
+    bool need_shadow = false;
+    std::vector<Window> wins;
+    uint64_t shadow_cell_bytes = 0;
+    uint64_t table_bytes = 0;               // tables uploaded by plan_create
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+
+    ~cusan_plan() {
+        if (ev0) cudaEventDestroy(ev0);
+        if (ev1) cudaEventDestroy(ev1);
+        if (own) cudaFree(own);
+        if (d_runs_own) cudaFree(d_runs_own);
+        if (d_heap_own) cudaFree(d_heap_own);
+    }
+};
+
+static int plan_device_setup(cusan_plan* p) {
+    HostPlan& hp = p->hp;
+    const cusan_check_opts& o = hp.opts;
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess || ndev == 0)
+        return fail(CUSAN_ECUDA, std::string("no CUDA device available: ") + cudaGetErrorString(e));
+    if (o.device < 0 || o.device >= ndev) return fail(CUSAN_EINVAL, "bad device ordinal");
+    p->device = o.device;
+    CK(cudaSetDevice(p->device));
+    p->stream = (cudaStream_t)o.stream;
+    int sms = 0, per_sm = 0;
+    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, p->device));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, shadow_check_window, THREADS, 0));
+    p->max_blocks = sms * std::max(per_sm, 1);
+
+    // device-side span tables: per window its spans plus a sentinel, with range / weight prefixes
+    std::vector<DSpan> ds;
+    ds.reserve(hp.spans.size() + hp.win_span_off.size());
+    p->need_shadow = false;
+    p->shadow_cell_bytes = 0;
+    for (size_t w = 0; w + 1 < hp.win_span_off.size(); w++) {
+        Window win{};
+        win.span_off = ds.size();
+        uint64_t tiles = 0, weight = 0;
+        for (uint64_t i = hp.win_span_off[w]; i < hp.win_span_off[w + 1]; i++) {
+            const Span& s = hp.spans[i];
+            DSpan d{};
+            d.abs_begin = s.abs_begin;
+            d.dense_begin = s.dense_begin;
+            d.len = s.len;
+            d.list_off = s.list_off;
+            d.list_cnt = s.list_cnt;
+            d.flags = s.flags;
+            d.rec = s.rec;
+            d.rec_units = s.rec_units;
+            // warp range: long enough that replaying the window's accesses once per range stays
+            // cheap next to streaming its cells (≈ 64 granules per access), capped for balance;
+            // spans that move no cells are one range each
+            uint64_t rs;
+            if (s.flags & (SPAN_LOAD | SPAN_STORE))
+                rs = std::min<uint64_t>(std::max<uint64_t>(64ull * s.list_cnt, 2048), 1ull << 16);
+            else
+                rs = std::max<uint64_t>(s.len, 1);
+            rs = std::min<uint64_t>((rs + CHUNK - 1) / CHUNK * CHUNK, 1ull << 31);
+            d.rsize = (uint32_t)rs;
+            const uint64_t nt = (s.len + rs - 1) / rs;
+            const uint64_t mem = (s.flags & (SPAN_LOAD | SPAN_STORE)) ? rs / 32 : 0;
+            d.rweight = (uint32_t)std::min<uint64_t>(mem + 4ull * s.list_cnt + 8, 0xffffffffull);
+            d.tile0 = tiles;
+            d.weight0 = weight;
+            tiles += nt;
+            weight += nt * d.rweight;
+            if (s.flags) p->need_shadow = true;
+            p->shadow_cell_bytes += s.len * (((s.flags & SPAN_LOAD) ? 16 : 0) + ((s.flags & SPAN_STORE) ? 16 : 0));
+            ds.push_back(d);
+        }
+        win.nspans = (uint32_t)(ds.size() - win.span_off);
+        DSpan sent{};
+        sent.tile0 = tiles;
+        sent.weight0 = weight;
+        ds.push_back(sent);
+        win.tiles = tiles;
+        win.weight = weight;
+        win.grid = (uint32_t)std::min<uint64_t>((uint64_t)p->max_blocks, (tiles + WARPS - 1) / WARPS);
+        if (win.grid == 0) win.grid = 1;
+        p->wins.push_back(win);
+    }
+
+    // workspace layout
+    p->heap_cap = hp.rec_units + (1ull << 16);             // pre-assigned records + lane-path room
+    uint64_t off = 0;
+    const uint64_t o_inc = off;     off = align_up(off + hp.inc.size() * sizeof(AccRec));
+    const uint64_t o_seg = off;     off = align_up(off + hp.segvc.size() * sizeof(uint32_t));
+    const uint64_t o_spans = off;   off = align_up(off + ds.size() * sizeof(DSpan));
+    const uint64_t o_cnt = off;     off = align_up(off + N_COUNTERS * sizeof(unsigned long long));
+    const uint64_t o_heap = off;    off = align_up(off + p->heap_cap * REC_WORDS * sizeof(uint32_t));
+    const uint64_t o_shadow = off;  off = align_up(off + (p->need_shadow ? hp.shard_granules * 16 : 0));
+    p->run_cap = std::max<uint64_t>(1ull << 16, 4 * p->wins.size() + 1024);
+    const uint64_t o_runs = off;    off = align_up(off + p->run_cap * sizeof(cusan_race_run));
+    p->ws_bytes = off;
+    if (o.workspace) {
+        if (o.workspace_bytes < off)
+            return fail(CUSAN_ENOMEM, "workspace too small: need " + std::to_string(off) + " bytes");
+        p->ws = (char*)o.workspace;
+    } else {
+        cudaError_t me = cudaMalloc((void**)&p->own, std::max<uint64_t>(off, ALIGN));
+        if (me != cudaSuccess) return fail(CUSAN_ENOMEM, std::string("cudaMalloc workspace: ") + cudaGetErrorString(me));
+        p->ws = p->own;
+    }
+    p->d_inc = (AccRec*)(p->ws + o_inc);
+    p->d_segvc = (uint32_t*)(p->ws + o_seg);
+    p->d_spans = (DSpan*)(p->ws + o_spans);
+    p->d_counters = (unsigned long long*)(p->ws + o_cnt);
+    p->d_heap = (uint32_t*)(p->ws + o_heap);
+    p->d_shadow = p->need_shadow ? (uint4*)(p->ws + o_shadow) : nullptr;
+    p->d_runs = (cusan_race_run*)(p->ws + o_runs);
+    CK(cudaMemcpyAsync(p->d_inc, hp.inc.data(), hp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, p->stream));
+    CK(cudaMemcpyAsync(p->d_segvc, hp.segvc.data(), hp.segvc.size() * sizeof(uint32_t), cudaMemcpyHostToDevice, p->stream));
+    CK(cudaMemcpyAsync(p->d_spans, ds.data(), ds.size() * sizeof(DSpan), cudaMemcpyHostToDevice, p->stream));
+    p->table_bytes = hp.inc.size() * sizeof(AccRec) + hp.segvc.size() * sizeof(uint32_t) + ds.size() * sizeof(DSpan);
+    CK(cudaEventCreate(&p->ev0));
+    CK(cudaEventCreate(&p->ev1));
+    CK(cudaStreamSynchronize(p->stream));
+    hp.ctr.shadow_bytes = p->need_shadow ? hp.shard_granules * 16 : 0;
+    hp.ctr.workspace_bytes = p->ws_bytes;
+    return CUSAN_OK;
+}
+
+static int launch_all(cusan_plan* p) {
+    // counters: race granules, runs, heap top (after the pre-assigned records), overflow flag
+    const unsigned long long init[N_COUNTERS] = {0, 0, p->hp.rec_units, 0};
+    CK(cudaMemcpyAsync(p->d_counters, init, sizeof(init), cudaMemcpyHostToDevice, p->stream));
+    CK(cudaEventRecord(p->ev0, p->stream));
+    Ctx k;
+    k.inc = p->d_inc;
+    k.segvc = p->d_segvc;
+    k.F = p->hp.F;
+    k.shadow = p->d_shadow;
+    k.heap = p->d_heap;
+    k.heap_cap = p->heap_cap;
+    k.runs = p->d_runs;
+    k.counters = p->d_counters;
+    k.run_cap = p->run_cap;
+    const int force_lanes = (p->hp.opts.flags & CUSAN_CHECK_FORCE_LANES) ? 1 : 0;
+    for (const Window& w : p->wins)
+        shadow_check_window<<<w.grid, THREADS, 0, p->stream>>>(p->d_spans + w.span_off, w.nspans, w.tiles,
+                                                               w.weight, k, force_lanes);
+    CK(cudaGetLastError());
+    CK(cudaEventRecord(p->ev1, p->stream));
+    return CUSAN_OK;
+}
+
+extern "C" {
+
+int cusan_plan_create(const cusan_trace* t, const cusan_check_opts* o, cusan_plan** out) {
+    if (!t || !o || !out) return fail(CUSAN_EINVAL, "null argument");
+    *out = nullptr;
+    cusan_plan* p = new (std::nothrow) cusan_plan;
+    if (!p) return fail(CUSAN_ENOMEM, "cannot allocate plan");
+    p->trace = t;
+    int st;
+    try {
+        st = build_host_plan(t->t, *o, p->hp);
+    } catch (const std::bad_alloc&) {
+        st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
+    }
+    if (!st) st = plan_device_setup(p);
+    if (st) {
+        delete p;
+        return st;
+    }
+    *out = p;
+    return CUSAN_OK;
+}
+
+int cusan_plan_describe(const cusan_trace* t, const cusan_check_opts* o, cusan_counters* out) {
+    if (!t || !o || !out) return fail(CUSAN_EINVAL, "null argument");
+    HostPlan hp;
+    int st;
+    try {
+        st = build_host_plan(t->t, *o, hp);
+    } catch (const std::bad_alloc&) {
+        st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
+    }
+    if (!st) *out = hp.ctr;
+    return st;
+}
+
+int cusan_plan_workspace_bytes(const cusan_plan* p, uint64_t* bytes) {
+    if (!p || !bytes) return fail(CUSAN_EINVAL, "null argument");
+    *bytes = p->ws_bytes;
+    return CUSAN_OK;
+}
+
+int cusan_plan_run(cusan_plan* p, cusan_report** out) {
+    if (!p || !out) return fail(CUSAN_EINVAL, "null argument");
+    *out = nullptr;
+    const auto t_start = std::chrono::steady_clock::now();
+    CK(cudaSetDevice(p->device));
+    unsigned long long cnt[N_COUNTERS];
+    for (int attempt = 0;; attempt++) {
+        int st = launch_all(p);
+        if (st) return st;
+        CK(cudaMemcpyAsync(cnt, p->d_counters, sizeof(cnt), cudaMemcpyDeviceToHost, p->stream));
+        CK(cudaStreamSynchronize(p->stream));
+        const bool runs_ovf = cnt[C_RUNS] > p->run_cap, heap_ovf = cnt[C_HEAP_OVF] != 0;
+        if (!runs_ovf && !heap_ovf) break;
+        if (attempt >= 8) return fail(CUSAN_ENOMEM, "run buffer / spill heap keeps overflowing");
+        if (runs_ovf) {                        // grow the run buffer and re-run (counts are exact)
+            if (p->d_runs_own) cudaFree(p->d_runs_own);
+            p->d_runs_own = nullptr;
+            const uint64_t cap = cnt[C_RUNS] + cnt[C_RUNS] / 8 + 1024;
+            if (cudaMalloc((void**)&p->d_runs_own, cap * sizeof(cusan_race_run)) != cudaSuccess)
+                return fail(CUSAN_ENOMEM, "cannot grow the run buffer");
+            p->d_runs = p->d_runs_own;
+            p->run_cap = cap;
+        }
+        if (heap_ovf) {                        // grow the spill heap (24-bit record index)
+            const uint64_t cap = std::min<uint64_t>(2 * p->heap_cap, (1ull << 24) - 1);
+            if (cap <= p->heap_cap) return fail(CUSAN_ENOMEM, "spill heap exceeds the 24-bit record index");
+            uint32_t* nh = nullptr;
+            if (cudaMalloc((void**)&nh, cap * REC_WORDS * sizeof(uint32_t)) != cudaSuccess)
+                return fail(CUSAN_ENOMEM, "cannot grow the spill heap");
+            if (p->d_heap_own) cudaFree(p->d_heap_own);
+            p->d_heap_own = nh;
+            p->d_heap = nh;
+            p->heap_cap = cap;
+        }
+    }
+    float kms = 0.f;
+    CK(cudaEventElapsedTime(&kms, p->ev0, p->ev1));
+    cusan_report* r = new (std::nothrow) cusan_report;
+    if (!r) return fail(CUSAN_ENOMEM, "cannot allocate report");
+    try {
+        r->runs.resize(cnt[C_RUNS]);
+    } catch (...) {
+        delete r;
+        return fail(CUSAN_ENOMEM, "cannot allocate report runs");
+    }
+    if (cnt[C_RUNS]) {
+        cudaError_t ce = cudaMemcpyAsync(r->runs.data(), p->d_runs, cnt[C_RUNS] * sizeof(cusan_race_run),
+                                         cudaMemcpyDeviceToHost, p->stream);
+        if (ce == cudaSuccess) ce = cudaStreamSynchronize(p->stream);
+        if (ce != cudaSuccess) {
+            delete r;
+            return cuda_fail(ce, "run download");
+        }
+    }
+    canonicalize_runs(r->runs);
+    r->n_runs = r->runs.size();
+    r->n_race_granules = cnt[C_RACE];
+    const uint64_t max_runs = p->hp.opts.max_runs;
+    if (max_runs && r->runs.size() > max_runs) {
+        r->runs.resize(max_runs);
+        r->truncated = 1;
+    }
+    r->ctr = p->hp.ctr;
+    r->ctr.raw_runs = cnt[C_RUNS];
+    r->ctr.kernel_ms = kms;
+    r->ctr.kernel_launches = p->wins.size();
+    r->ctr.shadow_cell_bytes = p->shadow_cell_bytes;
+    r->ctr.h2d_bytes = p->table_bytes + sizeof(unsigned long long) * N_COUNTERS;
+    r->ctr.d2h_bytes = sizeof(cnt) + cnt[C_RUNS] * sizeof(cusan_race_run);
+    r->ctr.run_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count();
+    *out = r;
+    return CUSAN_OK;
+}
+
+int cusan_plan_destroy(cusan_plan* p) {
+    if (!p) return fail(CUSAN_EINVAL, "plan is null");
+    if (p->stream) cudaStreamSynchronize(p->stream);
+    delete p;
+    return CUSAN_OK;
+}
+
+int cusan_check(const cusan_trace* t, const cusan_check_opts* o, cusan_report** out) {
+    cusan_plan* p = nullptr;
+    int st = cusan_plan_create(t, o, &p);
+    if (st) return st;
+    st = cusan_plan_run(p, out);
+    cusan_plan_destroy(p);
+    return st;
+}
+
+}  // extern "C"

@@ -1,0 +1,100 @@
+// Internal declarations shared by the library's translation units (not part of the C ABI).
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/cusan.h"
+
+namespace cusan {
+
+// thread-local last error (cusan_last_error)
+int fail(int status, const std::string& msg);
+
+struct Trace {
+    uint32_t max_fibers = 1;
+    std::vector<cusan_event> ev;
+};
+
+// ----------------------------------------------------------------------------------------------
+// Shadow slot encoding: u32 = fiber:8 | (event id + 1):24, 0 = empty.
+// Fiber 0xFF is reserved: in a cell's third read slot, 0xFF:24-bit index tags a spill record.
+// ----------------------------------------------------------------------------------------------
+inline uint32_t pack_epoch(uint32_t fiber, uint32_t event_id) { return (fiber << 24) | (event_id + 1); }
+constexpr uint32_t SPILL_TAG = 0xFF000000u;
+constexpr uint32_t REC_WORDS = 8;        // spill-record allocation unit (u32 words)
+
+// Per access event, what the shadow kernel needs (8 B, one per interval incidence):
+//   epoch  = pack_epoch(fiber, event id)
+//   segm   = segment id (bits 0..30) | is_write << 31
+struct AccRec {
+    uint32_t epoch;
+    uint32_t segm;
+};
+
+// One elementary interval of the granule space (a maximal granule range no access endpoint splits),
+// clipped to the plan's shard.
+struct Interval {
+    uint64_t abs_begin;   // absolute granule (address >> 3) of the first granule in the shard clip
+    uint64_t dense_begin; // index of that granule in the shard's shadow array
+    uint64_t len;         // granules in the shard clip
+    uint32_t list_off;    // first incidence (into the AccRec table) — all windows
+    uint32_t list_cnt;
+};
+
+// A window's piece of work on one interval: the interval's incidences inside the window.
+struct Span {
+    uint64_t abs_begin, dense_begin, len;
+    uint32_t list_off;    // into the AccRec table
+    uint32_t list_cnt;
+    uint32_t flags;       // SPAN_LOAD: cells hold state from an earlier window; SPAN_STORE: write back
+    uint32_t rec;         // pre-assigned spill record (REC_WORDS-word units) for the final state
+    uint32_t rec_units;   // its size; 0 = the final state needs no record (≤ 3 readers)
+};
+enum : uint32_t { SPAN_LOAD = 1u, SPAN_STORE = 2u };
+
+struct HostPlan {
+    // options
+    cusan_check_opts opts{};
+    // a1
+    uint32_t F = 1;                       // fibers (row length of segvc)
+    std::vector<uint32_t> segvc;          // nseg × F
+    uint64_t nseg = 0;
+    // accesses in trace order
+    std::vector<uint64_t> acc_g0, acc_g1; // granule ranges
+    std::vector<uint32_t> acc_event;      // trace position
+    std::vector<AccRec> acc_rec;
+    // a2
+    std::vector<Interval> iv;             // shard-clipped intervals (len > 0)
+    std::vector<AccRec> inc;              // incidence table: per interval, its accesses in trace order
+    std::vector<uint32_t> inc_acc;        // access index of each incidence
+    uint64_t shard_granules = 0;
+    uint64_t rec_units = 0;               // pre-assigned spill-record units
+    uint64_t spill_spans = 0;
+    // windows
+    std::vector<Span> spans;              // all windows, window-major
+    std::vector<uint64_t> win_span_off;   // nwin + 1
+    uint64_t window_accesses = 0;
+    // counters
+    cusan_counters ctr{};
+};
+
+int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp);
+
+// canonical merge of runs (sort by (later, earlier, g_begin), merge abutting) — a4 host part
+void canonicalize_runs(std::vector<cusan_race_run>& runs);
+
+}  // namespace cusan
+
+struct cusan_trace {
+    cusan::Trace t;
+};
+
+struct cusan_report {
+    uint64_t n_race_granules = 0;
+    uint64_t n_runs = 0;
+    int truncated = 0;
+    std::vector<cusan_race_run> runs;
+    cusan_counters ctr{};
+};

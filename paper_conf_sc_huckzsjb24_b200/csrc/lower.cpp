@@ -1,0 +1,349 @@
+// Lowering of CUDA / CUDA-aware MPI calls to happens-before primitives (step a0).
+//
+// CuSan runtime semantics (§IV-A, 606-734) plus MUST's MPI modelling,
+// in the form of SURVEY.md §8(b)'s table.  Every operation on a stream s is bracketed by
+//   prologue:  FORK(H -> s)                         issue order (Fig. 4 rank 1)
+//              s blocking user stream: ACQUIRE(s, K(S0))       legacy barrier (Fig. 3 (i))
+//              s = S0: ACQUIRE(S0, K(u)) ∀ blocking user u     legacy barrier (Fig. 3 (ii))
+//   epilogue:  RELEASE(s, K(s))                     AnnotateHappensBefore
+#include <algorithm>
+#include <map>
+#include <new>
+#include <set>
+#include <unordered_map>
+
+#include "../../include/cusan_lower.h"
+#include "common.h"
+
+using namespace cusan;
+
+namespace {
+constexpr uint32_t H = 0, S0 = 1;
+inline uint64_t K_stream(uint32_t f) { return (1ull << 56) | f; }
+inline uint64_t K_event(uint64_t e) { return (2ull << 56) | e; }
+inline uint64_t K_req(uint64_t r) { return (3ull << 56) | r; }
+}  // namespace
+
+struct cusan_lowering {
+    cusan_trace* trace;
+    std::unordered_map<uint64_t, uint32_t> stream_fiber;   // stream handle -> fiber
+    std::vector<uint32_t> streams;                         // S0, then user streams (creation order)
+    std::vector<uint32_t> blocking;                        // blocking user streams (creation order)
+    std::vector<char> is_blocking;                         // by fiber
+    uint32_t next_fiber = 2;
+    std::set<uint32_t> mpi_free;                           // pool of completed request fibers
+    std::unordered_map<uint64_t, uint32_t> req_fiber;
+    std::map<uint64_t, std::pair<uint64_t, int>> allocs;   // base -> (size, kind)
+
+    // --- primitives ---------------------------------------------------------------------------
+    int access(uint32_t f, int mode, uint64_t addr, uint64_t n) {
+        return cusan_trace_append_access(trace, f, (cusan_mode)mode, addr, n, nullptr);
+    }
+    int sync(cusan_sync k, uint32_t f, uint64_t key) {
+        return cusan_trace_append_sync(trace, k, f, key, nullptr);
+    }
+
+    // --- helpers -------------------------------------------------------------------------------
+    // allocation containing p (TypeART's extent lookup)
+    const std::pair<const uint64_t, std::pair<uint64_t, int>>* find(uint64_t p) const {
+        auto it = allocs.upper_bound(p);
+        if (it == allocs.begin()) return nullptr;
+        --it;
+        if (p >= it->first && p < it->first + it->second.first) return &*it;
+        return nullptr;
+    }
+    int fiber_of(uint64_t stream, uint32_t* f) const {
+        auto it = stream_fiber.find(stream);
+        if (it == stream_fiber.end()) return fail(CUSAN_EINVAL, "unknown stream handle");
+        *f = it->second;
+        return CUSAN_OK;
+    }
+    int new_fiber(uint32_t* f) {
+        uint32_t mf = 0;
+        cusan_trace_size(trace, nullptr, &mf);
+        if (next_fiber >= mf) return fail(CUSAN_EINVAL, "more fibers than the trace's max_fibers");
+        *f = next_fiber++;
+        if (is_blocking.size() <= *f) is_blocking.resize(*f + 1, 0);
+        return CUSAN_OK;
+    }
+    int prologue(uint32_t f) {
+        int st = sync(CUSAN_FORK, f, H);
+        if (st) return st;
+        if (f != S0 && f < is_blocking.size() && is_blocking[f]) return sync(CUSAN_ACQUIRE, f, K_stream(S0));
+        if (f == S0)
+            for (uint32_t u : blocking)
+                if ((st = sync(CUSAN_ACQUIRE, S0, K_stream(u)))) return st;
+        return CUSAN_OK;
+    }
+    int epilogue(uint32_t f) { return sync(CUSAN_RELEASE, f, K_stream(f)); }
+    // cudaStreamSynchronize; on S0 also every blocking stream (724-727)
+    int host_sync_stream(uint32_t f) {
+        int st = sync(CUSAN_ACQUIRE, H, K_stream(f));
+        if (st || f != S0) return st;
+        for (uint32_t u : blocking)
+            if ((st = sync(CUSAN_ACQUIRE, H, K_stream(u)))) return st;
+        return CUSAN_OK;
+    }
+    // cudaDeviceSynchronize: every stream
+    int host_sync_device() {
+        for (uint32_t f : streams) {
+            int st = sync(CUSAN_ACQUIRE, H, K_stream(f));
+            if (st) return st;
+        }
+        return CUSAN_OK;
+    }
+    bool tracked(uint64_t p, uint64_t n) const { return n > 0 && find(p) != nullptr; }
+};
+
+extern "C" {
+
+int cusan_lowering_create(cusan_trace* trace, cusan_lowering** out) {
+    if (!trace || !out) return fail(CUSAN_EINVAL, "null argument");
+    uint32_t mf = 0;
+    cusan_trace_size(trace, nullptr, &mf);
+    if (mf < 2) return fail(CUSAN_EINVAL, "a lowering needs max_fibers >= 2 (host + default stream)");
+    cusan_lowering* l = new (std::nothrow) cusan_lowering;
+    if (!l) return fail(CUSAN_ENOMEM, "cannot allocate lowering");
+    l->trace = trace;
+    l->stream_fiber[0] = S0;
+    l->streams.push_back(S0);
+    l->is_blocking.assign(2, 0);
+    *out = l;
+    return CUSAN_OK;
+}
+
+int cusan_lowering_destroy(cusan_lowering* l) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    delete l;
+    return CUSAN_OK;
+}
+
+int cusan_lowering_fibers(const cusan_lowering* l, uint32_t* n) {
+    if (!l || !n) return fail(CUSAN_EINVAL, "null argument");
+    *n = l->next_fiber;
+    return CUSAN_OK;
+}
+
+int cusan_on_malloc(cusan_lowering* l, uint64_t ptr, uint64_t size, enum cusan_mem_kind kind) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    if ((unsigned)kind > 3) return fail(CUSAN_EINVAL, "bad memory kind");
+    l->allocs[ptr] = {size, (int)kind};   // allocation is not an access
+    return CUSAN_OK;
+}
+
+int cusan_on_free(cusan_lowering* l, uint64_t) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    return l->host_sync_device();
+}
+
+int cusan_on_stream_create(cusan_lowering* l, uint64_t stream, int nonblocking) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    uint32_t f = 0;
+    int st = l->new_fiber(&f);
+    if (st) return st;
+    l->stream_fiber[stream] = f;
+    l->streams.push_back(f);
+    if (!nonblocking) {                    // track the non-blocking attribute
+        l->blocking.push_back(f);
+        l->is_blocking[f] = 1;
+    }
+    return CUSAN_OK;
+}
+
+int cusan_on_kernel(cusan_lowering* l, uint64_t stream, uint32_t nargs, const uint64_t* ptrs,
+                    const uint32_t* modes) {
+    if (!l || (nargs && (!ptrs || !modes))) return fail(CUSAN_EINVAL, "null argument");
+    uint32_t f = 0;
+    int st = l->fiber_of(stream, &f);
+    if (st || (st = l->prologue(f))) return st;
+    // (ii) of PAPER.md:650-654: each argument's whole allocation, by its R/W attribute
+    for (uint32_t i = 0; i < nargs; i++) {
+        auto* a = l->find(ptrs[i]);
+        if (!a) continue;
+        if (modes[i] > 2) return fail(CUSAN_EINVAL, "bad argument mode");
+        int mode = modes[i] == 0 ? CUSAN_READ : CUSAN_WRITE;   // RW -> WRITE
+        if ((st = l->access(f, mode, a->first, a->second.first))) return st;
+    }
+    return l->epilogue(f);
+}
+
+int cusan_on_stream_sync(cusan_lowering* l, uint64_t stream) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    uint32_t f = 0;
+    int st = l->fiber_of(stream, &f);
+    return st ? st : l->host_sync_stream(f);
+}
+
+int cusan_on_device_sync(cusan_lowering* l) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    return l->host_sync_device();
+}
+
+int cusan_on_event_record(cusan_lowering* l, uint64_t event, uint64_t stream) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    uint32_t f = 0;
+    int st = l->fiber_of(stream, &f);
+    if (st || (st = l->prologue(f))) return st;
+    return l->sync(CUSAN_RELEASE_STORE, f, K_event(event));
+}
+
+int cusan_on_event_sync(cusan_lowering* l, uint64_t event) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    return l->sync(CUSAN_ACQUIRE, H, K_event(event));
+}
+
+int cusan_on_stream_wait_event(cusan_lowering* l, uint64_t stream, uint64_t event) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    uint32_t f = 0;
+    int st = l->fiber_of(stream, &f);
+    if (st || (st = l->prologue(f))) return st;
+    return l->sync(CUSAN_ACQUIRE, f, K_event(event));
+}
+
+int cusan_on_stream_query(cusan_lowering* l, uint64_t stream, int success) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    uint32_t f = 0;
+    int st = l->fiber_of(stream, &f);
+    if (st || !success) return st;
+    return l->host_sync_stream(f);
+}
+
+int cusan_on_memcpy(cusan_lowering* l, uint64_t dst, uint64_t src, uint64_t n,
+                    enum cusan_copy_kind kind, int async, uint64_t stream) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    if ((unsigned)kind > 3) return fail(CUSAN_EINVAL, "bad copy kind");
+    uint32_t f = S0;
+    int st = async ? l->fiber_of(stream, &f) : CUSAN_OK;
+    if (st || (st = l->prologue(f))) return st;
+    if (l->tracked(dst, n) && (st = l->access(f, CUSAN_WRITE, dst, n))) return st;
+    if (l->tracked(src, n) && (st = l->access(f, CUSAN_READ, src, n))) return st;
+    if ((st = l->epilogue(f))) return st;
+    if (!async && kind != CUSAN_D2D)
+        return l->sync(CUSAN_ACQUIRE, H, K_stream(S0));
+    return CUSAN_OK;
+}
+
+int cusan_on_memset(cusan_lowering* l, uint64_t ptr, uint64_t n, int async, uint64_t stream) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    uint32_t f = S0;
+    int st = async ? l->fiber_of(stream, &f) : CUSAN_OK;
+    if (st || (st = l->prologue(f))) return st;
+    auto* a = l->find(ptr);
+    if (l->tracked(ptr, n) && (st = l->access(f, CUSAN_WRITE, ptr, n))) return st;
+    if ((st = l->epilogue(f))) return st;
+    if (!async && a && a->second.second == CUSAN_MEM_PINNED)
+        return l->sync(CUSAN_ACQUIRE, H, K_stream(S0));
+    return CUSAN_OK;
+}
+
+int cusan_on_host_access(cusan_lowering* l, uint64_t addr, uint64_t n, enum cusan_mode mode) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    return l->access(H, mode ? CUSAN_WRITE : CUSAN_READ, addr, n);
+}
+
+static int mpi_nonblocking(cusan_lowering* l, uint64_t buf, uint64_t n, uint64_t req, int mode) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    uint32_t m = 0;
+    if (!l->mpi_free.empty()) {            // recycled only after completion
+        m = *l->mpi_free.begin();
+        l->mpi_free.erase(l->mpi_free.begin());
+    } else {
+        int st = l->new_fiber(&m);
+        if (st) return st;
+    }
+    l->req_fiber[req] = m;
+    int st = l->sync(CUSAN_FORK, m, H);    // fiber per non-blocking request
+    if (st || (st = l->access(m, mode, buf, n))) return st;
+    return l->sync(CUSAN_RELEASE, m, K_req(req));
+}
+
+int cusan_on_mpi_isend(cusan_lowering* l, uint64_t buf, uint64_t n, uint64_t req) {
+    return mpi_nonblocking(l, buf, n, req, CUSAN_READ);
+}
+
+int cusan_on_mpi_irecv(cusan_lowering* l, uint64_t buf, uint64_t n, uint64_t req) {
+    return mpi_nonblocking(l, buf, n, req, CUSAN_WRITE);
+}
+
+int cusan_on_mpi_wait(cusan_lowering* l, uint64_t req) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    int st = l->sync(CUSAN_ACQUIRE, H, K_req(req));
+    if (st) return st;
+    auto it = l->req_fiber.find(req);
+    if (it != l->req_fiber.end()) {
+        l->mpi_free.insert(it->second);
+        l->req_fiber.erase(it);
+    }
+    return CUSAN_OK;
+}
+
+int cusan_on_mpi_test(cusan_lowering* l, uint64_t req, int flag) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    return flag ? cusan_on_mpi_wait(l, req) : CUSAN_OK;
+}
+
+int cusan_on_mpi_send(cusan_lowering* l, uint64_t buf, uint64_t n) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    return l->access(H, CUSAN_READ, buf, n);
+}
+
+int cusan_on_mpi_recv(cusan_lowering* l, uint64_t buf, uint64_t n) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    return l->access(H, CUSAN_WRITE, buf, n);
+}
+
+int cusan_lower_program(cusan_lowering* l, const cusan_api_call* calls, uint64_t n,
+                        const cusan_api_arg* args, uint64_t nargs, uint32_t* op_first_event) {
+    if (!l || (n && !calls) || (nargs && !args)) return fail(CUSAN_EINVAL, "null argument");
+    std::vector<uint64_t> ptrs;
+    std::vector<uint32_t> modes;
+    for (uint64_t i = 0; i < n; i++) {
+        const cusan_api_call& c = calls[i];
+        if (op_first_event) {
+            uint64_t ne = 0;
+            cusan_trace_size(l->trace, &ne, nullptr);
+            op_first_event[i] = (uint32_t)ne;
+        }
+        int st = CUSAN_OK;
+        switch (c.op) {
+            case CUSAN_OP_MALLOC: st = cusan_on_malloc(l, c.a, c.b, (cusan_mem_kind)c.x); break;
+            case CUSAN_OP_FREE: st = cusan_on_free(l, c.a); break;
+            case CUSAN_OP_STREAM_CREATE: st = cusan_on_stream_create(l, c.s, c.x & 1); break;
+            case CUSAN_OP_KERNEL: {
+                if (c.b + c.x > nargs) return fail(CUSAN_EINVAL, "kernel arguments out of range");
+                ptrs.resize(c.x);
+                modes.resize(c.x);
+                for (uint32_t j = 0; j < c.x; j++) {
+                    ptrs[j] = args[c.b + j].ptr;
+                    modes[j] = args[c.b + j].mode;
+                }
+                st = cusan_on_kernel(l, c.s, c.x, ptrs.data(), modes.data());
+                break;
+            }
+            case CUSAN_OP_STREAM_SYNC: st = cusan_on_stream_sync(l, c.s); break;
+            case CUSAN_OP_DEVICE_SYNC: st = cusan_on_device_sync(l); break;
+            case CUSAN_OP_EVENT_RECORD: st = cusan_on_event_record(l, c.c, c.s); break;
+            case CUSAN_OP_EVENT_SYNC: st = cusan_on_event_sync(l, c.c); break;
+            case CUSAN_OP_STREAM_WAIT_EVENT: st = cusan_on_stream_wait_event(l, c.s, c.c); break;
+            case CUSAN_OP_STREAM_QUERY: st = cusan_on_stream_query(l, c.s, (int)c.x); break;
+            case CUSAN_OP_MEMCPY: st = cusan_on_memcpy(l, c.a, c.b, c.c, (cusan_copy_kind)c.x, 0, 0); break;
+            case CUSAN_OP_MEMCPY_ASYNC:
+                st = cusan_on_memcpy(l, c.a, c.b, c.c, (cusan_copy_kind)c.x, 1, c.s);
+                break;
+            case CUSAN_OP_MEMSET: st = cusan_on_memset(l, c.a, c.c, 0, 0); break;
+            case CUSAN_OP_MEMSET_ASYNC: st = cusan_on_memset(l, c.a, c.c, 1, c.s); break;
+            case CUSAN_OP_HOST_ACCESS: st = cusan_on_host_access(l, c.a, c.c, (cusan_mode)(c.x ? 1 : 0)); break;
+            case CUSAN_OP_MPI_ISEND: st = cusan_on_mpi_isend(l, c.a, c.c, c.b); break;
+            case CUSAN_OP_MPI_IRECV: st = cusan_on_mpi_irecv(l, c.a, c.c, c.b); break;
+            case CUSAN_OP_MPI_WAIT: st = cusan_on_mpi_wait(l, c.b); break;
+            case CUSAN_OP_MPI_TEST: st = cusan_on_mpi_test(l, c.b, (int)c.x); break;
+            case CUSAN_OP_MPI_SEND: st = cusan_on_mpi_send(l, c.a, c.c); break;
+            case CUSAN_OP_MPI_RECV: st = cusan_on_mpi_recv(l, c.a, c.c); break;
+            default: return fail(CUSAN_EINVAL, "unknown API op");
+        }
+        if (st) return st;
+    }
+    return CUSAN_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,274 @@
+// Host preparation of a check (steps a1 and a2).
+//
+// a1  vector-clock / segment pass.  One pass over the trace keeps the current vector clock C_f of
+//     every fiber and the sync clock SC_k of every key (TSan annotation semantics, PAPER.md:164-173;
+//     fibers PAPER.md:178-186).  A fiber's clock entries for *other* fibers change only at an
+//     ACQUIRE or an incoming FORK, so the accesses of a fiber between two such events share one
+//     "segment" row segvc[seg][0..F) = C_f.  The shadow kernel's happens-before test for an earlier
+//     epoch (g, i+1) against a later access of fiber f in segment s is then
+//         g == f  ||  i+1 <= segvc[s][g]
+//     Rows are created lazily at the first access after a segment opens (no row for a segment
+//     without accesses).
+//
+// a2  range -> granule expansion and compaction.  Granule = addr >> 3 and an access covers
+//     [addr >> 3, (addr + n + 7) >> 3).  All access endpoints split the granule space into
+//     elementary intervals; the covered ones are numbered densely (the shadow index space), each with
+//     its list of covering accesses in trace order (its "incidences").  The space is cut into
+//     `nshards` contiguous dense ranges of equal coverage weight (Σ granules × incidences), and this
+//     plan keeps the clip of its shard.  Windows are runs of `window_events` consecutive accesses;
+//     a window's spans are its incidences grouped by interval.
+#include <algorithm>
+#include <bitset>
+#include <unordered_map>
+
+#include "common.h"
+
+namespace cusan {
+
+int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp) {
+    if (o.nshards < 1 || o.shard < 0 || o.shard >= o.nshards)
+        return fail(CUSAN_EINVAL, "need 0 <= shard < nshards");
+    if (o.window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
+    hp.opts = o;
+    const uint32_t F = t.max_fibers;
+    hp.F = F;
+    cusan_counters& c = hp.ctr;
+    c = cusan_counters{};
+    c.n_events = t.ev.size();
+    c.n_fibers = F;
+
+    // ---------------------------------------------------------------- a1: clocks and segments --
+    std::vector<uint32_t> C((size_t)F * F, 0);
+    std::unordered_map<uint64_t, uint32_t> key_slot;
+    std::vector<uint32_t> sc;                       // sync clocks, F entries per key
+    const uint32_t NO_SEG = 0xffffffffu;
+    std::vector<uint32_t> cur_seg(F, NO_SEG);
+    auto sync_clock = [&](uint64_t key) -> uint32_t* {
+        auto it = key_slot.find(key);
+        if (it == key_slot.end()) {
+            it = key_slot.emplace(key, (uint32_t)(sc.size() / F)).first;
+            sc.resize(sc.size() + F, 0);
+        }
+        return &sc[(size_t)it->second * F];
+    };
+    uint64_t n_acc = 0;
+    for (const auto& e : t.ev) n_acc += e.kind == CUSAN_EV_ACCESS;
+    hp.acc_g0.reserve(n_acc);
+    hp.acc_g1.reserve(n_acc);
+    hp.acc_event.reserve(n_acc);
+    hp.acc_rec.reserve(n_acc);
+    for (uint64_t i = 0; i < t.ev.size(); i++) {
+        const cusan_event& e = t.ev[i];
+        const uint32_t f = e.fiber;
+        uint32_t* Cf = &C[(size_t)f * F];
+        if (e.kind == CUSAN_EV_FORK) {              // an event of the source fiber's program order
+            const uint32_t s = (uint32_t)e.a;
+            uint32_t* Cs = &C[(size_t)s * F];
+            Cs[s] = (uint32_t)(i + 1);
+            for (uint32_t g = 0; g < F; g++) Cf[g] = std::max(Cf[g], Cs[g]);
+            cur_seg[f] = NO_SEG;                    // incoming edge opens a segment on dst
+            c.n_fork++;
+            continue;
+        }
+        Cf[f] = (uint32_t)(i + 1);
+        switch (e.kind) {
+            case CUSAN_EV_ACCESS: {
+                if (cur_seg[f] == NO_SEG) {
+                    if (hp.nseg >= 0x7fffffffu) return fail(CUSAN_ERANGE, "too many segments");
+                    cur_seg[f] = (uint32_t)hp.nseg++;
+                    hp.segvc.insert(hp.segvc.end(), Cf, Cf + F);
+                }
+                const uint64_t g0 = e.a >> 3;
+                const uint64_t g1 = e.b ? (e.a + e.b + 7) >> 3 : g0;
+                hp.acc_g0.push_back(g0);
+                hp.acc_g1.push_back(g1);
+                hp.acc_event.push_back((uint32_t)i);
+                hp.acc_rec.push_back({pack_epoch(f, (uint32_t)i), cur_seg[f] | ((uint32_t)e.mode << 31)});
+                const uint64_t bytes = 8 * (g1 - g0);
+                c.n_access++;
+                c.tracked_bytes += bytes;
+                if (e.mode) { c.n_write++; c.bytes_written += bytes; }
+                else { c.n_read++; c.bytes_read += bytes; }
+                break;
+            }
+            case CUSAN_EV_RELEASE: {                // SC_k := SC_k ⊔ C_f
+                uint32_t* S = sync_clock(e.a);
+                for (uint32_t g = 0; g < F; g++) S[g] = std::max(S[g], Cf[g]);
+                c.n_release++;
+                break;
+            }
+            case CUSAN_EV_RELEASE_STORE: {          // SC_k := C_f
+                uint32_t* S = sync_clock(e.a);
+                std::copy(Cf, Cf + F, S);
+                c.n_release_store++;
+                break;
+            }
+            case CUSAN_EV_ACQUIRE: {                // C_f := C_f ⊔ SC_k
+                uint32_t* S = sync_clock(e.a);
+                for (uint32_t g = 0; g < F; g++) Cf[g] = std::max(Cf[g], S[g]);
+                cur_seg[f] = NO_SEG;
+                c.n_acquire++;
+                break;
+            }
+            default:
+                return fail(CUSAN_EINVAL, "bad event kind in trace");
+        }
+    }
+    c.n_segments = hp.nseg;
+
+    // ---------------------------------------------------------------- a2: elementary intervals --
+    std::vector<uint64_t> B;
+    B.reserve(2 * n_acc);
+    for (uint64_t k = 0; k < n_acc; k++)
+        if (hp.acc_g1[k] > hp.acc_g0[k]) { B.push_back(hp.acc_g0[k]); B.push_back(hp.acc_g1[k]); }
+    std::sort(B.begin(), B.end());
+    B.erase(std::unique(B.begin(), B.end()), B.end());
+    const uint64_t nb = B.size();
+    std::vector<int64_t> diff(nb + 1, 0);
+    std::vector<uint32_t> b0(n_acc), b1(n_acc);
+    for (uint64_t k = 0; k < n_acc; k++) {
+        if (hp.acc_g1[k] <= hp.acc_g0[k]) { b0[k] = b1[k] = 0; continue; }
+        b0[k] = (uint32_t)(std::lower_bound(B.begin(), B.end(), hp.acc_g0[k]) - B.begin());
+        b1[k] = (uint32_t)(std::lower_bound(B.begin(), B.end(), hp.acc_g1[k]) - B.begin());
+        diff[b0[k]]++;
+        diff[b1[k]]--;
+    }
+    // elementary interval j = [B[j], B[j+1]); covered ones get ids in ascending address order
+    std::vector<uint32_t> iv_of(nb ? nb - 1 : 0, 0xffffffffu);
+    struct GIv { uint64_t abs_begin, dense_begin, len; uint32_t cnt, off; };
+    std::vector<GIv> giv;
+    {
+        int64_t cov = 0;
+        uint64_t dense = 0;
+        for (uint64_t j = 0; j + 1 < nb; j++) {
+            cov += diff[j];
+            if (cov > 0) {
+                iv_of[j] = (uint32_t)giv.size();
+                giv.push_back({B[j], dense, B[j + 1] - B[j], 0, 0});
+                dense += B[j + 1] - B[j];
+            }
+        }
+    }
+    c.n_intervals = giv.size();
+    // incidences: per interval, covering accesses in trace order (CSR)
+    for (uint64_t k = 0; k < n_acc; k++)
+        for (uint32_t j = b0[k]; j < b1[k]; j++) giv[iv_of[j]].cnt++;
+    uint64_t n_inc = 0;
+    for (auto& g : giv) {
+        if (n_inc + g.cnt > 0xffffffffull) return fail(CUSAN_ERANGE, "too many interval incidences");
+        g.off = (uint32_t)n_inc;
+        n_inc += g.cnt;
+    }
+    c.n_incidences = n_inc;
+    hp.inc.resize(n_inc);
+    hp.inc_acc.resize(n_inc);
+    {
+        std::vector<uint32_t> fill(giv.size());
+        for (size_t i = 0; i < giv.size(); i++) fill[i] = giv[i].off;
+        for (uint64_t k = 0; k < n_acc; k++)
+            for (uint32_t j = b0[k]; j < b1[k]; j++) {
+                uint32_t q = fill[iv_of[j]]++;
+                hp.inc[q] = hp.acc_rec[k];
+                hp.inc_acc[q] = (uint32_t)k;
+            }
+    }
+
+    // ---------------------------------------------------------------- a2: shard clip ------------
+    const uint64_t total_dense = giv.empty() ? 0 : giv.back().dense_begin + giv.back().len;
+    uint64_t d_lo = 0, d_hi = total_dense;
+    if (o.nshards > 1 && !giv.empty()) {
+        // boundaries at equal cumulative coverage weight Σ len × cnt
+        unsigned __int128 wtot = 0;
+        for (auto& g : giv) wtot += (unsigned __int128)g.len * g.cnt;
+        auto boundary = [&](int k) -> uint64_t {
+            if (k <= 0) return 0;
+            if (k >= o.nshards) return total_dense;
+            unsigned __int128 target = wtot * (unsigned)k / (unsigned)o.nshards, acc = 0;
+            for (auto& g : giv) {
+                unsigned __int128 w = (unsigned __int128)g.len * g.cnt;
+                if (acc + w >= target) {
+                    uint64_t x = (uint64_t)((target - acc + g.cnt - 1) / g.cnt);
+                    return g.dense_begin + std::min<uint64_t>(x, g.len);
+                }
+                acc += w;
+            }
+            return total_dense;
+        };
+        d_lo = boundary(o.shard);
+        d_hi = boundary(o.shard + 1);
+    }
+    hp.iv.clear();
+    for (auto& g : giv) {
+        uint64_t lo = std::max(g.dense_begin, d_lo), hi = std::min(g.dense_begin + g.len, d_hi);
+        if (lo >= hi) continue;
+        Interval v{};
+        v.abs_begin = g.abs_begin + (lo - g.dense_begin);
+        v.dense_begin = lo - d_lo;
+        v.len = hi - lo;
+        v.list_off = g.off;
+        v.list_cnt = g.cnt;
+        hp.iv.push_back(v);
+        c.tracked_bytes_shard += 8 * v.len * g.cnt;
+    }
+    hp.shard_granules = d_hi - d_lo;
+    c.shard_granules = hp.shard_granules;
+
+    // ---------------------------------------------------------------- windows and spans ---------
+    // A span that stores its final cells and ends with more than three reader fibers since the
+    // interval's last write gets a pre-assigned spill record: the cell keeps W, R0, R1 inline and
+    // the third slot points at the record holding the other readers (the reader *set* depends only
+    // on the fibers and modes covering the interval, never on happens-before, so its size is known
+    // here exactly).
+    const uint64_t W = o.window_events > 0 ? (uint64_t)o.window_events : std::max<uint64_t>(n_acc, 1);
+    hp.window_accesses = W;
+    const uint64_t nwin = n_acc ? (n_acc + W - 1) / W : 0;
+    std::vector<std::vector<Span>> per(nwin);
+    hp.rec_units = 0;
+    hp.spill_spans = 0;
+    for (const Interval& v : hp.iv) {
+        std::bitset<CUSAN_MAX_FIBERS + 1> readers;
+        uint32_t q = v.list_off, qe = v.list_off + v.list_cnt;
+        while (q < qe) {
+            uint64_t w = hp.inc_acc[q] / W;
+            uint32_t q2 = q;
+            while (q2 < qe && hp.inc_acc[q2] / W == w) {
+                const AccRec& r = hp.inc[q2];
+                if (r.segm >> 31) readers.reset();
+                else readers.set(r.epoch >> 24);
+                q2++;
+            }
+            Span s{};
+            s.abs_begin = v.abs_begin;
+            s.dense_begin = v.dense_begin;
+            s.len = v.len;
+            s.list_off = q;
+            s.list_cnt = q2 - q;
+            s.flags = (q > v.list_off ? SPAN_LOAD : 0u) | ((q2 < qe || o.persist_shadow) ? SPAN_STORE : 0u);
+            const uint64_t nr = readers.count();
+            if ((s.flags & SPAN_STORE) && nr > 3) {
+                s.rec = (uint32_t)hp.rec_units;
+                s.rec_units = (uint32_t)((nr - 2 + 1 + REC_WORDS - 1) / REC_WORDS);
+                hp.rec_units += s.rec_units;
+                hp.spill_spans++;
+            }
+            per[w].push_back(s);
+            q = q2;
+        }
+    }
+    if (hp.rec_units >= (1u << 24) - 1)
+        return fail(CUSAN_ERANGE, "too many spill records for the 24-bit record index");
+    c.spill_spans = hp.spill_spans;
+    c.spill_heap_bytes = hp.rec_units * REC_WORDS * 4;
+    hp.spans.clear();
+    hp.win_span_off.assign(1, 0);
+    for (uint64_t w = 0; w < nwin; w++) {
+        if (per[w].empty()) continue;              // windows with nothing in this shard
+        hp.spans.insert(hp.spans.end(), per[w].begin(), per[w].end());
+        hp.win_span_off.push_back(hp.spans.size());
+    }
+    c.n_windows = hp.win_span_off.size() - 1;
+    c.n_spans = hp.spans.size();
+    return CUSAN_OK;
+}
+
+}  // namespace cusan

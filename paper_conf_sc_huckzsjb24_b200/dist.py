@@ -1,0 +1,72 @@
+"""Multi-GPU check: the shadow space is sharded by granule range, one shard per rank.
+
+Granules are independent, so every rank builds the same host plan from the same trace (no table
+broadcast is needed: the trace is the input each rank holds), checks only its shard on its own GPU
+with no communication inside the check, and the race runs are gathered to rank 0 — the one real
+exchange step — with torch.distributed (NCCL over NVLink on GPUs, gloo in CPU tests).  Rank 0
+stitches runs that abut across shard boundaries and sorts them canonically (cusan_report_merge).
+"""
+from __future__ import annotations
+
+import numpy as np
+import torch
+import torch.distributed as dist
+
+from . import RUN_DTYPE, Plan, Report, Trace, report_merge
+
+_RUN_U64 = RUN_DTYPE.itemsize // 8          # a run record as three u64 words
+
+
+def gather_runs(runs: np.ndarray, n_race: int, device: torch.device | None = None,
+                group=None) -> tuple[np.ndarray, int] | None:
+    """All-gather every rank's runs and race-granule count; returns (runs, count) on rank 0."""
+    dev = device if device is not None else torch.device("cpu")
+    words = torch.from_numpy(np.ascontiguousarray(runs, RUN_DTYPE).view(np.uint64).astype(np.int64)).to(dev)
+    world = dist.get_world_size(group)
+    meta = torch.tensor([len(runs), n_race], dtype=torch.int64, device=dev)
+    metas = [torch.zeros_like(meta) for _ in range(world)]
+    dist.all_gather(metas, meta, group=group)
+    counts = [int(m[0]) for m in metas]
+    cap = max(max(counts), 1)
+    buf = torch.zeros(cap * _RUN_U64, dtype=torch.int64, device=dev)
+    buf[: words.numel()] = words
+    parts = [torch.zeros_like(buf) for _ in range(world)]
+    dist.all_gather(parts, buf, group=group)
+    if dist.get_rank(group) != 0:
+        return None
+    allw = [p[: c * _RUN_U64].cpu().numpy().astype(np.uint64) for p, c in zip(parts, counts)]
+    merged = np.concatenate(allw).view(RUN_DTYPE) if allw else np.zeros(0, RUN_DTYPE)
+    return merged, int(sum(int(m[1]) for m in metas))
+
+
+class ShardedPlan:
+    """One rank's shard of a multi-GPU check.  run() checks the shard on this rank's GPU, gathers
+    the runs and returns the canonical whole-trace Report on rank 0 (None elsewhere)."""
+
+    def __init__(self, trace: Trace, device: int = 0, group=None, comm_device: torch.device | None = None,
+                 **kw):
+        self.group = group
+        self.rank = dist.get_rank(group)
+        self.world = dist.get_world_size(group)
+        self.comm_device = comm_device
+        self.max_runs = kw.pop("max_runs", 0)
+        self.plan = Plan(trace, nshards=self.world, shard=self.rank, device=device, **kw)
+        self.last_shard_report: Report | None = None
+
+    def run(self) -> Report | None:
+        rep = self.plan.run()
+        self.last_shard_report = rep
+        out = gather_runs(rep.runs, rep.n_race_granules, self.comm_device, self.group)
+        if out is None:
+            return None
+        runs, n_race = out
+        return report_merge(runs, n_race, self.max_runs)
+
+    def close(self):
+        self.plan.close()
+
+
+def merge_shard_reports(parts: list[Report], max_runs: int = 0) -> Report:
+    """Single-process form of the gather + stitch (used when shards run one after another)."""
+    runs = np.concatenate([p.runs for p in parts]) if parts else np.zeros(0, RUN_DTYPE)
+    return report_merge(runs, sum(p.n_race_granules for p in parts), max_runs)

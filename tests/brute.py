@@ -127,3 +127,16 @@ def runs_to_triples(runs) -> set[tuple[int, int, int]]:
         for g in range(int(r["g_begin"]), int(r["g_end"])):
             out.add((g, int(r["earlier"]), int(r["later"])))
     return out
+
+
+def runs_to_triples_in(runs, granules: set) -> set[tuple[int, int, int]]:
+    """Triples of `runs` restricted to the given granules (runs may span billions of granules)."""
+    import bisect
+    gs = sorted(granules)
+    out = set()
+    for r in runs:
+        lo = bisect.bisect_left(gs, int(r["g_begin"]))
+        hi = bisect.bisect_left(gs, int(r["g_end"]))
+        for g in gs[lo:hi]:
+            out.add((g, int(r["earlier"]), int(r["later"])))
+    return out

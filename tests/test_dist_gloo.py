@@ -1,0 +1,110 @@
+"""Multi-GPU host logic on CPU: world_size-2 gloo process group.
+
+The kernels need a GPU, so here the two ranks exercise everything around them: the host shard
+partition (cusan_plan_describe), the run gather (dist.gather_runs over gloo) and rank 0's stitch
+and canonical sort (cusan_report_merge).  Each rank's shard runs are the oracle's runs clipped to
+that rank's granule range, so a stitch that failed to re-join runs cut at the shard boundary, or
+lost a rank's runs, would not reproduce the oracle's whole report.
+"""
+from __future__ import annotations
+
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _clip(runs, lo, hi):
+    out = runs.copy()
+    out["g_begin"] = np.maximum(out["g_begin"], np.uint64(lo))
+    out["g_end"] = np.minimum(out["g_end"], np.uint64(hi))
+    return out[out["g_begin"] < out["g_end"]]
+
+
+def _worker(rank, world, port, q):
+    import sys
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import oracle
+        import paper_conf_sc_huckzsjb24_b200 as cs
+        from paper_conf_sc_huckzsjb24_b200.dist import gather_runs
+        from tracegen import configs
+        w = configs.make(4, "small")
+        ops, args = w.arrays(True)
+        tr = cs.Trace(255)
+        cs.Lowering(tr).cusan_lower_program(ops, args)
+        ev = tr.cusan_trace_read()
+        ref = oracle.check_events(ev, 255, threads=2)
+        # shard boundary at the middle of the covered granule space (absolute granules)
+        acc = ev[ev["kind"] == 0]
+        g_lo = int(acc["a"].min()) >> 3
+        g_hi = int((acc["a"] + acc["b"]).max() + 7) >> 3
+        cut = (g_lo + g_hi) // 2 + 3
+        lo, hi = (g_lo, cut) if rank == 0 else (cut, g_hi)
+        mine = _clip(ref["runs"], lo, hi)
+        n_mine = int(np.sum(mine["g_end"] - mine["g_begin"]))
+        out = gather_runs(mine, n_mine)
+        # host shard partition of the product: the two shards tile the granule space and the
+        # coverage weight
+        parts = [cs.describe(tr, nshards=world, shard=s) for s in range(world)]
+        whole = cs.describe(tr)
+        part_ok = (sum(p["shard_granules"] for p in parts) == whole["shard_granules"] and
+                   sum(p["tracked_bytes_shard"] for p in parts) == whole["tracked_bytes"])
+        if rank == 0:
+            runs, n = out
+            merged = cs.report_merge(runs, n)
+            q.put(dict(ok=bool(np.array_equal(merged.runs, ref["runs"].astype(merged.runs.dtype))
+                               and merged.n_race_granules == ref["n_race_granules"]
+                               and merged.n_runs == ref["n_runs"] and ref["n_runs"] > 0),
+                       part_ok=part_ok, split_runs=len(runs)))
+        else:
+            q.put(dict(ok=out is None, part_ok=part_ok))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_two_rank_gather_and_stitch():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert all(r["ok"] for r in res), res
+    assert all(r["part_ok"] for r in res), res
+
+
+@pytest.mark.parametrize("nshards", [2, 3, 8])
+def test_shard_partition_balances_coverage(nshards):
+    import paper_conf_sc_huckzsjb24_b200 as cs
+    from tracegen import configs
+    w = configs.make(5, "small")
+    ops, args = w.arrays(False)
+    tr = cs.Trace(255)
+    cs.Lowering(tr).cusan_lower_program(ops, args)
+    whole = cs.describe(tr)
+    parts = [cs.describe(tr, nshards=nshards, shard=s) for s in range(nshards)]
+    assert sum(p["shard_granules"] for p in parts) == whole["shard_granules"]
+    assert sum(p["tracked_bytes_shard"] for p in parts) == whole["tracked_bytes"]
+    ideal = whole["tracked_bytes"] / nshards
+    # equal coverage weight up to one interval's granule boundary rounding
+    assert max(abs(p["tracked_bytes_shard"] - ideal) for p in parts) <= 0.01 * ideal + 8 * 1000

@@ -1,0 +1,185 @@
+"""GPU parity: the sm_100a path (through the C ABI) against the oracle, bit-exact.
+
+Integer work, so the bar is equality of the canonical run list and of the race-granule count
+(SURVEY.md §8(c) step 4).  Inputs come only from tracegen; expected values only from oracle/.
+"""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_sc_huckzsjb24_b200 as cs
+from tracegen import configs, fuzz
+from tracegen.program import EV_ACCESS
+
+import brute
+import listing_dsl
+
+pytestmark = pytest.mark.gpu
+
+
+def gpu_report(events, max_fibers=255, **kw):
+    tr = cs.Trace(max_fibers)
+    tr.cusan_trace_append_events(events)
+    return cs.check(tr, **kw)
+
+
+def assert_equal(rep, ref):
+    assert rep.n_race_granules == ref["n_race_granules"]
+    assert rep.n_runs == ref["n_runs"]
+    assert np.array_equal(rep.runs, ref["runs"].astype(rep.runs.dtype))
+
+
+def lower_product(ops, args):
+    tr = cs.Trace(255)
+    first = cs.Lowering(tr).cusan_lower_program(ops, args)
+    return tr, first
+
+
+# ---------------------------------------------------------------------------------------------
+LISTINGS = listing_dsl.parse()
+
+
+@pytest.mark.parametrize("lst", LISTINGS, ids=[l.name for l in LISTINGS])
+def test_listing_on_gpu(lst):
+    ops, args = lst.program.arrays()
+    tr, first = lower_product(ops, args)
+    ev = tr.cusan_trace_read()
+    rep = cs.check(tr)
+    got = listing_dsl.observed_pairs(rep.runs, listing_dsl.label_events(lst, ev, list(first)))
+    assert set(got) == {(a, b) for a, b, _ in lst.expect}
+    assert_equal(rep, oracle.check_events(ev, 256, threads=1))
+
+
+@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_FORCE_LANES], ids=["ranges", "lanes"])
+@pytest.mark.parametrize("window", [0, 1, 2, 7])
+def test_fuzz_primitive_traces(window, flags):
+    """Random traces spanning several lane steps (128 granules) with ragged tails; both the
+    equal-cells range path and the lane-parallel path."""
+    rng = np.random.default_rng(40 + window)
+    for i in range(60):
+        nf = int(rng.integers(2, 9))
+        ev = fuzz.random_primitive_trace(rng, int(rng.integers(1, 80)), nf, n_keys=3,
+                                         n_granules=int(rng.integers(1, 1500)), unaligned=bool(i % 3 == 0))
+        rep = gpu_report(ev, nf, window_events=window, flags=flags)
+        assert_equal(rep, oracle.check_events(ev, nf, threads=2))
+
+
+def test_spill_path_many_readers():
+    """More than three reader fibers between writes exercises the exact spill slots."""
+    rng = np.random.default_rng(77)
+    hit_spill = 0
+    for i in range(40):
+        nf = int(rng.integers(5, 40))
+        ev = fuzz.random_primitive_trace(rng, int(rng.integers(20, 200)), nf, n_keys=4,
+                                         n_granules=int(rng.integers(50, 700)), p_access=0.8)
+        # mostly reads: flip 75% of writes to reads
+        acc = ev["kind"] == EV_ACCESS
+        flip = acc & (rng.random(len(ev)) < 0.75)
+        ev["mode"][flip] = 0
+        ref = oracle.check_events(ev, nf, threads=2)
+        for window in (0, 3):
+            for flags in (0, cs.CUSAN_CHECK_FORCE_LANES):
+                rep = gpu_report(ev, nf, window_events=window, flags=flags)
+                assert_equal(rep, ref)
+                hit_spill += rep.counters["spill_spans"] > 0
+    assert hit_spill > 0
+
+
+@pytest.mark.parametrize("nshards", [2, 3, 5])
+def test_shards_merge_to_the_whole(nshards):
+    rng = np.random.default_rng(5 + nshards)
+    for _ in range(20):
+        nf = int(rng.integers(2, 7))
+        ev = fuzz.random_primitive_trace(rng, int(rng.integers(5, 80)), nf, n_keys=3,
+                                         n_granules=int(rng.integers(100, 2000)))
+        parts = [gpu_report(ev, nf, nshards=nshards, shard=s) for s in range(nshards)]
+        runs = np.concatenate([p.runs for p in parts])
+        merged = cs.report_merge(runs, sum(p.n_race_granules for p in parts))
+        assert_equal(merged, oracle.check_events(ev, nf, threads=2))
+        whole = gpu_report(ev, nf)
+        assert sum(p.counters["shard_granules"] for p in parts) == whole.counters["shard_granules"]
+        assert sum(p.counters["tracked_bytes_shard"] for p in parts) == parts[0].counters["tracked_bytes"]
+
+
+@pytest.mark.parametrize("c", [1, 2, 3, 4, 5])
+@pytest.mark.parametrize("racy", [False, True])
+def test_small_configs(c, racy):
+    w = configs.make(c, "small")
+    ops, args = w.arrays(racy)
+    tr, _ = lower_product(ops, args)
+    ev = tr.cusan_trace_read()
+    ref = oracle.check_events(ev, 256)
+    for window in (0, 97):
+        for flags in (0, cs.CUSAN_CHECK_FORCE_LANES):
+            assert_equal(cs.check(tr, window_events=window, flags=flags), ref)
+    assert (ref["n_race_granules"] > 0) == racy
+
+
+def test_edge_cases():
+    # empty trace, trace without accesses, zero-length access
+    assert cs.check(cs.Trace(4)).n_race_granules == 0
+    t = cs.Trace(4)
+    t.cusan_trace_append_sync(cs.CUSAN_RELEASE, 0, 5)
+    assert cs.check(t).n_runs == 0
+    t = cs.Trace(4)
+    t.cusan_trace_append_access(0, 1, 0x1000, 0)
+    t.cusan_trace_append_access(1, 1, 0x1000, 0)
+    assert cs.check(t).n_race_granules == 0
+    # 255 fibers (the maximum), all reading one granule, then one write: 254 races, exact spill
+    t = cs.Trace(255)
+    for f in range(255):
+        t.cusan_trace_append_access(f, 0, 0x2000, 8)
+    t.cusan_trace_append_access(0, 1, 0x2000, 8)
+    ref = oracle.check_events(t.cusan_trace_read(), 255)
+    for window in (0, 1, 100):
+        for flags in (0, cs.CUSAN_CHECK_FORCE_LANES):
+            rep = cs.check(t, window_events=window, flags=flags)
+            assert rep.n_race_granules == 254
+            assert_equal(rep, ref)
+    # truncation keeps counts exact
+    rep = cs.check(t, max_runs=10)
+    assert rep.truncated and len(rep.runs) == 10 and rep.n_runs == 254 and rep.n_race_granules == 254
+
+
+def test_repeated_runs_of_a_plan_are_identical():
+    w = configs.make(3, "small")
+    ops, args = w.arrays(True)
+    tr, _ = lower_product(ops, args)
+    plan = cs.Plan(tr, window_events=50)
+    a, b = plan.run(), plan.run()
+    assert np.array_equal(a.runs, b.runs) and a.n_race_granules == b.n_race_granules
+    plan.close()
+
+
+def _sample_granules(rep_runs, ev, rng, n_random=1500):
+    acc = ev[ev["kind"] == EV_ACCESS]
+    g0 = (acc["a"] >> np.uint64(3)).astype(np.uint64)
+    g1 = ((acc["a"] + acc["b"] + np.uint64(7)) >> np.uint64(3)).astype(np.uint64)
+    pick = rng.integers(0, len(acc), n_random)
+    inner = g0[pick] + (rng.random(n_random) * (g1[pick] - g0[pick]).astype(np.float64)).astype(np.uint64)
+    s = [inner, g0[pick], g1[pick] - np.uint64(1)]
+    if len(rep_runs):
+        k = rng.integers(0, len(rep_runs), min(300, len(rep_runs)))
+        s += [rep_runs["g_begin"][k], rep_runs["g_end"][k] - np.uint64(1), rep_runs["g_end"][k]]
+    return np.unique(np.concatenate(s).astype(np.uint64))
+
+
+@pytest.mark.parametrize("c", [2, 3, 4, 5])
+def test_full_size_configs_sampled(c):
+    """BASELINE.json sizes, bench launch configuration; oracle on sampled granules (run edges,
+    access edges and random interior granules)."""
+    w = configs.make(c, "full")
+    ops, args = w.arrays(True)
+    tr, _ = lower_product(ops, args)
+    ev = tr.cusan_trace_read()
+    rep = cs.check(tr)
+    assert rep.n_race_granules > 0
+    assert rep.n_race_granules == int(np.sum(rep.runs["g_end"] - rep.runs["g_begin"]))
+    sample = _sample_granules(rep.runs, ev, np.random.default_rng(c))
+    ref = oracle.check_events(ev, 256, sample=sample)
+    sset = set(int(x) for x in sample)
+    got = {t for t in brute.runs_to_triples_in(rep.runs, sset)}
+    want = brute.runs_to_triples(ref["runs"])
+    assert got == want
