@@ -3,8 +3,8 @@
 // K1 shadow_check_window — one launch per window of consecutive access events.
 //   Shadow cell: 16 B per 8-byte granule {W, R0, R1, R2}, each u32 = fiber:8 | (event id + 1):24,
 //   0 = empty.  When more than three fibers have read since the last write,
-//   R2 holds SPILL_TAG | r: the readers beyond R0, R1 live in an immutable spill record r of the
-//   device heap ({n, epoch_1..epoch_n}), so the read set stays exact with a fixed 16-B cell.
+//   R2 holds SPILL_TAG | r: the readers beyond R0, R1 live in spill record r of the device heap
+//   ({header with n, epoch_1..epoch_n}), so the read set stays exact with a fixed 16-B cell.
 //   The per-granule rule is the FastTrack-style check of SURVEY.md §8(c) step 3:
 //       any access b:      W ≠ ∅ ∧ ¬HB(W, b)            → race (W, b)
 //       write b:           ∀ read r ≠ ∅ ∧ ¬HB(r, b)     → race (r, b);   W := b, R := ∅
@@ -20,7 +20,8 @@
 //             hit is a run over the whole range;
 //     pass 3  stream the final cell out (128-bit stores; skipped when no later window needs it).
 //   Ranges whose cells differ take the exact lane-parallel path: 32 lanes × 4 consecutive granules
-//   per step, each lane its own cell and spill record (copy-on-write), hits compacted in the warp
+//   per step, each lane its own cell and private spill record (shared records are copied before
+//   they are modified), hits compacted in the warp
 //   (__ballot_sync over hit lanes, __shfl_up_sync comparison with the left neighbour, run heads
 //   sized from the continuation mask).  Both paths feed a 32-entry per-warp run cache (one entry
 //   per lane) that extends runs across steps and ranges before appending them to global memory.
@@ -159,10 +160,17 @@ __device__ __forceinline__ bool same(const uint4& a, const uint4& b) {
     return ((a.x ^ b.x) | (a.y ^ b.y) | (a.z ^ b.z) | (a.w ^ b.w)) == 0u;
 }
 
-// ---- lane path: per-lane spill records, copy-on-write ------------------------------------------
-// allocate a record of n entries; returns the tagged slot value, or 0 on heap overflow (flagged)
-__device__ __forceinline__ uint32_t rec_alloc(const Ctx& k, uint32_t n, uint32_t** out) {
-    const uint32_t units = (n + 1 + REC_WORDS - 1) / REC_WORDS;
+// ---- lane path: per-granule spill records -------------------------------------------------------
+// Record header word: n (bits 0..15) | units (bits 16..23) | PRIVATE (bit 31).  Records written by
+// the range path are shared by every granule of a range (never modified in place); records the
+// lane path allocates belong to one granule's cell and are updated in place while they have room.
+constexpr uint32_t REC_PRIVATE = 0x80000000u;
+__device__ __forceinline__ uint32_t rec_n(uint32_t hdr) { return hdr & 0xffffu; }
+
+// allocate a private record with room for `cap` entries holding n; returns the tagged slot value,
+// or 0 on heap overflow (flagged; the host grows the heap and re-runs)
+__device__ __forceinline__ uint32_t rec_alloc(const Ctx& k, uint32_t n, uint32_t cap, uint32_t** out) {
+    const uint32_t units = (cap + 1 + REC_WORDS - 1) / REC_WORDS;
     const unsigned long long at = atomicAdd(&k.counters[C_HEAP], (unsigned long long)units);
     if (at + units > k.heap_cap) {
         k.counters[C_HEAP_OVF] = 1ull;
@@ -170,7 +178,7 @@ __device__ __forceinline__ uint32_t rec_alloc(const Ctx& k, uint32_t n, uint32_t
         return 0;
     }
     *out = k.heap + at * REC_WORDS;
-    (*out)[0] = n;
+    (*out)[0] = REC_PRIVATE | (units << 16) | n;
     return SPILL_TAG | (uint32_t)at;
 }
 
@@ -184,18 +192,24 @@ __device__ void lane_read_update(uint4& c, uint32_t ep, uint32_t f, const Ctx& k
     if (!c.w) { c.w = ep; return; }
     uint32_t* dst;
     if (!is_spill(c.w)) {                      // fourth reader: record {R2, ep}
-        const uint32_t v = rec_alloc(k, 2, &dst);
+        const uint32_t v = rec_alloc(k, 2, 2 * REC_WORDS - 1, &dst);
         if (dst) { dst[1] = c.w; dst[2] = ep; }
         c.w = v;
         return;
     }
-    const uint32_t* src = rec_ptr(k, c.w);
-    const uint32_t n = src[0];
+    uint32_t* src = rec_ptr(k, c.w);
+    const uint32_t hdr = src[0];
+    const uint32_t n = rec_n(hdr);
     int pos = -1;
     for (uint32_t j = 0; j < n; j++)
         if ((src[1 + j] >> 24) == f) { pos = (int)j; break; }
     if (pos >= 0 && src[1 + pos] == ep) return;
-    const uint32_t v = rec_alloc(k, pos >= 0 ? n : n + 1, &dst);   // copy-on-write
+    if (hdr & REC_PRIVATE) {                   // this granule's own record: update in place
+        const uint32_t cap = ((hdr >> 16) & 0xffu) * REC_WORDS - 1;
+        if (pos >= 0) { src[1 + pos] = ep; return; }
+        if (n < cap) { src[1 + n] = ep; src[0] = hdr + 1; return; }
+    }
+    const uint32_t v = rec_alloc(k, pos >= 0 ? n : n + 1, 2 * (n + 1), &dst);   // copy, with room
     if (dst) {
         for (uint32_t j = 0; j < n; j++) dst[1 + j] = src[1 + j];
         if (pos >= 0) dst[1 + pos] = ep; else dst[1 + n] = ep;
@@ -231,14 +245,21 @@ __device__ void check_lanes(const DSpan& sp, uint64_t x0, uint64_t n, int lane, 
                     emit(valid[c] && unordered(cell[c].z, f, row), cell[c].z, later, g, lane, rc, k);
                     const bool sp_w = valid[c] && is_spill(cell[c].w);
                     emit(valid[c] && !sp_w && unordered(cell[c].w, f, row), cell[c].w, later, g, lane, rc, k);
-                    const uint32_t* rp = sp_w ? rec_ptr(k, cell[c].w) : nullptr;
-                    const uint32_t nr = sp_w ? rp[0] : 0u;
+                    uint32_t* rp = sp_w ? rec_ptr(k, cell[c].w) : nullptr;
+                    const uint32_t nr = sp_w ? rec_n(rp[0]) : 0u;
                     const uint32_t nmax = __reduce_max_sync(FULL, nr);
                     for (uint32_t j = 0; j < nmax; j++) {
                         const uint32_t v = j < nr ? rp[1 + j] : 0u;
                         emit(unordered(v, f, row), v, later, g, lane, rc, k);
                     }
-                    cell[c] = make_uint4(r.epoch, 0, 0, 0);
+                    // R := ∅.  A private record stays attached, emptied, for this granule's next
+                    // readers (a spilled cell with n = 0 is the empty read set); shared ones detach.
+                    uint32_t keep = 0;
+                    if (sp_w && (rp[0] & REC_PRIVATE)) {
+                        rp[0] &= ~0xffffu;
+                        keep = cell[c].w;
+                    }
+                    cell[c] = make_uint4(r.epoch, 0, 0, keep);
                 } else if (valid[c]) {
                     lane_read_update(cell[c], r.epoch, f, k);
                 }
@@ -327,7 +348,7 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
             if (c.w) {
                 if (is_spill(c.w)) {
                     const uint32_t* rp = rec_ptr(k, c.w);
-                    ns = rp[0];
+                    ns = rec_n(rp[0]);
                     for (uint32_t j = lane; j < ns; j += 32) lst[j] = rp[1 + j];
                 } else {
                     if (lane == 0) lst[0] = c.w;
@@ -384,7 +405,7 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                         v = SPILL_TAG | sp.rec;
                         dst = k.heap + (uint64_t)sp.rec * REC_WORDS;
                     } else {
-                        if (lane == 0) v = rec_alloc(k, ns, &dst);
+                        if (lane == 0) v = rec_alloc(k, ns, ns, &dst);
                         v = __shfl_sync(FULL, v, 0);
                         dst = v ? rec_ptr(k, v) : nullptr;
                     }
