@@ -1,10 +1,11 @@
 // Device part of the check (steps a3, a4) and the plan / check C ABI.
 //
 // K1 shadow_check_window — one launch per window of consecutive access events.
-//   Shadow cell: 16 B per 8-byte granule {W, R0, R1, R2}, each u32 = fiber:8 | (event id + 1):24,
-//   0 = empty.  When more than three fibers have read since the last write,
-//   R2 holds SPILL_TAG | r: the readers beyond R0, R1 live in spill record r of the device heap
-//   ({header with n, epoch_1..epoch_n}), so the read set stays exact with a fixed 16-B cell.
+//   Shadow cell: 8 B per 8-byte granule {W, R} (FastTrack's representation: the last write as an
+//   epoch, the reads as an epoch while one fiber reads, a read vector when several do), each u32 =
+//   fiber:8 | (event id + 1):24, 0 = empty.  When two or more fibers have read since the last
+//   write, R = SPILL_TAG | r names a read-set record r in the device heap ({header with n,
+//   epoch_1..epoch_n}), so the read set stays exact with a fixed 8-B cell.
 //   The per-granule rule is the FastTrack-style check of SURVEY.md §8(c) step 3:
 //       any access b:      W ≠ ∅ ∧ ¬HB(W, b)            → race (W, b)
 //       write b:           ∀ read r ≠ ∅ ∧ ¬HB(r, b)     → race (r, b);   W := b, R := ∅
@@ -13,18 +14,18 @@
 //   Work unit = a warp range: consecutive granules of one elementary interval, all covered by the
 //   same accesses of the window.  Warps own contiguous runs of ranges (coverage-weighted).
 //   Per range:
-//     pass 1  stream the cells in (coalesced 128-bit loads, 8 in flight per lane) and vote whether
-//             they are all equal (skipped in the interval's first window: known empty);
+//     pass 1  stream the cells in (coalesced 128-bit loads = 2 cells, 8 in flight per lane) and vote
+//             whether they are all equal (skipped in the interval's first window: known empty);
 //     pass 2  equal cells evolve identically under the same accesses, so the warp applies the
-//             window's accesses once to the common cell (spilled readers in shared memory); each
-//             hit is a run over the whole range;
+//             window's accesses once to the common cell (the read set in shared memory); each hit
+//             is a run over the whole range;
 //     pass 3  stream the final cell out (128-bit stores; skipped when no later window needs it).
 //   Ranges whose cells differ take the exact lane-parallel path: 32 lanes × 4 consecutive granules
-//   per step, each lane its own cell and private spill record (shared records are copied before
-//   they are modified), hits compacted in the warp
-//   (__ballot_sync over hit lanes, __shfl_up_sync comparison with the left neighbour, run heads
-//   sized from the continuation mask).  Both paths feed a 32-entry per-warp run cache (one entry
-//   per lane) that extends runs across steps and ranges before appending them to global memory.
+//   per step, each lane its own cell and private read-set record (shared records are copied before
+//   they are modified), hits compacted in the warp (__ballot_sync over hit lanes, __shfl_up_sync
+//   comparison with the left neighbour, run heads sized from the continuation mask).  Both paths
+//   feed a 32-entry per-warp run cache (one entry per lane) that extends runs across steps and
+//   ranges before appending them to global memory.
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -44,8 +45,9 @@ constexpr int CHUNK = 32 * U;           // granules per lane-parallel step
 constexpr int UL = 8;                   // 16-B loads / stores in flight per lane when streaming
 constexpr int WARPS = 8;                // warps per block
 constexpr int THREADS = 32 * WARPS;
-constexpr int MAXS = 256;               // shared-memory spill list per warp (≥ 255 − 2 readers)
+constexpr int MAXS = 256;               // shared-memory read set per warp (≥ 255 readers)
 constexpr unsigned FULL = 0xffffffffu;
+static_assert(CHUNK % CELL_ALIGN == 0, "ranges start on aligned shadow slots");
 
 // counters[]: 0 race granules, 1 raw runs, 2 heap top (record units), 3 heap overflow flag
 enum { C_RACE = 0, C_RUNS = 1, C_HEAP = 2, C_HEAP_OVF = 3, N_COUNTERS = 4 };
@@ -63,7 +65,7 @@ struct Ctx {                     // kernel-wide pointers
     const AccRec* __restrict__ inc;
     const uint32_t* __restrict__ segvc;
     uint32_t F;
-    uint4* __restrict__ shadow;
+    uint2* __restrict__ shadow;
     uint32_t* __restrict__ heap;
     unsigned long long heap_cap;  // record units
     cusan_race_run* __restrict__ runs;
@@ -156,11 +158,7 @@ __device__ __forceinline__ bool unordered(uint32_t e, uint32_t f, const uint32_t
     return g != f && (e & 0xffffffu) > __ldg(row + g);
 }
 
-__device__ __forceinline__ bool same(const uint4& a, const uint4& b) {
-    return ((a.x ^ b.x) | (a.y ^ b.y) | (a.z ^ b.z) | (a.w ^ b.w)) == 0u;
-}
-
-// ---- lane path: per-granule spill records -------------------------------------------------------
+// ---- lane path: per-granule read-set records ----------------------------------------------------
 // Record header word: n (bits 0..15) | units (bits 16..23) | PRIVATE (bit 31).  Records written by
 // the range path are shared by every granule of a range (never modified in place); records the
 // lane path allocates belong to one granule's cell and are updated in place while they have room.
@@ -183,21 +181,17 @@ __device__ __forceinline__ uint32_t rec_alloc(const Ctx& k, uint32_t n, uint32_t
 }
 
 // R[f] := ep on one lane's cell
-__device__ void lane_read_update(uint4& c, uint32_t ep, uint32_t f, const Ctx& k) {
-    if (c.y && (c.y >> 24) == f) { c.y = ep; return; }
-    if (c.z && (c.z >> 24) == f) { c.z = ep; return; }
-    if (c.w && !is_spill(c.w) && (c.w >> 24) == f) { c.w = ep; return; }
+__device__ void lane_read_update(uint2& c, uint32_t ep, uint32_t f, const Ctx& k) {
     if (!c.y) { c.y = ep; return; }
-    if (!c.z) { c.z = ep; return; }
-    if (!c.w) { c.w = ep; return; }
     uint32_t* dst;
-    if (!is_spill(c.w)) {                      // fourth reader: record {R2, ep}
-        const uint32_t v = rec_alloc(k, 2, 2 * REC_WORDS - 1, &dst);
-        if (dst) { dst[1] = c.w; dst[2] = ep; }
-        c.w = v;
+    if (!is_spill(c.y)) {
+        if ((c.y >> 24) == f) { c.y = ep; return; }
+        const uint32_t v = rec_alloc(k, 2, 2 * REC_WORDS - 1, &dst);   // second reader: {R, ep}
+        if (dst) { dst[1] = c.y; dst[2] = ep; }
+        c.y = v;
         return;
     }
-    uint32_t* src = rec_ptr(k, c.w);
+    uint32_t* src = rec_ptr(k, c.y);
     const uint32_t hdr = src[0];
     const uint32_t n = rec_n(hdr);
     int pos = -1;
@@ -214,19 +208,19 @@ __device__ void lane_read_update(uint4& c, uint32_t ep, uint32_t f, const Ctx& k
         for (uint32_t j = 0; j < n; j++) dst[1 + j] = src[1 + j];
         if (pos >= 0) dst[1 + pos] = ep; else dst[1 + n] = ep;
     }
-    c.w = v;
+    c.y = v;
 }
 
 // Lane-parallel exact path for granules [x0, x0 + n) of span sp (each lane its own cells).
 __device__ void check_lanes(const DSpan& sp, uint64_t x0, uint64_t n, int lane, RunCache& rc, const Ctx& k) {
     for (uint64_t xc = x0; xc < x0 + n; xc += CHUNK) {
-        uint4 cell[U];
+        uint2 cell[U];
         bool valid[U];
 #pragma unroll
         for (int c = 0; c < U; c++) {
             const uint64_t x = xc + c * 32 + lane;
             valid[c] = x < x0 + n;
-            cell[c] = make_uint4(0, 0, 0, 0);
+            cell[c] = make_uint2(0, 0);
             if (valid[c] && (sp.flags & SPAN_LOAD)) cell[c] = __ldcs(k.shadow + sp.dense_begin + x);
         }
         const uint32_t qe = sp.list_off + sp.list_cnt;
@@ -241,25 +235,23 @@ __device__ void check_lanes(const DSpan& sp, uint64_t x0, uint64_t n, int lane, 
                 const uint64_t g = sp.abs_begin + xc + c * 32 + lane;
                 emit(valid[c] && unordered(cell[c].x, f, row), cell[c].x, later, g, lane, rc, k);
                 if (wr) {
-                    emit(valid[c] && unordered(cell[c].y, f, row), cell[c].y, later, g, lane, rc, k);
-                    emit(valid[c] && unordered(cell[c].z, f, row), cell[c].z, later, g, lane, rc, k);
-                    const bool sp_w = valid[c] && is_spill(cell[c].w);
-                    emit(valid[c] && !sp_w && unordered(cell[c].w, f, row), cell[c].w, later, g, lane, rc, k);
-                    uint32_t* rp = sp_w ? rec_ptr(k, cell[c].w) : nullptr;
-                    const uint32_t nr = sp_w ? rec_n(rp[0]) : 0u;
+                    const bool sp_r = valid[c] && is_spill(cell[c].y);
+                    emit(valid[c] && !sp_r && unordered(cell[c].y, f, row), cell[c].y, later, g, lane, rc, k);
+                    uint32_t* rp = sp_r ? rec_ptr(k, cell[c].y) : nullptr;
+                    const uint32_t nr = sp_r ? rec_n(rp[0]) : 0u;
                     const uint32_t nmax = __reduce_max_sync(FULL, nr);
                     for (uint32_t j = 0; j < nmax; j++) {
                         const uint32_t v = j < nr ? rp[1 + j] : 0u;
                         emit(unordered(v, f, row), v, later, g, lane, rc, k);
                     }
                     // R := ∅.  A private record stays attached, emptied, for this granule's next
-                    // readers (a spilled cell with n = 0 is the empty read set); shared ones detach.
+                    // readers (a record with n = 0 is the empty read set); shared ones detach.
                     uint32_t keep = 0;
-                    if (sp_w && (rp[0] & REC_PRIVATE)) {
+                    if (sp_r && (rp[0] & REC_PRIVATE)) {
                         rp[0] &= ~0xffffu;
-                        keep = cell[c].w;
+                        keep = cell[c].y;
                     }
-                    cell[c] = make_uint4(r.epoch, 0, 0, keep);
+                    cell[c] = make_uint2(r.epoch, keep);
                 } else if (valid[c]) {
                     lane_read_update(cell[c], r.epoch, f, k);
                 }
@@ -322,19 +314,27 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
             const DSpan sp = spans[s];
             const uint64_t x0 = (t - sp.tile0) * sp.rsize;
             const uint64_t n = min((uint64_t)sp.rsize, sp.len - x0);
-            uint4* cells = k.shadow + sp.dense_begin + x0;
+            uint2* cells = k.shadow + sp.dense_begin + x0;      // 256-B aligned (CELL_ALIGN)
+            const uint4* cells2 = reinterpret_cast<const uint4*>(cells);
+            const uint64_t n2 = n >> 1;                         // cell pairs
             // ---- pass 1: stream the range's cells in and vote that they are all equal ----------
-            uint4 c = make_uint4(0, 0, 0, 0);      // first window of the interval: known empty
+            uint2 c = make_uint2(0, 0);            // first window of the interval: known empty
             bool uniform = !force_lanes;
             if (uniform && (sp.flags & SPAN_LOAD)) {
                 c = cells[0];
                 bool ok = true;
-                for (uint64_t i = lane; i < n; i += 32 * UL) {
+                for (uint64_t i = lane; i < n2; i += 32 * UL) {
                     uint4 v[UL];
 #pragma unroll
-                    for (int u = 0; u < UL; u++) v[u] = (i + u * 32 < n) ? __ldcs(cells + i + u * 32) : c;
+                    for (int u = 0; u < UL; u++)
+                        v[u] = (i + u * 32 < n2) ? __ldcs(cells2 + i + u * 32) : make_uint4(c.x, c.y, c.x, c.y);
 #pragma unroll
-                    for (int u = 0; u < UL; u++) ok &= same(v[u], c);
+                    for (int u = 0; u < UL; u++)
+                        ok &= ((v[u].x ^ c.x) | (v[u].y ^ c.y) | (v[u].z ^ c.x) | (v[u].w ^ c.y)) == 0u;
+                }
+                if ((n & 1) && lane == 0) {
+                    const uint2 tl = __ldcs(cells + n - 1);
+                    ok &= tl.x == c.x && tl.y == c.y;
                 }
                 uniform = __all_sync(FULL, ok);
             }
@@ -343,18 +343,17 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                 continue;
             }
             // ---- pass 2: all cells of the range equal `c`: apply the window's accesses once -----
-            // readers beyond R0, R1 are kept as a list in shared memory (ns entries)
+            // the read set is kept in shared memory (ns entries); c.x = W
             uint32_t ns = 0;
-            if (c.w) {
-                if (is_spill(c.w)) {
-                    const uint32_t* rp = rec_ptr(k, c.w);
+            if (c.y) {
+                if (is_spill(c.y)) {
+                    const uint32_t* rp = rec_ptr(k, c.y);
                     ns = rec_n(rp[0]);
                     for (uint32_t j = lane; j < ns; j += 32) lst[j] = rp[1 + j];
                 } else {
-                    if (lane == 0) lst[0] = c.w;
+                    if (lane == 0) lst[0] = c.y;
                     ns = 1;
                 }
-                c.w = 0;
                 __syncwarp();
             }
             const uint64_t gb = sp.abs_begin + x0, ge = gb + n;
@@ -368,18 +367,12 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                 const uint32_t* row = k.segvc + (uint64_t)(r.segm & 0x7fffffffu) * k.F;
                 emit_range(unordered(c.x, f, row), c.x, later, gb, ge, lane, rc, k);
                 if (r.segm >> 31) {
-                    emit_range(unordered(c.y, f, row), c.y, later, gb, ge, lane, rc, k);
-                    emit_range(unordered(c.z, f, row), c.z, later, gb, ge, lane, rc, k);
                     for (uint32_t j = 0; j < ns; j++) {
                         const uint32_t v = lst[j];
                         emit_range(unordered(v, f, row), v, later, gb, ge, lane, rc, k);
                     }
-                    c = make_uint4(r.epoch, 0, 0, 0);
+                    c.x = r.epoch;
                     ns = 0;
-                } else if (c.y && (c.y >> 24) == f) {
-                    c.y = r.epoch;
-                } else if (c.z && (c.z >> 24) == f) {
-                    c.z = r.epoch;
                 } else {
                     int pos = -1;
                     for (uint32_t b = 0; b < ns; b += 32) {
@@ -387,18 +380,18 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                         const unsigned m = __ballot_sync(FULL, j < ns && (lst[j] >> 24) == f);
                         if (m) { pos = (int)(b + __ffs(m) - 1); break; }
                     }
-                    if (pos >= 0) { if (lane == 0) lst[pos] = r.epoch; }
-                    else if (!c.y) c.y = r.epoch;
-                    else if (!c.z) c.z = r.epoch;
-                    else { if (lane == 0) lst[ns] = r.epoch; ns++; }
+                    if (lane == 0) lst[pos >= 0 ? pos : ns] = r.epoch;
+                    if (pos < 0) ns++;
                     __syncwarp();
                 }
             }
             // ---- pass 3: stream the final cell out -----------------------------------------------
             if (sp.flags & SPAN_STORE) {
-                if (ns == 1) {
-                    c.w = lst[0];
-                } else if (ns > 1) {
+                if (ns == 0) {
+                    c.y = 0;
+                } else if (ns == 1) {
+                    c.y = lst[0];
+                } else {
                     uint32_t* dst = nullptr;
                     uint32_t v = 0;
                     if (ns + 1 <= sp.rec_units * REC_WORDS) {      // the span's pre-assigned record
@@ -410,16 +403,19 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                         dst = v ? rec_ptr(k, v) : nullptr;
                     }
                     if (dst) {
-                        if (lane == 0) dst[0] = ns;
+                        if (lane == 0) dst[0] = ns;                 // shared: no PRIVATE bit
                         for (uint32_t j = lane; j < ns; j += 32) dst[1 + j] = lst[j];
                     }
-                    c.w = v;
+                    c.y = v;
                 }
-                for (uint64_t i = lane; i < n; i += 32 * UL) {
+                uint4* out2 = reinterpret_cast<uint4*>(cells);
+                const uint4 cc = make_uint4(c.x, c.y, c.x, c.y);
+                for (uint64_t i = lane; i < n2; i += 32 * UL) {
 #pragma unroll
                     for (int u = 0; u < UL; u++)
-                        if (i + u * 32 < n) __stcs(cells + i + u * 32, c);
+                        if (i + u * 32 < n2) __stcs(out2 + i + u * 32, cc);
                 }
+                if ((n & 1) && lane == 0) __stcs(cells + n - 1, c);
             }
             __syncwarp();
         }
@@ -463,7 +459,7 @@ struct cusan_plan {
     uint32_t* d_segvc = nullptr;
     DSpan* d_spans = nullptr;
     unsigned long long* d_counters = nullptr;
-    uint4* d_shadow = nullptr;
+    uint2* d_shadow = nullptr;
     uint32_t* d_heap = nullptr;
     uint64_t heap_cap = 0;                  // record units
     uint32_t* d_heap_own = nullptr;         // grown heap after an overflow
@@ -539,7 +535,7 @@ static int plan_device_setup(cusan_plan* p) {
             tiles += nt;
             weight += nt * d.rweight;
             if (s.flags) p->need_shadow = true;
-            p->shadow_cell_bytes += s.len * (((s.flags & SPAN_LOAD) ? 16 : 0) + ((s.flags & SPAN_STORE) ? 16 : 0));
+            p->shadow_cell_bytes += s.len * (((s.flags & SPAN_LOAD) ? 8 : 0) + ((s.flags & SPAN_STORE) ? 8 : 0));
             ds.push_back(d);
         }
         win.nspans = (uint32_t)(ds.size() - win.span_off);
@@ -562,7 +558,7 @@ static int plan_device_setup(cusan_plan* p) {
     const uint64_t o_spans = off;   off = align_up(off + ds.size() * sizeof(DSpan));
     const uint64_t o_cnt = off;     off = align_up(off + N_COUNTERS * sizeof(unsigned long long));
     const uint64_t o_heap = off;    off = align_up(off + p->heap_cap * REC_WORDS * sizeof(uint32_t));
-    const uint64_t o_shadow = off;  off = align_up(off + (p->need_shadow ? hp.shard_granules * 16 : 0));
+    const uint64_t o_shadow = off;  off = align_up(off + (p->need_shadow ? hp.shadow_cells * sizeof(uint2) : 0));
     p->run_cap = std::max<uint64_t>(1ull << 16, 4 * p->wins.size() + 1024);
     const uint64_t o_runs = off;    off = align_up(off + p->run_cap * sizeof(cusan_race_run));
     p->ws_bytes = off;
@@ -580,7 +576,7 @@ static int plan_device_setup(cusan_plan* p) {
     p->d_spans = (DSpan*)(p->ws + o_spans);
     p->d_counters = (unsigned long long*)(p->ws + o_cnt);
     p->d_heap = (uint32_t*)(p->ws + o_heap);
-    p->d_shadow = p->need_shadow ? (uint4*)(p->ws + o_shadow) : nullptr;
+    p->d_shadow = p->need_shadow ? (uint2*)(p->ws + o_shadow) : nullptr;
     p->d_runs = (cusan_race_run*)(p->ws + o_runs);
     CK(cudaMemcpyAsync(p->d_inc, hp.inc.data(), hp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, p->stream));
     CK(cudaMemcpyAsync(p->d_segvc, hp.segvc.data(), hp.segvc.size() * sizeof(uint32_t), cudaMemcpyHostToDevice, p->stream));
@@ -589,7 +585,7 @@ static int plan_device_setup(cusan_plan* p) {
     CK(cudaEventCreate(&p->ev0));
     CK(cudaEventCreate(&p->ev1));
     CK(cudaStreamSynchronize(p->stream));
-    hp.ctr.shadow_bytes = p->need_shadow ? hp.shard_granules * 16 : 0;
+    hp.ctr.shadow_bytes = p->need_shadow ? hp.shadow_cells * sizeof(uint2) : 0;
     hp.ctr.workspace_bytes = p->ws_bytes;
     return CUSAN_OK;
 }

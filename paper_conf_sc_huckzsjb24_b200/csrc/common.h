@@ -18,12 +18,15 @@ struct Trace {
 };
 
 // ----------------------------------------------------------------------------------------------
-// Shadow slot encoding: u32 = fiber:8 | (event id + 1):24, 0 = empty.
-// Fiber 0xFF is reserved: in a cell's third read slot, 0xFF:24-bit index tags a spill record.
+// Shadow cell (FastTrack's epoch / read-VC representation): 8 B per granule
+// {W, R}, each u32 = fiber:8 | (event id + 1):24, 0 = empty.  R is the single reader's epoch, or —
+// when two or more fibers have read since the last write — 0xFF:24-bit index of a read-set record
+// (fiber 0xFF is reserved for this tag).
 // ----------------------------------------------------------------------------------------------
 inline uint32_t pack_epoch(uint32_t fiber, uint32_t event_id) { return (fiber << 24) | (event_id + 1); }
 constexpr uint32_t SPILL_TAG = 0xFF000000u;
-constexpr uint32_t REC_WORDS = 8;        // spill-record allocation unit (u32 words)
+constexpr uint32_t REC_WORDS = 8;        // read-set record allocation unit (u32 words)
+constexpr uint64_t CELL_ALIGN = 32;      // interval shadow slots start on 32-cell (256-B) boundaries
 
 // Per access event, what the shadow kernel needs (8 B, one per interval incidence):
 //   epoch  = pack_epoch(fiber, event id)
@@ -69,8 +72,9 @@ struct HostPlan {
     std::vector<Interval> iv;             // shard-clipped intervals (len > 0)
     std::vector<AccRec> inc;              // incidence table: per interval, its accesses in trace order
     std::vector<uint32_t> inc_acc;        // access index of each incidence
-    uint64_t shard_granules = 0;
-    uint64_t rec_units = 0;               // pre-assigned spill-record units
+    uint64_t shard_granules = 0;          // covered granules in this shard
+    uint64_t shadow_cells = 0;            // shadow slots incl. alignment padding
+    uint64_t rec_units = 0;               // pre-assigned read-set record units
     uint64_t spill_spans = 0;
     // windows
     std::vector<Span> spans;              // all windows, window-major

@@ -197,28 +197,32 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp) {
         d_lo = boundary(o.shard);
         d_hi = boundary(o.shard + 1);
     }
+    // shard-local shadow slots: each clipped interval starts on a CELL_ALIGN boundary so warp
+    // ranges can move their cells with aligned 128-bit accesses (≤ CELL_ALIGN−1 unused cells each)
     hp.iv.clear();
+    uint64_t slot = 0;
     for (auto& g : giv) {
         uint64_t lo = std::max(g.dense_begin, d_lo), hi = std::min(g.dense_begin + g.len, d_hi);
         if (lo >= hi) continue;
         Interval v{};
         v.abs_begin = g.abs_begin + (lo - g.dense_begin);
-        v.dense_begin = lo - d_lo;
+        v.dense_begin = slot;
         v.len = hi - lo;
         v.list_off = g.off;
         v.list_cnt = g.cnt;
+        slot = (slot + v.len + CELL_ALIGN - 1) / CELL_ALIGN * CELL_ALIGN;
         hp.iv.push_back(v);
         c.tracked_bytes_shard += 8 * v.len * g.cnt;
     }
     hp.shard_granules = d_hi - d_lo;
+    hp.shadow_cells = slot;
     c.shard_granules = hp.shard_granules;
 
     // ---------------------------------------------------------------- windows and spans ---------
-    // A span that stores its final cells and ends with more than three reader fibers since the
-    // interval's last write gets a pre-assigned spill record: the cell keeps W, R0, R1 inline and
-    // the third slot points at the record holding the other readers (the reader *set* depends only
-    // on the fibers and modes covering the interval, never on happens-before, so its size is known
-    // here exactly).
+    // A span that stores its final cells and ends with two or more reader fibers since the
+    // interval's last write gets a pre-assigned read-set record: the cell keeps W inline and its R
+    // slot points at the record holding the readers (the reader *set* depends only on the fibers
+    // and modes covering the interval, never on happens-before, so its size is known here exactly).
     const uint64_t W = o.window_events > 0 ? (uint64_t)o.window_events : std::max<uint64_t>(n_acc, 1);
     hp.window_accesses = W;
     const uint64_t nwin = n_acc ? (n_acc + W - 1) / W : 0;
@@ -245,9 +249,9 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp) {
             s.list_cnt = q2 - q;
             s.flags = (q > v.list_off ? SPAN_LOAD : 0u) | ((q2 < qe || o.persist_shadow) ? SPAN_STORE : 0u);
             const uint64_t nr = readers.count();
-            if ((s.flags & SPAN_STORE) && nr > 3) {
+            if ((s.flags & SPAN_STORE) && nr >= 2) {
                 s.rec = (uint32_t)hp.rec_units;
-                s.rec_units = (uint32_t)((nr - 2 + 1 + REC_WORDS - 1) / REC_WORDS);
+                s.rec_units = (uint32_t)((nr + 1 + REC_WORDS - 1) / REC_WORDS);
                 hp.rec_units += s.rec_units;
                 hp.spill_spans++;
             }
