@@ -44,6 +44,7 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=15.0, help="target oracle sample time")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"])
     return ap.parse_args()
 
 
@@ -211,10 +212,18 @@ def run_ours(args):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    # one rank per GPU; --dist-backend gloo lets several ranks share GPUs (testing the sharded
+    # path on a 1-GPU box: shards checked concurrently, runs gathered over gloo)
+    local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    comm_dev = dev
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
+            comm_dev = torch.device("cpu")
     stream = torch.cuda.current_stream(dev)
 
     w, ops, args_, wname = workload(args)
@@ -228,13 +237,14 @@ def run_ours(args):
     def max_over_ranks(x: float) -> float:
         if world == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        t = torch.tensor([x], dtype=torch.float64, device=comm_dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
-    kw = dict(window_events=args.window, device=local, stream=stream.cuda_stream)
+    # device memory for every plan comes from PyTorch's caching allocator
+    kw = dict(window_events=args.window, device=local, stream=stream.cuda_stream, workspace="torch")
     if world > 1:
-        plan = ShardedPlan(tr, comm_device=dev, **kw)
+        plan = ShardedPlan(tr, comm_device=comm_dev, **kw)
         run = plan.run
     else:
         plan = cs.Plan(tr, **kw)
@@ -283,7 +293,7 @@ def run_ours(args):
         t2 = cs.Trace(255)
         cs.Lowering(t2).cusan_lower_program(ops, args_)
         if world > 1:
-            p2 = ShardedPlan(t2, comm_device=dev, **kw)
+            p2 = ShardedPlan(t2, comm_device=comm_dev, **kw)
             r2 = p2.run()
             c2 = p2.last_shard_report.counters
             p2.close()
@@ -300,7 +310,7 @@ def run_ours(args):
     # ---- post-mortem variant (extra, for context): one window, no shadow traffic --------------------
     pm = None
     if world == 1:
-        p3 = cs.Plan(tr, window_events=0, device=local, stream=stream.cuda_stream)
+        p3 = cs.Plan(tr, window_events=0, device=local, stream=stream.cuda_stream, workspace="torch")
         p3.run()
         torch.cuda.synchronize(dev)
         t0 = time.perf_counter()

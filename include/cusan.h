@@ -115,6 +115,10 @@ typedef struct cusan_check_opts {
 /* Diagnostics: disable the equal-cells range path so every granule takes the lane-parallel
  * per-granule path (used by the parity tests to exercise both paths; results are identical). */
 #define CUSAN_CHECK_FORCE_LANES 1
+/* cusan_plan_create computes the plan but neither allocates nor uploads: the caller queries
+ * cusan_plan_workspace_bytes, allocates device memory (e.g. a torch tensor from PyTorch's caching
+ * allocator) and calls cusan_plan_bind_workspace before cusan_plan_run. */
+#define CUSAN_CHECK_DEFER_WORKSPACE 2
 
 /* Defaults: nshards 1, shard 0, device 0, window_events 0, persist 0, max_runs 0, all NULL. */
 void cusan_check_opts_init(cusan_check_opts* o);
@@ -125,8 +129,12 @@ int cusan_check(const cusan_trace* t, const cusan_check_opts* o, cusan_report** 
 /* Host preparation (a1, a2) and upload of the event / clock / interval tables to the device.
  * The trace must stay alive and unmodified while the plan exists. */
 int cusan_plan_create(const cusan_trace* t, const cusan_check_opts* o, cusan_plan** out);
-/* Device bytes the plan needs (tables + shadow + ext slots + run buffer). */
+/* Device bytes the plan needs (tables + shadow + read-set heap + run buffer). */
 int cusan_plan_workspace_bytes(const cusan_plan* p, uint64_t* bytes);
+/* Binds caller-owned device memory (>= cusan_plan_workspace_bytes, 256-B aligned, on the plan's
+ * device) to a plan created with CUSAN_CHECK_DEFER_WORKSPACE and uploads the tables.  The memory
+ * must stay valid until cusan_plan_destroy.  CUSAN_ESTATE if the plan owns a workspace. */
+int cusan_plan_bind_workspace(cusan_plan* p, void* workspace, uint64_t bytes);
 /* Device part (a3, a4) and the report (a5).  May be called repeatedly (each run starts from an
  * empty shadow); asynchronous work is complete when it returns. */
 int cusan_plan_run(cusan_plan* p, cusan_report** out);

@@ -170,16 +170,31 @@ def _report(h, max_runs):
     return Report(h, max_runs)
 
 
-class Plan:
-    """cusan_plan: host preparation (a1, a2) + device tables; run() does a3-a5 on the GPU."""
+CUSAN_CHECK_DEFER_WORKSPACE = 2
 
-    def __init__(self, trace: Trace, **kw):
+
+class Plan:
+    """cusan_plan: host preparation (a1, a2) + device tables; run() does a3-a5 on the GPU.
+
+    workspace="torch" takes the plan's device memory from PyTorch's caching allocator (a uint8
+    tensor held by the plan) instead of the library's own cudaMalloc."""
+
+    def __init__(self, trace: Trace, workspace: str | None = None, **kw):
         self.trace = trace            # must outlive the plan
         self.max_runs = kw.get("max_runs", 0)
+        self.workspace = None
+        if workspace == "torch":
+            kw["flags"] = kw.get("flags", 0) | CUSAN_CHECK_DEFER_WORKSPACE
         o = _opts(**kw)
         h = C.c_void_p()
         _ck(lib.cusan_plan_create(trace.h, C.byref(o), C.byref(h)))
         self.h = h
+        if workspace == "torch":
+            import torch
+            nbytes = self.workspace_bytes()
+            self.workspace = torch.empty(max(nbytes, 256), dtype=torch.uint8,
+                                         device=torch.device("cuda", kw.get("device", 0)))
+            _ck(lib.cusan_plan_bind_workspace(self.h, C.c_void_p(self.workspace.data_ptr()), nbytes))
 
     def workspace_bytes(self) -> int:
         b = C.c_uint64()
@@ -195,6 +210,7 @@ class Plan:
         if getattr(self, "h", None):
             lib.cusan_plan_destroy(self.h)
             self.h = None
+        self.workspace = None
 
     __del__ = close
 
@@ -207,9 +223,16 @@ def describe(trace: Trace, **kw) -> dict:
     return {n: getattr(ctr, n) for n, _ in cusan_counters._fields_}
 
 
-def check(trace: Trace, **kw) -> Report:
+def check(trace: Trace, workspace: str | None = None, **kw) -> Report:
     """cusan_check: plan + run + destroy.  kw: nshards, shard, device, window_events,
-    persist_shadow, max_runs, stream (a cudaStream_t as int, e.g. torch's current stream)."""
+    persist_shadow, max_runs, stream (a cudaStream_t as int, e.g. torch's current stream), flags;
+    workspace="torch" allocates the device memory through PyTorch."""
+    if workspace is not None:
+        p = Plan(trace, workspace=workspace, **kw)
+        try:
+            return p.run()
+        finally:
+            p.close()
     o = _opts(**kw)
     h = C.c_void_p()
     _ck(lib.cusan_check(trace.h, C.byref(o), C.byref(h)))

@@ -9,7 +9,7 @@ import ctypes as C
 import os
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libcusan.so")
+LIB_PATH = os.environ.get("CUSAN_LIBRARY", os.path.join(HERE, "libcusan.so"))
 
 
 class CusanError(RuntimeError):
@@ -79,6 +79,7 @@ PROTOS = {
     "cusan_check": [P, C.POINTER(cusan_check_opts), PP],
     "cusan_plan_create": [P, C.POINTER(cusan_check_opts), PP],
     "cusan_plan_workspace_bytes": [P, pu64],
+    "cusan_plan_bind_workspace": [P, P, u64],
     "cusan_plan_run": [P, PP],
     "cusan_plan_destroy": [P],
     "cusan_plan_describe": [P, C.POINTER(cusan_check_opts), C.POINTER(cusan_counters)],

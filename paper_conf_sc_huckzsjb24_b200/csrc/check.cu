@@ -42,7 +42,26 @@ namespace {
 
 constexpr int U = 4;                    // 32-granule chunks per lane-parallel step
 constexpr int CHUNK = 32 * U;           // granules per lane-parallel step
-constexpr int UL = 8;                   // 16-B loads / stores in flight per lane when streaming
+#ifndef CUSAN_UL
+#define CUSAN_UL 4
+#endif
+#ifndef CUSAN_MIN_BLOCKS
+#define CUSAN_MIN_BLOCKS 3
+#endif
+constexpr int UL = CUSAN_UL;            // 16-B loads / stores in flight per lane when streaming
+#ifndef CUSAN_DYNAMIC
+#define CUSAN_DYNAMIC 0
+#endif
+#ifndef CUSAN_RANGE_PER_ACCESS
+#define CUSAN_RANGE_PER_ACCESS 512
+#endif
+#ifndef CUSAN_RANGE_MIN
+#define CUSAN_RANGE_MIN 16384
+#endif
+#ifndef CUSAN_RANGE_MAX
+#define CUSAN_RANGE_MAX 262144
+#endif
+constexpr int GRAB = 2;                 // ranges a warp takes per dynamic-scheduler grab
 constexpr int WARPS = 8;                // warps per block
 constexpr int THREADS = 32 * WARPS;
 constexpr int MAXS = 256;               // shared-memory read set per warp (≥ 255 readers)
@@ -289,27 +308,47 @@ __device__ __forceinline__ uint64_t tile_at_weight(const DSpan* __restrict__ sp,
     return sp[lo].tile0 + (pos - sp[lo].weight0 + w - 1) / w;
 }
 
-__global__ void __launch_bounds__(THREADS, 3)
+__global__ void __launch_bounds__(THREADS, CUSAN_MIN_BLOCKS)
 shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t total_tiles,
-                    uint64_t total_weight, Ctx k, int force_lanes) {
+                    uint64_t total_weight, Ctx k, int force_lanes, unsigned long long* sched) {
     __shared__ uint32_t s_list[WARPS][MAXS];
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
     uint32_t* lst = s_list[warp];
-    const uint64_t nwarps = (uint64_t)gridDim.x * WARPS;
-    const uint64_t wid = (uint64_t)blockIdx.x * WARPS + warp;
-    const uint64_t t0 = tile_at_weight(spans, nspans, (uint64_t)((unsigned __int128)total_weight * wid / nwarps),
-                                       total_weight, total_tiles);
-    const uint64_t t1 = tile_at_weight(spans, nspans, (uint64_t)((unsigned __int128)total_weight * (wid + 1) / nwarps),
-                                       total_weight, total_tiles);
     RunCache rc;
     rc.e = rc.l = 0;
     rc.gb = rc.ge = 0;
     rc.rr = 0;
     rc.nrace = 0;
-    if (t0 < t1) {
-        uint32_t s = find_span_by_tile(spans, nspans, t0);
-        for (uint64_t t = t0; t < t1; t++) {
+    // Range assignment: with `sched`, warps grab GRAB consecutive ranges at a time from a per-launch
+    // counter (dynamic balance); without, each warp owns one coverage-weighted contiguous slice.
+    uint64_t tend = 0;
+    uint32_t s = 0;
+    bool first = true;
+    {
+        for (uint64_t t = 0;; t++) {
+            if (t >= tend) {
+                uint64_t b, e;
+                if (sched) {
+                    unsigned long long base = 0;
+                    if (lane == 0) base = atomicAdd(sched, (unsigned long long)GRAB);
+                    b = __shfl_sync(FULL, base, 0);
+                    e = min(b + (uint64_t)GRAB, total_tiles);
+                } else {
+                    if (!first) break;
+                    const uint64_t nwarps = (uint64_t)gridDim.x * WARPS;
+                    const uint64_t wid = (uint64_t)blockIdx.x * WARPS + warp;
+                    b = tile_at_weight(spans, nspans, (uint64_t)((unsigned __int128)total_weight * wid / nwarps),
+                                       total_weight, total_tiles);
+                    e = tile_at_weight(spans, nspans, (uint64_t)((unsigned __int128)total_weight * (wid + 1) / nwarps),
+                                       total_weight, total_tiles);
+                    first = false;
+                }
+                if (b >= e) break;
+                t = b;
+                tend = e;
+                s = find_span_by_tile(spans, nspans, t);
+            }
             while (t >= spans[s + 1].tile0) s++;   // spans[nspans] is a sentinel
             const DSpan sp = spans[s];
             const uint64_t x0 = (t - sp.tile0) * sp.rsize;
@@ -467,9 +506,13 @@ struct cusan_plan {
     cusan_race_run* d_runs_own = nullptr;   // grown run buffer after an overflow
     uint64_t run_cap = 0;
     bool need_shadow = false;
+    bool bound = false;                     // workspace carved and tables uploaded
+    uint64_t o_inc = 0, o_seg = 0, o_spans = 0, o_cnt = 0, o_heap = 0, o_shadow = 0, o_runs = 0;
+    std::vector<DSpan> ds;                  // device span tables (host copy, uploaded at bind)
     std::vector<Window> wins;
     uint64_t shadow_cell_bytes = 0;
     uint64_t table_bytes = 0;               // tables uploaded by plan_create
+    std::vector<unsigned long long> counter_init;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
 
     ~cusan_plan() {
@@ -480,6 +523,8 @@ struct cusan_plan {
         if (d_heap_own) cudaFree(d_heap_own);
     }
 };
+
+static int plan_bind(cusan_plan* p, char* ws, uint64_t bytes);
 
 static int plan_device_setup(cusan_plan* p) {
     HostPlan& hp = p->hp;
@@ -522,7 +567,9 @@ static int plan_device_setup(cusan_plan* p) {
             // spans that move no cells are one range each
             uint64_t rs;
             if (s.flags & (SPAN_LOAD | SPAN_STORE))
-                rs = std::min<uint64_t>(std::max<uint64_t>(64ull * s.list_cnt, 2048), 1ull << 16);
+                rs = std::min<uint64_t>(std::max<uint64_t>((uint64_t)CUSAN_RANGE_PER_ACCESS * s.list_cnt,
+                                                           (uint64_t)CUSAN_RANGE_MIN),
+                                        (uint64_t)CUSAN_RANGE_MAX);
             else
                 rs = std::max<uint64_t>(s.len, 1);
             rs = std::min<uint64_t>((rs + CHUNK - 1) / CHUNK * CHUNK, 1ull << 31);
@@ -556,44 +603,63 @@ static int plan_device_setup(cusan_plan* p) {
     const uint64_t o_inc = off;     off = align_up(off + hp.inc.size() * sizeof(AccRec));
     const uint64_t o_seg = off;     off = align_up(off + hp.segvc.size() * sizeof(uint32_t));
     const uint64_t o_spans = off;   off = align_up(off + ds.size() * sizeof(DSpan));
-    const uint64_t o_cnt = off;     off = align_up(off + N_COUNTERS * sizeof(unsigned long long));
+    const uint64_t o_cnt = off;     off = align_up(off + (N_COUNTERS + p->wins.size()) * sizeof(unsigned long long));
     const uint64_t o_heap = off;    off = align_up(off + p->heap_cap * REC_WORDS * sizeof(uint32_t));
     const uint64_t o_shadow = off;  off = align_up(off + (p->need_shadow ? hp.shadow_cells * sizeof(uint2) : 0));
     p->run_cap = std::max<uint64_t>(1ull << 16, 4 * p->wins.size() + 1024);
     const uint64_t o_runs = off;    off = align_up(off + p->run_cap * sizeof(cusan_race_run));
     p->ws_bytes = off;
-    if (o.workspace) {
-        if (o.workspace_bytes < off)
-            return fail(CUSAN_ENOMEM, "workspace too small: need " + std::to_string(off) + " bytes");
-        p->ws = (char*)o.workspace;
-    } else {
-        cudaError_t me = cudaMalloc((void**)&p->own, std::max<uint64_t>(off, ALIGN));
-        if (me != cudaSuccess) return fail(CUSAN_ENOMEM, std::string("cudaMalloc workspace: ") + cudaGetErrorString(me));
-        p->ws = p->own;
-    }
-    p->d_inc = (AccRec*)(p->ws + o_inc);
-    p->d_segvc = (uint32_t*)(p->ws + o_seg);
-    p->d_spans = (DSpan*)(p->ws + o_spans);
-    p->d_counters = (unsigned long long*)(p->ws + o_cnt);
-    p->d_heap = (uint32_t*)(p->ws + o_heap);
-    p->d_shadow = p->need_shadow ? (uint2*)(p->ws + o_shadow) : nullptr;
-    p->d_runs = (cusan_race_run*)(p->ws + o_runs);
-    CK(cudaMemcpyAsync(p->d_inc, hp.inc.data(), hp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, p->stream));
-    CK(cudaMemcpyAsync(p->d_segvc, hp.segvc.data(), hp.segvc.size() * sizeof(uint32_t), cudaMemcpyHostToDevice, p->stream));
-    CK(cudaMemcpyAsync(p->d_spans, ds.data(), ds.size() * sizeof(DSpan), cudaMemcpyHostToDevice, p->stream));
-    p->table_bytes = hp.inc.size() * sizeof(AccRec) + hp.segvc.size() * sizeof(uint32_t) + ds.size() * sizeof(DSpan);
-    CK(cudaEventCreate(&p->ev0));
-    CK(cudaEventCreate(&p->ev1));
-    CK(cudaStreamSynchronize(p->stream));
+    p->o_inc = o_inc;
+    p->o_seg = o_seg;
+    p->o_spans = o_spans;
+    p->o_cnt = o_cnt;
+    p->o_heap = o_heap;
+    p->o_shadow = o_shadow;
+    p->o_runs = o_runs;
+    p->ds = std::move(ds);
+    p->table_bytes = hp.inc.size() * sizeof(AccRec) + hp.segvc.size() * sizeof(uint32_t) +
+                     p->ds.size() * sizeof(DSpan);
     hp.ctr.shadow_bytes = p->need_shadow ? hp.shadow_cells * sizeof(uint2) : 0;
     hp.ctr.workspace_bytes = p->ws_bytes;
+    CK(cudaEventCreate(&p->ev0));
+    CK(cudaEventCreate(&p->ev1));
+    if (o.workspace) return plan_bind(p, (char*)o.workspace, o.workspace_bytes);
+    if (o.flags & CUSAN_CHECK_DEFER_WORKSPACE) return CUSAN_OK;   // caller binds later
+    cudaError_t me = cudaMalloc((void**)&p->own, std::max<uint64_t>(off, ALIGN));
+    if (me != cudaSuccess) return fail(CUSAN_ENOMEM, std::string("cudaMalloc workspace: ") + cudaGetErrorString(me));
+    return plan_bind(p, p->own, off);
+}
+
+// Carve the workspace and upload the tables (a2 -> HBM).
+static int plan_bind(cusan_plan* p, char* ws, uint64_t bytes) {
+    if (bytes < p->ws_bytes)
+        return fail(CUSAN_ENOMEM, "workspace too small: need " + std::to_string(p->ws_bytes) + " bytes");
+    const HostPlan& hp = p->hp;
+    CK(cudaSetDevice(p->device));
+    p->ws = ws;
+    p->d_inc = (AccRec*)(p->ws + p->o_inc);
+    p->d_segvc = (uint32_t*)(p->ws + p->o_seg);
+    p->d_spans = (DSpan*)(p->ws + p->o_spans);
+    p->d_counters = (unsigned long long*)(p->ws + p->o_cnt);
+    p->d_shadow = p->need_shadow ? (uint2*)(p->ws + p->o_shadow) : nullptr;
+    if (!p->d_runs_own) p->d_runs = (cusan_race_run*)(p->ws + p->o_runs);
+    if (!p->d_heap_own) p->d_heap = (uint32_t*)(p->ws + p->o_heap);
+    else p->d_heap = p->d_heap_own;
+    CK(cudaMemcpyAsync(p->d_inc, hp.inc.data(), hp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, p->stream));
+    CK(cudaMemcpyAsync(p->d_segvc, hp.segvc.data(), hp.segvc.size() * sizeof(uint32_t), cudaMemcpyHostToDevice, p->stream));
+    CK(cudaMemcpyAsync(p->d_spans, p->ds.data(), p->ds.size() * sizeof(DSpan), cudaMemcpyHostToDevice, p->stream));
+    CK(cudaStreamSynchronize(p->stream));
+    p->bound = true;
     return CUSAN_OK;
 }
 
 static int launch_all(cusan_plan* p) {
     // counters: race granules, runs, heap top (after the pre-assigned records), overflow flag
-    const unsigned long long init[N_COUNTERS] = {0, 0, p->hp.rec_units, 0};
-    CK(cudaMemcpyAsync(p->d_counters, init, sizeof(init), cudaMemcpyHostToDevice, p->stream));
+    // + one dynamic-scheduler counter per window
+    p->counter_init.assign(N_COUNTERS + p->wins.size(), 0ull);
+    p->counter_init[C_HEAP] = p->hp.rec_units;
+    CK(cudaMemcpyAsync(p->d_counters, p->counter_init.data(), p->counter_init.size() * sizeof(unsigned long long),
+                       cudaMemcpyHostToDevice, p->stream));
     CK(cudaEventRecord(p->ev0, p->stream));
     Ctx k;
     k.inc = p->d_inc;
@@ -606,9 +672,12 @@ static int launch_all(cusan_plan* p) {
     k.counters = p->d_counters;
     k.run_cap = p->run_cap;
     const int force_lanes = (p->hp.opts.flags & CUSAN_CHECK_FORCE_LANES) ? 1 : 0;
-    for (const Window& w : p->wins)
+    for (size_t i = 0; i < p->wins.size(); i++) {
+        const Window& w = p->wins[i];
+        unsigned long long* sched = CUSAN_DYNAMIC ? p->d_counters + N_COUNTERS + i : nullptr;
         shadow_check_window<<<w.grid, THREADS, 0, p->stream>>>(p->d_spans + w.span_off, w.nspans, w.tiles,
-                                                               w.weight, k, force_lanes);
+                                                               w.weight, k, force_lanes, sched);
+    }
     CK(cudaGetLastError());
     CK(cudaEventRecord(p->ev1, p->stream));
     return CUSAN_OK;
@@ -656,9 +725,16 @@ int cusan_plan_workspace_bytes(const cusan_plan* p, uint64_t* bytes) {
     return CUSAN_OK;
 }
 
+int cusan_plan_bind_workspace(cusan_plan* p, void* workspace, uint64_t bytes) {
+    if (!p || !workspace) return fail(CUSAN_EINVAL, "null argument");
+    if (p->own) return fail(CUSAN_ESTATE, "plan already owns a workspace");
+    return plan_bind(p, (char*)workspace, bytes);
+}
+
 int cusan_plan_run(cusan_plan* p, cusan_report** out) {
     if (!p || !out) return fail(CUSAN_EINVAL, "null argument");
     *out = nullptr;
+    if (!p->bound) return fail(CUSAN_ESTATE, "plan has no workspace: call cusan_plan_bind_workspace");
     const auto t_start = std::chrono::steady_clock::now();
     CK(cudaSetDevice(p->device));
     unsigned long long cnt[N_COUNTERS];

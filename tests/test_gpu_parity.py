@@ -183,3 +183,21 @@ def test_full_size_configs_sampled(c):
     got = {t for t in brute.runs_to_triples_in(rep.runs, sset)}
     want = brute.runs_to_triples(ref["runs"])
     assert got == want
+
+
+def test_torch_workspace_and_stream():
+    """Device memory from PyTorch's caching allocator, work on torch's current stream."""
+    import torch
+    w = configs.make(5, "small")
+    ops, args = w.arrays(True)
+    tr, _ = lower_product(ops, args)
+    ref = oracle.check_events(tr.cusan_trace_read(), 255)
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        for window in (0, 50):
+            rep = cs.check(tr, workspace="torch", window_events=window, stream=s.cuda_stream)
+            assert_equal(rep, ref)
+    plan = cs.Plan(tr, workspace="torch", window_events=50)
+    assert plan.workspace is not None and plan.workspace.numel() >= plan.workspace_bytes()
+    assert_equal(plan.run(), ref)
+    plan.close()
