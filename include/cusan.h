@@ -143,6 +143,22 @@ int cusan_plan_destroy(cusan_plan* p);
  * plan_create would compute (shard clip, intervals, segments, windows, spill records). */
 int cusan_plan_describe(const cusan_trace* t, const cusan_check_opts* o, cusan_counters* out);
 
+/* ---- incremental (online) checking: SURVEY.md §8(f) f1 ------------------------------------------
+ * CuSan checks while the program runs.  A session keeps the shadow on the device
+ * between calls; each cusan_session_check() checks the accesses appended to the trace since the
+ * previous call (in windows of opts.window_events, 0 = one window) against it and reports the races
+ * whose later access is among them.  The union of all calls' reports equals one cusan_check of the
+ * final trace; n_race_granules of the calls add up to its count.  The trace may only grow.
+ * Each call re-plans the interval layout of the whole trace (host) and moves the shadow to it
+ * (device copy of untouched intervals), so the device holds two shadows; a call can be re-run
+ * internally after a buffer overflow because it never modifies the previous shadow.
+ * Restrictions: nshards = 1, no caller workspace.  Report counter tracked_bytes_shard = bytes
+ * checked by this call. */
+typedef struct cusan_session cusan_session;
+int cusan_session_create(const cusan_trace* t, const cusan_check_opts* o, cusan_session** out);
+int cusan_session_check(cusan_session* s, cusan_report** out);
+int cusan_session_destroy(cusan_session* s);
+
 /* ---- report (a5) ------------------------------------------------------------------------------ */
 typedef struct cusan_counters {
     /* trace counters, cf. CuSan's Table I */

@@ -215,6 +215,31 @@ class Plan:
     __del__ = close
 
 
+class Session:
+    """cusan_session: incremental (online) checking with the shadow kept on the device between
+    calls; check() checks the accesses appended to the trace since the previous call."""
+
+    def __init__(self, trace: Trace, **kw):
+        self.trace = trace            # must outlive the session; may only grow
+        self.max_runs = kw.get("max_runs", 0)
+        o = _opts(**kw)
+        h = C.c_void_p()
+        _ck(lib.cusan_session_create(trace.h, C.byref(o), C.byref(h)))
+        self.h = h
+
+    def check(self) -> Report:
+        h = C.c_void_p()
+        _ck(lib.cusan_session_check(self.h, C.byref(h)))
+        return _report(h, self.max_runs)
+
+    def close(self):
+        if getattr(self, "h", None):
+            lib.cusan_session_destroy(self.h)
+            self.h = None
+
+    __del__ = close
+
+
 def describe(trace: Trace, **kw) -> dict:
     """cusan_plan_describe: the host steps a1/a2 only (no GPU) — plan counters of a shard."""
     o = _opts(**kw)

@@ -83,6 +83,9 @@ PROTOS = {
     "cusan_plan_run": [P, PP],
     "cusan_plan_destroy": [P],
     "cusan_plan_describe": [P, C.POINTER(cusan_check_opts), C.POINTER(cusan_counters)],
+    "cusan_session_create": [P, C.POINTER(cusan_check_opts), PP],
+    "cusan_session_check": [P, PP],
+    "cusan_session_destroy": [P],
     "cusan_report_get": [P, pu64, pu64, C.POINTER(C.POINTER(cusan_race_run)), pi32],
     "cusan_report_counters": [P, C.POINTER(cusan_counters)],
     "cusan_report_merge": [P, u64, u64, u64, PP],

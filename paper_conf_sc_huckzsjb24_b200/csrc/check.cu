@@ -77,19 +77,23 @@ struct DSpan {
     uint64_t tile0, weight0;     // prefix of ranges / of range weights over the window's spans
     uint32_t rsize, rweight;     // granules per range (multiple of CHUNK), weight of one range
     uint32_t list_off, list_cnt, flags, rec, rec_units, pad;
+    uint64_t src_begin;          // where LOAD reads the cells: `shadow` (or `shadow_old` with SPAN_SRC_OLD)
 };
-static_assert(sizeof(DSpan) == 72, "DSpan layout");
+static_assert(sizeof(DSpan) == 80, "DSpan layout");
 
 struct Ctx {                     // kernel-wide pointers
     const AccRec* __restrict__ inc;
     const uint32_t* __restrict__ segvc;
     uint32_t F;
     uint2* __restrict__ shadow;
+    const uint2* __restrict__ shadow_old;   // previous layout (incremental sessions), else null
     uint32_t* __restrict__ heap;
     unsigned long long heap_cap;  // record units
     cusan_race_run* __restrict__ runs;
     unsigned long long* __restrict__ counters;
     unsigned long long run_cap;
+    int cow_all;                  // sessions: never modify a record in place (the previous check's
+                                  // shadow must stay a consistent snapshot so a check can re-run)
 };
 
 struct RunCache {
@@ -217,7 +221,7 @@ __device__ void lane_read_update(uint2& c, uint32_t ep, uint32_t f, const Ctx& k
     for (uint32_t j = 0; j < n; j++)
         if ((src[1 + j] >> 24) == f) { pos = (int)j; break; }
     if (pos >= 0 && src[1 + pos] == ep) return;
-    if (hdr & REC_PRIVATE) {                   // this granule's own record: update in place
+    if ((hdr & REC_PRIVATE) && !k.cow_all) {   // this granule's own record: update in place
         const uint32_t cap = ((hdr >> 16) & 0xffu) * REC_WORDS - 1;
         if (pos >= 0) { src[1 + pos] = ep; return; }
         if (n < cap) { src[1 + n] = ep; src[0] = hdr + 1; return; }
@@ -230,6 +234,11 @@ __device__ void lane_read_update(uint2& c, uint32_t ep, uint32_t f, const Ctx& k
     c.y = v;
 }
 
+// Where a span's LOAD reads its cells (SPAN_SRC_OLD: the previous check's shadow of a session).
+__device__ __forceinline__ const uint2* src_cells(const DSpan& sp, const Ctx& k) {
+    return ((sp.flags & SPAN_SRC_OLD) ? k.shadow_old : k.shadow) + sp.src_begin;
+}
+
 // Lane-parallel exact path for granules [x0, x0 + n) of span sp (each lane its own cells).
 __device__ void check_lanes(const DSpan& sp, uint64_t x0, uint64_t n, int lane, RunCache& rc, const Ctx& k) {
     for (uint64_t xc = x0; xc < x0 + n; xc += CHUNK) {
@@ -240,7 +249,7 @@ __device__ void check_lanes(const DSpan& sp, uint64_t x0, uint64_t n, int lane, 
             const uint64_t x = xc + c * 32 + lane;
             valid[c] = x < x0 + n;
             cell[c] = make_uint2(0, 0);
-            if (valid[c] && (sp.flags & SPAN_LOAD)) cell[c] = __ldcs(k.shadow + sp.dense_begin + x);
+            if (valid[c] && (sp.flags & SPAN_LOAD)) cell[c] = __ldcs(src_cells(sp, k) + x);
         }
         const uint32_t qe = sp.list_off + sp.list_cnt;
         for (uint32_t q = sp.list_off; q < qe; q++) {
@@ -266,7 +275,7 @@ __device__ void check_lanes(const DSpan& sp, uint64_t x0, uint64_t n, int lane, 
                     // R := ∅.  A private record stays attached, emptied, for this granule's next
                     // readers (a record with n = 0 is the empty read set); shared ones detach.
                     uint32_t keep = 0;
-                    if (sp_r && (rp[0] & REC_PRIVATE)) {
+                    if (sp_r && (rp[0] & REC_PRIVATE) && !k.cow_all) {
                         rp[0] &= ~0xffffu;
                         keep = cell[c].y;
                     }
@@ -354,26 +363,34 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
             const uint64_t x0 = (t - sp.tile0) * sp.rsize;
             const uint64_t n = min((uint64_t)sp.rsize, sp.len - x0);
             uint2* cells = k.shadow + sp.dense_begin + x0;      // 256-B aligned (CELL_ALIGN)
-            const uint4* cells2 = reinterpret_cast<const uint4*>(cells);
+            const uint2* src = src_cells(sp, k) + x0;
+            const uint4* cells2 = reinterpret_cast<const uint4*>(src);
             const uint64_t n2 = n >> 1;                         // cell pairs
             // ---- pass 1: stream the range's cells in and vote that they are all equal ----------
             uint2 c = make_uint2(0, 0);            // first window of the interval: known empty
             bool uniform = !force_lanes;
             if (uniform && (sp.flags & SPAN_LOAD)) {
-                c = cells[0];
+                c = src[0];
                 bool ok = true;
-                for (uint64_t i = lane; i < n2; i += 32 * UL) {
-                    uint4 v[UL];
+                if ((reinterpret_cast<uintptr_t>(src) & 15u) == 0) {
+                    for (uint64_t i = lane; i < n2; i += 32 * UL) {
+                        uint4 v[UL];
 #pragma unroll
-                    for (int u = 0; u < UL; u++)
-                        v[u] = (i + u * 32 < n2) ? __ldcs(cells2 + i + u * 32) : make_uint4(c.x, c.y, c.x, c.y);
+                        for (int u = 0; u < UL; u++)
+                            v[u] = (i + u * 32 < n2) ? __ldcs(cells2 + i + u * 32) : make_uint4(c.x, c.y, c.x, c.y);
 #pragma unroll
-                    for (int u = 0; u < UL; u++)
-                        ok &= ((v[u].x ^ c.x) | (v[u].y ^ c.y) | (v[u].z ^ c.x) | (v[u].w ^ c.y)) == 0u;
-                }
-                if ((n & 1) && lane == 0) {
-                    const uint2 tl = __ldcs(cells + n - 1);
-                    ok &= tl.x == c.x && tl.y == c.y;
+                        for (int u = 0; u < UL; u++)
+                            ok &= ((v[u].x ^ c.x) | (v[u].y ^ c.y) | (v[u].z ^ c.x) | (v[u].w ^ c.y)) == 0u;
+                    }
+                    if ((n & 1) && lane == 0) {
+                        const uint2 tl = __ldcs(src + n - 1);
+                        ok &= tl.x == c.x && tl.y == c.y;
+                    }
+                } else {                           // a session's old-layout source off a 16-B boundary
+                    for (uint64_t i = lane; i < n; i += 32) {
+                        const uint2 v = __ldcs(src + i);
+                        ok &= v.x == c.x && v.y == c.y;
+                    }
                 }
                 uniform = __all_sync(FULL, ok);
             }
@@ -526,27 +543,21 @@ struct cusan_plan {
 
 static int plan_bind(cusan_plan* p, char* ws, uint64_t bytes);
 
-static int plan_device_setup(cusan_plan* p) {
-    HostPlan& hp = p->hp;
-    const cusan_check_opts& o = hp.opts;
-    int ndev = 0;
-    cudaError_t e = cudaGetDeviceCount(&ndev);
-    if (e != cudaSuccess || ndev == 0)
-        return fail(CUSAN_ECUDA, std::string("no CUDA device available: ") + cudaGetErrorString(e));
-    if (o.device < 0 || o.device >= ndev) return fail(CUSAN_EINVAL, "bad device ordinal");
-    p->device = o.device;
-    CK(cudaSetDevice(p->device));
-    p->stream = (cudaStream_t)o.stream;
-    int sms = 0, per_sm = 0;
-    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, p->device));
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, shadow_check_window, THREADS, 0));
-    p->max_blocks = sms * std::max(per_sm, 1);
-
-    // device-side span tables: per window its spans plus a sentinel, with range / weight prefixes
+// Device-side span tables: per window its spans plus a sentinel, with range / weight prefixes.
+struct SpanTables {
     std::vector<DSpan> ds;
+    std::vector<Window> wins;
+    bool need_shadow = false;
+    uint64_t cell_bytes = 0;      // algorithmic shadow bytes (8 B per LOAD + 8 B per STORE cell)
+};
+
+static void build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& out) {
+    std::vector<DSpan>& ds = out.ds;
+    ds.clear();
     ds.reserve(hp.spans.size() + hp.win_span_off.size());
-    p->need_shadow = false;
-    p->shadow_cell_bytes = 0;
+    out.wins.clear();
+    out.need_shadow = false;
+    out.cell_bytes = 0;
     for (size_t w = 0; w + 1 < hp.win_span_off.size(); w++) {
         Window win{};
         win.span_off = ds.size();
@@ -562,11 +573,13 @@ static int plan_device_setup(cusan_plan* p) {
             d.flags = s.flags;
             d.rec = s.rec;
             d.rec_units = s.rec_units;
+            d.src_begin = s.src_begin;
             // warp range: long enough that replaying the window's accesses once per range stays
-            // cheap next to streaming its cells (≈ 64 granules per access), capped for balance;
-            // spans that move no cells are one range each
+            // small next to streaming its cells, capped for balance; spans that move no cells
+            // are one range each
+            const bool moves = s.flags & (SPAN_LOAD | SPAN_STORE);
             uint64_t rs;
-            if (s.flags & (SPAN_LOAD | SPAN_STORE))
+            if (moves)
                 rs = std::min<uint64_t>(std::max<uint64_t>((uint64_t)CUSAN_RANGE_PER_ACCESS * s.list_cnt,
                                                            (uint64_t)CUSAN_RANGE_MIN),
                                         (uint64_t)CUSAN_RANGE_MAX);
@@ -575,14 +588,14 @@ static int plan_device_setup(cusan_plan* p) {
             rs = std::min<uint64_t>((rs + CHUNK - 1) / CHUNK * CHUNK, 1ull << 31);
             d.rsize = (uint32_t)rs;
             const uint64_t nt = (s.len + rs - 1) / rs;
-            const uint64_t mem = (s.flags & (SPAN_LOAD | SPAN_STORE)) ? rs / 32 : 0;
+            const uint64_t mem = moves ? rs / 32 : 0;
             d.rweight = (uint32_t)std::min<uint64_t>(mem + 4ull * s.list_cnt + 8, 0xffffffffull);
             d.tile0 = tiles;
             d.weight0 = weight;
             tiles += nt;
             weight += nt * d.rweight;
-            if (s.flags) p->need_shadow = true;
-            p->shadow_cell_bytes += s.len * (((s.flags & SPAN_LOAD) ? 8 : 0) + ((s.flags & SPAN_STORE) ? 8 : 0));
+            if (moves) out.need_shadow = true;
+            out.cell_bytes += s.len * (((s.flags & SPAN_LOAD) ? 8 : 0) + ((s.flags & SPAN_STORE) ? 8 : 0));
             ds.push_back(d);
         }
         win.nspans = (uint32_t)(ds.size() - win.span_off);
@@ -592,10 +605,40 @@ static int plan_device_setup(cusan_plan* p) {
         ds.push_back(sent);
         win.tiles = tiles;
         win.weight = weight;
-        win.grid = (uint32_t)std::min<uint64_t>((uint64_t)p->max_blocks, (tiles + WARPS - 1) / WARPS);
+        win.grid = (uint32_t)std::min<uint64_t>((uint64_t)max_blocks, (tiles + WARPS - 1) / WARPS);
         if (win.grid == 0) win.grid = 1;
-        p->wins.push_back(win);
+        out.wins.push_back(win);
     }
+}
+
+static int device_info(int device, int* max_blocks) {
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess || ndev == 0)
+        return fail(CUSAN_ECUDA, std::string("no CUDA device available: ") + cudaGetErrorString(e));
+    if (device < 0 || device >= ndev) return fail(CUSAN_EINVAL, "bad device ordinal");
+    CK(cudaSetDevice(device));
+    int sms = 0, per_sm = 0;
+    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, shadow_check_window, THREADS, 0));
+    *max_blocks = sms * std::max(per_sm, 1);
+    return CUSAN_OK;
+}
+
+static int plan_device_setup(cusan_plan* p) {
+    HostPlan& hp = p->hp;
+    const cusan_check_opts& o = hp.opts;
+    int st0 = device_info(o.device, &p->max_blocks);
+    if (st0) return st0;
+    p->device = o.device;
+    p->stream = (cudaStream_t)o.stream;
+
+    SpanTables st;
+    build_span_tables(hp, p->max_blocks, st);
+    std::vector<DSpan>& ds = st.ds;
+    p->wins = st.wins;
+    p->need_shadow = st.need_shadow;
+    p->shadow_cell_bytes = st.cell_bytes;
 
     // workspace layout
     p->heap_cap = hp.rec_units + (1ull << 16);             // pre-assigned records + lane-path room
@@ -666,6 +709,8 @@ static int launch_all(cusan_plan* p) {
     k.segvc = p->d_segvc;
     k.F = p->hp.F;
     k.shadow = p->d_shadow;
+    k.shadow_old = nullptr;
+    k.cow_all = 0;
     k.heap = p->d_heap;
     k.heap_cap = p->heap_cap;
     k.runs = p->d_runs;
@@ -820,6 +865,318 @@ int cusan_check(const cusan_trace* t, const cusan_check_opts* o, cusan_report** 
     st = cusan_plan_run(p, out);
     cusan_plan_destroy(p);
     return st;
+}
+
+}  // extern "C"
+
+// ================================================================================================
+// Incremental sessions: CuSan checks while the program runs
+// (PAPER.md:606-612); a session keeps the shadow on the device between calls and each call checks
+// only the accesses appended since the previous one.
+//
+// New accesses can split elementary intervals or add new ones, so every call re-plans the layout
+// (a1, a2 over the whole trace; host cost only).  The previous call's shadow stays untouched as
+// the source: intervals the call does not touch are copied to the new layout (copy_cells), the
+// first span of a touched interval loads its cells from the old layout (SPAN_SRC_OLD), and read-set
+// records are never modified in place (cow_all).  A call therefore only writes the new buffer and
+// can be re-run as a whole after a run-buffer or heap overflow.  The buffers then swap.
+// ================================================================================================
+namespace {
+
+struct CopySeg {
+    uint64_t prefix, src, dst, len;       // cells [prefix, prefix + len) of the copy space
+};
+
+constexpr uint64_t COPY_CHUNK = 8192;     // cells per warp work item
+
+__global__ void __launch_bounds__(THREADS)
+copy_cells(const uint2* __restrict__ src, uint2* __restrict__ dst, const CopySeg* __restrict__ segs,
+           uint32_t nseg, uint64_t total) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t nwarps = (uint64_t)gridDim.x * WARPS;
+    const uint64_t nchunks = (total + COPY_CHUNK - 1) / COPY_CHUNK;
+    for (uint64_t ch = (uint64_t)blockIdx.x * WARPS + (threadIdx.x >> 5); ch < nchunks; ch += nwarps) {
+        const uint64_t c0 = ch * COPY_CHUNK, c1 = min(c0 + COPY_CHUNK, total);
+        uint32_t lo = 0, hi = nseg;                       // last segment with prefix <= c0
+        while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (segs[mid].prefix <= c0) lo = mid; else hi = mid;
+        }
+        for (uint64_t c = c0; c < c1; lo++) {
+            const CopySeg sg = segs[lo];
+            const uint64_t end = min(c1, sg.prefix + sg.len);
+            for (uint64_t i = c + lane; i < end; i += 32)
+                __stcs(dst + sg.dst + (i - sg.prefix), __ldcs(src + sg.src + (i - sg.prefix)));
+            c = end;
+        }
+    }
+}
+
+}  // namespace
+
+struct cusan_session {
+    const cusan_trace* trace = nullptr;
+    cusan_check_opts opts{};
+    int device = 0, max_blocks = 0;
+    cudaStream_t stream = nullptr;
+    std::vector<Interval> layout;                   // layout of `shadow`
+    uint2* shadow = nullptr;
+    uint64_t shadow_cap = 0;                        // cells
+    uint2* spare = nullptr;
+    uint64_t spare_cap = 0;
+    uint32_t* heap = nullptr;
+    uint64_t heap_cap = 0, heap_top = 0;            // record units
+    char* scratch = nullptr;
+    uint64_t scratch_cap = 0;
+    cusan_race_run* runs = nullptr;
+    uint64_t run_cap = 0;
+    uint64_t checked_access = 0, checked_events = 0, n_calls = 0;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+
+    ~cusan_session() {
+        if (ev0) cudaEventDestroy(ev0);
+        if (ev1) cudaEventDestroy(ev1);
+        cudaFree(shadow);
+        cudaFree(spare);
+        cudaFree(heap);
+        cudaFree(scratch);
+        cudaFree(runs);
+    }
+};
+
+template <class T>
+static int ensure(T** p, uint64_t* cap, uint64_t need, const char* what) {
+    if (*cap >= need && *p) return CUSAN_OK;
+    cudaFree(*p);
+    *p = nullptr;
+    *cap = 0;
+    const uint64_t n = std::max<uint64_t>(need, 1);
+    if (cudaMalloc((void**)p, n * sizeof(T)) != cudaSuccess)
+        return fail(CUSAN_ENOMEM, std::string("cannot allocate ") + what);
+    *cap = n;
+    return CUSAN_OK;
+}
+
+// grow the heap keeping records [0, heap_top)
+static int grow_heap(cusan_session* s, uint64_t need) {
+    if (s->heap_cap >= need && s->heap) return CUSAN_OK;
+    if (need >= (1ull << 24)) return fail(CUSAN_ENOMEM, "read-set heap exceeds the 24-bit record index");
+    const uint64_t cap = std::min<uint64_t>(std::max<uint64_t>(need, 2 * s->heap_cap), (1ull << 24) - 1);
+    uint32_t* nh = nullptr;
+    if (cudaMalloc((void**)&nh, cap * REC_WORDS * sizeof(uint32_t)) != cudaSuccess)
+        return fail(CUSAN_ENOMEM, "cannot grow the read-set heap");
+    if (s->heap && s->heap_top)
+        CK(cudaMemcpyAsync(nh, s->heap, s->heap_top * REC_WORDS * sizeof(uint32_t), cudaMemcpyDeviceToDevice,
+                           s->stream));
+    CK(cudaStreamSynchronize(s->stream));
+    cudaFree(s->heap);
+    s->heap = nh;
+    s->heap_cap = cap;
+    return CUSAN_OK;
+}
+
+extern "C" {
+
+int cusan_session_create(const cusan_trace* t, const cusan_check_opts* o, cusan_session** out) {
+    if (!t || !o || !out) return fail(CUSAN_EINVAL, "null argument");
+    *out = nullptr;
+    if (o->nshards != 1 || o->shard != 0)
+        return fail(CUSAN_EINVAL, "sessions check the whole granule space (nshards = 1)");
+    if (o->workspace) return fail(CUSAN_EINVAL, "sessions manage their own device memory");
+    cusan_session* s = new (std::nothrow) cusan_session;
+    if (!s) return fail(CUSAN_ENOMEM, "cannot allocate session");
+    s->trace = t;
+    s->opts = *o;
+    s->opts.persist_shadow = 1;
+    int st = device_info(o->device, &s->max_blocks);
+    if (!st) {
+        s->device = o->device;
+        s->stream = (cudaStream_t)o->stream;
+        if (cudaEventCreate(&s->ev0) != cudaSuccess || cudaEventCreate(&s->ev1) != cudaSuccess)
+            st = fail(CUSAN_ECUDA, "cannot create events");
+    }
+    if (st) {
+        delete s;
+        return st;
+    }
+    *out = s;
+    return CUSAN_OK;
+}
+
+int cusan_session_check(cusan_session* s, cusan_report** out) {
+    if (!s || !out) return fail(CUSAN_EINVAL, "null argument");
+    *out = nullptr;
+    const auto t_start = std::chrono::steady_clock::now();
+    CK(cudaSetDevice(s->device));
+    const Trace& tr = s->trace->t;
+    if (tr.ev.size() < s->checked_events) return fail(CUSAN_ESTATE, "the trace shrank");
+
+    // ---- a1 + a2 over the whole trace; spans only for the new accesses ------------------------
+    HostPlan hp;
+    int st;
+    try {
+        st = build_host_plan(tr, s->opts, hp, s->checked_access, s->heap_top);
+    } catch (const std::bad_alloc&) {
+        st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
+    }
+    if (st) return st;
+    const uint64_t first = s->checked_access, n_acc = hp.acc_g0.size();
+    uint64_t new_tracked = 0;
+    for (uint64_t k = first; k < n_acc; k++) new_tracked += 8 * (hp.acc_g1[k] - hp.acc_g0[k]);
+
+    // ---- old layout -> new layout ----------------------------------------------------------------
+    // intervals are elementary for all accesses so far, so each new interval lies inside one old
+    // interval or outside the old coverage
+    std::vector<uint64_t> old_src(hp.iv.size(), UINT64_MAX);
+    std::vector<CopySeg> segs;
+    uint64_t copy_cells_n = 0;
+    {
+        size_t j = 0;
+        for (size_t i = 0; i < hp.iv.size(); i++) {
+            const Interval& v = hp.iv[i];
+            while (j < s->layout.size() && s->layout[j].abs_begin + s->layout[j].len <= v.abs_begin) j++;
+            if (j < s->layout.size() && s->layout[j].abs_begin <= v.abs_begin) {
+                const Interval& u = s->layout[j];
+                old_src[i] = u.dense_begin + (v.abs_begin - u.abs_begin);
+                const bool touched = v.list_cnt && hp.inc_acc[v.list_off + v.list_cnt - 1] >= first;
+                if (!touched) {
+                    segs.push_back({copy_cells_n, old_src[i], v.dense_begin, v.len});
+                    copy_cells_n += v.len;
+                }
+            }
+        }
+    }
+    for (Span& sp : hp.spans) {
+        if (!(sp.flags & SPAN_FIRST_IN_CALL) || !(sp.flags & SPAN_LOAD)) continue;
+        auto it = std::lower_bound(hp.iv.begin(), hp.iv.end(), sp.dense_begin,
+                                   [](const Interval& a, uint64_t d) { return a.dense_begin < d; });
+        const size_t i = it - hp.iv.begin();
+        if (i >= hp.iv.size() || old_src[i] == UINT64_MAX)
+            return fail(CUSAN_ESTATE, "internal: a loaded interval has no previous state");
+        sp.flags |= SPAN_SRC_OLD;
+        sp.src_begin = old_src[i];
+    }
+    SpanTables tabs;
+    build_span_tables(hp, s->max_blocks, tabs);
+
+    // ---- device memory ---------------------------------------------------------------------------
+    if ((st = ensure(&s->spare, &s->spare_cap, hp.shadow_cells, "shadow"))) return st;
+    if ((st = grow_heap(s, s->heap_top + hp.rec_units + (1ull << 16)))) return st;
+    if ((st = ensure(&s->runs, &s->run_cap, std::max<uint64_t>(s->run_cap, 1ull << 16), "run buffer"))) return st;
+    const uint64_t nwin = tabs.wins.size();
+    uint64_t off = 0;
+    const uint64_t o_inc = off;   off = align_up(off + hp.inc.size() * sizeof(AccRec));
+    const uint64_t o_seg = off;   off = align_up(off + hp.segvc.size() * sizeof(uint32_t));
+    const uint64_t o_spans = off; off = align_up(off + tabs.ds.size() * sizeof(DSpan));
+    const uint64_t o_copy = off;  off = align_up(off + segs.size() * sizeof(CopySeg));
+    const uint64_t o_cnt = off;   off = align_up(off + (N_COUNTERS + nwin) * sizeof(unsigned long long));
+    if ((st = ensure(&s->scratch, &s->scratch_cap, off, "plan tables"))) return st;
+    AccRec* d_inc = (AccRec*)(s->scratch + o_inc);
+    uint32_t* d_seg = (uint32_t*)(s->scratch + o_seg);
+    DSpan* d_spans = (DSpan*)(s->scratch + o_spans);
+    CopySeg* d_copy = (CopySeg*)(s->scratch + o_copy);
+    unsigned long long* d_cnt = (unsigned long long*)(s->scratch + o_cnt);
+    CK(cudaMemcpyAsync(d_inc, hp.inc.data(), hp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, s->stream));
+    CK(cudaMemcpyAsync(d_seg, hp.segvc.data(), hp.segvc.size() * sizeof(uint32_t), cudaMemcpyHostToDevice, s->stream));
+    CK(cudaMemcpyAsync(d_spans, tabs.ds.data(), tabs.ds.size() * sizeof(DSpan), cudaMemcpyHostToDevice, s->stream));
+    CK(cudaMemcpyAsync(d_copy, segs.data(), segs.size() * sizeof(CopySeg), cudaMemcpyHostToDevice, s->stream));
+
+    // ---- a3 / a4 (re-runnable: only `spare` and fresh heap units are written) ----------------------
+    std::vector<unsigned long long> init(N_COUNTERS + nwin, 0ull), cnt(N_COUNTERS, 0ull);
+    float kms = 0.f;
+    for (int attempt = 0;; attempt++) {
+        init[C_HEAP] = s->heap_top + hp.rec_units;
+        CK(cudaMemcpyAsync(d_cnt, init.data(), init.size() * sizeof(unsigned long long), cudaMemcpyHostToDevice,
+                           s->stream));
+        CK(cudaEventRecord(s->ev0, s->stream));
+        if (copy_cells_n)
+            copy_cells<<<s->max_blocks, THREADS, 0, s->stream>>>(s->shadow, s->spare, d_copy, (uint32_t)segs.size(),
+                                                                  copy_cells_n);
+        Ctx k;
+        k.inc = d_inc;
+        k.segvc = d_seg;
+        k.F = hp.F;
+        k.shadow = s->spare;
+        k.shadow_old = s->shadow;
+        k.heap = s->heap;
+        k.heap_cap = s->heap_cap;
+        k.runs = s->runs;
+        k.counters = d_cnt;
+        k.run_cap = s->run_cap;
+        k.cow_all = 1;
+        const int force_lanes = (s->opts.flags & CUSAN_CHECK_FORCE_LANES) ? 1 : 0;
+        for (size_t i = 0; i < nwin; i++) {
+            const Window& w = tabs.wins[i];
+            unsigned long long* sched = CUSAN_DYNAMIC ? d_cnt + N_COUNTERS + i : nullptr;
+            shadow_check_window<<<w.grid, THREADS, 0, s->stream>>>(d_spans + w.span_off, w.nspans, w.tiles, w.weight,
+                                                                   k, force_lanes, sched);
+        }
+        CK(cudaGetLastError());
+        CK(cudaEventRecord(s->ev1, s->stream));
+        CK(cudaMemcpyAsync(cnt.data(), d_cnt, N_COUNTERS * sizeof(unsigned long long), cudaMemcpyDeviceToHost,
+                           s->stream));
+        CK(cudaStreamSynchronize(s->stream));
+        const bool runs_ovf = cnt[C_RUNS] > s->run_cap, heap_ovf = cnt[C_HEAP_OVF] != 0;
+        if (!runs_ovf && !heap_ovf) break;
+        if (attempt >= 8) return fail(CUSAN_ENOMEM, "run buffer / read-set heap keeps overflowing");
+        if (runs_ovf && (st = ensure(&s->runs, &s->run_cap, cnt[C_RUNS] + cnt[C_RUNS] / 8 + 1024, "run buffer")))
+            return st;
+        if (heap_ovf && (st = grow_heap(s, 2 * s->heap_cap))) return st;
+    }
+    CK(cudaEventElapsedTime(&kms, s->ev0, s->ev1));
+
+    // ---- commit: the new buffer becomes the shadow ------------------------------------------------
+    std::swap(s->shadow, s->spare);
+    std::swap(s->shadow_cap, s->spare_cap);
+    s->layout = hp.iv;
+    s->heap_top = cnt[C_HEAP];
+    s->checked_access = n_acc;
+    s->checked_events = tr.ev.size();
+    s->n_calls++;
+
+    cusan_report* r = new (std::nothrow) cusan_report;
+    if (!r) return fail(CUSAN_ENOMEM, "cannot allocate report");
+    try {
+        r->runs.resize(cnt[C_RUNS]);
+    } catch (...) {
+        delete r;
+        return fail(CUSAN_ENOMEM, "cannot allocate report runs");
+    }
+    if (cnt[C_RUNS]) {
+        cudaError_t ce = cudaMemcpy(r->runs.data(), s->runs, cnt[C_RUNS] * sizeof(cusan_race_run),
+                                    cudaMemcpyDeviceToHost);
+        if (ce != cudaSuccess) {
+            delete r;
+            return cuda_fail(ce, "run download");
+        }
+    }
+    canonicalize_runs(r->runs);
+    r->n_runs = r->runs.size();
+    r->n_race_granules = cnt[C_RACE];
+    if (s->opts.max_runs && r->runs.size() > s->opts.max_runs) {
+        r->runs.resize(s->opts.max_runs);
+        r->truncated = 1;
+    }
+    r->ctr = hp.ctr;
+    r->ctr.tracked_bytes_shard = new_tracked;       // checked by this call
+    r->ctr.raw_runs = cnt[C_RUNS];
+    r->ctr.kernel_ms = kms;
+    r->ctr.kernel_launches = nwin + (copy_cells_n ? 1 : 0);
+    r->ctr.shadow_cell_bytes = tabs.cell_bytes + 16 * copy_cells_n;
+    r->ctr.shadow_bytes = hp.shadow_cells * sizeof(uint2);
+    r->ctr.h2d_bytes = hp.inc.size() * sizeof(AccRec) + hp.segvc.size() * sizeof(uint32_t) +
+                       tabs.ds.size() * sizeof(DSpan) + segs.size() * sizeof(CopySeg);
+    r->ctr.d2h_bytes = N_COUNTERS * sizeof(unsigned long long) + cnt[C_RUNS] * sizeof(cusan_race_run);
+    r->ctr.run_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count();
+    *out = r;
+    return CUSAN_OK;
+}
+
+int cusan_session_destroy(cusan_session* s) {
+    if (!s) return fail(CUSAN_EINVAL, "session is null");
+    if (s->stream) cudaStreamSynchronize(s->stream);
+    delete s;
+    return CUSAN_OK;
 }
 
 }  // extern "C"

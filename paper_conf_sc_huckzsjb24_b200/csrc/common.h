@@ -52,10 +52,14 @@ struct Span {
     uint32_t list_off;    // into the AccRec table
     uint32_t list_cnt;
     uint32_t flags;       // SPAN_LOAD: cells hold state from an earlier window; SPAN_STORE: write back
-    uint32_t rec;         // pre-assigned spill record (REC_WORDS-word units) for the final state
-    uint32_t rec_units;   // its size; 0 = the final state needs no record (≤ 3 readers)
+    uint32_t rec;         // pre-assigned read-set record (REC_WORDS-word units) for the final state
+    uint32_t rec_units;   // its size; 0 = the final state needs no record (≤ 1 reader)
+    uint64_t src_begin;   // shadow index LOAD reads from (= dense_begin except in sessions)
 };
-enum : uint32_t { SPAN_LOAD = 1u, SPAN_STORE = 2u };
+// SPAN_LOAD: cells hold state from an earlier window; SPAN_STORE: a later window needs the result;
+// SPAN_FIRST_IN_CALL: the interval's first span of this check (incremental sessions);
+// SPAN_SRC_OLD: LOAD from the previous check's shadow at src_begin (sessions).
+enum : uint32_t { SPAN_LOAD = 1u, SPAN_STORE = 2u, SPAN_SRC_OLD = 4u, SPAN_FIRST_IN_CALL = 8u };
 
 struct HostPlan {
     // options
@@ -84,7 +88,10 @@ struct HostPlan {
     cusan_counters ctr{};
 };
 
-int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp);
+// a1 + a2.  Spans (windows) are planned for the accesses from `first_access` on (0 = all);
+// pre-assigned read-set records are numbered from `rec_base`.
+int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uint64_t first_access = 0,
+                    uint64_t rec_base = 0);
 
 // canonical merge of runs (sort by (later, earlier, g_begin), merge abutting) — a4 host part
 void canonicalize_runs(std::vector<cusan_race_run>& runs);

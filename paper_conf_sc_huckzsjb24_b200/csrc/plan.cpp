@@ -25,7 +25,8 @@
 
 namespace cusan {
 
-int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp) {
+int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uint64_t first_access,
+                    uint64_t rec_base) {
     if (o.nshards < 1 || o.shard < 0 || o.shard >= o.nshards)
         return fail(CUSAN_EINVAL, "need 0 <= shard < nshards");
     if (o.window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
@@ -223,19 +224,29 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp) {
     // interval's last write gets a pre-assigned read-set record: the cell keeps W inline and its R
     // slot points at the record holding the readers (the reader *set* depends only on the fibers
     // and modes covering the interval, never on happens-before, so its size is known here exactly).
-    const uint64_t W = o.window_events > 0 ? (uint64_t)o.window_events : std::max<uint64_t>(n_acc, 1);
+    // Incremental checks (f1) plan only the accesses from `first_access` on; earlier incidences
+    // still count for the LOAD flag and the reader sets, and records are numbered from `rec_base`.
+    const uint64_t first = std::min<uint64_t>(first_access, n_acc);
+    const uint64_t n_new = n_acc - first;
+    const uint64_t W = o.window_events > 0 ? (uint64_t)o.window_events : std::max<uint64_t>(n_new, 1);
     hp.window_accesses = W;
-    const uint64_t nwin = n_acc ? (n_acc + W - 1) / W : 0;
+    const uint64_t nwin = n_new ? (n_new + W - 1) / W : 0;
     std::vector<std::vector<Span>> per(nwin);
     hp.rec_units = 0;
     hp.spill_spans = 0;
     for (const Interval& v : hp.iv) {
         std::bitset<CUSAN_MAX_FIBERS + 1> readers;
         uint32_t q = v.list_off, qe = v.list_off + v.list_cnt;
+        for (; q < qe && hp.inc_acc[q] < first; q++) {
+            const AccRec& r = hp.inc[q];
+            if (r.segm >> 31) readers.reset();
+            else readers.set(r.epoch >> 24);
+        }
+        const uint32_t first_new = q;
         while (q < qe) {
-            uint64_t w = hp.inc_acc[q] / W;
+            uint64_t w = (hp.inc_acc[q] - first) / W;
             uint32_t q2 = q;
-            while (q2 < qe && hp.inc_acc[q2] / W == w) {
+            while (q2 < qe && (hp.inc_acc[q2] - first) / W == w) {
                 const AccRec& r = hp.inc[q2];
                 if (r.segm >> 31) readers.reset();
                 else readers.set(r.epoch >> 24);
@@ -247,10 +258,12 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp) {
             s.len = v.len;
             s.list_off = q;
             s.list_cnt = q2 - q;
-            s.flags = (q > v.list_off ? SPAN_LOAD : 0u) | ((q2 < qe || o.persist_shadow) ? SPAN_STORE : 0u);
+            s.src_begin = v.dense_begin;
+            s.flags = (q > v.list_off ? SPAN_LOAD : 0u) | ((q2 < qe || o.persist_shadow) ? SPAN_STORE : 0u) |
+                      (q == first_new ? SPAN_FIRST_IN_CALL : 0u);
             const uint64_t nr = readers.count();
             if ((s.flags & SPAN_STORE) && nr >= 2) {
-                s.rec = (uint32_t)hp.rec_units;
+                s.rec = (uint32_t)(rec_base + hp.rec_units);
                 s.rec_units = (uint32_t)((nr + 1 + REC_WORDS - 1) / REC_WORDS);
                 hp.rec_units += s.rec_units;
                 hp.spill_spans++;
@@ -259,8 +272,8 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp) {
             q = q2;
         }
     }
-    if (hp.rec_units >= (1u << 24) - 1)
-        return fail(CUSAN_ERANGE, "too many spill records for the 24-bit record index");
+    if (rec_base + hp.rec_units >= (1u << 24) - 1)
+        return fail(CUSAN_ERANGE, "too many read-set records for the 24-bit record index");
     c.spill_spans = hp.spill_spans;
     c.spill_heap_bytes = hp.rec_units * REC_WORDS * 4;
     hp.spans.clear();

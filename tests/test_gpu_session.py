@@ -1,0 +1,92 @@
+"""Incremental (online) checking: a session checks the accesses appended since its
+previous call against the shadow it keeps on the device.  Each call's report must equal the oracle's
+report of the final trace restricted to races whose later access belongs to that call."""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_sc_huckzsjb24_b200 as cs
+from tracegen import configs, fuzz
+from tracegen.program import EV_ACCESS
+
+pytestmark = pytest.mark.gpu
+
+
+def _by_later(runs, lo, hi):
+    m = (runs["later"] >= lo) & (runs["later"] < hi)
+    return runs[m]
+
+
+def _run_session(ev, nf, cuts, **kw):
+    """Append ev in pieces ending at `cuts`, check after each; compare with the oracle."""
+    ref = oracle.check_events(ev, nf, threads=2)
+    tr = cs.Trace(nf)
+    ses = cs.Session(tr, **kw)
+    start, total = 0, 0
+    for end in list(cuts) + [len(ev)]:
+        if end <= start:
+            continue
+        tr.cusan_trace_append_events(ev[start:end])
+        rep = ses.check()
+        want = _by_later(ref["runs"], start, end)
+        assert np.array_equal(rep.runs, want.astype(rep.runs.dtype)), (start, end)
+        assert rep.n_race_granules == int(np.sum(want["g_end"] - want["g_begin"]))
+        total += rep.n_race_granules
+        start = end
+    ses.close()
+    assert total == ref["n_race_granules"]
+    return ref
+
+
+@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_FORCE_LANES], ids=["ranges", "lanes"])
+@pytest.mark.parametrize("window", [0, 3])
+def test_session_fuzz(window, flags):
+    rng = np.random.default_rng(600 + window)
+    for _ in range(25):
+        nf = int(rng.integers(2, 9))
+        n = int(rng.integers(2, 90))
+        ev = fuzz.random_primitive_trace(rng, n, nf, n_keys=3, n_granules=int(rng.integers(1, 900)),
+                                         unaligned=bool(rng.integers(2)))
+        k = int(rng.integers(1, 6))
+        cuts = sorted(int(x) for x in rng.integers(1, n, size=k))
+        _run_session(ev, nf, cuts, window_events=window, flags=flags)
+
+
+def test_session_many_readers_across_calls():
+    """Read sets that spill into records survive from one call to the next."""
+    rng = np.random.default_rng(77)
+    for _ in range(15):
+        nf = int(rng.integers(6, 40))
+        ev = fuzz.random_primitive_trace(rng, int(rng.integers(30, 200)), nf, n_keys=4,
+                                         n_granules=int(rng.integers(50, 700)), p_access=0.85)
+        acc = ev["kind"] == EV_ACCESS
+        ev["mode"][acc & (rng.random(len(ev)) < 0.8)] = 0
+        cuts = sorted(int(x) for x in rng.integers(1, len(ev), size=4))
+        for flags in (0, cs.CUSAN_CHECK_FORCE_LANES):
+            _run_session(ev, nf, cuts, flags=flags)
+
+
+@pytest.mark.parametrize("c", [2, 3, 5])
+def test_session_small_configs(c):
+    w = configs.make(c, "small")
+    ops, args = w.arrays(True)
+    tr = cs.Trace(255)
+    cs.Lowering(tr).cusan_lower_program(ops, args)
+    ev = tr.cusan_trace_read()
+    cuts = list(np.linspace(0, len(ev), 7).astype(int)[1:-1])
+    ref = _run_session(ev, 255, cuts, window_events=64)
+    assert ref["n_race_granules"] > 0
+
+
+def test_session_rejects_shards_and_shrinking():
+    tr = cs.Trace(4)
+    with pytest.raises(cs.CusanError):
+        cs.Session(tr, nshards=2)
+    ses = cs.Session(tr)
+    tr.cusan_trace_append_access(0, 1, 0x1000, 64)
+    tr.cusan_trace_append_access(1, 1, 0x1000, 64)
+    assert ses.check().n_race_granules == 8
+    assert ses.check().n_race_granules == 0          # nothing new
+    ses.close()
