@@ -119,6 +119,12 @@ typedef struct cusan_check_opts {
  * cusan_plan_workspace_bytes, allocates device memory (e.g. a torch tensor from PyTorch's caching
  * allocator) and calls cusan_plan_bind_workspace before cusan_plan_run. */
 #define CUSAN_CHECK_DEFER_WORKSPACE 2
+/* Interval-compressed tracking (the paper's proposed remedy for the cost of
+ * tracking whole allocations): one shadow cell per elementary interval instead
+ * of one per granule.  Exact — every granule of an elementary interval is covered by the same
+ * accesses, so all its cells would hold the same state — and the shadow shrinks from
+ * 8 B × granules to 8 B × intervals.  Results are identical to the per-granule shadow. */
+#define CUSAN_CHECK_INTERVAL_SHADOW 4
 
 /* Defaults: nshards 1, shard 0, device 0, window_events 0, persist 0, max_runs 0, all NULL. */
 void cusan_check_opts_init(cusan_check_opts* o);

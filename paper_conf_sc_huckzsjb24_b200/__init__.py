@@ -171,6 +171,7 @@ def _report(h, max_runs):
 
 
 CUSAN_CHECK_DEFER_WORKSPACE = 2
+CUSAN_CHECK_INTERVAL_SHADOW = 4
 
 
 class Plan:

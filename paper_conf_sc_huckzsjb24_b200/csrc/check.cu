@@ -361,14 +361,16 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
             while (t >= spans[s + 1].tile0) s++;   // spans[nspans] is a sentinel
             const DSpan sp = spans[s];
             const uint64_t x0 = (t - sp.tile0) * sp.rsize;
-            const uint64_t n = min((uint64_t)sp.rsize, sp.len - x0);
+            const uint64_t n = min((uint64_t)sp.rsize, sp.len - x0);   // granules of the range
+            const bool comp = sp.flags & SPAN_COMPRESSED;           // f3: one cell per interval
+            const uint64_t ncell = comp ? 1 : n;
             uint2* cells = k.shadow + sp.dense_begin + x0;      // 256-B aligned (CELL_ALIGN)
             const uint2* src = src_cells(sp, k) + x0;
             const uint4* cells2 = reinterpret_cast<const uint4*>(src);
-            const uint64_t n2 = n >> 1;                         // cell pairs
+            const uint64_t n2 = ncell >> 1;                     // cell pairs
             // ---- pass 1: stream the range's cells in and vote that they are all equal ----------
             uint2 c = make_uint2(0, 0);            // first window of the interval: known empty
-            bool uniform = !force_lanes;
+            bool uniform = comp || !force_lanes;
             if (uniform && (sp.flags & SPAN_LOAD)) {
                 c = src[0];
                 bool ok = true;
@@ -382,12 +384,12 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                         for (int u = 0; u < UL; u++)
                             ok &= ((v[u].x ^ c.x) | (v[u].y ^ c.y) | (v[u].z ^ c.x) | (v[u].w ^ c.y)) == 0u;
                     }
-                    if ((n & 1) && lane == 0) {
-                        const uint2 tl = __ldcs(src + n - 1);
+                    if ((ncell & 1) && lane == 0) {
+                        const uint2 tl = __ldcs(src + ncell - 1);
                         ok &= tl.x == c.x && tl.y == c.y;
                     }
                 } else {                           // a session's old-layout source off a 16-B boundary
-                    for (uint64_t i = lane; i < n; i += 32) {
+                    for (uint64_t i = lane; i < ncell; i += 32) {
                         const uint2 v = __ldcs(src + i);
                         ok &= v.x == c.x && v.y == c.y;
                     }
@@ -471,7 +473,7 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                     for (int u = 0; u < UL; u++)
                         if (i + u * 32 < n2) __stcs(out2 + i + u * 32, cc);
                 }
-                if ((n & 1) && lane == 0) __stcs(cells + n - 1, c);
+                if ((ncell & 1) && lane == 0) __stcs(cells + ncell - 1, c);
             }
             __syncwarp();
         }
@@ -577,7 +579,8 @@ static void build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& ou
             // warp range: long enough that replaying the window's accesses once per range stays
             // small next to streaming its cells, capped for balance; spans that move no cells
             // are one range each
-            const bool moves = s.flags & (SPAN_LOAD | SPAN_STORE);
+            const bool comp = s.flags & SPAN_COMPRESSED;
+            const bool moves = !comp && (s.flags & (SPAN_LOAD | SPAN_STORE));
             uint64_t rs;
             if (moves)
                 rs = std::min<uint64_t>(std::max<uint64_t>((uint64_t)CUSAN_RANGE_PER_ACCESS * s.list_cnt,
@@ -594,8 +597,8 @@ static void build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& ou
             d.weight0 = weight;
             tiles += nt;
             weight += nt * d.rweight;
-            if (moves) out.need_shadow = true;
-            out.cell_bytes += s.len * (((s.flags & SPAN_LOAD) ? 8 : 0) + ((s.flags & SPAN_STORE) ? 8 : 0));
+            if (s.flags & (SPAN_LOAD | SPAN_STORE)) out.need_shadow = true;
+            out.cell_bytes += (comp ? 1 : s.len) * (((s.flags & SPAN_LOAD) ? 8 : 0) + ((s.flags & SPAN_STORE) ? 8 : 0));
             ds.push_back(d);
         }
         win.nspans = (uint32_t)(ds.size() - win.span_off);
@@ -1030,6 +1033,7 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
     std::vector<uint64_t> old_src(hp.iv.size(), UINT64_MAX);
     std::vector<CopySeg> segs;
     uint64_t copy_cells_n = 0;
+    const bool compressed = (s->opts.flags & CUSAN_CHECK_INTERVAL_SHADOW) != 0;
     {
         size_t j = 0;
         for (size_t i = 0; i < hp.iv.size(); i++) {
@@ -1037,11 +1041,13 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
             while (j < s->layout.size() && s->layout[j].abs_begin + s->layout[j].len <= v.abs_begin) j++;
             if (j < s->layout.size() && s->layout[j].abs_begin <= v.abs_begin) {
                 const Interval& u = s->layout[j];
-                old_src[i] = u.dense_begin + (v.abs_begin - u.abs_begin);
+                // compressed layouts (f3) keep one cell per interval: a split piece copies it
+                old_src[i] = compressed ? u.dense_begin : u.dense_begin + (v.abs_begin - u.abs_begin);
+                const uint64_t ncell = compressed ? 1 : v.len;
                 const bool touched = v.list_cnt && hp.inc_acc[v.list_off + v.list_cnt - 1] >= first;
                 if (!touched) {
-                    segs.push_back({copy_cells_n, old_src[i], v.dense_begin, v.len});
-                    copy_cells_n += v.len;
+                    segs.push_back({copy_cells_n, old_src[i], v.dense_begin, ncell});
+                    copy_cells_n += ncell;
                 }
             }
         }

@@ -59,7 +59,9 @@ struct Span {
 // SPAN_LOAD: cells hold state from an earlier window; SPAN_STORE: a later window needs the result;
 // SPAN_FIRST_IN_CALL: the interval's first span of this check (incremental sessions);
 // SPAN_SRC_OLD: LOAD from the previous check's shadow at src_begin (sessions).
-enum : uint32_t { SPAN_LOAD = 1u, SPAN_STORE = 2u, SPAN_SRC_OLD = 4u, SPAN_FIRST_IN_CALL = 8u };
+// SPAN_COMPRESSED: the interval keeps one shadow cell for all its granules (f3).
+enum : uint32_t { SPAN_LOAD = 1u, SPAN_STORE = 2u, SPAN_SRC_OLD = 4u, SPAN_FIRST_IN_CALL = 8u,
+                  SPAN_COMPRESSED = 16u };
 
 struct HostPlan {
     // options

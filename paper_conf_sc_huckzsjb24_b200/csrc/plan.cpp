@@ -200,8 +200,10 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
     }
     // shard-local shadow slots: each clipped interval starts on a CELL_ALIGN boundary so warp
     // ranges can move their cells with aligned 128-bit accesses (≤ CELL_ALIGN−1 unused cells each)
+    // (interval-compressed tracking, f3: one slot per interval)
     hp.iv.clear();
     uint64_t slot = 0;
+    const bool compressed = (o.flags & CUSAN_CHECK_INTERVAL_SHADOW) != 0;
     for (auto& g : giv) {
         uint64_t lo = std::max(g.dense_begin, d_lo), hi = std::min(g.dense_begin + g.len, d_hi);
         if (lo >= hi) continue;
@@ -211,7 +213,7 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
         v.len = hi - lo;
         v.list_off = g.off;
         v.list_cnt = g.cnt;
-        slot = (slot + v.len + CELL_ALIGN - 1) / CELL_ALIGN * CELL_ALIGN;
+        slot = compressed ? slot + 1 : (slot + v.len + CELL_ALIGN - 1) / CELL_ALIGN * CELL_ALIGN;
         hp.iv.push_back(v);
         c.tracked_bytes_shard += 8 * v.len * g.cnt;
     }
@@ -260,7 +262,7 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
             s.list_cnt = q2 - q;
             s.src_begin = v.dense_begin;
             s.flags = (q > v.list_off ? SPAN_LOAD : 0u) | ((q2 < qe || o.persist_shadow) ? SPAN_STORE : 0u) |
-                      (q == first_new ? SPAN_FIRST_IN_CALL : 0u);
+                      (q == first_new ? SPAN_FIRST_IN_CALL : 0u) | (compressed ? SPAN_COMPRESSED : 0u);
             const uint64_t nr = readers.count();
             if ((s.flags & SPAN_STORE) && nr >= 2) {
                 s.rec = (uint32_t)(rec_base + hp.rec_units);

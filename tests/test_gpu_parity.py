@@ -201,3 +201,23 @@ def test_torch_workspace_and_stream():
     assert plan.workspace is not None and plan.workspace.numel() >= plan.workspace_bytes()
     assert_equal(plan.run(), ref)
     plan.close()
+
+
+@pytest.mark.parametrize("window", [0, 1, 5])
+def test_interval_compressed_shadow_matches(window):
+    """f3: one shadow cell per elementary interval gives exactly the per-granule result."""
+    rng = np.random.default_rng(900 + window)
+    for i in range(40):
+        nf = int(rng.integers(2, 12))
+        ev = fuzz.random_primitive_trace(rng, int(rng.integers(1, 90)), nf, n_keys=3,
+                                         n_granules=int(rng.integers(1, 1500)), unaligned=bool(i % 2),
+                                         p_access=0.7)
+        rep = gpu_report(ev, nf, window_events=window, flags=cs.CUSAN_CHECK_INTERVAL_SHADOW)
+        assert_equal(rep, oracle.check_events(ev, nf, threads=2))
+        assert rep.counters["shadow_bytes"] <= 8 * rep.counters["n_intervals"] or window == 0
+    for c in (2, 3, 4, 5):
+        w = configs.make(c, "small")
+        ops, args = w.arrays(True)
+        tr, _ = lower_product(ops, args)
+        ref = oracle.check_events(tr.cusan_trace_read(), 255)
+        assert_equal(cs.check(tr, window_events=max(window, 1) * 40, flags=cs.CUSAN_CHECK_INTERVAL_SHADOW), ref)

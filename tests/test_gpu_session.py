@@ -90,3 +90,13 @@ def test_session_rejects_shards_and_shrinking():
     assert ses.check().n_race_granules == 8
     assert ses.check().n_race_granules == 0          # nothing new
     ses.close()
+
+
+def test_session_interval_compressed():
+    rng = np.random.default_rng(31)
+    for _ in range(20):
+        nf = int(rng.integers(2, 9))
+        n = int(rng.integers(2, 90))
+        ev = fuzz.random_primitive_trace(rng, n, nf, n_keys=3, n_granules=int(rng.integers(1, 900)))
+        cuts = sorted(int(x) for x in rng.integers(1, n, size=int(rng.integers(1, 6))))
+        _run_session(ev, nf, cuts, window_events=int(rng.integers(0, 4)), flags=cs.CUSAN_CHECK_INTERVAL_SHADOW)
