@@ -69,6 +69,23 @@ int cusan_on_mpi_test(cusan_lowering* l, uint64_t request, int flag);
 int cusan_on_mpi_send(cusan_lowering* l, uint64_t buf, uint64_t nbytes);
 int cusan_on_mpi_recv(cusan_lowering* l, uint64_t buf, uint64_t nbytes);
 
+/* ---- host threads and the per-thread default stream ----
+ * Every host thread is a fiber (thread 0 = fiber 0, the others get fibers when first seen).  The
+ * calls after cusan_on_thread(t) are made by thread t: their host-side edges (issue FORKs, host
+ * syncs, MPI requests, host accesses) use t's fiber.  cudaDeviceSynchronize covers the work
+ * submitted so far; work other threads submit after it is not covered.
+ * Stream handles: 1 = cudaStreamLegacy (S0), 2 = cudaStreamPerThread (the calling thread's
+ * per-thread default stream, a blocking stream: "not a non-blocking stream and will synchronize
+ * with the legacy default stream"), 0 = the default stream of the mode set by
+ * cusan_lowering_set_default_stream (legacy unless per_thread != 0).  User stream handles must be
+ * > 2.  K(thread t) = 4<<56 | t. */
+int cusan_on_thread(cusan_lowering* l, uint64_t thread);
+/* pthread_create by the calling thread: issue edge FORK(parent -> child) */
+int cusan_on_thread_create(cusan_lowering* l, uint64_t child);
+/* pthread_join by the calling thread: RELEASE(child, K(child)) + ACQUIRE(caller, K(child)) */
+int cusan_on_thread_join(cusan_lowering* l, uint64_t child);
+int cusan_lowering_set_default_stream(cusan_lowering* l, int per_thread);
+
 /* ---- bulk form: a recorded API program (same layout as tracegen.OP_DTYPE / ARG_DTYPE) -------- */
 enum cusan_api_op {
     CUSAN_OP_MALLOC = 1, CUSAN_OP_FREE = 2, CUSAN_OP_STREAM_CREATE = 3, CUSAN_OP_KERNEL = 4,
@@ -77,14 +94,16 @@ enum cusan_api_op {
     CUSAN_OP_MEMCPY = 11, CUSAN_OP_MEMCPY_ASYNC = 12, CUSAN_OP_MEMSET = 13,
     CUSAN_OP_MEMSET_ASYNC = 14, CUSAN_OP_HOST_ACCESS = 15, CUSAN_OP_MPI_ISEND = 16,
     CUSAN_OP_MPI_IRECV = 17, CUSAN_OP_MPI_WAIT = 18, CUSAN_OP_MPI_SEND = 19,
-    CUSAN_OP_MPI_RECV = 20, CUSAN_OP_MPI_TEST = 21
+    CUSAN_OP_MPI_RECV = 20, CUSAN_OP_MPI_TEST = 21, CUSAN_OP_SET_THREAD = 22,
+    CUSAN_OP_THREAD_CREATE = 23, CUSAN_OP_THREAD_JOIN = 24, CUSAN_OP_DEFAULT_STREAM = 25
 };
 /* 40-byte call record; field use per op is listed in DESIGN.md §"Input formats":
  *   MALLOC a=ptr b=size x=kind | FREE a=ptr | STREAM_CREATE s=stream x=nonblocking
  *   KERNEL s=stream b=first arg x=nargs | STREAM_SYNC s | DEVICE_SYNC | EVENT_RECORD c=event s
  *   EVENT_SYNC c | STREAM_WAIT_EVENT s c | STREAM_QUERY s x=success | MEMCPY a=dst b=src c=n x=kind
  *   MEMCPY_ASYNC + s | MEMSET a=ptr c=n | MEMSET_ASYNC + s | HOST_ACCESS a c x=mode
- *   MPI_ISEND / MPI_IRECV a=buf c=n b=request | MPI_WAIT b | MPI_TEST b x=flag | MPI_SEND/RECV a c */
+ *   MPI_ISEND / MPI_IRECV a=buf c=n b=request | MPI_WAIT b | MPI_TEST b x=flag | MPI_SEND/RECV a c
+ *   SET_THREAD a=thread | THREAD_CREATE a=child | THREAD_JOIN a=child | DEFAULT_STREAM x=per_thread */
 typedef struct cusan_api_call {
     uint32_t op, x;
     uint64_t a, b, c, s;

@@ -95,6 +95,9 @@ class Lowering:
             lib.cusan_lowering_destroy(self.h)
             self.h = None
 
+    def cusan_lowering_set_default_stream(self, per_thread: bool):
+        _ck(lib.cusan_lowering_set_default_stream(self.h, int(per_thread)))
+
     def cusan_lowering_fibers(self) -> int:
         n = C.c_uint32()
         _ck(lib.cusan_lowering_fibers(self.h, C.byref(n)))

@@ -114,6 +114,10 @@ PROTOS = {
     "cusan_on_mpi_test": [P, u64, i32],
     "cusan_on_mpi_send": [P, u64, u64],
     "cusan_on_mpi_recv": [P, u64, u64],
+    "cusan_on_thread": [P, u64],
+    "cusan_on_thread_create": [P, u64],
+    "cusan_on_thread_join": [P, u64],
+    "cusan_lowering_set_default_stream": [P, i32],
     "cusan_lower_program": [P, P, u64, P, u64, pu32],
 }
 VOID = {"cusan_check_opts_init"}

@@ -3,9 +3,15 @@
 // CuSan runtime semantics (§IV-A, 606-734) plus MUST's MPI modelling,
 // in the form of SURVEY.md §8(b)'s table.  Every operation on a stream s is bracketed by
 //   prologue:  FORK(H -> s)                         issue order (Fig. 4 rank 1)
-//              s blocking user stream: ACQUIRE(s, K(S0))       legacy barrier (Fig. 3 (i))
-//              s = S0: ACQUIRE(S0, K(u)) ∀ blocking user u     legacy barrier (Fig. 3 (ii))
+//              s blocking stream: ACQUIRE(s, K(S0))            legacy barrier (Fig. 3 (i))
+//              s = S0: ACQUIRE(S0, K(u)) ∀ blocking u          legacy barrier (Fig. 3 (ii))
 //   epilogue:  RELEASE(s, K(s))                     AnnotateHappensBefore
+// H is the calling host thread's fiber.  Host threads and per-thread default streams (SURVEY §8(f)
+// f4): thread creation is an issue edge FORK(parent -> child), a join is
+// RELEASE(child, K(thread)) + ACQUIRE(parent, K(thread)); a per-thread default stream is a blocking
+// stream of its thread ("not a non-blocking stream and will synchronize with the legacy default
+// stream").  Stream handle 1 = cudaStreamLegacy, 2 = cudaStreamPerThread,
+// 0 = the default stream of the selected mode.
 #include <algorithm>
 #include <map>
 #include <new>
@@ -18,22 +24,30 @@
 using namespace cusan;
 
 namespace {
-constexpr uint32_t H = 0, S0 = 1;
+constexpr uint32_t S0 = 1;
+constexpr uint64_t STREAM_LEGACY = 1, STREAM_PER_THREAD = 2;
 inline uint64_t K_stream(uint32_t f) { return (1ull << 56) | f; }
 inline uint64_t K_event(uint64_t e) { return (2ull << 56) | e; }
 inline uint64_t K_req(uint64_t r) { return (3ull << 56) | r; }
+inline uint64_t K_thread(uint64_t t) { return (4ull << 56) | t; }
 }  // namespace
 
 struct cusan_lowering {
     cusan_trace* trace;
-    std::unordered_map<uint64_t, uint32_t> stream_fiber;   // stream handle -> fiber
-    std::vector<uint32_t> streams;                         // S0, then user streams (creation order)
-    std::vector<uint32_t> blocking;                        // blocking user streams (creation order)
+    std::unordered_map<uint64_t, uint32_t> stream_fiber;   // user stream handle -> fiber
+    std::vector<uint32_t> streams;                         // S0, then streams (creation order)
+    std::vector<uint32_t> blocking;                        // blocking streams (creation order)
     std::vector<char> is_blocking;                         // by fiber
     uint32_t next_fiber = 2;
     std::set<uint32_t> mpi_free;                           // pool of completed request fibers
     std::unordered_map<uint64_t, uint32_t> req_fiber;
     std::map<uint64_t, std::pair<uint64_t, int>> allocs;   // base -> (size, kind)
+    std::unordered_map<uint64_t, uint32_t> thread_fiber;   // host thread -> fiber (thread 0 -> 0)
+    std::unordered_map<uint64_t, uint32_t> ptds;           // host thread -> per-thread default stream
+    uint64_t thread = 0;                                   // calling host thread
+    bool per_thread_mode = false;
+
+    uint32_t H() const { return thread_fiber.at(thread); }
 
     // --- primitives ---------------------------------------------------------------------------
     int access(uint32_t f, int mode, uint64_t addr, uint64_t n) {
@@ -52,12 +66,6 @@ struct cusan_lowering {
         if (p >= it->first && p < it->first + it->second.first) return &*it;
         return nullptr;
     }
-    int fiber_of(uint64_t stream, uint32_t* f) const {
-        auto it = stream_fiber.find(stream);
-        if (it == stream_fiber.end()) return fail(CUSAN_EINVAL, "unknown stream handle");
-        *f = it->second;
-        return CUSAN_OK;
-    }
     int new_fiber(uint32_t* f) {
         uint32_t mf = 0;
         cusan_trace_size(trace, nullptr, &mf);
@@ -66,8 +74,55 @@ struct cusan_lowering {
         if (is_blocking.size() <= *f) is_blocking.resize(*f + 1, 0);
         return CUSAN_OK;
     }
+    int add_stream(uint32_t* f, bool blocking_stream) {
+        int st = new_fiber(f);
+        if (st) return st;
+        streams.push_back(*f);
+        if (blocking_stream) {
+            blocking.push_back(*f);
+            is_blocking[*f] = 1;
+        }
+        return CUSAN_OK;
+    }
+    // the calling thread's per-thread default stream (a blocking stream), created on first use
+    int thread_ptds(uint32_t* f) {
+        auto it = ptds.find(thread);
+        if (it != ptds.end()) {
+            *f = it->second;
+            return CUSAN_OK;
+        }
+        int st = add_stream(f, true);
+        if (!st) ptds[thread] = *f;
+        return st;
+    }
+    int fiber_of(uint64_t stream, uint32_t* f) {
+        if (stream == 0) {
+            if (per_thread_mode) return thread_ptds(f);
+            *f = S0;
+            return CUSAN_OK;
+        }
+        if (stream == STREAM_LEGACY) {
+            *f = S0;
+            return CUSAN_OK;
+        }
+        if (stream == STREAM_PER_THREAD) return thread_ptds(f);
+        auto it = stream_fiber.find(stream);
+        if (it == stream_fiber.end()) return fail(CUSAN_EINVAL, "unknown stream handle");
+        *f = it->second;
+        return CUSAN_OK;
+    }
+    int thread_fiber_of(uint64_t t, uint32_t* f) {
+        auto it = thread_fiber.find(t);
+        if (it != thread_fiber.end()) {
+            *f = it->second;
+            return CUSAN_OK;
+        }
+        int st = new_fiber(f);
+        if (!st) thread_fiber[t] = *f;
+        return st;
+    }
     int prologue(uint32_t f) {
-        int st = sync(CUSAN_FORK, f, H);
+        int st = sync(CUSAN_FORK, f, H());
         if (st) return st;
         if (f != S0 && f < is_blocking.size() && is_blocking[f]) return sync(CUSAN_ACQUIRE, f, K_stream(S0));
         if (f == S0)
@@ -78,16 +133,17 @@ struct cusan_lowering {
     int epilogue(uint32_t f) { return sync(CUSAN_RELEASE, f, K_stream(f)); }
     // cudaStreamSynchronize; on S0 also every blocking stream (724-727)
     int host_sync_stream(uint32_t f) {
-        int st = sync(CUSAN_ACQUIRE, H, K_stream(f));
+        int st = sync(CUSAN_ACQUIRE, H(), K_stream(f));
         if (st || f != S0) return st;
         for (uint32_t u : blocking)
-            if ((st = sync(CUSAN_ACQUIRE, H, K_stream(u)))) return st;
+            if ((st = sync(CUSAN_ACQUIRE, H(), K_stream(u)))) return st;
         return CUSAN_OK;
     }
-    // cudaDeviceSynchronize: every stream
+    // cudaDeviceSynchronize: every stream; work other threads submit
+    // afterwards comes later in the trace and is not covered
     int host_sync_device() {
         for (uint32_t f : streams) {
-            int st = sync(CUSAN_ACQUIRE, H, K_stream(f));
+            int st = sync(CUSAN_ACQUIRE, H(), K_stream(f));
             if (st) return st;
         }
         return CUSAN_OK;
@@ -105,9 +161,9 @@ int cusan_lowering_create(cusan_trace* trace, cusan_lowering** out) {
     cusan_lowering* l = new (std::nothrow) cusan_lowering;
     if (!l) return fail(CUSAN_ENOMEM, "cannot allocate lowering");
     l->trace = trace;
-    l->stream_fiber[0] = S0;
     l->streams.push_back(S0);
     l->is_blocking.assign(2, 0);
+    l->thread_fiber[0] = 0;
     *out = l;
     return CUSAN_OK;
 }
@@ -138,15 +194,11 @@ int cusan_on_free(cusan_lowering* l, uint64_t) {
 
 int cusan_on_stream_create(cusan_lowering* l, uint64_t stream, int nonblocking) {
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    if (stream <= STREAM_PER_THREAD) return fail(CUSAN_EINVAL, "stream handles 0, 1, 2 are reserved");
     uint32_t f = 0;
-    int st = l->new_fiber(&f);
+    int st = l->add_stream(&f, !nonblocking);   // track the non-blocking attribute
     if (st) return st;
     l->stream_fiber[stream] = f;
-    l->streams.push_back(f);
-    if (!nonblocking) {                    // track the non-blocking attribute
-        l->blocking.push_back(f);
-        l->is_blocking[f] = 1;
-    }
     return CUSAN_OK;
 }
 
@@ -189,7 +241,7 @@ int cusan_on_event_record(cusan_lowering* l, uint64_t event, uint64_t stream) {
 
 int cusan_on_event_sync(cusan_lowering* l, uint64_t event) {
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
-    return l->sync(CUSAN_ACQUIRE, H, K_event(event));
+    return l->sync(CUSAN_ACQUIRE, l->H(), K_event(event));
 }
 
 int cusan_on_stream_wait_event(cusan_lowering* l, uint64_t stream, uint64_t event) {
@@ -212,33 +264,33 @@ int cusan_on_memcpy(cusan_lowering* l, uint64_t dst, uint64_t src, uint64_t n,
                     enum cusan_copy_kind kind, int async, uint64_t stream) {
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
     if ((unsigned)kind > 3) return fail(CUSAN_EINVAL, "bad copy kind");
-    uint32_t f = S0;
-    int st = async ? l->fiber_of(stream, &f) : CUSAN_OK;
+    uint32_t f = 0;
+    int st = l->fiber_of(async ? stream : 0, &f);              // cudaMemcpy: the default stream
     if (st || (st = l->prologue(f))) return st;
     if (l->tracked(dst, n) && (st = l->access(f, CUSAN_WRITE, dst, n))) return st;
     if (l->tracked(src, n) && (st = l->access(f, CUSAN_READ, src, n))) return st;
     if ((st = l->epilogue(f))) return st;
     if (!async && kind != CUSAN_D2D)
-        return l->sync(CUSAN_ACQUIRE, H, K_stream(S0));
+        return l->sync(CUSAN_ACQUIRE, l->H(), K_stream(f));
     return CUSAN_OK;
 }
 
 int cusan_on_memset(cusan_lowering* l, uint64_t ptr, uint64_t n, int async, uint64_t stream) {
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
-    uint32_t f = S0;
-    int st = async ? l->fiber_of(stream, &f) : CUSAN_OK;
+    uint32_t f = 0;
+    int st = l->fiber_of(async ? stream : 0, &f);
     if (st || (st = l->prologue(f))) return st;
     auto* a = l->find(ptr);
     if (l->tracked(ptr, n) && (st = l->access(f, CUSAN_WRITE, ptr, n))) return st;
     if ((st = l->epilogue(f))) return st;
     if (!async && a && a->second.second == CUSAN_MEM_PINNED)
-        return l->sync(CUSAN_ACQUIRE, H, K_stream(S0));
+        return l->sync(CUSAN_ACQUIRE, l->H(), K_stream(f));
     return CUSAN_OK;
 }
 
 int cusan_on_host_access(cusan_lowering* l, uint64_t addr, uint64_t n, enum cusan_mode mode) {
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
-    return l->access(H, mode ? CUSAN_WRITE : CUSAN_READ, addr, n);
+    return l->access(l->H(), mode ? CUSAN_WRITE : CUSAN_READ, addr, n);
 }
 
 static int mpi_nonblocking(cusan_lowering* l, uint64_t buf, uint64_t n, uint64_t req, int mode) {
@@ -252,7 +304,7 @@ static int mpi_nonblocking(cusan_lowering* l, uint64_t buf, uint64_t n, uint64_t
         if (st) return st;
     }
     l->req_fiber[req] = m;
-    int st = l->sync(CUSAN_FORK, m, H);    // fiber per non-blocking request
+    int st = l->sync(CUSAN_FORK, m, l->H());   // fiber per non-blocking request
     if (st || (st = l->access(m, mode, buf, n))) return st;
     return l->sync(CUSAN_RELEASE, m, K_req(req));
 }
@@ -267,7 +319,7 @@ int cusan_on_mpi_irecv(cusan_lowering* l, uint64_t buf, uint64_t n, uint64_t req
 
 int cusan_on_mpi_wait(cusan_lowering* l, uint64_t req) {
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
-    int st = l->sync(CUSAN_ACQUIRE, H, K_req(req));
+    int st = l->sync(CUSAN_ACQUIRE, l->H(), K_req(req));
     if (st) return st;
     auto it = l->req_fiber.find(req);
     if (it != l->req_fiber.end()) {
@@ -284,12 +336,41 @@ int cusan_on_mpi_test(cusan_lowering* l, uint64_t req, int flag) {
 
 int cusan_on_mpi_send(cusan_lowering* l, uint64_t buf, uint64_t n) {
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
-    return l->access(H, CUSAN_READ, buf, n);
+    return l->access(l->H(), CUSAN_READ, buf, n);
 }
 
 int cusan_on_mpi_recv(cusan_lowering* l, uint64_t buf, uint64_t n) {
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
-    return l->access(H, CUSAN_WRITE, buf, n);
+    return l->access(l->H(), CUSAN_WRITE, buf, n);
+}
+
+int cusan_on_thread(cusan_lowering* l, uint64_t thread) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    uint32_t f = 0;
+    int st = l->thread_fiber_of(thread, &f);
+    if (!st) l->thread = thread;
+    return st;
+}
+
+int cusan_on_thread_create(cusan_lowering* l, uint64_t child) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    uint32_t f = 0;
+    int st = l->thread_fiber_of(child, &f);
+    return st ? st : l->sync(CUSAN_FORK, f, l->H());           // creation is an issue edge
+}
+
+int cusan_on_thread_join(cusan_lowering* l, uint64_t child) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    auto it = l->thread_fiber.find(child);
+    if (it == l->thread_fiber.end()) return CUSAN_OK;
+    int st = l->sync(CUSAN_RELEASE, it->second, K_thread(child));   // the child's end ...
+    return st ? st : l->sync(CUSAN_ACQUIRE, l->H(), K_thread(child));   // ... HB the join
+}
+
+int cusan_lowering_set_default_stream(cusan_lowering* l, int per_thread) {
+    if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    l->per_thread_mode = per_thread != 0;
+    return CUSAN_OK;
 }
 
 int cusan_lower_program(cusan_lowering* l, const cusan_api_call* calls, uint64_t n,
@@ -339,6 +420,10 @@ int cusan_lower_program(cusan_lowering* l, const cusan_api_call* calls, uint64_t
             case CUSAN_OP_MPI_TEST: st = cusan_on_mpi_test(l, c.b, (int)c.x); break;
             case CUSAN_OP_MPI_SEND: st = cusan_on_mpi_send(l, c.a, c.c); break;
             case CUSAN_OP_MPI_RECV: st = cusan_on_mpi_recv(l, c.a, c.c); break;
+            case CUSAN_OP_SET_THREAD: st = cusan_on_thread(l, c.a); break;
+            case CUSAN_OP_THREAD_CREATE: st = cusan_on_thread_create(l, c.a); break;
+            case CUSAN_OP_THREAD_JOIN: st = cusan_on_thread_join(l, c.a); break;
+            case CUSAN_OP_DEFAULT_STREAM: st = cusan_lowering_set_default_stream(l, (int)c.x); break;
             default: return fail(CUSAN_EINVAL, "unknown API op");
         }
         if (st) return st;

@@ -50,7 +50,7 @@ def parse(path: str = GOLDEN) -> list[Listing]:
         if cmd == "listing":
             cur = Listing(rest[0], Program())
             listings.append(cur)
-            env = {"default": 0}
+            env = {"default": 0, "legacy": 1, "ptds": 2}   # CUDA's stream handles
             continue
         p = cur.program
 
@@ -112,6 +112,14 @@ def parse(path: str = GOLDEN) -> list[Listing]:
             labels = [label] if label else None
         elif cmd == "free":
             p.free(env[rest[0]])
+        elif cmd == "mode":
+            p.default_stream_mode(rest[0] == "per-thread")
+        elif cmd == "thread":
+            p.set_thread(int(rest[0]))
+        elif cmd == "tcreate":
+            p.thread_create(int(rest[0]))
+        elif cmd == "tjoin":
+            p.thread_join(int(rest[0]))
         elif cmd == "expect":
             if rest[0] == "race":
                 cur.expect.append((rest[1], rest[2], int(rest[3]) if len(rest) > 3 else None))

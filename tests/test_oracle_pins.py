@@ -117,7 +117,8 @@ def test_fully_synchronised_programs_are_race_free():
     """DeviceSynchronize + completion of every request after each call orders everything."""
     rng = np.random.default_rng(11)
     for _ in range(40):
-        p = fuzz.random_program(rng, int(rng.integers(5, 40)))
+        # single host thread: concurrent host threads would need joins, not device syncs
+        p = fuzz.random_program(rng, int(rng.integers(5, 40)), threads=False)
         ops, args = p.arrays()
         from tracegen.program import Program, OP_MPI_ISEND, OP_MPI_IRECV, OP_MPI_WAIT, OP_MPI_TEST
         q = Program()

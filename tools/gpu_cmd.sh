@@ -1,1 +1,2 @@
-timeout 900 python -m pytest tests/test_gpu_capture.py -x -q 2>&1 | tail -30
+timeout 1500 python -m pytest tests -m gpu -x -q 2>&1 | tail -5
+python __graft_entry__.py smoke 2>&1 | tail -3

@@ -43,15 +43,21 @@ def random_primitive_trace(rng: np.random.Generator, n_events: int, n_fibers: in
 
 
 def random_program(rng: np.random.Generator, n_ops: int, n_allocs: int = 3, n_streams: int = 3,
-                   alloc_bytes: int = 512) -> Program:
+                   alloc_bytes: int = 512, threads: bool | None = None) -> Program:
     """Random CUDA-aware MPI call sequence over a few allocations, blocking and non-blocking
     streams, events and requests (no attempt at correctness: most traces are racy)."""
     p = Program()
+    threads_on = rng.random() < 0.4 if threads is None else threads   # host threads / PTDS
+    if threads_on and rng.random() < 0.5:
+        p.default_stream_mode(True)
     kinds = [MEM_DEVICE, MEM_DEVICE, MEM_MANAGED, MEM_PINNED]
     allocs = [p.malloc(alloc_bytes + 8 * int(rng.integers(0, 16)), kind=kinds[i % len(kinds)])
               for i in range(n_allocs)]
     sizes = dict((a, s) for a, s, _ in p.allocs)
-    streams = [0] + [p.stream_create(nonblocking=bool(i % 2)) for i in range(n_streams)]
+    streams = [0, 1, 2] + [p.stream_create(nonblocking=bool(i % 2)) for i in range(n_streams)]
+    if not threads_on:
+        streams = [0] + streams[3:]
+    live_threads = [0]
     events = [p.new_event() for _ in range(3)]
     open_reqs: list[int] = []
 
@@ -62,6 +68,17 @@ def random_program(rng: np.random.Generator, n_ops: int, n_allocs: int = 3, n_st
         return a + off, ln
 
     for _ in range(n_ops):
+        if threads_on and rng.random() < 0.15:       # thread create / switch / join
+            u = rng.random()
+            if u < 0.4 and len(live_threads) < 4:
+                child = max(live_threads) + 1
+                p.thread_create(child)
+                live_threads.append(child)
+            elif u < 0.8:
+                p.set_thread(int(rng.choice(live_threads)))
+            elif len(live_threads) > 1:
+                p.thread_join(int(rng.choice(live_threads[1:])))
+            continue
         op = int(rng.integers(16))
         s = streams[int(rng.integers(len(streams)))]
         a = allocs[int(rng.integers(n_allocs))]

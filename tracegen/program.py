@@ -44,6 +44,10 @@ OP_MPI_WAIT = 18         # b=request
 OP_MPI_SEND = 19         # a=buf c=nbytes
 OP_MPI_RECV = 20         # a=buf c=nbytes
 OP_MPI_TEST = 21         # b=request x=1 if flag returned true
+OP_SET_THREAD = 22       # a=host thread id: the calls that follow are made by this thread
+OP_THREAD_CREATE = 23    # a=child thread id (created by the current thread)
+OP_THREAD_JOIN = 24      # a=child thread id (joined by the current thread)
+OP_DEFAULT_STREAM = 25   # x=1: per-thread default stream mode (handle 0), x=0: legacy (default)
 
 OPS = {v: k for k, v in dict(globals()).items() if k.startswith("OP_") and isinstance(v, int)}
 
@@ -54,7 +58,10 @@ CPY_H2H, CPY_H2D, CPY_D2H, CPY_D2D = 0, 1, 2, 3
 # access modes of kernel arguments (R, W or RW)
 MODE_R, MODE_W, MODE_RW = 0, 1, 2
 STREAM_NONBLOCKING = 1
-DEFAULT_STREAM = 0       # stream handle 0 = legacy default stream
+DEFAULT_STREAM = 0       # stream handle 0 = the default stream (legacy, or per-thread in that mode)
+STREAM_LEGACY = 1        # cudaStreamLegacy
+STREAM_PER_THREAD = 2    # cudaStreamPerThread
+FIRST_USER_STREAM = 16   # generated user-stream handles start here (clear of CUDA's special handles)
 
 # ---------------------------------------------------------------------------------------------
 # Primitive trace records (24 B): kind u8, mode u8, pad u16, fiber u32, a u64, b u64
@@ -75,7 +82,7 @@ class Program:
         self.ops: list[tuple] = []
         self.args: list[tuple] = []
         self._next_addr = base
-        self._next_stream = 1
+        self._next_stream = FIRST_USER_STREAM
         self._next_event = 1
         self._next_req = 1
         self.allocs: list[tuple[int, int, int]] = []   # (ptr, size, kind)
@@ -167,6 +174,19 @@ class Program:
 
     def recv(self, buf: int, n: int):
         self.ops.append((OP_MPI_RECV, 0, buf, 0, n, 0))
+
+    # -- host threads and the per-thread default stream --------------------
+    def set_thread(self, thread: int):
+        self.ops.append((OP_SET_THREAD, 0, thread, 0, 0, 0))
+
+    def thread_create(self, child: int):
+        self.ops.append((OP_THREAD_CREATE, 0, child, 0, 0, 0))
+
+    def thread_join(self, child: int):
+        self.ops.append((OP_THREAD_JOIN, 0, child, 0, 0, 0))
+
+    def default_stream_mode(self, per_thread: bool):
+        self.ops.append((OP_DEFAULT_STREAM, 1 if per_thread else 0, 0, 0, 0, 0))
 
     # -- output -------------------------------------------------------------------------------
     def arrays(self) -> tuple[np.ndarray, np.ndarray]:
