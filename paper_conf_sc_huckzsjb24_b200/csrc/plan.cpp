@@ -31,7 +31,12 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
         return fail(CUSAN_EINVAL, "need 0 <= shard < nshards");
     if (o.window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
     hp.opts = o;
-    const uint32_t F = t.max_fibers;
+    // clock width = fibers the trace actually uses (≤ max_fibers)
+    uint32_t F = 1;
+    for (const auto& e : t.ev) {
+        F = std::max<uint32_t>(F, e.fiber + 1);
+        if (e.kind == CUSAN_EV_FORK) F = std::max<uint32_t>(F, (uint32_t)e.a + 1);
+    }
     hp.F = F;
     cusan_counters& c = hp.ctr;
     c = cusan_counters{};
