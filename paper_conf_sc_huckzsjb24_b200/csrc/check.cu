@@ -61,6 +61,12 @@ constexpr int UL = CUSAN_UL;            // 16-B loads / stores in flight per lan
 #ifndef CUSAN_RANGE_MAX
 #define CUSAN_RANGE_MAX 262144
 #endif
+#ifndef CUSAN_RANGES_PER_WARP
+#define CUSAN_RANGES_PER_WARP 1
+#endif
+#ifndef CUSAN_RANGE_BAL_MIN
+#define CUSAN_RANGE_BAL_MIN 4096
+#endif
 constexpr int GRAB = 2;                 // ranges a warp takes per dynamic-scheduler grab
 constexpr int WARPS = 8;                // warps per block
 constexpr int THREADS = 32 * WARPS;
@@ -564,6 +570,13 @@ static void build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& ou
         Window win{};
         win.span_off = ds.size();
         uint64_t tiles = 0, weight = 0;
+        // balance: at least RANGES_PER_WARP ranges per warp of a full grid in this window
+        uint64_t moving = 0;
+        for (uint64_t i = hp.win_span_off[w]; i < hp.win_span_off[w + 1]; i++)
+            if (!(hp.spans[i].flags & SPAN_COMPRESSED) && (hp.spans[i].flags & (SPAN_LOAD | SPAN_STORE)))
+                moving += hp.spans[i].len;
+        const uint64_t rs_cap = std::max<uint64_t>(
+            CUSAN_RANGE_BAL_MIN, moving / ((uint64_t)CUSAN_RANGES_PER_WARP * WARPS * std::max(max_blocks, 1)));
         for (uint64_t i = hp.win_span_off[w]; i < hp.win_span_off[w + 1]; i++) {
             const Span& s = hp.spans[i];
             DSpan d{};
@@ -583,9 +596,10 @@ static void build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& ou
             const bool moves = !comp && (s.flags & (SPAN_LOAD | SPAN_STORE));
             uint64_t rs;
             if (moves)
-                rs = std::min<uint64_t>(std::max<uint64_t>((uint64_t)CUSAN_RANGE_PER_ACCESS * s.list_cnt,
-                                                           (uint64_t)CUSAN_RANGE_MIN),
-                                        (uint64_t)CUSAN_RANGE_MAX);
+                rs = std::min<uint64_t>(std::min<uint64_t>(std::max<uint64_t>((uint64_t)CUSAN_RANGE_PER_ACCESS * s.list_cnt,
+                                                                              (uint64_t)CUSAN_RANGE_MIN),
+                                                           (uint64_t)CUSAN_RANGE_MAX),
+                                        rs_cap);
             else
                 rs = std::max<uint64_t>(s.len, 1);
             rs = std::min<uint64_t>((rs + CHUNK - 1) / CHUNK * CHUNK, 1ull << 31);
