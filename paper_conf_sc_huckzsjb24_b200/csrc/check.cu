@@ -61,6 +61,14 @@ constexpr int UL = CUSAN_UL;            // 16-B loads / stores in flight per lan
 #ifndef CUSAN_RANGE_MAX
 #define CUSAN_RANGE_MAX 262144
 #endif
+#ifndef CUSAN_TMA
+#define CUSAN_TMA 1
+#endif
+constexpr uint32_t TMA_CHUNK = 4096;    // bytes per bulk load (double-buffered per warp)
+constexpr uint32_t TMA_PAT = 2048;      // bytes of the store tile per warp
+constexpr uint32_t TMA_MIN_BYTES = 8192; // ranges smaller than this stream through registers
+constexpr uint32_t TMA_WARP_BYTES = 2 * TMA_CHUNK + TMA_PAT + 128;
+constexpr size_t DYN_SMEM = CUSAN_TMA ? (size_t)8 * TMA_WARP_BYTES : 0;   // 8 = WARPS
 #ifndef CUSAN_RANGES_PER_WARP
 #define CUSAN_RANGES_PER_WARP 1
 #endif
@@ -186,6 +194,38 @@ __device__ __forceinline__ bool unordered(uint32_t e, uint32_t f, const uint32_t
     const uint32_t g = e >> 24;
     return g != f && (e & 0xffffffu) > __ldg(row + g);
 }
+
+// ---- TMA bulk copies (cp.async.bulk, sm_90+; SASS UBLKCP) --------------------------------------
+// Used by the streaming passes when CUSAN_TMA: pass 1 pulls the range's cells into a per-warp
+// double buffer in shared memory (mbarrier completion), pass 3 pushes a shared-memory tile filled
+// with the final cell out in bulk.  Addresses 16-B aligned, sizes multiples of 16.
+__device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n .reg .pred p;\n"
+        "WAIT_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra WAIT_%=;\n}\n"
+        ::"r"(smem_u32(bar)), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void bulk_load(void* dst_smem, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(dst_smem)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void bulk_store(void* dst, const void* src_smem, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
+                 ::"l"(dst), "r"(smem_u32(src_smem)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
 // ---- lane path: per-granule read-set records ----------------------------------------------------
 // Record header word: n (bits 0..15) | units (bits 16..23) | PRIVATE (bit 31).  Records written by
@@ -330,6 +370,21 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
     uint32_t* lst = s_list[warp];
+#if CUSAN_TMA
+    extern __shared__ __align__(128) unsigned char dsm[];
+    unsigned char* wsm = dsm + (size_t)warp * TMA_WARP_BYTES;
+    uint4* s_ld0 = reinterpret_cast<uint4*>(wsm);
+    uint4* s_ld1 = reinterpret_cast<uint4*>(wsm + TMA_CHUNK);
+    uint4* s_pat = reinterpret_cast<uint4*>(wsm + 2 * TMA_CHUNK);
+    uint64_t* s_bar = reinterpret_cast<uint64_t*>(wsm + 2 * TMA_CHUNK + TMA_PAT);
+    if (lane == 0) {
+        mbar_init(&s_bar[0]);
+        mbar_init(&s_bar[1]);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+    uint32_t ph0 = 0, ph1 = 0;              // mbarrier phases (warp-uniform)
+#endif
     RunCache rc;
     rc.e = rc.l = 0;
     rc.gb = rc.ge = 0;
@@ -380,6 +435,42 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
             if (uniform && (sp.flags & SPAN_LOAD)) {
                 c = src[0];
                 bool ok = true;
+#if CUSAN_TMA
+                if ((reinterpret_cast<uintptr_t>(src) & 15u) == 0 && n2 * 16 >= TMA_MIN_BYTES) {
+                    // bulk copies through a double buffer in shared memory (TMA engine)
+                    const uint64_t bytes = n2 * 16;
+                    const uint64_t nch = (bytes + TMA_CHUNK - 1) / TMA_CHUNK;
+                    const unsigned char* gsrc = reinterpret_cast<const unsigned char*>(src);
+                    if (lane == 0) {
+                        const uint32_t sz = (uint32_t)umin64(TMA_CHUNK, bytes);
+                        mbar_arrive_expect_tx(&s_bar[0], sz);
+                        bulk_load(s_ld0, gsrc, sz, &s_bar[0]);
+                    }
+                    const uint4 cc = make_uint4(c.x, c.y, c.x, c.y);
+                    for (uint64_t q = 0; q < nch; q++) {
+                        const int st = (int)(q & 1);
+                        if (q + 1 < nch && lane == 0) {          // prefetch the next chunk
+                            const uint64_t off = (q + 1) * TMA_CHUNK;
+                            const uint32_t sz = (uint32_t)umin64(TMA_CHUNK, bytes - off);
+                            mbar_arrive_expect_tx(&s_bar[st ^ 1], sz);
+                            bulk_load(st ? s_ld0 : s_ld1, gsrc + off, sz, &s_bar[st ^ 1]);
+                        }
+                        if (st == 0) { mbar_wait(&s_bar[0], ph0); ph0 ^= 1u; }
+                        else { mbar_wait(&s_bar[1], ph1); ph1 ^= 1u; }
+                        const uint4* buf = st ? s_ld1 : s_ld0;
+                        const uint32_t nv = (uint32_t)(umin64(TMA_CHUNK, bytes - q * TMA_CHUNK) / 16);
+                        for (uint32_t j = lane; j < nv; j += 32) {
+                            const uint4 v = buf[j];
+                            ok &= ((v.x ^ cc.x) | (v.y ^ cc.y) | (v.z ^ cc.z) | (v.w ^ cc.w)) == 0u;
+                        }
+                        __syncwarp();
+                    }
+                    if ((ncell & 1) && lane == 0) {
+                        const uint2 tl = __ldcs(src + ncell - 1);
+                        ok &= tl.x == c.x && tl.y == c.y;
+                    }
+                } else
+#endif
                 if ((reinterpret_cast<uintptr_t>(src) & 15u) == 0) {
                     for (uint64_t i = lane; i < n2; i += 32 * UL) {
                         uint4 v[UL];
@@ -474,6 +565,23 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                 }
                 uint4* out2 = reinterpret_cast<uint4*>(cells);
                 const uint4 cc = make_uint4(c.x, c.y, c.x, c.y);
+#if CUSAN_TMA
+                if (n2 * 16 >= TMA_MIN_BYTES) {
+                    // a shared-memory tile of the final cell, pushed out by bulk copies
+                    if (lane == 0) bulk_wait_read();          // the previous range's stores read the tile
+                    __syncwarp();
+                    for (uint32_t j = lane; j < TMA_PAT / 16; j += 32) s_pat[j] = cc;
+                    fence_async_smem();
+                    __syncwarp();
+                    if (lane == 0) {
+                        unsigned char* gdst = reinterpret_cast<unsigned char*>(out2);
+                        const uint64_t bytes = n2 * 16;
+                        for (uint64_t off = 0; off < bytes; off += TMA_PAT)
+                            bulk_store(gdst + off, s_pat, (uint32_t)umin64(TMA_PAT, bytes - off));
+                        bulk_commit();
+                    }
+                } else
+#endif
                 for (uint64_t i = lane; i < n2; i += 32 * UL) {
 #pragma unroll
                     for (int u = 0; u < UL; u++)
@@ -484,6 +592,10 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
             __syncwarp();
         }
     }
+#if CUSAN_TMA
+    if (lane == 0) bulk_wait_all();                 // bulk stores done before the tile goes away
+    __syncwarp();
+#endif
     if (rc.ge > rc.gb) flush_entry(rc, k);
     if (lane == 0 && rc.nrace) atomicAdd(&k.counters[C_RACE], rc.nrace);
 }
@@ -637,7 +749,9 @@ static int device_info(int device, int* max_blocks) {
     CK(cudaSetDevice(device));
     int sms = 0, per_sm = 0;
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device));
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, shadow_check_window, THREADS, 0));
+    if (DYN_SMEM)
+        CK(cudaFuncSetAttribute(shadow_check_window, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)DYN_SMEM));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, shadow_check_window, THREADS, DYN_SMEM));
     *max_blocks = sms * std::max(per_sm, 1);
     return CUSAN_OK;
 }
@@ -737,7 +851,7 @@ static int launch_all(cusan_plan* p) {
     for (size_t i = 0; i < p->wins.size(); i++) {
         const Window& w = p->wins[i];
         unsigned long long* sched = CUSAN_DYNAMIC ? p->d_counters + N_COUNTERS + i : nullptr;
-        shadow_check_window<<<w.grid, THREADS, 0, p->stream>>>(p->d_spans + w.span_off, w.nspans, w.tiles,
+        shadow_check_window<<<w.grid, THREADS, DYN_SMEM, p->stream>>>(p->d_spans + w.span_off, w.nspans, w.tiles,
                                                                w.weight, k, force_lanes, sched);
     }
     CK(cudaGetLastError());
@@ -1128,7 +1242,7 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
         for (size_t i = 0; i < nwin; i++) {
             const Window& w = tabs.wins[i];
             unsigned long long* sched = CUSAN_DYNAMIC ? d_cnt + N_COUNTERS + i : nullptr;
-            shadow_check_window<<<w.grid, THREADS, 0, s->stream>>>(d_spans + w.span_off, w.nspans, w.tiles, w.weight,
+            shadow_check_window<<<w.grid, THREADS, DYN_SMEM, s->stream>>>(d_spans + w.span_off, w.nspans, w.tiles, w.weight,
                                                                    k, force_lanes, sched);
         }
         CK(cudaGetLastError());
