@@ -64,8 +64,14 @@ constexpr int UL = CUSAN_UL;            // 16-B loads / stores in flight per lan
 #ifndef CUSAN_TMA
 #define CUSAN_TMA 1
 #endif
-constexpr uint32_t TMA_CHUNK = 4096;    // bytes per bulk load (double-buffered per warp)
-constexpr uint32_t TMA_PAT = 2048;      // bytes of the store tile per warp
+#ifndef CUSAN_TMA_CHUNK
+#define CUSAN_TMA_CHUNK 4096
+#endif
+#ifndef CUSAN_TMA_PAT
+#define CUSAN_TMA_PAT 2048
+#endif
+constexpr uint32_t TMA_CHUNK = CUSAN_TMA_CHUNK;   // bytes per bulk load (double-buffered per warp)
+constexpr uint32_t TMA_PAT = CUSAN_TMA_PAT;       // bytes of the store tile per warp
 constexpr uint32_t TMA_MIN_BYTES = 8192; // ranges smaller than this stream through registers
 constexpr uint32_t TMA_WARP_BYTES = 2 * TMA_CHUNK + TMA_PAT + 128;
 constexpr size_t DYN_SMEM = CUSAN_TMA ? (size_t)8 * TMA_WARP_BYTES : 0;   // 8 = WARPS

@@ -183,17 +183,37 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
     const uint64_t total_dense = giv.empty() ? 0 : giv.back().dense_begin + giv.back().len;
     uint64_t d_lo = 0, d_hi = total_dense;
     if (o.nshards > 1 && !giv.empty()) {
-        // boundaries at equal cumulative coverage weight Σ len × cnt
+        // Boundaries at equal cumulative cost.  Per granule: with several windows
+        // the kernel moves the cell 2(k−1) times for an interval touched in k windows (memory-bound);
+        // with one window (or one cell per interval, f3) the work is the accesses replayed, so the
+        // weight is the coverage (accesses covering the granule).
+        const uint64_t Ws = o.window_events > 0 ? (uint64_t)o.window_events : std::max<uint64_t>(n_acc, 1);
+        const bool windowed = Ws < n_acc && !(o.flags & CUSAN_CHECK_INTERVAL_SHADOW);
+        std::vector<uint64_t> wpg(giv.size());
+        for (size_t i = 0; i < giv.size(); i++) {
+            const GIv& g = giv[i];
+            if (!windowed) {
+                wpg[i] = std::max<uint64_t>(g.cnt, 1);
+                continue;
+            }
+            uint64_t k = 0, last = UINT64_MAX;
+            for (uint32_t q = g.off; q < g.off + g.cnt; q++) {
+                const uint64_t w = hp.inc_acc[q] / Ws;
+                if (w != last) { k++; last = w; }
+            }
+            wpg[i] = 2 * (k ? k - 1 : 0) + 1;
+        }
         unsigned __int128 wtot = 0;
-        for (auto& g : giv) wtot += (unsigned __int128)g.len * g.cnt;
+        for (size_t i = 0; i < giv.size(); i++) wtot += (unsigned __int128)giv[i].len * wpg[i];
         auto boundary = [&](int k) -> uint64_t {
             if (k <= 0) return 0;
             if (k >= o.nshards) return total_dense;
             unsigned __int128 target = wtot * (unsigned)k / (unsigned)o.nshards, acc = 0;
-            for (auto& g : giv) {
-                unsigned __int128 w = (unsigned __int128)g.len * g.cnt;
+            for (size_t i = 0; i < giv.size(); i++) {
+                const GIv& g = giv[i];
+                unsigned __int128 w = (unsigned __int128)g.len * wpg[i];
                 if (acc + w >= target) {
-                    uint64_t x = (uint64_t)((target - acc + g.cnt - 1) / g.cnt);
+                    uint64_t x = (uint64_t)((target - acc + wpg[i] - 1) / wpg[i]);
                     return g.dense_begin + std::min<uint64_t>(x, g.len);
                 }
                 acc += w;

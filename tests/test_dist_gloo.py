@@ -108,3 +108,20 @@ def test_shard_partition_balances_coverage(nshards):
     ideal = whole["tracked_bytes"] / nshards
     # equal coverage weight up to one interval's granule boundary rounding
     assert max(abs(p["tracked_bytes_shard"] - ideal) for p in parts) <= 0.01 * ideal + 8 * 1000
+
+
+@pytest.mark.parametrize("nshards", [2, 8])
+def test_windowed_shards_balance_moved_cells(nshards):
+    """Windowed checks are bound by the cells moved, so shards balance granules × windows."""
+    import paper_conf_sc_huckzsjb24_b200 as cs
+    from tracegen import configs
+    w = configs.make(5, "small")
+    ops, args = w.arrays(False)
+    tr = cs.Trace(255)
+    cs.Lowering(tr).cusan_lower_program(ops, args)
+    parts = [cs.describe(tr, nshards=nshards, shard=s, window_events=64) for s in range(nshards)]
+    whole = cs.describe(tr, window_events=64)
+    assert sum(p["shard_granules"] for p in parts) == whole["shard_granules"]
+    assert sum(p["tracked_bytes_shard"] for p in parts) == whole["tracked_bytes"]
+    g = [p["shard_granules"] for p in parts]
+    assert min(g) > 0.5 * max(g)
