@@ -1,1 +1,2 @@
-for v in tools/var_*.so; do echo "== $v"; CUSAN_LIBRARY=$v timeout 300 python tools/quick_timing.py 5,4,3 4096 2>&1 | cut -c1-90; done
+timeout 900 python tools/shard_scaling.py --config 5 --window 4096 2>&1 | tail -6
+timeout 900 python tools/shard_scaling.py --config 4 --window 4096 2>&1 | tail -1
