@@ -1,0 +1,380 @@
+// Plan / check C ABI (host side of steps a3-a5): device span tables, workspace layout and binding,
+// the window launches, overflow re-runs, run download and the canonical report.
+#include <algorithm>
+#include <chrono>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "kernel.cuh"
+
+using namespace cusan;
+
+struct cusan_plan {
+    const cusan_trace* trace = nullptr;
+    HostPlan hp;
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    int max_blocks = 0;
+    // device memory
+    char* own = nullptr;          // library-allocated workspace (null when the caller's is used)
+    char* ws = nullptr;
+    uint64_t ws_bytes = 0;
+    AccRec* d_inc = nullptr;
+    uint32_t* d_segvc = nullptr;
+    DSpan* d_spans = nullptr;
+    unsigned long long* d_counters = nullptr;
+    uint2* d_shadow = nullptr;
+    uint32_t* d_heap = nullptr;
+    uint64_t heap_cap = 0;                  // record units
+    uint32_t* d_heap_own = nullptr;         // grown heap after an overflow
+    cusan_race_run* d_runs = nullptr;
+    cusan_race_run* d_runs_own = nullptr;   // grown run buffer after an overflow
+    uint64_t run_cap = 0;
+    bool need_shadow = false;
+    bool bound = false;                     // workspace carved and tables uploaded
+    uint64_t o_inc = 0, o_seg = 0, o_spans = 0, o_cnt = 0, o_heap = 0, o_shadow = 0, o_runs = 0;
+    std::vector<DSpan> ds;                  // device span tables (host copy, uploaded at bind)
+    std::vector<Window> wins;
+    uint64_t shadow_cell_bytes = 0;
+    uint64_t table_bytes = 0;               // tables uploaded by plan_create
+    std::vector<unsigned long long> counter_init;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+
+    ~cusan_plan() {
+        if (ev0) cudaEventDestroy(ev0);
+        if (ev1) cudaEventDestroy(ev1);
+        if (own) cudaFree(own);
+        if (d_runs_own) cudaFree(d_runs_own);
+        if (d_heap_own) cudaFree(d_heap_own);
+    }
+};
+
+static int plan_bind(cusan_plan* p, char* ws, uint64_t bytes);
+
+void cusan::build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& out) {
+    std::vector<DSpan>& ds = out.ds;
+    ds.clear();
+    ds.reserve(hp.spans.size() + hp.win_span_off.size());
+    out.wins.clear();
+    out.need_shadow = false;
+    out.cell_bytes = 0;
+    for (size_t w = 0; w + 1 < hp.win_span_off.size(); w++) {
+        Window win{};
+        win.span_off = ds.size();
+        uint64_t tiles = 0, weight = 0;
+        // balance: at least RANGES_PER_WARP ranges per warp of a full grid in this window
+        uint64_t moving = 0;
+        for (uint64_t i = hp.win_span_off[w]; i < hp.win_span_off[w + 1]; i++)
+            if (!(hp.spans[i].flags & SPAN_COMPRESSED) && (hp.spans[i].flags & (SPAN_LOAD | SPAN_STORE)))
+                moving += hp.spans[i].len;
+        const uint64_t rs_cap = std::max<uint64_t>(
+            CUSAN_RANGE_BAL_MIN, moving / ((uint64_t)CUSAN_RANGES_PER_WARP * WARPS * std::max(max_blocks, 1)));
+        for (uint64_t i = hp.win_span_off[w]; i < hp.win_span_off[w + 1]; i++) {
+            const Span& s = hp.spans[i];
+            DSpan d{};
+            d.abs_begin = s.abs_begin;
+            d.dense_begin = s.dense_begin;
+            d.len = s.len;
+            d.list_off = s.list_off;
+            d.list_cnt = s.list_cnt;
+            d.flags = s.flags;
+            d.rec = s.rec;
+            d.rec_units = s.rec_units;
+            d.src_begin = s.src_begin;
+            // warp range: long enough that replaying the window's accesses once per range stays
+            // small next to streaming its cells, capped for balance; spans that move no cells
+            // are one range each
+            const bool comp = s.flags & SPAN_COMPRESSED;
+            const bool moves = !comp && (s.flags & (SPAN_LOAD | SPAN_STORE));
+            uint64_t rs;
+            if (moves)
+                rs = std::min<uint64_t>(std::min<uint64_t>(std::max<uint64_t>((uint64_t)CUSAN_RANGE_PER_ACCESS * s.list_cnt,
+                                                                              (uint64_t)CUSAN_RANGE_MIN),
+                                                           (uint64_t)CUSAN_RANGE_MAX),
+                                        rs_cap);
+            else
+                rs = std::max<uint64_t>(s.len, 1);
+            rs = std::min<uint64_t>((rs + CHUNK - 1) / CHUNK * CHUNK, 1ull << 31);
+            d.rsize = (uint32_t)rs;
+            const uint64_t nt = (s.len + rs - 1) / rs;
+            const uint64_t mem = moves ? rs / 32 : 0;
+            d.rweight = (uint32_t)std::min<uint64_t>(mem + 4ull * s.list_cnt + 8, 0xffffffffull);
+            d.tile0 = tiles;
+            d.weight0 = weight;
+            tiles += nt;
+            weight += nt * d.rweight;
+            if (s.flags & (SPAN_LOAD | SPAN_STORE)) out.need_shadow = true;
+            out.cell_bytes += (comp ? 1 : s.len) * (((s.flags & SPAN_LOAD) ? 8 : 0) + ((s.flags & SPAN_STORE) ? 8 : 0));
+            ds.push_back(d);
+        }
+        win.nspans = (uint32_t)(ds.size() - win.span_off);
+        DSpan sent{};
+        sent.tile0 = tiles;
+        sent.weight0 = weight;
+        ds.push_back(sent);
+        win.tiles = tiles;
+        win.weight = weight;
+        win.grid = (uint32_t)std::min<uint64_t>((uint64_t)max_blocks, (tiles + WARPS - 1) / WARPS);
+        if (win.grid == 0) win.grid = 1;
+        out.wins.push_back(win);
+    }
+}
+
+int cusan::device_info(int device, int* max_blocks) {
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess || ndev == 0)
+        return fail(CUSAN_ECUDA, std::string("no CUDA device available: ") + cudaGetErrorString(e));
+    if (device < 0 || device >= ndev) return fail(CUSAN_EINVAL, "bad device ordinal");
+    CK(cudaSetDevice(device));
+    int sms = 0, per_sm = 0;
+    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device));
+    CK(shadow_check_blocks_per_sm(&per_sm));
+    *max_blocks = sms * std::max(per_sm, 1);
+    return CUSAN_OK;
+}
+
+static int plan_device_setup(cusan_plan* p) {
+    HostPlan& hp = p->hp;
+    const cusan_check_opts& o = hp.opts;
+    int st0 = device_info(o.device, &p->max_blocks);
+    if (st0) return st0;
+    p->device = o.device;
+    p->stream = (cudaStream_t)o.stream;
+
+    SpanTables st;
+    build_span_tables(hp, p->max_blocks, st);
+    std::vector<DSpan>& ds = st.ds;
+    p->wins = st.wins;
+    p->need_shadow = st.need_shadow;
+    p->shadow_cell_bytes = st.cell_bytes;
+
+    // workspace layout
+    p->heap_cap = hp.rec_units + (1ull << 16);             // pre-assigned records + lane-path room
+    uint64_t off = 0;
+    const uint64_t o_inc = off;     off = align_up(off + hp.inc.size() * sizeof(AccRec));
+    const uint64_t o_seg = off;     off = align_up(off + hp.segvc.size() * sizeof(uint32_t));
+    const uint64_t o_spans = off;   off = align_up(off + ds.size() * sizeof(DSpan));
+    const uint64_t o_cnt = off;     off = align_up(off + (N_COUNTERS + p->wins.size()) * sizeof(unsigned long long));
+    const uint64_t o_heap = off;    off = align_up(off + p->heap_cap * REC_WORDS * sizeof(uint32_t));
+    const uint64_t o_shadow = off;  off = align_up(off + (p->need_shadow ? hp.shadow_cells * sizeof(uint2) : 0));
+    p->run_cap = std::max<uint64_t>(1ull << 16, 4 * p->wins.size() + 1024);
+    const uint64_t o_runs = off;    off = align_up(off + p->run_cap * sizeof(cusan_race_run));
+    p->ws_bytes = off;
+    p->o_inc = o_inc;
+    p->o_seg = o_seg;
+    p->o_spans = o_spans;
+    p->o_cnt = o_cnt;
+    p->o_heap = o_heap;
+    p->o_shadow = o_shadow;
+    p->o_runs = o_runs;
+    p->ds = std::move(ds);
+    p->table_bytes = hp.inc.size() * sizeof(AccRec) + hp.segvc.size() * sizeof(uint32_t) +
+                     p->ds.size() * sizeof(DSpan);
+    hp.ctr.shadow_bytes = p->need_shadow ? hp.shadow_cells * sizeof(uint2) : 0;
+    hp.ctr.workspace_bytes = p->ws_bytes;
+    CK(cudaEventCreate(&p->ev0));
+    CK(cudaEventCreate(&p->ev1));
+    if (o.workspace) return plan_bind(p, (char*)o.workspace, o.workspace_bytes);
+    if (o.flags & CUSAN_CHECK_DEFER_WORKSPACE) return CUSAN_OK;   // caller binds later
+    cudaError_t me = cudaMalloc((void**)&p->own, std::max<uint64_t>(off, ALIGN));
+    if (me != cudaSuccess) return fail(CUSAN_ENOMEM, std::string("cudaMalloc workspace: ") + cudaGetErrorString(me));
+    return plan_bind(p, p->own, off);
+}
+
+// Carve the workspace and upload the tables (a2 -> HBM).
+static int plan_bind(cusan_plan* p, char* ws, uint64_t bytes) {
+    if (bytes < p->ws_bytes)
+        return fail(CUSAN_ENOMEM, "workspace too small: need " + std::to_string(p->ws_bytes) + " bytes");
+    const HostPlan& hp = p->hp;
+    CK(cudaSetDevice(p->device));
+    p->ws = ws;
+    p->d_inc = (AccRec*)(p->ws + p->o_inc);
+    p->d_segvc = (uint32_t*)(p->ws + p->o_seg);
+    p->d_spans = (DSpan*)(p->ws + p->o_spans);
+    p->d_counters = (unsigned long long*)(p->ws + p->o_cnt);
+    p->d_shadow = p->need_shadow ? (uint2*)(p->ws + p->o_shadow) : nullptr;
+    if (!p->d_runs_own) p->d_runs = (cusan_race_run*)(p->ws + p->o_runs);
+    if (!p->d_heap_own) p->d_heap = (uint32_t*)(p->ws + p->o_heap);
+    else p->d_heap = p->d_heap_own;
+    CK(cudaMemcpyAsync(p->d_inc, hp.inc.data(), hp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, p->stream));
+    CK(cudaMemcpyAsync(p->d_segvc, hp.segvc.data(), hp.segvc.size() * sizeof(uint32_t), cudaMemcpyHostToDevice, p->stream));
+    CK(cudaMemcpyAsync(p->d_spans, p->ds.data(), p->ds.size() * sizeof(DSpan), cudaMemcpyHostToDevice, p->stream));
+    CK(cudaStreamSynchronize(p->stream));
+    p->bound = true;
+    return CUSAN_OK;
+}
+
+static int launch_all(cusan_plan* p) {
+    // counters: race granules, runs, heap top (after the pre-assigned records), overflow flag
+    // + one dynamic-scheduler counter per window
+    p->counter_init.assign(N_COUNTERS + p->wins.size(), 0ull);
+    p->counter_init[C_HEAP] = p->hp.rec_units;
+    CK(cudaMemcpyAsync(p->d_counters, p->counter_init.data(), p->counter_init.size() * sizeof(unsigned long long),
+                       cudaMemcpyHostToDevice, p->stream));
+    CK(cudaEventRecord(p->ev0, p->stream));
+    Ctx k;
+    k.inc = p->d_inc;
+    k.segvc = p->d_segvc;
+    k.F = p->hp.F;
+    k.shadow = p->d_shadow;
+    k.shadow_old = nullptr;
+    k.cow_all = 0;
+    k.heap = p->d_heap;
+    k.heap_cap = p->heap_cap;
+    k.runs = p->d_runs;
+    k.counters = p->d_counters;
+    k.run_cap = p->run_cap;
+    const int force_lanes = (p->hp.opts.flags & CUSAN_CHECK_FORCE_LANES) ? 1 : 0;
+    for (size_t i = 0; i < p->wins.size(); i++) {
+        const Window& w = p->wins[i];
+        unsigned long long* sched = CUSAN_DYNAMIC ? p->d_counters + N_COUNTERS + i : nullptr;
+        CK(launch_shadow_check(w.grid, p->stream, p->d_spans + w.span_off, w.nspans, w.tiles, w.weight, k, force_lanes,
+                               sched));
+    }
+    CK(cudaGetLastError());
+    CK(cudaEventRecord(p->ev1, p->stream));
+    return CUSAN_OK;
+}
+
+extern "C" {
+
+int cusan_plan_create(const cusan_trace* t, const cusan_check_opts* o, cusan_plan** out) {
+    if (!t || !o || !out) return fail(CUSAN_EINVAL, "null argument");
+    *out = nullptr;
+    cusan_plan* p = new (std::nothrow) cusan_plan;
+    if (!p) return fail(CUSAN_ENOMEM, "cannot allocate plan");
+    p->trace = t;
+    int st;
+    try {
+        st = build_host_plan(t->t, *o, p->hp);
+    } catch (const std::bad_alloc&) {
+        st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
+    }
+    if (!st) st = plan_device_setup(p);
+    if (st) {
+        delete p;
+        return st;
+    }
+    *out = p;
+    return CUSAN_OK;
+}
+
+int cusan_plan_describe(const cusan_trace* t, const cusan_check_opts* o, cusan_counters* out) {
+    if (!t || !o || !out) return fail(CUSAN_EINVAL, "null argument");
+    HostPlan hp;
+    int st;
+    try {
+        st = build_host_plan(t->t, *o, hp);
+    } catch (const std::bad_alloc&) {
+        st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
+    }
+    if (!st) *out = hp.ctr;
+    return st;
+}
+
+int cusan_plan_workspace_bytes(const cusan_plan* p, uint64_t* bytes) {
+    if (!p || !bytes) return fail(CUSAN_EINVAL, "null argument");
+    *bytes = p->ws_bytes;
+    return CUSAN_OK;
+}
+
+int cusan_plan_bind_workspace(cusan_plan* p, void* workspace, uint64_t bytes) {
+    if (!p || !workspace) return fail(CUSAN_EINVAL, "null argument");
+    if (p->own) return fail(CUSAN_ESTATE, "plan already owns a workspace");
+    return plan_bind(p, (char*)workspace, bytes);
+}
+
+int cusan_plan_run(cusan_plan* p, cusan_report** out) {
+    if (!p || !out) return fail(CUSAN_EINVAL, "null argument");
+    *out = nullptr;
+    if (!p->bound) return fail(CUSAN_ESTATE, "plan has no workspace: call cusan_plan_bind_workspace");
+    const auto t_start = std::chrono::steady_clock::now();
+    CK(cudaSetDevice(p->device));
+    unsigned long long cnt[N_COUNTERS];
+    for (int attempt = 0;; attempt++) {
+        int st = launch_all(p);
+        if (st) return st;
+        CK(cudaMemcpyAsync(cnt, p->d_counters, sizeof(cnt), cudaMemcpyDeviceToHost, p->stream));
+        CK(cudaStreamSynchronize(p->stream));
+        const bool runs_ovf = cnt[C_RUNS] > p->run_cap, heap_ovf = cnt[C_HEAP_OVF] != 0;
+        if (!runs_ovf && !heap_ovf) break;
+        if (attempt >= 8) return fail(CUSAN_ENOMEM, "run buffer / spill heap keeps overflowing");
+        if (runs_ovf) {                        // grow the run buffer and re-run (counts are exact)
+            if (p->d_runs_own) cudaFree(p->d_runs_own);
+            p->d_runs_own = nullptr;
+            const uint64_t cap = cnt[C_RUNS] + cnt[C_RUNS] / 8 + 1024;
+            if (cudaMalloc((void**)&p->d_runs_own, cap * sizeof(cusan_race_run)) != cudaSuccess)
+                return fail(CUSAN_ENOMEM, "cannot grow the run buffer");
+            p->d_runs = p->d_runs_own;
+            p->run_cap = cap;
+        }
+        if (heap_ovf) {                        // grow the spill heap (24-bit record index)
+            const uint64_t cap = std::min<uint64_t>(2 * p->heap_cap, (1ull << 24) - 1);
+            if (cap <= p->heap_cap) return fail(CUSAN_ENOMEM, "spill heap exceeds the 24-bit record index");
+            uint32_t* nh = nullptr;
+            if (cudaMalloc((void**)&nh, cap * REC_WORDS * sizeof(uint32_t)) != cudaSuccess)
+                return fail(CUSAN_ENOMEM, "cannot grow the spill heap");
+            if (p->d_heap_own) cudaFree(p->d_heap_own);
+            p->d_heap_own = nh;
+            p->d_heap = nh;
+            p->heap_cap = cap;
+        }
+    }
+    float kms = 0.f;
+    CK(cudaEventElapsedTime(&kms, p->ev0, p->ev1));
+    cusan_report* r = new (std::nothrow) cusan_report;
+    if (!r) return fail(CUSAN_ENOMEM, "cannot allocate report");
+    try {
+        r->runs.resize(cnt[C_RUNS]);
+    } catch (...) {
+        delete r;
+        return fail(CUSAN_ENOMEM, "cannot allocate report runs");
+    }
+    if (cnt[C_RUNS]) {
+        cudaError_t ce = cudaMemcpyAsync(r->runs.data(), p->d_runs, cnt[C_RUNS] * sizeof(cusan_race_run),
+                                         cudaMemcpyDeviceToHost, p->stream);
+        if (ce == cudaSuccess) ce = cudaStreamSynchronize(p->stream);
+        if (ce != cudaSuccess) {
+            delete r;
+            return cuda_fail(ce, "run download");
+        }
+    }
+    canonicalize_runs(r->runs);
+    r->n_runs = r->runs.size();
+    r->n_race_granules = cnt[C_RACE];
+    const uint64_t max_runs = p->hp.opts.max_runs;
+    if (max_runs && r->runs.size() > max_runs) {
+        r->runs.resize(max_runs);
+        r->truncated = 1;
+    }
+    r->ctr = p->hp.ctr;
+    r->ctr.raw_runs = cnt[C_RUNS];
+    r->ctr.kernel_ms = kms;
+    r->ctr.kernel_launches = p->wins.size();
+    r->ctr.shadow_cell_bytes = p->shadow_cell_bytes;
+    r->ctr.h2d_bytes = p->table_bytes + sizeof(unsigned long long) * N_COUNTERS;
+    r->ctr.d2h_bytes = sizeof(cnt) + cnt[C_RUNS] * sizeof(cusan_race_run);
+    r->ctr.run_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count();
+    *out = r;
+    return CUSAN_OK;
+}
+
+int cusan_plan_destroy(cusan_plan* p) {
+    if (!p) return fail(CUSAN_EINVAL, "plan is null");
+    if (p->stream) cudaStreamSynchronize(p->stream);
+    delete p;
+    return CUSAN_OK;
+}
+
+int cusan_check(const cusan_trace* t, const cusan_check_opts* o, cusan_report** out) {
+    cusan_plan* p = nullptr;
+    int st = cusan_plan_create(t, o, &p);
+    if (st) return st;
+    st = cusan_plan_run(p, out);
+    cusan_plan_destroy(p);
+    return st;
+}
+
+}  // extern "C"

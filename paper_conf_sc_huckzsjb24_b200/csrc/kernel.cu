@@ -1,0 +1,579 @@
+// The shadow-check kernels (steps a3, a4) and their launch wrappers.
+//
+// K1 shadow_check_window — one launch per window of consecutive access events.
+//   Shadow cell: 8 B per 8-byte granule {W, R} (FastTrack's representation: the last write as an
+//   epoch, the reads as an epoch while one fiber reads, a read vector when several do), each u32 =
+//   fiber:8 | (event id + 1):24, 0 = empty.  When two or more fibers have read since the last
+//   write, R = SPILL_TAG | r names a read-set record r in the device heap ({header with n,
+//   epoch_1..epoch_n}), so the read set stays exact with a fixed 8-B cell.
+//   The per-granule rule is the FastTrack-style check of SURVEY.md §8(c) step 3:
+//       any access b:      W ≠ ∅ ∧ ¬HB(W, b)            → race (W, b)
+//       write b:           ∀ read r ≠ ∅ ∧ ¬HB(r, b)     → race (r, b);   W := b, R := ∅
+//       read b on fiber f: R[f] := b
+//   with HB(e = (g, i+1), b in segment s of fiber f) ⇔ g = f ∨ i+1 ≤ segvc[s][g].
+//   Work unit = a warp range: consecutive granules of one elementary interval, all covered by the
+//   same accesses of the window.  Warps own contiguous runs of ranges (coverage-weighted).
+//   Per range:
+//     pass 1  stream the cells in (coalesced 128-bit loads = 2 cells, 8 in flight per lane) and vote
+//             whether they are all equal (skipped in the interval's first window: known empty);
+//     pass 2  equal cells evolve identically under the same accesses, so the warp applies the
+//             window's accesses once to the common cell (the read set in shared memory); each hit
+//             is a run over the whole range;
+//     pass 3  stream the final cell out (128-bit stores; skipped when no later window needs it).
+//   Ranges whose cells differ take the exact lane-parallel path: 32 lanes × 4 consecutive granules
+//   per step, each lane its own cell and private read-set record (shared records are copied before
+//   they are modified), hits compacted in the warp (__ballot_sync over hit lanes, __shfl_up_sync
+//   comparison with the left neighbour, run heads sized from the continuation mask).  Both paths
+//   feed a 32-entry per-warp run cache (one entry per lane) that extends runs across steps and
+//   ranges before appending them to global memory.
+#include "kernel.cuh"
+
+using namespace cusan;
+
+namespace {
+
+struct RunCache {
+    uint32_t e, l;       // earlier / later event id
+    uint64_t gb, ge;     // [gb, ge), empty when ge == gb
+    uint32_t rr;         // round-robin victim lane (warp-uniform)
+    unsigned long long nrace;
+};
+
+__device__ __forceinline__ bool is_spill(uint32_t v) { return (v >> 24) == 0xFFu; }
+__device__ __forceinline__ uint32_t* rec_ptr(const Ctx& k, uint32_t v) {
+    return k.heap + (uint64_t)(v & 0xffffffu) * REC_WORDS;
+}
+
+__device__ __forceinline__ void flush_entry(const RunCache& c, const Ctx& k) {
+    unsigned long long idx = atomicAdd(&k.counters[C_RUNS], 1ull);
+    if (idx < k.run_cap) {
+        cusan_race_run r;
+        r.g_begin = c.gb;
+        r.g_end = c.ge;
+        r.earlier = c.e;
+        r.later = c.l;
+        k.runs[idx] = r;
+    }
+}
+
+// Warp-collective: add run [rgb, rge) of (re, rl) to the per-warp run cache (one entry per lane):
+// extend an entry that ends where the run begins, else evict the round-robin victim.
+__device__ __forceinline__ void cache_insert(uint32_t re, uint32_t rl, uint64_t rgb, uint64_t rge, int lane,
+                                             RunCache& rc, const Ctx& k) {
+    const unsigned mm = __ballot_sync(FULL, rc.ge > rc.gb && rc.e == re && rc.l == rl && rc.ge == rgb);
+    if (mm) {
+        if (lane == __ffs(mm) - 1) rc.ge = rge;
+    } else {
+        if (lane == (int)rc.rr) {
+            if (rc.ge > rc.gb) flush_entry(rc, k);
+            rc.e = re;
+            rc.l = rl;
+            rc.gb = rgb;
+            rc.ge = rge;
+        }
+        rc.rr = (rc.rr + 1) & 31u;
+    }
+}
+
+// Warp-collective, lane-parallel granules: every lane passes its own hit flag (false for lanes
+// without a granule).  Lanes hold consecutive granules g.
+__device__ __forceinline__ void emit(bool hit, uint32_t earlier_epoch, uint32_t later_id, uint64_t g,
+                                     int lane, RunCache& rc, const Ctx& k) {
+    const unsigned m = __ballot_sync(FULL, hit);
+    if (!m) return;
+    rc.nrace += __popc(m);
+    const uint32_t e_id = (earlier_epoch & 0xffffffu) - 1u;
+    const uint32_t prev = __shfl_up_sync(FULL, e_id, 1);
+    const bool cont = hit && lane > 0 && ((m >> (lane - 1)) & 1u) && prev == e_id;
+    const unsigned cm = __ballot_sync(FULL, cont);
+    unsigned heads = m & ~cm;
+    uint32_t len = 0;
+    if (hit && !cont) {
+        const unsigned long long rest = (unsigned long long)cm >> (lane + 1);
+        len = (uint32_t)__ffsll((long long)~rest);   // 1 + number of continuing lanes
+    }
+    while (heads) {
+        const int h = __ffs(heads) - 1;
+        heads &= heads - 1;
+        const uint32_t re = __shfl_sync(FULL, e_id, h);
+        const uint64_t rgb = __shfl_sync(FULL, g, h);
+        const uint32_t rl = __shfl_sync(FULL, len, h);
+        cache_insert(re, later_id, rgb, rgb + rl, lane, rc, k);
+    }
+}
+
+// Warp-uniform: one hit covering every granule of [gb, ge).
+__device__ __forceinline__ void emit_range(bool hit, uint32_t earlier_epoch, uint32_t later_id, uint64_t gb,
+                                           uint64_t ge, int lane, RunCache& rc, const Ctx& k) {
+    if (!hit) return;
+    rc.nrace += ge - gb;
+    cache_insert((earlier_epoch & 0xffffffu) - 1u, later_id, gb, ge, lane, rc, k);
+}
+
+// ¬HB(earlier epoch e, later access of fiber f whose segment row is `row`)
+__device__ __forceinline__ bool unordered(uint32_t e, uint32_t f, const uint32_t* __restrict__ row) {
+    if (!e) return false;
+    const uint32_t g = e >> 24;
+    return g != f && (e & 0xffffffu) > __ldg(row + g);
+}
+
+// ---- TMA bulk copies (cp.async.bulk, sm_90+; SASS UBLKCP) --------------------------------------
+// Used by the streaming passes when CUSAN_TMA: pass 1 pulls the range's cells into a per-warp
+// double buffer in shared memory (mbarrier completion), pass 3 pushes a shared-memory tile filled
+// with the final cell out in bulk.  Addresses 16-B aligned, sizes multiples of 16.
+__device__ __forceinline__ uint64_t umin64(uint64_t a, uint64_t b) { return a < b ? a : b; }
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* bar) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n .reg .pred p;\n"
+        "WAIT_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra WAIT_%=;\n}\n"
+        ::"r"(smem_u32(bar)), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void bulk_load(void* dst_smem, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                 ::"r"(smem_u32(dst_smem)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void bulk_store(void* dst, const void* src_smem, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
+                 ::"l"(dst), "r"(smem_u32(src_smem)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+
+// ---- lane path: per-granule read-set records ----------------------------------------------------
+// Record header word: n (bits 0..15) | units (bits 16..23) | PRIVATE (bit 31).  Records written by
+// the range path are shared by every granule of a range (never modified in place); records the
+// lane path allocates belong to one granule's cell and are updated in place while they have room.
+constexpr uint32_t REC_PRIVATE = 0x80000000u;
+__device__ __forceinline__ uint32_t rec_n(uint32_t hdr) { return hdr & 0xffffu; }
+
+// allocate a private record with room for `cap` entries holding n; returns the tagged slot value,
+// or 0 on heap overflow (flagged; the host grows the heap and re-runs)
+__device__ __forceinline__ uint32_t rec_alloc(const Ctx& k, uint32_t n, uint32_t cap, uint32_t** out) {
+    const uint32_t units = (cap + 1 + REC_WORDS - 1) / REC_WORDS;
+    const unsigned long long at = atomicAdd(&k.counters[C_HEAP], (unsigned long long)units);
+    if (at + units > k.heap_cap) {
+        k.counters[C_HEAP_OVF] = 1ull;
+        *out = nullptr;
+        return 0;
+    }
+    *out = k.heap + at * REC_WORDS;
+    (*out)[0] = REC_PRIVATE | (units << 16) | n;
+    return SPILL_TAG | (uint32_t)at;
+}
+
+// R[f] := ep on one lane's cell
+__device__ void lane_read_update(uint2& c, uint32_t ep, uint32_t f, const Ctx& k) {
+    if (!c.y) { c.y = ep; return; }
+    uint32_t* dst;
+    if (!is_spill(c.y)) {
+        if ((c.y >> 24) == f) { c.y = ep; return; }
+        const uint32_t v = rec_alloc(k, 2, 2 * REC_WORDS - 1, &dst);   // second reader: {R, ep}
+        if (dst) { dst[1] = c.y; dst[2] = ep; }
+        c.y = v;
+        return;
+    }
+    uint32_t* src = rec_ptr(k, c.y);
+    const uint32_t hdr = src[0];
+    const uint32_t n = rec_n(hdr);
+    int pos = -1;
+    for (uint32_t j = 0; j < n; j++)
+        if ((src[1 + j] >> 24) == f) { pos = (int)j; break; }
+    if (pos >= 0 && src[1 + pos] == ep) return;
+    if ((hdr & REC_PRIVATE) && !k.cow_all) {   // this granule's own record: update in place
+        const uint32_t cap = ((hdr >> 16) & 0xffu) * REC_WORDS - 1;
+        if (pos >= 0) { src[1 + pos] = ep; return; }
+        if (n < cap) { src[1 + n] = ep; src[0] = hdr + 1; return; }
+    }
+    const uint32_t v = rec_alloc(k, pos >= 0 ? n : n + 1, 2 * (n + 1), &dst);   // copy, with room
+    if (dst) {
+        for (uint32_t j = 0; j < n; j++) dst[1 + j] = src[1 + j];
+        if (pos >= 0) dst[1 + pos] = ep; else dst[1 + n] = ep;
+    }
+    c.y = v;
+}
+
+// Where a span's LOAD reads its cells (SPAN_SRC_OLD: the previous check's shadow of a session).
+__device__ __forceinline__ const uint2* src_cells(const DSpan& sp, const Ctx& k) {
+    return ((sp.flags & SPAN_SRC_OLD) ? k.shadow_old : k.shadow) + sp.src_begin;
+}
+
+// Lane-parallel exact path for granules [x0, x0 + n) of span sp (each lane its own cells).
+__device__ void check_lanes(const DSpan& sp, uint64_t x0, uint64_t n, int lane, RunCache& rc, const Ctx& k) {
+    for (uint64_t xc = x0; xc < x0 + n; xc += CHUNK) {
+        uint2 cell[U];
+        bool valid[U];
+#pragma unroll
+        for (int c = 0; c < U; c++) {
+            const uint64_t x = xc + c * 32 + lane;
+            valid[c] = x < x0 + n;
+            cell[c] = make_uint2(0, 0);
+            if (valid[c] && (sp.flags & SPAN_LOAD)) cell[c] = __ldcs(src_cells(sp, k) + x);
+        }
+        const uint32_t qe = sp.list_off + sp.list_cnt;
+        for (uint32_t q = sp.list_off; q < qe; q++) {
+            const AccRec r = k.inc[q];
+            const uint32_t f = r.epoch >> 24;
+            const uint32_t later = (r.epoch & 0xffffffu) - 1u;
+            const uint32_t* row = k.segvc + (uint64_t)(r.segm & 0x7fffffffu) * k.F;
+            const bool wr = r.segm >> 31;
+#pragma unroll
+            for (int c = 0; c < U; c++) {
+                const uint64_t g = sp.abs_begin + xc + c * 32 + lane;
+                emit(valid[c] && unordered(cell[c].x, f, row), cell[c].x, later, g, lane, rc, k);
+                if (wr) {
+                    const bool sp_r = valid[c] && is_spill(cell[c].y);
+                    emit(valid[c] && !sp_r && unordered(cell[c].y, f, row), cell[c].y, later, g, lane, rc, k);
+                    uint32_t* rp = sp_r ? rec_ptr(k, cell[c].y) : nullptr;
+                    const uint32_t nr = sp_r ? rec_n(rp[0]) : 0u;
+                    const uint32_t nmax = __reduce_max_sync(FULL, nr);
+                    for (uint32_t j = 0; j < nmax; j++) {
+                        const uint32_t v = j < nr ? rp[1 + j] : 0u;
+                        emit(unordered(v, f, row), v, later, g, lane, rc, k);
+                    }
+                    // R := ∅.  A private record stays attached, emptied, for this granule's next
+                    // readers (a record with n = 0 is the empty read set); shared ones detach.
+                    uint32_t keep = 0;
+                    if (sp_r && (rp[0] & REC_PRIVATE) && !k.cow_all) {
+                        rp[0] &= ~0xffffu;
+                        keep = cell[c].y;
+                    }
+                    cell[c] = make_uint2(r.epoch, keep);
+                } else if (valid[c]) {
+                    lane_read_update(cell[c], r.epoch, f, k);
+                }
+            }
+        }
+        if (sp.flags & SPAN_STORE) {
+#pragma unroll
+            for (int c = 0; c < U; c++) {
+                const uint64_t x = xc + c * 32 + lane;
+                if (valid[c]) __stcs(k.shadow + sp.dense_begin + x, cell[c]);
+            }
+        }
+    }
+}
+
+__device__ __forceinline__ uint32_t find_span_by_tile(const DSpan* __restrict__ sp, uint32_t n, uint64_t t) {
+    uint32_t lo = 0, hi = n;        // last span with tile0 <= t
+    while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (sp[mid].tile0 <= t) lo = mid; else hi = mid;
+    }
+    return lo;
+}
+
+// first range whose start weight is >= pos
+__device__ __forceinline__ uint64_t tile_at_weight(const DSpan* __restrict__ sp, uint32_t n,
+                                                   uint64_t pos, uint64_t total_w, uint64_t total_t) {
+    if (pos >= total_w) return total_t;
+    uint32_t lo = 0, hi = n;
+    while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (sp[mid].weight0 <= pos) lo = mid; else hi = mid;
+    }
+    const uint64_t w = sp[lo].rweight;
+    return sp[lo].tile0 + (pos - sp[lo].weight0 + w - 1) / w;
+}
+
+__global__ void __launch_bounds__(THREADS, CUSAN_MIN_BLOCKS)
+shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t total_tiles,
+                    uint64_t total_weight, Ctx k, int force_lanes, unsigned long long* sched) {
+    __shared__ uint32_t s_list[WARPS][MAXS];
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    uint32_t* lst = s_list[warp];
+#if CUSAN_TMA
+    extern __shared__ __align__(128) unsigned char dsm[];
+    unsigned char* wsm = dsm + (size_t)warp * TMA_WARP_BYTES;
+    uint4* s_ld0 = reinterpret_cast<uint4*>(wsm);
+    uint4* s_ld1 = reinterpret_cast<uint4*>(wsm + TMA_CHUNK);
+    uint4* s_pat = reinterpret_cast<uint4*>(wsm + 2 * TMA_CHUNK);
+    uint64_t* s_bar = reinterpret_cast<uint64_t*>(wsm + 2 * TMA_CHUNK + TMA_PAT);
+    if (lane == 0) {
+        mbar_init(&s_bar[0]);
+        mbar_init(&s_bar[1]);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncwarp();
+    uint32_t ph0 = 0, ph1 = 0;              // mbarrier phases (warp-uniform)
+#endif
+    RunCache rc;
+    rc.e = rc.l = 0;
+    rc.gb = rc.ge = 0;
+    rc.rr = 0;
+    rc.nrace = 0;
+    // Range assignment: with `sched`, warps grab GRAB consecutive ranges at a time from a per-launch
+    // counter (dynamic balance); without, each warp owns one coverage-weighted contiguous slice.
+    uint64_t tend = 0;
+    uint32_t s = 0;
+    bool first = true;
+    {
+        for (uint64_t t = 0;; t++) {
+            if (t >= tend) {
+                uint64_t b, e;
+                if (sched) {
+                    unsigned long long base = 0;
+                    if (lane == 0) base = atomicAdd(sched, (unsigned long long)GRAB);
+                    b = __shfl_sync(FULL, base, 0);
+                    e = min(b + (uint64_t)GRAB, total_tiles);
+                } else {
+                    if (!first) break;
+                    const uint64_t nwarps = (uint64_t)gridDim.x * WARPS;
+                    const uint64_t wid = (uint64_t)blockIdx.x * WARPS + warp;
+                    b = tile_at_weight(spans, nspans, (uint64_t)((unsigned __int128)total_weight * wid / nwarps),
+                                       total_weight, total_tiles);
+                    e = tile_at_weight(spans, nspans, (uint64_t)((unsigned __int128)total_weight * (wid + 1) / nwarps),
+                                       total_weight, total_tiles);
+                    first = false;
+                }
+                if (b >= e) break;
+                t = b;
+                tend = e;
+                s = find_span_by_tile(spans, nspans, t);
+            }
+            while (t >= spans[s + 1].tile0) s++;   // spans[nspans] is a sentinel
+            const DSpan sp = spans[s];
+            const uint64_t x0 = (t - sp.tile0) * sp.rsize;
+            const uint64_t n = min((uint64_t)sp.rsize, sp.len - x0);   // granules of the range
+            const bool comp = sp.flags & SPAN_COMPRESSED;           // f3: one cell per interval
+            const uint64_t ncell = comp ? 1 : n;
+            uint2* cells = k.shadow + sp.dense_begin + x0;      // 256-B aligned (CELL_ALIGN)
+            const uint2* src = src_cells(sp, k) + x0;
+            const uint4* cells2 = reinterpret_cast<const uint4*>(src);
+            const uint64_t n2 = ncell >> 1;                     // cell pairs
+            // ---- pass 1: stream the range's cells in and vote that they are all equal ----------
+            uint2 c = make_uint2(0, 0);            // first window of the interval: known empty
+            bool uniform = comp || !force_lanes;
+            if (uniform && (sp.flags & SPAN_LOAD)) {
+                c = src[0];
+                bool ok = true;
+#if CUSAN_TMA
+                if ((reinterpret_cast<uintptr_t>(src) & 15u) == 0 && n2 * 16 >= TMA_MIN_BYTES) {
+                    // bulk copies through a double buffer in shared memory (TMA engine)
+                    const uint64_t bytes = n2 * 16;
+                    const uint64_t nch = (bytes + TMA_CHUNK - 1) / TMA_CHUNK;
+                    const unsigned char* gsrc = reinterpret_cast<const unsigned char*>(src);
+                    if (lane == 0) {
+                        const uint32_t sz = (uint32_t)umin64(TMA_CHUNK, bytes);
+                        mbar_arrive_expect_tx(&s_bar[0], sz);
+                        bulk_load(s_ld0, gsrc, sz, &s_bar[0]);
+                    }
+                    const uint4 cc = make_uint4(c.x, c.y, c.x, c.y);
+                    for (uint64_t q = 0; q < nch; q++) {
+                        const int st = (int)(q & 1);
+                        if (q + 1 < nch && lane == 0) {          // prefetch the next chunk
+                            const uint64_t off = (q + 1) * TMA_CHUNK;
+                            const uint32_t sz = (uint32_t)umin64(TMA_CHUNK, bytes - off);
+                            mbar_arrive_expect_tx(&s_bar[st ^ 1], sz);
+                            bulk_load(st ? s_ld0 : s_ld1, gsrc + off, sz, &s_bar[st ^ 1]);
+                        }
+                        if (st == 0) { mbar_wait(&s_bar[0], ph0); ph0 ^= 1u; }
+                        else { mbar_wait(&s_bar[1], ph1); ph1 ^= 1u; }
+                        const uint4* buf = st ? s_ld1 : s_ld0;
+                        const uint32_t nv = (uint32_t)(umin64(TMA_CHUNK, bytes - q * TMA_CHUNK) / 16);
+                        for (uint32_t j = lane; j < nv; j += 32) {
+                            const uint4 v = buf[j];
+                            ok &= ((v.x ^ cc.x) | (v.y ^ cc.y) | (v.z ^ cc.z) | (v.w ^ cc.w)) == 0u;
+                        }
+                        __syncwarp();
+                    }
+                    if ((ncell & 1) && lane == 0) {
+                        const uint2 tl = __ldcs(src + ncell - 1);
+                        ok &= tl.x == c.x && tl.y == c.y;
+                    }
+                } else
+#endif
+                if ((reinterpret_cast<uintptr_t>(src) & 15u) == 0) {
+                    for (uint64_t i = lane; i < n2; i += 32 * UL) {
+                        uint4 v[UL];
+#pragma unroll
+                        for (int u = 0; u < UL; u++)
+                            v[u] = (i + u * 32 < n2) ? __ldcs(cells2 + i + u * 32) : make_uint4(c.x, c.y, c.x, c.y);
+#pragma unroll
+                        for (int u = 0; u < UL; u++)
+                            ok &= ((v[u].x ^ c.x) | (v[u].y ^ c.y) | (v[u].z ^ c.x) | (v[u].w ^ c.y)) == 0u;
+                    }
+                    if ((ncell & 1) && lane == 0) {
+                        const uint2 tl = __ldcs(src + ncell - 1);
+                        ok &= tl.x == c.x && tl.y == c.y;
+                    }
+                } else {                           // a session's old-layout source off a 16-B boundary
+                    for (uint64_t i = lane; i < ncell; i += 32) {
+                        const uint2 v = __ldcs(src + i);
+                        ok &= v.x == c.x && v.y == c.y;
+                    }
+                }
+                uniform = __all_sync(FULL, ok);
+            }
+            if (!uniform) {
+                check_lanes(sp, x0, n, lane, rc, k);
+                continue;
+            }
+            // ---- pass 2: all cells of the range equal `c`: apply the window's accesses once -----
+            // the read set is kept in shared memory (ns entries); c.x = W
+            uint32_t ns = 0;
+            if (c.y) {
+                if (is_spill(c.y)) {
+                    const uint32_t* rp = rec_ptr(k, c.y);
+                    ns = rec_n(rp[0]);
+                    for (uint32_t j = lane; j < ns; j += 32) lst[j] = rp[1 + j];
+                } else {
+                    if (lane == 0) lst[0] = c.y;
+                    ns = 1;
+                }
+                __syncwarp();
+            }
+            const uint64_t gb = sp.abs_begin + x0, ge = gb + n;
+            const uint32_t qe = sp.list_off + sp.list_cnt;
+            AccRec nxt = k.inc[sp.list_off];
+            for (uint32_t q = sp.list_off; q < qe; q++) {
+                const AccRec r = nxt;
+                if (q + 1 < qe) nxt = k.inc[q + 1];
+                const uint32_t f = r.epoch >> 24;
+                const uint32_t later = (r.epoch & 0xffffffu) - 1u;
+                const uint32_t* row = k.segvc + (uint64_t)(r.segm & 0x7fffffffu) * k.F;
+                emit_range(unordered(c.x, f, row), c.x, later, gb, ge, lane, rc, k);
+                if (r.segm >> 31) {
+                    for (uint32_t j = 0; j < ns; j++) {
+                        const uint32_t v = lst[j];
+                        emit_range(unordered(v, f, row), v, later, gb, ge, lane, rc, k);
+                    }
+                    c.x = r.epoch;
+                    ns = 0;
+                    __syncwarp();                          // reads of lst before later writes
+                } else {
+                    int pos = -1;
+                    for (uint32_t b = 0; b < ns; b += 32) {
+                        const uint32_t j = b + lane;
+                        const unsigned m = __ballot_sync(FULL, j < ns && (lst[j] >> 24) == f);
+                        if (m) { pos = (int)(b + __ffs(m) - 1); break; }
+                    }
+                    __syncwarp();                          // (ballots do not order memory)
+                    if (lane == 0) lst[pos >= 0 ? pos : ns] = r.epoch;
+                    if (pos < 0) ns++;
+                    __syncwarp();
+                }
+            }
+            // ---- pass 3: stream the final cell out -----------------------------------------------
+            if (sp.flags & SPAN_STORE) {
+                if (ns == 0) {
+                    c.y = 0;
+                } else if (ns == 1) {
+                    c.y = lst[0];
+                } else {
+                    uint32_t* dst = nullptr;
+                    uint32_t v = 0;
+                    if (ns + 1 <= sp.rec_units * REC_WORDS) {      // the span's pre-assigned record
+                        v = SPILL_TAG | sp.rec;
+                        dst = k.heap + (uint64_t)sp.rec * REC_WORDS;
+                    } else {
+                        if (lane == 0) v = rec_alloc(k, ns, ns, &dst);
+                        v = __shfl_sync(FULL, v, 0);
+                        dst = v ? rec_ptr(k, v) : nullptr;
+                    }
+                    if (dst) {
+                        if (lane == 0) dst[0] = ns;                 // shared: no PRIVATE bit
+                        for (uint32_t j = lane; j < ns; j += 32) dst[1 + j] = lst[j];
+                    }
+                    c.y = v;
+                }
+                uint4* out2 = reinterpret_cast<uint4*>(cells);
+                const uint4 cc = make_uint4(c.x, c.y, c.x, c.y);
+#if CUSAN_TMA
+                if (n2 * 16 >= TMA_MIN_BYTES) {
+                    // a shared-memory tile of the final cell, pushed out by bulk copies
+                    if (lane == 0) bulk_wait_read();          // the previous range's stores read the tile
+                    __syncwarp();
+                    for (uint32_t j = lane; j < TMA_PAT / 16; j += 32) s_pat[j] = cc;
+                    fence_async_smem();
+                    __syncwarp();
+                    if (lane == 0) {
+                        unsigned char* gdst = reinterpret_cast<unsigned char*>(out2);
+                        const uint64_t bytes = n2 * 16;
+                        for (uint64_t off = 0; off < bytes; off += TMA_PAT)
+                            bulk_store(gdst + off, s_pat, (uint32_t)umin64(TMA_PAT, bytes - off));
+                        bulk_commit();
+                    }
+                } else
+#endif
+                for (uint64_t i = lane; i < n2; i += 32 * UL) {
+#pragma unroll
+                    for (int u = 0; u < UL; u++)
+                        if (i + u * 32 < n2) __stcs(out2 + i + u * 32, cc);
+                }
+                if ((ncell & 1) && lane == 0) __stcs(cells + ncell - 1, c);
+            }
+            __syncwarp();
+        }
+    }
+#if CUSAN_TMA
+    if (lane == 0) bulk_wait_all();                 // bulk stores done before the tile goes away
+    __syncwarp();
+#endif
+    if (rc.ge > rc.gb) flush_entry(rc, k);
+    if (lane == 0 && rc.nrace) atomicAdd(&k.counters[C_RACE], rc.nrace);
+}
+
+constexpr uint64_t COPY_CHUNK = 8192;     // cells per warp work item
+
+__global__ void __launch_bounds__(THREADS)
+copy_cells(const uint2* __restrict__ src, uint2* __restrict__ dst, const CopySeg* __restrict__ segs,
+           uint32_t nseg, uint64_t total) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t nwarps = (uint64_t)gridDim.x * WARPS;
+    const uint64_t nchunks = (total + COPY_CHUNK - 1) / COPY_CHUNK;
+    for (uint64_t ch = (uint64_t)blockIdx.x * WARPS + (threadIdx.x >> 5); ch < nchunks; ch += nwarps) {
+        const uint64_t c0 = ch * COPY_CHUNK, c1 = min(c0 + COPY_CHUNK, total);
+        uint32_t lo = 0, hi = nseg;                       // last segment with prefix <= c0
+        while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (segs[mid].prefix <= c0) lo = mid; else hi = mid;
+        }
+        for (uint64_t c = c0; c < c1; lo++) {
+            const CopySeg sg = segs[lo];
+            const uint64_t end = min(c1, sg.prefix + sg.len);
+            for (uint64_t i = c + lane; i < end; i += 32)
+                __stcs(dst + sg.dst + (i - sg.prefix), __ldcs(src + sg.src + (i - sg.prefix)));
+            c = end;
+        }
+    }
+}
+
+
+}  // namespace
+
+namespace cusan {
+
+cudaError_t launch_shadow_check(uint32_t grid, cudaStream_t stream, const DSpan* spans, uint32_t nspans,
+                                uint64_t tiles, uint64_t weight, const Ctx& k, int force_lanes,
+                                unsigned long long* sched) {
+    shadow_check_window<<<grid, THREADS, DYN_SMEM, stream>>>(spans, nspans, tiles, weight, k, force_lanes, sched);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_copy_cells(uint32_t grid, cudaStream_t stream, const uint2* src, uint2* dst,
+                              const CopySeg* segs, uint32_t nseg, uint64_t total) {
+    copy_cells<<<grid, THREADS, 0, stream>>>(src, dst, segs, nseg, total);
+    return cudaGetLastError();
+}
+
+cudaError_t shadow_check_blocks_per_sm(int* per_sm) {
+    if (DYN_SMEM) {
+        cudaError_t e = cudaFuncSetAttribute(shadow_check_window, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             (int)DYN_SMEM);
+        if (e != cudaSuccess) return e;
+    }
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, shadow_check_window, THREADS, DYN_SMEM);
+}
+
+}  // namespace cusan

@@ -1,0 +1,39 @@
+"""Small workloads for compute-sanitizer runs over the library's kernels (both kernel paths, windows,
+sessions, spill records, the interval-compressed shadow).  Asserts parity with the oracle too."""
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import numpy as np  # noqa: E402
+
+import oracle  # noqa: E402
+import paper_conf_sc_huckzsjb24_b200 as cs  # noqa: E402
+from tracegen import configs, fuzz  # noqa: E402
+
+rng = np.random.default_rng(5)
+n = 0
+for c in (1, 3, 5):
+    w = configs.make(c, "small" if c > 1 else "full")
+    ops, args = w.arrays(True)
+    tr = cs.Trace(255)
+    cs.Lowering(tr).cusan_lower_program(ops, args)
+    ref = oracle.check_events(tr.cusan_trace_read(), 255)
+    for kw in (dict(), dict(window_events=40), dict(window_events=40, flags=cs.CUSAN_CHECK_FORCE_LANES),
+               dict(window_events=40, flags=cs.CUSAN_CHECK_INTERVAL_SHADOW), dict(nshards=3, shard=1)):
+        rep = cs.check(tr, **kw)
+        if "nshards" not in kw:
+            assert rep.n_race_granules == ref["n_race_granules"], (c, kw)
+        n += 1
+for _ in range(10):
+    nf = int(rng.integers(5, 30))
+    ev = fuzz.random_primitive_trace(rng, 120, nf, n_keys=3, n_granules=600, p_access=0.8)
+    ev["mode"][(ev["kind"] == 0) & (rng.random(len(ev)) < 0.7)] = 0
+    tr = cs.Trace(nf)
+    ses = cs.Session(tr, window_events=7)
+    for a, b in ((0, 40), (40, 90), (90, 120)):
+        tr.cusan_trace_append_events(ev[a:b])
+        ses.check()
+        n += 1
+    ses.close()
+print("sanitize workloads ok:", n)
