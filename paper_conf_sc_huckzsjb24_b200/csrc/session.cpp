@@ -72,10 +72,16 @@ static int grow_heap(cusan_session* s, uint64_t need) {
     uint32_t* nh = nullptr;
     if (cudaMalloc((void**)&nh, cap * REC_WORDS * sizeof(uint32_t)) != cudaSuccess)
         return fail(CUSAN_ENOMEM, "cannot grow the read-set heap");
-    if (s->heap && s->heap_top)
-        CK(cudaMemcpyAsync(nh, s->heap, s->heap_top * REC_WORDS * sizeof(uint32_t), cudaMemcpyDeviceToDevice,
-                           s->stream));
-    CK(cudaStreamSynchronize(s->stream));
+    // zeroed, so the copy below never moves uninitialised words (unused tails of records)
+    cudaError_t e = cudaMemsetAsync(nh, 0, cap * REC_WORDS * sizeof(uint32_t), s->stream);
+    if (e == cudaSuccess && s->heap && s->heap_top)
+        e = cudaMemcpyAsync(nh, s->heap, s->heap_top * REC_WORDS * sizeof(uint32_t), cudaMemcpyDeviceToDevice,
+                            s->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s->stream);
+    if (e != cudaSuccess) {
+        cudaFree(nh);
+        return cuda_fail(e, "grow_heap");
+    }
     cudaFree(s->heap);
     s->heap = nh;
     s->heap_cap = cap;
