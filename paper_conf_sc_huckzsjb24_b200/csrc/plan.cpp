@@ -19,11 +19,28 @@
 //     a window's spans are its incidences grouped by interval.
 #include <algorithm>
 #include <bitset>
+#include <thread>
 #include <unordered_map>
 
 #include "common.h"
 
 namespace cusan {
+
+// Host threads for the planning loops (1 for small traces).
+static unsigned plan_threads(uint64_t work) {
+    if (work < (1u << 15)) return 1;
+    const unsigned hw = std::max(1u, std::thread::hardware_concurrency());
+    return std::min<unsigned>(hw, 16);
+}
+
+template <class Fn>
+static void parallel_for(unsigned T, Fn&& fn) {
+    std::vector<std::thread> th;
+    th.reserve(T ? T - 1 : 0);
+    for (unsigned t = 1; t < T; t++) th.emplace_back(fn, t);
+    fn(0u);
+    for (auto& x : th) x.join();
+}
 
 int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uint64_t first_access,
                     uint64_t rec_base) {
@@ -156,28 +173,43 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
         }
     }
     c.n_intervals = giv.size();
-    // incidences: per interval, covering accesses in trace order (CSR)
-    for (uint64_t k = 0; k < n_acc; k++)
-        for (uint32_t j = b0[k]; j < b1[k]; j++) giv[iv_of[j]].cnt++;
+    // incidences: per interval, covering accesses in trace order (CSR).  Threads take contiguous
+    // chunks of accesses; per-chunk counts give every chunk its slots, so the order is the serial one.
+    const unsigned T = plan_threads(n_acc);
+    std::vector<std::vector<uint32_t>> cnt_t(T, std::vector<uint32_t>(giv.size(), 0));
+    auto chunk = [&](unsigned t, uint64_t n) { return std::make_pair(n * t / T, n * (t + 1) / T); };
+    parallel_for(T, [&](unsigned t) {
+        auto [ka, kb] = chunk(t, n_acc);
+        for (uint64_t k = ka; k < kb; k++)
+            for (uint32_t j = b0[k]; j < b1[k]; j++) cnt_t[t][iv_of[j]]++;
+    });
     uint64_t n_inc = 0;
-    for (auto& g : giv) {
-        if (n_inc + g.cnt > 0xffffffffull) return fail(CUSAN_ERANGE, "too many interval incidences");
+    for (size_t i = 0; i < giv.size(); i++) {
+        GIv& g = giv[i];
         g.off = (uint32_t)n_inc;
-        n_inc += g.cnt;
+        uint64_t at = n_inc;
+        for (unsigned t = 0; t < T; t++) {           // counts -> each chunk's first slot
+            const uint32_t n = cnt_t[t][i];
+            cnt_t[t][i] = (uint32_t)at;
+            at += n;
+        }
+        if (at > 0xffffffffull) return fail(CUSAN_ERANGE, "too many interval incidences");
+        g.cnt = (uint32_t)(at - n_inc);
+        n_inc = at;
     }
     c.n_incidences = n_inc;
     hp.inc.resize(n_inc);
     hp.inc_acc.resize(n_inc);
-    {
-        std::vector<uint32_t> fill(giv.size());
-        for (size_t i = 0; i < giv.size(); i++) fill[i] = giv[i].off;
-        for (uint64_t k = 0; k < n_acc; k++)
+    parallel_for(T, [&](unsigned t) {
+        auto [ka, kb] = chunk(t, n_acc);
+        std::vector<uint32_t>& slot = cnt_t[t];
+        for (uint64_t k = ka; k < kb; k++)
             for (uint32_t j = b0[k]; j < b1[k]; j++) {
-                uint32_t q = fill[iv_of[j]]++;
+                const uint32_t q = slot[iv_of[j]]++;
                 hp.inc[q] = hp.acc_rec[k];
                 hp.inc_acc[q] = (uint32_t)k;
             }
-    }
+    });
 
     // ---------------------------------------------------------------- a2: shard clip ------------
     const uint64_t total_dense = giv.empty() ? 0 : giv.back().dense_begin + giv.back().len;
@@ -258,58 +290,73 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
     const uint64_t W = o.window_events > 0 ? (uint64_t)o.window_events : std::max<uint64_t>(n_new, 1);
     hp.window_accesses = W;
     const uint64_t nwin = n_new ? (n_new + W - 1) / W : 0;
-    std::vector<std::vector<Span>> per(nwin);
-    hp.rec_units = 0;
-    hp.spill_spans = 0;
-    for (const Interval& v : hp.iv) {
-        std::bitset<CUSAN_MAX_FIBERS + 1> readers;
-        uint32_t q = v.list_off, qe = v.list_off + v.list_cnt;
-        for (; q < qe && hp.inc_acc[q] < first; q++) {
-            const AccRec& r = hp.inc[q];
-            if (r.segm >> 31) readers.reset();
-            else readers.set(r.epoch >> 24);
-        }
-        const uint32_t first_new = q;
-        while (q < qe) {
-            uint64_t w = (hp.inc_acc[q] - first) / W;
-            uint32_t q2 = q;
-            while (q2 < qe && (hp.inc_acc[q2] - first) / W == w) {
-                const AccRec& r = hp.inc[q2];
+    // Threads take contiguous chunks of intervals and emit (window, span) in interval order; a
+    // stable counting sort by window then gives the window-major order of the serial loop.
+    const unsigned TS = plan_threads(hp.iv.size() * 8);
+    std::vector<std::vector<std::pair<uint64_t, Span>>> part(TS);
+    parallel_for(TS, [&](unsigned t) {
+        const size_t ia = hp.iv.size() * t / TS, ib = hp.iv.size() * (t + 1) / TS;
+        for (size_t i = ia; i < ib; i++) {
+            const Interval& v = hp.iv[i];
+            std::bitset<CUSAN_MAX_FIBERS + 1> readers;
+            uint32_t q = v.list_off, qe = v.list_off + v.list_cnt;
+            for (; q < qe && hp.inc_acc[q] < first; q++) {
+                const AccRec& r = hp.inc[q];
                 if (r.segm >> 31) readers.reset();
                 else readers.set(r.epoch >> 24);
-                q2++;
             }
-            Span s{};
-            s.abs_begin = v.abs_begin;
-            s.dense_begin = v.dense_begin;
-            s.len = v.len;
-            s.list_off = q;
-            s.list_cnt = q2 - q;
-            s.src_begin = v.dense_begin;
-            s.flags = (q > v.list_off ? SPAN_LOAD : 0u) | ((q2 < qe || o.persist_shadow) ? SPAN_STORE : 0u) |
-                      (q == first_new ? SPAN_FIRST_IN_CALL : 0u) | (compressed ? SPAN_COMPRESSED : 0u);
-            const uint64_t nr = readers.count();
-            if ((s.flags & SPAN_STORE) && nr >= 2) {
-                s.rec = (uint32_t)(rec_base + hp.rec_units);
-                s.rec_units = (uint32_t)((nr + 1 + REC_WORDS - 1) / REC_WORDS);
-                hp.rec_units += s.rec_units;
-                hp.spill_spans++;
+            const uint32_t first_new = q;
+            while (q < qe) {
+                uint64_t w = (hp.inc_acc[q] - first) / W;
+                uint32_t q2 = q;
+                while (q2 < qe && (hp.inc_acc[q2] - first) / W == w) {
+                    const AccRec& r = hp.inc[q2];
+                    if (r.segm >> 31) readers.reset();
+                    else readers.set(r.epoch >> 24);
+                    q2++;
+                }
+                Span s{};
+                s.abs_begin = v.abs_begin;
+                s.dense_begin = v.dense_begin;
+                s.len = v.len;
+                s.list_off = q;
+                s.list_cnt = q2 - q;
+                s.src_begin = v.dense_begin;
+                s.flags = (q > v.list_off ? SPAN_LOAD : 0u) | ((q2 < qe || o.persist_shadow) ? SPAN_STORE : 0u) |
+                          (q == first_new ? SPAN_FIRST_IN_CALL : 0u) | (compressed ? SPAN_COMPRESSED : 0u);
+                const uint64_t nr = readers.count();
+                if ((s.flags & SPAN_STORE) && nr >= 2)         // record index assigned below
+                    s.rec_units = (uint32_t)((nr + 1 + REC_WORDS - 1) / REC_WORDS);
+                part[t].emplace_back(w, s);
+                q = q2;
             }
-            per[w].push_back(s);
-            q = q2;
         }
+    });
+    std::vector<uint64_t> wstart(nwin + 1, 0);
+    for (const auto& pt : part)
+        for (const auto& ws : pt) wstart[ws.first + 1]++;
+    for (uint64_t w = 0; w < nwin; w++) wstart[w + 1] += wstart[w];
+    hp.spans.assign(wstart[nwin], Span{});
+    {
+        std::vector<uint64_t> at(wstart.begin(), wstart.end() - 1);
+        for (const auto& pt : part)
+            for (const auto& ws : pt) hp.spans[at[ws.first]++] = ws.second;
     }
+    hp.rec_units = 0;
+    hp.spill_spans = 0;
+    for (Span& s : hp.spans)
+        if (s.rec_units) {
+            s.rec = (uint32_t)(rec_base + hp.rec_units);
+            hp.rec_units += s.rec_units;
+            hp.spill_spans++;
+        }
     if (rec_base + hp.rec_units >= (1u << 24) - 1)
         return fail(CUSAN_ERANGE, "too many read-set records for the 24-bit record index");
     c.spill_spans = hp.spill_spans;
     c.spill_heap_bytes = hp.rec_units * REC_WORDS * 4;
-    hp.spans.clear();
     hp.win_span_off.assign(1, 0);
-    for (uint64_t w = 0; w < nwin; w++) {
-        if (per[w].empty()) continue;              // windows with nothing in this shard
-        hp.spans.insert(hp.spans.end(), per[w].begin(), per[w].end());
-        hp.win_span_off.push_back(hp.spans.size());
-    }
+    for (uint64_t w = 0; w < nwin; w++)
+        if (wstart[w + 1] > wstart[w]) hp.win_span_off.push_back(wstart[w + 1]);   // skip empty windows
     c.n_windows = hp.win_span_off.size() - 1;
     c.n_spans = hp.spans.size();
     return CUSAN_OK;
