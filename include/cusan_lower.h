@@ -86,6 +86,12 @@ int cusan_on_thread_create(cusan_lowering* l, uint64_t child);
 int cusan_on_thread_join(cusan_lowering* l, uint64_t child);
 int cusan_lowering_set_default_stream(cusan_lowering* l, int per_thread);
 
+/* What a fiber stands for, for race reports: kind = CUSAN_FIBER_*, handle = the thread id, stream
+ * handle or (latest) MPI request of the fiber.  CUSAN_EINVAL for a fiber the lowering never made. */
+enum cusan_fiber_kind { CUSAN_FIBER_HOST = 0, CUSAN_FIBER_LEGACY_STREAM = 1, CUSAN_FIBER_STREAM = 2,
+                        CUSAN_FIBER_PER_THREAD_STREAM = 3, CUSAN_FIBER_MPI_REQUEST = 4 };
+int cusan_lowering_fiber_info(const cusan_lowering* l, uint32_t fiber, int* kind, uint64_t* handle);
+
 /* ---- bulk form: a recorded API program (same layout as tracegen.OP_DTYPE / ARG_DTYPE) -------- */
 enum cusan_api_op {
     CUSAN_OP_MALLOC = 1, CUSAN_OP_FREE = 2, CUSAN_OP_STREAM_CREATE = 3, CUSAN_OP_KERNEL = 4,

@@ -95,6 +95,12 @@ class Lowering:
             lib.cusan_lowering_destroy(self.h)
             self.h = None
 
+    def cusan_lowering_fiber_info(self, fiber: int) -> tuple[int, int]:
+        """(cusan_fiber_kind, handle) of a fiber: thread id, stream handle or MPI request."""
+        kind, handle = C.c_int(), C.c_uint64()
+        _ck(lib.cusan_lowering_fiber_info(self.h, fiber, C.byref(kind), C.byref(handle)))
+        return kind.value, handle.value
+
     def cusan_lowering_set_default_stream(self, per_thread: bool):
         _ck(lib.cusan_lowering_set_default_stream(self.h, int(per_thread)))
 

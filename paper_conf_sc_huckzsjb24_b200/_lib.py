@@ -118,6 +118,7 @@ PROTOS = {
     "cusan_on_thread_create": [P, u64],
     "cusan_on_thread_join": [P, u64],
     "cusan_lowering_set_default_stream": [P, i32],
+    "cusan_lowering_fiber_info": [P, u32, pi32, pu64],
     "cusan_lower_program": [P, P, u64, P, u64, pu32],
 }
 VOID = {"cusan_check_opts_init"}

@@ -46,6 +46,12 @@ struct cusan_lowering {
     std::unordered_map<uint64_t, uint32_t> ptds;           // host thread -> per-thread default stream
     uint64_t thread = 0;                                   // calling host thread
     bool per_thread_mode = false;
+    std::vector<std::pair<int, uint64_t>> fiber_info;      // by fiber: (cusan_fiber_kind, handle)
+
+    void note(uint32_t f, int kind, uint64_t handle) {
+        if (fiber_info.size() <= f) fiber_info.resize(f + 1, {-1, 0});
+        fiber_info[f] = {kind, handle};
+    }
 
     uint32_t H() const { return thread_fiber.at(thread); }
 
@@ -92,7 +98,10 @@ struct cusan_lowering {
             return CUSAN_OK;
         }
         int st = add_stream(f, true);
-        if (!st) ptds[thread] = *f;
+        if (!st) {
+            ptds[thread] = *f;
+            note(*f, CUSAN_FIBER_PER_THREAD_STREAM, thread);
+        }
         return st;
     }
     int fiber_of(uint64_t stream, uint32_t* f) {
@@ -118,7 +127,10 @@ struct cusan_lowering {
             return CUSAN_OK;
         }
         int st = new_fiber(f);
-        if (!st) thread_fiber[t] = *f;
+        if (!st) {
+            thread_fiber[t] = *f;
+            note(*f, CUSAN_FIBER_HOST, t);
+        }
         return st;
     }
     int prologue(uint32_t f) {
@@ -164,6 +176,8 @@ int cusan_lowering_create(cusan_trace* trace, cusan_lowering** out) {
     l->streams.push_back(S0);
     l->is_blocking.assign(2, 0);
     l->thread_fiber[0] = 0;
+    l->note(0, CUSAN_FIBER_HOST, 0);
+    l->note(S0, CUSAN_FIBER_LEGACY_STREAM, 0);
     *out = l;
     return CUSAN_OK;
 }
@@ -199,6 +213,16 @@ int cusan_on_stream_create(cusan_lowering* l, uint64_t stream, int nonblocking) 
     int st = l->add_stream(&f, !nonblocking);   // track the non-blocking attribute
     if (st) return st;
     l->stream_fiber[stream] = f;
+    l->note(f, CUSAN_FIBER_STREAM, stream);
+    return CUSAN_OK;
+}
+
+int cusan_lowering_fiber_info(const cusan_lowering* l, uint32_t fiber, int* kind, uint64_t* handle) {
+    if (!l || !kind || !handle) return fail(CUSAN_EINVAL, "null argument");
+    if (fiber >= l->fiber_info.size() || l->fiber_info[fiber].first < 0)
+        return fail(CUSAN_EINVAL, "unknown fiber");
+    *kind = l->fiber_info[fiber].first;
+    *handle = l->fiber_info[fiber].second;
     return CUSAN_OK;
 }
 
@@ -304,6 +328,7 @@ static int mpi_nonblocking(cusan_lowering* l, uint64_t buf, uint64_t n, uint64_t
         if (st) return st;
     }
     l->req_fiber[req] = m;
+    l->note(m, CUSAN_FIBER_MPI_REQUEST, req);
     int st = l->sync(CUSAN_FORK, m, l->H());   // fiber per non-blocking request
     if (st || (st = l->access(m, mode, buf, n))) return st;
     return l->sync(CUSAN_RELEASE, m, K_req(req));

@@ -82,6 +82,45 @@ def test_check_without_gpu_fails_loudly():
     assert e.value.status == -4
 
 
+def test_fiber_info_and_text_report():
+    """Fibers are named by what they stand for; the text report names the racing calls."""
+    from paper_conf_sc_huckzsjb24_b200.report import format_report
+    import oracle
+    w = configs.make(1)
+    ops, args = w.arrays(True)
+    tr = cs.Trace(255)
+    low = cs.Lowering(tr)
+    first = low.cusan_lower_program(ops, args)
+    assert low.cusan_lowering_fiber_info(0) == (0, 0)        # host thread 0
+    assert low.cusan_lowering_fiber_info(1) == (1, 0)        # legacy default stream
+    assert low.cusan_lowering_fiber_info(2)[0] == 2           # the user stream
+    assert low.cusan_lowering_fiber_info(3) == (4, 1)        # MPI request 1
+    with pytest.raises(cs.CusanError):
+        low.cusan_lowering_fiber_info(9)
+    ref = oracle.check_events(tr.cusan_trace_read(), 255)
+
+    class Rep:
+        n_race_granules, n_runs, truncated, runs = ref["n_race_granules"], ref["n_runs"], False, ref["runs"]
+    text = format_report(Rep, tr, lowering=low, calls=ops, first_event=first)
+    assert "4096 bytes" in text and "MPI_Isend" in text and "kernel launch" in text
+
+
+def test_event_index_limit():
+    """Maximum trace length: event id + 1 must fit the 24-bit epoch field."""
+    n = (1 << 24) - 2
+    ev = np.zeros(n, EVENT_DTYPE)
+    ev["kind"] = 1                                       # RELEASE on key 0 by fiber 0
+    t = cs.Trace(2)
+    t.cusan_trace_append_events(ev)
+    assert len(t) == n
+    with pytest.raises(cs.CusanError) as e:
+        t.cusan_trace_append_sync(cs.CUSAN_RELEASE, 0, 1)
+    assert e.value.status == -2
+    d = cs.describe(t)                                   # the planner takes the longest trace
+    assert d["n_events"] == n and d["n_release"] == n
+    del ev, t
+
+
 def test_trace_roundtrip_and_event_ids():
     t = cs.Trace(8)
     assert t.cusan_trace_append_access(1, 1, 0x100, 24) == 0
