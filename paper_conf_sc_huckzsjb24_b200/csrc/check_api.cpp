@@ -81,7 +81,6 @@ void cusan::build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& ou
             d.flags = s.flags;
             d.rec = s.rec;
             d.rec_units = s.rec_units;
-            d.src_begin = s.src_begin;
             // warp range: long enough that replaying the window's accesses once per range stays
             // small next to streaming its cells, capped for balance; spans that move no cells
             // are one range each
@@ -219,8 +218,6 @@ static int launch_all(cusan_plan* p) {
     k.segvc = p->d_segvc;
     k.F = p->hp.F;
     k.shadow = p->d_shadow;
-    k.shadow_old = nullptr;
-    k.cow_all = 0;
     k.heap = p->d_heap;
     k.heap_cap = p->heap_cap;
     k.runs = p->d_runs;

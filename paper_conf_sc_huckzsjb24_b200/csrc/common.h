@@ -54,13 +54,11 @@ struct Span {
     uint32_t flags;       // SPAN_LOAD: cells hold state from an earlier window; SPAN_STORE: write back
     uint32_t rec;         // pre-assigned read-set record (REC_WORDS-word units) for the final state
     uint32_t rec_units;   // its size; 0 = the final state needs no record (≤ 1 reader)
-    uint64_t src_begin;   // shadow index LOAD reads from (= dense_begin except in sessions)
 };
 // SPAN_LOAD: cells hold state from an earlier window; SPAN_STORE: a later window needs the result;
 // SPAN_FIRST_IN_CALL: the interval's first span of this check (incremental sessions);
-// SPAN_SRC_OLD: LOAD from the previous check's shadow at src_begin (sessions).
 // SPAN_COMPRESSED: the interval keeps one shadow cell for all its granules (f3).
-enum : uint32_t { SPAN_LOAD = 1u, SPAN_STORE = 2u, SPAN_SRC_OLD = 4u, SPAN_FIRST_IN_CALL = 8u,
+enum : uint32_t { SPAN_LOAD = 1u, SPAN_STORE = 2u, SPAN_FIRST_IN_CALL = 8u,
                   SPAN_COMPRESSED = 16u };
 
 struct HostPlan {

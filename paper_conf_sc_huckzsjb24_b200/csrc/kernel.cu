@@ -189,7 +189,7 @@ __device__ void lane_read_update(uint2& c, uint32_t ep, uint32_t f, const Ctx& k
     for (uint32_t j = 0; j < n; j++)
         if ((src[1 + j] >> 24) == f) { pos = (int)j; break; }
     if (pos >= 0 && src[1 + pos] == ep) return;
-    if ((hdr & REC_PRIVATE) && !k.cow_all) {   // this granule's own record: update in place
+    if (hdr & REC_PRIVATE) {   // this granule's own record: update in place
         const uint32_t cap = ((hdr >> 16) & 0xffu) * REC_WORDS - 1;
         if (pos >= 0) { src[1 + pos] = ep; return; }
         if (n < cap) { src[1 + n] = ep; src[0] = hdr + 1; return; }
@@ -202,9 +202,9 @@ __device__ void lane_read_update(uint2& c, uint32_t ep, uint32_t f, const Ctx& k
     c.y = v;
 }
 
-// Where a span's LOAD reads its cells (SPAN_SRC_OLD: the previous check's shadow of a session).
+// Where a span's cells live in the shadow.
 __device__ __forceinline__ const uint2* src_cells(const DSpan& sp, const Ctx& k) {
-    return ((sp.flags & SPAN_SRC_OLD) ? k.shadow_old : k.shadow) + sp.src_begin;
+    return k.shadow + sp.dense_begin;
 }
 
 // Lane-parallel exact path for granules [x0, x0 + n) of span sp (each lane its own cells).
@@ -243,7 +243,7 @@ __device__ void check_lanes(const DSpan& sp, uint64_t x0, uint64_t n, int lane, 
                     // R := ∅.  A private record stays attached, emptied, for this granule's next
                     // readers (a record with n = 0 is the empty read set); shared ones detach.
                     uint32_t keep = 0;
-                    if (sp_r && (rp[0] & REC_PRIVATE) && !k.cow_all) {
+                    if (sp_r && (rp[0] & REC_PRIVATE)) {
                         rp[0] &= ~0xffffu;
                         keep = cell[c].y;
                     }
@@ -347,10 +347,13 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
             const uint64_t n = min((uint64_t)sp.rsize, sp.len - x0);   // granules of the range
             const bool comp = sp.flags & SPAN_COMPRESSED;           // f3: one cell per interval
             const uint64_t ncell = comp ? 1 : n;
-            uint2* cells = k.shadow + sp.dense_begin + x0;      // 256-B aligned (CELL_ALIGN)
+            uint2* cells = k.shadow + sp.dense_begin + x0;      // 8-B aligned (256-B for plan layouts)
             const uint2* src = src_cells(sp, k) + x0;
-            const uint4* cells2 = reinterpret_cast<const uint4*>(src);
-            const uint64_t n2 = ncell >> 1;                     // cell pairs
+            // 128-bit / bulk streaming needs 16-B alignment: a cell off it is handled on its own
+            const uint64_t shead = (reinterpret_cast<uintptr_t>(src) & 15u) ? 1 : 0;
+            const uint4* cells2 = reinterpret_cast<const uint4*>(src + shead);
+            const uint64_t n2 = ncell > shead ? (ncell - shead) >> 1 : 0;   // aligned cell pairs
+            const bool stail = ncell > shead && ((ncell - shead) & 1);
             // ---- pass 1: stream the range's cells in and vote that they are all equal ----------
             uint2 c = make_uint2(0, 0);            // first window of the interval: known empty
             bool uniform = comp || !force_lanes;
@@ -358,11 +361,11 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                 c = src[0];
                 bool ok = true;
 #if CUSAN_TMA
-                if ((reinterpret_cast<uintptr_t>(src) & 15u) == 0 && n2 * 16 >= TMA_MIN_BYTES) {
+                if (n2 * 16 >= TMA_MIN_BYTES) {
                     // bulk copies through a double buffer in shared memory (TMA engine)
                     const uint64_t bytes = n2 * 16;
                     const uint64_t nch = (bytes + TMA_CHUNK - 1) / TMA_CHUNK;
-                    const unsigned char* gsrc = reinterpret_cast<const unsigned char*>(src);
+                    const unsigned char* gsrc = reinterpret_cast<const unsigned char*>(cells2);
                     if (lane == 0) {
                         const uint32_t sz = (uint32_t)umin64(TMA_CHUNK, bytes);
                         mbar_arrive_expect_tx(&s_bar[0], sz);
@@ -387,13 +390,9 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                         }
                         __syncwarp();
                     }
-                    if ((ncell & 1) && lane == 0) {
-                        const uint2 tl = __ldcs(src + ncell - 1);
-                        ok &= tl.x == c.x && tl.y == c.y;
-                    }
                 } else
 #endif
-                if ((reinterpret_cast<uintptr_t>(src) & 15u) == 0) {
+                {
                     for (uint64_t i = lane; i < n2; i += 32 * UL) {
                         uint4 v[UL];
 #pragma unroll
@@ -403,15 +402,10 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                         for (int u = 0; u < UL; u++)
                             ok &= ((v[u].x ^ c.x) | (v[u].y ^ c.y) | (v[u].z ^ c.x) | (v[u].w ^ c.y)) == 0u;
                     }
-                    if ((ncell & 1) && lane == 0) {
-                        const uint2 tl = __ldcs(src + ncell - 1);
-                        ok &= tl.x == c.x && tl.y == c.y;
-                    }
-                } else {                           // a session's old-layout source off a 16-B boundary
-                    for (uint64_t i = lane; i < ncell; i += 32) {
-                        const uint2 v = __ldcs(src + i);
-                        ok &= v.x == c.x && v.y == c.y;
-                    }
+                }
+                if (stail && lane == 0) {                  // (the head cell is src[0] = c itself)
+                    const uint2 tl = __ldcs(src + ncell - 1);
+                    ok &= tl.x == c.x && tl.y == c.y;
                 }
                 uniform = __all_sync(FULL, ok);
             }
@@ -487,10 +481,14 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                     }
                     c.y = v;
                 }
-                uint4* out2 = reinterpret_cast<uint4*>(cells);
+                const uint64_t dhead = (reinterpret_cast<uintptr_t>(cells) & 15u) ? 1 : 0;
+                uint4* out2 = reinterpret_cast<uint4*>(cells + dhead);
+                const uint64_t m2 = ncell > dhead ? (ncell - dhead) >> 1 : 0;
+                const bool dtail = ncell > dhead && ((ncell - dhead) & 1);
                 const uint4 cc = make_uint4(c.x, c.y, c.x, c.y);
+                if (dhead && lane == 0) __stcs(cells, c);
 #if CUSAN_TMA
-                if (n2 * 16 >= TMA_MIN_BYTES) {
+                if (m2 * 16 >= TMA_MIN_BYTES) {
                     // a shared-memory tile of the final cell, pushed out by bulk copies
                     if (lane == 0) bulk_wait_read();          // the previous range's stores read the tile
                     __syncwarp();
@@ -499,19 +497,19 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                     __syncwarp();
                     if (lane == 0) {
                         unsigned char* gdst = reinterpret_cast<unsigned char*>(out2);
-                        const uint64_t bytes = n2 * 16;
+                        const uint64_t bytes = m2 * 16;
                         for (uint64_t off = 0; off < bytes; off += TMA_PAT)
                             bulk_store(gdst + off, s_pat, (uint32_t)umin64(TMA_PAT, bytes - off));
                         bulk_commit();
                     }
                 } else
 #endif
-                for (uint64_t i = lane; i < n2; i += 32 * UL) {
+                for (uint64_t i = lane; i < m2; i += 32 * UL) {
 #pragma unroll
                     for (int u = 0; u < UL; u++)
-                        if (i + u * 32 < n2) __stcs(out2 + i + u * 32, cc);
+                        if (i + u * 32 < m2) __stcs(out2 + i + u * 32, cc);
                 }
-                if ((ncell & 1) && lane == 0) __stcs(cells + ncell - 1, c);
+                if (dtail && lane == 0) __stcs(cells + ncell - 1, c);
             }
             __syncwarp();
         }
@@ -526,9 +524,12 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
 
 constexpr uint64_t COPY_CHUNK = 8192;     // cells per warp work item
 
+// Copy cells between layouts.  With `heap` set (a session splitting a compressed interval in place,
+// so source and copy both stay live) a copied private read-set record becomes shared: neither cell
+// may then update it in place (lane_read_update copies it on its next change).
 __global__ void __launch_bounds__(THREADS)
-copy_cells(const uint2* __restrict__ src, uint2* __restrict__ dst, const CopySeg* __restrict__ segs,
-           uint32_t nseg, uint64_t total) {
+copy_cells(const uint2* src, uint2* dst, const CopySeg* __restrict__ segs, uint32_t nseg, uint64_t total,
+           uint32_t* heap) {
     const int lane = threadIdx.x & 31;
     const uint64_t nwarps = (uint64_t)gridDim.x * WARPS;
     const uint64_t nchunks = (total + COPY_CHUNK - 1) / COPY_CHUNK;
@@ -542,8 +543,11 @@ copy_cells(const uint2* __restrict__ src, uint2* __restrict__ dst, const CopySeg
         for (uint64_t c = c0; c < c1; lo++) {
             const CopySeg sg = segs[lo];
             const uint64_t end = min(c1, sg.prefix + sg.len);
-            for (uint64_t i = c + lane; i < end; i += 32)
-                __stcs(dst + sg.dst + (i - sg.prefix), __ldcs(src + sg.src + (i - sg.prefix)));
+            for (uint64_t i = c + lane; i < end; i += 32) {
+                const uint2 v = __ldcs(src + sg.src + (i - sg.prefix));
+                if (heap && is_spill(v.y)) atomicAnd(heap + (uint64_t)(v.y & 0xffffffu) * REC_WORDS, ~REC_PRIVATE);
+                __stcs(dst + sg.dst + (i - sg.prefix), v);
+            }
             c = end;
         }
     }
@@ -562,8 +566,8 @@ cudaError_t launch_shadow_check(uint32_t grid, cudaStream_t stream, const DSpan*
 }
 
 cudaError_t launch_copy_cells(uint32_t grid, cudaStream_t stream, const uint2* src, uint2* dst,
-                              const CopySeg* segs, uint32_t nseg, uint64_t total) {
-    copy_cells<<<grid, THREADS, 0, stream>>>(src, dst, segs, nseg, total);
+                              const CopySeg* segs, uint32_t nseg, uint64_t total, uint32_t* heap) {
+    copy_cells<<<grid, THREADS, 0, stream>>>(src, dst, segs, nseg, total, heap);
     return cudaGetLastError();
 }
 

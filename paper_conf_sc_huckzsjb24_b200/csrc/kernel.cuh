@@ -68,27 +68,23 @@ struct DSpan {
     uint64_t tile0, weight0;     // prefix of ranges / of range weights over the window's spans
     uint32_t rsize, rweight;     // granules per range (multiple of CHUNK), weight of one range
     uint32_t list_off, list_cnt, flags, rec, rec_units, pad;
-    uint64_t src_begin;          // where LOAD reads the cells: `shadow` (or `shadow_old` with SPAN_SRC_OLD)
 };
-static_assert(sizeof(DSpan) == 80, "DSpan layout");
+static_assert(sizeof(DSpan) == 72, "DSpan layout");
 
 struct Ctx {                     // kernel-wide pointers
     const AccRec* __restrict__ inc;
     const uint32_t* __restrict__ segvc;
     uint32_t F;
     uint2* __restrict__ shadow;
-    const uint2* __restrict__ shadow_old;   // previous layout (incremental sessions), else null
     uint32_t* __restrict__ heap;
     unsigned long long heap_cap;  // record units
     cusan_race_run* __restrict__ runs;
     unsigned long long* __restrict__ counters;
     unsigned long long run_cap;
-    int cow_all;                  // sessions: never modify a record in place (the previous check's
-                                  // shadow must stay a consistent snapshot so a check can re-run)
 };
 
 
-// Copy of untouched intervals' cells from a session's previous layout to the new one.
+// Cells copied inside a session's shadow (pieces of a split compressed interval, f3).
 struct CopySeg {
     uint64_t prefix, src, dst, len;       // cells [prefix, prefix + len) of the copy space
 };
@@ -120,7 +116,7 @@ cudaError_t launch_shadow_check(uint32_t grid, cudaStream_t stream, const DSpan*
                                 unsigned long long* sched);
 // sessions: move untouched intervals' cells to the new layout
 cudaError_t launch_copy_cells(uint32_t grid, cudaStream_t stream, const uint2* src, uint2* dst,
-                              const CopySeg* segs, uint32_t nseg, uint64_t total);
+                              const CopySeg* segs, uint32_t nseg, uint64_t total, uint32_t* heap);
 // resident blocks of K1 per SM (sets K1's dynamic shared memory limit first)
 cudaError_t shadow_check_blocks_per_sm(int* per_sm);
 

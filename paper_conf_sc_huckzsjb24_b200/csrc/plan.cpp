@@ -321,7 +321,6 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
                 s.len = v.len;
                 s.list_off = q;
                 s.list_cnt = q2 - q;
-                s.src_begin = v.dense_begin;
                 s.flags = (q > v.list_off ? SPAN_LOAD : 0u) | ((q2 < qe || o.persist_shadow) ? SPAN_STORE : 0u) |
                           (q == first_new ? SPAN_FIRST_IN_CALL : 0u) | (compressed ? SPAN_COMPRESSED : 0u);
                 const uint64_t nr = readers.count();

@@ -1,9 +1,13 @@
 // Incremental (online) sessions — SURVEY.md §8(f) f1.
 #include <algorithm>
+#include <bitset>
 #include <chrono>
 #include <cstring>
 #include <new>
 #include <string>
+#include <unordered_map>
+
+#include <cuda.h>
 
 #include "kernel.cuh"
 
@@ -14,40 +18,186 @@ using namespace cusan;
 // (PAPER.md:606-612); a session keeps the shadow on the device between calls and each call checks
 // only the accesses appended since the previous one.
 //
-// New accesses can split elementary intervals or add new ones, so every call re-plans the layout
-// (a1, a2 over the whole trace; host cost only).  The previous call's shadow stays untouched as
-// the source: intervals the call does not touch are copied to the new layout (copy_cells), the
-// first span of a touched interval loads its cells from the old layout (SPAN_SRC_OLD), and read-set
-// records are never modified in place (cow_all).  A call therefore only writes the new buffer and
-// can be re-run as a whole after a run-buffer or heap overflow.  The buffers then swap.
+// The host plan is incremental too: the vector clocks, sync clocks and segment rows (a1) carry over
+// between calls, and so does the layout (a2) — the elementary intervals seen so far, each with the
+// set of fibers that read it since its last write.  A call processes only the new events: its
+// accesses' endpoints split old intervals (a split piece inherits the state) or open new ones, the
+// new incidences are grouped into windows and spans, and only new segment rows are uploaded.  Host
+// cost per call is O(new events × fibers + intervals).
+//
+// On the device the layout is stable: a piece of a split interval keeps its cells where they are
+// (the pieces of an interval are consecutive sub-ranges of it), memory touched for the first time
+// gets new cells appended to the shadow, and the check updates the cells in place.  A call costs
+// only the cells its accesses touch (the shadow grows in place, see Vmm below).  With the
+// interval-compressed shadow (f3) an interval has one cell, so a split piece other than the first
+// gets a new cell copied from it (copy_cells).  In-place updates cannot be re-run: if the run buffer
+// overflows, the call's run list is marked truncated (race-granule counts stay exact) and the buffer
+// grows for later calls; a read-set heap overflow (only possible on the lane-parallel path) fails
+// the session.
 // ================================================================================================
+namespace {
+
+constexpr uint32_t NO_SEG = 0xffffffffu;
+
+// ---- growable shadow in a reserved virtual range (CUDA virtual memory management) --------------
+// The session reserves a virtual range as large as the device's memory once and maps physical
+// chunks at its end as the shadow grows, so growth neither copies the cells nor needs room for two
+// copies (a 70 GB shadow could not be re-allocated next to itself in 180 GB).  Driver entry points
+// come from the runtime (no link against libcuda); if they are unavailable the shadow falls back to
+// re-allocation with a copy.
+struct Vmm {
+    decltype(&cuMemAddressReserve) reserve = nullptr;
+    decltype(&cuMemAddressFree) addr_free = nullptr;
+    decltype(&cuMemCreate) create = nullptr;
+    decltype(&cuMemMap) map = nullptr;
+    decltype(&cuMemSetAccess) set_access = nullptr;
+    decltype(&cuMemUnmap) unmap = nullptr;
+    decltype(&cuMemRelease) release = nullptr;
+    decltype(&cuMemGetAllocationGranularity) granularity = nullptr;
+    bool ok = false;
+};
+
+const Vmm& vmm() {
+    static const Vmm v = [] {
+        Vmm r;
+        auto get = [](const char* name, void** fn) {
+            cudaDriverEntryPointQueryResult q;
+            return cudaGetDriverEntryPoint(name, fn, cudaEnableDefault, &q) == cudaSuccess &&
+                   q == cudaDriverEntryPointSuccess && *fn;
+        };
+        r.ok = get("cuMemAddressReserve", (void**)&r.reserve) && get("cuMemAddressFree", (void**)&r.addr_free) &&
+               get("cuMemCreate", (void**)&r.create) && get("cuMemMap", (void**)&r.map) &&
+               get("cuMemSetAccess", (void**)&r.set_access) && get("cuMemUnmap", (void**)&r.unmap) &&
+               get("cuMemRelease", (void**)&r.release) &&
+               get("cuMemGetAllocationGranularity", (void**)&r.granularity);
+        return r;
+    }();
+    return v;
+}
+
+struct VmRange {
+    CUdeviceptr base = 0;
+    size_t reserved = 0, mapped = 0, gran = 0;
+    std::vector<std::pair<CUmemGenericAllocationHandle, size_t>> chunks;   // mapped back to back
+
+    ~VmRange() {
+        const Vmm& v = vmm();
+        size_t off = 0;
+        for (auto& c : chunks) {
+            v.unmap(base + off, c.second);
+            v.release(c.first);
+            off += c.second;
+        }
+        if (base) v.addr_free(base, reserved);
+    }
+};
+
+}  // namespace
+
+// make at least `bytes` of the range usable (maps one new chunk with 1/8 headroom); false = not
+// possible (no VMM support, or out of memory)
+static bool vm_grow(VmRange& r, int device, size_t bytes) {
+    if (bytes <= r.mapped) return true;
+    const Vmm& v = vmm();
+    if (!v.ok) return false;
+    CUmemAllocationProp prop{};
+    prop.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+    prop.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+    prop.location.id = device;
+    if (!r.base) {
+        size_t free_b = 0, total_b = 0;
+        if (v.granularity(&r.gran, &prop, CU_MEM_ALLOC_GRANULARITY_RECOMMENDED) != CUDA_SUCCESS ||
+            cudaMemGetInfo(&free_b, &total_b) != cudaSuccess)
+            return false;
+        r.reserved = (std::max(total_b, bytes) + r.gran - 1) / r.gran * r.gran;
+        if (v.reserve(&r.base, r.reserved, 0, 0, 0) != CUDA_SUCCESS) {
+            r.base = 0;
+            return false;
+        }
+    }
+    size_t want = bytes + bytes / 8;
+    want = std::min(std::max(want, bytes), r.reserved);
+    if (bytes > r.reserved) return false;
+    const size_t sz = (want - r.mapped + r.gran - 1) / r.gran * r.gran;
+    if (r.mapped + sz > r.reserved) return false;
+    CUmemGenericAllocationHandle h;
+    if (v.create(&h, sz, &prop, 0) != CUDA_SUCCESS) return false;
+    if (v.map(r.base + r.mapped, sz, 0, h, 0) != CUDA_SUCCESS) {
+        v.release(h);
+        return false;
+    }
+    CUmemAccessDesc acc{};
+    acc.location = prop.location;
+    acc.flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+    if (v.set_access(r.base + r.mapped, sz, &acc, 1) != CUDA_SUCCESS) {
+        v.unmap(r.base + r.mapped, sz);
+        v.release(h);
+        return false;
+    }
+    r.chunks.push_back({h, sz});
+    r.mapped += sz;
+    return true;
+}
+
+namespace {
+
+// one elementary interval of the session's layout
+struct SIv {
+    uint64_t abs_begin, len, dense;
+    std::bitset<CUSAN_MAX_FIBERS + 1> readers;   // fibers that read it since its last write
+};
+
+}  // namespace
+
 struct cusan_session {
     const cusan_trace* trace = nullptr;
     cusan_check_opts opts{};
     int device = 0, max_blocks = 0;
     cudaStream_t stream = nullptr;
-    std::vector<Interval> layout;                   // layout of `shadow`
+    // ---- host state carried between calls ----
+    uint32_t F = 1;                                 // clock width = the trace's max_fibers
+    std::vector<uint32_t> C;                        // F × F fiber clocks
+    std::unordered_map<uint64_t, uint32_t> key_slot;
+    std::vector<uint32_t> sc;                       // sync clocks, F per key
+    std::vector<uint32_t> cur_seg;                  // open segment per fiber
+    std::vector<uint32_t> segvc;                    // all segment rows (host copy)
+    uint64_t nseg = 0;
+    std::vector<SIv> ivs;                           // layout of `shadow`
+    uint64_t used = 0;                              // cells of `shadow` in use
+    uint64_t checked_access = 0, checked_events = 0, n_calls = 0;
+    bool broken = false;                            // a call failed after changing the state
+    // ---- device state ----
+    VmRange vm;                                     // the shadow's virtual range (if VMM works)
+    bool vm_shadow = true;
     uint2* shadow = nullptr;
     uint64_t shadow_cap = 0;                        // cells
-    uint2* spare = nullptr;
-    uint64_t spare_cap = 0;
+    uint32_t* d_segvc = nullptr;
+    uint64_t d_segvc_cap = 0, seg_uploaded = 0;     // u32 words / rows on the device
     uint32_t* heap = nullptr;
     uint64_t heap_cap = 0, heap_top = 0;            // record units
     char* scratch = nullptr;
     uint64_t scratch_cap = 0;
     cusan_race_run* runs = nullptr;
     uint64_t run_cap = 0;
-    uint64_t checked_access = 0, checked_events = 0, n_calls = 0;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
 
     ~cusan_session() {
         if (ev0) cudaEventDestroy(ev0);
         if (ev1) cudaEventDestroy(ev1);
-        cudaFree(shadow);
-        cudaFree(spare);
+        if (!vm_shadow) cudaFree(shadow);
+        cudaFree(d_segvc);
         cudaFree(heap);
         cudaFree(scratch);
         cudaFree(runs);
+    }
+
+    uint32_t* sync_clock(uint64_t key) {
+        auto it = key_slot.find(key);
+        if (it == key_slot.end()) {
+            it = key_slot.emplace(key, (uint32_t)(sc.size() / F)).first;
+            sc.resize(sc.size() + F, 0);
+        }
+        return &sc[(size_t)it->second * F];
     }
 };
 
@@ -64,27 +214,272 @@ static int ensure(T** p, uint64_t* cap, uint64_t need, const char* what) {
     return CUSAN_OK;
 }
 
+// grow a device buffer keeping its first `keep` elements.  small = doubling and zero-filled (so
+// the copy never moves uninitialised words, e.g. unused tails of records); !small (the shadow,
+// tens of GB) = exactly `need` and not filled: every cell past `keep` is stored before it is read
+template <class T>
+static int grow_keep(cusan_session* s, T** p, uint64_t* cap, uint64_t need, uint64_t keep, const char* what,
+                     bool small = true) {
+    if (*cap >= need && *p) return CUSAN_OK;
+    const uint64_t n = small ? std::max<uint64_t>(std::max<uint64_t>(need, 2 * *cap), 64) : std::max<uint64_t>(need, 64);
+    T* np = nullptr;
+    if (cudaMalloc((void**)&np, n * sizeof(T)) != cudaSuccess)
+        return fail(CUSAN_ENOMEM, std::string("cannot grow ") + what);
+    cudaError_t e = small ? cudaMemsetAsync(np, 0, n * sizeof(T), s->stream) : cudaSuccess;
+    if (e == cudaSuccess && *p && keep)
+        e = cudaMemcpyAsync(np, *p, keep * sizeof(T), cudaMemcpyDeviceToDevice, s->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s->stream);
+    if (e != cudaSuccess) {
+        cudaFree(np);
+        return cuda_fail(e, what);
+    }
+    cudaFree(*p);
+    *p = np;
+    *cap = n;
+    return CUSAN_OK;
+}
+
 // grow the heap keeping records [0, heap_top)
 static int grow_heap(cusan_session* s, uint64_t need) {
     if (s->heap_cap >= need && s->heap) return CUSAN_OK;
     if (need >= (1ull << 24)) return fail(CUSAN_ENOMEM, "read-set heap exceeds the 24-bit record index");
-    const uint64_t cap = std::min<uint64_t>(std::max<uint64_t>(need, 2 * s->heap_cap), (1ull << 24) - 1);
-    uint32_t* nh = nullptr;
-    if (cudaMalloc((void**)&nh, cap * REC_WORDS * sizeof(uint32_t)) != cudaSuccess)
-        return fail(CUSAN_ENOMEM, "cannot grow the read-set heap");
-    // zeroed, so the copy below never moves uninitialised words (unused tails of records)
-    cudaError_t e = cudaMemsetAsync(nh, 0, cap * REC_WORDS * sizeof(uint32_t), s->stream);
-    if (e == cudaSuccess && s->heap && s->heap_top)
-        e = cudaMemcpyAsync(nh, s->heap, s->heap_top * REC_WORDS * sizeof(uint32_t), cudaMemcpyDeviceToDevice,
-                            s->stream);
-    if (e == cudaSuccess) e = cudaStreamSynchronize(s->stream);
-    if (e != cudaSuccess) {
-        cudaFree(nh);
-        return cuda_fail(e, "grow_heap");
+    uint64_t words = s->heap_cap * REC_WORDS;
+    int st = grow_keep(s, &s->heap, &words, std::min<uint64_t>(need, (1ull << 24) - 1) * REC_WORDS,
+                       s->heap_top * REC_WORDS, "the read-set heap");
+    if (!st) s->heap_cap = std::min<uint64_t>(words / REC_WORDS, (1ull << 24) - 1);
+    return st;
+}
+
+// The incremental host plan of one call (a1 + a2 for the new events).
+struct CallPlan {
+    std::vector<uint64_t> g0, g1;                   // new accesses (granule ranges)
+    std::vector<AccRec> rec;
+    std::vector<SIv> ivs;                           // new layout
+    std::vector<char> has_state;                    // per new interval: covered before this call
+    std::vector<uint32_t> inc_off, inc_cnt;         // per new interval: new incidences (CSR)
+    std::vector<AccRec> inc;
+    std::vector<uint32_t> inc_acc;                  // call-local access index of each incidence
+    HostPlan hp;                                    // spans, windows and counters for the launches
+    std::vector<CopySeg> segs;                      // cells to copy (compressed split pieces)
+    uint64_t copy_cells = 0, used = 0, tracked = 0; // used: shadow cells in use after the call
+};
+
+static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
+    const uint32_t F = s->F;
+    cusan_counters& c = cp.hp.ctr;
+    c = cusan_counters{};
+    c.n_fibers = F;
+    // ---- a1: clocks and segments for the new events (build_host_plan's pass, resumed) ----------
+    for (uint64_t i = s->checked_events; i < tr.ev.size(); i++) {
+        const cusan_event& e = tr.ev[i];
+        const uint32_t f = e.fiber;
+        uint32_t* Cf = &s->C[(size_t)f * F];
+        c.n_events++;
+        if (e.kind == CUSAN_EV_FORK) {
+            const uint32_t src = (uint32_t)e.a;
+            uint32_t* Cs = &s->C[(size_t)src * F];
+            Cs[src] = (uint32_t)(i + 1);
+            for (uint32_t g = 0; g < F; g++) Cf[g] = std::max(Cf[g], Cs[g]);
+            s->cur_seg[f] = NO_SEG;
+            c.n_fork++;
+            continue;
+        }
+        Cf[f] = (uint32_t)(i + 1);
+        switch (e.kind) {
+            case CUSAN_EV_ACCESS: {
+                if (s->cur_seg[f] == NO_SEG) {
+                    if (s->nseg >= 0x7fffffffu) return fail(CUSAN_ERANGE, "too many segments");
+                    s->cur_seg[f] = (uint32_t)s->nseg++;
+                    s->segvc.insert(s->segvc.end(), Cf, Cf + F);
+                }
+                const uint64_t g0 = e.a >> 3, g1 = e.b ? (e.a + e.b + 7) >> 3 : g0;
+                cp.g0.push_back(g0);
+                cp.g1.push_back(g1);
+                cp.rec.push_back({pack_epoch(f, (uint32_t)i), s->cur_seg[f] | ((uint32_t)e.mode << 31)});
+                const uint64_t bytes = 8 * (g1 - g0);
+                c.n_access++;
+                cp.tracked += bytes;
+                if (e.mode) { c.n_write++; c.bytes_written += bytes; }
+                else { c.n_read++; c.bytes_read += bytes; }
+                break;
+            }
+            case CUSAN_EV_RELEASE: {
+                uint32_t* S = s->sync_clock(e.a);
+                for (uint32_t g = 0; g < F; g++) S[g] = std::max(S[g], Cf[g]);
+                c.n_release++;
+                break;
+            }
+            case CUSAN_EV_RELEASE_STORE: {
+                uint32_t* S = s->sync_clock(e.a);
+                std::copy(Cf, Cf + F, S);
+                c.n_release_store++;
+                break;
+            }
+            case CUSAN_EV_ACQUIRE: {
+                uint32_t* S = s->sync_clock(e.a);
+                for (uint32_t g = 0; g < F; g++) Cf[g] = std::max(Cf[g], S[g]);
+                s->cur_seg[f] = NO_SEG;
+                c.n_acquire++;
+                break;
+            }
+            default:
+                return fail(CUSAN_EINVAL, "bad event kind in trace");
+        }
     }
-    cudaFree(s->heap);
-    s->heap = nh;
-    s->heap_cap = cap;
+    c.tracked_bytes = cp.tracked;
+    c.n_segments = s->nseg;
+
+    // ---- a2: refine the layout by the new endpoints -----------------------------------------------
+    const uint64_t n_new = cp.g0.size();
+    std::vector<uint64_t> P;
+    P.reserve(2 * (n_new + s->ivs.size()));
+    for (uint64_t k = 0; k < n_new; k++)
+        if (cp.g1[k] > cp.g0[k]) { P.push_back(cp.g0[k]); P.push_back(cp.g1[k]); }
+    for (const SIv& u : s->ivs) { P.push_back(u.abs_begin); P.push_back(u.abs_begin + u.len); }
+    std::sort(P.begin(), P.end());
+    P.erase(std::unique(P.begin(), P.end()), P.end());
+    const uint64_t np = P.size();
+    std::vector<int64_t> diff(np + 1, 0);
+    std::vector<uint32_t> b0(n_new, 0), b1(n_new, 0);
+    for (uint64_t k = 0; k < n_new; k++) {
+        if (cp.g1[k] <= cp.g0[k]) continue;
+        b0[k] = (uint32_t)(std::lower_bound(P.begin(), P.end(), cp.g0[k]) - P.begin());
+        b1[k] = (uint32_t)(std::lower_bound(P.begin(), P.end(), cp.g1[k]) - P.begin());
+        diff[b0[k]]++;
+        diff[b1[k]]--;
+    }
+    const bool compressed = (s->opts.flags & CUSAN_CHECK_INTERVAL_SHADOW) != 0;
+    std::vector<uint32_t> iv_of(np ? np - 1 : 0, 0xffffffffu);
+    uint64_t used = s->used;
+    {
+        int64_t cov = 0;
+        size_t u = 0;
+        for (uint64_t j = 0; j + 1 < np; j++) {
+            cov += diff[j];
+            while (u < s->ivs.size() && s->ivs[u].abs_begin + s->ivs[u].len <= P[j]) u++;
+            const bool old = u < s->ivs.size() && s->ivs[u].abs_begin <= P[j];
+            if (cov <= 0 && !old) continue;
+            SIv v;
+            v.abs_begin = P[j];
+            v.len = P[j + 1] - P[j];
+            if (old) {                 // a piece of an old interval: its state, its cells in place
+                const SIv& o = s->ivs[u];
+                v.readers = o.readers;
+                if (!compressed) {
+                    v.dense = o.dense + (P[j] - o.abs_begin);
+                } else if (P[j] == o.abs_begin) {
+                    v.dense = o.dense;
+                } else {               // compressed: a further piece gets a copy of the one cell
+                    v.dense = used++;
+                    cp.segs.push_back({cp.copy_cells, o.dense, v.dense, 1});
+                    cp.copy_cells++;
+                }
+            } else {                   // memory touched for the first time: new cells at the end
+                if (compressed) {
+                    v.dense = used++;
+                } else {
+                    v.dense = (used + CELL_ALIGN - 1) / CELL_ALIGN * CELL_ALIGN;
+                    used = v.dense + v.len;
+                }
+            }
+            iv_of[j] = (uint32_t)cp.ivs.size();
+            cp.ivs.push_back(v);
+            cp.has_state.push_back(old ? 1 : 0);
+        }
+    }
+    cp.used = used;
+    const size_t niv = cp.ivs.size();
+    c.n_intervals = niv;
+    // new incidences per interval, in trace order
+    cp.inc_cnt.assign(niv, 0);
+    for (uint64_t k = 0; k < n_new; k++)
+        for (uint32_t j = b0[k]; j < b1[k]; j++) cp.inc_cnt[iv_of[j]]++;
+    cp.inc_off.assign(niv, 0);
+    uint64_t n_inc = 0;
+    for (size_t i = 0; i < niv; i++) {
+        cp.inc_off[i] = (uint32_t)n_inc;
+        n_inc += cp.inc_cnt[i];
+    }
+    if (n_inc > 0xffffffffull) return fail(CUSAN_ERANGE, "too many interval incidences");
+    c.n_incidences = n_inc;
+    cp.inc.resize(n_inc);
+    cp.inc_acc.resize(n_inc);
+    {
+        std::vector<uint32_t> at(cp.inc_off);
+        for (uint64_t k = 0; k < n_new; k++)
+            for (uint32_t j = b0[k]; j < b1[k]; j++) {
+                const uint32_t q = at[iv_of[j]]++;
+                cp.inc[q] = cp.rec[k];
+                cp.inc_acc[q] = (uint32_t)k;
+            }
+    }
+    uint64_t granules = 0;
+    for (const SIv& v : cp.ivs) granules += v.len;
+    c.shard_granules = granules;
+    c.tracked_bytes_shard = cp.tracked;
+
+    // ---- windows and spans for the new incidences; moves for the untouched intervals ---------------
+    const uint64_t W = s->opts.window_events > 0 ? (uint64_t)s->opts.window_events : std::max<uint64_t>(n_new, 1);
+    const uint64_t nwin = n_new ? (n_new + W - 1) / W : 0;
+    std::vector<std::pair<uint64_t, Span>> out;
+    for (size_t i = 0; i < niv; i++) {
+        SIv& v = cp.ivs[i];
+        const bool has_state = cp.has_state[i];
+        const uint32_t qa = cp.inc_off[i], qe = qa + cp.inc_cnt[i];
+        if (qa == qe) continue;                      // untouched: its cells stay where they are
+        for (uint32_t q = qa; q < qe;) {
+            const uint64_t w = cp.inc_acc[q] / W;
+            uint32_t q2 = q;
+            while (q2 < qe && cp.inc_acc[q2] / W == w) {
+                const AccRec& r = cp.inc[q2];
+                if (r.segm >> 31) v.readers.reset();
+                else v.readers.set(r.epoch >> 24);
+                q2++;
+            }
+            Span sp{};
+            sp.abs_begin = v.abs_begin;
+            sp.dense_begin = v.dense;
+            sp.len = v.len;
+            sp.list_off = q;
+            sp.list_cnt = q2 - q;
+            const bool first_span = q == qa;
+            sp.flags = ((!first_span || has_state) ? SPAN_LOAD : 0u) | SPAN_STORE |
+                       (first_span ? SPAN_FIRST_IN_CALL : 0u) | (compressed ? SPAN_COMPRESSED : 0u);
+            const uint64_t nr = v.readers.count();
+            if (nr >= 2) sp.rec_units = (uint32_t)((nr + 1 + REC_WORDS - 1) / REC_WORDS);
+            out.emplace_back(w, sp);
+            q = q2;
+        }
+    }
+    // window-major (stable by interval), records numbered from the heap top
+    std::vector<uint64_t> wstart(nwin + 1, 0);
+    for (const auto& ws : out) wstart[ws.first + 1]++;
+    for (uint64_t w = 0; w < nwin; w++) wstart[w + 1] += wstart[w];
+    HostPlan& hp = cp.hp;
+    hp.spans.assign(out.size(), Span{});
+    {
+        std::vector<uint64_t> at(wstart.begin(), wstart.end() - 1);
+        for (const auto& ws : out) hp.spans[at[ws.first]++] = ws.second;
+    }
+    hp.rec_units = 0;
+    hp.spill_spans = 0;
+    for (Span& sp : hp.spans)
+        if (sp.rec_units) {
+            sp.rec = (uint32_t)(s->heap_top + hp.rec_units);
+            hp.rec_units += sp.rec_units;
+            hp.spill_spans++;
+        }
+    if (s->heap_top + hp.rec_units >= (1u << 24) - 1)
+        return fail(CUSAN_ERANGE, "too many read-set records for the 24-bit record index");
+    hp.win_span_off.assign(1, 0);
+    for (uint64_t w = 0; w < nwin; w++)
+        if (wstart[w + 1] > wstart[w]) hp.win_span_off.push_back(wstart[w + 1]);
+    hp.F = F;
+    hp.window_accesses = W;
+    c.n_windows = hp.win_span_off.size() - 1;
+    c.n_spans = hp.spans.size();
+    c.spill_spans = hp.spill_spans;
+    c.spill_heap_bytes = hp.rec_units * REC_WORDS * 4;
     return CUSAN_OK;
 }
 
@@ -96,11 +491,15 @@ int cusan_session_create(const cusan_trace* t, const cusan_check_opts* o, cusan_
     if (o->nshards != 1 || o->shard != 0)
         return fail(CUSAN_EINVAL, "sessions check the whole granule space (nshards = 1)");
     if (o->workspace) return fail(CUSAN_EINVAL, "sessions manage their own device memory");
+    if (o->window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
     cusan_session* s = new (std::nothrow) cusan_session;
     if (!s) return fail(CUSAN_ENOMEM, "cannot allocate session");
     s->trace = t;
     s->opts = *o;
     s->opts.persist_shadow = 1;
+    s->F = t->t.max_fibers;
+    s->C.assign((size_t)s->F * s->F, 0);
+    s->cur_seg.assign(s->F, NO_SEG);
     int st = device_info(o->device, &s->max_blocks);
     if (!st) {
         s->device = o->device;
@@ -123,144 +522,116 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
     CK(cudaSetDevice(s->device));
     const Trace& tr = s->trace->t;
     if (tr.ev.size() < s->checked_events) return fail(CUSAN_ESTATE, "the trace shrank");
+    if (s->broken) return fail(CUSAN_ESTATE, "an earlier call failed after changing the session's state");
+    s->broken = true;   // cleared when this call commits
 
-    // ---- a1 + a2 over the whole trace; spans only for the new accesses ------------------------
-    HostPlan hp;
+    // ---- host: incremental a1 + a2 (the clocks and the layout carry over) -------------------------
+    CallPlan cp;
     int st;
     try {
-        st = build_host_plan(tr, s->opts, hp, s->checked_access, s->heap_top);
+        st = plan_call(s, tr, cp);
     } catch (const std::bad_alloc&) {
         st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
     }
     if (st) return st;
-    const uint64_t first = s->checked_access, n_acc = hp.acc_g0.size();
-    uint64_t new_tracked = 0;
-    for (uint64_t k = first; k < n_acc; k++) new_tracked += 8 * (hp.acc_g1[k] - hp.acc_g0[k]);
-
-    // ---- old layout -> new layout ----------------------------------------------------------------
-    // intervals are elementary for all accesses so far, so each new interval lies inside one old
-    // interval or outside the old coverage
-    std::vector<uint64_t> old_src(hp.iv.size(), UINT64_MAX);
-    std::vector<CopySeg> segs;
-    uint64_t copy_cells_n = 0;
-    const bool compressed = (s->opts.flags & CUSAN_CHECK_INTERVAL_SHADOW) != 0;
-    {
-        size_t j = 0;
-        for (size_t i = 0; i < hp.iv.size(); i++) {
-            const Interval& v = hp.iv[i];
-            while (j < s->layout.size() && s->layout[j].abs_begin + s->layout[j].len <= v.abs_begin) j++;
-            if (j < s->layout.size() && s->layout[j].abs_begin <= v.abs_begin) {
-                const Interval& u = s->layout[j];
-                // compressed layouts (f3) keep one cell per interval: a split piece copies it
-                old_src[i] = compressed ? u.dense_begin : u.dense_begin + (v.abs_begin - u.abs_begin);
-                const uint64_t ncell = compressed ? 1 : v.len;
-                const bool touched = v.list_cnt && hp.inc_acc[v.list_off + v.list_cnt - 1] >= first;
-                if (!touched) {
-                    segs.push_back({copy_cells_n, old_src[i], v.dense_begin, ncell});
-                    copy_cells_n += ncell;
-                }
-            }
-        }
-    }
-    for (Span& sp : hp.spans) {
-        if (!(sp.flags & SPAN_FIRST_IN_CALL) || !(sp.flags & SPAN_LOAD)) continue;
-        auto it = std::lower_bound(hp.iv.begin(), hp.iv.end(), sp.dense_begin,
-                                   [](const Interval& a, uint64_t d) { return a.dense_begin < d; });
-        const size_t i = it - hp.iv.begin();
-        if (i >= hp.iv.size() || old_src[i] == UINT64_MAX)
-            return fail(CUSAN_ESTATE, "internal: a loaded interval has no previous state");
-        sp.flags |= SPAN_SRC_OLD;
-        sp.src_begin = old_src[i];
-    }
+    HostPlan& hp = cp.hp;
     SpanTables tabs;
     build_span_tables(hp, s->max_blocks, tabs);
 
     // ---- device memory ---------------------------------------------------------------------------
-    if ((st = ensure(&s->spare, &s->spare_cap, hp.shadow_cells, "shadow"))) return st;
+    // the shadow grows as new memory is touched: new chunks mapped in place, else re-allocated
+    // with its cells moved (1/8 headroom either way)
+    if (cp.used > s->shadow_cap) {
+        if (s->vm_shadow && vm_grow(s->vm, s->device, cp.used * sizeof(uint2))) {
+            s->shadow = (uint2*)s->vm.base;
+            s->shadow_cap = s->vm.mapped / sizeof(uint2);
+        } else {
+            if (s->vm_shadow && s->vm.mapped)
+                return fail(CUSAN_ENOMEM, "cannot map more shadow memory");
+            s->vm_shadow = false;
+            if ((st = grow_keep(s, &s->shadow, &s->shadow_cap, cp.used + cp.used / 8, s->used, "shadow", false)))
+                return st;
+        }
+    }
     if ((st = grow_heap(s, s->heap_top + hp.rec_units + (1ull << 16)))) return st;
-    if ((st = ensure(&s->runs, &s->run_cap, std::max<uint64_t>(s->run_cap, 1ull << 16), "run buffer"))) return st;
+    if ((st = ensure(&s->runs, &s->run_cap, std::max<uint64_t>(s->run_cap, 1ull << 20), "run buffer"))) return st;
+    const uint64_t seg_words = s->nseg * s->F, up_words = s->seg_uploaded * s->F;
+    const uint64_t new_row_bytes = (seg_words - up_words) * sizeof(uint32_t);
+    if ((st = grow_keep(s, &s->d_segvc, &s->d_segvc_cap, seg_words, up_words, "segment rows"))) return st;
+    if (seg_words > up_words)                        // only the rows new since the last call
+        CK(cudaMemcpyAsync(s->d_segvc + up_words, s->segvc.data() + up_words,
+                           (seg_words - up_words) * sizeof(uint32_t), cudaMemcpyHostToDevice, s->stream));
     const uint64_t nwin = tabs.wins.size();
     uint64_t off = 0;
-    const uint64_t o_inc = off;   off = align_up(off + hp.inc.size() * sizeof(AccRec));
-    const uint64_t o_seg = off;   off = align_up(off + hp.segvc.size() * sizeof(uint32_t));
+    const uint64_t o_inc = off;   off = align_up(off + cp.inc.size() * sizeof(AccRec));
     const uint64_t o_spans = off; off = align_up(off + tabs.ds.size() * sizeof(DSpan));
-    const uint64_t o_copy = off;  off = align_up(off + segs.size() * sizeof(CopySeg));
+    const uint64_t o_copy = off;  off = align_up(off + cp.segs.size() * sizeof(CopySeg));
     const uint64_t o_cnt = off;   off = align_up(off + (N_COUNTERS + nwin) * sizeof(unsigned long long));
     if ((st = ensure(&s->scratch, &s->scratch_cap, off, "plan tables"))) return st;
     AccRec* d_inc = (AccRec*)(s->scratch + o_inc);
-    uint32_t* d_seg = (uint32_t*)(s->scratch + o_seg);
     DSpan* d_spans = (DSpan*)(s->scratch + o_spans);
     CopySeg* d_copy = (CopySeg*)(s->scratch + o_copy);
     unsigned long long* d_cnt = (unsigned long long*)(s->scratch + o_cnt);
-    CK(cudaMemcpyAsync(d_inc, hp.inc.data(), hp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, s->stream));
-    CK(cudaMemcpyAsync(d_seg, hp.segvc.data(), hp.segvc.size() * sizeof(uint32_t), cudaMemcpyHostToDevice, s->stream));
+    CK(cudaMemcpyAsync(d_inc, cp.inc.data(), cp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, s->stream));
     CK(cudaMemcpyAsync(d_spans, tabs.ds.data(), tabs.ds.size() * sizeof(DSpan), cudaMemcpyHostToDevice, s->stream));
-    CK(cudaMemcpyAsync(d_copy, segs.data(), segs.size() * sizeof(CopySeg), cudaMemcpyHostToDevice, s->stream));
+    CK(cudaMemcpyAsync(d_copy, cp.segs.data(), cp.segs.size() * sizeof(CopySeg), cudaMemcpyHostToDevice, s->stream));
 
-    // ---- a3 / a4 (re-runnable: only `spare` and fresh heap units are written) ----------------------
+    // ---- a3 / a4, in place ------------------------------------------------------------------------
     std::vector<unsigned long long> init(N_COUNTERS + nwin, 0ull), cnt(N_COUNTERS, 0ull);
-    float kms = 0.f;
-    for (int attempt = 0;; attempt++) {
-        init[C_HEAP] = s->heap_top + hp.rec_units;
-        CK(cudaMemcpyAsync(d_cnt, init.data(), init.size() * sizeof(unsigned long long), cudaMemcpyHostToDevice,
-                           s->stream));
-        CK(cudaEventRecord(s->ev0, s->stream));
-        if (copy_cells_n)
-            CK(launch_copy_cells(s->max_blocks, s->stream, s->shadow, s->spare, d_copy, (uint32_t)segs.size(),
-                                  copy_cells_n));
-        Ctx k;
-        k.inc = d_inc;
-        k.segvc = d_seg;
-        k.F = hp.F;
-        k.shadow = s->spare;
-        k.shadow_old = s->shadow;
-        k.heap = s->heap;
-        k.heap_cap = s->heap_cap;
-        k.runs = s->runs;
-        k.counters = d_cnt;
-        k.run_cap = s->run_cap;
-        k.cow_all = 1;
-        const int force_lanes = (s->opts.flags & CUSAN_CHECK_FORCE_LANES) ? 1 : 0;
-        for (size_t i = 0; i < nwin; i++) {
-            const Window& w = tabs.wins[i];
-            unsigned long long* sched = CUSAN_DYNAMIC ? d_cnt + N_COUNTERS + i : nullptr;
-            CK(launch_shadow_check(w.grid, s->stream, d_spans + w.span_off, w.nspans, w.tiles, w.weight, k,
-                                   force_lanes, sched));
-        }
-        CK(cudaGetLastError());
-        CK(cudaEventRecord(s->ev1, s->stream));
-        CK(cudaMemcpyAsync(cnt.data(), d_cnt, N_COUNTERS * sizeof(unsigned long long), cudaMemcpyDeviceToHost,
-                           s->stream));
-        CK(cudaStreamSynchronize(s->stream));
-        const bool runs_ovf = cnt[C_RUNS] > s->run_cap, heap_ovf = cnt[C_HEAP_OVF] != 0;
-        if (!runs_ovf && !heap_ovf) break;
-        if (attempt >= 8) return fail(CUSAN_ENOMEM, "run buffer / read-set heap keeps overflowing");
-        if (runs_ovf && (st = ensure(&s->runs, &s->run_cap, cnt[C_RUNS] + cnt[C_RUNS] / 8 + 1024, "run buffer")))
-            return st;
-        if (heap_ovf && (st = grow_heap(s, 2 * s->heap_cap))) return st;
+    init[C_HEAP] = s->heap_top + hp.rec_units;
+    CK(cudaMemcpyAsync(d_cnt, init.data(), init.size() * sizeof(unsigned long long), cudaMemcpyHostToDevice,
+                       s->stream));
+    CK(cudaEventRecord(s->ev0, s->stream));
+    if (cp.copy_cells)
+        CK(launch_copy_cells(s->max_blocks, s->stream, s->shadow, s->shadow, d_copy, (uint32_t)cp.segs.size(),
+                             cp.copy_cells, s->heap));
+    Ctx k;
+    k.inc = d_inc;
+    k.segvc = s->d_segvc;
+    k.F = s->F;
+    k.shadow = s->shadow;
+    k.heap = s->heap;
+    k.heap_cap = s->heap_cap;
+    k.runs = s->runs;
+    k.counters = d_cnt;
+    k.run_cap = s->run_cap;
+    const int force_lanes = (s->opts.flags & CUSAN_CHECK_FORCE_LANES) ? 1 : 0;
+    for (size_t i = 0; i < nwin; i++) {
+        const Window& w = tabs.wins[i];
+        unsigned long long* sched = CUSAN_DYNAMIC ? d_cnt + N_COUNTERS + i : nullptr;
+        CK(launch_shadow_check(w.grid, s->stream, d_spans + w.span_off, w.nspans, w.tiles, w.weight, k, force_lanes,
+                               sched));
     }
+    CK(cudaEventRecord(s->ev1, s->stream));
+    CK(cudaMemcpyAsync(cnt.data(), d_cnt, N_COUNTERS * sizeof(unsigned long long), cudaMemcpyDeviceToHost,
+                       s->stream));
+    CK(cudaStreamSynchronize(s->stream));
+    float kms = 0.f;
     CK(cudaEventElapsedTime(&kms, s->ev0, s->ev1));
+    if (cnt[C_HEAP_OVF]) return fail(CUSAN_ENOMEM, "read-set heap overflow: the session's state is lost");
+    const bool runs_ovf = cnt[C_RUNS] > s->run_cap;
+    const uint64_t kept_runs = std::min<uint64_t>(cnt[C_RUNS], s->run_cap);
 
-    // ---- commit: the new buffer becomes the shadow ------------------------------------------------
-    std::swap(s->shadow, s->spare);
-    std::swap(s->shadow_cap, s->spare_cap);
-    s->layout = hp.iv;
+    // ---- commit: the new layout becomes the session's ---------------------------------------------
+    s->ivs.swap(cp.ivs);
+    s->used = cp.used;
+    s->seg_uploaded = s->nseg;
     s->heap_top = cnt[C_HEAP];
-    s->checked_access = n_acc;
+    s->checked_access += cp.g0.size();
     s->checked_events = tr.ev.size();
     s->n_calls++;
 
     cusan_report* r = new (std::nothrow) cusan_report;
     if (!r) return fail(CUSAN_ENOMEM, "cannot allocate report");
     try {
-        r->runs.resize(cnt[C_RUNS]);
+        r->runs.resize(kept_runs);
     } catch (...) {
         delete r;
         return fail(CUSAN_ENOMEM, "cannot allocate report runs");
     }
-    if (cnt[C_RUNS]) {
-        cudaError_t ce = cudaMemcpy(r->runs.data(), s->runs, cnt[C_RUNS] * sizeof(cusan_race_run),
-                                    cudaMemcpyDeviceToHost);
+    if (kept_runs) {
+        cudaError_t ce =
+            cudaMemcpy(r->runs.data(), s->runs, kept_runs * sizeof(cusan_race_run), cudaMemcpyDeviceToHost);
         if (ce != cudaSuccess) {
             delete r;
             return cuda_fail(ce, "run download");
@@ -268,23 +639,26 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
     }
     canonicalize_runs(r->runs);
     r->n_runs = r->runs.size();
-    r->n_race_granules = cnt[C_RACE];
+    r->n_race_granules = cnt[C_RACE];   // exact even when the run list overflowed
+    if (runs_ovf) r->truncated = 1;     // the state is committed; the call cannot be re-run
     if (s->opts.max_runs && r->runs.size() > s->opts.max_runs) {
         r->runs.resize(s->opts.max_runs);
         r->truncated = 1;
     }
     r->ctr = hp.ctr;
-    r->ctr.tracked_bytes_shard = new_tracked;       // checked by this call
     r->ctr.raw_runs = cnt[C_RUNS];
     r->ctr.kernel_ms = kms;
-    r->ctr.kernel_launches = nwin + (copy_cells_n ? 1 : 0);
-    r->ctr.shadow_cell_bytes = tabs.cell_bytes + 16 * copy_cells_n;
-    r->ctr.shadow_bytes = hp.shadow_cells * sizeof(uint2);
-    r->ctr.h2d_bytes = hp.inc.size() * sizeof(AccRec) + hp.segvc.size() * sizeof(uint32_t) +
-                       tabs.ds.size() * sizeof(DSpan) + segs.size() * sizeof(CopySeg);
-    r->ctr.d2h_bytes = N_COUNTERS * sizeof(unsigned long long) + cnt[C_RUNS] * sizeof(cusan_race_run);
+    r->ctr.kernel_launches = nwin + (cp.copy_cells ? 1 : 0);
+    r->ctr.shadow_cell_bytes = tabs.cell_bytes + 16 * cp.copy_cells;
+    r->ctr.shadow_bytes = s->used * sizeof(uint2);
+    r->ctr.h2d_bytes = cp.inc.size() * sizeof(AccRec) + tabs.ds.size() * sizeof(DSpan) +
+                       cp.segs.size() * sizeof(CopySeg) + new_row_bytes;
+    r->ctr.d2h_bytes = N_COUNTERS * sizeof(unsigned long long) + kept_runs * sizeof(cusan_race_run);
     r->ctr.run_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count();
+    s->broken = false;
     *out = r;
+    // a run list that overflowed is sized for the next call (best effort: this call succeeded)
+    if (runs_ovf) ensure(&s->runs, &s->run_cap, cnt[C_RUNS] + cnt[C_RUNS] / 8 + 1024, "run buffer");
     return CUSAN_OK;
 }
 
@@ -296,4 +670,3 @@ int cusan_session_destroy(cusan_session* s) {
 }
 
 }  // extern "C"
-

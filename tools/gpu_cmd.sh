@@ -1,3 +1,8 @@
-mkdir -p gpurun_out
-echo "== racecheck"; timeout 1500 compute-sanitizer --tool racecheck --racecheck-report hazard --error-exitcode 9 --print-limit 10 python tools/sanitize_small.py > gpurun_out/sanitizer_racecheck.log 2>&1; echo "exit $?"; tail -3 gpurun_out/sanitizer_racecheck.log
-echo "== initcheck (no TMA build)"; CUSAN_LIBRARY=tools/var_notma.so timeout 1500 compute-sanitizer --tool initcheck --error-exitcode 9 --print-limit 10 python tools/sanitize_small.py > gpurun_out/sanitizer_initcheck_notma.log 2>&1; echo "exit $?"; tail -3 gpurun_out/sanitizer_initcheck_notma.log
+timeout 900 python -m pytest tests/test_gpu_session.py -x -q 2>&1 | tail -3
+timeout 600 python tools/session_bench.py --config 5 --chunk 4096 > gpurun_out/session_c5_4096.json; cut -c1-300 gpurun_out/session_c5_4096.json
+timeout 600 python tools/session_bench.py --config 5 --chunk 512 > gpurun_out/session_c5_512.json; cut -c1-300 gpurun_out/session_c5_512.json
+python - <<'P'
+import json
+d=json.load(open('gpurun_out/session_c5_4096.json'))
+for c in d['per_call']: print(round(c['seconds']*1e3,1), round(c['kernel_ms'],1), c['launches'])
+P
