@@ -46,9 +46,9 @@ class Trace:
         _ck(lib.cusan_trace_create(max_fibers, reserve_events, C.byref(h)))
         self.h = h
 
-    def __del__(self):
+    def __del__(self, _destroy=lib.cusan_trace_destroy):   # bound now: safe at interpreter exit
         if getattr(self, "h", None):
-            lib.cusan_trace_destroy(self.h)
+            _destroy(self.h)
             self.h = None
 
     def cusan_trace_append_access(self, fiber: int, mode: int, addr: int, nbytes: int) -> int:
@@ -90,9 +90,9 @@ class Lowering:
         self.h = h
         self.trace = trace
 
-    def __del__(self):
+    def __del__(self, _destroy=lib.cusan_lowering_destroy):
         if getattr(self, "h", None):
-            lib.cusan_lowering_destroy(self.h)
+            _destroy(self.h)
             self.h = None
 
     def cusan_lowering_fiber_info(self, fiber: int) -> tuple[int, int]:
@@ -156,9 +156,9 @@ class Report:
         else:
             self.runs = np.zeros(0, RUN_DTYPE)
 
-    def __del__(self):
+    def __del__(self, _free=lib.cusan_report_free):
         if getattr(self, "h", None):
-            lib.cusan_report_free(self.h)
+            _free(self.h)
             self.h = None
 
 
@@ -216,9 +216,9 @@ class Plan:
         _ck(lib.cusan_plan_run(self.h, C.byref(h)))
         return _report(h, self.max_runs)
 
-    def close(self):
+    def close(self, _destroy=lib.cusan_plan_destroy):
         if getattr(self, "h", None):
-            lib.cusan_plan_destroy(self.h)
+            _destroy(self.h)
             self.h = None
         self.workspace = None
 
@@ -242,9 +242,9 @@ class Session:
         _ck(lib.cusan_session_check(self.h, C.byref(h)))
         return _report(h, self.max_runs)
 
-    def close(self):
+    def close(self, _destroy=lib.cusan_session_destroy):
         if getattr(self, "h", None):
-            lib.cusan_session_destroy(self.h)
+            _destroy(self.h)
             self.h = None
 
     __del__ = close

@@ -2,6 +2,8 @@
 // the window launches, overflow re-runs, run download and the canonical report.
 #include <algorithm>
 #include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -39,6 +41,7 @@ struct cusan_plan {
     uint64_t shadow_cell_bytes = 0;
     uint64_t table_bytes = 0;               // tables uploaded by plan_create
     std::vector<unsigned long long> counter_init;
+    RunMerge merge;                         // a4 scratch (device run merge)
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
 
     ~cusan_plan() {
@@ -158,7 +161,12 @@ static int plan_device_setup(cusan_plan* p) {
     const uint64_t o_cnt = off;     off = align_up(off + (N_COUNTERS + p->wins.size()) * sizeof(unsigned long long));
     const uint64_t o_heap = off;    off = align_up(off + p->heap_cap * REC_WORDS * sizeof(uint32_t));
     const uint64_t o_shadow = off;  off = align_up(off + (p->need_shadow ? hp.shadow_cells * sizeof(uint2) : 0));
-    p->run_cap = std::max<uint64_t>(1ull << 16, 4 * p->wins.size() + 1024);
+    // raw runs: a range with equal cells emits one run per racing pair, and ranges taken by different
+    // warps are not joined before the device merge, so the buffer is sized from the ranges (an
+    // overflow re-runs the check with a larger buffer)
+    uint64_t tiles = 0;
+    for (const Window& w : p->wins) tiles += w.tiles;
+    p->run_cap = std::min<uint64_t>(std::max<uint64_t>(1ull << 16, 2 * tiles + 4 * p->wins.size() + 1024), 1ull << 24);
     const uint64_t o_runs = off;    off = align_up(off + p->run_cap * sizeof(cusan_race_run));
     p->ws_bytes = off;
     p->o_inc = o_inc;
@@ -290,7 +298,9 @@ int cusan_plan_run(cusan_plan* p, cusan_report** out) {
     const auto t_start = std::chrono::steady_clock::now();
     CK(cudaSetDevice(p->device));
     unsigned long long cnt[N_COUNTERS];
+    int attempts = 0;
     for (int attempt = 0;; attempt++) {
+        attempts = attempt + 1;
         int st = launch_all(p);
         if (st) return st;
         CK(cudaMemcpyAsync(cnt, p->d_counters, sizeof(cnt), cudaMemcpyDeviceToHost, p->stream));
@@ -323,22 +333,19 @@ int cusan_plan_run(cusan_plan* p, cusan_report** out) {
     CK(cudaEventElapsedTime(&kms, p->ev0, p->ev1));
     cusan_report* r = new (std::nothrow) cusan_report;
     if (!r) return fail(CUSAN_ENOMEM, "cannot allocate report");
-    try {
-        r->runs.resize(cnt[C_RUNS]);
-    } catch (...) {
+    uint64_t d2h = sizeof(cnt);
+    const auto t_checked = std::chrono::steady_clock::now();
+    const int mst = merge_runs_device(p->merge, p->stream, p->d_runs, cnt[C_RUNS], r->runs, &d2h);   // a4
+    if (std::getenv("CUSAN_DEBUG_TIMING")) {
+        using ms = std::chrono::duration<double, std::milli>;
+        std::fprintf(stderr, "cusan_plan_run: %d attempt(s), check %.3f ms (kernels %.3f), merge %.3f ms of %llu raw runs\n",
+                     attempts, ms(t_checked - t_start).count(), kms, ms(std::chrono::steady_clock::now() - t_checked).count(),
+                     (unsigned long long)cnt[C_RUNS]);
+    }
+    if (mst) {
         delete r;
-        return fail(CUSAN_ENOMEM, "cannot allocate report runs");
+        return mst;
     }
-    if (cnt[C_RUNS]) {
-        cudaError_t ce = cudaMemcpyAsync(r->runs.data(), p->d_runs, cnt[C_RUNS] * sizeof(cusan_race_run),
-                                         cudaMemcpyDeviceToHost, p->stream);
-        if (ce == cudaSuccess) ce = cudaStreamSynchronize(p->stream);
-        if (ce != cudaSuccess) {
-            delete r;
-            return cuda_fail(ce, "run download");
-        }
-    }
-    canonicalize_runs(r->runs);
     r->n_runs = r->runs.size();
     r->n_race_granules = cnt[C_RACE];
     const uint64_t max_runs = p->hp.opts.max_runs;
@@ -349,10 +356,10 @@ int cusan_plan_run(cusan_plan* p, cusan_report** out) {
     r->ctr = p->hp.ctr;
     r->ctr.raw_runs = cnt[C_RUNS];
     r->ctr.kernel_ms = kms;
-    r->ctr.kernel_launches = p->wins.size();
+    r->ctr.kernel_launches = p->wins.size() + (cnt[C_RUNS] ? MERGE_LAUNCHES : 0);
     r->ctr.shadow_cell_bytes = p->shadow_cell_bytes;
     r->ctr.h2d_bytes = p->table_bytes + sizeof(unsigned long long) * N_COUNTERS;
-    r->ctr.d2h_bytes = sizeof(cnt) + cnt[C_RUNS] * sizeof(cusan_race_run);
+    r->ctr.d2h_bytes = d2h;
     r->ctr.run_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count();
     *out = r;
     return CUSAN_OK;

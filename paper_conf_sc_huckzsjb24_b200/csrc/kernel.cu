@@ -12,7 +12,7 @@
 //       read b on fiber f: R[f] := b
 //   with HB(e = (g, i+1), b in segment s of fiber f) ⇔ g = f ∨ i+1 ≤ segvc[s][g].
 //   Work unit = a warp range: consecutive granules of one elementary interval, all covered by the
-//   same accesses of the window.  Warps own contiguous runs of ranges (coverage-weighted).
+//   same accesses of the window.  Warps take ranges one at a time from a per-launch counter.
 //   Per range:
 //     pass 1  stream the cells in (coalesced 128-bit loads = 2 cells, 8 in flight per lane) and vote
 //             whether they are all equal (skipped in the interval's first window: known empty);

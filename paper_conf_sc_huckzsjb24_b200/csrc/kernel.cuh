@@ -21,7 +21,7 @@ constexpr int CHUNK = 32 * U;           // granules per lane-parallel step
 #endif
 constexpr int UL = CUSAN_UL;            // 16-B loads / stores in flight per lane when streaming
 #ifndef CUSAN_DYNAMIC
-#define CUSAN_DYNAMIC 0
+#define CUSAN_DYNAMIC 1
 #endif
 #ifndef CUSAN_RANGE_PER_ACCESS
 #define CUSAN_RANGE_PER_ACCESS 512
@@ -52,7 +52,10 @@ constexpr size_t DYN_SMEM = CUSAN_TMA ? (size_t)8 * TMA_WARP_BYTES : 0;   // 8 =
 #ifndef CUSAN_RANGE_BAL_MIN
 #define CUSAN_RANGE_BAL_MIN 4096
 #endif
-constexpr int GRAB = 2;                 // ranges a warp takes per dynamic-scheduler grab
+#ifndef CUSAN_GRAB
+#define CUSAN_GRAB 1
+#endif
+constexpr int GRAB = CUSAN_GRAB;        // ranges a warp takes per dynamic-scheduler grab
 constexpr int WARPS = 8;                // warps per block
 constexpr int THREADS = 32 * WARPS;
 constexpr int MAXS = 256;               // shared-memory read set per warp (≥ 255 readers)
@@ -114,7 +117,7 @@ struct Window {
 cudaError_t launch_shadow_check(uint32_t grid, cudaStream_t stream, const DSpan* spans, uint32_t nspans,
                                 uint64_t tiles, uint64_t weight, const Ctx& k, int force_lanes,
                                 unsigned long long* sched);
-// sessions: move untouched intervals' cells to the new layout
+// sessions: copy the cell of a split compressed interval to its new piece
 cudaError_t launch_copy_cells(uint32_t grid, cudaStream_t stream, const uint2* src, uint2* dst,
                               const CopySeg* segs, uint32_t nseg, uint64_t total, uint32_t* heap);
 // resident blocks of K1 per SM (sets K1's dynamic shared memory limit first)
@@ -130,5 +133,15 @@ struct SpanTables {
 };
 void build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& out);
 int device_info(int device, int* max_blocks);
+
+// ---- a4 on the device (merge.cu): raw runs -> canonical runs, downloaded into `out` -------------
+struct RunMerge {                 // scratch, grown on demand and kept for the next call
+    char* buf = nullptr;
+    uint64_t cap = 0;
+    ~RunMerge();
+};
+constexpr int MERGE_LAUNCHES = 4; // own kernels per merge (plus CUB's sort / scan kernels)
+int merge_runs_device(RunMerge& m, cudaStream_t stream, const cusan_race_run* d_runs, uint64_t n,
+                      std::vector<cusan_race_run>& out, uint64_t* d2h_bytes);
 
 }  // namespace cusan

@@ -179,6 +179,7 @@ struct cusan_session {
     uint64_t scratch_cap = 0;
     cusan_race_run* runs = nullptr;
     uint64_t run_cap = 0;
+    RunMerge merge;                                 // a4 scratch (device run merge)
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
 
     ~cusan_session() {
@@ -554,7 +555,11 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
         }
     }
     if ((st = grow_heap(s, s->heap_top + hp.rec_units + (1ull << 16)))) return st;
-    if ((st = ensure(&s->runs, &s->run_cap, std::max<uint64_t>(s->run_cap, 1ull << 20), "run buffer"))) return st;
+    uint64_t tiles = 0;                 // raw-run bound heuristic, as in plans (an overflow truncates)
+    for (const Window& w : tabs.wins) tiles += w.tiles;
+    if ((st = ensure(&s->runs, &s->run_cap, std::max<uint64_t>(std::max<uint64_t>(s->run_cap, 1ull << 20), 2 * tiles + 1024),
+                     "run buffer")))
+        return st;
     const uint64_t seg_words = s->nseg * s->F, up_words = s->seg_uploaded * s->F;
     const uint64_t new_row_bytes = (seg_words - up_words) * sizeof(uint32_t);
     if ((st = grow_keep(s, &s->d_segvc, &s->d_segvc_cap, seg_words, up_words, "segment rows"))) return st;
@@ -621,23 +626,16 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
     s->checked_events = tr.ev.size();
     s->n_calls++;
 
+    s->broken = false;                  // the state is consistent from here on
+
     cusan_report* r = new (std::nothrow) cusan_report;
     if (!r) return fail(CUSAN_ENOMEM, "cannot allocate report");
-    try {
-        r->runs.resize(kept_runs);
-    } catch (...) {
+    uint64_t d2h = N_COUNTERS * sizeof(unsigned long long);
+    const int mst = merge_runs_device(s->merge, s->stream, s->runs, kept_runs, r->runs, &d2h);   // a4
+    if (mst) {
         delete r;
-        return fail(CUSAN_ENOMEM, "cannot allocate report runs");
+        return mst;
     }
-    if (kept_runs) {
-        cudaError_t ce =
-            cudaMemcpy(r->runs.data(), s->runs, kept_runs * sizeof(cusan_race_run), cudaMemcpyDeviceToHost);
-        if (ce != cudaSuccess) {
-            delete r;
-            return cuda_fail(ce, "run download");
-        }
-    }
-    canonicalize_runs(r->runs);
     r->n_runs = r->runs.size();
     r->n_race_granules = cnt[C_RACE];   // exact even when the run list overflowed
     if (runs_ovf) r->truncated = 1;     // the state is committed; the call cannot be re-run
@@ -648,14 +646,13 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
     r->ctr = hp.ctr;
     r->ctr.raw_runs = cnt[C_RUNS];
     r->ctr.kernel_ms = kms;
-    r->ctr.kernel_launches = nwin + (cp.copy_cells ? 1 : 0);
+    r->ctr.kernel_launches = nwin + (cp.copy_cells ? 1 : 0) + (kept_runs ? MERGE_LAUNCHES : 0);
     r->ctr.shadow_cell_bytes = tabs.cell_bytes + 16 * cp.copy_cells;
     r->ctr.shadow_bytes = s->used * sizeof(uint2);
     r->ctr.h2d_bytes = cp.inc.size() * sizeof(AccRec) + tabs.ds.size() * sizeof(DSpan) +
                        cp.segs.size() * sizeof(CopySeg) + new_row_bytes;
-    r->ctr.d2h_bytes = N_COUNTERS * sizeof(unsigned long long) + kept_runs * sizeof(cusan_race_run);
+    r->ctr.d2h_bytes = d2h;
     r->ctr.run_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count();
-    s->broken = false;
     *out = r;
     // a run list that overflowed is sized for the next call (best effort: this call succeeded)
     if (runs_ovf) ensure(&s->runs, &s->run_cap, cnt[C_RUNS] + cnt[C_RUNS] / 8 + 1024, "run buffer");

@@ -221,3 +221,44 @@ def test_interval_compressed_shadow_matches(window):
         tr, _ = lower_product(ops, args)
         ref = oracle.check_events(tr.cusan_trace_read(), 255)
         assert_equal(cs.check(tr, window_events=max(window, 1) * 40, flags=cs.CUSAN_CHECK_INTERVAL_SHADOW), ref)
+
+
+def _events(rows):
+    from tracegen.program import EVENT_DTYPE
+    ev = np.zeros(len(rows), EVENT_DTYPE)
+    for i, (k, m, f, a, b) in enumerate(rows):
+        ev[i]["kind"], ev[i]["mode"], ev[i]["fiber"], ev[i]["a"], ev[i]["b"] = k, m, f, a, b
+    return ev
+
+
+def test_run_buffer_overflow_reruns_exactly():
+    """More raw runs than the first run buffer holds (65536 here): the plan grows it and re-runs;
+    the report is exact.  Closed form: 200 unsynchronised whole-range writes on 200 fibers race pairwise with
+    their predecessor only (each write resets the state), 199 runs of the whole range."""
+    n_gran, n_fib, base = 1 << 21, 200, 1 << 36
+    ev = _events([(EV_ACCESS, 1, f, base, 8 * n_gran) for f in range(n_fib)])
+    tr = cs.Trace(255)
+    tr.cusan_trace_append_events(ev)
+    p = cs.Plan(tr, window_events=50)         # 4 windows, 512 ranges each, 50 racing pairs per range
+    rep = p.run()
+    assert rep.counters["raw_runs"] > (1 << 16)                 # beyond the initial buffer
+    assert rep.n_race_granules == (n_fib - 1) * n_gran
+    assert rep.n_runs == n_fib - 1
+    want = [(base >> 3, (base >> 3) + n_gran, e, e + 1) for e in range(n_fib - 1)]
+    assert [tuple(int(x) for x in r) for r in rep.runs] == want
+    rep2 = p.run()                                              # the grown buffer is kept
+    assert np.array_equal(rep2.runs, rep.runs)
+    p.close()
+
+
+def test_heap_overflow_reruns_exactly():
+    """Lane path with three readers per granule: the second reader of every granule allocates a
+    record, more than the plan's initial heap room; the plan grows the heap and re-runs.  A final
+    unsynchronised write races with each read: 3 runs of the whole range."""
+    n_gran, base = 1 << 17, 1 << 36
+    rows = [(EV_ACCESS, 0, f, base, 8 * n_gran) for f in (0, 1, 2)] + [(EV_ACCESS, 1, 3, base, 8 * n_gran)]
+    tr = cs.Trace(8)
+    tr.cusan_trace_append_events(_events(rows))
+    rep = cs.check(tr, flags=cs.CUSAN_CHECK_FORCE_LANES, window_events=1)
+    assert rep.n_race_granules == 3 * n_gran
+    assert [tuple(int(x) for x in r) for r in rep.runs] == [(base >> 3, (base >> 3) + n_gran, e, 3) for e in range(3)]

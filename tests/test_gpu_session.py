@@ -100,3 +100,41 @@ def test_session_interval_compressed():
         ev = fuzz.random_primitive_trace(rng, n, nf, n_keys=3, n_granules=int(rng.integers(1, 900)))
         cuts = sorted(int(x) for x in rng.integers(1, n, size=int(rng.integers(1, 6))))
         _run_session(ev, nf, cuts, window_events=int(rng.integers(0, 4)), flags=cs.CUSAN_CHECK_INTERVAL_SHADOW)
+
+
+def test_session_compressed_shared_records_across_splits():
+    """f3 sessions: a split compressed interval copies its cell; a read-set record it names becomes
+    shared, so an update through either cell must not show through the other."""
+    rng = np.random.default_rng(91)
+    for _ in range(15):
+        nf = int(rng.integers(6, 30))
+        ev = fuzz.random_primitive_trace(rng, int(rng.integers(40, 200)), nf, n_keys=3,
+                                         n_granules=int(rng.integers(20, 400)), p_access=0.85)
+        acc = ev["kind"] == EV_ACCESS
+        ev["mode"][acc & (rng.random(len(ev)) < 0.8)] = 0
+        cuts = sorted(set(int(x) for x in rng.integers(1, len(ev), size=10)))
+        for flags in (0, cs.CUSAN_CHECK_FORCE_LANES):
+            _run_session(ev, nf, cuts, flags=flags | cs.CUSAN_CHECK_INTERVAL_SHADOW)
+
+
+def test_session_shadow_growth_many_calls():
+    """Every call touches new memory, so the shadow grows (new mapped chunks) call after call;
+    the cells of the first call survive every growth."""
+    from tracegen.program import EVENT_DTYPE, EV_RELEASE, EV_ACQUIRE
+    rows = []
+    base, size = 1 << 32, 1 << 20                      # 1 MiB = 131072 granules per call
+    n_calls = 40
+    order = [c for c in range(n_calls) if c % 2 == 0] + [c for c in range(n_calls) if c % 2]
+    for i, c in enumerate(order):                      # fiber 0 writes region c; the even ones
+        if i == n_calls // 2:                          # before its release
+            rows.append((EV_RELEASE, 0, 0, 7, 0))
+        rows.append((EV_ACCESS, 1, 0, base + c * 3 * size, size))
+    rows.append((EV_ACQUIRE, 0, 1, 7, 0))
+    for c in range(n_calls):                           # fiber 1 reads part of every region: the
+        rows.append((EV_ACCESS, 0, 1, base + c * 3 * size + 8 * c, size // 2))   # odd ones race
+    ev = np.zeros(len(rows), EVENT_DTYPE)
+    for i, (k, m, f, a, b) in enumerate(rows):
+        ev[i]["kind"], ev[i]["mode"], ev[i]["fiber"], ev[i]["a"], ev[i]["b"] = k, m, f, a, b
+    cuts = list(range(1, n_calls)) + [n_calls + 2 + 5 * i for i in range(8)]
+    ref = _run_session(ev, 2, cuts)
+    assert ref["n_race_granules"] == (n_calls // 2) * (size // 2) // 8

@@ -29,11 +29,16 @@ for _ in range(10):
     nf = int(rng.integers(5, 30))
     ev = fuzz.random_primitive_trace(rng, 120, nf, n_keys=3, n_granules=600, p_access=0.8)
     ev["mode"][(ev["kind"] == 0) & (rng.random(len(ev)) < 0.7)] = 0
-    tr = cs.Trace(nf)
-    ses = cs.Session(tr, window_events=7)
-    for a, b in ((0, 40), (40, 90), (90, 120)):
-        tr.cusan_trace_append_events(ev[a:b])
-        ses.check()
-        n += 1
-    ses.close()
+    ref = oracle.check_events(ev, nf)
+    for flags in (0, cs.CUSAN_CHECK_FORCE_LANES, cs.CUSAN_CHECK_INTERVAL_SHADOW,
+                  cs.CUSAN_CHECK_INTERVAL_SHADOW | cs.CUSAN_CHECK_FORCE_LANES):
+        tr = cs.Trace(nf)
+        ses = cs.Session(tr, window_events=7, flags=flags)
+        total = 0
+        for a, b in ((0, 40), (40, 90), (90, 120)):
+            tr.cusan_trace_append_events(ev[a:b])
+            total += ses.check().n_race_granules
+            n += 1
+        ses.close()
+        assert total == ref["n_race_granules"], flags
 print("sanitize workloads ok:", n)
