@@ -2,8 +2,9 @@
 """bench.py — race-checked GB/s of the B200 happens-before race check (DESIGN.md §"Measurement").
 
 One step = one pass of the whole hot path over the workload: the shadow-check kernels (a3) with
-in-warp run compaction (a4), the run download, the canonical merge and the report (a5), with the
-event / clock / interval tables (a1, a2) already resident in HBM.  `e2e` repeats the metric
+in-warp run compaction, the device merge into canonical runs (a4), their download and the report
+(a5), with the event / clock / interval tables (a1, a2) already resident in HBM.  Extra keys, for
+context only: `postmortem` (one window) and `interval_compressed` (f3: one cell per interval).  `e2e` repeats the metric
 through the public C ABI from host buffers: lowering of the recorded CUDA/MPI call program (a0),
 planning (a1, a2), table upload, check and report, every step.
 
@@ -281,7 +282,7 @@ def run_ours(args):
     cell_bytes = ctr["shadow_cell_bytes"]
     peak, peak_src = measured_peaks()
     achieved = cell_bytes / (k_ms / 1e3) / 1e9 if k_ms > 0 else 0.0
-    nl = max(1, int(ctr["kernel_launches"]))
+    nl = max(1, int(ctr["n_windows"]))                  # K1 launches per step (one per window)
     traffic, _ = ncu_traffic()
 
     # ---- e2e: public C ABI from host buffers, every step: lower + plan + upload + check + report ----
@@ -321,6 +322,22 @@ def run_ours(args):
               "kernel_ms": r3.counters["kernel_ms"], "window_events": "all (one window)"}
         p3.close()
 
+    # ---- interval-compressed shadow (f3, extra, for context): same windows, one cell per interval --
+    ic = None
+    if world == 1:
+        p4 = cs.Plan(tr, window_events=args.window, device=local, stream=stream.cuda_stream, workspace="torch",
+                     flags=cs.CUSAN_CHECK_INTERVAL_SHADOW)
+        p4.run()
+        torch.cuda.synchronize(dev)
+        t0 = time.perf_counter()
+        r4 = p4.run()
+        ic_s = time.perf_counter() - t0
+        assert r4.n_race_granules == final.n_race_granules and np.array_equal(r4.runs, final.runs)
+        ic = {"value": tracked / ic_s / 1e9, "unit": "GB/s", "ms_per_step": ic_s * 1e3,
+              "kernel_ms": r4.counters["kernel_ms"], "shadow_bytes": int(r4.counters["shadow_bytes"]),
+              "window_events": args.window}
+        p4.close()
+
     if rank != 0:
         if world > 1:
             dist.destroy_process_group()
@@ -356,6 +373,7 @@ def run_ours(args):
         "gpu_launches": launches,
         "clocks": clk,
         "postmortem": pm,
+        "interval_compressed": ic,
     }
     print(json.dumps(line), flush=True)
     if world > 1:

@@ -35,7 +35,8 @@ struct cusan_plan {
     uint64_t run_cap = 0;
     bool need_shadow = false;
     bool bound = false;                     // workspace carved and tables uploaded
-    uint64_t o_inc = 0, o_seg = 0, o_spans = 0, o_cnt = 0, o_heap = 0, o_shadow = 0, o_runs = 0;
+    uint64_t o_inc = 0, o_seg = 0, o_spans = 0, o_cnt = 0, o_heap = 0, o_shadow = 0, o_runs = 0, o_merge = 0;
+    uint64_t merge_bytes = 0;
     std::vector<DSpan> ds;                  // device span tables (host copy, uploaded at bind)
     std::vector<Window> wins;
     uint64_t shadow_cell_bytes = 0;
@@ -168,6 +169,10 @@ static int plan_device_setup(cusan_plan* p) {
     for (const Window& w : p->wins) tiles += w.tiles;
     p->run_cap = std::min<uint64_t>(std::max<uint64_t>(1ull << 16, 2 * tiles + 4 * p->wins.size() + 1024), 1ull << 24);
     const uint64_t o_runs = off;    off = align_up(off + p->run_cap * sizeof(cusan_race_run));
+    // a4 scratch for merging up to run_cap raw runs (no allocation per run)
+    const int mst = merge_scratch_bytes(p->run_cap, &p->merge_bytes);
+    if (mst) return mst;
+    const uint64_t o_merge = off;   off = align_up(off + p->merge_bytes);
     p->ws_bytes = off;
     p->o_inc = o_inc;
     p->o_seg = o_seg;
@@ -176,6 +181,7 @@ static int plan_device_setup(cusan_plan* p) {
     p->o_heap = o_heap;
     p->o_shadow = o_shadow;
     p->o_runs = o_runs;
+    p->o_merge = o_merge;
     p->ds = std::move(ds);
     p->table_bytes = hp.inc.size() * sizeof(AccRec) + hp.segvc.size() * sizeof(uint32_t) +
                      p->ds.size() * sizeof(DSpan);
@@ -203,6 +209,10 @@ static int plan_bind(cusan_plan* p, char* ws, uint64_t bytes) {
     p->d_counters = (unsigned long long*)(p->ws + p->o_cnt);
     p->d_shadow = p->need_shadow ? (uint2*)(p->ws + p->o_shadow) : nullptr;
     if (!p->d_runs_own) p->d_runs = (cusan_race_run*)(p->ws + p->o_runs);
+    if (!p->merge.own) {
+        p->merge.buf = p->ws + p->o_merge;
+        p->merge.cap = p->merge_bytes;
+    }
     if (!p->d_heap_own) p->d_heap = (uint32_t*)(p->ws + p->o_heap);
     else p->d_heap = p->d_heap_own;
     CK(cudaMemcpyAsync(p->d_inc, hp.inc.data(), hp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, p->stream));

@@ -135,11 +135,13 @@ void build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& out);
 int device_info(int device, int* max_blocks);
 
 // ---- a4 on the device (merge.cu): raw runs -> canonical runs, downloaded into `out` -------------
-struct RunMerge {                 // scratch, grown on demand and kept for the next call
+struct RunMerge {                 // scratch: the caller's (plan workspace) or own, grown on demand
     char* buf = nullptr;
     uint64_t cap = 0;
+    bool own = false;
     ~RunMerge();
 };
+int merge_scratch_bytes(uint64_t n, uint64_t* bytes);   // scratch for merging n raw runs
 constexpr int MERGE_LAUNCHES = 4; // own kernels per merge (plus CUB's sort / scan kernels)
 int merge_runs_device(RunMerge& m, cudaStream_t stream, const cusan_race_run* d_runs, uint64_t n,
                       std::vector<cusan_race_run>& out, uint64_t* d2h_bytes);

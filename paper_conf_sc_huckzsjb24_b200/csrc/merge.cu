@@ -61,12 +61,48 @@ __global__ void run_scatter(const cusan_race_run* __restrict__ runs, const uint3
 
 inline uint64_t up(uint64_t x) { return (x + 255) & ~255ull; }
 
+struct Layout {
+    uint64_t o_ka, o_kb, o_ia, o_ib, o_hd, o_sg, o_out, o_cnt, o_tmp, total;
+    size_t temp;
+};
+
+int layout(uint32_t n, cudaStream_t stream, Layout& L) {
+    using cusan::cuda_fail;
+    // temp storage of the three CUB calls (sizes depend only on n)
+    size_t t1 = 0, t2 = 0, t3 = 0;
+    CK(cub::DeviceRadixSort::SortPairs(nullptr, t1, (const uint64_t*)nullptr, (uint64_t*)nullptr,
+                                       (const uint32_t*)nullptr, (uint32_t*)nullptr, (int)n, 0, 64, stream));
+    CK(cub::DeviceRadixSort::SortPairs(nullptr, t2, (const uint64_t*)nullptr, (uint64_t*)nullptr,
+                                       (const uint32_t*)nullptr, (uint32_t*)nullptr, (int)n, 0, 48, stream));
+    CK(cub::DeviceScan::InclusiveSum(nullptr, t3, (const uint32_t*)nullptr, (uint32_t*)nullptr, (int)n, stream));
+    L.temp = std::max(t1, std::max(t2, t3));
+    L.o_ka = 0;
+    L.o_kb = L.o_ka + up(8ull * n);
+    L.o_ia = L.o_kb + up(8ull * n);
+    L.o_ib = L.o_ia + up(4ull * n);
+    L.o_hd = L.o_ib + up(4ull * n);
+    L.o_sg = L.o_hd + up(4ull * n);
+    L.o_out = L.o_sg + up(4ull * n);
+    L.o_cnt = L.o_out + up(sizeof(cusan_race_run) * n);
+    L.o_tmp = L.o_cnt + 256;
+    L.total = L.o_tmp + up(L.temp);
+    return CUSAN_OK;
+}
+
 }  // namespace
 
 namespace cusan {
 
 RunMerge::~RunMerge() {
-    if (buf) cudaFree(buf);
+    if (own && buf) cudaFree(buf);
+}
+
+int merge_scratch_bytes(uint64_t n, uint64_t* bytes) {
+    if (n >= (1ull << 31)) return fail(CUSAN_ENOMEM, "more than 2^31 raw race runs");
+    Layout L;
+    const int st = layout((uint32_t)std::max<uint64_t>(n, 1), nullptr, L);
+    if (!st) *bytes = L.total;
+    return st;
 }
 
 int merge_runs_device(RunMerge& m, cudaStream_t stream, const cusan_race_run* d_runs, uint64_t n64,
@@ -75,35 +111,29 @@ int merge_runs_device(RunMerge& m, cudaStream_t stream, const cusan_race_run* d_
     if (n64 == 0) return CUSAN_OK;
     if (n64 >= (1ull << 31)) return fail(CUSAN_ENOMEM, "more than 2^31 raw race runs");
     const uint32_t n = (uint32_t)n64;
-    // temp storage of the three CUB calls (sizes depend only on n)
-    size_t t1 = 0, t2 = 0, t3 = 0;
-    CK(cub::DeviceRadixSort::SortPairs(nullptr, t1, (const uint64_t*)nullptr, (uint64_t*)nullptr,
-                                       (const uint32_t*)nullptr, (uint32_t*)nullptr, (int)n, 0, 64, stream));
-    CK(cub::DeviceRadixSort::SortPairs(nullptr, t2, (const uint64_t*)nullptr, (uint64_t*)nullptr,
-                                       (const uint32_t*)nullptr, (uint32_t*)nullptr, (int)n, 0, 48, stream));
-    CK(cub::DeviceScan::InclusiveSum(nullptr, t3, (const uint32_t*)nullptr, (uint32_t*)nullptr, (int)n, stream));
-    const size_t temp = std::max(t1, std::max(t2, t3));
-    const uint64_t o_ka = 0, o_kb = o_ka + up(8ull * n), o_ia = o_kb + up(8ull * n), o_ib = o_ia + up(4ull * n);
-    const uint64_t o_hd = o_ib + up(4ull * n), o_sg = o_hd + up(4ull * n), o_out = o_sg + up(4ull * n);
-    const uint64_t o_cnt = o_out + up(sizeof(cusan_race_run) * n), o_tmp = o_cnt + 256, total = o_tmp + up(temp);
-    if (m.cap < total) {
-        if (m.buf) cudaFree(m.buf);
+    Layout L;
+    int st = layout(n, stream, L);
+    if (st) return st;
+    if (m.cap < L.total) {              // the caller's scratch is too small: own, grown buffer
+        if (m.own && m.buf) cudaFree(m.buf);
         m.buf = nullptr;
         m.cap = 0;
-        const uint64_t want = total + total / 4;
+        m.own = true;
+        const uint64_t want = L.total + L.total / 4;
         if (cudaMalloc((void**)&m.buf, want) != cudaSuccess) return fail(CUSAN_ENOMEM, "cannot allocate run merge buffers");
         m.cap = want;
     }
     char* b = m.buf;
-    uint64_t* ka = (uint64_t*)(b + o_ka);
-    uint64_t* kb = (uint64_t*)(b + o_kb);
-    uint32_t* ia = (uint32_t*)(b + o_ia);
-    uint32_t* ib = (uint32_t*)(b + o_ib);
-    uint32_t* hd = (uint32_t*)(b + o_hd);
-    uint32_t* sg = (uint32_t*)(b + o_sg);
-    cusan_race_run* d_out = (cusan_race_run*)(b + o_out);
-    unsigned long long* d_cnt = (unsigned long long*)(b + o_cnt);
-    void* tmp = b + o_tmp;
+    uint64_t* ka = (uint64_t*)(b + L.o_ka);
+    uint64_t* kb = (uint64_t*)(b + L.o_kb);
+    uint32_t* ia = (uint32_t*)(b + L.o_ia);
+    uint32_t* ib = (uint32_t*)(b + L.o_ib);
+    uint32_t* hd = (uint32_t*)(b + L.o_hd);
+    uint32_t* sg = (uint32_t*)(b + L.o_sg);
+    cusan_race_run* d_out = (cusan_race_run*)(b + L.o_out);
+    unsigned long long* d_cnt = (unsigned long long*)(b + L.o_cnt);
+    void* tmp = b + L.o_tmp;
+    const size_t temp = L.temp;
     size_t tb = temp;
     const uint32_t grid = (n + MT - 1) / MT;
     keys_by_begin<<<grid, MT, 0, stream>>>(d_runs, n, ka, ia);

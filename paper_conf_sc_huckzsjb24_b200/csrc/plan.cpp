@@ -19,6 +19,13 @@
 //     a window's spans are its incidences grouped by interval.
 #include <algorithm>
 #include <bitset>
+#include <chrono>
+#include <condition_variable>
+#include <cstdio>
+#include <cstdlib>
+#include <functional>
+#include <future>
+#include <mutex>
 #include <thread>
 #include <unordered_map>
 
@@ -33,10 +40,76 @@ static unsigned plan_threads(uint64_t work) {
     return std::min<unsigned>(hw, 16);
 }
 
+// A persistent pool of planning threads (created on first use, never torn down): a parallel loop
+// costs a wake-up instead of thread creation.  One loop at a time; a concurrent caller (another host
+// thread planning) falls back to its own threads.
+class Pool {
+  public:
+    explicit Pool(unsigned workers) {
+        for (unsigned i = 0; i < workers; i++) th_.emplace_back([this] { loop(); });
+    }
+    unsigned size() const { return (unsigned)th_.size() + 1; }
+    std::mutex busy;                                // held by the caller for a whole loop
+    void run(unsigned T, const std::function<void(unsigned)>& fn) {
+        {
+            std::lock_guard<std::mutex> lk(m_);
+            job_ = &fn;
+            njobs_ = T;
+            next_ = 1;
+            pending_ = T - 1;
+            gen_++;
+        }
+        cv_.notify_all();
+        fn(0u);
+        std::unique_lock<std::mutex> lk(m_);
+        done_.wait(lk, [&] { return pending_ == 0; });
+        job_ = nullptr;
+    }
+
+  private:
+    void loop() {
+        uint64_t seen = 0;
+        std::unique_lock<std::mutex> lk(m_);
+        for (;;) {
+            cv_.wait(lk, [&] { return gen_ != seen; });
+            seen = gen_;
+            while (job_ && next_ < njobs_) {
+                const unsigned t = next_++;
+                const std::function<void(unsigned)>* f = job_;
+                lk.unlock();
+                (*f)(t);
+                lk.lock();
+                if (--pending_ == 0) done_.notify_one();
+            }
+        }
+    }
+    std::vector<std::thread> th_;
+    std::mutex m_;
+    std::condition_variable cv_, done_;
+    const std::function<void(unsigned)>* job_ = nullptr;
+    unsigned njobs_ = 0, next_ = 0, pending_ = 0;
+    uint64_t gen_ = 0;
+};
+
+static Pool& pool() {
+    static Pool* p = new Pool(std::min<unsigned>(std::max(1u, std::thread::hardware_concurrency()), 16) - 1);
+    return *p;
+}
+
 template <class Fn>
 static void parallel_for(unsigned T, Fn&& fn) {
+    if (T <= 1) {
+        fn(0u);
+        return;
+    }
+    Pool& P = pool();
+    std::unique_lock<std::mutex> lk(P.busy, std::try_to_lock);
+    if (lk && T <= P.size()) {
+        P.run(T, std::function<void(unsigned)>(fn));
+        return;
+    }
     std::vector<std::thread> th;
-    th.reserve(T ? T - 1 : 0);
+    th.reserve(T - 1);
     for (unsigned t = 1; t < T; t++) th.emplace_back(fn, t);
     fn(0u);
     for (auto& x : th) x.join();
@@ -48,96 +121,131 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
         return fail(CUSAN_EINVAL, "need 0 <= shard < nshards");
     if (o.window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
     hp.opts = o;
-    // clock width = fibers the trace actually uses (≤ max_fibers)
+    const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
+    auto tick = [t0 = std::chrono::steady_clock::now(), dbg](const char* what) {
+        if (dbg)
+            std::fprintf(stderr, "build_host_plan: %-12s %8.3f ms\n", what,
+                         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+    };
+    // clock width = fibers the trace actually uses (≤ max_fibers); the accesses' granule ranges
     uint32_t F = 1;
+    uint64_t n_acc = 0;
     for (const auto& e : t.ev) {
         F = std::max<uint32_t>(F, e.fiber + 1);
         if (e.kind == CUSAN_EV_FORK) F = std::max<uint32_t>(F, (uint32_t)e.a + 1);
+        n_acc += e.kind == CUSAN_EV_ACCESS;
     }
     hp.F = F;
     cusan_counters& c = hp.ctr;
     c = cusan_counters{};
     c.n_events = t.ev.size();
     c.n_fibers = F;
-
-    // ---------------------------------------------------------------- a1: clocks and segments --
-    std::vector<uint32_t> C((size_t)F * F, 0);
-    std::unordered_map<uint64_t, uint32_t> key_slot;
-    std::vector<uint32_t> sc;                       // sync clocks, F entries per key
-    const uint32_t NO_SEG = 0xffffffffu;
-    std::vector<uint32_t> cur_seg(F, NO_SEG);
-    auto sync_clock = [&](uint64_t key) -> uint32_t* {
-        auto it = key_slot.find(key);
-        if (it == key_slot.end()) {
-            it = key_slot.emplace(key, (uint32_t)(sc.size() / F)).first;
-            sc.resize(sc.size() + F, 0);
-        }
-        return &sc[(size_t)it->second * F];
-    };
-    uint64_t n_acc = 0;
-    for (const auto& e : t.ev) n_acc += e.kind == CUSAN_EV_ACCESS;
-    hp.acc_g0.reserve(n_acc);
-    hp.acc_g1.reserve(n_acc);
-    hp.acc_event.reserve(n_acc);
-    hp.acc_rec.reserve(n_acc);
-    for (uint64_t i = 0; i < t.ev.size(); i++) {
-        const cusan_event& e = t.ev[i];
-        const uint32_t f = e.fiber;
-        uint32_t* Cf = &C[(size_t)f * F];
-        if (e.kind == CUSAN_EV_FORK) {              // an event of the source fiber's program order
-            const uint32_t s = (uint32_t)e.a;
-            uint32_t* Cs = &C[(size_t)s * F];
-            Cs[s] = (uint32_t)(i + 1);
-            for (uint32_t g = 0; g < F; g++) Cf[g] = std::max(Cf[g], Cs[g]);
-            cur_seg[f] = NO_SEG;                    // incoming edge opens a segment on dst
-            c.n_fork++;
-            continue;
-        }
-        Cf[f] = (uint32_t)(i + 1);
-        switch (e.kind) {
-            case CUSAN_EV_ACCESS: {
-                if (cur_seg[f] == NO_SEG) {
-                    if (hp.nseg >= 0x7fffffffu) return fail(CUSAN_ERANGE, "too many segments");
-                    cur_seg[f] = (uint32_t)hp.nseg++;
-                    hp.segvc.insert(hp.segvc.end(), Cf, Cf + F);
-                }
-                const uint64_t g0 = e.a >> 3;
-                const uint64_t g1 = e.b ? (e.a + e.b + 7) >> 3 : g0;
-                hp.acc_g0.push_back(g0);
-                hp.acc_g1.push_back(g1);
-                hp.acc_event.push_back((uint32_t)i);
-                hp.acc_rec.push_back({pack_epoch(f, (uint32_t)i), cur_seg[f] | ((uint32_t)e.mode << 31)});
-                const uint64_t bytes = 8 * (g1 - g0);
-                c.n_access++;
-                c.tracked_bytes += bytes;
-                if (e.mode) { c.n_write++; c.bytes_written += bytes; }
-                else { c.n_read++; c.bytes_read += bytes; }
-                break;
-            }
-            case CUSAN_EV_RELEASE: {                // SC_k := SC_k ⊔ C_f
-                uint32_t* S = sync_clock(e.a);
-                for (uint32_t g = 0; g < F; g++) S[g] = std::max(S[g], Cf[g]);
-                c.n_release++;
-                break;
-            }
-            case CUSAN_EV_RELEASE_STORE: {          // SC_k := C_f
-                uint32_t* S = sync_clock(e.a);
-                std::copy(Cf, Cf + F, S);
-                c.n_release_store++;
-                break;
-            }
-            case CUSAN_EV_ACQUIRE: {                // C_f := C_f ⊔ SC_k
-                uint32_t* S = sync_clock(e.a);
-                for (uint32_t g = 0; g < F; g++) Cf[g] = std::max(Cf[g], S[g]);
-                cur_seg[f] = NO_SEG;
-                c.n_acquire++;
-                break;
-            }
-            default:
-                return fail(CUSAN_EINVAL, "bad event kind in trace");
+    hp.acc_g0.resize(n_acc);
+    hp.acc_g1.resize(n_acc);
+    hp.acc_event.resize(n_acc);
+    hp.acc_rec.resize(n_acc);
+    {
+        uint64_t k = 0;
+        for (uint64_t i = 0; i < t.ev.size(); i++) {
+            const cusan_event& e = t.ev[i];
+            if (e.kind != CUSAN_EV_ACCESS) continue;
+            hp.acc_g0[k] = e.a >> 3;
+            hp.acc_g1[k] = e.b ? (e.a + e.b + 7) >> 3 : e.a >> 3;
+            hp.acc_event[k] = (uint32_t)i;
+            k++;
         }
     }
-    c.n_segments = hp.nseg;
+
+    // ---------------------------------------------------------------- a1: clocks and segments --
+    // Runs on its own thread while a2 builds the intervals (a2 needs a1's records only to fill the
+    // incidence table at the end).  Errors come back as (status, message).
+    auto a1 = [&]() -> std::pair<int, std::string> {
+        std::vector<uint32_t> C((size_t)F * F, 0);
+        std::unordered_map<uint64_t, uint32_t> key_slot;
+        std::vector<uint32_t> sc;                   // sync clocks, F entries per key
+        const uint32_t NO_SEG = 0xffffffffu;
+        std::vector<uint32_t> cur_seg(F, NO_SEG);
+        auto sync_clock = [&](uint64_t key) -> uint32_t* {
+            auto it = key_slot.find(key);
+            if (it == key_slot.end()) {
+                it = key_slot.emplace(key, (uint32_t)(sc.size() / F)).first;
+                sc.resize(sc.size() + F, 0);
+            }
+            return &sc[(size_t)it->second * F];
+        };
+        uint64_t k = 0;
+        for (uint64_t i = 0; i < t.ev.size(); i++) {
+            const cusan_event& e = t.ev[i];
+            const uint32_t f = e.fiber;
+            uint32_t* Cf = &C[(size_t)f * F];
+            if (e.kind == CUSAN_EV_FORK) {          // an event of the source fiber's program order
+                const uint32_t s = (uint32_t)e.a;
+                uint32_t* Cs = &C[(size_t)s * F];
+                Cs[s] = (uint32_t)(i + 1);
+                for (uint32_t g = 0; g < F; g++) Cf[g] = std::max(Cf[g], Cs[g]);
+                cur_seg[f] = NO_SEG;                // incoming edge opens a segment on dst
+                c.n_fork++;
+                continue;
+            }
+            Cf[f] = (uint32_t)(i + 1);
+            switch (e.kind) {
+                case CUSAN_EV_ACCESS: {
+                    if (cur_seg[f] == NO_SEG) {
+                        if (hp.nseg >= 0x7fffffffu) return {CUSAN_ERANGE, "too many segments"};
+                        cur_seg[f] = (uint32_t)hp.nseg++;
+                        hp.segvc.insert(hp.segvc.end(), Cf, Cf + F);
+                    }
+                    hp.acc_rec[k] = {pack_epoch(f, (uint32_t)i), cur_seg[f] | ((uint32_t)e.mode << 31)};
+                    const uint64_t bytes = 8 * (hp.acc_g1[k] - hp.acc_g0[k]);
+                    k++;
+                    c.n_access++;
+                    c.tracked_bytes += bytes;
+                    if (e.mode) { c.n_write++; c.bytes_written += bytes; }
+                    else { c.n_read++; c.bytes_read += bytes; }
+                    break;
+                }
+                case CUSAN_EV_RELEASE: {            // SC_k := SC_k ⊔ C_f
+                    uint32_t* S = sync_clock(e.a);
+                    for (uint32_t g = 0; g < F; g++) S[g] = std::max(S[g], Cf[g]);
+                    c.n_release++;
+                    break;
+                }
+                case CUSAN_EV_RELEASE_STORE: {      // SC_k := C_f
+                    uint32_t* S = sync_clock(e.a);
+                    std::copy(Cf, Cf + F, S);
+                    c.n_release_store++;
+                    break;
+                }
+                case CUSAN_EV_ACQUIRE: {            // C_f := C_f ⊔ SC_k
+                    uint32_t* S = sync_clock(e.a);
+                    for (uint32_t g = 0; g < F; g++) Cf[g] = std::max(Cf[g], S[g]);
+                    cur_seg[f] = NO_SEG;
+                    c.n_acquire++;
+                    break;
+                }
+                default:
+                    return {CUSAN_EINVAL, "bad event kind in trace"};
+            }
+        }
+        c.n_segments = hp.nseg;
+        return {CUSAN_OK, ""};
+    };
+    const bool concurrent = n_acc >= (1u << 12);
+    std::future<std::pair<int, std::string>> a1_done;
+    std::pair<int, std::string> a1_status{CUSAN_OK, ""};
+    if (concurrent) a1_done = std::async(std::launch::async, a1);
+    else a1_status = a1();
+    // joins a1 (at the latest when the plan is left early)
+    struct Join {
+        std::future<std::pair<int, std::string>>* f;
+        std::pair<int, std::string>* out;
+        ~Join() { if (f->valid()) *out = f->get(); }
+    } a1_join{&a1_done, &a1_status};
+    auto a1_finish = [&]() -> int {
+        if (a1_done.valid()) a1_status = a1_done.get();
+        tick("a1 clocks");
+        return a1_status.first ? fail(a1_status.first, a1_status.second) : CUSAN_OK;
+    };
 
     // ---------------------------------------------------------------- a2: elementary intervals --
     std::vector<uint64_t> B;
@@ -146,16 +254,24 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
         if (hp.acc_g1[k] > hp.acc_g0[k]) { B.push_back(hp.acc_g0[k]); B.push_back(hp.acc_g1[k]); }
     std::sort(B.begin(), B.end());
     B.erase(std::unique(B.begin(), B.end()), B.end());
+    tick("a2 sort");
     const uint64_t nb = B.size();
     std::vector<int64_t> diff(nb + 1, 0);
     std::vector<uint32_t> b0(n_acc), b1(n_acc);
-    for (uint64_t k = 0; k < n_acc; k++) {
-        if (hp.acc_g1[k] <= hp.acc_g0[k]) { b0[k] = b1[k] = 0; continue; }
-        b0[k] = (uint32_t)(std::lower_bound(B.begin(), B.end(), hp.acc_g0[k]) - B.begin());
-        b1[k] = (uint32_t)(std::lower_bound(B.begin(), B.end(), hp.acc_g1[k]) - B.begin());
-        diff[b0[k]]++;
-        diff[b1[k]]--;
+    {
+        const unsigned TB = plan_threads(n_acc * 8);
+        parallel_for(TB, [&](unsigned t) {
+            const uint64_t ka = n_acc * t / TB, kb = n_acc * (t + 1) / TB;
+            for (uint64_t k = ka; k < kb; k++) {
+                if (hp.acc_g1[k] <= hp.acc_g0[k]) { b0[k] = b1[k] = 0; continue; }
+                b0[k] = (uint32_t)(std::lower_bound(B.begin(), B.end(), hp.acc_g0[k]) - B.begin());
+                b1[k] = (uint32_t)(std::lower_bound(B.begin(), B.end(), hp.acc_g1[k]) - B.begin());
+            }
+        });
+        for (uint64_t k = 0; k < n_acc; k++)
+            if (b1[k] > b0[k]) { diff[b0[k]]++; diff[b1[k]]--; }
     }
+    tick("a2 bounds");
     // elementary interval j = [B[j], B[j+1]); covered ones get ids in ascending address order
     std::vector<uint32_t> iv_of(nb ? nb - 1 : 0, 0xffffffffu);
     struct GIv { uint64_t abs_begin, dense_begin, len; uint32_t cnt, off; };
@@ -173,11 +289,18 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
         }
     }
     c.n_intervals = giv.size();
+    tick("a2 intervals");
     // incidences: per interval, covering accesses in trace order (CSR).  Threads take contiguous
     // chunks of accesses; per-chunk counts give every chunk its slots, so the order is the serial one.
-    const unsigned T = plan_threads(n_acc);
+    // Chunks hold equal numbers of incidences (an access covering many intervals is more work).
+    std::vector<uint64_t> wk(n_acc + 1, 0);
+    for (uint64_t k = 0; k < n_acc; k++) wk[k + 1] = wk[k] + (b1[k] - b0[k]);
+    const unsigned T = plan_threads(std::max<uint64_t>(n_acc, wk[n_acc]));
     std::vector<std::vector<uint32_t>> cnt_t(T, std::vector<uint32_t>(giv.size(), 0));
-    auto chunk = [&](unsigned t, uint64_t n) { return std::make_pair(n * t / T, n * (t + 1) / T); };
+    std::vector<uint64_t> cut(T + 1, n_acc);
+    for (unsigned t = 0; t < T; t++)
+        cut[t] = (uint64_t)(std::lower_bound(wk.begin(), wk.end(), wk[n_acc] * t / T) - wk.begin());
+    auto chunk = [&](unsigned t, uint64_t) { return std::make_pair(std::min(cut[t], n_acc), std::min(cut[t + 1], n_acc)); };
     parallel_for(T, [&](unsigned t) {
         auto [ka, kb] = chunk(t, n_acc);
         for (uint64_t k = ka; k < kb; k++)
@@ -204,13 +327,17 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
         auto [ka, kb] = chunk(t, n_acc);
         std::vector<uint32_t>& slot = cnt_t[t];
         for (uint64_t k = ka; k < kb; k++)
-            for (uint32_t j = b0[k]; j < b1[k]; j++) {
-                const uint32_t q = slot[iv_of[j]]++;
-                hp.inc[q] = hp.acc_rec[k];
-                hp.inc_acc[q] = (uint32_t)k;
-            }
+            for (uint32_t j = b0[k]; j < b1[k]; j++) hp.inc_acc[slot[iv_of[j]]++] = (uint32_t)k;
     });
-
+    tick("a2 incidence");
+    if (int st = a1_finish()) return st;                 // a1's records fill the incidence table
+    {
+        const unsigned TI = plan_threads(n_inc);
+        parallel_for(TI, [&](unsigned t) {
+            const uint64_t qa = n_inc * t / TI, qb = n_inc * (t + 1) / TI;
+            for (uint64_t q = qa; q < qb; q++) hp.inc[q] = hp.acc_rec[hp.inc_acc[q]];
+        });
+    }
     // ---------------------------------------------------------------- a2: shard clip ------------
     const uint64_t total_dense = giv.empty() ? 0 : giv.back().dense_begin + giv.back().len;
     uint64_t d_lo = 0, d_hi = total_dense;
@@ -278,6 +405,7 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
     hp.shadow_cells = slot;
     c.shard_granules = hp.shard_granules;
 
+    tick("a2 clip");
     // ---------------------------------------------------------------- windows and spans ---------
     // A span that stores its final cells and ends with two or more reader fibers since the
     // interval's last write gets a pre-assigned read-set record: the cell keeps W inline and its R
@@ -292,10 +420,16 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
     const uint64_t nwin = n_new ? (n_new + W - 1) / W : 0;
     // Threads take contiguous chunks of intervals and emit (window, span) in interval order; a
     // stable counting sort by window then gives the window-major order of the serial loop.
-    const unsigned TS = plan_threads(hp.iv.size() * 8);
+    // Chunks hold equal numbers of incidences.
+    std::vector<uint64_t> wi(hp.iv.size() + 1, 0);
+    for (size_t i = 0; i < hp.iv.size(); i++) wi[i + 1] = wi[i] + hp.iv[i].list_cnt + 1;
+    const unsigned TS = plan_threads(wi.back() * 2);
+    std::vector<size_t> icut(TS + 1, hp.iv.size());
+    for (unsigned t = 0; t < TS; t++)
+        icut[t] = (size_t)(std::lower_bound(wi.begin(), wi.end(), wi.back() * t / TS) - wi.begin());
     std::vector<std::vector<std::pair<uint64_t, Span>>> part(TS);
     parallel_for(TS, [&](unsigned t) {
-        const size_t ia = hp.iv.size() * t / TS, ib = hp.iv.size() * (t + 1) / TS;
+        const size_t ia = std::min(icut[t], hp.iv.size()), ib = std::min(icut[t + 1], hp.iv.size());
         for (size_t i = ia; i < ib; i++) {
             const Interval& v = hp.iv[i];
             std::bitset<CUSAN_MAX_FIBERS + 1> readers;
@@ -358,6 +492,7 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
         if (wstart[w + 1] > wstart[w]) hp.win_span_off.push_back(wstart[w + 1]);   // skip empty windows
     c.n_windows = hp.win_span_off.size() - 1;
     c.n_spans = hp.spans.size();
+    tick("spans");
     return CUSAN_OK;
 }
 
