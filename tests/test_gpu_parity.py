@@ -174,7 +174,11 @@ def test_full_size_configs_sampled(c):
     ops, args = w.arrays(True)
     tr, _ = lower_product(ops, args)
     ev = tr.cusan_trace_read()
-    rep = cs.check(tr)
+    import torch
+    s = torch.cuda.Stream()
+    rep = cs.check(tr, window_events=4096, workspace="torch", stream=s.cuda_stream)   # as bench.py runs it
+    one = cs.check(tr)                                                                # post-mortem: one window
+    assert one.n_race_granules == rep.n_race_granules and np.array_equal(one.runs, rep.runs)
     assert rep.n_race_granules > 0
     assert rep.n_race_granules == int(np.sum(rep.runs["g_end"] - rep.runs["g_begin"]))
     sample = _sample_granules(rep.runs, ev, np.random.default_rng(c))
@@ -262,3 +266,35 @@ def test_heap_overflow_reruns_exactly():
     rep = cs.check(tr, flags=cs.CUSAN_CHECK_FORCE_LANES, window_events=1)
     assert rep.n_race_granules == 3 * n_gran
     assert [tuple(int(x) for x in r) for r in rep.runs] == [(base >> 3, (base >> 3) + n_gran, e, 3) for e in range(3)]
+
+
+def test_largest_event_id_on_the_gpu():
+    """Maximum trace length: the last event id 2^24 - 3 packs as epoch 2^24 - 2 in the
+    24-bit field; it must race with event 0.  Closed form: one run of the range, (0, last)."""
+    from tracegen.program import EV_RELEASE
+    n = (1 << 24) - 2
+    base, n_gran = 1 << 33, 4096
+    ev = np.zeros(n, dtype=_events([]).dtype)
+    ev["kind"] = EV_RELEASE                                   # fiber 0 releases key 0, n-2 times
+    ev[0]["kind"], ev[0]["mode"], ev[0]["a"], ev[0]["b"] = EV_ACCESS, 1, base, 8 * n_gran
+    ev[n - 1]["kind"], ev[n - 1]["mode"], ev[n - 1]["fiber"] = EV_ACCESS, 1, 1
+    ev[n - 1]["a"], ev[n - 1]["b"] = base, 8 * n_gran
+    tr = cs.Trace(2)
+    tr.cusan_trace_append_events(ev)
+    for kw in ({}, {"flags": cs.CUSAN_CHECK_FORCE_LANES}, {"flags": cs.CUSAN_CHECK_INTERVAL_SHADOW}):
+        rep = cs.check(tr, **kw)
+        assert [tuple(int(x) for x in r) for r in rep.runs] == [(base >> 3, (base >> 3) + n_gran, 0, n - 1)]
+
+
+@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_FORCE_LANES], ids=["ranges", "lanes"])
+def test_maximum_fibers_read_set(flags):
+    """255 fibers (the most an epoch encodes) read a range, then fiber 0 writes it: the full read
+    set (254 other readers) lives in a record and every unordered reader races."""
+    base, n_gran = 1 << 34, 1000
+    rows = [(EV_ACCESS, 0, f, base + 8 * (f % 3), 8 * n_gran) for f in range(255)]
+    rows.append((EV_ACCESS, 1, 0, base, 8 * (n_gran + 2)))
+    ev = _events(rows)
+    ref = oracle.check_events(ev, 255)
+    assert ref["n_runs"] >= 254
+    for window in (0, 7):
+        assert_equal(gpu_report(ev, 255, window_events=window, flags=flags), ref)
