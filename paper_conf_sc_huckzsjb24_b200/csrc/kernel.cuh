@@ -142,6 +142,7 @@ struct RunMerge {                 // scratch: the caller's (plan workspace) or o
     ~RunMerge();
 };
 int merge_scratch_bytes(uint64_t n, uint64_t* bytes);   // scratch for merging n raw runs
+int merge_reserve(RunMerge& m, uint64_t n);               // own scratch for n raw runs
 constexpr int MERGE_LAUNCHES = 4; // own kernels per merge (plus CUB's sort / scan kernels)
 int merge_runs_device(RunMerge& m, cudaStream_t stream, const cusan_race_run* d_runs, uint64_t n,
                       std::vector<cusan_race_run>& out, uint64_t* d2h_bytes);

@@ -105,6 +105,19 @@ int merge_scratch_bytes(uint64_t n, uint64_t* bytes) {
     return st;
 }
 
+int merge_reserve(RunMerge& m, uint64_t n) {
+    uint64_t need = 0;
+    if (int st = merge_scratch_bytes(n, &need)) return st;
+    if (m.cap >= need) return CUSAN_OK;
+    if (m.own && m.buf) cudaFree(m.buf);
+    m.buf = nullptr;
+    m.cap = 0;
+    m.own = true;
+    if (cudaMalloc((void**)&m.buf, need) != cudaSuccess) return fail(CUSAN_ENOMEM, "cannot allocate run merge buffers");
+    m.cap = need;
+    return CUSAN_OK;
+}
+
 int merge_runs_device(RunMerge& m, cudaStream_t stream, const cusan_race_run* d_runs, uint64_t n64,
                       std::vector<cusan_race_run>& out, uint64_t* d2h_bytes) {
     out.clear();

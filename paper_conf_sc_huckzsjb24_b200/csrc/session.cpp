@@ -2,6 +2,8 @@
 #include <algorithm>
 #include <bitset>
 #include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -92,11 +94,27 @@ struct VmRange {
     }
 };
 
+// A growable device buffer.  With VMM: a virtual range of `reserve` bytes (0 = the device's memory)
+// whose end gets physical chunks mapped as it grows — the address and contents stay, nothing is
+// copied or freed (cudaMalloc / cudaFree next to a tens-of-GB shadow cost up to 100s of ms).
+// Without: cudaMalloc + copy of the kept prefix.  Contents past the kept prefix are undefined.
+template <class T>
+struct DevBuf {
+    VmRange vr;
+    T* p = nullptr;
+    uint64_t cap = 0;             // elements
+    uint64_t reserve = 0;         // bytes of virtual range
+    bool vm = false;
+    ~DevBuf() {
+        if (!vm && p) cudaFree(p);
+    }
+};
+
 }  // namespace
 
 // make at least `bytes` of the range usable (maps one new chunk with 1/8 headroom); false = not
 // possible (no VMM support, or out of memory)
-static bool vm_grow(VmRange& r, int device, size_t bytes) {
+static bool vm_grow(VmRange& r, int device, size_t bytes, size_t reserve = 0) {
     if (bytes <= r.mapped) return true;
     const Vmm& v = vmm();
     if (!v.ok) return false;
@@ -109,7 +127,7 @@ static bool vm_grow(VmRange& r, int device, size_t bytes) {
         if (v.granularity(&r.gran, &prop, CU_MEM_ALLOC_GRANULARITY_RECOMMENDED) != CUDA_SUCCESS ||
             cudaMemGetInfo(&free_b, &total_b) != cudaSuccess)
             return false;
-        r.reserved = (std::max(total_b, bytes) + r.gran - 1) / r.gran * r.gran;
+        r.reserved = (std::max(reserve ? reserve : total_b, bytes) + r.gran - 1) / r.gran * r.gran;
         if (v.reserve(&r.base, r.reserved, 0, 0, 0) != CUDA_SUCCESS) {
             r.base = 0;
             return false;
@@ -166,31 +184,23 @@ struct cusan_session {
     uint64_t used = 0;                              // cells of `shadow` in use
     uint64_t checked_access = 0, checked_events = 0, n_calls = 0;
     bool broken = false;                            // a call failed after changing the state
-    // ---- device state ----
-    VmRange vm;                                     // the shadow's virtual range (if VMM works)
-    bool vm_shadow = true;
-    uint2* shadow = nullptr;
-    uint64_t shadow_cap = 0;                        // cells
-    uint32_t* d_segvc = nullptr;
-    uint64_t d_segvc_cap = 0, seg_uploaded = 0;     // u32 words / rows on the device
-    uint32_t* heap = nullptr;
-    uint64_t heap_cap = 0, heap_top = 0;            // record units
-    char* scratch = nullptr;
-    uint64_t scratch_cap = 0;
-    cusan_race_run* runs = nullptr;
-    uint64_t run_cap = 0;
-    RunMerge merge;                                 // a4 scratch (device run merge)
+    // ---- device state (every buffer grows in place, see DevBuf) ----
+    DevBuf<uint2> shadow;                           // cells
+    DevBuf<uint32_t> segvc_d;                       // segment rows, u32 words
+    uint64_t seg_uploaded = 0;                      // rows on the device
+    DevBuf<uint32_t> heap;                          // read-set records, u32 words
+    uint64_t heap_top = 0;                          // record units in use
+    DevBuf<char> scratch;                           // one call's tables and counters
+    DevBuf<cusan_race_run> runs;                    // raw runs of one call
+    DevBuf<char> merge_buf;                         // a4 scratch
+    RunMerge merge;                                 // views merge_buf
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
 
     ~cusan_session() {
         if (ev0) cudaEventDestroy(ev0);
         if (ev1) cudaEventDestroy(ev1);
-        if (!vm_shadow) cudaFree(shadow);
-        cudaFree(d_segvc);
-        cudaFree(heap);
-        cudaFree(scratch);
-        cudaFree(runs);
     }
+    uint64_t heap_cap() const { return std::min<uint64_t>(heap.cap / REC_WORDS, (1ull << 24) - 1); }
 
     uint32_t* sync_clock(uint64_t key) {
         auto it = key_slot.find(key);
@@ -202,53 +212,55 @@ struct cusan_session {
     }
 };
 
+// grow a buffer to at least `need` elements keeping the first `keep` (see DevBuf)
 template <class T>
-static int ensure(T** p, uint64_t* cap, uint64_t need, const char* what) {
-    if (*cap >= need && *p) return CUSAN_OK;
-    cudaFree(*p);
-    *p = nullptr;
-    *cap = 0;
-    const uint64_t n = std::max<uint64_t>(need, 1);
-    if (cudaMalloc((void**)p, n * sizeof(T)) != cudaSuccess)
-        return fail(CUSAN_ENOMEM, std::string("cannot allocate ") + what);
-    *cap = n;
-    return CUSAN_OK;
-}
-
-// grow a device buffer keeping its first `keep` elements.  small = doubling and zero-filled (so
-// the copy never moves uninitialised words, e.g. unused tails of records); !small (the shadow,
-// tens of GB) = exactly `need` and not filled: every cell past `keep` is stored before it is read
-template <class T>
-static int grow_keep(cusan_session* s, T** p, uint64_t* cap, uint64_t need, uint64_t keep, const char* what,
-                     bool small = true) {
-    if (*cap >= need && *p) return CUSAN_OK;
-    const uint64_t n = small ? std::max<uint64_t>(std::max<uint64_t>(need, 2 * *cap), 64) : std::max<uint64_t>(need, 64);
+static int grow_buf(cusan_session* s, DevBuf<T>& b, uint64_t need, uint64_t keep, const char* what) {
+    if (b.cap >= need && b.p) return CUSAN_OK;
+    need = std::max<uint64_t>(need, 1);
+    if (b.vm || (!b.p && vmm().ok)) {
+        if (vm_grow(b.vr, s->device, need * sizeof(T), b.reserve)) {
+            b.vm = true;
+            b.p = (T*)b.vr.base;
+            b.cap = b.vr.mapped / sizeof(T);
+            return CUSAN_OK;
+        }
+        if (b.vm) return fail(CUSAN_ENOMEM, std::string("cannot map more device memory for ") + what);
+    }
+    const uint64_t n = std::max<uint64_t>(need + need / 8, 64);
     T* np = nullptr;
     if (cudaMalloc((void**)&np, n * sizeof(T)) != cudaSuccess)
-        return fail(CUSAN_ENOMEM, std::string("cannot grow ") + what);
-    cudaError_t e = small ? cudaMemsetAsync(np, 0, n * sizeof(T), s->stream) : cudaSuccess;
-    if (e == cudaSuccess && *p && keep)
-        e = cudaMemcpyAsync(np, *p, keep * sizeof(T), cudaMemcpyDeviceToDevice, s->stream);
+        return fail(CUSAN_ENOMEM, std::string("cannot allocate ") + what);
+    cudaError_t e = cudaSuccess;
+    if (b.p && keep) e = cudaMemcpyAsync(np, b.p, std::min(keep, b.cap) * sizeof(T), cudaMemcpyDeviceToDevice, s->stream);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s->stream);
     if (e != cudaSuccess) {
         cudaFree(np);
         return cuda_fail(e, what);
     }
-    cudaFree(*p);
-    *p = np;
-    *cap = n;
+    cudaFree(b.p);
+    b.p = np;
+    b.cap = n;
     return CUSAN_OK;
 }
 
 // grow the heap keeping records [0, heap_top)
-static int grow_heap(cusan_session* s, uint64_t need) {
-    if (s->heap_cap >= need && s->heap) return CUSAN_OK;
-    if (need >= (1ull << 24)) return fail(CUSAN_ENOMEM, "read-set heap exceeds the 24-bit record index");
-    uint64_t words = s->heap_cap * REC_WORDS;
-    int st = grow_keep(s, &s->heap, &words, std::min<uint64_t>(need, (1ull << 24) - 1) * REC_WORDS,
-                       s->heap_top * REC_WORDS, "the read-set heap");
-    if (!st) s->heap_cap = std::min<uint64_t>(words / REC_WORDS, (1ull << 24) - 1);
-    return st;
+static int grow_heap(cusan_session* s, uint64_t need_units) {
+    if (s->heap_cap() >= need_units && s->heap.p) return CUSAN_OK;
+    if (need_units >= (1ull << 24)) return fail(CUSAN_ENOMEM, "read-set heap exceeds the 24-bit record index");
+    return grow_buf(s, s->heap, need_units * REC_WORDS, s->heap_top * REC_WORDS, "the read-set heap");
+}
+
+// run buffer for `n` raw runs and the a4 scratch to merge them
+static int grow_runs(cusan_session* s, uint64_t n) {
+    if (int st = grow_buf(s, s->runs, n, 0, "the run buffer")) return st;
+    uint64_t mb = 0;
+    if (int st = merge_scratch_bytes(s->runs.cap, &mb)) return st;
+    if (int st = grow_buf(s, s->merge_buf, mb, 0, "the run merge scratch")) return st;
+    if (!s->merge.own) {
+        s->merge.buf = s->merge_buf.p;
+        s->merge.cap = s->merge_buf.cap;
+    }
+    return CUSAN_OK;
 }
 
 // The incremental host plan of one call (a1 + a2 for the new events).
@@ -508,6 +520,17 @@ int cusan_session_create(const cusan_trace* t, const cusan_check_opts* o, cusan_
         if (cudaEventCreate(&s->ev0) != cudaSuccess || cudaEventCreate(&s->ev1) != cudaSuccess)
             st = fail(CUSAN_ECUDA, "cannot create events");
     }
+    // run buffer and its merge scratch now, while allocation is cheap (before the shadow is mapped)
+    if (!st) {
+        size_t free_b = 0, total_b = 0;
+        cudaMemGetInfo(&free_b, &total_b);
+        s->heap.reserve = (1ull << 24) * REC_WORDS * sizeof(uint32_t);   // the 24-bit record index
+        s->segvc_d.reserve = s->scratch.reserve = total_b / 8;
+        s->runs.reserve = s->merge_buf.reserve = total_b / 16;
+        st = grow_runs(s, 1ull << 20);
+    }
+    if (!st) st = grow_heap(s, 1ull << 16);
+    if (!st) st = grow_buf(s, s->scratch, 16ull << 20, 0, "plan tables");
     if (st) {
         delete s;
         return st;
@@ -520,6 +543,12 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
     if (!s || !out) return fail(CUSAN_EINVAL, "null argument");
     *out = nullptr;
     const auto t_start = std::chrono::steady_clock::now();
+    const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
+    auto tick = [&](const char* what) {
+        if (dbg)
+            std::fprintf(stderr, "cusan_session_check: %-10s %8.3f ms\n", what,
+                         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count());
+    };
     CK(cudaSetDevice(s->device));
     const Trace& tr = s->trace->t;
     if (tr.ev.size() < s->checked_events) return fail(CUSAN_ESTATE, "the trace shrank");
@@ -537,34 +566,23 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
     if (st) return st;
     HostPlan& hp = cp.hp;
     SpanTables tabs;
+    tick("plan");
     build_span_tables(hp, s->max_blocks, tabs);
+    tick("tables");
 
     // ---- device memory ---------------------------------------------------------------------------
     // the shadow grows as new memory is touched: new chunks mapped in place, else re-allocated
     // with its cells moved (1/8 headroom either way)
-    if (cp.used > s->shadow_cap) {
-        if (s->vm_shadow && vm_grow(s->vm, s->device, cp.used * sizeof(uint2))) {
-            s->shadow = (uint2*)s->vm.base;
-            s->shadow_cap = s->vm.mapped / sizeof(uint2);
-        } else {
-            if (s->vm_shadow && s->vm.mapped)
-                return fail(CUSAN_ENOMEM, "cannot map more shadow memory");
-            s->vm_shadow = false;
-            if ((st = grow_keep(s, &s->shadow, &s->shadow_cap, cp.used + cp.used / 8, s->used, "shadow", false)))
-                return st;
-        }
-    }
+    if ((st = grow_buf(s, s->shadow, cp.used, s->used, "the shadow"))) return st;
     if ((st = grow_heap(s, s->heap_top + hp.rec_units + (1ull << 16)))) return st;
     uint64_t tiles = 0;                 // raw-run bound heuristic, as in plans (an overflow truncates)
     for (const Window& w : tabs.wins) tiles += w.tiles;
-    if ((st = ensure(&s->runs, &s->run_cap, std::max<uint64_t>(std::max<uint64_t>(s->run_cap, 1ull << 20), 2 * tiles + 1024),
-                     "run buffer")))
-        return st;
+    if ((st = grow_runs(s, 2 * tiles + 1024))) return st;
     const uint64_t seg_words = s->nseg * s->F, up_words = s->seg_uploaded * s->F;
     const uint64_t new_row_bytes = (seg_words - up_words) * sizeof(uint32_t);
-    if ((st = grow_keep(s, &s->d_segvc, &s->d_segvc_cap, seg_words, up_words, "segment rows"))) return st;
+    if ((st = grow_buf(s, s->segvc_d, seg_words, up_words, "segment rows"))) return st;
     if (seg_words > up_words)                        // only the rows new since the last call
-        CK(cudaMemcpyAsync(s->d_segvc + up_words, s->segvc.data() + up_words,
+        CK(cudaMemcpyAsync(s->segvc_d.p + up_words, s->segvc.data() + up_words,
                            (seg_words - up_words) * sizeof(uint32_t), cudaMemcpyHostToDevice, s->stream));
     const uint64_t nwin = tabs.wins.size();
     uint64_t off = 0;
@@ -572,14 +590,15 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
     const uint64_t o_spans = off; off = align_up(off + tabs.ds.size() * sizeof(DSpan));
     const uint64_t o_copy = off;  off = align_up(off + cp.segs.size() * sizeof(CopySeg));
     const uint64_t o_cnt = off;   off = align_up(off + (N_COUNTERS + nwin) * sizeof(unsigned long long));
-    if ((st = ensure(&s->scratch, &s->scratch_cap, off, "plan tables"))) return st;
-    AccRec* d_inc = (AccRec*)(s->scratch + o_inc);
-    DSpan* d_spans = (DSpan*)(s->scratch + o_spans);
-    CopySeg* d_copy = (CopySeg*)(s->scratch + o_copy);
-    unsigned long long* d_cnt = (unsigned long long*)(s->scratch + o_cnt);
+    if ((st = grow_buf(s, s->scratch, off, 0, "plan tables"))) return st;
+    AccRec* d_inc = (AccRec*)(s->scratch.p + o_inc);
+    DSpan* d_spans = (DSpan*)(s->scratch.p + o_spans);
+    CopySeg* d_copy = (CopySeg*)(s->scratch.p + o_copy);
+    unsigned long long* d_cnt = (unsigned long long*)(s->scratch.p + o_cnt);
     CK(cudaMemcpyAsync(d_inc, cp.inc.data(), cp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, s->stream));
     CK(cudaMemcpyAsync(d_spans, tabs.ds.data(), tabs.ds.size() * sizeof(DSpan), cudaMemcpyHostToDevice, s->stream));
     CK(cudaMemcpyAsync(d_copy, cp.segs.data(), cp.segs.size() * sizeof(CopySeg), cudaMemcpyHostToDevice, s->stream));
+    tick("memory");
 
     // ---- a3 / a4, in place ------------------------------------------------------------------------
     std::vector<unsigned long long> init(N_COUNTERS + nwin, 0ull), cnt(N_COUNTERS, 0ull);
@@ -588,18 +607,18 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
                        s->stream));
     CK(cudaEventRecord(s->ev0, s->stream));
     if (cp.copy_cells)
-        CK(launch_copy_cells(s->max_blocks, s->stream, s->shadow, s->shadow, d_copy, (uint32_t)cp.segs.size(),
-                             cp.copy_cells, s->heap));
+        CK(launch_copy_cells(s->max_blocks, s->stream, s->shadow.p, s->shadow.p, d_copy, (uint32_t)cp.segs.size(),
+                             cp.copy_cells, s->heap.p));
     Ctx k;
     k.inc = d_inc;
-    k.segvc = s->d_segvc;
+    k.segvc = s->segvc_d.p;
     k.F = s->F;
-    k.shadow = s->shadow;
-    k.heap = s->heap;
-    k.heap_cap = s->heap_cap;
-    k.runs = s->runs;
+    k.shadow = s->shadow.p;
+    k.heap = s->heap.p;
+    k.heap_cap = s->heap_cap();
+    k.runs = s->runs.p;
     k.counters = d_cnt;
-    k.run_cap = s->run_cap;
+    k.run_cap = s->runs.cap;
     const int force_lanes = (s->opts.flags & CUSAN_CHECK_FORCE_LANES) ? 1 : 0;
     for (size_t i = 0; i < nwin; i++) {
         const Window& w = tabs.wins[i];
@@ -611,11 +630,12 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
     CK(cudaMemcpyAsync(cnt.data(), d_cnt, N_COUNTERS * sizeof(unsigned long long), cudaMemcpyDeviceToHost,
                        s->stream));
     CK(cudaStreamSynchronize(s->stream));
+    tick("check");
     float kms = 0.f;
     CK(cudaEventElapsedTime(&kms, s->ev0, s->ev1));
     if (cnt[C_HEAP_OVF]) return fail(CUSAN_ENOMEM, "read-set heap overflow: the session's state is lost");
-    const bool runs_ovf = cnt[C_RUNS] > s->run_cap;
-    const uint64_t kept_runs = std::min<uint64_t>(cnt[C_RUNS], s->run_cap);
+    const bool runs_ovf = cnt[C_RUNS] > s->runs.cap;
+    const uint64_t kept_runs = std::min<uint64_t>(cnt[C_RUNS], s->runs.cap);
 
     // ---- commit: the new layout becomes the session's ---------------------------------------------
     s->ivs.swap(cp.ivs);
@@ -631,7 +651,8 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
     cusan_report* r = new (std::nothrow) cusan_report;
     if (!r) return fail(CUSAN_ENOMEM, "cannot allocate report");
     uint64_t d2h = N_COUNTERS * sizeof(unsigned long long);
-    const int mst = merge_runs_device(s->merge, s->stream, s->runs, kept_runs, r->runs, &d2h);   // a4
+    const int mst = merge_runs_device(s->merge, s->stream, s->runs.p, kept_runs, r->runs, &d2h);   // a4
+    tick("merge");
     if (mst) {
         delete r;
         return mst;
@@ -655,7 +676,7 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
     r->ctr.run_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count();
     *out = r;
     // a run list that overflowed is sized for the next call (best effort: this call succeeded)
-    if (runs_ovf) ensure(&s->runs, &s->run_cap, cnt[C_RUNS] + cnt[C_RUNS] / 8 + 1024, "run buffer");
+    if (runs_ovf) grow_runs(s, cnt[C_RUNS] + cnt[C_RUNS] / 8 + 1024);
     return CUSAN_OK;
 }
 

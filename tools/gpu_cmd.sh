@@ -1,10 +1,3 @@
-mkdir -p gpurun_out/r01_configs
-for c in 5 4 3 2; do
-  for t in racy clean; do
-    fl=""; [ $t = clean ] && fl="--clean"
-    cb=""; [ $t = clean ] && cb="--no-cpu-baseline"
-    timeout 600 python bench.py --config $c $fl $cb --steps 10 --warmup 3 > gpurun_out/r01_configs/bench_config${c}_$t.json 2> gpurun_out/r01_configs/bench_config${c}_$t.err
-    echo "config $c $t rc=$?"
-  done
-done
-timeout 900 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/bench_reference.json 2> gpurun_out/bench_reference.err; cut -c1-300 gpurun_out/bench_reference.json
+timeout 900 python -m pytest tests/test_gpu_session.py tests/test_gpu_capture.py -x -q 2>&1 | tail -2
+CUSAN_DEBUG_TIMING=1 timeout 600 python tools/session_bench.py --config 5 --chunk 4096 2>gpurun_out/sess_dbg.txt > gpurun_out/session_c5_4096.json; cut -c1-330 gpurun_out/session_c5_4096.json
+timeout 600 python tools/session_bench.py --config 5 --chunk 512 > gpurun_out/session_c5_512.json; cut -c1-330 gpurun_out/session_c5_512.json
