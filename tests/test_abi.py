@@ -187,3 +187,45 @@ def test_lowering_single_call_api():
         low.cusan_on_kernel(77, [0x1000], [1])          # unknown stream
     with pytest.raises(cs.CusanError):
         low.cusan_on_memcpy(0, 0, 8, 9, 0, 0)             # bad copy kind
+
+
+def test_concurrent_planning_threads():
+    """Host planning from several threads at once (ctypes releases the GIL): the shared pool of
+    planning threads serves one caller, the others run their own threads; results are identical."""
+    import threading
+    w = configs.make(3, "full")
+    ops, args = w.arrays(True)
+    tr = cs.Trace(255)
+    cs.Lowering(tr).cusan_lower_program(ops, args)
+    want = cs.describe(tr, window_events=512)
+    out, errs = [], []
+
+    def work():
+        try:
+            for _ in range(3):
+                out.append(cs.describe(tr, window_events=512))
+        except Exception as e:               # pragma: no cover - reported below
+            errs.append(e)
+    th = [threading.Thread(target=work) for _ in range(4)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join(timeout=120)
+    assert not errs and len(out) == 12
+    assert all(d == want for d in out)
+
+
+def test_planning_with_the_clock_thread():
+    """From 4096 accesses on, a1 runs on its own thread next to a2; the plan is the same as the
+    serial one would give (one interval and one segment row per disjoint write)."""
+    n = 1 << 13
+    ev = np.zeros(n, EVENT_DTYPE)
+    ev["kind"] = 0
+    ev["mode"] = 1
+    ev["a"] = np.arange(n, dtype=np.uint64) * 64
+    ev["b"] = 64
+    t = cs.Trace(4)
+    t.cusan_trace_append_events(ev)
+    d = cs.describe(t, window_events=100)
+    assert d["n_access"] == n and d["n_intervals"] == n and d["n_windows"] == (n + 99) // 100
+    assert d["n_segments"] == 1 and d["n_incidences"] == n and d["tracked_bytes"] == 64 * n
