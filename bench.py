@@ -193,9 +193,20 @@ def run_reference(args):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot_s / args.steps,
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
         "data": "synthetic", "config": ref_config,
-        "cpu_baseline": {"value": value, "unit": "GB/s", "cores": threads, "kind": "oracle", "sample": sample},
+        "cpu_baseline": {"value": value, "unit": "GB/s", "cores": threads, "kind": "oracle", "cpu_model": cpu_model(),
+                         "sample": sample},
         "e2e": {"value": value, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }))
+
+
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
 
 
 def oracle_sample_step(ev, nf, s, threads):
@@ -354,7 +365,9 @@ def run_ours(args):
     if world == 1 and not args.no_cpu_baseline:
         ev = tr.cusan_trace_read()
         s = oracle_sample(ev, 255, args.cpu_seconds, os.cpu_count() or 1)
+        s1 = oracle_sample(ev, 255, 2.0, 1)          # single-thread rate on a smaller slice
         cpu = {"value": s["rate_gbs"], "unit": "GB/s", "cores": os.cpu_count() or 1, "kind": "oracle",
+               "cpu_model": cpu_model(), "single_thread_value": s1["rate_gbs"],
                "sample": (f"contiguous granule range [{s['range'][0]}, {s['range'][1]}) of the same trace: "
                           f"{s['granules']} granules, {s['checked_bytes'] / 1e9:.1f} GB checked in "
                           f"{s['seconds']:.1f} s")}
