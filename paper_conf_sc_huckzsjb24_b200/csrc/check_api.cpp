@@ -5,6 +5,8 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <map>
+#include <mutex>
 #include <new>
 #include <string>
 
@@ -37,7 +39,7 @@ struct cusan_plan {
     bool bound = false;                     // workspace carved and tables uploaded
     uint64_t o_inc = 0, o_seg = 0, o_spans = 0, o_cnt = 0, o_heap = 0, o_shadow = 0, o_runs = 0, o_merge = 0;
     uint64_t merge_bytes = 0;
-    std::vector<DSpan> ds;                  // device span tables (host copy, uploaded at bind)
+    pinned_vector<DSpan> ds;                // device span tables (host copy, uploaded at bind)
     std::vector<Window> wins;
     uint64_t shadow_cell_bytes = 0;
     uint64_t table_bytes = 0;               // tables uploaded by plan_create
@@ -56,8 +58,75 @@ struct cusan_plan {
 
 static int plan_bind(cusan_plan* p, char* ws, uint64_t bytes);
 
+// ---- pinned host blocks for uploaded tables (common.h) ------------------------------------------
+// Every block carries a 64-byte header {size class, pinned?}.  Freed blocks go back to a cache by
+// size class (powers of two from 64 KiB) up to PINNED_CACHE_MAX bytes; a process without a usable
+// CUDA device gets heap blocks.
+namespace {
+constexpr size_t PIN_HDR = 64, PINNED_CACHE_MAX = size_t(1) << 30;
+struct PinHdr { size_t cls; int pinned; };
+struct PinCache {
+    std::mutex m;
+    std::map<size_t, std::vector<void*>> free_by_cls;
+    size_t cached = 0;
+    int device_ok = -1;      // -1 unknown, 0 no CUDA device, 1 cudaHostAlloc works
+};
+PinCache& pin_cache() { static PinCache* c = new PinCache; return *c; }
+}  // namespace
+
+void* cusan::pinned_alloc(size_t bytes) {
+    size_t cls = size_t(1) << 16;
+    while (cls < bytes + PIN_HDR) cls <<= 1;
+    PinCache& c = pin_cache();
+    {
+        std::lock_guard<std::mutex> lk(c.m);
+        auto it = c.free_by_cls.find(cls);
+        if (it != c.free_by_cls.end() && !it->second.empty()) {
+            void* b = it->second.back();
+            it->second.pop_back();
+            c.cached -= cls;
+            return (char*)b + PIN_HDR;
+        }
+    }
+    void* b = nullptr;
+    int pinned = 0;
+    if (c.device_ok != 0) {
+        if (cudaHostAlloc(&b, cls, cudaHostAllocPortable) == cudaSuccess) {
+            pinned = 1;
+            c.device_ok = 1;
+        } else {
+            (void)cudaGetLastError();
+            b = nullptr;
+            int n = 0;
+            if (c.device_ok == -1 && (cudaGetDeviceCount(&n) != cudaSuccess || n == 0)) c.device_ok = 0;
+            (void)cudaGetLastError();
+        }
+    }
+    if (!b) b = std::malloc(cls);
+    if (!b) throw std::bad_alloc();
+    *(PinHdr*)b = PinHdr{cls, pinned};
+    return (char*)b + PIN_HDR;
+}
+
+void cusan::pinned_free(void* p) noexcept {
+    if (!p) return;
+    void* b = (char*)p - PIN_HDR;
+    const PinHdr h = *(const PinHdr*)b;
+    PinCache& c = pin_cache();
+    {
+        std::lock_guard<std::mutex> lk(c.m);
+        if (c.cached + h.cls <= PINNED_CACHE_MAX) {
+            c.free_by_cls[h.cls].push_back(b);
+            c.cached += h.cls;
+            return;
+        }
+    }
+    if (h.pinned) cudaFreeHost(b);
+    else std::free(b);
+}
+
 void cusan::build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& out) {
-    std::vector<DSpan>& ds = out.ds;
+    pinned_vector<DSpan>& ds = out.ds;
     ds.clear();
     ds.reserve(hp.spans.size() + hp.win_span_off.size());
     out.wins.clear();
@@ -148,7 +217,7 @@ static int plan_device_setup(cusan_plan* p) {
 
     SpanTables st;
     build_span_tables(hp, p->max_blocks, st);
-    std::vector<DSpan>& ds = st.ds;
+    pinned_vector<DSpan>& ds = st.ds;
     p->wins = st.wins;
     p->need_shadow = st.need_shadow;
     p->shadow_cell_bytes = st.cell_bytes;

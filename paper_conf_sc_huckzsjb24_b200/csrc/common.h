@@ -12,6 +12,70 @@ namespace cusan {
 // thread-local last error (cusan_last_error)
 int fail(int status, const std::string& msg);
 
+// Host memory for the tables a plan or session uploads to the device: page-locked
+// (cudaHostAlloc) so every upload is a DMA transfer, taken from a process-wide cache of blocks
+// (pinning costs milliseconds per call); plain heap memory in a process without a CUDA device
+// (host planning only: cusan_plan_describe).
+void* pinned_alloc(size_t bytes);
+void pinned_free(void* p) noexcept;
+template <class T>
+struct PinnedAllocator {
+    using value_type = T;
+    PinnedAllocator() = default;
+    template <class U> PinnedAllocator(const PinnedAllocator<U>&) noexcept {}
+    T* allocate(size_t n) { return static_cast<T*>(pinned_alloc(n * sizeof(T))); }
+    void deallocate(T* p, size_t) noexcept { pinned_free(p); }
+    template <class U> bool operator==(const PinnedAllocator<U>&) const noexcept { return true; }
+    template <class U> bool operator!=(const PinnedAllocator<U>&) const noexcept { return false; }
+};
+template <class T>
+using pinned_vector = std::vector<T, PinnedAllocator<T>>;
+
+// Sync-clock slot of each key (open addressing, linear probing): keys are arbitrary u64 values,
+// slots are numbered 0, 1, 2 ... in order of first use.
+class KeySlots {
+  public:
+    uint32_t size() const { return n_; }
+    // slot of `key`; a new key gets the next slot and *fresh = true
+    uint32_t get(uint64_t key, bool* fresh) {
+        if (2 * (n_ + 1) > cap_) grow();
+        for (size_t i = hash(key) & (cap_ - 1);; i = (i + 1) & (cap_ - 1)) {
+            if (val_[i] == EMPTY) {
+                key_[i] = key;
+                val_[i] = n_;
+                *fresh = true;
+                return n_++;
+            }
+            if (key_[i] == key) {
+                *fresh = false;
+                return val_[i];
+            }
+        }
+    }
+
+  private:
+    static constexpr uint32_t EMPTY = 0xffffffffu;
+    static size_t hash(uint64_t k) { return (size_t)((k * 0x9E3779B97F4A7C15ull) >> 20); }
+    void grow() {
+        std::vector<uint64_t> k = std::move(key_);
+        std::vector<uint32_t> v = std::move(val_);
+        cap_ = cap_ ? 2 * cap_ : 1024;
+        key_.assign(cap_, 0);
+        val_.assign(cap_, EMPTY);
+        for (size_t j = 0; j < v.size(); j++) {
+            if (v[j] == EMPTY) continue;
+            size_t i = hash(k[j]) & (cap_ - 1);
+            while (val_[i] != EMPTY) i = (i + 1) & (cap_ - 1);
+            key_[i] = k[j];
+            val_[i] = v[j];
+        }
+    }
+    std::vector<uint64_t> key_;
+    std::vector<uint32_t> val_;
+    size_t cap_ = 0;
+    uint32_t n_ = 0;
+};
+
 struct Trace {
     uint32_t max_fibers = 1;
     std::vector<cusan_event> ev;
@@ -66,7 +130,7 @@ struct HostPlan {
     cusan_check_opts opts{};
     // a1
     uint32_t F = 1;                       // fibers (row length of segvc)
-    std::vector<uint32_t> segvc;          // nseg × F
+    pinned_vector<uint32_t> segvc;        // nseg × F (uploaded)
     uint64_t nseg = 0;
     // accesses in trace order
     std::vector<uint64_t> acc_g0, acc_g1; // granule ranges
@@ -74,7 +138,7 @@ struct HostPlan {
     std::vector<AccRec> acc_rec;
     // a2
     std::vector<Interval> iv;             // shard-clipped intervals (len > 0)
-    std::vector<AccRec> inc;              // incidence table: per interval, its accesses in trace order
+    pinned_vector<AccRec> inc;            // incidence table: per interval, its accesses in trace order (uploaded)
     std::vector<uint32_t> inc_acc;        // access index of each incidence
     uint64_t shard_granules = 0;          // covered granules in this shard
     uint64_t shadow_cells = 0;            // shadow slots incl. alignment padding

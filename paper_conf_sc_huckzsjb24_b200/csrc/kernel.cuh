@@ -126,7 +126,7 @@ cudaError_t shadow_check_blocks_per_sm(int* per_sm);
 // ---- host helpers shared by check_api.cpp and session.cpp -----------------------------------------
 // Device-side span tables: per window its spans plus a sentinel, with range / weight prefixes.
 struct SpanTables {
-    std::vector<DSpan> ds;
+    pinned_vector<DSpan> ds;
     std::vector<Window> wins;
     bool need_shadow = false;
     uint64_t cell_bytes = 0;      // algorithmic shadow bytes (8 B per LOAD + 8 B per STORE cell)

@@ -115,6 +115,30 @@ static void parallel_for(unsigned T, Fn&& fn) {
     for (auto& x : th) x.join();
 }
 
+// Stable LSD radix sort of (key, id) pairs by key: 11-bit digits over the bits in which the keys
+// differ (granule numbers of one address space: a few passes).
+static void radix_sort_pairs(std::vector<uint64_t>& key, std::vector<uint32_t>& id) {
+    const size_t n = key.size();
+    if (n < 2) return;
+    const auto mm = std::minmax_element(key.begin(), key.end());
+    const uint64_t mn = *mm.first, span = *mm.second - mn;
+    const int bits = span ? 64 - __builtin_clzll(span) : 0;
+    std::vector<uint64_t> k2(n);
+    std::vector<uint32_t> i2(n);
+    for (int sh = 0; sh < bits; sh += 11) {
+        std::vector<size_t> cnt(2049, 0);
+        for (size_t i = 0; i < n; i++) cnt[((key[i] - mn) >> sh & 2047) + 1]++;
+        for (int d = 0; d < 2048; d++) cnt[d + 1] += cnt[d];
+        for (size_t i = 0; i < n; i++) {
+            const size_t at = cnt[(key[i] - mn) >> sh & 2047]++;
+            k2[at] = key[i];
+            i2[at] = id[i];
+        }
+        key.swap(k2);
+        id.swap(i2);
+    }
+}
+
 int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uint64_t first_access,
                     uint64_t rec_base) {
     if (o.nshards < 1 || o.shard < 0 || o.shard >= o.nshards)
@@ -161,17 +185,15 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
     // incidence table at the end).  Errors come back as (status, message).
     auto a1 = [&]() -> std::pair<int, std::string> {
         std::vector<uint32_t> C((size_t)F * F, 0);
-        std::unordered_map<uint64_t, uint32_t> key_slot;
+        KeySlots key_slot;
         std::vector<uint32_t> sc;                   // sync clocks, F entries per key
         const uint32_t NO_SEG = 0xffffffffu;
         std::vector<uint32_t> cur_seg(F, NO_SEG);
         auto sync_clock = [&](uint64_t key) -> uint32_t* {
-            auto it = key_slot.find(key);
-            if (it == key_slot.end()) {
-                it = key_slot.emplace(key, (uint32_t)(sc.size() / F)).first;
-                sc.resize(sc.size() + F, 0);
-            }
-            return &sc[(size_t)it->second * F];
+            bool fresh;
+            const uint32_t slot = key_slot.get(key, &fresh);
+            if (fresh) sc.resize(sc.size() + F, 0);
+            return &sc[(size_t)slot * F];
         };
         uint64_t k = 0;
         for (uint64_t i = 0; i < t.ev.size(); i++) {
@@ -248,96 +270,53 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
     };
 
     // ---------------------------------------------------------------- a2: elementary intervals --
+    // Endpoints of the non-empty accesses, radix-sorted with their access ids: the distinct values
+    // are the interval boundaries B, and each endpoint's rank is its boundary index (b0, b1).
+    std::vector<uint32_t> b0(n_acc, 0), b1(n_acc, 0);
     std::vector<uint64_t> B;
-    B.reserve(2 * n_acc);
-    for (uint64_t k = 0; k < n_acc; k++)
-        if (hp.acc_g1[k] > hp.acc_g0[k]) { B.push_back(hp.acc_g0[k]); B.push_back(hp.acc_g1[k]); }
-    std::sort(B.begin(), B.end());
-    B.erase(std::unique(B.begin(), B.end()), B.end());
-    tick("a2 sort");
-    const uint64_t nb = B.size();
-    std::vector<int64_t> diff(nb + 1, 0);
-    std::vector<uint32_t> b0(n_acc), b1(n_acc);
     {
-        const unsigned TB = plan_threads(n_acc * 8);
-        parallel_for(TB, [&](unsigned t) {
-            const uint64_t ka = n_acc * t / TB, kb = n_acc * (t + 1) / TB;
-            for (uint64_t k = ka; k < kb; k++) {
-                if (hp.acc_g1[k] <= hp.acc_g0[k]) { b0[k] = b1[k] = 0; continue; }
-                b0[k] = (uint32_t)(std::lower_bound(B.begin(), B.end(), hp.acc_g0[k]) - B.begin());
-                b1[k] = (uint32_t)(std::lower_bound(B.begin(), B.end(), hp.acc_g1[k]) - B.begin());
-            }
-        });
+        std::vector<uint64_t> ek;
+        std::vector<uint32_t> eid;
+        ek.reserve(2 * n_acc);
+        eid.reserve(2 * n_acc);
         for (uint64_t k = 0; k < n_acc; k++)
-            if (b1[k] > b0[k]) { diff[b0[k]]++; diff[b1[k]]--; }
+            if (hp.acc_g1[k] > hp.acc_g0[k]) {
+                ek.push_back(hp.acc_g0[k]);
+                eid.push_back((uint32_t)(2 * k));
+                ek.push_back(hp.acc_g1[k]);
+                eid.push_back((uint32_t)(2 * k + 1));
+            }
+        radix_sort_pairs(ek, eid);
+        B.reserve(ek.size());
+        for (size_t i = 0; i < ek.size(); i++) {
+            if (i == 0 || ek[i] != ek[i - 1]) B.push_back(ek[i]);
+            ((eid[i] & 1) ? b1 : b0)[eid[i] >> 1] = (uint32_t)(B.size() - 1);
+        }
     }
     tick("a2 bounds");
-    // elementary interval j = [B[j], B[j+1]); covered ones get ids in ascending address order
-    std::vector<uint32_t> iv_of(nb ? nb - 1 : 0, 0xffffffffu);
-    struct GIv { uint64_t abs_begin, dense_begin, len; uint32_t cnt, off; };
+    const uint64_t nb = B.size();
+    // coverage of elementary interval j = [B[j], B[j+1]) = the accesses covering it (difference
+    // array); covered ones get ids in ascending address order.  An interval's incidence count is
+    // its coverage.
+    struct GIv { uint64_t abs_begin, dense_begin, len; uint32_t cnt, j; };
     std::vector<GIv> giv;
     {
+        std::vector<int64_t> diff(nb + 1, 0);
+        for (uint64_t k = 0; k < n_acc; k++)
+            if (b1[k] > b0[k]) { diff[b0[k]]++; diff[b1[k]]--; }
         int64_t cov = 0;
         uint64_t dense = 0;
         for (uint64_t j = 0; j + 1 < nb; j++) {
             cov += diff[j];
             if (cov > 0) {
-                iv_of[j] = (uint32_t)giv.size();
-                giv.push_back({B[j], dense, B[j + 1] - B[j], 0, 0});
+                if (cov > 0xffffffffll) return fail(CUSAN_ERANGE, "too many interval incidences");
+                giv.push_back({B[j], dense, B[j + 1] - B[j], (uint32_t)cov, (uint32_t)j});
                 dense += B[j + 1] - B[j];
             }
         }
     }
     c.n_intervals = giv.size();
     tick("a2 intervals");
-    // incidences: per interval, covering accesses in trace order (CSR).  Threads take contiguous
-    // chunks of accesses; per-chunk counts give every chunk its slots, so the order is the serial one.
-    // Chunks hold equal numbers of incidences (an access covering many intervals is more work).
-    std::vector<uint64_t> wk(n_acc + 1, 0);
-    for (uint64_t k = 0; k < n_acc; k++) wk[k + 1] = wk[k] + (b1[k] - b0[k]);
-    const unsigned T = plan_threads(std::max<uint64_t>(n_acc, wk[n_acc]));
-    std::vector<std::vector<uint32_t>> cnt_t(T, std::vector<uint32_t>(giv.size(), 0));
-    std::vector<uint64_t> cut(T + 1, n_acc);
-    for (unsigned t = 0; t < T; t++)
-        cut[t] = (uint64_t)(std::lower_bound(wk.begin(), wk.end(), wk[n_acc] * t / T) - wk.begin());
-    auto chunk = [&](unsigned t, uint64_t) { return std::make_pair(std::min(cut[t], n_acc), std::min(cut[t + 1], n_acc)); };
-    parallel_for(T, [&](unsigned t) {
-        auto [ka, kb] = chunk(t, n_acc);
-        for (uint64_t k = ka; k < kb; k++)
-            for (uint32_t j = b0[k]; j < b1[k]; j++) cnt_t[t][iv_of[j]]++;
-    });
-    uint64_t n_inc = 0;
-    for (size_t i = 0; i < giv.size(); i++) {
-        GIv& g = giv[i];
-        g.off = (uint32_t)n_inc;
-        uint64_t at = n_inc;
-        for (unsigned t = 0; t < T; t++) {           // counts -> each chunk's first slot
-            const uint32_t n = cnt_t[t][i];
-            cnt_t[t][i] = (uint32_t)at;
-            at += n;
-        }
-        if (at > 0xffffffffull) return fail(CUSAN_ERANGE, "too many interval incidences");
-        g.cnt = (uint32_t)(at - n_inc);
-        n_inc = at;
-    }
-    c.n_incidences = n_inc;
-    hp.inc.resize(n_inc);
-    hp.inc_acc.resize(n_inc);
-    parallel_for(T, [&](unsigned t) {
-        auto [ka, kb] = chunk(t, n_acc);
-        std::vector<uint32_t>& slot = cnt_t[t];
-        for (uint64_t k = ka; k < kb; k++)
-            for (uint32_t j = b0[k]; j < b1[k]; j++) hp.inc_acc[slot[iv_of[j]]++] = (uint32_t)k;
-    });
-    tick("a2 incidence");
-    if (int st = a1_finish()) return st;                 // a1's records fill the incidence table
-    {
-        const unsigned TI = plan_threads(n_inc);
-        parallel_for(TI, [&](unsigned t) {
-            const uint64_t qa = n_inc * t / TI, qb = n_inc * (t + 1) / TI;
-            for (uint64_t q = qa; q < qb; q++) hp.inc[q] = hp.acc_rec[hp.inc_acc[q]];
-        });
-    }
     // ---------------------------------------------------------------- a2: shard clip ------------
     const uint64_t total_dense = giv.empty() ? 0 : giv.back().dense_begin + giv.back().len;
     uint64_t d_lo = 0, d_hi = total_dense;
@@ -349,18 +328,35 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
         const uint64_t Ws = o.window_events > 0 ? (uint64_t)o.window_events : std::max<uint64_t>(n_acc, 1);
         const bool windowed = Ws < n_acc && !(o.flags & CUSAN_CHECK_INTERVAL_SHADOW);
         std::vector<uint64_t> wpg(giv.size());
-        for (size_t i = 0; i < giv.size(); i++) {
-            const GIv& g = giv[i];
-            if (!windowed) {
-                wpg[i] = std::max<uint64_t>(g.cnt, 1);
-                continue;
+        if (!windowed) {
+            for (size_t i = 0; i < giv.size(); i++) wpg[i] = std::max<uint64_t>(giv[i].cnt, 1);
+        } else {
+            // k per interval = windows whose accesses cover it: each window's covered boundary
+            // ranges (its accesses' [b0, b1) merged) add one on a difference array
+            const uint64_t nw = (n_acc + Ws - 1) / Ws;
+            std::vector<std::vector<std::pair<uint32_t, uint32_t>>> wr(nw);
+            const unsigned TW = (unsigned)std::min<uint64_t>(plan_threads(n_acc * 4), nw);
+            parallel_for(TW, [&](unsigned t) {
+                for (uint64_t w = t; w < nw; w += TW) {
+                    std::vector<std::pair<uint32_t, uint32_t>> r;
+                    for (uint64_t k = w * Ws; k < std::min(n_acc, (w + 1) * Ws); k++)
+                        if (b1[k] > b0[k]) r.emplace_back(b0[k], b1[k]);
+                    std::sort(r.begin(), r.end());
+                    auto& out = wr[w];
+                    for (const auto& x : r) {
+                        if (!out.empty() && x.first <= out.back().second) out.back().second = std::max(out.back().second, x.second);
+                        else out.push_back(x);
+                    }
+                }
+            });
+            std::vector<int64_t> kd(nb + 1, 0);
+            for (const auto& out : wr)
+                for (const auto& x : out) { kd[x.first]++; kd[x.second]--; }
+            for (uint64_t j = 1; j <= nb; j++) kd[j] += kd[j - 1];
+            for (size_t i = 0; i < giv.size(); i++) {
+                const uint64_t k = (uint64_t)kd[giv[i].j];
+                wpg[i] = 2 * (k ? k - 1 : 0) + 1;
             }
-            uint64_t k = 0, last = UINT64_MAX;
-            for (uint32_t q = g.off; q < g.off + g.cnt; q++) {
-                const uint64_t w = hp.inc_acc[q] / Ws;
-                if (w != last) { k++; last = w; }
-            }
-            wpg[i] = 2 * (k ? k - 1 : 0) + 1;
         }
         unsigned __int128 wtot = 0;
         for (size_t i = 0; i < giv.size(); i++) wtot += (unsigned __int128)giv[i].len * wpg[i];
@@ -384,9 +380,11 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
     }
     // shard-local shadow slots: each clipped interval starts on a CELL_ALIGN boundary so warp
     // ranges can move their cells with aligned 128-bit accesses (≤ CELL_ALIGN−1 unused cells each)
-    // (interval-compressed tracking, f3: one slot per interval)
+    // (interval-compressed tracking, f3: one slot per interval).  The incidence table holds only
+    // the shard's intervals, so a rank of a multi-GPU check builds and uploads only its part.
     hp.iv.clear();
-    uint64_t slot = 0;
+    std::vector<uint32_t> iv_j;                      // elementary interval of each shard interval
+    uint64_t slot = 0, n_inc = 0;
     const bool compressed = (o.flags & CUSAN_CHECK_INTERVAL_SHADOW) != 0;
     for (auto& g : giv) {
         uint64_t lo = std::max(g.dense_begin, d_lo), hi = std::min(g.dense_begin + g.len, d_hi);
@@ -395,17 +393,65 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
         v.abs_begin = g.abs_begin + (lo - g.dense_begin);
         v.dense_begin = slot;
         v.len = hi - lo;
-        v.list_off = g.off;
+        v.list_off = (uint32_t)n_inc;
         v.list_cnt = g.cnt;
+        n_inc += g.cnt;
+        if (n_inc > 0xffffffffull) return fail(CUSAN_ERANGE, "too many interval incidences");
         slot = compressed ? slot + 1 : (slot + v.len + CELL_ALIGN - 1) / CELL_ALIGN * CELL_ALIGN;
         hp.iv.push_back(v);
+        iv_j.push_back(g.j);
         c.tracked_bytes_shard += 8 * v.len * g.cnt;
     }
     hp.shard_granules = d_hi - d_lo;
     hp.shadow_cells = slot;
     c.shard_granules = hp.shard_granules;
-
+    c.n_incidences = n_inc;
     tick("a2 clip");
+    // incidences: per shard interval, its covering accesses in trace order (CSR).  Threads own
+    // contiguous chunks of the shard's intervals (equal numbers of incidences) and each scans the
+    // accesses in trace order, so every list comes out in the serial order.
+    hp.inc.resize(n_inc);
+    hp.inc_acc.resize(n_inc);
+    {
+        const size_t niv = hp.iv.size();
+        const unsigned T = niv ? std::min<unsigned>(plan_threads(std::max<uint64_t>(n_acc, n_inc)), (unsigned)niv) : 1;
+        std::vector<size_t> icut(T + 1, niv);
+        icut[0] = 0;
+        for (unsigned t = 1; t < T; t++) {
+            const uint64_t want = n_inc * t / T;
+            size_t lo = 0, hi = niv;                 // first interval whose list starts at >= want
+            while (lo < hi) {
+                const size_t m = (lo + hi) / 2;
+                if (hp.iv[m].list_off < want) lo = m + 1;
+                else hi = m;
+            }
+            icut[t] = std::max(lo, icut[t - 1]);
+        }
+        parallel_for(T, [&](unsigned t) {
+            const size_t ia = icut[t], ib = icut[t + 1];
+            if (ia >= ib) return;
+            const uint32_t ja = iv_j[ia], jb = iv_j[ib - 1] + 1;
+            // elementary j -> shard interval (the clip keeps at most one piece per j)
+            std::vector<uint32_t> at(jb - ja, 0xffffffffu);
+            for (size_t i = ia; i < ib; i++) at[iv_j[i] - ja] = hp.iv[i].list_off;
+            for (uint64_t k = 0; k < n_acc; k++) {
+                const uint32_t lo = std::max(b0[k], ja), hi = std::min(b1[k], jb);
+                for (uint32_t j = lo; j < hi; j++) {
+                    uint32_t& s = at[j - ja];
+                    if (s != 0xffffffffu) hp.inc_acc[s++] = (uint32_t)k;
+                }
+            }
+        });
+    }
+    tick("a2 incidence");
+    if (int st = a1_finish()) return st;                 // a1's records fill the incidence table
+    {
+        const unsigned TI = plan_threads(n_inc);
+        parallel_for(TI, [&](unsigned t) {
+            const uint64_t qa = n_inc * t / TI, qb = n_inc * (t + 1) / TI;
+            for (uint64_t q = qa; q < qb; q++) hp.inc[q] = hp.acc_rec[hp.inc_acc[q]];
+        });
+    }
     // ---------------------------------------------------------------- windows and spans ---------
     // A span that stores its final cells and ends with two or more reader fibers since the
     // interval's last write gets a pre-assigned read-set record: the cell keeps W inline and its R
@@ -418,18 +464,50 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
     const uint64_t W = o.window_events > 0 ? (uint64_t)o.window_events : std::max<uint64_t>(n_new, 1);
     hp.window_accesses = W;
     const uint64_t nwin = n_new ? (n_new + W - 1) / W : 0;
-    // Threads take contiguous chunks of intervals and emit (window, span) in interval order; a
-    // stable counting sort by window then gives the window-major order of the serial loop.
-    // Chunks hold equal numbers of incidences.
+    // Two passes over contiguous chunks of intervals (equal numbers of incidences): the first counts
+    // each chunk's spans per window; a prefix over (window, chunk) gives every chunk its slots in the
+    // window-major order of the serial loop; the second writes the spans straight into them.
     std::vector<uint64_t> wi(hp.iv.size() + 1, 0);
     for (size_t i = 0; i < hp.iv.size(); i++) wi[i + 1] = wi[i] + hp.iv[i].list_cnt + 1;
-    const unsigned TS = plan_threads(wi.back() * 2);
+    unsigned TS = plan_threads(wi.back() * 2);
+    TS = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>(TS, (1ull << 24) / std::max<uint64_t>(nwin, 1)));
     std::vector<size_t> icut(TS + 1, hp.iv.size());
     for (unsigned t = 0; t < TS; t++)
         icut[t] = (size_t)(std::lower_bound(wi.begin(), wi.end(), wi.back() * t / TS) - wi.begin());
-    std::vector<std::vector<std::pair<uint64_t, Span>>> part(TS);
+    std::vector<std::vector<uint64_t>> at(TS, std::vector<uint64_t>(nwin, 0));
+    auto window_of = [&](uint32_t q) { return (hp.inc_acc[q] - first) / W; };
     parallel_for(TS, [&](unsigned t) {
         const size_t ia = std::min(icut[t], hp.iv.size()), ib = std::min(icut[t + 1], hp.iv.size());
+        std::vector<uint64_t>& n = at[t];
+        for (size_t i = ia; i < ib; i++) {
+            const Interval& v = hp.iv[i];
+            uint32_t q = v.list_off;
+            const uint32_t qe = v.list_off + v.list_cnt;
+            while (q < qe && hp.inc_acc[q] < first) q++;
+            uint64_t last = UINT64_MAX;
+            for (; q < qe; q++) {
+                const uint64_t w = window_of(q);
+                if (w != last) { n[w]++; last = w; }
+            }
+        }
+    });
+    std::vector<uint64_t> wstart(nwin + 1, 0);
+    {
+        uint64_t pos = 0;
+        for (uint64_t w = 0; w < nwin; w++) {
+            wstart[w] = pos;
+            for (unsigned t = 0; t < TS; t++) {
+                const uint64_t n = at[t][w];
+                at[t][w] = pos;
+                pos += n;
+            }
+        }
+        wstart[nwin] = pos;
+    }
+    hp.spans.resize(wstart[nwin]);
+    parallel_for(TS, [&](unsigned t) {
+        const size_t ia = std::min(icut[t], hp.iv.size()), ib = std::min(icut[t + 1], hp.iv.size());
+        std::vector<uint64_t>& slot = at[t];
         for (size_t i = ia; i < ib; i++) {
             const Interval& v = hp.iv[i];
             std::bitset<CUSAN_MAX_FIBERS + 1> readers;
@@ -441,15 +519,16 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
             }
             const uint32_t first_new = q;
             while (q < qe) {
-                uint64_t w = (hp.inc_acc[q] - first) / W;
+                const uint64_t w = window_of(q);
                 uint32_t q2 = q;
-                while (q2 < qe && (hp.inc_acc[q2] - first) / W == w) {
+                while (q2 < qe && window_of(q2) == w) {
                     const AccRec& r = hp.inc[q2];
                     if (r.segm >> 31) readers.reset();
                     else readers.set(r.epoch >> 24);
                     q2++;
                 }
-                Span s{};
+                Span& s = hp.spans[slot[w]++];
+                s = Span{};
                 s.abs_begin = v.abs_begin;
                 s.dense_begin = v.dense_begin;
                 s.len = v.len;
@@ -460,21 +539,10 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
                 const uint64_t nr = readers.count();
                 if ((s.flags & SPAN_STORE) && nr >= 2)         // record index assigned below
                     s.rec_units = (uint32_t)((nr + 1 + REC_WORDS - 1) / REC_WORDS);
-                part[t].emplace_back(w, s);
                 q = q2;
             }
         }
     });
-    std::vector<uint64_t> wstart(nwin + 1, 0);
-    for (const auto& pt : part)
-        for (const auto& ws : pt) wstart[ws.first + 1]++;
-    for (uint64_t w = 0; w < nwin; w++) wstart[w + 1] += wstart[w];
-    hp.spans.assign(wstart[nwin], Span{});
-    {
-        std::vector<uint64_t> at(wstart.begin(), wstart.end() - 1);
-        for (const auto& pt : part)
-            for (const auto& ws : pt) hp.spans[at[ws.first]++] = ws.second;
-    }
     hp.rec_units = 0;
     hp.spill_spans = 0;
     for (Span& s : hp.spans)

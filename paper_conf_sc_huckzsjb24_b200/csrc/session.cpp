@@ -175,10 +175,10 @@ struct cusan_session {
     // ---- host state carried between calls ----
     uint32_t F = 1;                                 // clock width = the trace's max_fibers
     std::vector<uint32_t> C;                        // F × F fiber clocks
-    std::unordered_map<uint64_t, uint32_t> key_slot;
+    KeySlots key_slot;
     std::vector<uint32_t> sc;                       // sync clocks, F per key
     std::vector<uint32_t> cur_seg;                  // open segment per fiber
-    std::vector<uint32_t> segvc;                    // all segment rows (host copy)
+    pinned_vector<uint32_t> segvc;                  // all segment rows (host copy, uploaded)
     uint64_t nseg = 0;
     std::vector<SIv> ivs;                           // layout of `shadow`
     uint64_t used = 0;                              // cells of `shadow` in use
@@ -203,12 +203,10 @@ struct cusan_session {
     uint64_t heap_cap() const { return std::min<uint64_t>(heap.cap / REC_WORDS, (1ull << 24) - 1); }
 
     uint32_t* sync_clock(uint64_t key) {
-        auto it = key_slot.find(key);
-        if (it == key_slot.end()) {
-            it = key_slot.emplace(key, (uint32_t)(sc.size() / F)).first;
-            sc.resize(sc.size() + F, 0);
-        }
-        return &sc[(size_t)it->second * F];
+        bool fresh;
+        const uint32_t slot = key_slot.get(key, &fresh);
+        if (fresh) sc.resize(sc.size() + F, 0);
+        return &sc[(size_t)slot * F];
     }
 };
 
@@ -270,7 +268,7 @@ struct CallPlan {
     std::vector<SIv> ivs;                           // new layout
     std::vector<char> has_state;                    // per new interval: covered before this call
     std::vector<uint32_t> inc_off, inc_cnt;         // per new interval: new incidences (CSR)
-    std::vector<AccRec> inc;
+    pinned_vector<AccRec> inc;                      // uploaded
     std::vector<uint32_t> inc_acc;                  // call-local access index of each incidence
     HostPlan hp;                                    // spans, windows and counters for the launches
     std::vector<CopySeg> segs;                      // cells to copy (compressed split pieces)

@@ -8,6 +8,7 @@ import argparse
 import json
 import os
 import sys
+import time
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 
@@ -29,9 +30,11 @@ out = {"config": a.config, "window": a.window, "n": {}}
 t1 = None
 ref = None
 for n in [int(x) for x in a.ns.split(",")]:
-    times, runs, races = [], [], 0
+    times, plan_ms, runs, races = [], [], [], 0
     for s in range(n):
+        t0 = time.perf_counter()
         p = cs.Plan(tr, nshards=n, shard=s, window_events=a.window, workspace="torch")
+        plan_ms.append(1e3 * (time.perf_counter() - t0))
         p.run()
         r = min((p.run() for _ in range(3)), key=lambda r: r.counters["run_ms"])
         times.append(r.counters["run_ms"])
@@ -45,7 +48,7 @@ for n in [int(x) for x in a.ns.split(",")]:
     step = max(times)
     if n == 1:
         t1 = step
-    out["n"][n] = {"max_shard_ms": step, "min_shard_ms": min(times), "speedup": t1 / step if t1 else None,
+    out["n"][n] = {"max_shard_ms": step, "min_shard_ms": min(times), "max_plan_create_ms": max(plan_ms), "speedup": t1 / step if t1 else None,
                    "efficiency": t1 / step / n if t1 else None}
     print(n, out["n"][n], flush=True)
 print(json.dumps(out))
