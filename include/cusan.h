@@ -173,8 +173,10 @@ typedef struct cusan_counters {
     uint64_t tracked_bytes_shard;  /* the part of it inside this report's shard                    */
     uint64_t bytes_read, bytes_written;
     /* plan */
+    /* n_intervals: covered elementary intervals of the whole trace; n_incidences, n_spans: the    */
+    /* (interval, access) pairs and (window, interval) pieces of this plan's shard               */
     uint64_t n_fibers, n_segments, n_intervals, n_incidences, n_windows, n_spans;
-    uint64_t shard_granules, spill_heap_bytes, spill_spans; /* spill records: > 3 reader fibers */
+    uint64_t shard_granules, spill_heap_bytes, spill_spans; /* read-set records: >= 2 reader fibers since the last write */
     uint64_t shadow_bytes, workspace_bytes, raw_runs;
     /* device timings of the last run, CUDA events on the plan's stream, milliseconds */
     double kernel_ms;              /* all shadow-check launches                                  */

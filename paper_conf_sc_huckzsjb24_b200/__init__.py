@@ -26,7 +26,7 @@ ARG_DTYPE = np.dtype([("ptr", "<u8"), ("mode", "<u4"), ("pad", "<u4")])
 
 CUSAN_READ, CUSAN_WRITE = 0, 1
 CUSAN_RELEASE, CUSAN_RELEASE_STORE, CUSAN_ACQUIRE, CUSAN_FORK = 0, 1, 2, 3
-__all__ = ["Trace", "Lowering", "Plan", "Report", "check", "report_merge", "CusanError", "version",
+__all__ = ["Trace", "Lowering", "Plan", "Report", "check", "pipelined_checks", "report_merge", "CusanError", "version",
            "RUN_DTYPE", "EVENT_DTYPE"]
 
 
@@ -211,6 +211,15 @@ class Plan:
         _ck(lib.cusan_plan_workspace_bytes(self.h, C.byref(b)))
         return b.value
 
+    def cusan_plan_bind_workspace(self, workspace) -> None:
+        """Bind device memory (a CUDA uint8 tensor of at least workspace_bytes(), held by the plan)
+        to a plan created with CUSAN_CHECK_DEFER_WORKSPACE and upload its tables."""
+        nbytes = self.workspace_bytes()
+        if workspace.numel() * workspace.element_size() < nbytes:
+            raise ValueError("workspace smaller than workspace_bytes()")
+        self.workspace = workspace
+        _ck(lib.cusan_plan_bind_workspace(self.h, C.c_void_p(workspace.data_ptr()), nbytes))
+
     def run(self) -> Report:
         h = C.c_void_p()
         _ck(lib.cusan_plan_run(self.h, C.byref(h)))
@@ -272,6 +281,44 @@ def check(trace: Trace, workspace: str | None = None, **kw) -> Report:
     h = C.c_void_p()
     _ck(lib.cusan_check(trace.h, C.byref(o), C.byref(h)))
     return _report(h, kw.get("max_runs", 0))
+
+
+def pipelined_checks(make_trace, steps: int, device: int = 0, **kw):
+    """Check `steps` traces one after another with the host and the GPU overlapped: while the GPU
+    checks trace i (a3-a5), a host thread builds trace i+1 (`make_trace(i+1)`, e.g. lowering the
+    next batch of recorded calls, a0) and its plan (a1, a2).  This is how an online checker keeps
+    both busy.  Every plan's tables are uploaded (host -> device) when it is bound, after the
+    previous plan's run completed, and every run downloads its report, so each step still pays
+    its own transfers.  All plans share one workspace from PyTorch's caching allocator (a plan's
+    shadow and records are scratch for its own run).  Yields (trace, report) per step; kw as for
+    Plan (window_events, nshards, shard, stream, flags, ...)."""
+    from concurrent.futures import ThreadPoolExecutor
+
+    import torch
+    kw = dict(kw)
+    kw["flags"] = kw.get("flags", 0) | CUSAN_CHECK_DEFER_WORKSPACE
+
+    def prepare(i):
+        tr = make_trace(i)
+        return tr, Plan(tr, device=device, **kw)
+
+    ws = None
+    with ThreadPoolExecutor(1) as ex:
+        nxt = ex.submit(prepare, 0) if steps > 0 else None
+        for i in range(steps):
+            tr, p = nxt.result()
+            if i + 1 < steps:
+                nxt = ex.submit(prepare, i + 1)
+            need = max(p.workspace_bytes(), 256)
+            if ws is None or ws.numel() < need:
+                ws = None
+                ws = torch.empty(need, dtype=torch.uint8, device=torch.device("cuda", device))
+            try:
+                p.cusan_plan_bind_workspace(ws)
+                rep = p.run()
+            finally:
+                p.close()
+            yield tr, rep
 
 
 def report_merge(runs: np.ndarray, n_race_granules: int, max_runs: int = 0) -> Report:

@@ -1,6 +1,7 @@
 // Plan / check C ABI (host side of steps a3-a5): device span tables, workspace layout and binding,
 // the window launches, overflow re-runs, run download and the canonical report.
 #include <algorithm>
+#include <atomic>
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
@@ -69,7 +70,7 @@ struct PinCache {
     std::mutex m;
     std::map<size_t, std::vector<void*>> free_by_cls;
     size_t cached = 0;
-    int device_ok = -1;      // -1 unknown, 0 no CUDA device, 1 cudaHostAlloc works
+    std::atomic<int> device_ok{-1};   // -1 unknown, 0 no CUDA device, 1 cudaHostAlloc works
 };
 PinCache& pin_cache() { static PinCache* c = new PinCache; return *c; }
 }  // namespace

@@ -88,19 +88,37 @@ def test_spill_path_many_readers():
 
 
 @pytest.mark.parametrize("nshards", [2, 3, 5])
-def test_shards_merge_to_the_whole(nshards):
+@pytest.mark.parametrize("window,flags", [(0, 0), (3, 0), (3, cs.CUSAN_CHECK_INTERVAL_SHADOW)],
+                         ids=["one-window", "windowed", "windowed-compressed"])
+def test_shards_merge_to_the_whole(nshards, window, flags):
+    """Shard boundaries come from the coverage (one window) or from the windows touching each
+    interval (windowed); either way the shards' merged runs are the whole trace's."""
     rng = np.random.default_rng(5 + nshards)
     for _ in range(20):
         nf = int(rng.integers(2, 7))
         ev = fuzz.random_primitive_trace(rng, int(rng.integers(5, 80)), nf, n_keys=3,
                                          n_granules=int(rng.integers(100, 2000)))
-        parts = [gpu_report(ev, nf, nshards=nshards, shard=s) for s in range(nshards)]
+        kw = dict(window_events=window, flags=flags)
+        parts = [gpu_report(ev, nf, nshards=nshards, shard=s, **kw) for s in range(nshards)]
         runs = np.concatenate([p.runs for p in parts])
         merged = cs.report_merge(runs, sum(p.n_race_granules for p in parts))
         assert_equal(merged, oracle.check_events(ev, nf, threads=2))
-        whole = gpu_report(ev, nf)
+        whole = gpu_report(ev, nf, **kw)
         assert sum(p.counters["shard_granules"] for p in parts) == whole.counters["shard_granules"]
         assert sum(p.counters["tracked_bytes_shard"] for p in parts) == parts[0].counters["tracked_bytes"]
+        assert sum(p.counters["n_incidences"] for p in parts) >= whole.counters["n_incidences"]
+
+
+@pytest.mark.parametrize("c", [3, 5])
+def test_small_configs_sharded_windowed(c):
+    w = configs.make(c, "small")
+    ops, args = w.arrays(True)
+    tr, _ = lower_product(ops, args)
+    ref = oracle.check_events(tr.cusan_trace_read(), 256)
+    for nshards in (2, 8):
+        parts = [cs.check(tr, window_events=97, nshards=nshards, shard=s) for s in range(nshards)]
+        merged = cs.report_merge(np.concatenate([p.runs for p in parts]), sum(p.n_race_granules for p in parts))
+        assert_equal(merged, ref)
 
 
 @pytest.mark.parametrize("c", [1, 2, 3, 4, 5])
@@ -298,3 +316,27 @@ def test_maximum_fibers_read_set(flags):
     assert ref["n_runs"] >= 254
     for window in (0, 7):
         assert_equal(gpu_report(ev, 255, window_events=window, flags=flags), ref)
+
+
+def test_pipelined_checks_match_the_oracle_per_step():
+    """pipelined_checks: plans prepared on a host thread while the previous one runs, one shared
+    workspace — every step's report is that trace's oracle report (different sizes and windows per
+    step, so the shared workspace is re-carved and grown)."""
+    rng = np.random.default_rng(77)
+    traces = []
+    for i in range(6):
+        nf = int(rng.integers(2, 8))
+        ev = fuzz.random_primitive_trace(rng, int(rng.integers(5, 120)), nf, n_keys=3,
+                                         n_granules=int(rng.integers(50, 5000) * (i + 1)))
+        traces.append((ev, nf))
+
+    def make(i):
+        tr = cs.Trace(traces[i][1])
+        tr.cusan_trace_append_events(traces[i][0])
+        return tr
+
+    n = 0
+    for i, (tr, rep) in enumerate(cs.pipelined_checks(make, len(traces), window_events=3)):
+        assert_equal(rep, oracle.check_events(traces[i][0], traces[i][1], threads=2))
+        n += 1
+    assert n == len(traces)

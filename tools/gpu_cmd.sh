@@ -1,6 +1,4 @@
 python __graft_entry__.py build > /dev/null
 timeout 900 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1; echo pytest_rc=$?; tail -3 gpurun_out/pytest_gpu.log
-CUSAN_DEBUG_TIMING=1 timeout 300 python tools/e2e_breakdown.py --config 5 --steps 3 > gpurun_out/e2e_c5.txt 2>&1
-grep workspace=torch gpurun_out/e2e_c5.txt; grep build_host gpurun_out/e2e_c5.txt | tail -7
-timeout 600 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; echo bench_rc=$?; python -c "
+timeout 600 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; echo bench_rc=$?; tail -3 gpurun_out/bench.err; python -c "
 import json; d=json.load(open('gpurun_out/bench.json')); print(d['value'], d['e2e'], d['roofline']['frac'], d['clocks'])"
