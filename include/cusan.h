@@ -110,6 +110,8 @@ typedef struct cusan_check_opts {
     void* workspace;      /* optional caller-owned device memory (e.g. a torch tensor); NULL = the
                              library allocates with cudaMalloc                                     */
     uint64_t workspace_bytes;
+    uint64_t shard_block; /* sessions with nshards > 1: granules per block of the block-cyclic shard
+                             map, a power of two (0 = 2^21); one-shot checks shard by range instead */
 } cusan_check_opts;
 
 /* Diagnostics: disable the equal-cells range path so every granule takes the lane-parallel
@@ -155,11 +157,18 @@ int cusan_plan_describe(const cusan_trace* t, const cusan_check_opts* o, cusan_c
  * previous call (in windows of opts.window_events, 0 = one window) against it and reports the races
  * whose later access is among them.  The union of all calls' reports equals one cusan_check of the
  * final trace; n_race_granules of the calls add up to its count.  The trace may only grow.
- * Each call re-plans the interval layout of the whole trace (host) and moves the shadow to it
- * (device copy of untouched intervals), so the device holds two shadows; a call can be re-run
- * internally after a buffer overflow because it never modifies the previous shadow.
- * Restrictions: nshards = 1, no caller workspace.  Report counter tracked_bytes_shard = bytes
- * checked by this call. */
+ * The host plan is incremental (clocks, sync clocks and the interval layout carry over; a call
+ * processes only its new events) and the shadow layout is stable: cells are updated in place and
+ * memory touched for the first time gets cells appended (every device buffer grows inside a
+ * reserved virtual range).  Because a call updates the shadow in place it cannot be re-run: a run
+ * buffer overflow truncates that call's run list (counts stay exact) and grows the buffer; a
+ * read-set heap overflow fails the session (CUSAN_ESTATE afterwards).
+ * Multi-GPU sessions (nshards > 1, one session per rank, each on its own device): the address space
+ * is not known in advance, so the granule space is dealt out block-cyclically — granule g belongs
+ * to shard (g / shard_block) mod nshards, shard_block a power of two (0 = 2^21 granules = 16 MiB of
+ * address).  The shards' reports of one call, merged (cusan_report_merge), are the call's report.
+ * No caller workspace.  Report counter tracked_bytes = bytes checked by this call (all shards),
+ * tracked_bytes_shard = the part in this session's shard. */
 typedef struct cusan_session cusan_session;
 int cusan_session_create(const cusan_trace* t, const cusan_check_opts* o, cusan_session** out);
 int cusan_session_check(cusan_session* s, cusan_report** out);

@@ -166,12 +166,13 @@ CUSAN_CHECK_FORCE_LANES = 1
 
 
 def _opts(nshards=1, shard=0, device=0, window_events=0, persist_shadow=False, max_runs=0, stream=None,
-          flags=0):
+          flags=0, shard_block=0):
     o = cusan_check_opts()
     lib.cusan_check_opts_init(C.byref(o))
     o.nshards, o.shard, o.device, o.flags = nshards, shard, device, flags
     o.window_events, o.persist_shadow, o.max_runs = window_events, int(persist_shadow), max_runs
     o.stream = stream
+    o.shard_block = shard_block
     return o
 
 

@@ -32,7 +32,8 @@ class cusan_check_opts(C.Structure):
     _fields_ = [("nshards", C.c_int), ("shard", C.c_int), ("device", C.c_int),
                 ("window_events", C.c_int), ("persist_shadow", C.c_int), ("flags", C.c_int),
                 ("max_runs", C.c_uint64),
-                ("stream", C.c_void_p), ("workspace", C.c_void_p), ("workspace_bytes", C.c_uint64)]
+                ("stream", C.c_void_p), ("workspace", C.c_void_p), ("workspace_bytes", C.c_uint64),
+                ("shard_block", C.c_uint64)]
 
 
 _COUNTER_U64 = ["n_events", "n_access", "n_read", "n_write", "n_release", "n_release_store",

@@ -183,6 +183,7 @@ struct cusan_session {
     std::vector<SIv> ivs;                           // layout of `shadow`
     uint64_t used = 0;                              // cells of `shadow` in use
     uint64_t checked_access = 0, checked_events = 0, n_calls = 0;
+    uint32_t blk_log2 = 21;                         // block-cyclic shard map (nshards > 1)
     bool broken = false;                            // a call failed after changing the state
     // ---- device state (every buffer grows in place, see DevBuf) ----
     DevBuf<uint2> shadow;                           // cells
@@ -344,8 +345,17 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
     const uint64_t n_new = cp.g0.size();
     std::vector<uint64_t> P;
     P.reserve(2 * (n_new + s->ivs.size()));
+    // with shards, every block edge inside a new access is a boundary too, so each new elementary
+    // interval lies in one block and belongs to one shard (old intervals are this shard's already)
+    const int nsh = s->opts.nshards;
+    const uint32_t L = s->blk_log2;
     for (uint64_t k = 0; k < n_new; k++)
-        if (cp.g1[k] > cp.g0[k]) { P.push_back(cp.g0[k]); P.push_back(cp.g1[k]); }
+        if (cp.g1[k] > cp.g0[k]) {
+            P.push_back(cp.g0[k]);
+            P.push_back(cp.g1[k]);
+            if (nsh > 1)
+                for (uint64_t b = ((cp.g0[k] >> L) + 1) << L; b < cp.g1[k]; b += 1ull << L) P.push_back(b);
+        }
     for (const SIv& u : s->ivs) { P.push_back(u.abs_begin); P.push_back(u.abs_begin + u.len); }
     std::sort(P.begin(), P.end());
     P.erase(std::unique(P.begin(), P.end()), P.end());
@@ -370,6 +380,7 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
             while (u < s->ivs.size() && s->ivs[u].abs_begin + s->ivs[u].len <= P[j]) u++;
             const bool old = u < s->ivs.size() && s->ivs[u].abs_begin <= P[j];
             if (cov <= 0 && !old) continue;
+            if (!old && nsh > 1 && (int)((P[j] >> L) % (uint64_t)nsh) != s->opts.shard) continue;   // another shard's
             SIv v;
             v.abs_begin = P[j];
             v.len = P[j + 1] - P[j];
@@ -404,7 +415,8 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
     // new incidences per interval, in trace order
     cp.inc_cnt.assign(niv, 0);
     for (uint64_t k = 0; k < n_new; k++)
-        for (uint32_t j = b0[k]; j < b1[k]; j++) cp.inc_cnt[iv_of[j]]++;
+        for (uint32_t j = b0[k]; j < b1[k]; j++)
+            if (iv_of[j] != 0xffffffffu) cp.inc_cnt[iv_of[j]]++;
     cp.inc_off.assign(niv, 0);
     uint64_t n_inc = 0;
     for (size_t i = 0; i < niv; i++) {
@@ -419,15 +431,19 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
         std::vector<uint32_t> at(cp.inc_off);
         for (uint64_t k = 0; k < n_new; k++)
             for (uint32_t j = b0[k]; j < b1[k]; j++) {
+                if (iv_of[j] == 0xffffffffu) continue;
                 const uint32_t q = at[iv_of[j]]++;
                 cp.inc[q] = cp.rec[k];
                 cp.inc_acc[q] = (uint32_t)k;
             }
     }
-    uint64_t granules = 0;
-    for (const SIv& v : cp.ivs) granules += v.len;
+    uint64_t granules = 0, tracked_shard = 0;
+    for (size_t i = 0; i < niv; i++) {
+        granules += cp.ivs[i].len;
+        tracked_shard += 8 * cp.ivs[i].len * cp.inc_cnt[i];
+    }
     c.shard_granules = granules;
-    c.tracked_bytes_shard = cp.tracked;
+    c.tracked_bytes_shard = tracked_shard;
 
     // ---- windows and spans for the new incidences; moves for the untouched intervals ---------------
     const uint64_t W = s->opts.window_events > 0 ? (uint64_t)s->opts.window_events : std::max<uint64_t>(n_new, 1);
@@ -499,8 +515,10 @@ extern "C" {
 int cusan_session_create(const cusan_trace* t, const cusan_check_opts* o, cusan_session** out) {
     if (!t || !o || !out) return fail(CUSAN_EINVAL, "null argument");
     *out = nullptr;
-    if (o->nshards != 1 || o->shard != 0)
-        return fail(CUSAN_EINVAL, "sessions check the whole granule space (nshards = 1)");
+    if (o->nshards < 1 || o->shard < 0 || o->shard >= o->nshards)
+        return fail(CUSAN_EINVAL, "need 0 <= shard < nshards");
+    if (o->shard_block & (o->shard_block - 1))
+        return fail(CUSAN_EINVAL, "shard_block must be a power of two (or 0)");
     if (o->workspace) return fail(CUSAN_EINVAL, "sessions manage their own device memory");
     if (o->window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
     cusan_session* s = new (std::nothrow) cusan_session;
@@ -508,6 +526,7 @@ int cusan_session_create(const cusan_trace* t, const cusan_check_opts* o, cusan_
     s->trace = t;
     s->opts = *o;
     s->opts.persist_shadow = 1;
+    s->blk_log2 = o->shard_block ? (uint32_t)__builtin_ctzll(o->shard_block) : 21u;
     s->F = t->t.max_fibers;
     s->C.assign((size_t)s->F * s->F, 0);
     s->cur_seg.assign(s->F, NO_SEG);

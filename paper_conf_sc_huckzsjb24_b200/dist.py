@@ -12,7 +12,7 @@ import numpy as np
 import torch
 import torch.distributed as dist
 
-from . import RUN_DTYPE, Plan, Report, Trace, report_merge
+from . import RUN_DTYPE, Plan, Report, Session, Trace, report_merge
 
 _RUN_U64 = RUN_DTYPE.itemsize // 8          # a run record as three u64 words
 
@@ -64,6 +64,35 @@ class ShardedPlan:
 
     def close(self):
         self.plan.close()
+
+
+class ShardedSession:
+    """One rank's shard of a multi-GPU online check (f1 on N GPUs).  Every rank appends the same
+    events to its trace; its session keeps the shadow of its block-cyclic share of the granule
+    space (granule g -> shard (g / shard_block) mod N: the address space is not known in advance,
+    so a contiguous split cannot be balanced up front).  check() checks this rank's share of the
+    new accesses, gathers the runs and returns the call's canonical report on rank 0 (None
+    elsewhere)."""
+
+    def __init__(self, trace: Trace, device: int = 0, group=None, comm_device: torch.device | None = None,
+                 **kw):
+        self.group = group
+        self.comm_device = comm_device
+        self.max_runs = kw.pop("max_runs", 0)
+        self.session = Session(trace, nshards=dist.get_world_size(group), shard=dist.get_rank(group),
+                               device=device, **kw)
+        self.last_shard_report: Report | None = None
+
+    def check(self) -> Report | None:
+        rep = self.session.check()
+        self.last_shard_report = rep
+        out = gather_runs(rep.runs, rep.n_race_granules, self.comm_device, self.group)
+        if out is None:
+            return None
+        return report_merge(out[0], out[1], self.max_runs)
+
+    def close(self):
+        self.session.close()
 
 
 def merge_shard_reports(parts: list[Report], max_runs: int = 0) -> Report:

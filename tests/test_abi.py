@@ -69,6 +69,11 @@ def test_argument_validation():
     with pytest.raises(cs.CusanError):
         t.cusan_trace_append_events(bad)
     assert len(t) == 0                                   # bulk append is all-or-nothing
+    # session shard arguments are validated before any device work
+    for kw in (dict(nshards=2, shard=2), dict(nshards=0), dict(nshards=2, shard=1, shard_block=48)):
+        with pytest.raises(cs.CusanError) as e:
+            cs.Session(t, **kw)
+        assert e.value.status == -1
 
 
 def test_check_without_gpu_fails_loudly():

@@ -80,10 +80,12 @@ def test_session_small_configs(c):
     assert ref["n_race_granules"] > 0
 
 
-def test_session_rejects_shards_and_shrinking():
+def test_session_rejects_bad_shards_and_shrinking():
     tr = cs.Trace(4)
     with pytest.raises(cs.CusanError):
-        cs.Session(tr, nshards=2)
+        cs.Session(tr, nshards=2, shard=2)
+    with pytest.raises(cs.CusanError):
+        cs.Session(tr, nshards=2, shard=0, shard_block=48)      # not a power of two
     ses = cs.Session(tr)
     tr.cusan_trace_append_access(0, 1, 0x1000, 64)
     tr.cusan_trace_append_access(1, 1, 0x1000, 64)
@@ -138,3 +140,58 @@ def test_session_shadow_growth_many_calls():
     cuts = list(range(1, n_calls)) + [n_calls + 2 + 5 * i for i in range(8)]
     ref = _run_session(ev, 2, cuts)
     assert ref["n_race_granules"] == (n_calls // 2) * (size // 2) // 8
+
+
+@pytest.mark.parametrize("nshards,block", [(2, 64), (3, 32), (4, 1 << 12)])
+@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_INTERVAL_SHADOW], ids=["per-granule", "compressed"])
+def test_session_block_cyclic_shards_merge_per_call(nshards, block, flags):
+    """Multi-GPU sessions: per call, the merged reports of the block-cyclic shards equal the
+    one-shard session's report of that call (which the other session tests pin to the oracle);
+    shard granules and checked bytes add up."""
+    rng = np.random.default_rng(100 + nshards)
+    for _ in range(6):
+        nf = int(rng.integers(2, 7))
+        ev = fuzz.random_primitive_trace(rng, int(rng.integers(20, 150)), nf, n_keys=3,
+                                         n_granules=int(rng.integers(200, 6000)))
+        cuts = sorted({0, len(ev), *rng.integers(1, len(ev), 3).tolist()})
+        trs = [cs.Trace(nf) for _ in range(nshards + 1)]
+        whole = cs.Session(trs[0], window_events=3, flags=flags)
+        parts = [cs.Session(trs[1 + s], window_events=3, flags=flags, nshards=nshards, shard=s,
+                            shard_block=block) for s in range(nshards)]
+        for a, b in zip(cuts[:-1], cuts[1:]):
+            for t in trs:
+                t.cusan_trace_append_events(ev[a:b])
+            ref = whole.check()
+            reps = [p.check() for p in parts]
+            merged = cs.report_merge(np.concatenate([r.runs for r in reps]), sum(r.n_race_granules for r in reps))
+            assert merged.n_race_granules == ref.n_race_granules
+            assert np.array_equal(merged.runs, ref.runs)
+            assert sum(r.counters["tracked_bytes_shard"] for r in reps) == ref.counters["tracked_bytes"]
+            assert sum(r.counters["shard_granules"] for r in reps) == ref.counters["shard_granules"]
+        whole.close()
+        for p in parts:
+            p.close()
+
+
+def test_session_shards_small_config():
+    w = configs.make(5, "small")
+    ops, args = w.arrays(True)
+    tr = cs.Trace(255)
+    cs.Lowering(tr).cusan_lower_program(ops, args)
+    ev = tr.cusan_trace_read()
+    ref = oracle.check_events(ev, 256)
+    trs = [cs.Trace(255) for _ in range(3)]
+    ses = [cs.Session(trs[s], window_events=97, nshards=3, shard=s, shard_block=1 << 10) for s in range(3)]
+    runs, n = [], 0
+    for a in range(0, len(ev), len(ev) // 4 + 1):
+        for t in trs:
+            t.cusan_trace_append_events(ev[a:a + len(ev) // 4 + 1])
+        for s in ses:
+            r = s.check()
+            runs.append(r.runs)
+            n += r.n_race_granules
+    merged = cs.report_merge(np.concatenate(runs), n)
+    assert merged.n_race_granules == ref["n_race_granules"] > 0
+    assert np.array_equal(merged.runs, ref["runs"].astype(merged.runs.dtype))
+    for s in ses:
+        s.close()

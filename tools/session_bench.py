@@ -1,7 +1,12 @@
 """Online-checking throughput (f1): feed a config's trace to a cusan_session in chunks of
-`--chunk` accesses and time every session call (host re-planning + layout move + check).
+`--chunk` accesses and time every session call (incremental host plan + check).
 
-    python tools/session_bench.py --config 5 --chunk 4096
+    python tools/session_bench.py --config 5 --chunk 4096 [--nshards N]
+
+With --nshards N, N block-cyclic shard sessions (one per GPU in a multi-GPU run) are run one after
+another on this GPU; a call of the N-GPU session takes the slowest shard's time (the gather of a
+call's runs is a few KB), so Σ over calls of that max predicts the N-GPU online time.  Reports of
+the shards are merged per call and must add up to the one-shard race count.
 """
 import argparse
 import json
@@ -21,6 +26,8 @@ ap.add_argument("--config", type=int, default=5)
 ap.add_argument("--size", default="full")
 ap.add_argument("--chunk", type=int, default=4096, help="accesses per session call")
 ap.add_argument("--window", type=int, default=0)
+ap.add_argument("--nshards", type=int, default=1)
+ap.add_argument("--shard-block", type=int, default=0)
 a = ap.parse_args()
 
 w = configs.make(a.config, a.size)
@@ -31,25 +38,34 @@ ev = full.cusan_trace_read()
 acc_pos = np.flatnonzero(ev["kind"] == 0)
 cuts = [int(acc_pos[i]) for i in range(a.chunk, len(acc_pos), a.chunk)] + [len(ev)]
 
-tr = cs.Trace(255)
-ses = cs.Session(tr, window_events=a.window)
+trs = [cs.Trace(255) for _ in range(a.nshards)]
+sess = [cs.Session(trs[s], window_events=a.window, nshards=a.nshards, shard=s, shard_block=a.shard_block)
+        for s in range(a.nshards)]
 start, calls = 0, []
 for end in cuts:
-    tr.cusan_trace_append_events(ev[start:end])
-    t0 = time.perf_counter()
-    rep = ses.check()
-    dt = time.perf_counter() - t0
-    c = rep.counters
-    calls.append(dict(events=end - start, seconds=dt, kernel_ms=c["kernel_ms"], tracked=c["tracked_bytes_shard"],
-                      cell_bytes=c["shadow_cell_bytes"], races=rep.n_race_granules, launches=c["kernel_launches"]))
+    per = []
+    for t, ses in zip(trs, sess):
+        t.cusan_trace_append_events(ev[start:end])
+        t0 = time.perf_counter()
+        rep = ses.check()
+        dt = time.perf_counter() - t0
+        c = rep.counters
+        per.append(dict(seconds=dt, kernel_ms=c["kernel_ms"], tracked=c["tracked_bytes"],
+                        cell_bytes=c["shadow_cell_bytes"], races=rep.n_race_granules, launches=c["kernel_launches"]))
+    calls.append(dict(events=end - start, seconds=max(x["seconds"] for x in per),
+                      kernel_ms=max(x["kernel_ms"] for x in per), tracked=per[0]["tracked"],
+                      cell_bytes=sum(x["cell_bytes"] for x in per), races=sum(x["races"] for x in per),
+                      launches=max(x["launches"] for x in per),
+                      shard_seconds=[x["seconds"] for x in per] if a.nshards > 1 else None))
     start = end
-ses.close()
+for ses in sess:
+    ses.close()
 tot = sum(x["tracked"] for x in calls)
 secs = sum(x["seconds"] for x in calls)
 kms = sum(x["kernel_ms"] for x in calls)
 cell = sum(x["cell_bytes"] for x in calls)
-out = dict(config=a.config, chunk_accesses=a.chunk, calls=len(calls), tracked_bytes=tot,
+out = dict(config=a.config, chunk_accesses=a.chunk, nshards=a.nshards, calls=len(calls), tracked_bytes=tot,
            checked_gbs=tot / secs / 1e9, kernel_checked_gbs=tot / (kms / 1e3) / 1e9,
-           kernel_dram_gbs=cell / (kms / 1e3) / 1e9, seconds=secs, kernel_ms=kms,
+           kernel_dram_gbs_per_shard=cell / a.nshards / (kms / 1e3) / 1e9, seconds=secs, kernel_ms=kms,
            race_granules=sum(x["races"] for x in calls), per_call=calls)
 print(json.dumps(out))
