@@ -172,6 +172,15 @@ int cusan_plan_describe(const cusan_trace* t, const cusan_check_opts* o, cusan_c
 typedef struct cusan_session cusan_session;
 int cusan_session_create(const cusan_trace* t, const cusan_check_opts* o, cusan_session** out);
 int cusan_session_check(cusan_session* s, cusan_report** out);
+/* Pipelined form of cusan_session_check, so the host and the device work at the same time:
+ * cusan_session_submit plans the events appended since the previous submit on the host (while the
+ * call in flight runs on the device), then collects the call in flight (*prev = its report, NULL if
+ * there was none), then queues this call's uploads and check on the session's stream and returns
+ * without waiting.  cusan_session_finish waits for the call in flight and returns its report (NULL
+ * if none).  Reports are identical to cusan_session_check's; cusan_session_check fails with
+ * CUSAN_ESTATE while a submitted call is in flight.  *prev / *out are freed with cusan_report_free. */
+int cusan_session_submit(cusan_session* s, cusan_report** prev);
+int cusan_session_finish(cusan_session* s, cusan_report** out);
 int cusan_session_destroy(cusan_session* s);
 
 /* ---- report (a5) ------------------------------------------------------------------------------ */

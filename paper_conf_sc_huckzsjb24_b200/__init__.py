@@ -252,6 +252,19 @@ class Session:
         _ck(lib.cusan_session_check(self.h, C.byref(h)))
         return _report(h, self.max_runs)
 
+    def submit(self) -> Report | None:
+        """cusan_session_submit: plan the new events (overlapping the call in flight), collect the
+        call in flight and launch this one; returns the previous call's report (None if none)."""
+        h = C.c_void_p()
+        _ck(lib.cusan_session_submit(self.h, C.byref(h)))
+        return _report(h, self.max_runs) if h.value else None
+
+    def finish(self) -> Report | None:
+        """cusan_session_finish: wait for the call in flight and return its report (None if none)."""
+        h = C.c_void_p()
+        _ck(lib.cusan_session_finish(self.h, C.byref(h)))
+        return _report(h, self.max_runs) if h.value else None
+
     def close(self, _destroy=lib.cusan_session_destroy):
         if getattr(self, "h", None):
             _destroy(self.h)

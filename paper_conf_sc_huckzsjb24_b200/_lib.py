@@ -86,6 +86,8 @@ PROTOS = {
     "cusan_plan_describe": [P, C.POINTER(cusan_check_opts), C.POINTER(cusan_counters)],
     "cusan_session_create": [P, C.POINTER(cusan_check_opts), PP],
     "cusan_session_check": [P, PP],
+    "cusan_session_submit": [P, PP],
+    "cusan_session_finish": [P, PP],
     "cusan_session_destroy": [P],
     "cusan_report_get": [P, pu64, pu64, C.POINTER(C.POINTER(cusan_race_run)), pi32],
     "cusan_report_counters": [P, C.POINTER(cusan_counters)],

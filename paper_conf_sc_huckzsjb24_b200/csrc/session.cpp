@@ -5,6 +5,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <memory>
 #include <new>
 #include <string>
 #include <unordered_map>
@@ -167,6 +168,8 @@ struct SIv {
 
 }  // namespace
 
+struct PendingCall;
+
 struct cusan_session {
     const cusan_trace* trace = nullptr;
     cusan_check_opts opts{};
@@ -196,11 +199,9 @@ struct cusan_session {
     DevBuf<char> merge_buf;                         // a4 scratch
     RunMerge merge;                                 // views merge_buf
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    std::unique_ptr<PendingCall> pending;           // a submitted call not collected yet
 
-    ~cusan_session() {
-        if (ev0) cudaEventDestroy(ev0);
-        if (ev1) cudaEventDestroy(ev1);
-    }
+    ~cusan_session();
     uint64_t heap_cap() const { return std::min<uint64_t>(heap.cap / REC_WORDS, (1ull << 24) - 1); }
 
     uint32_t* sync_clock(uint64_t key) {
@@ -478,7 +479,7 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
             q = q2;
         }
     }
-    // window-major (stable by interval), records numbered from the heap top
+    // window-major (stable by interval), records numbered from 0 (the heap top at launch is added)
     std::vector<uint64_t> wstart(nwin + 1, 0);
     for (const auto& ws : out) wstart[ws.first + 1]++;
     for (uint64_t w = 0; w < nwin; w++) wstart[w + 1] += wstart[w];
@@ -492,12 +493,10 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
     hp.spill_spans = 0;
     for (Span& sp : hp.spans)
         if (sp.rec_units) {
-            sp.rec = (uint32_t)(s->heap_top + hp.rec_units);
+            sp.rec = (uint32_t)hp.rec_units;     // relative: the heap top is added at launch
             hp.rec_units += sp.rec_units;
             hp.spill_spans++;
         }
-    if (s->heap_top + hp.rec_units >= (1u << 24) - 1)
-        return fail(CUSAN_ERANGE, "too many read-set records for the 24-bit record index");
     hp.win_span_off.assign(1, 0);
     for (uint64_t w = 0; w < nwin; w++)
         if (wstart[w + 1] > wstart[w]) hp.win_span_off.push_back(wstart[w + 1]);
@@ -507,6 +506,185 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
     c.n_spans = hp.spans.size();
     c.spill_spans = hp.spill_spans;
     c.spill_heap_bytes = hp.rec_units * REC_WORDS * 4;
+    return CUSAN_OK;
+}
+
+// A call launched by cusan_session_submit and not collected yet.  Its host tables stay here until
+// the call completes: their uploads are asynchronous DMA transfers from page-locked memory.
+struct PendingCall {
+    CallPlan cp;
+    SpanTables tabs;
+    pinned_vector<uint32_t> seg_rows;               // segment rows new in this call (staged)
+    uint64_t seg_first_word = 0;                    // where they go in segvc_d
+    uint64_t used_before = 0;                       // shadow cells in use before the call
+    pinned_vector<unsigned long long> init, cnt;    // counter initial values / read-back
+    uint64_t h2d = 0;
+    std::chrono::steady_clock::time_point t_start;
+};
+
+cusan_session::~cusan_session() {
+    if (ev0) cudaEventDestroy(ev0);
+    if (ev1) cudaEventDestroy(ev1);
+}
+
+static void session_tick(const PendingCall& pc, const char* what) {
+    static const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
+    if (dbg)
+        std::fprintf(stderr, "cusan_session: %-10s %8.3f ms\n", what,
+                     std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - pc.t_start).count());
+}
+
+// Host part of a call: the incremental a1 + a2 of the events appended since the previous call.
+// The session's host state (clocks, layout, counts) moves on at once, so the next call can be
+// planned while this one runs on the device; only the read-set heap top waits for the device
+// (record numbers are relative until launch).
+static int session_plan(cusan_session* s, PendingCall& pc) {
+    const Trace& tr = s->trace->t;
+    if (tr.ev.size() < s->checked_events) return fail(CUSAN_ESTATE, "the trace shrank");
+    s->broken = true;                  // cleared once the call is launched
+    CallPlan& cp = pc.cp;
+    int st;
+    try {
+        st = plan_call(s, tr, cp);
+        if (!st) {
+            build_span_tables(cp.hp, s->max_blocks, pc.tabs);
+            pc.seg_first_word = s->seg_uploaded * s->F;
+            pc.seg_rows.assign(s->segvc.begin() + pc.seg_first_word, s->segvc.begin() + s->nseg * s->F);
+        }
+    } catch (const std::bad_alloc&) {
+        st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
+    }
+    if (st) return st;
+    session_tick(pc, "plan");
+    // the new layout becomes the session's
+    pc.used_before = s->used;
+    s->ivs.swap(cp.ivs);
+    s->used = cp.used;
+    s->seg_uploaded = s->nseg;
+    s->checked_access += cp.g0.size();
+    s->checked_events = tr.ev.size();
+    s->n_calls++;
+    return CUSAN_OK;
+}
+
+// Device part, asynchronous: buffers, uploads, the check launches and the counter read-back are
+// queued on the session's stream (a4's merge happens in session_finish).
+static int session_launch(cusan_session* s, PendingCall& pc) {
+    CallPlan& cp = pc.cp;
+    HostPlan& hp = cp.hp;
+    SpanTables& tabs = pc.tabs;
+    const uint64_t base = s->heap_top;                 // the previous call's records end here
+    if (base + hp.rec_units >= (1u << 24) - 1)
+        return fail(CUSAN_ERANGE, "too many read-set records for the 24-bit record index");
+    for (DSpan& d : tabs.ds)
+        if (d.rec_units) d.rec += (uint32_t)base;
+    // the shadow grows as new memory is touched: new chunks mapped in place, else re-allocated
+    // with its cells moved (1/8 headroom either way)
+    int st;
+    if ((st = grow_buf(s, s->shadow, cp.used, pc.used_before, "the shadow"))) return st;
+    if ((st = grow_heap(s, base + hp.rec_units + (1ull << 16)))) return st;
+    uint64_t tiles = 0;                 // raw-run bound heuristic, as in plans (an overflow truncates)
+    for (const Window& w : tabs.wins) tiles += w.tiles;
+    if ((st = grow_runs(s, 2 * tiles + 1024))) return st;
+    const uint64_t seg_words = pc.seg_first_word + pc.seg_rows.size();
+    if ((st = grow_buf(s, s->segvc_d, seg_words, pc.seg_first_word, "segment rows"))) return st;
+    if (!pc.seg_rows.empty())                        // only the rows new since the last call
+        CK(cudaMemcpyAsync(s->segvc_d.p + pc.seg_first_word, pc.seg_rows.data(), pc.seg_rows.size() * sizeof(uint32_t),
+                           cudaMemcpyHostToDevice, s->stream));
+    const uint64_t nwin = tabs.wins.size();
+    uint64_t off = 0;
+    const uint64_t o_inc = off;   off = align_up(off + cp.inc.size() * sizeof(AccRec));
+    const uint64_t o_spans = off; off = align_up(off + tabs.ds.size() * sizeof(DSpan));
+    const uint64_t o_copy = off;  off = align_up(off + cp.segs.size() * sizeof(CopySeg));
+    const uint64_t o_cnt = off;   off = align_up(off + (N_COUNTERS + nwin) * sizeof(unsigned long long));
+    if ((st = grow_buf(s, s->scratch, off, 0, "plan tables"))) return st;
+    AccRec* d_inc = (AccRec*)(s->scratch.p + o_inc);
+    DSpan* d_spans = (DSpan*)(s->scratch.p + o_spans);
+    CopySeg* d_copy = (CopySeg*)(s->scratch.p + o_copy);
+    unsigned long long* d_cnt = (unsigned long long*)(s->scratch.p + o_cnt);
+    CK(cudaMemcpyAsync(d_inc, cp.inc.data(), cp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, s->stream));
+    CK(cudaMemcpyAsync(d_spans, tabs.ds.data(), tabs.ds.size() * sizeof(DSpan), cudaMemcpyHostToDevice, s->stream));
+    CK(cudaMemcpyAsync(d_copy, cp.segs.data(), cp.segs.size() * sizeof(CopySeg), cudaMemcpyHostToDevice, s->stream));
+    pc.h2d = cp.inc.size() * sizeof(AccRec) + tabs.ds.size() * sizeof(DSpan) + cp.segs.size() * sizeof(CopySeg) +
+             pc.seg_rows.size() * sizeof(uint32_t);
+    session_tick(pc, "memory");
+
+    // ---- a3, in place ------------------------------------------------------------------------------
+    pc.init.assign(N_COUNTERS + nwin, 0ull);
+    pc.cnt.assign(N_COUNTERS, 0ull);
+    pc.init[C_HEAP] = base + hp.rec_units;
+    CK(cudaMemcpyAsync(d_cnt, pc.init.data(), pc.init.size() * sizeof(unsigned long long), cudaMemcpyHostToDevice,
+                       s->stream));
+    CK(cudaEventRecord(s->ev0, s->stream));
+    if (cp.copy_cells)
+        CK(launch_copy_cells(s->max_blocks, s->stream, s->shadow.p, s->shadow.p, d_copy, (uint32_t)cp.segs.size(),
+                             cp.copy_cells, s->heap.p));
+    Ctx k;
+    k.inc = d_inc;
+    k.segvc = s->segvc_d.p;
+    k.F = s->F;
+    k.shadow = s->shadow.p;
+    k.heap = s->heap.p;
+    k.heap_cap = s->heap_cap();
+    k.runs = s->runs.p;
+    k.counters = d_cnt;
+    k.run_cap = s->runs.cap;
+    const int force_lanes = (s->opts.flags & CUSAN_CHECK_FORCE_LANES) ? 1 : 0;
+    for (size_t i = 0; i < nwin; i++) {
+        const Window& w = tabs.wins[i];
+        unsigned long long* sched = CUSAN_DYNAMIC ? d_cnt + N_COUNTERS + i : nullptr;
+        CK(launch_shadow_check(w.grid, s->stream, d_spans + w.span_off, w.nspans, w.tiles, w.weight, k, force_lanes,
+                               sched));
+    }
+    CK(cudaEventRecord(s->ev1, s->stream));
+    CK(cudaMemcpyAsync(pc.cnt.data(), d_cnt, N_COUNTERS * sizeof(unsigned long long), cudaMemcpyDeviceToHost,
+                       s->stream));
+    return CUSAN_OK;
+}
+
+// Wait for a launched call, merge its runs on the device (a4) and build its report (a5).
+static int session_finish(cusan_session* s, PendingCall& pc, cusan_report** out) {
+    CK(cudaStreamSynchronize(s->stream));
+    session_tick(pc, "check");
+    const CallPlan& cp = pc.cp;
+    const uint64_t* cnt = (const uint64_t*)pc.cnt.data();
+    float kms = 0.f;
+    CK(cudaEventElapsedTime(&kms, s->ev0, s->ev1));
+    if (cnt[C_HEAP_OVF]) {
+        s->broken = true;
+        return fail(CUSAN_ENOMEM, "read-set heap overflow: the session's state is lost");
+    }
+    s->heap_top = cnt[C_HEAP];
+    const bool runs_ovf = cnt[C_RUNS] > s->runs.cap;
+    const uint64_t kept_runs = std::min<uint64_t>(cnt[C_RUNS], s->runs.cap);
+    cusan_report* r = new (std::nothrow) cusan_report;
+    if (!r) return fail(CUSAN_ENOMEM, "cannot allocate report");
+    uint64_t d2h = N_COUNTERS * sizeof(unsigned long long);
+    const int mst = merge_runs_device(s->merge, s->stream, s->runs.p, kept_runs, r->runs, &d2h);   // a4
+    session_tick(pc, "merge");
+    if (mst) {
+        delete r;
+        return mst;
+    }
+    r->n_runs = r->runs.size();
+    r->n_race_granules = cnt[C_RACE];   // exact even when the run list overflowed
+    if (runs_ovf) r->truncated = 1;     // the shadow moved on; the call cannot be re-run
+    if (s->opts.max_runs && r->runs.size() > s->opts.max_runs) {
+        r->runs.resize(s->opts.max_runs);
+        r->truncated = 1;
+    }
+    r->ctr = cp.hp.ctr;
+    r->ctr.raw_runs = cnt[C_RUNS];
+    r->ctr.kernel_ms = kms;
+    r->ctr.kernel_launches = pc.tabs.wins.size() + (cp.copy_cells ? 1 : 0) + (kept_runs ? MERGE_LAUNCHES : 0);
+    r->ctr.shadow_cell_bytes = pc.tabs.cell_bytes + 16 * cp.copy_cells;
+    r->ctr.shadow_bytes = cp.used * sizeof(uint2);
+    r->ctr.h2d_bytes = pc.h2d + pc.init.size() * sizeof(unsigned long long);
+    r->ctr.d2h_bytes = d2h;
+    r->ctr.run_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - pc.t_start).count();
+    *out = r;
+    // a run list that overflowed is sized for the next call (best effort: this call succeeded)
+    if (runs_ovf) grow_runs(s, cnt[C_RUNS] + cnt[C_RUNS] / 8 + 1024);
     return CUSAN_OK;
 }
 
@@ -556,150 +734,53 @@ int cusan_session_create(const cusan_trace* t, const cusan_check_opts* o, cusan_
     return CUSAN_OK;
 }
 
+int cusan_session_submit(cusan_session* s, cusan_report** prev) {
+    if (!s || !prev) return fail(CUSAN_EINVAL, "null argument");
+    *prev = nullptr;
+    if (s->broken) return fail(CUSAN_ESTATE, "an earlier call failed after changing the session's state");
+    CK(cudaSetDevice(s->device));
+    std::unique_ptr<PendingCall> next(new (std::nothrow) PendingCall);
+    if (!next) return fail(CUSAN_ENOMEM, "cannot allocate a call");
+    next->t_start = std::chrono::steady_clock::now();
+    int st = session_plan(s, *next);                 // host: overlaps the call in flight
+    if (st) return st;
+    if (s->pending) {                                // collect the call in flight
+        std::unique_ptr<PendingCall> done = std::move(s->pending);
+        st = session_finish(s, *done, prev);
+        if (st) {
+            s->broken = true;
+            return st;
+        }
+    }
+    st = session_launch(s, *next);
+    if (st) return st;
+    s->pending = std::move(next);
+    s->broken = false;
+    return CUSAN_OK;
+}
+
+int cusan_session_finish(cusan_session* s, cusan_report** out) {
+    if (!s || !out) return fail(CUSAN_EINVAL, "null argument");
+    *out = nullptr;
+    if (!s->pending) return CUSAN_OK;
+    CK(cudaSetDevice(s->device));
+    std::unique_ptr<PendingCall> done = std::move(s->pending);
+    return session_finish(s, *done, out);
+}
+
 int cusan_session_check(cusan_session* s, cusan_report** out) {
     if (!s || !out) return fail(CUSAN_EINVAL, "null argument");
     *out = nullptr;
-    const auto t_start = std::chrono::steady_clock::now();
-    const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
-    auto tick = [&](const char* what) {
-        if (dbg)
-            std::fprintf(stderr, "cusan_session_check: %-10s %8.3f ms\n", what,
-                         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count());
-    };
-    CK(cudaSetDevice(s->device));
-    const Trace& tr = s->trace->t;
-    if (tr.ev.size() < s->checked_events) return fail(CUSAN_ESTATE, "the trace shrank");
-    if (s->broken) return fail(CUSAN_ESTATE, "an earlier call failed after changing the session's state");
-    s->broken = true;   // cleared when this call commits
-
-    // ---- host: incremental a1 + a2 (the clocks and the layout carry over) -------------------------
-    CallPlan cp;
-    int st;
-    try {
-        st = plan_call(s, tr, cp);
-    } catch (const std::bad_alloc&) {
-        st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
-    }
+    if (s->pending) return fail(CUSAN_ESTATE, "a submitted call is in flight: collect it with cusan_session_finish");
+    cusan_report* none = nullptr;
+    int st = cusan_session_submit(s, &none);
     if (st) return st;
-    HostPlan& hp = cp.hp;
-    SpanTables tabs;
-    tick("plan");
-    build_span_tables(hp, s->max_blocks, tabs);
-    tick("tables");
-
-    // ---- device memory ---------------------------------------------------------------------------
-    // the shadow grows as new memory is touched: new chunks mapped in place, else re-allocated
-    // with its cells moved (1/8 headroom either way)
-    if ((st = grow_buf(s, s->shadow, cp.used, s->used, "the shadow"))) return st;
-    if ((st = grow_heap(s, s->heap_top + hp.rec_units + (1ull << 16)))) return st;
-    uint64_t tiles = 0;                 // raw-run bound heuristic, as in plans (an overflow truncates)
-    for (const Window& w : tabs.wins) tiles += w.tiles;
-    if ((st = grow_runs(s, 2 * tiles + 1024))) return st;
-    const uint64_t seg_words = s->nseg * s->F, up_words = s->seg_uploaded * s->F;
-    const uint64_t new_row_bytes = (seg_words - up_words) * sizeof(uint32_t);
-    if ((st = grow_buf(s, s->segvc_d, seg_words, up_words, "segment rows"))) return st;
-    if (seg_words > up_words)                        // only the rows new since the last call
-        CK(cudaMemcpyAsync(s->segvc_d.p + up_words, s->segvc.data() + up_words,
-                           (seg_words - up_words) * sizeof(uint32_t), cudaMemcpyHostToDevice, s->stream));
-    const uint64_t nwin = tabs.wins.size();
-    uint64_t off = 0;
-    const uint64_t o_inc = off;   off = align_up(off + cp.inc.size() * sizeof(AccRec));
-    const uint64_t o_spans = off; off = align_up(off + tabs.ds.size() * sizeof(DSpan));
-    const uint64_t o_copy = off;  off = align_up(off + cp.segs.size() * sizeof(CopySeg));
-    const uint64_t o_cnt = off;   off = align_up(off + (N_COUNTERS + nwin) * sizeof(unsigned long long));
-    if ((st = grow_buf(s, s->scratch, off, 0, "plan tables"))) return st;
-    AccRec* d_inc = (AccRec*)(s->scratch.p + o_inc);
-    DSpan* d_spans = (DSpan*)(s->scratch.p + o_spans);
-    CopySeg* d_copy = (CopySeg*)(s->scratch.p + o_copy);
-    unsigned long long* d_cnt = (unsigned long long*)(s->scratch.p + o_cnt);
-    CK(cudaMemcpyAsync(d_inc, cp.inc.data(), cp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, s->stream));
-    CK(cudaMemcpyAsync(d_spans, tabs.ds.data(), tabs.ds.size() * sizeof(DSpan), cudaMemcpyHostToDevice, s->stream));
-    CK(cudaMemcpyAsync(d_copy, cp.segs.data(), cp.segs.size() * sizeof(CopySeg), cudaMemcpyHostToDevice, s->stream));
-    tick("memory");
-
-    // ---- a3 / a4, in place ------------------------------------------------------------------------
-    std::vector<unsigned long long> init(N_COUNTERS + nwin, 0ull), cnt(N_COUNTERS, 0ull);
-    init[C_HEAP] = s->heap_top + hp.rec_units;
-    CK(cudaMemcpyAsync(d_cnt, init.data(), init.size() * sizeof(unsigned long long), cudaMemcpyHostToDevice,
-                       s->stream));
-    CK(cudaEventRecord(s->ev0, s->stream));
-    if (cp.copy_cells)
-        CK(launch_copy_cells(s->max_blocks, s->stream, s->shadow.p, s->shadow.p, d_copy, (uint32_t)cp.segs.size(),
-                             cp.copy_cells, s->heap.p));
-    Ctx k;
-    k.inc = d_inc;
-    k.segvc = s->segvc_d.p;
-    k.F = s->F;
-    k.shadow = s->shadow.p;
-    k.heap = s->heap.p;
-    k.heap_cap = s->heap_cap();
-    k.runs = s->runs.p;
-    k.counters = d_cnt;
-    k.run_cap = s->runs.cap;
-    const int force_lanes = (s->opts.flags & CUSAN_CHECK_FORCE_LANES) ? 1 : 0;
-    for (size_t i = 0; i < nwin; i++) {
-        const Window& w = tabs.wins[i];
-        unsigned long long* sched = CUSAN_DYNAMIC ? d_cnt + N_COUNTERS + i : nullptr;
-        CK(launch_shadow_check(w.grid, s->stream, d_spans + w.span_off, w.nspans, w.tiles, w.weight, k, force_lanes,
-                               sched));
-    }
-    CK(cudaEventRecord(s->ev1, s->stream));
-    CK(cudaMemcpyAsync(cnt.data(), d_cnt, N_COUNTERS * sizeof(unsigned long long), cudaMemcpyDeviceToHost,
-                       s->stream));
-    CK(cudaStreamSynchronize(s->stream));
-    tick("check");
-    float kms = 0.f;
-    CK(cudaEventElapsedTime(&kms, s->ev0, s->ev1));
-    if (cnt[C_HEAP_OVF]) return fail(CUSAN_ENOMEM, "read-set heap overflow: the session's state is lost");
-    const bool runs_ovf = cnt[C_RUNS] > s->runs.cap;
-    const uint64_t kept_runs = std::min<uint64_t>(cnt[C_RUNS], s->runs.cap);
-
-    // ---- commit: the new layout becomes the session's ---------------------------------------------
-    s->ivs.swap(cp.ivs);
-    s->used = cp.used;
-    s->seg_uploaded = s->nseg;
-    s->heap_top = cnt[C_HEAP];
-    s->checked_access += cp.g0.size();
-    s->checked_events = tr.ev.size();
-    s->n_calls++;
-
-    s->broken = false;                  // the state is consistent from here on
-
-    cusan_report* r = new (std::nothrow) cusan_report;
-    if (!r) return fail(CUSAN_ENOMEM, "cannot allocate report");
-    uint64_t d2h = N_COUNTERS * sizeof(unsigned long long);
-    const int mst = merge_runs_device(s->merge, s->stream, s->runs.p, kept_runs, r->runs, &d2h);   // a4
-    tick("merge");
-    if (mst) {
-        delete r;
-        return mst;
-    }
-    r->n_runs = r->runs.size();
-    r->n_race_granules = cnt[C_RACE];   // exact even when the run list overflowed
-    if (runs_ovf) r->truncated = 1;     // the state is committed; the call cannot be re-run
-    if (s->opts.max_runs && r->runs.size() > s->opts.max_runs) {
-        r->runs.resize(s->opts.max_runs);
-        r->truncated = 1;
-    }
-    r->ctr = hp.ctr;
-    r->ctr.raw_runs = cnt[C_RUNS];
-    r->ctr.kernel_ms = kms;
-    r->ctr.kernel_launches = nwin + (cp.copy_cells ? 1 : 0) + (kept_runs ? MERGE_LAUNCHES : 0);
-    r->ctr.shadow_cell_bytes = tabs.cell_bytes + 16 * cp.copy_cells;
-    r->ctr.shadow_bytes = s->used * sizeof(uint2);
-    r->ctr.h2d_bytes = cp.inc.size() * sizeof(AccRec) + tabs.ds.size() * sizeof(DSpan) +
-                       cp.segs.size() * sizeof(CopySeg) + new_row_bytes;
-    r->ctr.d2h_bytes = d2h;
-    r->ctr.run_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count();
-    *out = r;
-    // a run list that overflowed is sized for the next call (best effort: this call succeeded)
-    if (runs_ovf) grow_runs(s, cnt[C_RUNS] + cnt[C_RUNS] / 8 + 1024);
-    return CUSAN_OK;
+    return cusan_session_finish(s, out);
 }
 
 int cusan_session_destroy(cusan_session* s) {
     if (!s) return fail(CUSAN_EINVAL, "session is null");
-    if (s->stream) cudaStreamSynchronize(s->stream);
+    if (s->stream || s->pending) cudaStreamSynchronize(s->stream);
     delete s;
     return CUSAN_OK;
 }

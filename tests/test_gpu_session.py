@@ -195,3 +195,39 @@ def test_session_shards_small_config():
     assert np.array_equal(merged.runs, ref["runs"].astype(merged.runs.dtype))
     for s in ses:
         s.close()
+
+
+@pytest.mark.parametrize("flags,nshards", [(0, 1), (cs.CUSAN_CHECK_FORCE_LANES, 1),
+                                           (cs.CUSAN_CHECK_INTERVAL_SHADOW, 1), (0, 2)],
+                         ids=["ranges", "lanes", "compressed", "shards"])
+def test_session_submit_pipelines_and_matches_check(flags, nshards):
+    """submit/finish (host planning of call i+1 overlapping the device work of call i, records
+    numbered at launch) return, call by call, exactly what check() returns."""
+    rng = np.random.default_rng(300 + flags + nshards)
+    for _ in range(6):
+        nf = int(rng.integers(2, 9))
+        ev = fuzz.random_primitive_trace(rng, int(rng.integers(20, 160)), nf, n_keys=3,
+                                         n_granules=int(rng.integers(100, 4000)))
+        cuts = sorted({0, len(ev), *rng.integers(1, len(ev), 4).tolist()})
+        for shard in range(nshards):
+            kw = dict(window_events=2, flags=flags, nshards=nshards, shard=shard, shard_block=64)
+            ta, tb = cs.Trace(nf), cs.Trace(nf)
+            sa, sb = cs.Session(ta, **kw), cs.Session(tb, **kw)
+            want, got = [], []
+            for a, b in zip(cuts[:-1], cuts[1:]):
+                ta.cusan_trace_append_events(ev[a:b])
+                tb.cusan_trace_append_events(ev[a:b])
+                want.append(sa.check())
+                prev = sb.submit()
+                if prev is not None:
+                    got.append(prev)
+                with pytest.raises(cs.CusanError):
+                    sb.check()                   # a call is in flight
+            got.append(sb.finish())
+            assert sb.finish() is None
+            assert len(got) == len(want)
+            for x, y in zip(got, want):
+                assert x.n_race_granules == y.n_race_granules
+                assert np.array_equal(x.runs, y.runs)
+            sa.close()
+            sb.close()

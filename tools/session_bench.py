@@ -28,7 +28,11 @@ ap.add_argument("--chunk", type=int, default=4096, help="accesses per session ca
 ap.add_argument("--window", type=int, default=0)
 ap.add_argument("--nshards", type=int, default=1)
 ap.add_argument("--shard-block", type=int, default=0)
+ap.add_argument("--pipelined", action="store_true",
+                help="submit/finish: plan call i+1 on the host while the GPU checks call i (one shard)")
 a = ap.parse_args()
+if a.pipelined and a.nshards != 1:
+    raise SystemExit("--pipelined times one session (on N GPUs every shard pipelines on its own)")
 
 w = configs.make(a.config, a.size)
 ops, args = w.arrays(True)
@@ -37,6 +41,27 @@ cs.Lowering(full).cusan_lower_program(ops, args)
 ev = full.cusan_trace_read()
 acc_pos = np.flatnonzero(ev["kind"] == 0)
 cuts = [int(acc_pos[i]) for i in range(a.chunk, len(acc_pos), a.chunk)] + [len(ev)]
+
+if a.pipelined:
+    tr = cs.Trace(255)
+    ses = cs.Session(tr, window_events=a.window)
+    reps, start = [], 0
+    t0 = time.perf_counter()
+    for end in cuts:
+        tr.cusan_trace_append_events(ev[start:end])
+        r = ses.submit()
+        if r is not None:
+            reps.append(r)
+        start = end
+    reps.append(ses.finish())
+    secs = time.perf_counter() - t0
+    ses.close()
+    tot = sum(r.counters["tracked_bytes"] for r in reps)
+    kms = sum(r.counters["kernel_ms"] for r in reps)
+    print(json.dumps(dict(config=a.config, chunk_accesses=a.chunk, pipelined=True, calls=len(reps),
+                          tracked_bytes=tot, checked_gbs=tot / secs / 1e9, kernel_checked_gbs=tot / (kms / 1e3) / 1e9,
+                          seconds=secs, kernel_ms=kms, race_granules=sum(r.n_race_granules for r in reps))))
+    raise SystemExit(0)
 
 trs = [cs.Trace(255) for _ in range(a.nshards)]
 sess = [cs.Session(trs[s], window_events=a.window, nshards=a.nshards, shard=s, shard_block=a.shard_block)
