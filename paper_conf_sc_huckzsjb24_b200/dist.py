@@ -83,13 +83,26 @@ class ShardedSession:
                                device=device, **kw)
         self.last_shard_report: Report | None = None
 
-    def check(self) -> Report | None:
-        rep = self.session.check()
+    def _gather(self, rep: Report) -> Report | None:
         self.last_shard_report = rep
         out = gather_runs(rep.runs, rep.n_race_granules, self.comm_device, self.group)
         if out is None:
             return None
         return report_merge(out[0], out[1], self.max_runs)
+
+    def check(self) -> Report | None:
+        return self._gather(self.session.check())
+
+    def submit(self) -> Report | None:
+        """Pipelined check (cusan_session_submit on every rank): returns the previous call's merged
+        report on rank 0 (None elsewhere, and on the first call)."""
+        prev = self.session.submit()
+        has_prev = prev is not None          # the same on every rank: all ranks submit together
+        return self._gather(prev) if has_prev else None
+
+    def finish(self) -> Report | None:
+        rep = self.session.finish()
+        return self._gather(rep) if rep is not None else None
 
     def close(self):
         self.session.close()
