@@ -1,2 +1,5 @@
 python __graft_entry__.py build > /dev/null
-timeout 600 python -m pytest tests/test_gpu_dist.py -x -q > gpurun_out/pytest_dist.log 2>&1; echo rc=$?; tail -30 gpurun_out/pytest_dist.log
+timeout 300 python tools/sanitize_small.py 2>&1 | tail -2
+for t in memcheck synccheck racecheck; do
+timeout 1200 compute-sanitizer --tool $t --print-limit 20 python tools/sanitize_small.py > gpurun_out/san_$t.txt 2>&1; echo $t rc=$?; tail -4 gpurun_out/san_$t.txt
+done

@@ -41,4 +41,16 @@ for _ in range(10):
             n += 1
         ses.close()
         assert total == ref["n_race_granules"], flags
+        # pipelined calls (submit / finish) and a 2-shard block-cyclic session
+        for kw in (dict(), dict(nshards=2, shard=0, shard_block=64), dict(nshards=2, shard=1, shard_block=64)):
+            tr = cs.Trace(nf)
+            ses = cs.Session(tr, window_events=7, flags=flags, **kw)
+            for a, b in ((0, 40), (40, 90), (90, 120)):
+                tr.cusan_trace_append_events(ev[a:b])
+                r = ses.submit()
+                total -= r.n_race_granules if r is not None else 0
+            total -= ses.finish().n_race_granules
+            n += 1
+            ses.close()
+        assert total == -ref["n_race_granules"], flags       # 1 whole + 1 pipelined + 2 shard halves
 print("sanitize workloads ok:", n)
