@@ -1,5 +1,3 @@
 python __graft_entry__.py build > /dev/null
-timeout 300 python tools/sanitize_small.py 2>&1 | tail -2
-for t in memcheck synccheck racecheck; do
-timeout 1200 compute-sanitizer --tool $t --print-limit 20 python tools/sanitize_small.py > gpurun_out/san_$t.txt 2>&1; echo $t rc=$?; tail -4 gpurun_out/san_$t.txt
-done
+timeout 600 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; echo bench_rc=$?; tail -3 gpurun_out/bench.err; python -c "
+import json; d=json.load(open('gpurun_out/bench.json')); print(d['value'], d['e2e'], d['roofline']['frac'], d['clocks'])"
