@@ -278,9 +278,14 @@ int cusan_on_stream_wait_event(cusan_lowering* l, uint64_t stream, uint64_t even
 
 int cusan_on_stream_query(cusan_lowering* l, uint64_t stream, int success) {
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    if (!success) {            // no synchronisation, so no event and no (lazy) fiber either
+        if (stream == 0 || stream == STREAM_LEGACY || stream == STREAM_PER_THREAD || l->stream_fiber.count(stream))
+            return CUSAN_OK;
+        return fail(CUSAN_EINVAL, "unknown stream handle");
+    }
     uint32_t f = 0;
     int st = l->fiber_of(stream, &f);
-    if (st || !success) return st;
+    if (st) return st;
     return l->host_sync_stream(f);
 }
 

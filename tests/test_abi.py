@@ -163,6 +163,30 @@ def test_lowering_matches_oracle_lowering_configs(c):
         assert list(first_p) == first_o
 
 
+def test_failed_stream_query_uses_no_fiber():
+    """An unsuccessful cudaStreamQuery appends nothing (A9) and must not open the lazily created
+    per-thread default stream fiber either: the next fiber (an MPI request's) gets the same id in
+    the product and the oracle lowering (found by tools/fuzz_campaign.py)."""
+    from tracegen.program import Program, STREAM_PER_THREAD
+    for per_thread in (False, True):
+        p = Program()
+        p.default_stream_mode(per_thread)
+        a = p.malloc(512)
+        s = p.stream_create()
+        p.kernel(s, [(a, 1)])
+        p.stream_query(STREAM_PER_THREAD, False)
+        p.stream_query(0, False)
+        r = p.isend(a, 256)
+        p.wait(r)
+        ops, args = p.arrays()
+        ev_p, nf_p, first_p = _product_lower(ops, args)
+        ev_o, nf_o, first_o = _oracle_lower_first(ops, args)
+        assert nf_p == nf_o and np.array_equal(ev_p, ev_o) and list(first_p) == first_o
+    t = cs.Trace(8)
+    with pytest.raises(cs.CusanError):
+        cs.Lowering(t).cusan_on_stream_query(12345, 0)    # unknown handle, even when unsuccessful
+
+
 def test_lowering_matches_oracle_lowering_fuzz_and_listings():
     import listing_dsl
     progs = [l.program for l in listing_dsl.parse()]

@@ -1,3 +1,2 @@
 python __graft_entry__.py build > /dev/null
-timeout 600 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; echo bench_rc=$?; tail -3 gpurun_out/bench.err; python -c "
-import json; d=json.load(open('gpurun_out/bench.json')); print(d['value'], d['e2e'], d['roofline']['frac'], d['clocks'])"
+timeout 300 python tools/fuzz_campaign.py --minutes 1 --seed 7 > gpurun_out/fuzz_quick.json 2>gpurun_out/fuzz_quick.err; echo rc=$?; tail -3 gpurun_out/fuzz_quick.err; cat gpurun_out/fuzz_quick.json
