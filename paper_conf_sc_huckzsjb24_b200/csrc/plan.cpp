@@ -33,11 +33,15 @@
 
 namespace cusan {
 
-// Host threads for the planning loops (1 for small traces).
+// Host threads for the planning loops (1 for small traces).  One core stays free for the thread
+// that launches and waits on the device work (pipelined checks plan while a check runs).
+static unsigned max_plan_threads() {
+    const unsigned hw = std::max(1u, std::thread::hardware_concurrency());
+    return std::max(1u, std::min<unsigned>(hw > 2 ? hw - 1 : hw, 16));
+}
 static unsigned plan_threads(uint64_t work) {
     if (work < (1u << 15)) return 1;
-    const unsigned hw = std::max(1u, std::thread::hardware_concurrency());
-    return std::min<unsigned>(hw, 16);
+    return max_plan_threads();
 }
 
 // A persistent pool of planning threads (created on first use, never torn down): a parallel loop
@@ -92,7 +96,7 @@ class Pool {
 };
 
 static Pool& pool() {
-    static Pool* p = new Pool(std::min<unsigned>(std::max(1u, std::thread::hardware_concurrency()), 16) - 1);
+    static Pool* p = new Pool(max_plan_threads() - 1);
     return *p;
 }
 

@@ -1,3 +1,6 @@
 python __graft_entry__.py build > /dev/null
-timeout 1800 python tools/fuzz_campaign.py --minutes 25 --seed 11 > gpurun_out/fuzz_campaign.json 2>gpurun_out/fuzz_campaign.err; echo rc=$?; tail -3 gpurun_out/fuzz_campaign.err; python -c "
-import json; d=json.load(open('gpurun_out/fuzz_campaign.json')); print({k: d[k] for k in ('cases','checks','mismatches','racy_cases')}); print(d['first_failures'])"
+for i in 1 2; do
+timeout 600 python bench.py --no-cpu-baseline > gpurun_out/bench.json 2> gpurun_out/bench.err; echo bench_rc=$?; python -c "
+import json; d=json.load(open('gpurun_out/bench.json')); print(d['value'], d['e2e']['value'], d['e2e']['serial']['value'])"
+done
+timeout 600 python tools/e2e_pipeline_probe.py racy 2>&1 | tail -4
