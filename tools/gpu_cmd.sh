@@ -1,6 +1,7 @@
 python __graft_entry__.py build > /dev/null
-for i in 1 2; do
-timeout 600 python bench.py --no-cpu-baseline > gpurun_out/bench.json 2> gpurun_out/bench.err; echo bench_rc=$?; python -c "
-import json; d=json.load(open('gpurun_out/bench.json')); print(d['value'], d['e2e']['value'], d['e2e']['serial']['value'])"
+mkdir -p gpurun_out/r01_configs
+for c in 2 3 4 5; do
+  timeout 600 python bench.py --config $c > gpurun_out/r01_configs/bench_config${c}_racy.json 2>gpurun_out/r01_configs/err_${c}_racy.txt; echo c=$c racy rc=$?
+  timeout 600 python bench.py --config $c --clean --no-cpu-baseline > gpurun_out/r01_configs/bench_config${c}_clean.json 2>gpurun_out/r01_configs/err_${c}_clean.txt; echo c=$c clean rc=$?
 done
-timeout 600 python tools/e2e_pipeline_probe.py racy 2>&1 | tail -4
+timeout 600 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/bench_reference.json 2>gpurun_out/err_ref.txt; echo ref rc=$?
