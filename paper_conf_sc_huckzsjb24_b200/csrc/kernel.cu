@@ -110,6 +110,16 @@ __device__ __forceinline__ void emit_range(bool hit, uint32_t earlier_epoch, uin
     cache_insert((earlier_epoch & 0xffffffu) - 1u, later_id, gb, ge, lane, rc, k);
 }
 
+// Warp-collective: every lane with `hit` emits one run over the whole range [gb, ge) for its own
+// (earlier epoch, later event), one lane after another.
+__device__ __forceinline__ void emit_range_lanes(bool hit, uint32_t earlier_epoch, uint32_t later_id, uint64_t gb,
+                                                 uint64_t ge, int lane, RunCache& rc, const Ctx& k) {
+    for (unsigned m = __ballot_sync(FULL, hit); m; m &= m - 1) {
+        const int h = __ffs(m) - 1;
+        emit_range(true, __shfl_sync(FULL, earlier_epoch, h), __shfl_sync(FULL, later_id, h), gb, ge, lane, rc, k);
+    }
+}
+
 // ¬HB(earlier epoch e, later access of fiber f whose segment row is `row`)
 __device__ __forceinline__ bool unordered(uint32_t e, uint32_t f, const uint32_t* __restrict__ row) {
     if (!e) return false;
@@ -289,9 +299,13 @@ __global__ void __launch_bounds__(THREADS, CUSAN_MIN_BLOCKS)
 shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t total_tiles,
                     uint64_t total_weight, Ctx k, int force_lanes, unsigned long long* sched) {
     __shared__ uint32_t s_list[WARPS][MAXS];
+    __shared__ uint8_t s_slot[WARPS][256];
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
     uint32_t* lst = s_list[warp];
+    uint8_t* slot = s_slot[warp];
+    for (int i = lane; i < 256; i += 32) slot[i] = 0xFFu;
+    __syncwarp();
 #if CUSAN_TMA
     extern __shared__ __align__(128) unsigned char dsm[];
     unsigned char* wsm = dsm + (size_t)warp * TMA_WARP_BYTES;
@@ -414,50 +428,127 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                 continue;
             }
             // ---- pass 2: all cells of the range equal `c`: apply the window's accesses once -----
-            // the read set is kept in shared memory (ns entries); c.x = W
+            // 32 accesses at a time, lane l taking access q0 + l.  The state each access sees
+            // follows from the batch's pattern of writes and reads (ballots, __match_any_sync), so
+            // every happens-before test of a batch is one load per lane, issued in parallel.  The
+            // read set lives in shared memory (lst, ns entries, one per fiber; slot[fiber] = its
+            // index, 0xFF = absent); c.x = W.
             uint32_t ns = 0;
             if (c.y) {
                 if (is_spill(c.y)) {
                     const uint32_t* rp = rec_ptr(k, c.y);
                     ns = rec_n(rp[0]);
-                    for (uint32_t j = lane; j < ns; j += 32) lst[j] = rp[1 + j];
+                    for (uint32_t j = lane; j < ns; j += 32) {
+                        const uint32_t v = rp[1 + j];
+                        lst[j] = v;
+                        slot[v >> 24] = (uint8_t)j;
+                    }
                 } else {
-                    if (lane == 0) lst[0] = c.y;
+                    if (lane == 0) {
+                        lst[0] = c.y;
+                        slot[c.y >> 24] = 0;
+                    }
                     ns = 1;
                 }
                 __syncwarp();
             }
             const uint64_t gb = sp.abs_begin + x0, ge = gb + n;
             const uint32_t qe = sp.list_off + sp.list_cnt;
-            AccRec nxt = k.inc[sp.list_off];
-            for (uint32_t q = sp.list_off; q < qe; q++) {
-                const AccRec r = nxt;
-                if (q + 1 < qe) nxt = k.inc[q + 1];
+            const unsigned below = (1u << lane) - 1u;
+            for (uint32_t q0 = sp.list_off; q0 < qe; q0 += 32) {
+                const bool act = q0 + lane < qe;
+                AccRec r{0u, 0u};
+                if (act) r = k.inc[q0 + lane];
+                const bool isw = act && (r.segm >> 31);
+                const bool isr = act && !isw;
                 const uint32_t f = r.epoch >> 24;
                 const uint32_t later = (r.epoch & 0xffffffu) - 1u;
                 const uint32_t* row = k.segvc + (uint64_t)(r.segm & 0x7fffffffu) * k.F;
-                emit_range(unordered(c.x, f, row), c.x, later, gb, ge, lane, rc, k);
-                if (r.segm >> 31) {
-                    for (uint32_t j = 0; j < ns; j++) {
-                        const uint32_t v = lst[j];
-                        emit_range(unordered(v, f, row), v, later, gb, ge, lane, rc, k);
+                const unsigned wm = __ballot_sync(FULL, isw);
+                const unsigned rm = __ballot_sync(FULL, isr);
+                const unsigned pw = wm & below;
+                const int lw = pw ? 31 - __clz(pw) : -1;            // the last write before this access
+                const uint32_t w_ep = __shfl_sync(FULL, r.epoch, lw < 0 ? 0 : lw);
+                const uint32_t W = lw < 0 ? c.x : w_ep;
+                // (1) every access against the last write before it
+                emit_range_lanes(act && unordered(W, f, row), W, later, gb, ge, lane, rc, k);
+                // the next read by the same fiber in this batch (32 = none)
+                const unsigned same = __match_any_sync(FULL, isr ? f : 0x100u + (unsigned)lane);
+                const unsigned above = same & ~((2u << lane) - 1u);
+                const int nxt = above ? __ffs(above) - 1 : 32;
+                if (wm) {
+                    // (2) a write against the batch's reads since the last write before it that are
+                    //     the last read of their fiber before it
+                    if (rm) {
+                        const unsigned cand = isw ? (rm & below & ~(lw < 0 ? 0u : ((2u << lw) - 1u))) : 0u;
+                        unsigned hm = 0;
+#pragma unroll 8
+                        for (int p = 0; p < 32; p++) {
+                            const uint32_t ep = __shfl_sync(FULL, r.epoch, p);
+                            const int np = __shfl_sync(FULL, nxt, p);
+                            if (((cand >> p) & 1u) && np > lane && unordered(ep, f, row)) hm |= 1u << p;
+                        }
+                        for (;;) {                                   // one run per (read, write) hit
+                            const unsigned any = __ballot_sync(FULL, hm != 0);
+                            if (!any) break;
+                            const int h = __ffs(any) - 1;
+                            const int pr = __ffs(__shfl_sync(FULL, hm, h)) - 1;
+                            const uint32_t e = __shfl_sync(FULL, r.epoch, pr);
+                            const uint32_t l = __shfl_sync(FULL, later, h);
+                            emit_range(true, e, l, gb, ge, lane, rc, k);
+                            if (lane == h) hm &= hm - 1;
+                        }
                     }
-                    c.x = r.epoch;
-                    ns = 0;
-                    __syncwarp();                          // reads of lst before later writes
-                } else {
-                    int pos = -1;
-                    for (uint32_t b = 0; b < ns; b += 32) {
-                        const uint32_t j = b + lane;
-                        const unsigned m = __ballot_sync(FULL, j < ns && (lst[j] >> 24) == f);
-                        if (m) { pos = (int)(b + __ffs(m) - 1); break; }
+                    // (3) the first write of the batch against the incoming read set, except the
+                    //     fibers that read again in the batch before it
+                    if (ns) {
+                        const int l0 = __ffs(wm) - 1;
+                        const uint32_t f0 = __shfl_sync(FULL, f, l0);
+                        const uint32_t seg0 = __shfl_sync(FULL, r.segm & 0x7fffffffu, l0);
+                        const uint32_t later0 = __shfl_sync(FULL, later, l0);
+                        const uint32_t* row0 = k.segvc + (uint64_t)seg0 * k.F;
+                        const unsigned rb = rm & ((1u << l0) - 1u);
+                        for (uint32_t j0 = 0; j0 < ns; j0 += 32) {
+                            const uint32_t j = j0 + lane;
+                            const uint32_t v = j < ns ? lst[j] : 0u;
+                            bool shadowed = false;
+                            for (unsigned bb = rb; bb; bb &= bb - 1)
+                                shadowed |= (v >> 24) == __shfl_sync(FULL, f, __ffs(bb) - 1);
+                            emit_range_lanes(j < ns && !shadowed && unordered(v, f0, row0), v, later0, gb, ge,
+                                             lane, rc, k);
+                        }
                     }
-                    __syncwarp();                          // (ballots do not order memory)
-                    if (lane == 0) lst[pos >= 0 ? pos : ns] = r.epoch;
-                    if (pos < 0) ns++;
+                    // new state: W = the batch's last write, R = the reads after it (last per fiber)
+                    const int lwl = 31 - __clz(wm);
+                    c.x = __shfl_sync(FULL, r.epoch, lwl);
+                    const unsigned live = __ballot_sync(FULL, isr && lane > lwl && nxt == 32);
+                    __syncwarp();                          // reads of lst above before its rewrite
+                    for (uint32_t j = lane; j < ns; j += 32) slot[lst[j] >> 24] = 0xFFu;
+                    __syncwarp();
+                    if ((live >> lane) & 1u) {
+                        const uint32_t at = __popc(live & below);
+                        lst[at] = r.epoch;
+                        slot[f] = (uint8_t)at;
+                    }
+                    ns = __popc(live);
+                    __syncwarp();
+                } else if (rm) {
+                    // reads only: each fiber's last read of the batch replaces its entry or joins
+                    const bool last = isr && nxt == 32;
+                    const uint32_t pos = last ? slot[f] : 0xFFu;
+                    const unsigned app = __ballot_sync(FULL, last && pos == 0xFFu);
+                    __syncwarp();
+                    if (last) {
+                        const uint32_t at = pos != 0xFFu ? pos : ns + __popc(app & below);
+                        lst[at] = r.epoch;
+                        slot[f] = (uint8_t)at;
+                    }
+                    ns += __popc(app);
                     __syncwarp();
                 }
             }
+            for (uint32_t j = lane; j < ns; j += 32) slot[lst[j] >> 24] = 0xFFu;   // index empty again
+            __syncwarp();
             // ---- pass 3: stream the final cell out -----------------------------------------------
             if (sp.flags & SPAN_STORE) {
                 if (ns == 0) {

@@ -1,7 +1,5 @@
 python __graft_entry__.py build > /dev/null
-mkdir -p gpurun_out/r01_configs
-for c in 2 3 4 5; do
-  timeout 600 python bench.py --config $c > gpurun_out/r01_configs/bench_config${c}_racy.json 2>gpurun_out/r01_configs/err_${c}_racy.txt; echo c=$c racy rc=$?
-  timeout 600 python bench.py --config $c --clean --no-cpu-baseline > gpurun_out/r01_configs/bench_config${c}_clean.json 2>gpurun_out/r01_configs/err_${c}_clean.txt; echo c=$c clean rc=$?
-done
-timeout 600 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/bench_reference.json 2>gpurun_out/err_ref.txt; echo ref rc=$?
+timeout 900 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1; echo pytest_rc=$?; tail -5 gpurun_out/pytest_gpu.log
+timeout 600 python tools/quick_timing.py 2,3,4,5 1024,4096,16384 > gpurun_out/quick2.txt 2>&1; cat gpurun_out/quick2.txt | cut -c1-200
+timeout 600 python tools/fuzz_campaign.py --minutes 4 --seed 21 > gpurun_out/fuzz_quick.json 2>gpurun_out/fuzz_quick.err; python -c "
+import json; d=json.load(open('gpurun_out/fuzz_quick.json')); print({k: d[k] for k in ('cases','checks','mismatches','racy_cases')}); print(d['first_failures'][:3])"
