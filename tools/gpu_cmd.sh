@@ -1,5 +1,4 @@
 python __graft_entry__.py build > /dev/null
-timeout 900 python -m pytest tests -m gpu -x -q > gpurun_out/pytest_gpu.log 2>&1; echo pytest_rc=$?; tail -5 gpurun_out/pytest_gpu.log
-timeout 600 python tools/quick_timing.py 2,3,4,5 1024,4096,16384 > gpurun_out/quick2.txt 2>&1; cat gpurun_out/quick2.txt | cut -c1-200
-timeout 600 python tools/fuzz_campaign.py --minutes 4 --seed 21 > gpurun_out/fuzz_quick.json 2>gpurun_out/fuzz_quick.err; python -c "
-import json; d=json.load(open('gpurun_out/fuzz_quick.json')); print({k: d[k] for k in ('cases','checks','mismatches','racy_cases')}); print(d['first_failures'][:3])"
+timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/launches.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline --e2e-steps 1 > gpurun_out/b_ncu.log 2>&1; echo launches rc=$?
+timeout 2700 ncu --set full --clock-control none --import-source on -k regex:shadow_check_window --launch-skip 9 -c 9 -o gpurun_out/k1_c5 python tools/profile_k1.py --config 5 --nshards 1 --runs 1 > gpurun_out/ncu_c5.log 2>&1; echo full rc=$?; tail -4 gpurun_out/ncu_c5.log
+ls -la gpurun_out/*.ncu-rep
