@@ -1,4 +1,7 @@
 python __graft_entry__.py build > /dev/null
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file gpurun_out/launches.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline --e2e-steps 1 > gpurun_out/b_ncu.log 2>&1; echo launches rc=$?
-timeout 2700 ncu --set full --clock-control none --import-source on -k regex:shadow_check_window --launch-skip 9 -c 9 -o gpurun_out/k1_c5 python tools/profile_k1.py --config 5 --nshards 1 --runs 1 > gpurun_out/ncu_c5.log 2>&1; echo full rc=$?; tail -4 gpurun_out/ncu_c5.log
-ls -la gpurun_out/*.ncu-rep
+timeout 600 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; echo bench_rc=$?
+mkdir -p gpurun_out/r01_configs
+for c in 2 3 4 5; do
+  timeout 600 python bench.py --config $c > gpurun_out/r01_configs/bench_config${c}_racy.json 2>gpurun_out/r01_configs/err_${c}_racy.txt; echo c=$c racy rc=$?
+  timeout 600 python bench.py --config $c --clean --no-cpu-baseline > gpurun_out/r01_configs/bench_config${c}_clean.json 2>gpurun_out/r01_configs/err_${c}_clean.txt; echo c=$c clean rc=$?
+done
