@@ -10,7 +10,7 @@
  *   a1  vector-clock / segment pass (host)                             — cusan_plan_create
  *   a2  range → granule expansion, interval compaction, shard clip, windows (host) + upload
  *   a3  shadow check, one sm_100a kernel launch per window (device)    — cusan_plan_run
- *   a4  race-hit compaction into runs (kernel epilogue) + canonical merge (host)
+ *   a4  race-hit compaction into runs (in the kernel) + canonical merge (device sort / scan kernels)
  *   a5  report                                                          — cusan_report_*
  *
  * Conventions for every function:
