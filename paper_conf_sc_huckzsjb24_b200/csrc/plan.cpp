@@ -17,6 +17,8 @@
 //     `nshards` contiguous dense ranges of equal coverage weight (Σ granules × incidences), and this
 //     plan keeps the clip of its shard.  Windows are runs of `window_events` consecutive accesses;
 //     a window's spans are its incidences grouped by interval.
+#include <sched.h>
+
 #include <algorithm>
 #include <bitset>
 #include <chrono>
@@ -34,10 +36,26 @@
 namespace cusan {
 
 // Host threads for the planning loops (1 for small traces).  One core stays free for the thread
-// that launches and waits on the device work (pipelined checks plan while a check runs).
+// that launches and waits on the device work (pipelined checks plan while a check runs).  The cores
+// are those this process may run on (its affinity mask, which follows container cpusets), shared
+// among the ranks of the node when torchrun says how many there are (LOCAL_WORLD_SIZE), so 8 ranks
+// on one host do not each start a pool the size of the machine.  CUSAN_PLAN_THREADS overrides.
 static unsigned max_plan_threads() {
-    const unsigned hw = std::max(1u, std::thread::hardware_concurrency());
-    return std::max(1u, std::min<unsigned>(hw > 2 ? hw - 1 : hw, 16));
+    static const unsigned n = [] {
+        if (const char* e = std::getenv("CUSAN_PLAN_THREADS")) {
+            const long v = std::strtol(e, nullptr, 10);
+            if (v > 0) return (unsigned)std::min<long>(v, 256);
+        }
+        unsigned hw = std::max(1u, std::thread::hardware_concurrency());
+        cpu_set_t set;
+        if (sched_getaffinity(0, sizeof(set), &set) == 0) hw = std::max(1, CPU_COUNT(&set));
+        if (const char* e = std::getenv("LOCAL_WORLD_SIZE")) {
+            const long ranks = std::strtol(e, nullptr, 10);
+            if (ranks > 1) hw = std::max<unsigned>(1, hw / (unsigned)ranks);
+        }
+        return std::max(1u, std::min<unsigned>(hw > 2 ? hw - 1 : hw, 16));
+    }();
+    return n;
 }
 static unsigned plan_threads(uint64_t work) {
     if (work < (1u << 15)) return 1;
