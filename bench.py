@@ -226,7 +226,7 @@ def run_ours(args):
     import torch.distributed as dist
 
     import paper_conf_sc_huckzsjb24_b200 as cs
-    from paper_conf_sc_huckzsjb24_b200.dist import ShardedPlan, gather_runs
+    from paper_conf_sc_huckzsjb24_b200.dist import ShardedPlan, broadcast_trace, gather_runs
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -248,8 +248,11 @@ def run_ours(args):
     stream = torch.cuda.current_stream(dev)
 
     w, ops, args_, wname = workload(args)
-    tr = cs.Trace(255)
-    cs.Lowering(tr).cusan_lower_program(ops, args_)
+    if world == 1 or rank == 0:
+        tr = cs.Trace(255)
+        cs.Lowering(tr).cusan_lower_program(ops, args_)
+    if world > 1:      # rank 0 recorded the program; the other ranks receive its events
+        tr = broadcast_trace(tr if rank == 0 else None, device=comm_dev)
 
     def barrier():
         if world > 1:

@@ -1,7 +1,8 @@
 """Multi-GPU check: the shadow space is sharded by granule range, one shard per rank.
 
-Granules are independent, so every rank builds the same host plan from the same trace (no table
-broadcast is needed: the trace is the input each rank holds), checks only its shard on its own GPU
+Granules are independent, so every rank builds the same host plan from the same trace (each rank
+holds the trace, or the rank that recorded it broadcasts its events: broadcast_trace), checks only
+its shard on its own GPU
 with no communication inside the check, and the race runs are gathered to rank 0 — the one real
 exchange step — with torch.distributed (NCCL over NVLink on GPUs, gloo in CPU tests).  Rank 0
 stitches runs that abut across shard boundaries and sorts them canonically (cusan_report_merge).
@@ -37,6 +38,38 @@ def gather_runs(runs: np.ndarray, n_race: int, device: torch.device | None = Non
     allw = [p[: c * _RUN_U64].cpu().numpy().astype(np.uint64) for p, c in zip(parts, counts)]
     merged = np.concatenate(allw).view(RUN_DTYPE) if allw else np.zeros(0, RUN_DTYPE)
     return merged, int(sum(int(m[1]) for m in metas))
+
+
+def broadcast_trace(trace: Trace | None, src: int = 0, device: torch.device | None = None, group=None,
+                    first: int = 0) -> Trace:
+    """The recorded trace lives on rank ``src`` (the process that intercepted the application's
+    calls); every rank gets the same primitive events (24 B each, SURVEY §8(e) "broadcast the event
+    table") and returns a Trace holding them — ``src`` its own trace, the others a new Trace (or
+    ``trace`` extended, when given) with events ``first..`` of src's trace appended (same
+    max_fibers as src's).  One broadcast of (count, max_fibers), one of the raw event bytes (NCCL
+    over NVLink on GPUs)."""
+    from . import EVENT_DTYPE
+    dev = device if device is not None else torch.device("cpu")
+    me = dist.get_rank(group)
+    if me == src:
+        ev = trace.cusan_trace_read(first)
+        meta = torch.tensor([len(ev), trace.cusan_trace_size()[1]], dtype=torch.int64, device=dev)
+    else:
+        meta = torch.zeros(2, dtype=torch.int64, device=dev)
+    dist.broadcast(meta, dist.get_global_rank(group, src) if group is not None else src, group=group)
+    n, nf = int(meta[0]), int(meta[1])
+    if me == src:
+        buf = torch.from_numpy(np.ascontiguousarray(ev).view(np.uint8)).to(dev)
+    else:
+        buf = torch.empty(n * EVENT_DTYPE.itemsize, dtype=torch.uint8, device=dev)
+    if n:
+        dist.broadcast(buf, dist.get_global_rank(group, src) if group is not None else src, group=group)
+    if me == src:
+        return trace
+    out = trace if trace is not None else Trace(nf)
+    if n:
+        out.cusan_trace_append_events(buf.cpu().numpy().view(EVENT_DTYPE))
+    return out
 
 
 class ShardedPlan:

@@ -140,3 +140,58 @@ def runs_to_triples_in(runs, granules: set) -> set[tuple[int, int, int]]:
         for g in gs[lo:hi]:
             out.add((g, int(r["earlier"]), int(r["later"])))
     return out
+
+
+class HBGraph:
+    """The same happens-before graph as ``hb_closure`` for traces of any length, queried pair by
+    pair (forward search) instead of closed.  The acquire edges of a key are routed through a chain
+    of per-key nodes: RELEASE i links into the key's chain at its position, the chain runs forward in
+    trace order, a RELEASE_STORE starts a new chain, and ACQUIRE j links from the chain's last node —
+    so RELEASE i reaches ACQUIRE j through the chain iff i < j with no RELEASE_STORE on the key in
+    between (other than i itself being that store), exactly the edge set of ``hb_closure``."""
+
+    def __init__(self, events):
+        n = len(events)
+        kind = [int(k) for k in events["kind"]]
+        fib = [int(f) for f in events["fiber"]]
+        key = [int(a) for a in events["a"]]
+        self.n = n
+        self.succ: list[list[int]] = [[] for _ in range(n)]
+        self.t: list[int] = list(range(n))            # node time (trace position; chain nodes: creation)
+        last_on: dict[int, int] = {}
+        pending_fork: dict[int, list[int]] = {}
+        chain: dict[int, int] = {}                    # key -> last chain node
+        for i in range(n):
+            k = kind[i]
+            f = key[i] if k == EV_FORK else fib[i]
+            if f in last_on:
+                self.succ[last_on[f]].append(i)
+            last_on[f] = i
+            for src in pending_fork.pop(f, []):
+                self.succ[src].append(i)
+            if k == EV_FORK:
+                pending_fork.setdefault(fib[i], []).append(i)
+            elif k in (EV_RELEASE, EV_RELEASE_STORE):
+                node = len(self.succ)
+                self.succ.append([])
+                self.t.append(i)
+                if k == EV_RELEASE and key[i] in chain:
+                    self.succ[chain[key[i]]].append(node)
+                self.succ[i].append(node)
+                chain[key[i]] = node
+            elif k == EV_ACQUIRE and key[i] in chain:
+                self.succ[chain[key[i]]].append(i)
+
+    def hb(self, a: int, b: int) -> bool:
+        """a →hb b (a < b): b reachable from a over edges that never pass b's trace position."""
+        seen = {a}
+        stack = [a]
+        while stack:
+            x = stack.pop()
+            for y in self.succ[x]:
+                if y == b:
+                    return True
+                if y not in seen and self.t[y] < b:
+                    seen.add(y)
+                    stack.append(y)
+        return False

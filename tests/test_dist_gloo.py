@@ -125,3 +125,53 @@ def test_windowed_shards_balance_moved_cells(nshards):
     assert sum(p["tracked_bytes_shard"] for p in parts) == whole["tracked_bytes"]
     g = [p["shard_granules"] for p in parts]
     assert min(g) > 0.5 * max(g)
+
+
+def _bcast_worker(rank, world, port, q):
+    import sys
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import paper_conf_sc_huckzsjb24_b200 as cs
+        from paper_conf_sc_huckzsjb24_b200.dist import broadcast_trace
+        from tracegen import configs
+        w = configs.make(5, "small")
+        ops, args = w.arrays(True)
+        half = len(ops) // 2
+        mine = cs.Trace(255)                          # what every rank would have lowered itself
+        cs.Lowering(mine).cusan_lower_program(ops, args)
+        if rank == 0:                                 # only rank 0 records the program
+            tr = cs.Trace(255)
+            low = cs.Lowering(tr)
+            low.cusan_lower_program(ops[:half], args)
+            got = broadcast_trace(tr)
+            n0 = len(tr)
+            low.cusan_lower_program(ops[half:], args)
+            got = broadcast_trace(tr, first=n0)       # incremental: only the new events
+        else:
+            got = broadcast_trace(None)
+            got = broadcast_trace(got)
+        same = bool(np.array_equal(got.cusan_trace_read(), mine.cusan_trace_read()))
+        d_got = cs.describe(got, nshards=world, shard=rank, window_events=64)
+        d_mine = cs.describe(mine, nshards=world, shard=rank, window_events=64)
+        q.put(dict(rank=rank, same=same, plan_same=d_got == d_mine,
+                   fibers=got.cusan_trace_size()[1]))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_two_rank_trace_broadcast():
+    """Rank 0 records the program and broadcasts its events (whole, then incrementally); rank 1's
+    trace, and the shard plan it builds from it, equal what lowering the program itself gives."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_bcast_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert all(r["same"] and r["plan_same"] and r["fibers"] == 255 for r in res), res
