@@ -5,6 +5,9 @@ Integer work, so the bar is equality of the canonical run list and of the race-g
 """
 from __future__ import annotations
 
+import hashlib
+import os
+
 import numpy as np
 import pytest
 
@@ -205,6 +208,37 @@ def test_full_size_configs_sampled(c):
     got = {t for t in brute.runs_to_triples_in(rep.runs, sset)}
     want = brute.runs_to_triples(ref["runs"])
     assert got == want
+
+
+FULL_GOLDEN = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden", "full")
+
+
+@pytest.mark.parametrize("twin", ["racy", "clean"])
+@pytest.mark.parametrize("c", [1, 2, 3, 4, 5])
+def test_full_size_configs_exact(c, twin):
+    """Every BASELINE config at its full size, whole trace, bit-exact against the oracle's complete
+    report (every granule checked by oracle.c; written by tools/oracle_full_reports.py, which calls
+    only oracle/ and tracegen/).  The GPU runs in the bench launch configuration (4096-access
+    windows, torch workspace, a side stream) and, for the two largest traces, also as 8 granule-range
+    shards merged (result invariance under the GPU count)."""
+    g = np.load(os.path.join(FULL_GOLDEN, f"config{c}_{twin}.npz"))
+    w = configs.make(c, "full")
+    ops, args = w.arrays(twin == "racy")
+    tr, _ = lower_product(ops, args)
+    ev = tr.cusan_trace_read()
+    # the product lowering produced exactly the trace the oracle checked (oracle.lower)
+    assert hashlib.sha256(np.ascontiguousarray(ev).tobytes()).hexdigest() == str(g["events_sha256"])
+    ref = dict(n_race_granules=int(g["n_race_granules"]), n_runs=int(g["n_runs"]), runs=g["runs"])
+    assert (ref["n_race_granules"] > 0) == (twin == "racy")
+    import torch
+    s = torch.cuda.Stream()
+    rep = cs.check(tr, window_events=4096, workspace="torch", stream=s.cuda_stream)   # as bench.py runs it
+    assert rep.counters["tracked_bytes"] == int(g["tracked_bytes"])
+    assert_equal(rep, ref)
+    if c in (4, 5):
+        parts = [cs.check(tr, window_events=4096, nshards=8, shard=k) for k in range(8)]
+        merged = cs.report_merge(np.concatenate([p.runs for p in parts]), sum(p.n_race_granules for p in parts))
+        assert_equal(merged, ref)
 
 
 def test_torch_workspace_and_stream():

@@ -6,6 +6,9 @@ or from the mathematics of the definitions (subset / emptiness / relabelling / s
 """
 from __future__ import annotations
 
+import hashlib
+import os
+
 import numpy as np
 import pytest
 
@@ -292,3 +295,63 @@ def test_listings_reject_counterfactual_readings():
     assert _listing_failures(no_fork) > 0
     assert _listing_failures(back_edge) > 0
     assert _listing_failures(no_legacy) > 0
+
+
+# ------------------------------------------------------------------------------------------------
+# full-size goldens (tests/golden/full, written by tools/oracle_full_reports.py from oracle/ only)
+# ------------------------------------------------------------------------------------------------
+def test_hb_graph_equals_closure():
+    """brute.HBGraph (pairwise search, any trace length) == brute.hb_closure on tiny traces."""
+    rng = np.random.default_rng(9)
+    for _ in range(200):
+        nf = int(rng.integers(2, 6))
+        ev = fuzz.random_primitive_trace(rng, int(rng.integers(2, 50)), nf, n_keys=3, n_granules=16)
+        reach = brute.hb_closure(ev)
+        g = brute.HBGraph(ev)
+        for a in range(len(ev)):
+            for b in range(a + 1, len(ev)):
+                assert g.hb(a, b) == bool((reach[a] >> b) & 1)
+
+
+FULL_GOLDEN = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden", "full")
+
+
+@pytest.mark.parametrize("twin", ["racy", "clean"])
+@pytest.mark.parametrize("c", [1, 2, 3, 4, 5])
+def test_full_size_golden_reports(c, twin):
+    """The stored full-size oracle reports belong to today's generators (hash of the oracle's own
+    lowering of the full-size program) and every reported race is one by the paper's definition,
+    checked without vector clocks: earlier < later are accesses of different fibers, at least one a
+    write, both covering the whole run, and not ordered in the explicit HB graph.
+    Runs are canonical and maximal; the race-granule count is their total length; clean twins ∅."""
+    g = np.load(os.path.join(FULL_GOLDEN, f"config{c}_{twin}.npz"))
+    w = configs.make(c, "full")
+    ops, args = w.arrays(twin == "racy")
+    ev, nf = lower(ops, args)
+    assert hashlib.sha256(np.ascontiguousarray(ev).tobytes()).hexdigest() == str(g["events_sha256"])
+    assert int(g["n_events"]) == len(ev) and int(g["max_fibers"]) == nf
+    acc = ev[ev["kind"] == EV_ACCESS]
+    assert int(g["tracked_bytes"]) == 8 * int(np.sum(((acc["a"] + acc["b"] + np.uint64(7)) >> np.uint64(3))
+                                                     - (acc["a"] >> np.uint64(3))))
+    runs = g["runs"]
+    assert len(runs) == int(g["n_runs"])
+    assert int(np.sum(runs["g_end"] - runs["g_begin"])) == int(g["n_race_granules"])
+    if twin == "clean":
+        assert len(runs) == 0
+        return
+    assert len(runs) > 0
+    if c == 1:
+        assert len(runs) == 1 and int(g["n_race_granules"]) == 512     # closed form (SURVEY §8(c))
+    keys = [(int(r["later"]), int(r["earlier"]), int(r["g_begin"])) for r in runs]
+    assert keys == sorted(keys) and len(set(keys)) == len(keys)
+    for r0, r1 in zip(runs[:-1], runs[1:]):                         # maximal: no two runs abut
+        assert not (r0["later"] == r1["later"] and r0["earlier"] == r1["earlier"] and r0["g_end"] == r1["g_begin"])
+    graph = brute.HBGraph(ev)
+    for e, l in sorted({(int(r["earlier"]), int(r["later"])) for r in runs}):
+        a, b = ev[e], ev[l]
+        assert e < l and int(a["kind"]) == int(b["kind"]) == EV_ACCESS
+        assert int(a["fiber"]) != int(b["fiber"]) and (int(a["mode"]) == 1 or int(b["mode"]) == 1)
+        assert not graph.hb(e, l)
+    for r in runs:
+        for x in (ev[int(r["earlier"])], ev[int(r["later"])]):
+            assert int(x["a"]) >> 3 <= int(r["g_begin"]) and int(r["g_end"]) <= (int(x["a"]) + int(x["b"]) + 7) >> 3
