@@ -101,7 +101,7 @@ class ShardedPlan:
 
 class ShardedSession:
     """One rank's shard of a multi-GPU online check (f1 on N GPUs).  Every rank appends the same
-    events to its trace; its session keeps the shadow of its block-cyclic share of the granule
+    events to its trace (itself, or from the recording rank with pull()); its session keeps the shadow of its block-cyclic share of the granule
     space (granule g -> shard (g / shard_block) mod N: the address space is not known in advance,
     so a contiguous split cannot be balanced up front).  check() checks this rank's share of the
     new accesses, gathers the runs and returns the call's canonical report on rank 0 (None
@@ -114,7 +114,24 @@ class ShardedSession:
         self.max_runs = kw.pop("max_runs", 0)
         self.session = Session(trace, nshards=dist.get_world_size(group), shard=dist.get_rank(group),
                                device=device, **kw)
+        self.trace = trace
+        self._sent = 0
         self.last_shard_report: Report | None = None
+
+    def pull(self, src: int = 0) -> int:
+        """Bring every rank's trace up to date with rank ``src``'s, the one recording the
+        application: src broadcasts the events appended since its last pull (broadcast_trace with
+        ``first``), the others append them.  Call on every rank before check()/submit(); returns the
+        number of events moved."""
+        me = dist.get_rank(self.group)
+        n0 = len(self.trace)
+        broadcast_trace(self.trace, src=src, device=self.comm_device, group=self.group,
+                        first=self._sent if me == src else 0)
+        if me == src:
+            moved = n0 - self._sent
+            self._sent = n0
+            return moved
+        return len(self.trace) - n0
 
     def _gather(self, rep: Report) -> Report | None:
         self.last_shard_report = rep

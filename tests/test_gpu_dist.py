@@ -1,6 +1,7 @@
 """Multi-rank paths on the GPU: two processes (torch.distributed over gloo, both ranks on cuda:0 —
 the round's boxes have one GPU) run the sharded one-shot check (ShardedPlan) and the sharded
-online session (ShardedSession, check and submit/finish), gather the runs and compare rank 0's
+online session (ShardedSession, check and submit/finish; events recorded on rank 0 and pulled by
+rank 1 for check), gather the runs and compare rank 0's
 merged reports with the oracle.  The NCCL launch differs only in the process group backend and
 the device of the gathered tensors."""
 from __future__ import annotations
@@ -50,7 +51,9 @@ def _worker(rank, world, port, q):
         sb = ShardedSession(tb, window_events=64, shard_block=1 << 10)
         calls_a, calls_b = [], []
         for a, b in zip(cuts[:-1], cuts[1:]):
-            ta.cusan_trace_append_events(ev[a:b])
+            if rank == 0:                          # rank 0 records; rank 1 receives (pull)
+                ta.cusan_trace_append_events(ev[a:b])
+            assert sa.pull() == b - a
             tb.cusan_trace_append_events(ev[a:b])
             calls_a.append(sa.check())
             r = sb.submit()
