@@ -28,6 +28,8 @@ ap.add_argument("--chunk", type=int, default=4096, help="accesses per session ca
 ap.add_argument("--window", type=int, default=0)
 ap.add_argument("--nshards", type=int, default=1)
 ap.add_argument("--shard-block", type=int, default=0)
+ap.add_argument("--summary", action="store_true", help="omit the per-call list")
+ap.add_argument("--max-calls", type=int, default=0, help="stop after this many calls (0 = whole trace)")
 ap.add_argument("--pipelined", action="store_true",
                 help="submit/finish: plan call i+1 on the host while the GPU checks call i (one shard)")
 a = ap.parse_args()
@@ -41,6 +43,8 @@ cs.Lowering(full).cusan_lower_program(ops, args)
 ev = full.cusan_trace_read()
 acc_pos = np.flatnonzero(ev["kind"] == 0)
 cuts = [int(acc_pos[i]) for i in range(a.chunk, len(acc_pos), a.chunk)] + [len(ev)]
+if a.max_calls:
+    cuts = cuts[:a.max_calls]
 
 if a.pipelined:
     tr = cs.Trace(255)
@@ -93,4 +97,10 @@ out = dict(config=a.config, chunk_accesses=a.chunk, nshards=a.nshards, calls=len
            checked_gbs=tot / secs / 1e9, kernel_checked_gbs=tot / (kms / 1e3) / 1e9,
            kernel_dram_gbs_per_shard=cell / a.nshards / (kms / 1e3) / 1e9, seconds=secs, kernel_ms=kms,
            race_granules=sum(x["races"] for x in calls), per_call=calls)
+cs_ = sorted(x["seconds"] for x in calls)
+ks_ = sorted(x["kernel_ms"] for x in calls)
+out.update(call_ms_median=1e3 * cs_[len(cs_) // 2], call_ms_p90=1e3 * cs_[int(0.9 * (len(cs_) - 1))],
+           kernel_ms_median=ks_[len(ks_) // 2])
+if a.summary:
+    out.pop("per_call")
 print(json.dumps(out))
