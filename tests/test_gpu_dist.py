@@ -93,3 +93,54 @@ def test_two_ranks_sharded_plan_and_sessions_on_gpu():
         assert p.exitcode == 0
     assert res[0] == {"plan": True, "session": True, "submit": True}, res
     assert res[1] == {"others_none": True}, res
+
+
+def _nccl_worker(port, q):
+    import sys
+    sys.path.insert(0, ROOT)
+    import torch
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=dev)
+    try:
+        import oracle
+        import paper_conf_sc_huckzsjb24_b200 as cs
+        from paper_conf_sc_huckzsjb24_b200.dist import ShardedPlan, ShardedSession, broadcast_trace
+        from tracegen import configs
+        w = configs.make(5, "small")
+        ops, args = w.arrays(True)
+        tr = cs.Trace(255)
+        cs.Lowering(tr).cusan_lower_program(ops, args)
+        ev = tr.cusan_trace_read()
+        ref = oracle.check_events(ev, 256)
+        got = broadcast_trace(tr, device=dev)
+        rep = ShardedPlan(got, comm_device=dev, window_events=97).run()
+        res = {"plan": rep.n_race_granules == ref["n_race_granules"] > 0
+               and np.array_equal(rep.runs, ref["runs"].astype(rep.runs.dtype))}
+        t2 = cs.Trace(255)
+        ses = ShardedSession(t2, comm_device=dev, window_events=64)
+        t2.cusan_trace_append_events(ev)
+        res["pull"] = ses.pull() == len(ev)
+        r2 = ses.check()
+        ses.close()
+        res["session"] = r2.n_race_granules == ref["n_race_granules"] and np.array_equal(r2.runs, rep.runs)
+        q.put(res)
+    except Exception as e:                         # pragma: no cover - reported to the parent
+        q.put({"error": repr(e)})
+    finally:
+        dist.destroy_process_group()
+
+
+def test_nccl_collectives_on_one_gpu():
+    """The NCCL code path of the multi-GPU check (CUDA tensors in broadcast_trace, gather_runs,
+    ShardedPlan, ShardedSession.pull) in a one-rank NCCL group — the only NCCL group a one-GPU box
+    can form; the multi-rank logic itself is covered over gloo above."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    p = ctx.Process(target=_nccl_worker, args=(_free_port(), q))
+    p.start()
+    res = q.get(timeout=300)
+    p.join(timeout=60)
+    assert p.exitcode == 0
+    assert res == {"plan": True, "pull": True, "session": True}, res
