@@ -298,10 +298,11 @@ def check(trace: Trace, workspace: str | None = None, **kw) -> Report:
 
 
 def pipelined_checks(make_trace, steps: int, device: int = 0, **kw):
-    """Check `steps` traces one after another with the host and the GPU overlapped: while the GPU
-    checks trace i (a3-a5), a host thread builds trace i+1 (`make_trace(i+1)`, e.g. lowering the
-    next batch of recorded calls, a0) and its plan (a1, a2).  This is how an online checker keeps
-    both busy.  Every plan's tables are uploaded (host -> device) when it is bound, after the
+    """Check `steps` traces one after another with the host and the GPU overlapped, as a
+    three-stage pipeline: while the GPU checks trace i (a3-a5), one host thread plans trace i+1
+    (a1, a2) and another builds trace i+2 (`make_trace(i+2)`, e.g. lowering the next batch of
+    recorded calls, a0), so a step costs the slowest stage rather than their sum.  This is how an
+    online checker keeps host and GPU busy.  Every plan's tables are uploaded (host -> device) when it is bound, after the
     previous plan's run completed, and every run downloads its report, so each step still pays
     its own transfers.  All plans share one workspace from PyTorch's caching allocator (a plan's
     shadow and records are scratch for its own run).  Yields (trace, report) per step; kw as for
@@ -312,17 +313,21 @@ def pipelined_checks(make_trace, steps: int, device: int = 0, **kw):
     kw = dict(kw)
     kw["flags"] = kw.get("flags", 0) | CUSAN_CHECK_DEFER_WORKSPACE
 
-    def prepare(i):
-        tr = make_trace(i)
-        return tr, Plan(tr, device=device, **kw)
-
     ws = None
-    with ThreadPoolExecutor(1) as ex:
-        nxt = ex.submit(prepare, 0) if steps > 0 else None
+    with ThreadPoolExecutor(1) as lower_ex, ThreadPoolExecutor(1) as plan_ex:
+        traces = {j: lower_ex.submit(make_trace, j) for j in range(min(2, steps))}
+
+        def prepare(j):
+            tr = traces.pop(j).result()
+            return tr, Plan(tr, device=device, **kw)
+
+        nxt = plan_ex.submit(prepare, 0) if steps > 0 else None
         for i in range(steps):
             tr, p = nxt.result()
+            if i + 2 < steps:
+                traces[i + 2] = lower_ex.submit(make_trace, i + 2)
             if i + 1 < steps:
-                nxt = ex.submit(prepare, i + 1)
+                nxt = plan_ex.submit(prepare, i + 1)
             need = max(p.workspace_bytes(), 256)
             if ws is None or ws.numel() < need:
                 ws = None
