@@ -41,7 +41,11 @@ struct cusan_lowering {
     uint32_t next_fiber = 2;
     std::set<uint32_t> mpi_free;                           // pool of completed request fibers
     std::unordered_map<uint64_t, uint32_t> req_fiber;
-    std::map<uint64_t, std::pair<uint64_t, int>> allocs;   // base -> (size, kind)
+    struct Alloc {
+        uint64_t base, size;
+        int kind;
+    };
+    std::vector<Alloc> allocs;                             // registered allocations, sorted by base
     std::unordered_map<uint64_t, uint32_t> thread_fiber;   // host thread -> fiber (thread 0 -> 0)
     std::unordered_map<uint64_t, uint32_t> ptds;           // host thread -> per-thread default stream
     uint64_t thread = 0;                                   // calling host thread
@@ -65,12 +69,23 @@ struct cusan_lowering {
 
     // --- helpers -------------------------------------------------------------------------------
     // allocation containing p (TypeART's extent lookup)
-    const std::pair<const uint64_t, std::pair<uint64_t, int>>* find(uint64_t p) const {
-        auto it = allocs.upper_bound(p);
+    // (the allocation with the greatest base <= p, if it contains p; a flat sorted array: lookups
+    // happen for every kernel argument, registrations rarely)
+    const Alloc* find(uint64_t p) const {
+        auto it = std::upper_bound(allocs.begin(), allocs.end(), p,
+                                   [](uint64_t x, const Alloc& a) { return x < a.base; });
         if (it == allocs.begin()) return nullptr;
         --it;
-        if (p >= it->first && p < it->first + it->second.first) return &*it;
+        if (p >= it->base && p - it->base < it->size) return &*it;
         return nullptr;
+    }
+    void add_alloc(uint64_t base, uint64_t size, int kind) {
+        auto it = std::lower_bound(allocs.begin(), allocs.end(), base,
+                                   [](const Alloc& a, uint64_t x) { return a.base < x; });
+        if (it != allocs.end() && it->base == base)
+            *it = {base, size, kind};                      // re-registration replaces
+        else
+            allocs.insert(it, {base, size, kind});
     }
     int new_fiber(uint32_t* f) {
         uint32_t mf = 0;
@@ -197,7 +212,7 @@ int cusan_lowering_fibers(const cusan_lowering* l, uint32_t* n) {
 int cusan_on_malloc(cusan_lowering* l, uint64_t ptr, uint64_t size, enum cusan_mem_kind kind) {
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
     if ((unsigned)kind > 3) return fail(CUSAN_EINVAL, "bad memory kind");
-    l->allocs[ptr] = {size, (int)kind};   // allocation is not an access
+    l->add_alloc(ptr, size, (int)kind);   // allocation is not an access
     return CUSAN_OK;
 }
 
@@ -238,7 +253,7 @@ int cusan_on_kernel(cusan_lowering* l, uint64_t stream, uint32_t nargs, const ui
         if (!a) continue;
         if (modes[i] > 2) return fail(CUSAN_EINVAL, "bad argument mode");
         int mode = modes[i] == 0 ? CUSAN_READ : CUSAN_WRITE;   // RW -> WRITE
-        if ((st = l->access(f, mode, a->first, a->second.first))) return st;
+        if ((st = l->access(f, mode, a->base, a->size))) return st;
     }
     return l->epilogue(f);
 }
@@ -312,7 +327,7 @@ int cusan_on_memset(cusan_lowering* l, uint64_t ptr, uint64_t n, int async, uint
     auto* a = l->find(ptr);
     if (l->tracked(ptr, n) && (st = l->access(f, CUSAN_WRITE, ptr, n))) return st;
     if ((st = l->epilogue(f))) return st;
-    if (!async && a && a->second.second == CUSAN_MEM_PINNED)
+    if (!async && a && a->kind == CUSAN_MEM_PINNED)
         return l->sync(CUSAN_ACQUIRE, l->H(), K_stream(f));
     return CUSAN_OK;
 }
