@@ -272,8 +272,10 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
             }
         }
         c.n_segments = hp.nseg;
+        tick("a1 (thread)");
         return {CUSAN_OK, ""};
     };
+    tick("acc scan");
     const bool concurrent = n_acc >= (1u << 12);
     std::future<std::pair<int, std::string>> a1_done;
     std::pair<int, std::string> a1_status{CUSAN_OK, ""};
@@ -308,7 +310,9 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
                 ek.push_back(hp.acc_g1[k]);
                 eid.push_back((uint32_t)(2 * k + 1));
             }
+        tick("a2 endpoints");
         radix_sort_pairs(ek, eid);
+        tick("a2 sort");
         B.reserve(ek.size());
         for (size_t i = 0; i < ek.size(); i++) {
             if (i == 0 || ek[i] != ek[i - 1]) B.push_back(ek[i]);
