@@ -211,8 +211,15 @@ int cusan::device_info(int device, int* max_blocks) {
 static int plan_device_setup(cusan_plan* p) {
     HostPlan& hp = p->hp;
     const cusan_check_opts& o = hp.opts;
+    const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
+    auto tick = [t0 = std::chrono::steady_clock::now(), dbg](const char* what) {
+        if (dbg)
+            std::fprintf(stderr, "plan_device_setup: %-12s %8.3f ms\n", what,
+                         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+    };
     int st0 = device_info(o.device, &p->max_blocks);
     if (st0) return st0;
+    tick("device info");
     p->device = o.device;
     p->stream = (cudaStream_t)o.stream;
 
@@ -222,6 +229,7 @@ static int plan_device_setup(cusan_plan* p) {
     p->wins = st.wins;
     p->need_shadow = st.need_shadow;
     p->shadow_cell_bytes = st.cell_bytes;
+    tick("span tables");
 
     // workspace layout
     p->heap_cap = hp.rec_units + (1ull << 16);             // pre-assigned records + lane-path room
@@ -257,8 +265,10 @@ static int plan_device_setup(cusan_plan* p) {
                      p->ds.size() * sizeof(DSpan);
     hp.ctr.shadow_bytes = p->need_shadow ? hp.shadow_cells * sizeof(uint2) : 0;
     hp.ctr.workspace_bytes = p->ws_bytes;
-    CK(cudaEventCreate(&p->ev0));
-    CK(cudaEventCreate(&p->ev1));
+    tick("layout");
+    // (the timing events are created at the first run, on the thread that runs the plan:
+    // cudaEventCreate waits while another thread of the process synchronises with the device, so
+    // creating them here would stall a plan prepared while the previous check runs)
     if (o.workspace) return plan_bind(p, (char*)o.workspace, o.workspace_bytes);
     if (o.flags & CUSAN_CHECK_DEFER_WORKSPACE) return CUSAN_OK;   // caller binds later
     cudaError_t me = cudaMalloc((void**)&p->own, std::max<uint64_t>(off, ALIGN));
@@ -288,7 +298,8 @@ static int plan_bind(cusan_plan* p, char* ws, uint64_t bytes) {
     CK(cudaMemcpyAsync(p->d_inc, hp.inc.data(), hp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, p->stream));
     CK(cudaMemcpyAsync(p->d_segvc, hp.segvc.data(), hp.segvc.size() * sizeof(uint32_t), cudaMemcpyHostToDevice, p->stream));
     CK(cudaMemcpyAsync(p->d_spans, p->ds.data(), p->ds.size() * sizeof(DSpan), cudaMemcpyHostToDevice, p->stream));
-    CK(cudaStreamSynchronize(p->stream));
+    // no wait: the kernels follow on the same stream, and the page-locked tables live until the
+    // plan is destroyed (which synchronises the stream)
     p->bound = true;
     return CUSAN_OK;
 }
@@ -300,6 +311,8 @@ static int launch_all(cusan_plan* p) {
     p->counter_init[C_HEAP] = p->hp.rec_units;
     CK(cudaMemcpyAsync(p->d_counters, p->counter_init.data(), p->counter_init.size() * sizeof(unsigned long long),
                        cudaMemcpyHostToDevice, p->stream));
+    if (!p->ev0) CK(cudaEventCreate(&p->ev0));
+    if (!p->ev1) CK(cudaEventCreate(&p->ev1));
     CK(cudaEventRecord(p->ev0, p->stream));
     Ctx k;
     k.inc = p->d_inc;
@@ -447,7 +460,10 @@ int cusan_plan_run(cusan_plan* p, cusan_report** out) {
 
 int cusan_plan_destroy(cusan_plan* p) {
     if (!p) return fail(CUSAN_EINVAL, "plan is null");
-    if (p->stream) cudaStreamSynchronize(p->stream);
+    if (p->bound || p->stream) {          // pending uploads / work on the plan's stream
+        cudaSetDevice(p->device);
+        cudaStreamSynchronize(p->stream);
+    }
     delete p;
     return CUSAN_OK;
 }

@@ -26,6 +26,8 @@
 //   comparison with the left neighbour, run heads sized from the continuation mask).  Both paths
 //   feed a 32-entry per-warp run cache (one entry per lane) that extends runs across steps and
 //   ranges before appending them to global memory.
+#include <atomic>
+
 #include "kernel.cuh"
 
 using namespace cusan;
@@ -662,7 +664,26 @@ cudaError_t launch_copy_cells(uint32_t grid, cudaStream_t stream, const uint2* s
     return cudaGetLastError();
 }
 
+// Once per device: setting a function attribute while that kernel runs waits for it, so a plan
+// prepared on another host thread while a check runs (pipelined checks) would stall here.
 cudaError_t shadow_check_blocks_per_sm(int* per_sm) {
+    static std::atomic<int> known[256];
+    int dev = 0;
+    cudaError_t e0 = cudaGetDevice(&dev);
+    if (e0 != cudaSuccess) return e0;
+    if (dev >= 0 && dev < 256) {
+        const int k = known[dev].load(std::memory_order_acquire);
+        if (k > 0) {
+            *per_sm = k;
+            return cudaSuccess;
+        }
+    }
+    cudaError_t e1 = shadow_check_blocks_per_sm_query(per_sm);
+    if (e1 == cudaSuccess && dev >= 0 && dev < 256 && *per_sm > 0) known[dev].store(*per_sm, std::memory_order_release);
+    return e1;
+}
+
+cudaError_t shadow_check_blocks_per_sm_query(int* per_sm) {
     if (DYN_SMEM) {
         cudaError_t e = cudaFuncSetAttribute(shadow_check_window, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                              (int)DYN_SMEM);

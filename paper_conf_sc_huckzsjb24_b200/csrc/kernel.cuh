@@ -121,7 +121,8 @@ cudaError_t launch_shadow_check(uint32_t grid, cudaStream_t stream, const DSpan*
 cudaError_t launch_copy_cells(uint32_t grid, cudaStream_t stream, const uint2* src, uint2* dst,
                               const CopySeg* segs, uint32_t nseg, uint64_t total, uint32_t* heap);
 // resident blocks of K1 per SM (sets K1's dynamic shared memory limit first)
-cudaError_t shadow_check_blocks_per_sm(int* per_sm);
+cudaError_t shadow_check_blocks_per_sm(int* per_sm);        // cached per device
+cudaError_t shadow_check_blocks_per_sm_query(int* per_sm);  // sets the smem attribute, asks the occupancy API
 
 // ---- host helpers shared by check_api.cpp and session.cpp -----------------------------------------
 // Device-side span tables: per window its spans plus a sentinel, with range / weight prefixes.
