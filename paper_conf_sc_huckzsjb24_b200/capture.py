@@ -17,11 +17,17 @@ side streams with cudaStreamNonBlocking, so they are registered as non-blocking 
 the legacy default stream.  A host-blocking device->host copy (`.cpu()`, `.item()`) is a kernel on
 the current stream followed by a stream synchronisation, which is what PyTorch does.
 
-Point-to-point communication (`isend`, `irecv`, `send`, `recv`) can be recorded with
-`Capture.isend` / `irecv` / `send` / `recv` / `wait`: MPI semantics (a fiber per request, completed
-by the wait) — or, for NCCL (`stream_ordered=True`), NCCL's: the communication
-runs on a communication stream that waits on the current stream and the wait makes the current
-stream wait.
+Point-to-point communication through `torch.distributed` (`isend`, `irecv`, `send`, `recv`,
+`batch_isend_irecv`) is recorded automatically inside a capture: the functions are wrapped for its
+duration and the `Work` handles they return record the completion when waited on (or when
+`is_completed()` first returns True, MPI_Test).  Two semantics, by the process group's backend:
+MPI's for host-driven backends (a request fiber, completed by the wait) and
+NCCL's for `nccl` (the transfer runs on a communication stream that waits on the current stream,
+and `wait()` makes the current stream wait on it) — so a kernel that touches the buffer before
+the wait races with the transfer, as in Fig. 6A.  The same records can be made
+by hand with `Capture.isend` / `irecv` / `send` / `recv` / `wait` (e.g. for another communication
+library).  Collectives (`c10d::allreduce_` …) are recorded as an operation on the current stream
+(NCCL's stream-ordered semantics for synchronous collectives).
 """
 from __future__ import annotations
 
@@ -37,6 +43,7 @@ from . import Report, Trace, Lowering, check
 _aten = torch.ops.aten
 _COPY_OPS = ("aten::copy_", "aten::_to_copy", "aten::_local_scalar_dense", "aten::_copy_from",
              "aten::_copy_from_and_resize")
+_P2P_OPS = ("c10d::send", "c10d::recv_", "c10d::recv_any_source_")
 _ACTIVE: "Capture | None" = None
 _HOOKS_INSTALLED = False
 
@@ -86,7 +93,10 @@ class Capture:
         rep = cap.check()            # GPU happens-before race check of what ran
     """
 
-    def __init__(self, max_fibers: int = 255):
+    def __init__(self, max_fibers: int = 255, intercept_distributed: bool = True):
+        self.intercept_distributed = intercept_distributed
+        self._patched: list[tuple[Any, str, Any]] = []
+        self._in_p2p = False
         self.trace = Trace(max_fibers)
         self.low = Lowering(self.trace)
         self.streams: set[int] = {0}
@@ -105,6 +115,8 @@ class Capture:
         _install_hooks()
         torch.cuda.synchronize()                     # work issued before the capture is complete
         _ACTIVE = self
+        if self.intercept_distributed:
+            self._patch_distributed()
         self._mode = _Dispatch(self)
         self._mode.__enter__()
         return self
@@ -113,6 +125,9 @@ class Capture:
         global _ACTIVE
         self._mode.__exit__(*exc)
         self._mode = None
+        for mod, name, fn in reversed(self._patched):
+            setattr(mod, name, fn)
+        self._patched.clear()
         _ACTIVE = None
         return False
 
@@ -158,6 +173,8 @@ class Capture:
     def _on_op(self, func, args, kwargs, out):
         schema = func._schema
         name = schema.name
+        if self._in_p2p and name in _P2P_OPS:
+            return                                    # recorded by the torch.distributed wrapper
         # allocation only (no kernel touches the memory) / tensors passed only for their shape
         alloc_only = name in ("aten::empty", "aten::empty_like", "aten::empty_strided", "aten::new_empty",
                               "aten::new_empty_strided")
@@ -238,3 +255,104 @@ class Capture:
 
     def recv(self, tensor: torch.Tensor):
         self.low.cusan_on_mpi_recv(self._storage(tensor), tensor.untyped_storage().nbytes())
+
+    # ---- torch.distributed interception --------------------------------------------------------------
+    def _patch_distributed(self):
+        import torch.distributed as dist
+        if not dist.is_available():
+            return
+        import torch.distributed.distributed_c10d as c10d
+        cap = self
+
+        def nccl(group) -> bool:
+            try:
+                return dist.get_backend(group) == "nccl"
+            except Exception:                          # no default group yet
+                return False
+
+        def start(tensor, write, group):
+            if not isinstance(tensor, torch.Tensor) or not tensor.is_cuda:
+                return None                            # host tensors are not tracked
+            return cap._p2p(tensor, write, nccl(group))
+
+        def call(fn, *a, **k):
+            prev, cap._in_p2p = cap._in_p2p, True
+            try:
+                return fn(*a, **k)
+            finally:
+                cap._in_p2p = prev
+
+        orig = {n: getattr(c10d, n) for n in ("isend", "irecv", "send", "recv", "batch_isend_irecv")}
+
+        def nonblocking(name, write):
+            def wrapped(tensor, *a, **k):
+                if cap._in_p2p:                        # inside batch_isend_irecv: recorded there
+                    return orig[name](tensor, *a, **k)
+                h = start(tensor, write, k.get("group", a[1] if len(a) > 1 else None))
+                work = call(orig[name], tensor, *a, **k)
+                return _Work(work, cap, [h] if h else [])
+            wrapped.__name__ = name
+            return wrapped
+
+        def blocking(name, write):
+            def wrapped(tensor, *a, **k):
+                group = k.get("group", a[1] if len(a) > 1 else None)
+                out = call(orig[name], tensor, *a, **k)
+                if isinstance(tensor, torch.Tensor) and tensor.is_cuda:
+                    if nccl(group):                    # stream-ordered transfer, waited on
+                        cap.wait(cap._p2p(tensor, write, True))
+                    else:                              # host-blocking (MPI_Send / MPI_Recv)
+                        (cap.recv if write else cap.send)(tensor)
+                return out
+            wrapped.__name__ = name
+            return wrapped
+
+        def batch(p2p_op_list):
+            handles = []
+            for op in p2p_op_list:
+                write = getattr(op.op, "__name__", "") == "irecv"
+                h = start(op.tensor, write, op.group)
+                if h:
+                    handles.append(h)
+            works = call(orig["batch_isend_irecv"], p2p_op_list)
+            return [_Work(w, cap, handles) for w in works]
+
+        repl = {"isend": nonblocking("isend", 0), "irecv": nonblocking("irecv", 1),
+                "send": blocking("send", 0), "recv": blocking("recv", 1), "batch_isend_irecv": batch}
+        for mod in (c10d, dist):
+            for name, fn in repl.items():
+                if getattr(mod, name, None) is orig[name]:
+                    self._patched.append((mod, name, orig[name]))
+                    setattr(mod, name, fn)
+
+
+class _Work:
+    """A torch.distributed Work whose completion (wait, or is_completed() returning True) is
+    recorded in the capture: MPI_Wait / MPI_Test(success) for request fibers, the current stream
+    waiting on the transfer for NCCL.  Everything else is the wrapped Work's."""
+
+    def __init__(self, work, cap: Capture, handles: list):
+        self._work = work
+        self._cap = cap
+        self._handles = handles
+
+    def _complete(self):
+        for h in self._handles:
+            if not h[0].endswith("done"):
+                self._cap.wait(h)
+        self._handles[:] = [(k + "-done", v) for k, v in self._handles]
+
+    def wait(self, *a, **k):
+        out = self._work.wait(*a, **k) if self._work is not None else True
+        if _ACTIVE is self._cap:
+            self._complete()
+        return out
+
+    def is_completed(self):
+        done = self._work.is_completed() if self._work is not None else True
+        if done and _ACTIVE is self._cap:
+            self._complete()
+        return done
+
+    def __getattr__(self, name):
+        return getattr(self._work, name)

@@ -90,3 +90,73 @@ def test_nccl_style_p2p_is_stream_ordered():
         x.add_(1)
         torch.cuda.synchronize()
     assert _parity(cap).n_race_granules == 0
+
+
+def _dist_worker(port, q):
+    import os
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    sys.path.insert(0, root)
+    sys.path.insert(0, os.path.join(root, "tests"))
+    import torch.distributed as dist
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=dev)
+    res = {}
+    try:
+        from paper_conf_sc_huckzsjb24_b200.capture import Capture as Cap
+        n = 1 << 14
+        for name, fixed in (("racy", False), ("fixed", True)):
+            torch.cuda.synchronize()
+            with Cap() as cap:
+                x = torch.ones(n, device="cuda")
+                y = torch.zeros(n, device="cuda")
+                ops = [dist.P2POp(dist.isend, x, 0), dist.P2POp(dist.irecv, y, 0)]
+                works = dist.batch_isend_irecv(ops)   # recorded by the capture, no manual calls
+                if fixed:
+                    for w in works:
+                        w.wait()                      # current stream waits on the transfer
+                x.add_(1)                             # writes the buffer being sent
+                s = y.sum()                           # reads the buffer being received
+                for w in works:
+                    w.wait()
+                torch.cuda.synchronize()
+            rep = cap.check()
+            ref = oracle.check_events(cap.trace.cusan_trace_read(), 255, threads=2)
+            res[name] = dict(races=rep.n_race_granules, runs=rep.n_runs,
+                             parity=rep.n_race_granules == ref["n_race_granules"]
+                             and bool(np.array_equal(rep.runs, ref["runs"].astype(rep.runs.dtype))),
+                             value=float(s), patched_back=dist.isend.__module__ == "torch.distributed.distributed_c10d")
+        q.put(res)
+    except Exception as e:                          # pragma: no cover - reported to the parent
+        q.put({"error": repr(e)})
+    finally:
+        dist.destroy_process_group()
+
+
+def test_torch_distributed_p2p_is_captured():
+    """torch.distributed P2P inside a capture is recorded without manual calls (NCCL semantics in
+    a one-rank NCCL group, exchange with itself): a kernel writing the send buffer and one reading
+    the receive buffer before the works are waited on race with the transfer (Fig. 6A in
+    PyTorch/NCCL form); waiting first orders them."""
+    import socket
+
+    import torch.multiprocessing as mp
+    sk = socket.socket()
+    sk.bind(("127.0.0.1", 0))
+    port = sk.getsockname()[1]
+    sk.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    p = ctx.Process(target=_dist_worker, args=(port, q))
+    p.start()
+    res = q.get(timeout=300)
+    p.join(timeout=60)
+    assert p.exitcode == 0 and "error" not in res, res
+    n = 1 << 14
+    assert res["racy"]["parity"] and res["fixed"]["parity"], res
+    # racy: (isend read, add_ write) over x and (irecv write, sum read) over y
+    assert res["racy"]["races"] == 2 * n * 4 // 8 and res["racy"]["runs"] == 2, res
+    assert res["fixed"]["races"] == 0 and res["fixed"]["value"] == n, res
+    assert res["racy"]["patched_back"] and res["fixed"]["patched_back"], res
