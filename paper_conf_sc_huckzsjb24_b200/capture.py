@@ -28,10 +28,19 @@ the wait races with the transfer, as in Fig. 6A.  The same re
 by hand with `Capture.isend` / `irecv` / `send` / `recv` / `wait` (e.g. for another communication
 library).  Collectives (`c10d::allreduce_` …) are recorded as an operation on the current stream
 (NCCL's stream-ordered semantics for synchronous collectives).
+
+Host threads: every Python thread that issues CUDA work
+inside a capture is its own host fiber (`cusan_on_thread`); `threading.Thread.start` is recorded as
+an issue edge from the starting thread and a completed `join` as the joined thread's release
+acquired by the joiner, and threads started inside the capture get the operator-dispatch hook too
+(dispatch modes are thread-local).  Records are serialised by a lock, so the trace order is the
+order in which the threads issued their calls.
 """
 from __future__ import annotations
 
+import functools
 import itertools
+import threading
 from typing import Any
 
 import torch
@@ -72,6 +81,16 @@ def _install_hooks():
     _HOOKS_INSTALLED = True
 
 
+def _recording(fn):
+    """A recording entry point: serialised, and attributed to the calling host thread."""
+    @functools.wraps(fn)
+    def wrapped(self, *a, **k):
+        with self._lock:
+            self._as_current_thread()
+            return fn(self, *a, **k)
+    return wrapped
+
+
 class _Dispatch(TorchDispatchMode):
     def __init__(self, cap: "Capture"):
         super().__init__()
@@ -80,7 +99,7 @@ class _Dispatch(TorchDispatchMode):
     def __torch_dispatch__(self, func, types, args=(), kwargs=None):
         kwargs = kwargs or {}
         out = func(*args, **kwargs)
-        if func is not _aten.record_stream.default:
+        if func is not _aten.record_stream.default and _ACTIVE is self.cap:   # (threads may outlive it)
             self.cap._on_op(func, args, kwargs, out)
         return out
 
@@ -97,6 +116,9 @@ class Capture:
         self.intercept_distributed = intercept_distributed
         self._patched: list[tuple[Any, str, Any]] = []
         self._in_p2p = False
+        self._lock = threading.RLock()
+        self._tids: dict[threading.Thread, int] = {}   # host thread -> thread id in the trace
+        self._cur_tid = 0
         self.trace = Trace(max_fibers)
         self.low = Lowering(self.trace)
         self.streams: set[int] = {0}
@@ -115,8 +137,11 @@ class Capture:
         _install_hooks()
         torch.cuda.synchronize()                     # work issued before the capture is complete
         _ACTIVE = self
+        self._tids = {threading.current_thread(): 0}    # the capturing thread is thread 0 (fiber 0)
+        self._cur_tid = 0
         if self.intercept_distributed:
             self._patch_distributed()
+        self._patch_threads()
         self._mode = _Dispatch(self)
         self._mode.__enter__()
         return self
@@ -151,25 +176,32 @@ class Capture:
         return ptr
 
     # ---- CUDA trace callbacks -----------------------------------------------------------------------
+    @_recording
     def _on_stream_creation(self, stream: int):
         self._stream(stream)
 
+    @_recording
     def _on_event_record(self, event: int, stream: int):
         self.low.cusan_on_event_record(event, self._stream(stream))
 
+    @_recording
     def _on_event_wait(self, event: int, stream: int):
         self.low.cusan_on_stream_wait_event(self._stream(stream), event)
 
+    @_recording
     def _on_event_sync(self, event: int):
         self.low.cusan_on_event_sync(event)
 
+    @_recording
     def _on_stream_sync(self, stream: int):
         self.low.cusan_on_stream_sync(self._stream(stream))
 
+    @_recording
     def _on_device_sync(self):
         self.low.cusan_on_device_sync()
 
     # ---- operator dispatch ---------------------------------------------------------------------------
+    @_recording
     def _on_op(self, func, args, kwargs, out):
         schema = func._schema
         name = schema.name
@@ -219,9 +251,11 @@ class Capture:
             self.low.cusan_on_stream_sync(stream)     # blocking host<->device copy
 
     # ---- point-to-point communication ----------------------------------------------------------------
+    @_recording
     def isend(self, tensor: torch.Tensor, stream_ordered: bool = False):
         return self._p2p(tensor, 0, stream_ordered)
 
+    @_recording
     def irecv(self, tensor: torch.Tensor, stream_ordered: bool = False):
         return self._p2p(tensor, 1, stream_ordered)
 
@@ -243,6 +277,7 @@ class Capture:
         self.low.cusan_on_event_record(e2, comm)
         return ("nccl", e2)
 
+    @_recording
     def wait(self, handle: Any):
         kind, v = handle
         if kind == "mpi":
@@ -250,11 +285,53 @@ class Capture:
         else:
             self.low.cusan_on_stream_wait_event(self._stream(torch.cuda.current_stream().cuda_stream), v)
 
+    @_recording
     def send(self, tensor: torch.Tensor):
         self.low.cusan_on_mpi_send(self._storage(tensor), tensor.untyped_storage().nbytes())
 
+    @_recording
     def recv(self, tensor: torch.Tensor):
         self.low.cusan_on_mpi_recv(self._storage(tensor), tensor.untyped_storage().nbytes())
+
+    # ---- host threads ---------------------------------------------------------------------------------
+    def _thread_id(self, th: threading.Thread) -> int:
+        if th not in self._tids:
+            self._tids[th] = len(self._tids)
+        return self._tids[th]
+
+    def _as_current_thread(self):
+        tid = self._thread_id(threading.current_thread())
+        if tid != self._cur_tid:
+            self.low.cusan_on_thread(tid)
+            self._cur_tid = tid
+
+    def _patch_threads(self):
+        cap = self
+        orig_start, orig_join = threading.Thread.start, threading.Thread.join
+
+        def start(th):
+            with cap._lock:
+                cap._as_current_thread()
+                cap.low.cusan_on_thread_create(cap._thread_id(th))   # issue edge parent -> child
+            body = th.run
+
+            def run():
+                with _Dispatch(cap):               # dispatch modes are per thread
+                    body()
+            th.run = run
+            return orig_start(th)
+
+        def join(th, timeout=None):
+            out = orig_join(th, timeout)
+            if not th.is_alive() and th in cap._tids and _ACTIVE is cap:
+                with cap._lock:
+                    cap._as_current_thread()
+                    cap.low.cusan_on_thread_join(cap._tids[th])       # child release, caller acquire
+            return out
+
+        for name, fn, orig in (("start", start, orig_start), ("join", join, orig_join)):
+            self._patched.append((threading.Thread, name, orig))
+            setattr(threading.Thread, name, fn)
 
     # ---- torch.distributed interception --------------------------------------------------------------
     def _patch_distributed(self):

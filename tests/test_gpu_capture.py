@@ -160,3 +160,41 @@ def test_torch_distributed_p2p_is_captured():
     assert res["racy"]["races"] == 2 * n * 4 // 8 and res["racy"]["runs"] == 2, res
     assert res["fixed"]["races"] == 0 and res["fixed"]["value"] == n, res
     assert res["racy"]["patched_back"] and res["fixed"]["patched_back"], res
+
+
+@pytest.mark.parametrize("fixed", [False, True])
+def test_host_threads_are_fibers(fixed):
+    """A second Python thread issues work on a side stream (f4 in a captured PyTorch program,
+    PAPER.md:1202-1218).  Racy: the main thread, told by a host-level event (invisible to the
+    device), writes the tensor on the default stream while the side stream's write is unordered
+    with it.  Fixed: the default stream waits on the side stream first."""
+    import threading
+    torch.cuda.synchronize()
+    n = 1 << 14
+    s = torch.cuda.Stream()
+    done = threading.Event()
+    with Capture() as cap:
+        x = torch.ones(n, device="cuda")
+
+        def work():
+            with torch.cuda.stream(s):
+                s.wait_stream(torch.cuda.default_stream())   # after x's initialisation
+                x.mul_(2)
+            done.set()
+
+        t = threading.Thread(target=work)
+        t.start()
+        done.wait()
+        if fixed:
+            t.join()
+            torch.cuda.current_stream().wait_stream(s)
+        x.add_(1)
+        t.join()
+        torch.cuda.synchronize()
+    assert len(cap._tids) == 2                     # two host fibers
+    rep = _parity(cap)
+    if fixed:
+        assert rep.n_race_granules == 0
+    else:
+        assert rep.n_race_granules == n * 4 // 8 and rep.n_runs == 1
+    assert threading.Thread.start.__module__ == "threading"   # patches removed on exit
