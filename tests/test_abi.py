@@ -258,3 +258,14 @@ def test_planning_with_the_clock_thread():
     d = cs.describe(t, window_events=100)
     assert d["n_access"] == n and d["n_intervals"] == n and d["n_windows"] == (n + 99) // 100
     assert d["n_segments"] == 1 and d["n_incidences"] == n and d["tracked_bytes"] == 64 * n
+
+
+def test_c_example_host_steps():
+    """examples/fig6a.c drives the C ABI from C (lowering callbacks + cusan_plan_describe, no GPU)."""
+    import subprocess
+    import __graft_entry__ as g
+    exe = [e for e in g.build_examples() if e.endswith("fig6a")][0]
+    for extra in ([], ["--fixed"]):
+        r = subprocess.run([exe, "--describe", *extra], capture_output=True, text=True, timeout=60)
+        assert r.returncode == 0, (r.stdout, r.stderr)
+        assert "accesses 2" in r.stdout and "tracked 8192 B" in r.stdout

@@ -374,3 +374,15 @@ def test_pipelined_checks_match_the_oracle_per_step():
         assert_equal(rep, oracle.check_events(traces[i][0], traces[i][1], threads=2))
         n += 1
     assert n == len(traces)
+
+
+def test_c_example_fig6a():
+    """The paper's Fig. 6A through the C ABI from a C program (examples/fig6a.c): racy = one run
+    over the 4 KiB buffer, (Isend read, kernel write); fixed (MPI_Wait first) = none."""
+    import subprocess
+    import __graft_entry__ as g
+    exe = [e for e in g.build_examples() if e.endswith("fig6a")][0]
+    racy = subprocess.run([exe], capture_output=True, text=True, timeout=120)
+    assert racy.returncode == 0 and "racy: 512 race granules, 1 runs" in racy.stdout, (racy.stdout, racy.stderr)
+    fixed = subprocess.run([exe, "--fixed"], capture_output=True, text=True, timeout=120)
+    assert fixed.returncode == 0 and "fixed: 0 race granules, 0 runs" in fixed.stdout, (fixed.stdout, fixed.stderr)
