@@ -135,7 +135,8 @@ class Capture:
         if _ACTIVE is not None:
             raise RuntimeError("a Capture is already active")
         _install_hooks()
-        torch.cuda.synchronize()                     # work issued before the capture is complete
+        if torch.cuda.is_available():
+            torch.cuda.synchronize()                 # work issued before the capture is complete
         _ACTIVE = self
         self._tids = {threading.current_thread(): 0}    # the capturing thread is thread 0 (fiber 0)
         self._cur_tid = 0
