@@ -46,9 +46,11 @@ struct cusan_lowering {
         int kind;
     };
     std::vector<Alloc> allocs;                             // registered allocations, sorted by base
+    std::unordered_map<uint64_t, Alloc> by_base;           // the same, by exact base pointer
     std::unordered_map<uint64_t, uint32_t> thread_fiber;   // host thread -> fiber (thread 0 -> 0)
     std::unordered_map<uint64_t, uint32_t> ptds;           // host thread -> per-thread default stream
     uint64_t thread = 0;                                   // calling host thread
+    uint32_t h_fiber = 0;                                  // its fiber (thread_fiber[thread])
     bool per_thread_mode = false;
     std::vector<std::pair<int, uint64_t>> fiber_info;      // by fiber: (cusan_fiber_kind, handle)
 
@@ -57,7 +59,7 @@ struct cusan_lowering {
         fiber_info[f] = {kind, handle};
     }
 
-    uint32_t H() const { return thread_fiber.at(thread); }
+    uint32_t H() const { return h_fiber; }
 
     // --- primitives ---------------------------------------------------------------------------
     int access(uint32_t f, int mode, uint64_t addr, uint64_t n) {
@@ -72,6 +74,10 @@ struct cusan_lowering {
     // (the allocation with the greatest base <= p, if it contains p; a flat sorted array: lookups
     // happen for every kernel argument, registrations rarely)
     const Alloc* find(uint64_t p) const {
+        // kernel arguments are nearly always allocation bases: an exact hit is the allocation with
+        // the greatest base <= p, so it decides alone
+        const auto hit = by_base.find(p);
+        if (hit != by_base.end()) return hit->second.size ? &hit->second : nullptr;
         auto it = std::upper_bound(allocs.begin(), allocs.end(), p,
                                    [](uint64_t x, const Alloc& a) { return x < a.base; });
         if (it == allocs.begin()) return nullptr;
@@ -86,6 +92,7 @@ struct cusan_lowering {
             *it = {base, size, kind};                      // re-registration replaces
         else
             allocs.insert(it, {base, size, kind});
+        by_base[base] = {base, size, kind};
     }
     int new_fiber(uint32_t* f) {
         uint32_t mf = 0;
@@ -393,7 +400,10 @@ int cusan_on_thread(cusan_lowering* l, uint64_t thread) {
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
     uint32_t f = 0;
     int st = l->thread_fiber_of(thread, &f);
-    if (!st) l->thread = thread;
+    if (!st) {
+        l->thread = thread;
+        l->h_fiber = f;
+    }
     return st;
 }
 
@@ -421,6 +431,17 @@ int cusan_lowering_set_default_stream(cusan_lowering* l, int per_thread) {
 int cusan_lower_program(cusan_lowering* l, const cusan_api_call* calls, uint64_t n,
                         const cusan_api_arg* args, uint64_t nargs, uint32_t* op_first_event) {
     if (!l || (n && !calls) || (nargs && !args)) return fail(CUSAN_EINVAL, "null argument");
+    {   // room for the typical expansion (a launch is ~6 primitives), so the trace grows once
+        std::vector<cusan_event>& ev = l->trace->t.ev;
+        const uint64_t want = std::min<uint64_t>(ev.size() + 4 * n + nargs, CUSAN_MAX_EVENTS);
+        if (want > ev.capacity()) {
+            try {
+                ev.reserve(want);
+            } catch (...) {
+                return fail(CUSAN_ENOMEM, "cannot reserve the trace");
+            }
+        }
+    }
     std::vector<uint64_t> ptrs;
     std::vector<uint32_t> modes;
     for (uint64_t i = 0; i < n; i++) {
