@@ -140,12 +140,16 @@ int cusan_plan_create(const cusan_trace* t, const cusan_check_opts* o, cusan_pla
 /* Device bytes the plan needs (tables + shadow + read-set heap + run buffer). */
 int cusan_plan_workspace_bytes(const cusan_plan* p, uint64_t* bytes);
 /* Binds caller-owned device memory (>= cusan_plan_workspace_bytes, 256-B aligned, on the plan's
- * device) to a plan created with CUSAN_CHECK_DEFER_WORKSPACE and uploads the tables.  The memory
- * must stay valid until cusan_plan_destroy.  CUSAN_ESTATE if the plan owns a workspace. */
+ * device) to a plan created with CUSAN_CHECK_DEFER_WORKSPACE and uploads the tables (queued on the
+ * plan's stream, not waited for: the check follows on the same stream).  The memory must stay
+ * valid until cusan_plan_destroy.  CUSAN_ESTATE if the plan owns a workspace.
+ * cusan_plan_create calls no CUDA function that waits for the device, so a plan can be prepared on
+ * one host thread while another thread's check runs (pipelined checks). */
 int cusan_plan_bind_workspace(cusan_plan* p, void* workspace, uint64_t bytes);
 /* Device part (a3, a4) and the report (a5).  May be called repeatedly (each run starts from an
  * empty shadow); asynchronous work is complete when it returns. */
 int cusan_plan_run(cusan_plan* p, cusan_report** out);
+/* Waits for the plan's stream (pending uploads / work), then frees the plan. */
 int cusan_plan_destroy(cusan_plan* p);
 /* Host steps a1 and a2 only (no device needed): fills the trace / plan counters the same
  * plan_create would compute (shard clip, intervals, segments, windows, spill records). */
