@@ -149,8 +149,12 @@ int cusan_plan_bind_workspace(cusan_plan* p, void* workspace, uint64_t bytes);
 /* Device part (a3, a4) and the report (a5).  May be called repeatedly (each run starts from an
  * empty shadow); asynchronous work is complete when it returns. */
 int cusan_plan_run(cusan_plan* p, cusan_report** out);
-/* Waits for the plan's stream (pending uploads / work), then frees the plan. */
+/* Waits for the plan's stream (pending uploads / work), then frees the plan.  A library-allocated
+ * workspace is parked for the next plan on the device (one block per device, the largest) instead
+ * of freed: cudaMalloc / cudaFree of a tens-of-GB shadow cost tens of ms each. */
 int cusan_plan_destroy(cusan_plan* p);
+/* Frees the parked workspaces (all devices).  Set CUSAN_NO_WORKSPACE_CACHE=1 to never park. */
+int cusan_release_cached_memory(void);
 /* Host steps a1 and a2 only (no device needed): fills the trace / plan counters the same
  * plan_create would compute (shard clip, intervals, segments, windows, spill records). */
 int cusan_plan_describe(const cusan_trace* t, const cusan_check_opts* o, cusan_counters* out);

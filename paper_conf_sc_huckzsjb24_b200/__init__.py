@@ -27,7 +27,7 @@ ARG_DTYPE = np.dtype([("ptr", "<u8"), ("mode", "<u4"), ("pad", "<u4")])
 CUSAN_READ, CUSAN_WRITE = 0, 1
 CUSAN_RELEASE, CUSAN_RELEASE_STORE, CUSAN_ACQUIRE, CUSAN_FORK = 0, 1, 2, 3
 __all__ = ["Trace", "Lowering", "Plan", "Report", "check", "pipelined_checks", "report_merge", "CusanError", "version",
-           "RUN_DTYPE", "EVENT_DTYPE"]
+           "RUN_DTYPE", "EVENT_DTYPE", "release_cached_memory"]
 
 
 def version() -> str:
@@ -338,6 +338,11 @@ def pipelined_checks(make_trace, steps: int, device: int = 0, **kw):
             finally:
                 p.close()
             yield tr, rep
+
+
+def release_cached_memory() -> None:
+    """cusan_release_cached_memory: free the library's parked check workspaces (all devices)."""
+    _ck(lib.cusan_release_cached_memory())
 
 
 def report_merge(runs: np.ndarray, n_race_granules: int, max_runs: int = 0) -> Report:

@@ -15,6 +15,95 @@
 
 using namespace cusan;
 
+// ---- library-owned workspaces: one parked block per device ----------------------------------------
+// A check without a caller workspace needs up to tens of GB (the shadow); cudaMalloc / cudaFree of
+// that much cost tens of ms each and cudaFree waits for the device, so repeated cusan_check calls
+// would pay both every time.  A destroyed plan parks its workspace instead (one block per device,
+// the largest seen); the next plan on that device takes it when it is large enough.  Released by
+// cusan_release_cached_memory() (or set CUSAN_NO_WORKSPACE_CACHE=1 to disable).
+namespace {
+struct WsCache {
+    std::mutex m;
+    char* p[256] = {};
+    uint64_t bytes[256] = {};
+};
+WsCache& ws_cache() { static WsCache* c = new WsCache; return *c; }
+bool ws_cache_on() {
+    static const bool on = std::getenv("CUSAN_NO_WORKSPACE_CACHE") == nullptr;
+    return on;
+}
+// a block of >= bytes on `device` (the current device): the parked one if it fits, else a new one
+// (freeing a parked block that is too small first, so both never coexist)
+cudaError_t ws_acquire(int device, uint64_t bytes, char** out, uint64_t* got) {
+    *out = nullptr;
+    *got = 0;
+    if (ws_cache_on() && device >= 0 && device < 256) {
+        WsCache& c = ws_cache();
+        std::lock_guard<std::mutex> lk(c.m);
+        if (c.p[device] && c.bytes[device] >= bytes) {
+            *out = c.p[device];
+            *got = c.bytes[device];
+            c.p[device] = nullptr;
+            c.bytes[device] = 0;
+            return cudaSuccess;
+        }
+        if (c.p[device]) {
+            cudaFree(c.p[device]);
+            c.p[device] = nullptr;
+            c.bytes[device] = 0;
+        }
+    }
+    cudaError_t e = cudaMalloc((void**)out, bytes);
+    if (e == cudaErrorMemoryAllocation) {      // blocks parked on other devices do not matter, but
+        (void)cudaGetLastError();              // a racing thread may have parked one here: retry once
+        cusan::release_parked_workspace(device);
+        e = cudaMalloc((void**)out, bytes);
+    }
+    if (e == cudaSuccess) *got = bytes;
+    return e;
+}
+// park a block (the plan's work on it is complete); frees whichever of it and the parked one is smaller
+void ws_release(int device, char* p, uint64_t bytes) {
+    if (!p) return;
+    if (ws_cache_on() && device >= 0 && device < 256) {
+        WsCache& c = ws_cache();
+        std::lock_guard<std::mutex> lk(c.m);
+        if (!c.p[device] || c.bytes[device] < bytes) {
+            char* old = c.p[device];
+            c.p[device] = p;
+            c.bytes[device] = bytes;
+            if (old) {
+                int cur = 0;
+                cudaGetDevice(&cur);
+                cudaSetDevice(device);
+                cudaFree(old);
+                cudaSetDevice(cur);
+            }
+            return;
+        }
+    }
+    int cur = 0;
+    cudaGetDevice(&cur);
+    cudaSetDevice(device);
+    cudaFree(p);
+    cudaSetDevice(cur);
+}
+}  // namespace
+
+void cusan::release_parked_workspace(int device) {
+    if (device < 0 || device >= 256) return;
+    WsCache& c = ws_cache();
+    std::lock_guard<std::mutex> lk(c.m);
+    if (!c.p[device]) return;
+    int cur = 0;
+    cudaGetDevice(&cur);
+    cudaSetDevice(device);
+    cudaFree(c.p[device]);
+    cudaSetDevice(cur);
+    c.p[device] = nullptr;
+    c.bytes[device] = 0;
+}
+
 struct cusan_plan {
     const cusan_trace* trace = nullptr;
     HostPlan hp;
@@ -23,6 +112,7 @@ struct cusan_plan {
     int max_blocks = 0;
     // device memory
     char* own = nullptr;          // library-allocated workspace (null when the caller's is used)
+    uint64_t own_bytes = 0;
     char* ws = nullptr;
     uint64_t ws_bytes = 0;
     AccRec* d_inc = nullptr;
@@ -51,7 +141,7 @@ struct cusan_plan {
     ~cusan_plan() {
         if (ev0) cudaEventDestroy(ev0);
         if (ev1) cudaEventDestroy(ev1);
-        if (own) cudaFree(own);
+        if (own) ws_release(device, own, own_bytes);
         if (d_runs_own) cudaFree(d_runs_own);
         if (d_heap_own) cudaFree(d_heap_own);
     }
@@ -271,7 +361,7 @@ static int plan_device_setup(cusan_plan* p) {
     // creating them here would stall a plan prepared while the previous check runs)
     if (o.workspace) return plan_bind(p, (char*)o.workspace, o.workspace_bytes);
     if (o.flags & CUSAN_CHECK_DEFER_WORKSPACE) return CUSAN_OK;   // caller binds later
-    cudaError_t me = cudaMalloc((void**)&p->own, std::max<uint64_t>(off, ALIGN));
+    cudaError_t me = ws_acquire(p->device, std::max<uint64_t>(off, ALIGN), &p->own, &p->own_bytes);
     if (me != cudaSuccess) return fail(CUSAN_ENOMEM, std::string("cudaMalloc workspace: ") + cudaGetErrorString(me));
     return plan_bind(p, p->own, off);
 }
@@ -455,6 +545,22 @@ int cusan_plan_run(cusan_plan* p, cusan_report** out) {
     r->ctr.d2h_bytes = d2h;
     r->ctr.run_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count();
     *out = r;
+    return CUSAN_OK;
+}
+
+int cusan_release_cached_memory(void) {
+    WsCache& c = ws_cache();
+    std::lock_guard<std::mutex> lk(c.m);
+    int cur = 0;
+    cudaGetDevice(&cur);
+    for (int d = 0; d < 256; d++)
+        if (c.p[d]) {
+            cudaSetDevice(d);
+            cudaFree(c.p[d]);
+            c.p[d] = nullptr;
+            c.bytes[d] = 0;
+        }
+    cudaSetDevice(cur);
     return CUSAN_OK;
 }
 

@@ -17,6 +17,9 @@ int fail(int status, const std::string& msg);
 // (pinning costs milliseconds per call); plain heap memory in a process without a CUDA device
 // (host planning only: cusan_plan_describe).
 void* pinned_alloc(size_t bytes);
+// Frees the check workspace parked on `device` (check_api.cpp), e.g. before a session's shadow
+// growth fails for want of device memory.
+void release_parked_workspace(int device);
 void pinned_free(void* p) noexcept;
 template <class T>
 struct PinnedAllocator {

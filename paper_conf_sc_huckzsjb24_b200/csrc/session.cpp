@@ -140,7 +140,10 @@ static bool vm_grow(VmRange& r, int device, size_t bytes, size_t reserve = 0) {
     const size_t sz = (want - r.mapped + r.gran - 1) / r.gran * r.gran;
     if (r.mapped + sz > r.reserved) return false;
     CUmemGenericAllocationHandle h;
-    if (v.create(&h, sz, &prop, 0) != CUDA_SUCCESS) return false;
+    if (v.create(&h, sz, &prop, 0) != CUDA_SUCCESS) {
+        release_parked_workspace(device);      // a one-shot check's parked workspace, then retry
+        if (v.create(&h, sz, &prop, 0) != CUDA_SUCCESS) return false;
+    }
     if (v.map(r.base + r.mapped, sz, 0, h, 0) != CUDA_SUCCESS) {
         v.release(h);
         return false;

@@ -386,3 +386,20 @@ def test_c_example_fig6a():
     assert racy.returncode == 0 and "racy: 512 race granules, 1 runs" in racy.stdout, (racy.stdout, racy.stderr)
     fixed = subprocess.run([exe, "--fixed"], capture_output=True, text=True, timeout=120)
     assert fixed.returncode == 0 and "fixed: 0 race granules, 0 runs" in fixed.stdout, (fixed.stdout, fixed.stderr)
+
+
+def test_library_workspace_is_reused_and_released():
+    """Checks without a caller workspace park theirs for the next check (cusan_plan_destroy);
+    results are unchanged whether the block is reused, replaced by a larger one or released."""
+    small = configs.make(3, "small")
+    big = configs.make(5, "small")
+    reps = []
+    for w in (small, small, big, small, big):
+        ops, args = w.arrays(True)
+        tr, _ = lower_product(ops, args)
+        reps.append((cs.check(tr, window_events=50), oracle.check_events(tr.cusan_trace_read(), 256)))
+        if len(reps) == 4:
+            cs.release_cached_memory()
+    for rep, ref in reps:
+        assert_equal(rep, ref)
+    cs.release_cached_memory()
