@@ -216,7 +216,25 @@ void cusan::pinned_free(void* p) noexcept {
     else std::free(b);
 }
 
+// Work-unit (warp range) sizing, granules.  The compiled defaults (kernel.cuh) can be overridden
+// at run time by CUSAN_RANGE_MIN / CUSAN_RANGE_MAX / CUSAN_RANGE_PER_ACCESS / CUSAN_RANGE_BAL_MIN /
+// CUSAN_RANGES_PER_WARP: tuning sweeps, and the parity tests that check results do not depend on
+// the work decomposition.  Ranges are rounded up to whole lane steps (CHUNK granules).
+namespace {
+uint64_t env_u64(const char* name, uint64_t dflt) {
+    const char* e = std::getenv(name);
+    if (!e || !*e) return dflt;
+    const unsigned long long v = std::strtoull(e, nullptr, 10);
+    return v ? (uint64_t)v : dflt;
+}
+}  // namespace
+
 void cusan::build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& out) {
+    const uint64_t R_MIN = env_u64("CUSAN_RANGE_MIN", CUSAN_RANGE_MIN);
+    const uint64_t R_MAX = std::max<uint64_t>(env_u64("CUSAN_RANGE_MAX", CUSAN_RANGE_MAX), 1);
+    const uint64_t R_PER_ACC = env_u64("CUSAN_RANGE_PER_ACCESS", CUSAN_RANGE_PER_ACCESS);
+    const uint64_t R_BAL_MIN = env_u64("CUSAN_RANGE_BAL_MIN", CUSAN_RANGE_BAL_MIN);
+    const uint64_t R_PER_WARP = env_u64("CUSAN_RANGES_PER_WARP", CUSAN_RANGES_PER_WARP);
     pinned_vector<DSpan>& ds = out.ds;
     ds.clear();
     ds.reserve(hp.spans.size() + hp.win_span_off.size());
@@ -233,7 +251,7 @@ void cusan::build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& ou
             if (!(hp.spans[i].flags & SPAN_COMPRESSED) && (hp.spans[i].flags & (SPAN_LOAD | SPAN_STORE)))
                 moving += hp.spans[i].len;
         const uint64_t rs_cap = std::max<uint64_t>(
-            CUSAN_RANGE_BAL_MIN, moving / ((uint64_t)CUSAN_RANGES_PER_WARP * WARPS * std::max(max_blocks, 1)));
+            R_BAL_MIN, moving / (R_PER_WARP * WARPS * std::max(max_blocks, 1)));
         for (uint64_t i = hp.win_span_off[w]; i < hp.win_span_off[w + 1]; i++) {
             const Span& s = hp.spans[i];
             DSpan d{};
@@ -252,9 +270,7 @@ void cusan::build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& ou
             const bool moves = !comp && (s.flags & (SPAN_LOAD | SPAN_STORE));
             uint64_t rs;
             if (moves)
-                rs = std::min<uint64_t>(std::min<uint64_t>(std::max<uint64_t>((uint64_t)CUSAN_RANGE_PER_ACCESS * s.list_cnt,
-                                                                              (uint64_t)CUSAN_RANGE_MIN),
-                                                           (uint64_t)CUSAN_RANGE_MAX),
+                rs = std::min<uint64_t>(std::min<uint64_t>(std::max<uint64_t>(R_PER_ACC * s.list_cnt, R_MIN), R_MAX),
                                         rs_cap);
             else
                 rs = std::max<uint64_t>(s.len, 1);

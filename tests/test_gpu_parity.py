@@ -403,3 +403,30 @@ def test_library_workspace_is_reused_and_released():
     for rep, ref in reps:
         assert_equal(rep, ref)
     cs.release_cached_memory()
+
+
+@pytest.mark.parametrize("ranges", [
+    dict(CUSAN_RANGE_MAX="128", CUSAN_RANGE_BAL_MIN="128"),                  # one lane step per range
+    dict(CUSAN_RANGE_MIN="1024", CUSAN_RANGE_MAX="1024", CUSAN_RANGE_BAL_MIN="1024"),
+    dict(CUSAN_RANGE_PER_ACCESS="1", CUSAN_RANGE_MIN="128", CUSAN_RANGES_PER_WARP="64",
+         CUSAN_RANGE_BAL_MIN="128"),
+    dict(CUSAN_RANGE_MIN="2147483648", CUSAN_RANGE_MAX="2147483648",
+         CUSAN_RANGE_BAL_MIN="2147483648"),                                   # one range per span
+], ids=["lane-step", "1Ki", "balance", "whole-span"])
+def test_results_do_not_depend_on_the_work_decomposition(ranges, monkeypatch):
+    """SURVEY §8(c) pin "invariance under tile size": the warp range length (the kernel's work unit,
+    sized on the host) from one lane step to a whole span gives the oracle's report, on both kernel
+    paths and with shards."""
+    for k, v in ranges.items():
+        monkeypatch.setenv(k, v)
+    for c in (3, 5):
+        w = configs.make(c, "small")
+        ops, args = w.arrays(True)
+        tr, _ = lower_product(ops, args)
+        ref = oracle.check_events(tr.cusan_trace_read(), 256)
+        for window in (0, 97):
+            for flags in (0, cs.CUSAN_CHECK_FORCE_LANES):
+                assert_equal(cs.check(tr, window_events=window, flags=flags), ref)
+        parts = [cs.check(tr, window_events=97, nshards=3, shard=s) for s in range(3)]
+        assert_equal(cs.report_merge(np.concatenate([p.runs for p in parts]),
+                                     sum(p.n_race_granules for p in parts)), ref)
