@@ -351,7 +351,7 @@ class Capture:
         def start(tensor, write, group):
             if not isinstance(tensor, torch.Tensor) or not tensor.is_cuda:
                 return None                            # host tensors are not tracked
-            return cap._p2p(tensor, write, nccl(group))
+            return (cap.irecv if write else cap.isend)(tensor, nccl(group))   # serialised, this thread
 
         def call(fn, *a, **k):
             prev, cap._in_p2p = cap._in_p2p, True
@@ -378,7 +378,7 @@ class Capture:
                 out = call(orig[name], tensor, *a, **k)
                 if isinstance(tensor, torch.Tensor) and tensor.is_cuda:
                     if nccl(group):                    # stream-ordered transfer, waited on
-                        cap.wait(cap._p2p(tensor, write, True))
+                        cap.wait((cap.irecv if write else cap.isend)(tensor, True))
                     else:                              # host-blocking (MPI_Send / MPI_Recv)
                         (cap.recv if write else cap.send)(tensor)
                 return out
