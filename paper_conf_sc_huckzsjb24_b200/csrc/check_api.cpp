@@ -227,6 +227,11 @@ uint64_t env_u64(const char* name, uint64_t dflt) {
     const unsigned long long v = std::strtoull(e, nullptr, 10);
     return v ? (uint64_t)v : dflt;
 }
+uint64_t env_u64_or_zero(const char* name, uint64_t dflt) {
+    const char* e = std::getenv(name);
+    if (!e || !*e) return dflt;
+    return (uint64_t)std::strtoull(e, nullptr, 10);
+}
 }  // namespace
 
 void cusan::build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& out) {
@@ -235,7 +240,13 @@ void cusan::build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& ou
     const uint64_t R_PER_ACC = env_u64("CUSAN_RANGE_PER_ACCESS", CUSAN_RANGE_PER_ACCESS);
     const uint64_t R_BAL_MIN = env_u64("CUSAN_RANGE_BAL_MIN", CUSAN_RANGE_BAL_MIN);
     const uint64_t R_PER_WARP = env_u64("CUSAN_RANGES_PER_WARP", CUSAN_RANGES_PER_WARP);
+    // guided tail: the last TAIL_PCT % of each long span's ranges are cut TAIL_DIV times smaller and
+    // queued after every span's head, so the last work a launch hands out is small and the grid
+    // drains evenly (warps take ranges in queue order from the dynamic scheduler)
+    const uint64_t TAIL_PCT = std::min<uint64_t>(env_u64_or_zero("CUSAN_TAIL_PCT", CUSAN_TAIL_PCT), 99);
+    const uint64_t TAIL_DIV = std::max<uint64_t>(env_u64("CUSAN_TAIL_DIV", CUSAN_TAIL_DIV), 1);
     pinned_vector<DSpan>& ds = out.ds;
+    std::vector<DSpan> tails;
     ds.clear();
     ds.reserve(hp.spans.size() + hp.win_span_off.size());
     out.wins.clear();
@@ -275,18 +286,48 @@ void cusan::build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& ou
             else
                 rs = std::max<uint64_t>(s.len, 1);
             rs = std::min<uint64_t>((rs + CHUNK - 1) / CHUNK * CHUNK, 1ull << 31);
-            d.rsize = (uint32_t)rs;
-            const uint64_t nt = (s.len + rs - 1) / rs;
-            const uint64_t mem = moves ? rs / 32 : 0;
-            d.rweight = (uint32_t)std::min<uint64_t>(mem + 4ull * s.list_cnt + 8, 0xffffffffull);
-            d.tile0 = tiles;
-            d.weight0 = weight;
-            tiles += nt;
-            weight += nt * d.rweight;
             if (s.flags & (SPAN_LOAD | SPAN_STORE)) out.need_shadow = true;
             out.cell_bytes += (comp ? 1 : s.len) * (((s.flags & SPAN_LOAD) ? 8 : 0) + ((s.flags & SPAN_STORE) ? 8 : 0));
-            ds.push_back(d);
+            auto place = [&](DSpan x, uint64_t r) {       // x covers x.len granules in ranges of r
+                x.rsize = (uint32_t)r;
+                const uint64_t nt = (x.len + r - 1) / r;
+                const uint64_t mem = moves ? r / 32 : 0;
+                x.rweight = (uint32_t)std::min<uint64_t>(mem + 4ull * x.list_cnt + 8, 0xffffffffull);
+                x.tile0 = tiles;
+                x.weight0 = weight;
+                tiles += nt;
+                weight += nt * x.rweight;
+                ds.push_back(x);
+            };
+            const uint64_t nt_all = (s.len + rs - 1) / rs;
+            const uint64_t rs_t = std::max<uint64_t>((rs / TAIL_DIV + CHUNK - 1) / CHUNK * CHUNK, CHUNK);
+            const uint64_t n_tail = nt_all * TAIL_PCT / 100;
+            if (moves && TAIL_PCT && TAIL_DIV > 1 && rs_t < rs && n_tail >= 1 && n_tail < nt_all) {
+                const uint64_t head = (nt_all - n_tail) * rs;      // whole head ranges
+                DSpan t = d;
+                d.len = head;
+                t.abs_begin += head;
+                t.dense_begin += head;
+                t.len = s.len - head;
+                t.rsize = (uint32_t)rs_t;
+                place(d, rs);
+                tails.push_back(t);
+            } else {
+                place(d, rs);
+            }
         }
+        for (DSpan t : tails) {                          // the guided tail, after every head
+            const uint64_t r = t.rsize;
+            const bool mv = !(t.flags & SPAN_COMPRESSED) && (t.flags & (SPAN_LOAD | SPAN_STORE));
+            const uint64_t nt = (t.len + r - 1) / r;
+            t.rweight = (uint32_t)std::min<uint64_t>((mv ? r / 32 : 0) + 4ull * t.list_cnt + 8, 0xffffffffull);
+            t.tile0 = tiles;
+            t.weight0 = weight;
+            tiles += nt;
+            weight += nt * t.rweight;
+            ds.push_back(t);
+        }
+        tails.clear();
         win.nspans = (uint32_t)(ds.size() - win.span_off);
         DSpan sent{};
         sent.tile0 = tiles;

@@ -52,6 +52,12 @@ constexpr size_t DYN_SMEM = CUSAN_TMA ? (size_t)8 * TMA_WARP_BYTES : 0;   // 8 =
 #ifndef CUSAN_RANGE_BAL_MIN
 #define CUSAN_RANGE_BAL_MIN 4096
 #endif
+#ifndef CUSAN_TAIL_PCT
+#define CUSAN_TAIL_PCT 67         // guided tail (check_api.cpp build_span_tables): % of a span's ranges
+#endif
+#ifndef CUSAN_TAIL_DIV
+#define CUSAN_TAIL_DIV 3          // ... cut this many times smaller, queued after every head
+#endif
 #ifndef CUSAN_GRAB
 #define CUSAN_GRAB 1
 #endif
