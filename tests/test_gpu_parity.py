@@ -412,7 +412,9 @@ def test_library_workspace_is_reused_and_released():
          CUSAN_RANGE_BAL_MIN="128"),
     dict(CUSAN_RANGE_MIN="2147483648", CUSAN_RANGE_MAX="2147483648",
          CUSAN_RANGE_BAL_MIN="2147483648"),                                   # one range per span
-], ids=["lane-step", "1Ki", "balance", "whole-span"])
+    dict(CUSAN_TAIL_PCT="0"),                                                  # no guided tail
+    dict(CUSAN_TAIL_PCT="95", CUSAN_TAIL_DIV="16", CUSAN_RANGE_BAL_MIN="1024"),  # nearly all tail
+], ids=["lane-step", "1Ki", "balance", "whole-span", "no-tail", "all-tail"])
 def test_results_do_not_depend_on_the_work_decomposition(ranges, monkeypatch):
     """SURVEY §8(c) pin "invariance under tile size": the warp range length (the kernel's work unit,
     sized on the host) from one lane step to a whole span gives the oracle's report, on both kernel
