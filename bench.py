@@ -307,6 +307,8 @@ def run_ours(args):
     achieved = cell_bytes / (k_ms / 1e3) / 1e9 if k_ms > 0 else 0.0
     nl = max(1, int(ctr["n_windows"]))                  # K1 launches per step (one per window)
     traffic, _ = ncu_traffic()
+    if not (args.config == 5 and args.size == "full" and args.window == 4096 and world == 1):
+        traffic = None                                   # the committed capture is of the bench workload
 
     # ---- e2e: public API from host buffers, every step: lower + plan + upload + check + report ----
     # (a) pipelined (the value reported): pipelined_checks lowers step i+2 and plans step i+1 on
