@@ -329,6 +329,7 @@ def run_ours(args):
     barrier()
     torch.cuda.synchronize(dev)
     t0 = None
+    e2e_kernel_ms = []
     for i, (_tr, r2) in enumerate(cs.pipelined_checks(make_trace, n_e2e + 2, device=local, **pkw)):
         if i < 2:                                # warm-up steps: fill the pipeline
             if i == 1:
@@ -337,6 +338,7 @@ def run_ours(args):
             continue
         c2 = r2.counters
         h2d, d2h = int(c2["h2d_bytes"]), int(c2["d2h_bytes"])
+        e2e_kernel_ms.append(float(c2["kernel_ms"]))
         if world > 1:
             out = gather_runs(r2.runs, r2.n_race_granules, comm_dev)
             r2 = cs.report_merge(*out) if out is not None else None
@@ -428,6 +430,7 @@ def run_ours(args):
         "cpu_baseline": cpu,
         "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "ms_per_step": 1e3 * e2e_step_s, "steps": n_e2e,
+                "kernel_ms_per_step": statistics.mean(e2e_kernel_ms) if e2e_kernel_ms else None,
                 "mode": "pipelined_checks: lowering of step i+2 and planning of step i+1 (host threads) overlap the GPU check of step i; "
                         "pinned host tables uploaded and the report downloaded every step; 2 warm-up steps",
                 "serial": {"value": e2e_serial, "unit": "GB/s", "ms_per_step": 1e3 * statistics.mean(serial_s),
