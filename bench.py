@@ -323,8 +323,8 @@ def run_ours(args):
     pkw = dict(window_events=args.window, stream=stream.cuda_stream)
     if world > 1:
         pkw.update(nshards=world, shard=rank)
-    # at least --e2e-steps timed steps and ~1 s of them (short steps are noisy), two warm-up steps
-    n_e2e = max(1, args.e2e_steps, min(400, int(1000.0 / max(1e-3, 1e3 * elapsed_s / args.steps))))
+    # at least --e2e-steps timed steps and ~2 s of them (short steps are noisy), two warm-up steps
+    n_e2e = max(1, args.e2e_steps, min(800, int(2000.0 / max(1e-3, 1e3 * elapsed_s / args.steps))))
     h2d = d2h = 0
     barrier()
     torch.cuda.synchronize(dev)
