@@ -90,6 +90,9 @@ def parse(path: str = GOLDEN) -> list[Listing]:
         elif cmd == "memcpy":
             p.memcpy(ptr(rest[0]), ptr(rest[1]), int(rest[2]), CPY[rest[3]])
             labels = [f"{label}.w", f"{label}.r"] if label else None
+        elif cmd == "memcpya":                         # cudaMemcpyAsync(dst, src, n, kind, stream)
+            p.memcpy_async(ptr(rest[0]), ptr(rest[1]), int(rest[2]), CPY[rest[3]], env[rest[4]])
+            labels = [f"{label}.w", f"{label}.r"] if label else None
         elif cmd == "memset":
             if len(rest) > 2:
                 p.memset_async(ptr(rest[0]), int(rest[1]), env[rest[2]])

@@ -355,3 +355,64 @@ def test_full_size_golden_reports(c, twin):
     for r in runs:
         for x in (ev[int(r["earlier"])], ev[int(r["later"])]):
             assert int(x["a"]) >> 3 <= int(r["g_begin"]) and int(r["g_end"]) <= (int(x["a"]) + int(x["b"]) + 7) >> 3
+
+
+# ------------------------------------------------------------------------------------------------
+# lowering mutants: each plausible misreading of a sync rule in oracle/lower.py must turn some
+# paper listing red (the listings pin the oracle's lowering, not only its equality with the product)
+# ------------------------------------------------------------------------------------------------
+_LOWER_MUTANTS = {
+    # M1: cudaMemcpyAsync H2D/D2H made host-synchronous
+    "memcpy_async_host_sync": ("if kind == OP_MEMCPY and x in (CPY_H2H, CPY_H2D, CPY_D2H):",
+                               "if x in (CPY_H2H, CPY_H2D, CPY_D2H):"),
+    # M2: a failed MPI_Test treated as completion (Fig. 1)
+    "mpi_test_fail_completes": ("if kind == OP_MPI_WAIT or x:", "if True:"),
+    # M3: cudaMemsetAsync on pinned memory made host-synchronous (PAPER.md:438-440 vs 463-466)
+    "memset_async_pinned_sync": ("if kind == OP_MEMSET and al is not None and al[2] == MEM_PINNED:",
+                                 "if al is not None and al[2] == MEM_PINNED:"),
+    # reading ★A6: H2H cudaMemcpy left asynchronous
+    "memcpy_h2h_async": ("x in (CPY_H2H, CPY_H2D, CPY_D2H)", "x in (CPY_H2D, CPY_D2H)"),
+    # D2D made host-synchronous (only H2D / D2H / H2H block the host)
+    "memcpy_d2d_sync": ("x in (CPY_H2H, CPY_H2D, CPY_D2H)", "True"),
+    # synchronous cudaMemset on pinned memory left asynchronous
+    "memset_pinned_async": ("if kind == OP_MEMSET and al is not None and al[2] == MEM_PINNED:", "if False:"),
+    # a failed cudaStreamQuery treated as a sync (A9)
+    "stream_query_fail_syncs": ("if x:                                          # only a successful",
+                                "if True:                                       # only a successful"),
+    # event re-record joins instead of replacing (A4)
+    "event_record_joins": ("self.release_store(f, K_event(c))", "self.release(f, K_event(c))"),
+    # cudaFree without its device-wide sync (A8)
+    "free_no_sync": ("self.sync_device_host()                      # PAPER.md:448-450", "pass  #"),
+}
+
+
+def _mutant_lowering(name):
+    import importlib.util
+    import oracle.lower as ol
+    old, new = _LOWER_MUTANTS[name]
+    src = open(ol.__file__).read()
+    assert src.count(old) == 1, (name, "mutation site not found exactly once")
+    spec = importlib.util.spec_from_loader(f"oracle_lower_{name}", loader=None)
+    mod = importlib.util.module_from_spec(spec)
+    exec(compile(src.replace(old, new), ol.__file__, "exec"), mod.__dict__)
+    return mod.Lowering
+
+
+@pytest.mark.parametrize("name", sorted(_LOWER_MUTANTS))
+def test_listings_kill_lowering_mutants(name):
+    """A lowering with one sync rule misread misclassifies at least one paper listing."""
+    MutLowering = _mutant_lowering(name)
+    bad = []
+    for lst in LISTINGS:
+        ops, args = lst.program.arrays()
+        L = MutLowering()
+        first = []
+        for op in np.asarray(ops, OP_DTYPE):
+            first.append(len(L.ev))
+            L.call(op, args)
+        ev = L.events()
+        rep = oracle.check_events(ev, L.next_fiber, threads=1)
+        got = set(listing_dsl.observed_pairs(rep["runs"], listing_dsl.label_events(lst, ev, first)))
+        if got != {(a, b) for a, b, _ in lst.expect}:
+            bad.append(lst.name)
+    assert bad, f"mutant {name} passes every paper listing"
