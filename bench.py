@@ -3,12 +3,19 @@
 
 One step = one pass of the whole hot path over the workload: the shadow-check kernels (a3) with
 in-warp run compaction, the device merge into canonical runs (a4), their download and the report
-(a5), with the event / clock / interval tables (a1, a2) already resident in HBM.  Extra keys, for
-context only: `postmortem` (one window) and `interval_compressed` (f3: one cell per interval).
+(a5), with the event / clock / interval tables (a1, a2) already resident in HBM.
+
+Two shadow layouts give the identical report; the line carries both:
+  * `value`, `roofline`, `e2e`: the DENSE shadow (CUSAN_CHECK_DENSE_SHADOW, one 8-B cell per
+    granule, TSan's layout) — every covered granule's cell is read and written in every window
+    that touches it, the HBM-bound kernel SURVEY.md §8(d)'s roofline describes;
+  * `modes.interval_compressed`: the library DEFAULT (one cell per elementary interval, f3) — the
+    fastest exact path; its end-to-end time is host work (lowering, planning), not HBM.
 `e2e` repeats the metric through the public API from host buffers: lowering of the recorded
 CUDA/MPI call program (a0), planning (a1, a2), table upload from pinned host memory, check and
 report download, every step — pipelined (`pipelined_checks`: the host side of step i+1 overlaps
-the GPU side of step i), with the unpipelined per-call number under `e2e.serial`.
+the GPU side of step i), with the unpipelined per-call number under `e2e.serial` and a per-phase
+cost breakdown (lower / plan / upload / kernels / merge + download) under `breakdown`.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
     torchrun --nproc-per-node N bench.py --gpus N ...      (one rank per GPU, shards by granule range)
@@ -123,6 +130,14 @@ def workload(args):
     return w, ops, args_, f"{name} ({'clean' if args.clean else 'racy'} twin, {args.size} size)"
 
 
+def bench_config(wname, window, events, accesses, tracked):
+    """`config` of the JSON line: the workload only, identical in both arms (--impl ours|reference);
+    run-dependent figures go under `workload_stats`."""
+    return {"workload": wname, "window_events": window, "events": int(events), "accesses": int(accesses),
+            "fibers": 64, "tracked_bytes": int(tracked),
+            "l2": "inputs larger than L2 (dense shadow 64 GiB, streamed every window)"}
+
+
 # ------------------------------------------------------------------------------------------------
 # CPU baseline: the oracle (as it stands) on a bounded contiguous granule sample of the same trace
 # ------------------------------------------------------------------------------------------------
@@ -184,17 +199,15 @@ def run_reference(args):
     import numpy as np
     acc = ev[ev["kind"] == 0]
     tracked = int(8 * np.sum(((acc["a"] + acc["b"] + np.uint64(7)) >> np.uint64(3)) - (acc["a"] >> np.uint64(3))))
-    ref_config = {"workload": wname, "window_events": args.window, "events": int(len(ev)), "accesses": int(len(acc)),
-                  "fibers": 64, "tracked_bytes": tracked,
-                  "note": "the oracle checks the whole trace at once; the race set does not depend on windows",
-                  "parallelism": f"{threads} host threads"}
+    ref_config = bench_config(wname, args.window, len(ev), len(acc), tracked)
     sample = (f"granules [{s['range'][0]}, {s['range'][1]}) = {s['granules']} granules, "
               f"{s['checked_bytes'] / 1e9:.1f} GB checked per step")
     print(json.dumps({
         "impl": "reference", "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot_s / args.steps,
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "u32",
-        "data": "synthetic", "config": ref_config,
+        "data": "synthetic", "config": ref_config, "parallelism": f"{threads} host threads",
+        "note": "the oracle checks the whole trace at once; the race set does not depend on windows",
         "cpu_baseline": {"value": value, "unit": "GB/s", "cores": threads, "kind": "oracle", "cpu_model": cpu_model(),
                          "sample": sample},
         "e2e": {"value": value, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -266,7 +279,8 @@ def run_ours(args):
         return float(t.item())
 
     # device memory for every plan comes from PyTorch's caching allocator
-    kw = dict(window_events=args.window, device=local, stream=stream.cuda_stream, workspace="torch")
+    DENSE = cs.CUSAN_CHECK_DENSE_SHADOW
+    kw = dict(window_events=args.window, device=local, stream=stream.cuda_stream, workspace="torch", flags=DENSE)
     if world > 1:
         plan = ShardedPlan(tr, comm_device=comm_dev, **kw)
         run = plan.run
@@ -320,56 +334,82 @@ def run_ours(args):
         cs.Lowering(t).cusan_lower_program(ops, args_)
         return t
 
-    pkw = dict(window_events=args.window, stream=stream.cuda_stream)
-    if world > 1:
-        pkw.update(nshards=world, shard=rank)
-    # at least --e2e-steps timed steps and ~2 s of them (short steps are noisy), two warm-up steps
-    n_e2e = max(1, args.e2e_steps, min(800, int(2000.0 / max(1e-3, 1e3 * elapsed_s / args.steps))))
-    h2d = d2h = 0
-    barrier()
-    torch.cuda.synchronize(dev)
-    t0 = None
-    e2e_kernel_ms = []
-    for i, (_tr, r2) in enumerate(cs.pipelined_checks(make_trace, n_e2e + 2, device=local, **pkw)):
-        if i < 2:                                # warm-up steps: fill the pipeline
-            if i == 1:
-                barrier()
-                t0 = time.perf_counter()
-            continue
-        c2 = r2.counters
-        h2d, d2h = int(c2["h2d_bytes"]), int(c2["d2h_bytes"])
-        e2e_kernel_ms.append(float(c2["kernel_ms"]))
+    def e2e_pipelined(flags, step_s_hint):
+        """Pipelined end-to-end steps: (GB/s, s/step, h2d, d2h, mean kernel ms)."""
+        pkw = dict(window_events=args.window, stream=stream.cuda_stream, flags=flags)
         if world > 1:
-            out = gather_runs(r2.runs, r2.n_race_granules, comm_dev)
-            r2 = cs.report_merge(*out) if out is not None else None
-        if rank == 0:
-            assert r2.n_race_granules == final.n_race_granules and np.array_equal(r2.runs, final.runs)
-    torch.cuda.synchronize(dev)
-    e2e_step_s = max_over_ranks(time.perf_counter() - t0) / n_e2e
-    e2e_value = tracked / e2e_step_s / 1e9
-
-    serial_s = []
-    for _ in range(2):
+            pkw.update(nshards=world, shard=rank)
+        # at least --e2e-steps timed steps and ~2 s of them (short steps are noisy), two warm-up steps
+        n = max(1, args.e2e_steps, min(800, int(2.0 / max(1e-5, step_s_hint))))
+        h2d = d2h = 0
         barrier()
         torch.cuda.synchronize(dev)
-        t0 = time.perf_counter()
-        t2 = make_trace(0)
-        if world > 1:
-            p2 = ShardedPlan(t2, comm_device=comm_dev, **kw)
-            r2 = p2.run()
-            p2.close()
-        else:
-            r2 = cs.check(t2, **kw)
+        t0 = None
+        kms = []
+        for i, (_tr, r2) in enumerate(cs.pipelined_checks(make_trace, n + 2, device=local, **pkw)):
+            if i < 2:                                # warm-up steps: fill the pipeline
+                if i == 1:
+                    barrier()
+                    t0 = time.perf_counter()
+                continue
+            c2 = r2.counters
+            h2d, d2h = int(c2["h2d_bytes"]), int(c2["d2h_bytes"])
+            kms.append(float(c2["kernel_ms"]))
+            if world > 1:
+                out = gather_runs(r2.runs, r2.n_race_granules, comm_dev)
+                r2 = cs.report_merge(*out) if out is not None else None
+            if rank == 0:
+                assert r2.n_race_granules == final.n_race_granules and np.array_equal(r2.runs, final.runs)
         torch.cuda.synchronize(dev)
-        serial_s.append(max_over_ranks(time.perf_counter() - t0))
-        if rank == 0:
-            assert r2.n_race_granules == final.n_race_granules and np.array_equal(r2.runs, final.runs)
-    e2e_serial = tracked / statistics.mean(serial_s) / 1e9
+        step_s = max_over_ranks(time.perf_counter() - t0) / n
+        return tracked / step_s / 1e9, step_s, n, h2d, d2h, (statistics.mean(kms) if kms else None)
+
+    def e2e_serial_and_breakdown(flags, reps=3):
+        """One cusan_check after another (nothing overlapped), timed per phase; medians."""
+        ph = {"lower_ms": [], "plan_ms": [], "upload_ms": [], "kernel_ms": [], "merge_download_ms": [],
+              "total_ms": []}
+        for _ in range(reps):
+            barrier()
+            torch.cuda.synchronize(dev)
+            t0 = time.perf_counter()
+            t2 = make_trace(0)                                   # a0: lowering of the API program
+            t1 = time.perf_counter()
+            if world > 1:
+                p2 = ShardedPlan(t2, comm_device=comm_dev, **dict(kw, flags=flags))
+                t2b = t3 = time.perf_counter()
+                r2 = p2.run()
+                rc = p2.last_shard_report.counters
+            else:
+                p2 = cs.Plan(t2, **dict(kw, flags=flags, workspace=None)
+                             | {"flags": flags | cs.CUSAN_CHECK_DEFER_WORKSPACE})
+                t2b = time.perf_counter()                        # a1 + a2 on the host
+                ws = torch.empty(max(p2.workspace_bytes(), 256), dtype=torch.uint8, device=dev)
+                p2.cusan_plan_bind_workspace(ws)                 # table upload (pinned -> HBM)
+                torch.cuda.synchronize(dev)
+                t3 = time.perf_counter()
+                r2 = p2.run()                                    # a3 + a4 + a5
+                rc = r2.counters
+            p2.close()
+            torch.cuda.synchronize(dev)
+            t4 = time.perf_counter()
+            ph["lower_ms"].append(1e3 * (t1 - t0))
+            ph["plan_ms"].append(1e3 * (t2b - t1))
+            ph["upload_ms"].append(1e3 * (t3 - t2b))
+            ph["kernel_ms"].append(float(rc["kernel_ms"]))
+            ph["merge_download_ms"].append(max(0.0, 1e3 * (t4 - t3) - float(rc["kernel_ms"])))
+            ph["total_ms"].append(max_over_ranks(t4 - t0) * 1e3)
+            if rank == 0:
+                assert r2.n_race_granules == final.n_race_granules and np.array_equal(r2.runs, final.runs)
+        med = {k: statistics.median(v) for k, v in ph.items()}
+        return tracked / (med["total_ms"] / 1e3) / 1e9, med
+
+    e2e_value, e2e_step_s, n_e2e, h2d, d2h, e2e_kms = e2e_pipelined(DENSE, elapsed_s / args.steps)
+    e2e_serial, dense_breakdown = e2e_serial_and_breakdown(DENSE)
 
     # ---- post-mortem variant (extra, for context): one window, no shadow traffic --------------------
     pm = None
     if world == 1:
-        p3 = cs.Plan(tr, window_events=0, device=local, stream=stream.cuda_stream, workspace="torch")
+        p3 = cs.Plan(tr, window_events=0, device=local, stream=stream.cuda_stream, workspace="torch", flags=DENSE)
         p3.run()
         torch.cuda.synchronize(dev)
         t0 = time.perf_counter()
@@ -380,21 +420,40 @@ def run_ours(args):
               "kernel_ms": r3.counters["kernel_ms"], "window_events": "all (one window)"}
         p3.close()
 
-    # ---- interval-compressed shadow (f3, extra, for context): same windows, one cell per interval --
-    ic = None
-    if world == 1:
-        p4 = cs.Plan(tr, window_events=args.window, device=local, stream=stream.cuda_stream, workspace="torch",
-                     flags=cs.CUSAN_CHECK_INTERVAL_SHADOW)
+    # ---- interval-compressed shadow (f3, the library default): same windows, one cell per interval --
+    # device-timed steps (tables resident, CUDA events on the plan's stream), pipelined and serial
+    # end to end through the public API, and its cost breakdown
+    ckw = dict(kw, flags=cs.CUSAN_CHECK_INTERVAL_SHADOW)
+    p4 = ShardedPlan(tr, comm_device=comm_dev, **ckw) if world > 1 else cs.Plan(tr, **ckw)
+    for _ in range(max(3, args.warmup)):
         p4.run()
-        torch.cuda.synchronize(dev)
-        t0 = time.perf_counter()
+    n_ic = max(args.steps, 50)
+    barrier()
+    torch.cuda.synchronize(dev)
+    e0.record(stream)
+    ic_kms = []
+    for _ in range(n_ic):
         r4 = p4.run()
-        ic_s = time.perf_counter() - t0
+        ic_kms.append((p4.last_shard_report if world > 1 else r4).counters["kernel_ms"])
+    e1.record(stream)
+    torch.cuda.synchronize(dev)
+    ic_s = max_over_ranks(e0.elapsed_time(e1) / 1e3) / n_ic
+    ic_ctr = (p4.last_shard_report if world > 1 else r4).counters
+    if rank == 0:
         assert r4.n_race_granules == final.n_race_granules and np.array_equal(r4.runs, final.runs)
-        ic = {"value": tracked / ic_s / 1e9, "unit": "GB/s", "ms_per_step": ic_s * 1e3,
-              "kernel_ms": r4.counters["kernel_ms"], "shadow_bytes": int(r4.counters["shadow_bytes"]),
-              "window_events": args.window}
-        p4.close()
+    p4.close()
+    del p4
+    ic_e2e, ic_e2e_s, ic_n, ic_h2d, ic_d2h, ic_e2e_kms = e2e_pipelined(cs.CUSAN_CHECK_INTERVAL_SHADOW, 0.01)
+    ic_serial, ic_breakdown = e2e_serial_and_breakdown(cs.CUSAN_CHECK_INTERVAL_SHADOW, reps=5)
+    ic = {"value": tracked / ic_s / 1e9, "unit": "GB/s", "ms_per_step": ic_s * 1e3, "steps": n_ic,
+          "kernel_ms_per_step": statistics.mean(ic_kms), "kernel_launches_per_step": int(ic_ctr["kernel_launches"]),
+          "shadow_bytes_per_gpu": int(ic_ctr["shadow_bytes"]), "window_events": args.window,
+          "flags": "CUSAN_CHECK_INTERVAL_SHADOW (library default)",
+          "e2e": {"value": ic_e2e, "unit": "GB/s", "h2d_bytes_per_step": ic_h2d, "d2h_bytes_per_step": ic_d2h,
+                  "ms_per_step": 1e3 * ic_e2e_s, "steps": ic_n, "kernel_ms_per_step": ic_e2e_kms,
+                  "mode": "pipelined_checks, as the dense e2e",
+                  "serial": {"value": ic_serial, "unit": "GB/s", "ms_per_step": ic_breakdown["total_ms"]}},
+          "breakdown": ic_breakdown}
 
     if rank != 0:
         if world > 1:
@@ -416,13 +475,13 @@ def run_ours(args):
         "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": 1e3 * elapsed_s / args.steps, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
-        "config": {"workload": wname, "window_events": args.window, "windows": int(ctr["n_windows"]),
-                   "events": int(ctr["n_events"]), "accesses": int(ctr["n_access"]), "fibers": 64,
-                   "tracked_bytes": int(tracked), "shadow_bytes_per_gpu": int(ctr["shadow_bytes"]),
-                   "granules_per_gpu": int(ctr["shard_granules"]), "coverage_per_window": d_cov,
-                   "race_granules": int(final.n_race_granules), "race_runs": int(final.n_runs),
-                   "parallelism": f"granule-range shards x{world}",
-                   "l2": "inputs larger than L2 (shadow 128 GiB / n_gpus, streamed every window)"},
+        "config": bench_config(wname, args.window, ctr["n_events"], ctr["n_access"], tracked),
+        "parallelism": f"granule-range shards x{world}",
+        "workload_stats": {"windows": int(ctr["n_windows"]), "shadow_bytes_per_gpu": int(ctr["shadow_bytes"]),
+                           "granules_per_gpu": int(ctr["shard_granules"]), "coverage_per_window": d_cov,
+                           "race_granules": int(final.n_race_granules), "race_runs": int(final.n_runs),
+                           "shadow": "dense: one 8-B cell per 8-byte granule (modes.interval_compressed: "
+                                     "the library default)"},
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
                      "kernel": "shadow_check_window", "kernel_ms_per_step": k_ms, "launches_per_step": nl,
@@ -430,15 +489,17 @@ def run_ours(args):
         "cpu_baseline": cpu,
         "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "ms_per_step": 1e3 * e2e_step_s, "steps": n_e2e,
-                "kernel_ms_per_step": statistics.mean(e2e_kernel_ms) if e2e_kernel_ms else None,
+                "kernel_ms_per_step": e2e_kms,
                 "mode": "pipelined_checks: lowering of step i+2 and planning of step i+1 (host threads) overlap the GPU check of step i; "
                         "pinned host tables uploaded and the report downloaded every step; 2 warm-up steps",
-                "serial": {"value": e2e_serial, "unit": "GB/s", "ms_per_step": 1e3 * statistics.mean(serial_s),
-                           "mode": "cusan_check per step, nothing overlapped"}},
+                "serial": {"value": e2e_serial, "unit": "GB/s", "ms_per_step": dense_breakdown["total_ms"],
+                           "mode": "lower + plan + upload + check per step, nothing overlapped (median of 3)"},
+                "breakdown": dense_breakdown},
         "gpu_launches": launches,
         "clocks": clk,
         "postmortem": pm,
-        "interval_compressed": ic,
+        "modes": {"dense": {"value": value, "e2e": e2e_value, "flags": "CUSAN_CHECK_DENSE_SHADOW (value, roofline, e2e)"},
+                  "interval_compressed": ic},
     }
     print(json.dumps(line), flush=True)
     if world > 1:

@@ -104,7 +104,7 @@ typedef struct cusan_check_opts {
     int device;           /* CUDA device ordinal                                                   */
     int window_events;    /* access events per shadow window; 0 = library default (one window)    */
     int persist_shadow;   /* 1: store every window's final cells (shadow left valid after the run) */
-    int flags;            /* CUSAN_CHECK_* diagnostics flags (0 for normal use)                    */
+    int flags;            /* CUSAN_CHECK_* flags (0 = interval-compressed shadow, library-allocated) */
     uint64_t max_runs;    /* runs kept in the report (0 = all); counts stay exact when truncated   */
     void* stream;         /* cudaStream_t to run on (NULL = the legacy default stream)             */
     void* workspace;      /* optional caller-owned device memory (e.g. a torch tensor); NULL = the
@@ -114,19 +114,21 @@ typedef struct cusan_check_opts {
                              map, a power of two (0 = 2^21); one-shot checks shard by range instead */
 } cusan_check_opts;
 
-/* Diagnostics: disable the equal-cells range path so every granule takes the lane-parallel
- * per-granule path (used by the parity tests to exercise both paths; results are identical). */
-#define CUSAN_CHECK_FORCE_LANES 1
 /* cusan_plan_create computes the plan but neither allocates nor uploads: the caller queries
  * cusan_plan_workspace_bytes, allocates device memory (e.g. a torch tensor from PyTorch's caching
  * allocator) and calls cusan_plan_bind_workspace before cusan_plan_run. */
 #define CUSAN_CHECK_DEFER_WORKSPACE 2
-/* Interval-compressed tracking (the paper's proposed remedy for the cost of
- * tracking whole allocations): one shadow cell per elementary interval instead
- * of one per granule.  Exact — every granule of an elementary interval is covered by the same
- * accesses, so all its cells would hold the same state — and the shadow shrinks from
- * 8 B × granules to 8 B × intervals.  Results are identical to the per-granule shadow. */
+/* Shadow representation (results are identical):
+ *   CUSAN_CHECK_INTERVAL_SHADOW — the DEFAULT: one 8-B shadow cell per elementary interval (a maximal
+ *     granule range no access endpoint splits).  Exact, because every granule of an elementary
+ *     interval is covered by the same accesses, so all its cells would hold the same state; the
+ *     paper's proposed remedy for the cost of tracking whole allocations.
+ *   CUSAN_CHECK_DENSE_SHADOW — one 8-B cell per 8-byte granule, TSan's layout:
+ *     every covered granule's cell is read and written in every window that touches it (the HBM
+ *     roofline line of SURVEY.md §8(d)); the kernel verifies that the cells of each range agree.
+ * Passing both is CUSAN_EINVAL.  (Flag value 1, a removed diagnostic, is rejected too.) */
 #define CUSAN_CHECK_INTERVAL_SHADOW 4
+#define CUSAN_CHECK_DENSE_SHADOW 8
 
 /* Defaults: nshards 1, shard 0, device 0, window_events 0, persist 0, max_runs 0, all NULL. */
 void cusan_check_opts_init(cusan_check_opts* o);
@@ -211,6 +213,9 @@ typedef struct cusan_counters {
     uint64_t shadow_cell_bytes;    /* algorithmic shadow bytes moved by the check kernels          */
     uint64_t h2d_bytes;            /* host -> device bytes: plan tables (create) + counters (run)  */
     uint64_t d2h_bytes;            /* device -> host bytes of the last run (counters + runs)       */
+    /* sessions: read-set heap after this call — records some interval still names, and the heap's
+       high-water mark (dead records are reused from the next call on, so it tracks the live set) */
+    uint64_t heap_live_bytes, heap_bytes;
 } cusan_counters;
 
 int cusan_report_get(const cusan_report* r, uint64_t* n_race_granules, uint64_t* n_runs,

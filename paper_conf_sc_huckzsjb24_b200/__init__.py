@@ -162,9 +162,6 @@ class Report:
             self.h = None
 
 
-CUSAN_CHECK_FORCE_LANES = 1
-
-
 def _opts(nshards=1, shard=0, device=0, window_events=0, persist_shadow=False, max_runs=0, stream=None,
           flags=0, shard_block=0):
     o = cusan_check_opts()
@@ -181,7 +178,24 @@ def _report(h, max_runs):
 
 
 CUSAN_CHECK_DEFER_WORKSPACE = 2
-CUSAN_CHECK_INTERVAL_SHADOW = 4
+CUSAN_CHECK_INTERVAL_SHADOW = 4    # the default shadow: one cell per elementary interval (f3)
+CUSAN_CHECK_DENSE_SHADOW = 8       # one cell per 8-byte granule (TSan's layout, §8(d) roofline line)
+
+
+def _torch_workspace(nbytes: int, device: int, stream):
+    """A uint8 CUDA tensor of nbytes from PyTorch's caching allocator, allocated on the stream the
+    plan runs on (`stream`, a cudaStream_t as int), so the allocator orders its reuse after the plan."""
+    import torch
+    dev = torch.device("cuda", device)
+    with torch.cuda.stream(torch.cuda.ExternalStream(stream, device=dev)):
+        return torch.empty(max(nbytes, 256), dtype=torch.uint8, device=dev)
+
+
+def _default_torch_stream(kw: dict) -> None:
+    """A plan on torch memory runs on torch's current stream unless a stream is given."""
+    if kw.get("stream") is None:
+        import torch
+        kw["stream"] = torch.cuda.current_stream(kw.get("device", 0)).cuda_stream
 
 
 class Plan:
@@ -196,15 +210,15 @@ class Plan:
         self.workspace = None
         if workspace == "torch":
             kw["flags"] = kw.get("flags", 0) | CUSAN_CHECK_DEFER_WORKSPACE
+            _default_torch_stream(kw)
+        self.device, self.stream = kw.get("device", 0), kw.get("stream")
         o = _opts(**kw)
         h = C.c_void_p()
         _ck(lib.cusan_plan_create(trace.h, C.byref(o), C.byref(h)))
         self.h = h
         if workspace == "torch":
-            import torch
             nbytes = self.workspace_bytes()
-            self.workspace = torch.empty(max(nbytes, 256), dtype=torch.uint8,
-                                         device=torch.device("cuda", kw.get("device", 0)))
+            self.workspace = _torch_workspace(nbytes, self.device, self.stream)
             _ck(lib.cusan_plan_bind_workspace(self.h, C.c_void_p(self.workspace.data_ptr()), nbytes))
 
     def workspace_bytes(self) -> int:
@@ -312,6 +326,9 @@ def pipelined_checks(make_trace, steps: int, device: int = 0, **kw):
     import torch
     kw = dict(kw)
     kw["flags"] = kw.get("flags", 0) | CUSAN_CHECK_DEFER_WORKSPACE
+    kw["device"] = device
+    _default_torch_stream(kw)
+    kw.pop("device")
 
     ws = None
     with ThreadPoolExecutor(1) as lower_ex, ThreadPoolExecutor(1) as plan_ex:
@@ -331,7 +348,7 @@ def pipelined_checks(make_trace, steps: int, device: int = 0, **kw):
             need = max(p.workspace_bytes(), 256)
             if ws is None or ws.numel() < need:
                 ws = None
-                ws = torch.empty(need, dtype=torch.uint8, device=torch.device("cuda", device))
+                ws = _torch_workspace(need, device, kw["stream"])
             try:
                 p.cusan_plan_bind_workspace(ws)
                 rep = p.run()

@@ -290,7 +290,7 @@ void cusan::build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& ou
             out.cell_bytes += (comp ? 1 : s.len) * (((s.flags & SPAN_LOAD) ? 8 : 0) + ((s.flags & SPAN_STORE) ? 8 : 0));
             auto place = [&](DSpan x, uint64_t r) {       // x covers x.len granules in ranges of r
                 x.rsize = (uint32_t)r;
-                const uint64_t nt = (x.len + r - 1) / r;
+                const uint64_t nt = comp ? 1 : (x.len + r - 1) / r;   // a compressed span: one range
                 const uint64_t mem = moves ? r / 32 : 0;
                 x.rweight = (uint32_t)std::min<uint64_t>(mem + 4ull * x.list_cnt + 8, 0xffffffffull);
                 x.tile0 = tiles;
@@ -471,12 +471,10 @@ static int launch_all(cusan_plan* p) {
     k.runs = p->d_runs;
     k.counters = p->d_counters;
     k.run_cap = p->run_cap;
-    const int force_lanes = (p->hp.opts.flags & CUSAN_CHECK_FORCE_LANES) ? 1 : 0;
     for (size_t i = 0; i < p->wins.size(); i++) {
         const Window& w = p->wins[i];
         unsigned long long* sched = CUSAN_DYNAMIC ? p->d_counters + N_COUNTERS + i : nullptr;
-        CK(launch_shadow_check(w.grid, p->stream, p->d_spans + w.span_off, w.nspans, w.tiles, w.weight, k, force_lanes,
-                               sched));
+        CK(launch_shadow_check(w.grid, p->stream, p->d_spans + w.span_off, w.nspans, w.tiles, w.weight, k, sched));
     }
     CK(cudaGetLastError());
     CK(cudaEventRecord(p->ev1, p->stream));
@@ -545,6 +543,9 @@ int cusan_plan_run(cusan_plan* p, cusan_report** out) {
         if (st) return st;
         CK(cudaMemcpyAsync(cnt, p->d_counters, sizeof(cnt), cudaMemcpyDeviceToHost, p->stream));
         CK(cudaStreamSynchronize(p->stream));
+        if (cnt[C_INVARIANT])
+            return fail(CUSAN_ESTATE, "internal error: cells of one elementary interval differ (" +
+                                          std::to_string(cnt[C_INVARIANT]) + " ranges)");
         const bool runs_ovf = cnt[C_RUNS] > p->run_cap, heap_ovf = cnt[C_HEAP_OVF] != 0;
         if (!runs_ovf && !heap_ovf) break;
         if (attempt >= 8) return fail(CUSAN_ENOMEM, "run buffer / spill heap keeps overflowing");

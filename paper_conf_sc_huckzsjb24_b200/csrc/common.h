@@ -79,6 +79,11 @@ class KeySlots {
     uint32_t n_ = 0;
 };
 
+// Interval-compressed shadow (f3) unless the caller asks for the per-granule dense shadow.
+inline bool compressed_shadow(const cusan_check_opts& o) { return !(o.flags & CUSAN_CHECK_DENSE_SHADOW); }
+// CUSAN_EINVAL for unknown or contradictory flags
+int check_flags(const cusan_check_opts& o);
+
 struct Trace {
     uint32_t max_fibers = 1;
     std::vector<cusan_event> ev;

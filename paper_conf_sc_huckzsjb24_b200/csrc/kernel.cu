@@ -20,12 +20,13 @@
 //             window's accesses once to the common cell (the read set in shared memory); each hit
 //             is a run over the whole range;
 //     pass 3  stream the final cell out (128-bit stores; skipped when no later window needs it).
-//   Ranges whose cells differ take the exact lane-parallel path: 32 lanes × 4 consecutive granules
-//   per step, each lane its own cell and private read-set record (shared records are copied before
-//   they are modified), hits compacted in the warp (__ballot_sync over hit lanes, __shfl_up_sync
-//   comparison with the left neighbour, run heads sized from the continuation mask).  Both paths
-//   feed a 32-entry per-warp run cache (one entry per lane) that extends runs across steps and
-//   ranges before appending them to global memory.
+//   Every granule of a range is covered by the same accesses (ranges lie inside one elementary
+//   interval of the plan), so in the per-granule (dense) shadow all cells of a range are equal by
+//   construction; pass 1's vote verifies that invariant (a violation is counted and fails the check
+//   with CUSAN_ESTATE: it would be a planner bug).  With the interval-compressed shadow (f3, the
+//   default) the range is the whole interval and its one cell is loaded once.  Hits feed a 32-entry
+//   per-warp run cache (one entry per lane) that extends runs across ranges before appending them
+//   to global memory.
 #include <atomic>
 
 #include "kernel.cuh"
@@ -74,33 +75,6 @@ __device__ __forceinline__ void cache_insert(uint32_t re, uint32_t rl, uint64_t 
             rc.ge = rge;
         }
         rc.rr = (rc.rr + 1) & 31u;
-    }
-}
-
-// Warp-collective, lane-parallel granules: every lane passes its own hit flag (false for lanes
-// without a granule).  Lanes hold consecutive granules g.
-__device__ __forceinline__ void emit(bool hit, uint32_t earlier_epoch, uint32_t later_id, uint64_t g,
-                                     int lane, RunCache& rc, const Ctx& k) {
-    const unsigned m = __ballot_sync(FULL, hit);
-    if (!m) return;
-    rc.nrace += __popc(m);
-    const uint32_t e_id = (earlier_epoch & 0xffffffu) - 1u;
-    const uint32_t prev = __shfl_up_sync(FULL, e_id, 1);
-    const bool cont = hit && lane > 0 && ((m >> (lane - 1)) & 1u) && prev == e_id;
-    const unsigned cm = __ballot_sync(FULL, cont);
-    unsigned heads = m & ~cm;
-    uint32_t len = 0;
-    if (hit && !cont) {
-        const unsigned long long rest = (unsigned long long)cm >> (lane + 1);
-        len = (uint32_t)__ffsll((long long)~rest);   // 1 + number of continuing lanes
-    }
-    while (heads) {
-        const int h = __ffs(heads) - 1;
-        heads &= heads - 1;
-        const uint32_t re = __shfl_sync(FULL, e_id, h);
-        const uint64_t rgb = __shfl_sync(FULL, g, h);
-        const uint32_t rl = __shfl_sync(FULL, len, h);
-        cache_insert(re, later_id, rgb, rgb + rl, lane, rc, k);
     }
 }
 
@@ -161,15 +135,14 @@ __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.w
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_async_smem() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
-// ---- lane path: per-granule read-set records ----------------------------------------------------
-// Record header word: n (bits 0..15) | units (bits 16..23) | PRIVATE (bit 31).  Records written by
-// the range path are shared by every granule of a range (never modified in place); records the
-// lane path allocates belong to one granule's cell and are updated in place while they have room.
-constexpr uint32_t REC_PRIVATE = 0x80000000u;
+// ---- read-set records ---------------------------------------------------------------------------
+// Record = {header n, epoch_1 .. epoch_n} in REC_WORDS-word units, written once by the range that
+// ends with that read set (pass 3) and only read afterwards.  The host pre-assigns one per span;
+// rec_alloc is the fallback should a pre-assigned record be too small (never with an exact plan).
 __device__ __forceinline__ uint32_t rec_n(uint32_t hdr) { return hdr & 0xffffu; }
 
-// allocate a private record with room for `cap` entries holding n; returns the tagged slot value,
-// or 0 on heap overflow (flagged; the host grows the heap and re-runs)
+// allocate a record with room for `cap` entries holding n; returns the tagged slot value, or 0 on
+// heap overflow (flagged; a plan grows the heap and re-runs)
 __device__ __forceinline__ uint32_t rec_alloc(const Ctx& k, uint32_t n, uint32_t cap, uint32_t** out) {
     const uint32_t units = (cap + 1 + REC_WORDS - 1) / REC_WORDS;
     const unsigned long long at = atomicAdd(&k.counters[C_HEAP], (unsigned long long)units);
@@ -179,100 +152,8 @@ __device__ __forceinline__ uint32_t rec_alloc(const Ctx& k, uint32_t n, uint32_t
         return 0;
     }
     *out = k.heap + at * REC_WORDS;
-    (*out)[0] = REC_PRIVATE | (units << 16) | n;
+    (*out)[0] = n;
     return SPILL_TAG | (uint32_t)at;
-}
-
-// R[f] := ep on one lane's cell
-__device__ void lane_read_update(uint2& c, uint32_t ep, uint32_t f, const Ctx& k) {
-    if (!c.y) { c.y = ep; return; }
-    uint32_t* dst;
-    if (!is_spill(c.y)) {
-        if ((c.y >> 24) == f) { c.y = ep; return; }
-        const uint32_t v = rec_alloc(k, 2, 2 * REC_WORDS - 1, &dst);   // second reader: {R, ep}
-        if (dst) { dst[1] = c.y; dst[2] = ep; }
-        c.y = v;
-        return;
-    }
-    uint32_t* src = rec_ptr(k, c.y);
-    const uint32_t hdr = src[0];
-    const uint32_t n = rec_n(hdr);
-    int pos = -1;
-    for (uint32_t j = 0; j < n; j++)
-        if ((src[1 + j] >> 24) == f) { pos = (int)j; break; }
-    if (pos >= 0 && src[1 + pos] == ep) return;
-    if (hdr & REC_PRIVATE) {   // this granule's own record: update in place
-        const uint32_t cap = ((hdr >> 16) & 0xffu) * REC_WORDS - 1;
-        if (pos >= 0) { src[1 + pos] = ep; return; }
-        if (n < cap) { src[1 + n] = ep; src[0] = hdr + 1; return; }
-    }
-    const uint32_t v = rec_alloc(k, pos >= 0 ? n : n + 1, 2 * (n + 1), &dst);   // copy, with room
-    if (dst) {
-        for (uint32_t j = 0; j < n; j++) dst[1 + j] = src[1 + j];
-        if (pos >= 0) dst[1 + pos] = ep; else dst[1 + n] = ep;
-    }
-    c.y = v;
-}
-
-// Where a span's cells live in the shadow.
-__device__ __forceinline__ const uint2* src_cells(const DSpan& sp, const Ctx& k) {
-    return k.shadow + sp.dense_begin;
-}
-
-// Lane-parallel exact path for granules [x0, x0 + n) of span sp (each lane its own cells).
-__device__ void check_lanes(const DSpan& sp, uint64_t x0, uint64_t n, int lane, RunCache& rc, const Ctx& k) {
-    for (uint64_t xc = x0; xc < x0 + n; xc += CHUNK) {
-        uint2 cell[U];
-        bool valid[U];
-#pragma unroll
-        for (int c = 0; c < U; c++) {
-            const uint64_t x = xc + c * 32 + lane;
-            valid[c] = x < x0 + n;
-            cell[c] = make_uint2(0, 0);
-            if (valid[c] && (sp.flags & SPAN_LOAD)) cell[c] = __ldcs(src_cells(sp, k) + x);
-        }
-        const uint32_t qe = sp.list_off + sp.list_cnt;
-        for (uint32_t q = sp.list_off; q < qe; q++) {
-            const AccRec r = k.inc[q];
-            const uint32_t f = r.epoch >> 24;
-            const uint32_t later = (r.epoch & 0xffffffu) - 1u;
-            const uint32_t* row = k.segvc + (uint64_t)(r.segm & 0x7fffffffu) * k.F;
-            const bool wr = r.segm >> 31;
-#pragma unroll
-            for (int c = 0; c < U; c++) {
-                const uint64_t g = sp.abs_begin + xc + c * 32 + lane;
-                emit(valid[c] && unordered(cell[c].x, f, row), cell[c].x, later, g, lane, rc, k);
-                if (wr) {
-                    const bool sp_r = valid[c] && is_spill(cell[c].y);
-                    emit(valid[c] && !sp_r && unordered(cell[c].y, f, row), cell[c].y, later, g, lane, rc, k);
-                    uint32_t* rp = sp_r ? rec_ptr(k, cell[c].y) : nullptr;
-                    const uint32_t nr = sp_r ? rec_n(rp[0]) : 0u;
-                    const uint32_t nmax = __reduce_max_sync(FULL, nr);
-                    for (uint32_t j = 0; j < nmax; j++) {
-                        const uint32_t v = j < nr ? rp[1 + j] : 0u;
-                        emit(unordered(v, f, row), v, later, g, lane, rc, k);
-                    }
-                    // R := ∅.  A private record stays attached, emptied, for this granule's next
-                    // readers (a record with n = 0 is the empty read set); shared ones detach.
-                    uint32_t keep = 0;
-                    if (sp_r && (rp[0] & REC_PRIVATE)) {
-                        rp[0] &= ~0xffffu;
-                        keep = cell[c].y;
-                    }
-                    cell[c] = make_uint2(r.epoch, keep);
-                } else if (valid[c]) {
-                    lane_read_update(cell[c], r.epoch, f, k);
-                }
-            }
-        }
-        if (sp.flags & SPAN_STORE) {
-#pragma unroll
-            for (int c = 0; c < U; c++) {
-                const uint64_t x = xc + c * 32 + lane;
-                if (valid[c]) __stcs(k.shadow + sp.dense_begin + x, cell[c]);
-            }
-        }
-    }
 }
 
 __device__ __forceinline__ uint32_t find_span_by_tile(const DSpan* __restrict__ sp, uint32_t n, uint64_t t) {
@@ -299,7 +180,7 @@ __device__ __forceinline__ uint64_t tile_at_weight(const DSpan* __restrict__ sp,
 
 __global__ void __launch_bounds__(THREADS, CUSAN_MIN_BLOCKS)
 shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t total_tiles,
-                    uint64_t total_weight, Ctx k, int force_lanes, unsigned long long* sched) {
+                    uint64_t total_weight, Ctx k, unsigned long long* sched) {
     __shared__ uint32_t s_list[WARPS][MAXS];
     __shared__ uint8_t s_slot[WARPS][256];
     const int lane = threadIdx.x & 31;
@@ -359,12 +240,14 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
             }
             while (t >= spans[s + 1].tile0) s++;   // spans[nspans] is a sentinel
             const DSpan sp = spans[s];
-            const uint64_t x0 = (t - sp.tile0) * sp.rsize;
-            const uint64_t n = min((uint64_t)sp.rsize, sp.len - x0);   // granules of the range
-            const bool comp = sp.flags & SPAN_COMPRESSED;           // f3: one cell per interval
+            // f3: one cell per interval, and a compressed span is always a single range (its cell
+            // must have exactly one owner, whatever the interval's length)
+            const bool comp = sp.flags & SPAN_COMPRESSED;
+            const uint64_t x0 = comp ? 0 : (t - sp.tile0) * sp.rsize;
+            const uint64_t n = comp ? sp.len : min((uint64_t)sp.rsize, sp.len - x0);   // granules of the range
             const uint64_t ncell = comp ? 1 : n;
             uint2* cells = k.shadow + sp.dense_begin + x0;      // 8-B aligned (256-B for plan layouts)
-            const uint2* src = src_cells(sp, k) + x0;
+            const uint2* src = cells;
             // 128-bit / bulk streaming needs 16-B alignment: a cell off it is handled on its own
             const uint64_t shead = (reinterpret_cast<uintptr_t>(src) & 15u) ? 1 : 0;
             const uint4* cells2 = reinterpret_cast<const uint4*>(src + shead);
@@ -372,8 +255,8 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
             const bool stail = ncell > shead && ((ncell - shead) & 1);
             // ---- pass 1: stream the range's cells in and vote that they are all equal ----------
             uint2 c = make_uint2(0, 0);            // first window of the interval: known empty
-            bool uniform = comp || !force_lanes;
-            if (uniform && (sp.flags & SPAN_LOAD)) {
+            bool uniform = true;
+            if (sp.flags & SPAN_LOAD) {
                 c = src[0];
                 bool ok = true;
 #if CUSAN_TMA
@@ -425,8 +308,8 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                 }
                 uniform = __all_sync(FULL, ok);
             }
-            if (!uniform) {
-                check_lanes(sp, x0, n, lane, rc, k);
+            if (!uniform) {                        // planner invariant broken: fail the check
+                if (lane == 0) atomicAdd(&k.counters[C_INVARIANT], 1ull);
                 continue;
             }
             // ---- pass 2: all cells of the range equal `c`: apply the window's accesses once -----
@@ -617,12 +500,10 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
 
 constexpr uint64_t COPY_CHUNK = 8192;     // cells per warp work item
 
-// Copy cells between layouts.  With `heap` set (a session splitting a compressed interval in place,
-// so source and copy both stay live) a copied private read-set record becomes shared: neither cell
-// may then update it in place (lane_read_update copies it on its next change).
+// Copy cells between layouts (a session splitting a compressed interval in place: the copy names the
+// same read-set record, which is never modified after it is written).
 __global__ void __launch_bounds__(THREADS)
-copy_cells(const uint2* src, uint2* dst, const CopySeg* __restrict__ segs, uint32_t nseg, uint64_t total,
-           uint32_t* heap) {
+copy_cells(const uint2* src, uint2* dst, const CopySeg* __restrict__ segs, uint32_t nseg, uint64_t total) {
     const int lane = threadIdx.x & 31;
     const uint64_t nwarps = (uint64_t)gridDim.x * WARPS;
     const uint64_t nchunks = (total + COPY_CHUNK - 1) / COPY_CHUNK;
@@ -638,7 +519,6 @@ copy_cells(const uint2* src, uint2* dst, const CopySeg* __restrict__ segs, uint3
             const uint64_t end = min(c1, sg.prefix + sg.len);
             for (uint64_t i = c + lane; i < end; i += 32) {
                 const uint2 v = __ldcs(src + sg.src + (i - sg.prefix));
-                if (heap && is_spill(v.y)) atomicAnd(heap + (uint64_t)(v.y & 0xffffffu) * REC_WORDS, ~REC_PRIVATE);
                 __stcs(dst + sg.dst + (i - sg.prefix), v);
             }
             c = end;
@@ -652,15 +532,14 @@ copy_cells(const uint2* src, uint2* dst, const CopySeg* __restrict__ segs, uint3
 namespace cusan {
 
 cudaError_t launch_shadow_check(uint32_t grid, cudaStream_t stream, const DSpan* spans, uint32_t nspans,
-                                uint64_t tiles, uint64_t weight, const Ctx& k, int force_lanes,
-                                unsigned long long* sched) {
-    shadow_check_window<<<grid, THREADS, DYN_SMEM, stream>>>(spans, nspans, tiles, weight, k, force_lanes, sched);
+                                uint64_t tiles, uint64_t weight, const Ctx& k, unsigned long long* sched) {
+    shadow_check_window<<<grid, THREADS, DYN_SMEM, stream>>>(spans, nspans, tiles, weight, k, sched);
     return cudaGetLastError();
 }
 
 cudaError_t launch_copy_cells(uint32_t grid, cudaStream_t stream, const uint2* src, uint2* dst,
-                              const CopySeg* segs, uint32_t nseg, uint64_t total, uint32_t* heap) {
-    copy_cells<<<grid, THREADS, 0, stream>>>(src, dst, segs, nseg, total, heap);
+                              const CopySeg* segs, uint32_t nseg, uint64_t total) {
+    copy_cells<<<grid, THREADS, 0, stream>>>(src, dst, segs, nseg, total);
     return cudaGetLastError();
 }
 

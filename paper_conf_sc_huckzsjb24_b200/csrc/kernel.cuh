@@ -11,8 +11,7 @@
 namespace cusan {
 
 
-constexpr int U = 4;                    // 32-granule chunks per lane-parallel step
-constexpr int CHUNK = 32 * U;           // granules per lane-parallel step
+constexpr int CHUNK = 128;              // granule multiple of a warp range (16-B aligned cell pairs per lane)
 #ifndef CUSAN_UL
 #define CUSAN_UL 4
 #endif
@@ -68,8 +67,9 @@ constexpr int MAXS = 256;               // shared-memory read set per warp (≥ 
 constexpr unsigned FULL = 0xffffffffu;
 static_assert(CHUNK % CELL_ALIGN == 0, "ranges start on aligned shadow slots");
 
-// counters[]: 0 race granules, 1 raw runs, 2 heap top (record units), 3 heap overflow flag
-enum { C_RACE = 0, C_RUNS = 1, C_HEAP = 2, C_HEAP_OVF = 3, N_COUNTERS = 4 };
+// counters[]: 0 race granules, 1 raw runs, 2 heap top (record units), 3 heap overflow flag,
+// 4 ranges whose cells were not all equal (planner invariant violated: the check fails)
+enum { C_RACE = 0, C_RUNS = 1, C_HEAP = 2, C_HEAP_OVF = 3, C_INVARIANT = 4, N_COUNTERS = 5 };
 
 // A window's work on one elementary interval, cut into warp ranges of `rsize` granules.
 struct DSpan {
@@ -121,11 +121,10 @@ struct Window {
 // ---- launch wrappers (kernel.cu) ----------------------------------------------------------------
 // K1: one window of the shadow check
 cudaError_t launch_shadow_check(uint32_t grid, cudaStream_t stream, const DSpan* spans, uint32_t nspans,
-                                uint64_t tiles, uint64_t weight, const Ctx& k, int force_lanes,
-                                unsigned long long* sched);
+                                uint64_t tiles, uint64_t weight, const Ctx& k, unsigned long long* sched);
 // sessions: copy the cell of a split compressed interval to its new piece
 cudaError_t launch_copy_cells(uint32_t grid, cudaStream_t stream, const uint2* src, uint2* dst,
-                              const CopySeg* segs, uint32_t nseg, uint64_t total, uint32_t* heap);
+                              const CopySeg* segs, uint32_t nseg, uint64_t total);
 // resident blocks of K1 per SM (sets K1's dynamic shared memory limit first)
 cudaError_t shadow_check_blocks_per_sm(int* per_sm);        // cached per device
 cudaError_t shadow_check_blocks_per_sm_query(int* per_sm);  // sets the smem attribute, asks the occupancy API

@@ -161,11 +161,20 @@ static void radix_sort_pairs(std::vector<uint64_t>& key, std::vector<uint32_t>& 
     }
 }
 
+int check_flags(const cusan_check_opts& o) {
+    const int known = CUSAN_CHECK_DEFER_WORKSPACE | CUSAN_CHECK_INTERVAL_SHADOW | CUSAN_CHECK_DENSE_SHADOW;
+    if (o.flags & ~known) return fail(CUSAN_EINVAL, "unknown cusan_check_opts.flags bits");
+    if ((o.flags & CUSAN_CHECK_INTERVAL_SHADOW) && (o.flags & CUSAN_CHECK_DENSE_SHADOW))
+        return fail(CUSAN_EINVAL, "CUSAN_CHECK_INTERVAL_SHADOW and CUSAN_CHECK_DENSE_SHADOW exclude each other");
+    return CUSAN_OK;
+}
+
 int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uint64_t first_access,
                     uint64_t rec_base) {
     if (o.nshards < 1 || o.shard < 0 || o.shard >= o.nshards)
         return fail(CUSAN_EINVAL, "need 0 <= shard < nshards");
     if (o.window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
+    if (int st = check_flags(o)) return st;
     hp.opts = o;
     const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
     auto tick = [t0 = std::chrono::steady_clock::now(), dbg](const char* what) {
@@ -352,7 +361,7 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
         // with one window (or one cell per interval, f3) the work is the accesses replayed, so the
         // weight is the coverage (accesses covering the granule).
         const uint64_t Ws = o.window_events > 0 ? (uint64_t)o.window_events : std::max<uint64_t>(n_acc, 1);
-        const bool windowed = Ws < n_acc && !(o.flags & CUSAN_CHECK_INTERVAL_SHADOW);
+        const bool windowed = Ws < n_acc && !compressed_shadow(o);
         std::vector<uint64_t> wpg(giv.size());
         if (!windowed) {
             for (size_t i = 0; i < giv.size(); i++) wpg[i] = std::max<uint64_t>(giv[i].cnt, 1);
@@ -411,7 +420,7 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
     hp.iv.clear();
     std::vector<uint32_t> iv_j;                      // elementary interval of each shard interval
     uint64_t slot = 0, n_inc = 0;
-    const bool compressed = (o.flags & CUSAN_CHECK_INTERVAL_SHADOW) != 0;
+    const bool compressed = compressed_shadow(o);
     for (auto& g : giv) {
         uint64_t lo = std::max(g.dense_begin, d_lo), hi = std::min(g.dense_begin + g.len, d_hi);
         if (lo >= hi) continue;

@@ -163,10 +163,64 @@ static bool vm_grow(VmRange& r, int device, size_t bytes, size_t reserve = 0) {
 
 namespace {
 
+constexpr uint32_t NO_REC = 0xffffffffu;
+
 // one elementary interval of the session's layout
 struct SIv {
     uint64_t abs_begin, len, dense;
     std::bitset<CUSAN_MAX_FIBERS + 1> readers;   // fibers that read it since its last write
+    uint32_t rec = NO_REC;                       // read-set record its cells name (>= 2 readers)
+};
+
+// Read-set records of a session, allocated on the host.  A record is written once, by the span
+// that ends with its read set, and only read afterwards; it stays live while some interval's cells
+// name it (pieces of a split interval share their parent's record).  After each call's plan the
+// records no interval names any more are dead: they become reusable from the NEXT call's plan on —
+// the current call's kernels may still read them, and the next call's kernels run after them on
+// the same stream.  So the heap holds the live read sets (bounded by intervals × fibers) however
+// long the session runs, instead of growing with every call.
+struct RecAlloc {
+    uint64_t hwm = 0;                                       // units ever handed out = heap size needed
+    std::vector<std::vector<uint32_t>> free_by_units;       // reusable records by size (units)
+    std::vector<std::pair<uint32_t, uint32_t>> pending;     // dead in the current call: (rec, units)
+    std::unordered_map<uint32_t, uint32_t> live;            // allocated: rec -> units
+    uint64_t live_units = 0;
+
+    // a record of `units` units; false if the 24-bit record index is exhausted
+    bool alloc(uint32_t units, uint32_t* rec) {
+        if (units < free_by_units.size() && !free_by_units[units].empty()) {
+            *rec = free_by_units[units].back();
+            free_by_units[units].pop_back();
+        } else {
+            if (hwm + units >= (1ull << 24) - 1) return false;
+            *rec = (uint32_t)hwm;
+            hwm += units;
+        }
+        live.emplace(*rec, units);
+        live_units += units;
+        return true;
+    }
+    // records dead in the previous call become reusable (called when a call is planned)
+    void promote() {
+        for (const auto& d : pending) {
+            if (free_by_units.size() <= d.second) free_by_units.resize(d.second + 1);
+            free_by_units[d.second].push_back(d.first);
+        }
+        pending.clear();
+    }
+    // after a call's plan: every allocated record the layout no longer names is dead
+    template <class Layout>
+    void collect(const Layout& ivs) {
+        std::unordered_map<uint32_t, char> named;
+        for (const auto& v : ivs)
+            if (v.rec != NO_REC) named.emplace(v.rec, 1);
+        for (auto it = live.begin(); it != live.end();) {
+            if (named.count(it->first)) { ++it; continue; }
+            pending.emplace_back(it->first, it->second);
+            live_units -= it->second;
+            it = live.erase(it);
+        }
+    }
 };
 
 }  // namespace
@@ -196,7 +250,7 @@ struct cusan_session {
     DevBuf<uint32_t> segvc_d;                       // segment rows, u32 words
     uint64_t seg_uploaded = 0;                      // rows on the device
     DevBuf<uint32_t> heap;                          // read-set records, u32 words
-    uint64_t heap_top = 0;                          // record units in use
+    RecAlloc recs;                                  // which records are live / reusable
     DevBuf<char> scratch;                           // one call's tables and counters
     DevBuf<cusan_race_run> runs;                    // raw runs of one call
     DevBuf<char> merge_buf;                         // a4 scratch
@@ -246,11 +300,11 @@ static int grow_buf(cusan_session* s, DevBuf<T>& b, uint64_t need, uint64_t keep
     return CUSAN_OK;
 }
 
-// grow the heap keeping records [0, heap_top)
+// grow the heap keeping every record handed out so far
 static int grow_heap(cusan_session* s, uint64_t need_units) {
     if (s->heap_cap() >= need_units && s->heap.p) return CUSAN_OK;
-    if (need_units >= (1ull << 24)) return fail(CUSAN_ENOMEM, "read-set heap exceeds the 24-bit record index");
-    return grow_buf(s, s->heap, need_units * REC_WORDS, s->heap_top * REC_WORDS, "the read-set heap");
+    need_units = std::min<uint64_t>(need_units, (1ull << 24) - 1);
+    return grow_buf(s, s->heap, need_units * REC_WORDS, s->recs.hwm * REC_WORDS, "the read-set heap");
 }
 
 // run buffer for `n` raw runs and the a4 scratch to merge them
@@ -285,6 +339,7 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
     cusan_counters& c = cp.hp.ctr;
     c = cusan_counters{};
     c.n_fibers = F;
+    s->recs.promote();                 // records dead since the previous call's plan are free now
     // ---- a1: clocks and segments for the new events (build_host_plan's pass, resumed) ----------
     for (uint64_t i = s->checked_events; i < tr.ev.size(); i++) {
         const cusan_event& e = tr.ev[i];
@@ -373,7 +428,7 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
         diff[b0[k]]++;
         diff[b1[k]]--;
     }
-    const bool compressed = (s->opts.flags & CUSAN_CHECK_INTERVAL_SHADOW) != 0;
+    const bool compressed = compressed_shadow(s->opts);
     std::vector<uint32_t> iv_of(np ? np - 1 : 0, 0xffffffffu);
     uint64_t used = s->used;
     {
@@ -391,6 +446,7 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
             if (old) {                 // a piece of an old interval: its state, its cells in place
                 const SIv& o = s->ivs[u];
                 v.readers = o.readers;
+                v.rec = o.rec;
                 if (!compressed) {
                     v.dense = o.dense + (P[j] - o.abs_begin);
                 } else if (P[j] == o.abs_begin) {
@@ -477,7 +533,13 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
             sp.flags = ((!first_span || has_state) ? SPAN_LOAD : 0u) | SPAN_STORE |
                        (first_span ? SPAN_FIRST_IN_CALL : 0u) | (compressed ? SPAN_COMPRESSED : 0u);
             const uint64_t nr = v.readers.count();
-            if (nr >= 2) sp.rec_units = (uint32_t)((nr + 1 + REC_WORDS - 1) / REC_WORDS);
+            v.rec = NO_REC;                         // the span's store replaces the cells' R
+            if (nr >= 2) {
+                sp.rec_units = (uint32_t)((nr + 1 + REC_WORDS - 1) / REC_WORDS);
+                if (!s->recs.alloc(sp.rec_units, &sp.rec))
+                    return fail(CUSAN_ERANGE, "live read-set records exceed the 24-bit record index");
+                v.rec = sp.rec;
+            }
             out.emplace_back(w, sp);
             q = q2;
         }
@@ -496,7 +558,6 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
     hp.spill_spans = 0;
     for (Span& sp : hp.spans)
         if (sp.rec_units) {
-            sp.rec = (uint32_t)hp.rec_units;     // relative: the heap top is added at launch
             hp.rec_units += sp.rec_units;
             hp.spill_spans++;
         }
@@ -509,6 +570,9 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
     c.n_spans = hp.spans.size();
     c.spill_spans = hp.spill_spans;
     c.spill_heap_bytes = hp.rec_units * REC_WORDS * 4;
+    s->recs.collect(cp.ivs);           // records no interval of the new layout names are dead
+    c.heap_live_bytes = s->recs.live_units * REC_WORDS * 4;
+    c.heap_bytes = s->recs.hwm * REC_WORDS * 4;
     return CUSAN_OK;
 }
 
@@ -574,18 +638,12 @@ static int session_plan(cusan_session* s, PendingCall& pc) {
 // queued on the session's stream (a4's merge happens in session_finish).
 static int session_launch(cusan_session* s, PendingCall& pc) {
     CallPlan& cp = pc.cp;
-    HostPlan& hp = cp.hp;
     SpanTables& tabs = pc.tabs;
-    const uint64_t base = s->heap_top;                 // the previous call's records end here
-    if (base + hp.rec_units >= (1u << 24) - 1)
-        return fail(CUSAN_ERANGE, "too many read-set records for the 24-bit record index");
-    for (DSpan& d : tabs.ds)
-        if (d.rec_units) d.rec += (uint32_t)base;
     // the shadow grows as new memory is touched: new chunks mapped in place, else re-allocated
     // with its cells moved (1/8 headroom either way)
     int st;
     if ((st = grow_buf(s, s->shadow, cp.used, pc.used_before, "the shadow"))) return st;
-    if ((st = grow_heap(s, base + hp.rec_units + (1ull << 16)))) return st;
+    if ((st = grow_heap(s, s->recs.hwm + (s->recs.hwm >> 3) + 1024))) return st;
     uint64_t tiles = 0;                 // raw-run bound heuristic, as in plans (an overflow truncates)
     for (const Window& w : tabs.wins) tiles += w.tiles;
     if ((st = grow_runs(s, 2 * tiles + 1024))) return st;
@@ -615,13 +673,13 @@ static int session_launch(cusan_session* s, PendingCall& pc) {
     // ---- a3, in place ------------------------------------------------------------------------------
     pc.init.assign(N_COUNTERS + nwin, 0ull);
     pc.cnt.assign(N_COUNTERS, 0ull);
-    pc.init[C_HEAP] = base + hp.rec_units;
+    pc.init[C_HEAP] = s->heap_cap();     // records are host-assigned: no device allocation
     CK(cudaMemcpyAsync(d_cnt, pc.init.data(), pc.init.size() * sizeof(unsigned long long), cudaMemcpyHostToDevice,
                        s->stream));
     CK(cudaEventRecord(s->ev0, s->stream));
     if (cp.copy_cells)
         CK(launch_copy_cells(s->max_blocks, s->stream, s->shadow.p, s->shadow.p, d_copy, (uint32_t)cp.segs.size(),
-                             cp.copy_cells, s->heap.p));
+                             cp.copy_cells));
     Ctx k;
     k.inc = d_inc;
     k.segvc = s->segvc_d.p;
@@ -632,12 +690,10 @@ static int session_launch(cusan_session* s, PendingCall& pc) {
     k.runs = s->runs.p;
     k.counters = d_cnt;
     k.run_cap = s->runs.cap;
-    const int force_lanes = (s->opts.flags & CUSAN_CHECK_FORCE_LANES) ? 1 : 0;
     for (size_t i = 0; i < nwin; i++) {
         const Window& w = tabs.wins[i];
         unsigned long long* sched = CUSAN_DYNAMIC ? d_cnt + N_COUNTERS + i : nullptr;
-        CK(launch_shadow_check(w.grid, s->stream, d_spans + w.span_off, w.nspans, w.tiles, w.weight, k, force_lanes,
-                               sched));
+        CK(launch_shadow_check(w.grid, s->stream, d_spans + w.span_off, w.nspans, w.tiles, w.weight, k, sched));
     }
     CK(cudaEventRecord(s->ev1, s->stream));
     CK(cudaMemcpyAsync(pc.cnt.data(), d_cnt, N_COUNTERS * sizeof(unsigned long long), cudaMemcpyDeviceToHost,
@@ -653,11 +709,11 @@ static int session_finish(cusan_session* s, PendingCall& pc, cusan_report** out)
     const uint64_t* cnt = (const uint64_t*)pc.cnt.data();
     float kms = 0.f;
     CK(cudaEventElapsedTime(&kms, s->ev0, s->ev1));
-    if (cnt[C_HEAP_OVF]) {
+    if (cnt[C_HEAP_OVF] || cnt[C_INVARIANT]) {
         s->broken = true;
-        return fail(CUSAN_ENOMEM, "read-set heap overflow: the session's state is lost");
+        return fail(CUSAN_ESTATE, "internal error: a read set outgrew its record or cells of one interval "
+                                  "differ; the session's state is lost");
     }
-    s->heap_top = cnt[C_HEAP];
     const bool runs_ovf = cnt[C_RUNS] > s->runs.cap;
     const uint64_t kept_runs = std::min<uint64_t>(cnt[C_RUNS], s->runs.cap);
     cusan_report* r = new (std::nothrow) cusan_report;
@@ -702,6 +758,8 @@ int cusan_session_create(const cusan_trace* t, const cusan_check_opts* o, cusan_
         return fail(CUSAN_EINVAL, "shard_block must be a power of two (or 0)");
     if (o->workspace) return fail(CUSAN_EINVAL, "sessions manage their own device memory");
     if (o->window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
+    if (int st = check_flags(*o)) return st;
+    if (o->flags & CUSAN_CHECK_DEFER_WORKSPACE) return fail(CUSAN_EINVAL, "sessions manage their own device memory");
     cusan_session* s = new (std::nothrow) cusan_session;
     if (!s) return fail(CUSAN_ENOMEM, "cannot allocate session");
     s->trace = t;

@@ -55,11 +55,11 @@ def test_listing_on_gpu(lst):
     assert_equal(rep, oracle.check_events(ev, 256, threads=1))
 
 
-@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_FORCE_LANES], ids=["ranges", "lanes"])
+@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_DENSE_SHADOW], ids=["compressed", "dense"])
 @pytest.mark.parametrize("window", [0, 1, 2, 7])
 def test_fuzz_primitive_traces(window, flags):
-    """Random traces spanning several lane steps (128 granules) with ragged tails; both the
-    equal-cells range path and the lane-parallel path."""
+    """Random traces spanning several warp ranges with ragged tails; both shadow layouts (one cell
+    per elementary interval, the default, and one cell per granule)."""
     rng = np.random.default_rng(40 + window)
     for i in range(60):
         nf = int(rng.integers(2, 9))
@@ -83,7 +83,7 @@ def test_spill_path_many_readers():
         ev["mode"][flip] = 0
         ref = oracle.check_events(ev, nf, threads=2)
         for window in (0, 3):
-            for flags in (0, cs.CUSAN_CHECK_FORCE_LANES):
+            for flags in (0, cs.CUSAN_CHECK_DENSE_SHADOW):
                 rep = gpu_report(ev, nf, window_events=window, flags=flags)
                 assert_equal(rep, ref)
                 hit_spill += rep.counters["spill_spans"] > 0
@@ -91,8 +91,8 @@ def test_spill_path_many_readers():
 
 
 @pytest.mark.parametrize("nshards", [2, 3, 5])
-@pytest.mark.parametrize("window,flags", [(0, 0), (3, 0), (3, cs.CUSAN_CHECK_INTERVAL_SHADOW)],
-                         ids=["one-window", "windowed", "windowed-compressed"])
+@pytest.mark.parametrize("window,flags", [(0, cs.CUSAN_CHECK_DENSE_SHADOW), (3, cs.CUSAN_CHECK_DENSE_SHADOW), (3, 0)],
+                         ids=["one-window-dense", "windowed-dense", "windowed-compressed"])
 def test_shards_merge_to_the_whole(nshards, window, flags):
     """Shard boundaries come from the coverage (one window) or from the windows touching each
     interval (windowed); either way the shards' merged runs are the whole trace's."""
@@ -133,7 +133,7 @@ def test_small_configs(c, racy):
     ev = tr.cusan_trace_read()
     ref = oracle.check_events(ev, 256)
     for window in (0, 97):
-        for flags in (0, cs.CUSAN_CHECK_FORCE_LANES):
+        for flags in (0, cs.CUSAN_CHECK_DENSE_SHADOW):
             assert_equal(cs.check(tr, window_events=window, flags=flags), ref)
     assert (ref["n_race_granules"] > 0) == racy
 
@@ -155,7 +155,7 @@ def test_edge_cases():
     t.cusan_trace_append_access(0, 1, 0x2000, 8)
     ref = oracle.check_events(t.cusan_trace_read(), 255)
     for window in (0, 1, 100):
-        for flags in (0, cs.CUSAN_CHECK_FORCE_LANES):
+        for flags in (0, cs.CUSAN_CHECK_DENSE_SHADOW):
             rep = cs.check(t, window_events=window, flags=flags)
             assert rep.n_race_granules == 254
             assert_equal(rep, ref)
@@ -197,8 +197,9 @@ def test_full_size_configs_sampled(c):
     ev = tr.cusan_trace_read()
     import torch
     s = torch.cuda.Stream()
-    rep = cs.check(tr, window_events=4096, workspace="torch", stream=s.cuda_stream)   # as bench.py runs it
-    one = cs.check(tr)                                                                # post-mortem: one window
+    rep = cs.check(tr, window_events=4096, workspace="torch", stream=s.cuda_stream,
+                   flags=cs.CUSAN_CHECK_DENSE_SHADOW)                                # as bench.py runs it
+    one = cs.check(tr)                                                 # compressed, post-mortem: one window
     assert one.n_race_granules == rep.n_race_granules and np.array_equal(one.runs, rep.runs)
     assert rep.n_race_granules > 0
     assert rep.n_race_granules == int(np.sum(rep.runs["g_end"] - rep.runs["g_begin"]))
@@ -232,9 +233,10 @@ def test_full_size_configs_exact(c, twin):
     assert (ref["n_race_granules"] > 0) == (twin == "racy")
     import torch
     s = torch.cuda.Stream()
-    rep = cs.check(tr, window_events=4096, workspace="torch", stream=s.cuda_stream)   # as bench.py runs it
-    assert rep.counters["tracked_bytes"] == int(g["tracked_bytes"])
-    assert_equal(rep, ref)
+    for flags in (cs.CUSAN_CHECK_DENSE_SHADOW, 0):      # both bench lines: dense, compressed
+        rep = cs.check(tr, window_events=4096, workspace="torch", stream=s.cuda_stream, flags=flags)
+        assert rep.counters["tracked_bytes"] == int(g["tracked_bytes"])
+        assert_equal(rep, ref)
     if c in (4, 5):
         parts = [cs.check(tr, window_events=4096, nshards=8, shard=k) for k in range(8)]
         merged = cs.report_merge(np.concatenate([p.runs for p in parts]), sum(p.n_race_granules for p in parts))
@@ -295,7 +297,8 @@ def test_run_buffer_overflow_reruns_exactly():
     ev = _events([(EV_ACCESS, 1, f, base, 8 * n_gran) for f in range(n_fib)])
     tr = cs.Trace(255)
     tr.cusan_trace_append_events(ev)
-    p = cs.Plan(tr, window_events=50)         # 4 windows, 512 ranges each, 50 racing pairs per range
+    p = cs.Plan(tr, window_events=50, flags=cs.CUSAN_CHECK_DENSE_SHADOW)   # 4 windows, 512 ranges each,
+    #                                                                      50 racing pairs per range
     rep = p.run()
     assert rep.counters["raw_runs"] > (1 << 16)                 # beyond the initial buffer
     assert rep.n_race_granules == (n_fib - 1) * n_gran
@@ -307,17 +310,36 @@ def test_run_buffer_overflow_reruns_exactly():
     p.close()
 
 
-def test_heap_overflow_reruns_exactly():
-    """Lane path with three readers per granule: the second reader of every granule allocates a
-    record, more than the plan's initial heap room; the plan grows the heap and re-runs.  A final
-    unsynchronised write races with each read: 3 runs of the whole range."""
-    n_gran, base = 1 << 17, 1 << 36
-    rows = [(EV_ACCESS, 0, f, base, 8 * n_gran) for f in (0, 1, 2)] + [(EV_ACCESS, 1, 3, base, 8 * n_gran)]
-    tr = cs.Trace(8)
-    tr.cusan_trace_append_events(_events(rows))
-    rep = cs.check(tr, flags=cs.CUSAN_CHECK_FORCE_LANES, window_events=1)
-    assert rep.n_race_granules == 3 * n_gran
-    assert [tuple(int(x) for x in r) for r in rep.runs] == [(base >> 3, (base >> 3) + n_gran, e, 3) for e in range(3)]
+@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_DENSE_SHADOW], ids=["compressed", "dense"])
+def test_interval_longer_than_2_31_granules(flags):
+    """An elementary interval of more than 2^31 granules (17 GB of address): a compressed span is
+    one range owning its single cell, a dense span is cut into ranges at the right offsets.
+    Closed form: W f0, W f1, R f2 over the whole range, unsynchronised, each access in its own
+    window: runs (0 -> 1) and (1 -> 2) over all N granules.  The oracle checks sampled granules at
+    the 2^31 boundary and both ends."""
+    n_gran, base = (1 << 31) + 4096 + 40, 1 << 40
+    g0 = base >> 3
+    rows = [(EV_ACCESS, 1, 0, base, 8 * n_gran), (EV_ACCESS, 1, 1, base, 8 * n_gran),
+            (EV_ACCESS, 0, 2, base, 8 * n_gran)]
+    ev = _events(rows)
+    want = [(g0, g0 + n_gran, 0, 1), (g0, g0 + n_gran, 1, 2)]
+    sample = np.array([g0, g0 + 1, g0 + (1 << 31) - 1, g0 + (1 << 31), g0 + n_gran - 1], np.uint64)
+    ref = oracle.check_events(ev, 3, sample=sample)
+    assert brute.runs_to_triples(ref["runs"]) == {(int(g), e, l) for g in sample for _, _, e, l in want}
+    tr = cs.Trace(3)
+    tr.cusan_trace_append_events(ev)
+    rep = cs.check(tr, window_events=1, flags=flags)
+    assert [tuple(int(x) for x in r) for r in rep.runs] == want
+    assert rep.n_race_granules == 2 * n_gran
+    if flags == 0:
+        assert rep.counters["shadow_bytes"] <= 64
+        ses = cs.Session(cs.Trace(3), window_events=1)        # the in-place session path
+        got = []
+        for k in range(3):
+            ses.trace.cusan_trace_append_events(ev[k:k + 1])
+            got += [tuple(int(x) for x in r) for r in ses.check().runs]
+        assert got == want
+        ses.close()
 
 
 def test_largest_event_id_on_the_gpu():
@@ -333,12 +355,12 @@ def test_largest_event_id_on_the_gpu():
     ev[n - 1]["a"], ev[n - 1]["b"] = base, 8 * n_gran
     tr = cs.Trace(2)
     tr.cusan_trace_append_events(ev)
-    for kw in ({}, {"flags": cs.CUSAN_CHECK_FORCE_LANES}, {"flags": cs.CUSAN_CHECK_INTERVAL_SHADOW}):
+    for kw in ({}, {"flags": cs.CUSAN_CHECK_DENSE_SHADOW}, {"flags": cs.CUSAN_CHECK_INTERVAL_SHADOW}):
         rep = cs.check(tr, **kw)
         assert [tuple(int(x) for x in r) for r in rep.runs] == [(base >> 3, (base >> 3) + n_gran, 0, n - 1)]
 
 
-@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_FORCE_LANES], ids=["ranges", "lanes"])
+@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_DENSE_SHADOW], ids=["compressed", "dense"])
 def test_maximum_fibers_read_set(flags):
     """255 fibers (the most an epoch encodes) read a range, then fiber 0 writes it: the full read
     set (254 other readers) lives in a record and every unordered reader races."""
@@ -417,8 +439,8 @@ def test_library_workspace_is_reused_and_released():
 ], ids=["lane-step", "1Ki", "balance", "whole-span", "no-tail", "all-tail"])
 def test_results_do_not_depend_on_the_work_decomposition(ranges, monkeypatch):
     """SURVEY §8(c) pin "invariance under tile size": the warp range length (the kernel's work unit,
-    sized on the host) from one lane step to a whole span gives the oracle's report, on both kernel
-    paths and with shards."""
+    sized on the host) from one lane step to a whole span gives the oracle's report, in both shadow
+    layouts and with shards."""
     for k, v in ranges.items():
         monkeypatch.setenv(k, v)
     for c in (3, 5):
@@ -427,7 +449,7 @@ def test_results_do_not_depend_on_the_work_decomposition(ranges, monkeypatch):
         tr, _ = lower_product(ops, args)
         ref = oracle.check_events(tr.cusan_trace_read(), 256)
         for window in (0, 97):
-            for flags in (0, cs.CUSAN_CHECK_FORCE_LANES):
+            for flags in (0, cs.CUSAN_CHECK_DENSE_SHADOW):
                 assert_equal(cs.check(tr, window_events=window, flags=flags), ref)
         parts = [cs.check(tr, window_events=97, nshards=3, shard=s) for s in range(3)]
         assert_equal(cs.report_merge(np.concatenate([p.runs for p in parts]),

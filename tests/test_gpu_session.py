@@ -40,7 +40,7 @@ def _run_session(ev, nf, cuts, **kw):
     return ref
 
 
-@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_FORCE_LANES], ids=["ranges", "lanes"])
+@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_DENSE_SHADOW], ids=["compressed", "dense"])
 @pytest.mark.parametrize("window", [0, 3])
 def test_session_fuzz(window, flags):
     rng = np.random.default_rng(600 + window)
@@ -64,7 +64,7 @@ def test_session_many_readers_across_calls():
         acc = ev["kind"] == EV_ACCESS
         ev["mode"][acc & (rng.random(len(ev)) < 0.8)] = 0
         cuts = sorted(int(x) for x in rng.integers(1, len(ev), size=4))
-        for flags in (0, cs.CUSAN_CHECK_FORCE_LANES):
+        for flags in (0, cs.CUSAN_CHECK_DENSE_SHADOW):
             _run_session(ev, nf, cuts, flags=flags)
 
 
@@ -106,7 +106,7 @@ def test_session_interval_compressed():
 
 def test_session_compressed_shared_records_across_splits():
     """f3 sessions: a split compressed interval copies its cell; a read-set record it names becomes
-    shared, so an update through either cell must not show through the other."""
+    shared by both cells (records are written once and never updated in place)."""
     rng = np.random.default_rng(91)
     for _ in range(15):
         nf = int(rng.integers(6, 30))
@@ -115,8 +115,7 @@ def test_session_compressed_shared_records_across_splits():
         acc = ev["kind"] == EV_ACCESS
         ev["mode"][acc & (rng.random(len(ev)) < 0.8)] = 0
         cuts = sorted(set(int(x) for x in rng.integers(1, len(ev), size=10)))
-        for flags in (0, cs.CUSAN_CHECK_FORCE_LANES):
-            _run_session(ev, nf, cuts, flags=flags | cs.CUSAN_CHECK_INTERVAL_SHADOW)
+        _run_session(ev, nf, cuts, flags=cs.CUSAN_CHECK_INTERVAL_SHADOW)
 
 
 def test_session_shadow_growth_many_calls():
@@ -143,7 +142,7 @@ def test_session_shadow_growth_many_calls():
 
 
 @pytest.mark.parametrize("nshards,block", [(2, 64), (3, 32), (4, 1 << 12)])
-@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_INTERVAL_SHADOW], ids=["per-granule", "compressed"])
+@pytest.mark.parametrize("flags", [cs.CUSAN_CHECK_DENSE_SHADOW, 0], ids=["per-granule", "compressed"])
 def test_session_block_cyclic_shards_merge_per_call(nshards, block, flags):
     """Multi-GPU sessions: per call, the merged reports of the block-cyclic shards equal the
     one-shard session's report of that call (which the other session tests pin to the oracle);
@@ -197,9 +196,9 @@ def test_session_shards_small_config():
         s.close()
 
 
-@pytest.mark.parametrize("flags,nshards", [(0, 1), (cs.CUSAN_CHECK_FORCE_LANES, 1),
-                                           (cs.CUSAN_CHECK_INTERVAL_SHADOW, 1), (0, 2)],
-                         ids=["ranges", "lanes", "compressed", "shards"])
+@pytest.mark.parametrize("flags,nshards", [(cs.CUSAN_CHECK_DENSE_SHADOW, 1), (0, 1),
+                                           (cs.CUSAN_CHECK_DENSE_SHADOW, 2), (0, 2)],
+                         ids=["dense", "compressed", "dense-shards", "compressed-shards"])
 def test_session_submit_pipelines_and_matches_check(flags, nshards):
     """submit/finish (host planning of call i+1 overlapping the device work of call i, records
     numbered at launch) return, call by call, exactly what check() returns."""
@@ -231,3 +230,46 @@ def test_session_submit_pipelines_and_matches_check(flags, nshards):
                 assert np.array_equal(x.runs, y.runs)
             sa.close()
             sb.close()
+
+
+@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_DENSE_SHADOW], ids=["compressed", "dense"])
+def test_session_read_set_records_are_reclaimed(flags):
+    """Intervals read by several fibers in every call (weights read by forward and backward
+    streams) get a new read-set record per call; the records the layout no longer names are reused
+    from the next call on, so the heap stays at its high-water mark of the first calls instead of
+    growing call after call.  Every call still equals the oracle's report restricted to it."""
+    from tracegen.program import EVENT_DTYPE, EV_ACQUIRE, EV_RELEASE
+    rows = []
+    base, size, n_calls, per_call = 1 << 33, 1 << 16, 60, []
+    for c in range(n_calls):
+        start = len(rows)
+        for f in (1, 2, 3):                                   # three readers of both buffers
+            rows.append((EV_ACCESS, 0, f, base, size))
+            rows.append((EV_ACCESS, 0, f, base + 2 * size, size))
+        if c % 7 == 3:                                        # an unordered write now and then
+            rows.append((EV_ACCESS, 1, 4, base + 2 * size + 64, 256))
+        for f in (1, 2, 3):
+            rows.append((EV_RELEASE, 0, f, 100 + f, 0))
+            rows.append((EV_ACQUIRE, 0, 0, 100 + f, 0))
+        rows.append((EV_ACCESS, 1, 0, base + size // 2, size // 4))   # host writes part of buffer 0
+        rows.append((EV_RELEASE, 0, 0, 99, 0))
+        for f in (1, 2, 3, 4):
+            rows.append((EV_ACQUIRE, 0, f, 99, 0))
+        per_call.append((start, len(rows)))
+    ev = np.zeros(len(rows), EVENT_DTYPE)
+    for i, (k, m, f, a, b) in enumerate(rows):
+        ev[i]["kind"], ev[i]["mode"], ev[i]["fiber"], ev[i]["a"], ev[i]["b"] = k, m, f, a, b
+    ref = oracle.check_events(ev, 5, threads=2)
+    assert ref["n_race_granules"] > 0
+    tr = cs.Trace(5)
+    ses = cs.Session(tr, window_events=2, flags=flags)
+    heap = []
+    for a, b in per_call:
+        tr.cusan_trace_append_events(ev[a:b])
+        rep = ses.check()
+        want = _by_later(ref["runs"], a, b)
+        assert np.array_equal(rep.runs, want.astype(rep.runs.dtype)), (a, b)
+        heap.append(rep.counters["heap_bytes"])
+        assert rep.counters["heap_live_bytes"] <= rep.counters["heap_bytes"]
+    ses.close()
+    assert heap[-1] == heap[10] > 0, heap         # bounded: no growth once the layout is stable

@@ -30,7 +30,7 @@ a = ap.parse_args()
 
 rng = np.random.default_rng(a.seed)
 stats = {"cases": 0, "checks": 0, "mismatches": 0, "racy_cases": 0, "by_mode": {}, "first_failures": []}
-FL, IV = cs.CUSAN_CHECK_FORCE_LANES, cs.CUSAN_CHECK_INTERVAL_SHADOW
+FL, IV = cs.CUSAN_CHECK_DENSE_SHADOW, cs.CUSAN_CHECK_INTERVAL_SHADOW
 
 
 def same(rep_runs, rep_n, ref):
@@ -56,7 +56,7 @@ def one_case(ev, nf, case):
     n_acc = int(np.sum(ev["kind"] == 0))
     windows = [0, int(rng.integers(1, 6)), max(1, n_acc // 3)]
     for w in windows:
-        for flags in (0, FL, IV, IV | FL):
+        for flags in (0, FL, IV):
             r = cs.check(tr, window_events=w, flags=flags)
             record(f"oneshot w={'all' if w == 0 else 'small'} flags={flags}", same(r.runs, r.n_race_granules, ref), case)
     ns = int(rng.integers(2, 6))

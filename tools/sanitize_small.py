@@ -19,7 +19,7 @@ for c in (1, 3, 5):
     tr = cs.Trace(255)
     cs.Lowering(tr).cusan_lower_program(ops, args)
     ref = oracle.check_events(tr.cusan_trace_read(), 255)
-    for kw in (dict(), dict(window_events=40), dict(window_events=40, flags=cs.CUSAN_CHECK_FORCE_LANES),
+    for kw in (dict(), dict(window_events=40), dict(window_events=40, flags=cs.CUSAN_CHECK_DENSE_SHADOW),
                dict(window_events=40, flags=cs.CUSAN_CHECK_INTERVAL_SHADOW), dict(nshards=3, shard=1)):
         rep = cs.check(tr, **kw)
         if "nshards" not in kw:
@@ -30,8 +30,7 @@ for _ in range(10):
     ev = fuzz.random_primitive_trace(rng, 120, nf, n_keys=3, n_granules=600, p_access=0.8)
     ev["mode"][(ev["kind"] == 0) & (rng.random(len(ev)) < 0.7)] = 0
     ref = oracle.check_events(ev, nf)
-    for flags in (0, cs.CUSAN_CHECK_FORCE_LANES, cs.CUSAN_CHECK_INTERVAL_SHADOW,
-                  cs.CUSAN_CHECK_INTERVAL_SHADOW | cs.CUSAN_CHECK_FORCE_LANES):
+    for flags in (0, cs.CUSAN_CHECK_DENSE_SHADOW, cs.CUSAN_CHECK_INTERVAL_SHADOW):
         tr = cs.Trace(nf)
         ses = cs.Session(tr, window_events=7, flags=flags)
         total = 0
