@@ -129,6 +129,11 @@ typedef struct cusan_check_opts {
  * Passing both is CUSAN_EINVAL.  (Flag value 1, a removed diagnostic, is rejected too.) */
 #define CUSAN_CHECK_INTERVAL_SHADOW 4
 #define CUSAN_CHECK_DENSE_SHADOW 8
+/* Build the plan's interval, incidence and span tables (step a2) on the host instead of the device.
+ * By default cusan_plan_create runs a1 on the host and a2 on the GPU (sm_100a kernels + CUB sorts
+ * and scans, plan_dev.cu) and waits for it; the tables are identical either way (the host path is
+ * the reference the tests compare the device tables with, and what cusan_plan_describe runs). */
+#define CUSAN_CHECK_HOST_PLAN 16
 
 /* Defaults: nshards 1, shard 0, device 0, window_events 0, persist 0, max_runs 0, all NULL. */
 void cusan_check_opts_init(cusan_check_opts* o);
@@ -155,6 +160,13 @@ int cusan_plan_run(cusan_plan* p, cusan_report** out);
  * workspace is parked for the next plan on the device (one block per device, the largest) instead
  * of freed: cudaMalloc / cudaFree of a tens-of-GB shadow cost tens of ms each. */
 int cusan_plan_destroy(cusan_plan* p);
+/* Diagnostics: copies the plan's device tables to host memory — the incidence table (8-B records
+ * {epoch, segment | write << 31}, *n_inc of them) and the span tables of every window (72-B DSpan
+ * records incl. one sentinel per window, *n_spans of them) — if the buffers hold them (capacities
+ * in records; NULL buffers only report the counts).  Used to check that device-built tables equal
+ * host-built ones (CUSAN_CHECK_HOST_PLAN).  Waits for the plan's stream. */
+int cusan_plan_tables(const cusan_plan* p, void* inc, uint64_t inc_cap, void* spans, uint64_t spans_cap,
+                      uint64_t* n_inc, uint64_t* n_spans);
 /* Frees the parked workspaces (all devices).  Set CUSAN_NO_WORKSPACE_CACHE=1 to never park. */
 int cusan_release_cached_memory(void);
 /* Host steps a1 and a2 only (no device needed): fills the trace / plan counters the same

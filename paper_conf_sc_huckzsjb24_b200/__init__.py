@@ -180,6 +180,12 @@ def _report(h, max_runs):
 CUSAN_CHECK_DEFER_WORKSPACE = 2
 CUSAN_CHECK_INTERVAL_SHADOW = 4    # the default shadow: one cell per elementary interval (f3)
 CUSAN_CHECK_DENSE_SHADOW = 8       # one cell per 8-byte granule (TSan's layout, §8(d) roofline line)
+CUSAN_CHECK_HOST_PLAN = 16         # build the a2 tables on the host (default: on the device)
+DSPAN_DTYPE = np.dtype([("abs_begin", "<u8"), ("dense_begin", "<u8"), ("len", "<u8"), ("tile0", "<u8"),
+                        ("weight0", "<u8"), ("rsize", "<u4"), ("rweight", "<u4"), ("list_off", "<u4"),
+                        ("list_cnt", "<u4"), ("flags", "<u4"), ("rec", "<u4"), ("rec_units", "<u4"),
+                        ("pad", "<u4")])
+INC_DTYPE = np.dtype([("epoch", "<u4"), ("segm", "<u4")])
 
 
 def _torch_workspace(nbytes: int, device: int, stream):
@@ -239,6 +245,14 @@ class Plan:
         h = C.c_void_p()
         _ck(lib.cusan_plan_run(self.h, C.byref(h)))
         return _report(h, self.max_runs)
+
+    def cusan_plan_tables(self) -> tuple[np.ndarray, np.ndarray]:
+        """The plan's device tables (diagnostics): incidence records and span-table records."""
+        ni, ns = C.c_uint64(), C.c_uint64()
+        _ck(lib.cusan_plan_tables(self.h, None, 0, None, 0, C.byref(ni), C.byref(ns)))
+        inc, spans = np.zeros(ni.value, INC_DTYPE), np.zeros(ns.value, DSPAN_DTYPE)
+        _ck(lib.cusan_plan_tables(self.h, _ptr(inc), ni.value, _ptr(spans), ns.value, C.byref(ni), C.byref(ns)))
+        return inc, spans
 
     def close(self, _destroy=lib.cusan_plan_destroy):
         if getattr(self, "h", None):

@@ -84,6 +84,7 @@ PROTOS = {
     "cusan_plan_run": [P, PP],
     "cusan_plan_destroy": [P],
     "cusan_release_cached_memory": [],
+    "cusan_plan_tables": [P, P, u64, P, u64, pu64, pu64],
     "cusan_plan_describe": [P, C.POINTER(cusan_check_opts), C.POINTER(cusan_counters)],
     "cusan_session_create": [P, C.POINTER(cusan_check_opts), PP],
     "cusan_session_check": [P, PP],

@@ -12,6 +12,7 @@
 #include <string>
 
 #include "kernel.cuh"
+#include "plan_dev.h"
 
 using namespace cusan;
 
@@ -137,8 +138,12 @@ struct cusan_plan {
     std::vector<unsigned long long> counter_init;
     RunMerge merge;                         // a4 scratch (device run merge)
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    bool dev_planned = false;               // a2 ran on the device: tables live in dscr
+    DevScratch* dscr = nullptr;
+    uint64_t n_ds = 0;                      // span table records (device-planned)
 
     ~cusan_plan() {
+        if (dscr) plan_dev_release(dscr);
         if (ev0) cudaEventDestroy(ev0);
         if (ev1) cudaEventDestroy(ev1);
         if (own) ws_release(device, own, own_bytes);
@@ -234,17 +239,26 @@ uint64_t env_u64_or_zero(const char* name, uint64_t dflt) {
 }
 }  // namespace
 
+// guided tail: the last TAIL_PCT % of each long span's ranges are cut TAIL_DIV times smaller and
+// queued after every span's head, so the last work a launch hands out is small and the grid drains
+// evenly (warps take ranges in queue order from the dynamic scheduler)
+static DevPlanArgs span_args(int max_blocks) {
+    DevPlanArgs a;
+    a.R_MIN = env_u64("CUSAN_RANGE_MIN", CUSAN_RANGE_MIN);
+    a.R_MAX = std::max<uint64_t>(env_u64("CUSAN_RANGE_MAX", CUSAN_RANGE_MAX), 1);
+    a.R_PER_ACC = env_u64("CUSAN_RANGE_PER_ACCESS", CUSAN_RANGE_PER_ACCESS);
+    a.R_BAL_MIN = env_u64("CUSAN_RANGE_BAL_MIN", CUSAN_RANGE_BAL_MIN);
+    a.R_PER_WARP = env_u64("CUSAN_RANGES_PER_WARP", CUSAN_RANGES_PER_WARP);
+    a.TAIL_PCT = std::min<uint64_t>(env_u64_or_zero("CUSAN_TAIL_PCT", CUSAN_TAIL_PCT), 99);
+    a.TAIL_DIV = std::max<uint64_t>(env_u64("CUSAN_TAIL_DIV", CUSAN_TAIL_DIV), 1);
+    a.max_blocks = max_blocks;
+    return a;
+}
+
 void cusan::build_span_tables(const HostPlan& hp, int max_blocks, SpanTables& out) {
-    const uint64_t R_MIN = env_u64("CUSAN_RANGE_MIN", CUSAN_RANGE_MIN);
-    const uint64_t R_MAX = std::max<uint64_t>(env_u64("CUSAN_RANGE_MAX", CUSAN_RANGE_MAX), 1);
-    const uint64_t R_PER_ACC = env_u64("CUSAN_RANGE_PER_ACCESS", CUSAN_RANGE_PER_ACCESS);
-    const uint64_t R_BAL_MIN = env_u64("CUSAN_RANGE_BAL_MIN", CUSAN_RANGE_BAL_MIN);
-    const uint64_t R_PER_WARP = env_u64("CUSAN_RANGES_PER_WARP", CUSAN_RANGES_PER_WARP);
-    // guided tail: the last TAIL_PCT % of each long span's ranges are cut TAIL_DIV times smaller and
-    // queued after every span's head, so the last work a launch hands out is small and the grid
-    // drains evenly (warps take ranges in queue order from the dynamic scheduler)
-    const uint64_t TAIL_PCT = std::min<uint64_t>(env_u64_or_zero("CUSAN_TAIL_PCT", CUSAN_TAIL_PCT), 99);
-    const uint64_t TAIL_DIV = std::max<uint64_t>(env_u64("CUSAN_TAIL_DIV", CUSAN_TAIL_DIV), 1);
+    const DevPlanArgs a = span_args(max_blocks);
+    const uint64_t R_MIN = a.R_MIN, R_MAX = a.R_MAX, R_PER_ACC = a.R_PER_ACC, R_BAL_MIN = a.R_BAL_MIN;
+    const uint64_t R_PER_WARP = a.R_PER_WARP, TAIL_PCT = a.TAIL_PCT, TAIL_DIV = a.TAIL_DIV;
     pinned_vector<DSpan>& ds = out.ds;
     std::vector<DSpan> tails;
     ds.clear();
@@ -371,7 +385,44 @@ static int plan_device_setup(cusan_plan* p) {
     p->stream = (cudaStream_t)o.stream;
 
     SpanTables st;
-    build_span_tables(hp, p->max_blocks, st);
+    uint64_t dev_h2d = 0;
+    if (p->dev_planned) {
+        // a2 on the device: the tables stay in the plan's planning scratch
+        p->dscr = plan_dev_acquire(p->device);
+        if (!p->dscr) return fail(CUSAN_ENOMEM, "cannot create the device planning scratch");
+        DevPlanOut dp;
+        int e = device_plan_a2(hp, span_args(p->max_blocks), *p->dscr, dp);
+        if (e) return e;
+        cusan_counters& c = hp.ctr;
+        c.n_intervals = dp.n_intervals;
+        c.n_incidences = dp.n_inc;
+        c.shard_granules = hp.shard_granules = dp.shard_granules;
+        c.tracked_bytes_shard = dp.tracked_bytes_shard;
+        c.spill_spans = hp.spill_spans = dp.spill_spans;
+        hp.rec_units = dp.rec_units;
+        c.spill_heap_bytes = dp.rec_units * REC_WORDS * 4;
+        c.n_windows = dp.wins.size();
+        c.n_spans = dp.n_spans;
+        hp.shadow_cells = dp.shadow_cells;
+        for (const WinDesc& d : dp.wins) {
+            Window w{};
+            w.span_off = d.span_off;
+            w.nspans = d.nspans;
+            w.tiles = d.tiles;
+            w.weight = d.weight;
+            w.grid = (uint32_t)std::min<uint64_t>((uint64_t)p->max_blocks, (d.tiles + WARPS - 1) / WARPS);
+            if (w.grid == 0) w.grid = 1;
+            st.wins.push_back(w);
+        }
+        st.need_shadow = dp.need_shadow;
+        st.cell_bytes = dp.cell_bytes;
+        p->d_inc = const_cast<AccRec*>(dp.inc);
+        p->d_spans = const_cast<DSpan*>(dp.ds);
+        p->n_ds = dp.n_ds;
+        dev_h2d = dp.h2d_bytes;
+    } else {
+        build_span_tables(hp, p->max_blocks, st);
+    }
     pinned_vector<DSpan>& ds = st.ds;
     p->wins = st.wins;
     p->need_shadow = st.need_shadow;
@@ -409,7 +460,7 @@ static int plan_device_setup(cusan_plan* p) {
     p->o_merge = o_merge;
     p->ds = std::move(ds);
     p->table_bytes = hp.inc.size() * sizeof(AccRec) + hp.segvc.size() * sizeof(uint32_t) +
-                     p->ds.size() * sizeof(DSpan);
+                     p->ds.size() * sizeof(DSpan) + dev_h2d;
     hp.ctr.shadow_bytes = p->need_shadow ? hp.shadow_cells * sizeof(uint2) : 0;
     hp.ctr.workspace_bytes = p->ws_bytes;
     tick("layout");
@@ -430,9 +481,11 @@ static int plan_bind(cusan_plan* p, char* ws, uint64_t bytes) {
     const HostPlan& hp = p->hp;
     CK(cudaSetDevice(p->device));
     p->ws = ws;
-    p->d_inc = (AccRec*)(p->ws + p->o_inc);
+    if (!p->dev_planned) {
+        p->d_inc = (AccRec*)(p->ws + p->o_inc);
+        p->d_spans = (DSpan*)(p->ws + p->o_spans);
+    }
     p->d_segvc = (uint32_t*)(p->ws + p->o_seg);
-    p->d_spans = (DSpan*)(p->ws + p->o_spans);
     p->d_counters = (unsigned long long*)(p->ws + p->o_cnt);
     p->d_shadow = p->need_shadow ? (uint2*)(p->ws + p->o_shadow) : nullptr;
     if (!p->d_runs_own) p->d_runs = (cusan_race_run*)(p->ws + p->o_runs);
@@ -442,9 +495,11 @@ static int plan_bind(cusan_plan* p, char* ws, uint64_t bytes) {
     }
     if (!p->d_heap_own) p->d_heap = (uint32_t*)(p->ws + p->o_heap);
     else p->d_heap = p->d_heap_own;
-    CK(cudaMemcpyAsync(p->d_inc, hp.inc.data(), hp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, p->stream));
+    if (!p->dev_planned) {
+        CK(cudaMemcpyAsync(p->d_inc, hp.inc.data(), hp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, p->stream));
+        CK(cudaMemcpyAsync(p->d_spans, p->ds.data(), p->ds.size() * sizeof(DSpan), cudaMemcpyHostToDevice, p->stream));
+    }
     CK(cudaMemcpyAsync(p->d_segvc, hp.segvc.data(), hp.segvc.size() * sizeof(uint32_t), cudaMemcpyHostToDevice, p->stream));
-    CK(cudaMemcpyAsync(p->d_spans, p->ds.data(), p->ds.size() * sizeof(DSpan), cudaMemcpyHostToDevice, p->stream));
     // no wait: the kernels follow on the same stream, and the page-locked tables live until the
     // plan is destroyed (which synchronises the stream)
     p->bound = true;
@@ -489,9 +544,13 @@ int cusan_plan_create(const cusan_trace* t, const cusan_check_opts* o, cusan_pla
     cusan_plan* p = new (std::nothrow) cusan_plan;
     if (!p) return fail(CUSAN_ENOMEM, "cannot allocate plan");
     p->trace = t;
+    // a2 on the device unless asked for the host planner (or there are no accesses to plan)
+    uint64_t n_acc = 0;
+    for (const cusan_event& e : t->t.ev) n_acc += e.kind == CUSAN_EV_ACCESS;
+    p->dev_planned = !(o->flags & CUSAN_CHECK_HOST_PLAN) && n_acc > 0;
     int st;
     try {
-        st = build_host_plan(t->t, *o, p->hp);
+        st = build_host_plan(t->t, *o, p->hp, 0, 0, p->dev_planned);
     } catch (const std::bad_alloc&) {
         st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
     }
@@ -603,6 +662,21 @@ int cusan_plan_run(cusan_plan* p, cusan_report** out) {
     r->ctr.d2h_bytes = d2h;
     r->ctr.run_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count();
     *out = r;
+    return CUSAN_OK;
+}
+
+int cusan_plan_tables(const cusan_plan* p, void* inc, uint64_t inc_cap, void* spans, uint64_t spans_cap,
+                      uint64_t* n_inc, uint64_t* n_spans) {
+    if (!p || !n_inc || !n_spans) return fail(CUSAN_EINVAL, "null argument");
+    if (!p->bound) return fail(CUSAN_ESTATE, "plan has no workspace: call cusan_plan_bind_workspace");
+    CK(cudaSetDevice(p->device));
+    CK(cudaStreamSynchronize(p->stream));
+    *n_inc = p->dev_planned ? p->hp.ctr.n_incidences : p->hp.inc.size();
+    *n_spans = p->dev_planned ? p->n_ds : p->ds.size();
+    if (inc && inc_cap >= *n_inc && *n_inc)
+        CK(cudaMemcpy(inc, p->d_inc, *n_inc * sizeof(AccRec), cudaMemcpyDeviceToHost));
+    if (spans && spans_cap >= *n_spans && *n_spans)
+        CK(cudaMemcpy(spans, p->d_spans, *n_spans * sizeof(DSpan), cudaMemcpyDeviceToHost));
     return CUSAN_OK;
 }
 

@@ -58,7 +58,10 @@ class KeySlots {
 
   private:
     static constexpr uint32_t EMPTY = 0xffffffffu;
-    static size_t hash(uint64_t k) { return (size_t)((k * 0x9E3779B97F4A7C15ull) >> 20); }
+    static size_t hash(uint64_t k) {           // splitmix64 finalizer: every key bit reaches every slot bit
+        k ^= k >> 30; k *= 0xBF58476D1CE4E5B9ull; k ^= k >> 27; k *= 0x94D049BB133111EBull; k ^= k >> 31;
+        return (size_t)k;
+    }
     void grow() {
         std::vector<uint64_t> k = std::move(key_);
         std::vector<uint32_t> v = std::move(val_);
@@ -161,9 +164,10 @@ struct HostPlan {
 };
 
 // a1 + a2.  Spans (windows) are planned for the accesses from `first_access` on (0 = all);
-// pre-assigned read-set records are numbered from `rec_base`.
+// pre-assigned read-set records are numbered from `rec_base`.  a1_only: the accesses and a1 only
+// (a2 runs on the device, plan_dev.cu).
 int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uint64_t first_access = 0,
-                    uint64_t rec_base = 0);
+                    uint64_t rec_base = 0, bool a1_only = false);
 
 // canonical merge of runs (sort by (later, earlier, g_begin), merge abutting) — a4 host part
 void canonicalize_runs(std::vector<cusan_race_run>& runs);

@@ -117,6 +117,12 @@ struct Window {
     uint32_t grid;
 };
 
+// A window as the device planner describes it (plan_dev.cu; downloaded for the launches).
+struct WinDesc {
+    uint64_t span_off, tiles, weight;
+    uint32_t nspans, pad;
+};
+
 
 // ---- launch wrappers (kernel.cu) ----------------------------------------------------------------
 // K1: one window of the shadow check

@@ -161,8 +161,107 @@ static void radix_sort_pairs(std::vector<uint64_t>& key, std::vector<uint32_t>& 
     }
 }
 
+// a1.  Two passes.
+//  (1) Serial, cheap: which events open a segment (the first access of a fiber after an ACQUIRE or
+//      an incoming FORK), the segment id and epoch of every access (acc_rec), the sync-clock slot of
+//      every sync event, the Table I counters.
+//  (2) The vector clocks.  Column g of every clock (C_f[g] for all fibers f, SC_k[g] for all keys k)
+//      evolves independently of the other columns — each primitive is an element-wise max, copy or
+//      tick — so the columns are split among threads, each replaying the whole trace on its columns
+//      and writing them into the segment rows.  Same rows as one pass over whole clocks.
+std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned threads) {
+    const uint32_t F = hp.F;
+    const uint64_t n = t.ev.size();
+    cusan_counters& c = hp.ctr;
+    constexpr uint32_t NO_SEG = 0xffffffffu, NO_SLOT = 0xffffffffu;
+    std::vector<uint32_t> aux(n);          // per event: key slot (sync) or segment opened (access) or NO_SEG
+    std::vector<uint32_t> cur_seg(F, NO_SEG);
+    KeySlots key_slot;
+    hp.nseg = 0;
+    uint64_t k = 0;
+    for (uint64_t i = 0; i < n; i++) {
+        const cusan_event& e = t.ev[i];
+        const uint32_t f = e.fiber;
+        switch (e.kind) {
+            case CUSAN_EV_FORK:                    // an event of src's program order; opens a segment on dst
+                cur_seg[f] = NO_SEG;
+                aux[i] = NO_SLOT;
+                c.n_fork++;
+                break;
+            case CUSAN_EV_ACCESS: {
+                aux[i] = NO_SEG;
+                if (cur_seg[f] == NO_SEG) {
+                    if (hp.nseg >= 0x7fffffffu) return {CUSAN_ERANGE, "too many segments"};
+                    cur_seg[f] = (uint32_t)hp.nseg++;
+                    aux[i] = cur_seg[f];
+                }
+                hp.acc_rec[k] = {pack_epoch(f, (uint32_t)i), cur_seg[f] | ((uint32_t)e.mode << 31)};
+                const uint64_t bytes = 8 * (hp.acc_g1[k] - hp.acc_g0[k]);
+                k++;
+                c.n_access++;
+                c.tracked_bytes += bytes;
+                if (e.mode) { c.n_write++; c.bytes_written += bytes; }
+                else { c.n_read++; c.bytes_read += bytes; }
+                break;
+            }
+            case CUSAN_EV_RELEASE:
+            case CUSAN_EV_RELEASE_STORE:
+            case CUSAN_EV_ACQUIRE: {
+                bool fresh;
+                aux[i] = key_slot.get(e.a, &fresh);
+                if (e.kind == CUSAN_EV_ACQUIRE) { cur_seg[f] = NO_SEG; c.n_acquire++; }
+                else if (e.kind == CUSAN_EV_RELEASE) c.n_release++;
+                else c.n_release_store++;
+                break;
+            }
+            default:
+                return {CUSAN_EINVAL, "bad event kind in trace"};
+        }
+    }
+    c.n_segments = hp.nseg;
+    hp.segvc.resize(hp.nseg * F);
+    const uint32_t nkeys = key_slot.size();
+    // columns per thread: multiples of 8, at least 8 (one AVX2 vector of u32)
+    const unsigned T = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>({threads, (F + 7) / 8, n / 4096 + 1}));
+    parallel_for(T, [&](unsigned th) {
+        const uint32_t c0 = (uint32_t)((uint64_t)((F + 7) / 8) * th / T) * 8;
+        const uint32_t c1 = std::min<uint32_t>(F, (uint32_t)((uint64_t)((F + 7) / 8) * (th + 1) / T) * 8);
+        if (c0 >= c1) return;
+        const uint32_t G = c1 - c0;
+        std::vector<uint32_t> C((size_t)F * G, 0), S((size_t)nkeys * G, 0);
+        uint32_t* segvc = hp.segvc.data();
+        for (uint64_t i = 0; i < n; i++) {
+            const cusan_event& e = t.ev[i];
+            const uint32_t f = e.fiber;
+            uint32_t* __restrict__ Cf = &C[(size_t)f * G];
+            if (e.kind == CUSAN_EV_FORK) {         // C_src[src] := i+1; C_dst := C_dst ⊔ C_src
+                const uint32_t src = (uint32_t)e.a;
+                uint32_t* __restrict__ Cs = &C[(size_t)src * G];
+                if (src >= c0 && src < c1) Cs[src - c0] = (uint32_t)(i + 1);
+                if (src != f)
+                    for (uint32_t g = 0; g < G; g++) Cf[g] = std::max(Cf[g], Cs[g]);
+                continue;
+            }
+            if (f >= c0 && f < c1) Cf[f - c0] = (uint32_t)(i + 1);
+            if (e.kind == CUSAN_EV_ACCESS) {
+                if (aux[i] != NO_SEG) std::copy(Cf, Cf + G, segvc + (size_t)aux[i] * F + c0);
+                continue;
+            }
+            uint32_t* __restrict__ Sk = &S[(size_t)aux[i] * G];
+            if (e.kind == CUSAN_EV_RELEASE)        // SC_k := SC_k ⊔ C_f
+                for (uint32_t g = 0; g < G; g++) Sk[g] = std::max(Sk[g], Cf[g]);
+            else if (e.kind == CUSAN_EV_RELEASE_STORE)   // SC_k := C_f
+                std::copy(Cf, Cf + G, Sk);
+            else                                   // C_f := C_f ⊔ SC_k
+                for (uint32_t g = 0; g < G; g++) Cf[g] = std::max(Cf[g], Sk[g]);
+        }
+    });
+    return {CUSAN_OK, ""};
+}
+
 int check_flags(const cusan_check_opts& o) {
-    const int known = CUSAN_CHECK_DEFER_WORKSPACE | CUSAN_CHECK_INTERVAL_SHADOW | CUSAN_CHECK_DENSE_SHADOW;
+    const int known = CUSAN_CHECK_DEFER_WORKSPACE | CUSAN_CHECK_INTERVAL_SHADOW | CUSAN_CHECK_DENSE_SHADOW |
+                      CUSAN_CHECK_HOST_PLAN;
     if (o.flags & ~known) return fail(CUSAN_EINVAL, "unknown cusan_check_opts.flags bits");
     if ((o.flags & CUSAN_CHECK_INTERVAL_SHADOW) && (o.flags & CUSAN_CHECK_DENSE_SHADOW))
         return fail(CUSAN_EINVAL, "CUSAN_CHECK_INTERVAL_SHADOW and CUSAN_CHECK_DENSE_SHADOW exclude each other");
@@ -170,7 +269,7 @@ int check_flags(const cusan_check_opts& o) {
 }
 
 int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uint64_t first_access,
-                    uint64_t rec_base) {
+                    uint64_t rec_base, bool a1_only) {
     if (o.nshards < 1 || o.shard < 0 || o.shard >= o.nshards)
         return fail(CUSAN_EINVAL, "need 0 <= shard < nshards");
     if (o.window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
@@ -214,77 +313,22 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
     // ---------------------------------------------------------------- a1: clocks and segments --
     // Runs on its own thread while a2 builds the intervals (a2 needs a1's records only to fill the
     // incidence table at the end).  Errors come back as (status, message).
+    const unsigned a1_threads = plan_threads((uint64_t)t.ev.size() * F / 64);
     auto a1 = [&]() -> std::pair<int, std::string> {
-        std::vector<uint32_t> C((size_t)F * F, 0);
-        KeySlots key_slot;
-        std::vector<uint32_t> sc;                   // sync clocks, F entries per key
-        const uint32_t NO_SEG = 0xffffffffu;
-        std::vector<uint32_t> cur_seg(F, NO_SEG);
-        auto sync_clock = [&](uint64_t key) -> uint32_t* {
-            bool fresh;
-            const uint32_t slot = key_slot.get(key, &fresh);
-            if (fresh) sc.resize(sc.size() + F, 0);
-            return &sc[(size_t)slot * F];
-        };
-        uint64_t k = 0;
-        for (uint64_t i = 0; i < t.ev.size(); i++) {
-            const cusan_event& e = t.ev[i];
-            const uint32_t f = e.fiber;
-            uint32_t* Cf = &C[(size_t)f * F];
-            if (e.kind == CUSAN_EV_FORK) {          // an event of the source fiber's program order
-                const uint32_t s = (uint32_t)e.a;
-                uint32_t* Cs = &C[(size_t)s * F];
-                Cs[s] = (uint32_t)(i + 1);
-                for (uint32_t g = 0; g < F; g++) Cf[g] = std::max(Cf[g], Cs[g]);
-                cur_seg[f] = NO_SEG;                // incoming edge opens a segment on dst
-                c.n_fork++;
-                continue;
-            }
-            Cf[f] = (uint32_t)(i + 1);
-            switch (e.kind) {
-                case CUSAN_EV_ACCESS: {
-                    if (cur_seg[f] == NO_SEG) {
-                        if (hp.nseg >= 0x7fffffffu) return {CUSAN_ERANGE, "too many segments"};
-                        cur_seg[f] = (uint32_t)hp.nseg++;
-                        hp.segvc.insert(hp.segvc.end(), Cf, Cf + F);
-                    }
-                    hp.acc_rec[k] = {pack_epoch(f, (uint32_t)i), cur_seg[f] | ((uint32_t)e.mode << 31)};
-                    const uint64_t bytes = 8 * (hp.acc_g1[k] - hp.acc_g0[k]);
-                    k++;
-                    c.n_access++;
-                    c.tracked_bytes += bytes;
-                    if (e.mode) { c.n_write++; c.bytes_written += bytes; }
-                    else { c.n_read++; c.bytes_read += bytes; }
-                    break;
-                }
-                case CUSAN_EV_RELEASE: {            // SC_k := SC_k ⊔ C_f
-                    uint32_t* S = sync_clock(e.a);
-                    for (uint32_t g = 0; g < F; g++) S[g] = std::max(S[g], Cf[g]);
-                    c.n_release++;
-                    break;
-                }
-                case CUSAN_EV_RELEASE_STORE: {      // SC_k := C_f
-                    uint32_t* S = sync_clock(e.a);
-                    std::copy(Cf, Cf + F, S);
-                    c.n_release_store++;
-                    break;
-                }
-                case CUSAN_EV_ACQUIRE: {            // C_f := C_f ⊔ SC_k
-                    uint32_t* S = sync_clock(e.a);
-                    for (uint32_t g = 0; g < F; g++) Cf[g] = std::max(Cf[g], S[g]);
-                    cur_seg[f] = NO_SEG;
-                    c.n_acquire++;
-                    break;
-                }
-                default:
-                    return {CUSAN_EINVAL, "bad event kind in trace"};
-            }
-        }
-        c.n_segments = hp.nseg;
+        const auto a1_t0 = std::chrono::steady_clock::now();
+        std::pair<int, std::string> st = run_a1(t, hp, a1_threads);
         tick("a1 (thread)");
-        return {CUSAN_OK, ""};
+        if (dbg)
+            std::fprintf(stderr, "build_host_plan: a1 alone     %8.3f ms (%llu segments, %u threads)\n",
+                         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - a1_t0).count(),
+                         (unsigned long long)hp.nseg, a1_threads);
+        return st;
     };
     tick("acc scan");
+    if (a1_only) {                     // a2 runs on the device (plan_dev.cu)
+        const std::pair<int, std::string> st = a1();
+        return st.first ? fail(st.first, st.second) : CUSAN_OK;
+    }
     const bool concurrent = n_acc >= (1u << 12);
     std::future<std::pair<int, std::string>> a1_done;
     std::pair<int, std::string> a1_status{CUSAN_OK, ""};

@@ -1,0 +1,110 @@
+"""Step a2 on the device (plan_dev.cu): the interval, incidence and span tables the GPU builds are
+byte-identical to the host planner's (CUSAN_CHECK_HOST_PLAN, build_host_plan + build_span_tables),
+for one and many windows, both shadow layouts, granule-range shards and persisted shadows; the
+reports agree with each other and with the oracle."""
+from __future__ import annotations
+
+import numpy as np
+import pytest
+
+import oracle
+import paper_conf_sc_huckzsjb24_b200 as cs
+from tracegen import configs, fuzz
+
+pytestmark = pytest.mark.gpu
+
+HOST = cs.CUSAN_CHECK_HOST_PLAN
+COUNTERS = ["n_intervals", "n_incidences", "n_spans", "n_windows", "shard_granules", "tracked_bytes",
+            "tracked_bytes_shard", "spill_spans", "spill_heap_bytes", "shadow_bytes", "n_segments", "n_access",
+            "shadow_cell_bytes"]
+
+
+def _tables(tr, **kw):
+    p = cs.Plan(tr, **kw)
+    inc, spans = p.cusan_plan_tables()
+    rep = p.run()
+    p.close()
+    return inc, spans, rep
+
+
+def assert_same_plan(tr, **kw):
+    di, ds, dr = _tables(tr, **kw)
+    hi, hs, hr = _tables(tr, **dict(kw, flags=kw.get("flags", 0) | HOST))
+    assert di.tobytes() == hi.tobytes(), "incidence tables differ"
+    assert len(ds) == len(hs) and ds.tobytes() == hs.tobytes(), "span tables differ"
+    for k in COUNTERS:
+        assert dr.counters[k] == hr.counters[k], k
+    assert dr.n_race_granules == hr.n_race_granules and np.array_equal(dr.runs, hr.runs)
+    return dr
+
+
+@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_DENSE_SHADOW], ids=["compressed", "dense"])
+@pytest.mark.parametrize("window", [0, 1, 3, 17])
+def test_device_tables_equal_host_tables_fuzz(window, flags):
+    rng = np.random.default_rng(1200 + window + flags)
+    for i in range(30):
+        nf = int(rng.integers(2, 12))
+        ev = fuzz.random_primitive_trace(rng, int(rng.integers(1, 150)), nf, n_keys=3,
+                                         n_granules=int(rng.integers(1, 3000)), unaligned=bool(i % 3 == 0),
+                                         p_access=float(rng.uniform(0.3, 0.9)))
+        acc = ev["kind"] == 0
+        ev["mode"][acc & (rng.random(len(ev)) < 0.5)] = 0          # many readers: read-set records
+        tr = cs.Trace(nf)
+        tr.cusan_trace_append_events(ev)
+        kw = dict(window_events=window, flags=flags, persist_shadow=bool(i % 4 == 1))
+        rep = assert_same_plan(tr, **kw)
+        ref = oracle.check_events(ev, nf, threads=2)
+        assert rep.n_race_granules == ref["n_race_granules"]
+        assert np.array_equal(rep.runs, ref["runs"].astype(rep.runs.dtype))
+        for nshards in (2, 5):
+            for s in range(nshards):
+                assert_same_plan(tr, nshards=nshards, shard=s, **kw)
+
+
+@pytest.mark.parametrize("c", [1, 2, 3, 4, 5])
+def test_device_tables_equal_host_tables_configs(c):
+    w = configs.make(c, "small")
+    ops, args = w.arrays(True)
+    tr = cs.Trace(255)
+    cs.Lowering(tr).cusan_lower_program(ops, args)
+    for flags in (0, cs.CUSAN_CHECK_DENSE_SHADOW):
+        for window in (0, 97):
+            assert_same_plan(tr, window_events=window, flags=flags)
+        for s in range(3):
+            assert_same_plan(tr, window_events=97, flags=flags, nshards=3, shard=s)
+
+
+@pytest.mark.parametrize("c", [3, 5])
+def test_device_tables_equal_host_tables_full_size(c):
+    """BASELINE.json sizes in the bench launch configuration (4096-access windows), both layouts,
+    and one of 8 shards."""
+    import torch
+    torch.cuda.empty_cache()                 # earlier tests' 64 GiB torch workspaces
+    cs.release_cached_memory()
+    w = configs.make(c, "full")
+    ops, args = w.arrays(True)
+    tr = cs.Trace(255)
+    cs.Lowering(tr).cusan_lower_program(ops, args)
+    for flags in (0, cs.CUSAN_CHECK_DENSE_SHADOW):
+        assert_same_plan(tr, window_events=4096, flags=flags)
+    assert_same_plan(tr, window_events=4096, nshards=8, shard=5, flags=cs.CUSAN_CHECK_DENSE_SHADOW)
+
+
+def test_device_plan_edge_cases():
+    # no accesses / only empty accesses / one access
+    t = cs.Trace(4)
+    t.cusan_trace_append_sync(cs.CUSAN_RELEASE, 0, 5)
+    assert_same_plan(t)
+    t = cs.Trace(4)
+    t.cusan_trace_append_access(0, 1, 0x1000, 0)
+    t.cusan_trace_append_access(1, 1, 0x1000, 0)
+    assert_same_plan(t, window_events=1)
+    t = cs.Trace(4)
+    t.cusan_trace_append_access(0, 1, 0x1000, 64)
+    assert_same_plan(t, window_events=1)
+    # more shards than intervals: empty shards
+    t = cs.Trace(4)
+    t.cusan_trace_append_access(0, 1, 0x1000, 64)
+    t.cusan_trace_append_access(1, 0, 0x1000, 64)
+    for s in range(6):
+        assert_same_plan(t, nshards=6, shard=s, window_events=1)
