@@ -239,7 +239,7 @@ def run_ours(args):
     import torch.distributed as dist
 
     import paper_conf_sc_huckzsjb24_b200 as cs
-    from paper_conf_sc_huckzsjb24_b200.dist import ShardedPlan, broadcast_trace, gather_runs
+    from paper_conf_sc_huckzsjb24_b200.dist import ShardedPlan, broadcast_clocks, gather_runs
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -254,6 +254,10 @@ def run_ours(args):
     comm_dev = dev
     if world > 1:
         if args.dist_backend == "nccl":
+            # communicator lines (rank r of N) for the logs, on stderr so stdout stays one JSON line
+            os.environ.setdefault("NCCL_DEBUG", "INFO")
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
+            os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
             dist.init_process_group("nccl", device_id=dev)
         else:
             dist.init_process_group("gloo")
@@ -261,11 +265,14 @@ def run_ours(args):
     stream = torch.cuda.current_stream(dev)
 
     w, ops, args_, wname = workload(args)
+    tr = vc = None
     if world == 1 or rank == 0:
         tr = cs.Trace(255)
         cs.Lowering(tr).cusan_lower_program(ops, args_)
-    if world > 1:      # rank 0 recorded the program; the other ranks receive its events
-        tr = broadcast_trace(tr if rank == 0 else None, device=comm_dev)
+    if world > 1:      # rank 0 recorded the program: it computes the event clocks once (a1) and
+        #                broadcasts them; every rank plans its own shard from them on its GPU
+        vc = broadcast_clocks(cs.Clocks.compute(tr) if rank == 0 else None, device=comm_dev)
+        print(f"cusan bench: rank {rank} of {world} ({args.dist_backend}), device {local}", file=sys.stderr)
 
     def barrier():
         if world > 1:
@@ -282,7 +289,7 @@ def run_ours(args):
     DENSE = cs.CUSAN_CHECK_DENSE_SHADOW
     kw = dict(window_events=args.window, device=local, stream=stream.cuda_stream, workspace="torch", flags=DENSE)
     if world > 1:
-        plan = ShardedPlan(tr, comm_device=comm_dev, **kw)
+        plan = ShardedPlan(clocks=vc, comm_device=comm_dev, **kw)
         run = plan.run
     else:
         plan = cs.Plan(tr, **kw)
@@ -403,8 +410,44 @@ def run_ours(args):
         med = {k: statistics.median(v) for k, v in ph.items()}
         return tracked / (med["total_ms"] / 1e3) / 1e9, med
 
-    e2e_value, e2e_step_s, n_e2e, h2d, d2h, e2e_kms = e2e_pipelined(DENSE, elapsed_s / args.steps)
-    e2e_serial, dense_breakdown = e2e_serial_and_breakdown(DENSE)
+    def e2e_sharded(flags, reps):
+        """N ranks, every step: rank 0 lowers the program (a0) and computes the clocks (a1), broadcasts
+        them; every rank plans its shard on its GPU (a2), checks it (a3, a4), the runs are gathered
+        and stitched on rank 0 (a5).  Per-phase times are the max over ranks (medians of steps)."""
+        ph = {"lower_ms": [], "clocks_ms": [], "broadcast_ms": [], "plan_ms": [], "check_ms": [],
+              "gather_merge_ms": [], "total_ms": []}
+        h2d = d2h = 0
+        for _ in range(reps):
+            barrier()
+            torch.cuda.synchronize(dev)
+            t0 = time.perf_counter()
+            t2 = make_trace(0) if rank == 0 else None
+            t1 = time.perf_counter()
+            p2 = ShardedPlan(t2, clocks_src=0, comm_device=comm_dev, **dict(kw, flags=flags))
+            t3 = time.perf_counter()
+            shard = p2.plan.run()
+            torch.cuda.synchronize(dev)
+            t4 = time.perf_counter()
+            out = gather_runs(shard.runs, shard.n_race_granules, comm_dev)
+            r2 = cs.report_merge(*out) if out is not None else None
+            t5 = time.perf_counter()
+            p2.close()
+            for k, v in (("lower_ms", t1 - t0), ("clocks_ms", p2.timings["clocks_ms"] / 1e3),
+                         ("broadcast_ms", p2.timings["broadcast_ms"] / 1e3), ("plan_ms", p2.timings["plan_ms"] / 1e3),
+                         ("check_ms", t4 - t3), ("gather_merge_ms", t5 - t4), ("total_ms", t5 - t0)):
+                ph[k].append(max_over_ranks(v) * 1e3)
+            h2d, d2h = int(shard.counters["h2d_bytes"]), int(shard.counters["d2h_bytes"])
+            if rank == 0:
+                assert r2.n_race_granules == final.n_race_granules and np.array_equal(r2.runs, final.runs)
+        med = {k: statistics.median(v) for k, v in ph.items()}
+        return tracked / (med["total_ms"] / 1e3) / 1e9, med, h2d, d2h
+
+    if world == 1:
+        e2e_value, e2e_step_s, n_e2e, h2d, d2h, e2e_kms = e2e_pipelined(DENSE, elapsed_s / args.steps)
+        e2e_serial, dense_breakdown = e2e_serial_and_breakdown(DENSE)
+    else:
+        e2e_value, dense_breakdown, h2d, d2h = e2e_sharded(DENSE, 3)
+        e2e_serial, e2e_step_s, n_e2e, e2e_kms = e2e_value, dense_breakdown["total_ms"] / 1e3, 3, None
 
     # ---- post-mortem variant (extra, for context): one window, no shadow traffic --------------------
     pm = None
@@ -424,7 +467,7 @@ def run_ours(args):
     # device-timed steps (tables resident, CUDA events on the plan's stream), pipelined and serial
     # end to end through the public API, and its cost breakdown
     ckw = dict(kw, flags=cs.CUSAN_CHECK_INTERVAL_SHADOW)
-    p4 = ShardedPlan(tr, comm_device=comm_dev, **ckw) if world > 1 else cs.Plan(tr, **ckw)
+    p4 = ShardedPlan(clocks=vc, comm_device=comm_dev, **ckw) if world > 1 else cs.Plan(tr, **ckw)
     for _ in range(max(3, args.warmup)):
         p4.run()
     n_ic = max(args.steps, 50)
@@ -443,8 +486,12 @@ def run_ours(args):
         assert r4.n_race_granules == final.n_race_granules and np.array_equal(r4.runs, final.runs)
     p4.close()
     del p4
-    ic_e2e, ic_e2e_s, ic_n, ic_h2d, ic_d2h, ic_e2e_kms = e2e_pipelined(cs.CUSAN_CHECK_INTERVAL_SHADOW, 0.01)
-    ic_serial, ic_breakdown = e2e_serial_and_breakdown(cs.CUSAN_CHECK_INTERVAL_SHADOW, reps=5)
+    if world == 1:
+        ic_e2e, ic_e2e_s, ic_n, ic_h2d, ic_d2h, ic_e2e_kms = e2e_pipelined(cs.CUSAN_CHECK_INTERVAL_SHADOW, 0.01)
+        ic_serial, ic_breakdown = e2e_serial_and_breakdown(cs.CUSAN_CHECK_INTERVAL_SHADOW, reps=5)
+    else:
+        ic_e2e, ic_breakdown, ic_h2d, ic_d2h = e2e_sharded(cs.CUSAN_CHECK_INTERVAL_SHADOW, 5)
+        ic_serial, ic_e2e_s, ic_n, ic_e2e_kms = ic_e2e, ic_breakdown["total_ms"] / 1e3, 5, None
     ic = {"value": tracked / ic_s / 1e9, "unit": "GB/s", "ms_per_step": ic_s * 1e3, "steps": n_ic,
           "kernel_ms_per_step": statistics.mean(ic_kms), "kernel_launches_per_step": int(ic_ctr["kernel_launches"]),
           "shadow_bytes_per_gpu": int(ic_ctr["shadow_bytes"]), "window_events": args.window,
@@ -490,8 +537,10 @@ def run_ours(args):
         "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "ms_per_step": 1e3 * e2e_step_s, "steps": n_e2e,
                 "kernel_ms_per_step": e2e_kms,
-                "mode": "pipelined_checks: lowering of step i+2 and planning of step i+1 (host threads) overlap the GPU check of step i; "
-                        "pinned host tables uploaded and the report downloaded every step; 2 warm-up steps",
+                "mode": ("pipelined_checks: lowering of step i+2 and planning of step i+1 (host threads) overlap the GPU check of step i; "
+                         "pinned host tables uploaded and the report downloaded every step; 2 warm-up steps") if world == 1 else
+                        ("sharded, serial: rank 0 lowers + computes clocks, broadcast, every rank plans its shard on its GPU, "
+                         "checks, runs gathered to rank 0 (median of 3 steps, phases max over ranks)"),
                 "serial": {"value": e2e_serial, "unit": "GB/s", "ms_per_step": dense_breakdown["total_ms"],
                            "mode": "lower + plan + upload + check per step, nothing overlapped (median of 3)"},
                 "breakdown": dense_breakdown},

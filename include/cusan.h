@@ -169,6 +169,23 @@ int cusan_plan_tables(const cusan_plan* p, void* inc, uint64_t inc_cap, void* sp
                       uint64_t* n_inc, uint64_t* n_spans);
 /* Frees the parked workspaces (all devices).  Set CUSAN_NO_WORKSPACE_CACHE=1 to never park. */
 int cusan_release_cached_memory(void);
+/* ---- a1's products as a transferable object ("event clocks broadcast") ----------
+ * cusan_clocks_compute runs a1 over the whole trace (on all of the node's cores): per access its
+ * granule range and record {epoch, segment | write << 31}, the segment clock rows (u32 × fibers) and
+ * the trace counters.  On a multi-GPU node the rank that recorded the trace computes them once,
+ * exports a flat little-endian image (cusan_clocks_bytes / _export: header, g0[n], g1[n], records[n],
+ * rows[nseg × F]), broadcasts it (NCCL over NVLink) and every rank imports it and plans its own
+ * shard on its own GPU with cusan_plan_create_from_clocks (a2 on the device) — no rank repeats a1
+ * and no rank needs the trace.  The image is validated on import (CUSAN_EINVAL if corrupt). */
+typedef struct cusan_clocks cusan_clocks;
+int cusan_clocks_compute(const cusan_trace* t, cusan_clocks** out);
+int cusan_clocks_bytes(const cusan_clocks* c, uint64_t* bytes);
+int cusan_clocks_export(const cusan_clocks* c, void* buf, uint64_t bytes);
+int cusan_clocks_import(const void* buf, uint64_t bytes, cusan_clocks** out);
+int cusan_clocks_destroy(cusan_clocks* c);
+/* As cusan_plan_create, from clocks (the clocks need not outlive the plan); CUSAN_CHECK_HOST_PLAN
+ * is rejected.  Results equal cusan_plan_create's on the trace the clocks came from. */
+int cusan_plan_create_from_clocks(const cusan_clocks* c, const cusan_check_opts* o, cusan_plan** out);
 /* Host steps a1 and a2 only (no device needed): fills the trace / plan counters the same
  * plan_create would compute (shard clip, intervals, segments, windows, spill records). */
 int cusan_plan_describe(const cusan_trace* t, const cusan_check_opts* o, cusan_counters* out);

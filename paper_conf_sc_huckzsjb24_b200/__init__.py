@@ -26,7 +26,7 @@ ARG_DTYPE = np.dtype([("ptr", "<u8"), ("mode", "<u4"), ("pad", "<u4")])
 
 CUSAN_READ, CUSAN_WRITE = 0, 1
 CUSAN_RELEASE, CUSAN_RELEASE_STORE, CUSAN_ACQUIRE, CUSAN_FORK = 0, 1, 2, 3
-__all__ = ["Trace", "Lowering", "Plan", "Report", "check", "pipelined_checks", "report_merge", "CusanError", "version",
+__all__ = ["Trace", "Lowering", "Clocks", "Plan", "Report", "check", "pipelined_checks", "report_merge", "CusanError", "version",
            "RUN_DTYPE", "EVENT_DTYPE", "release_cached_memory"]
 
 
@@ -204,13 +204,47 @@ def _default_torch_stream(kw: dict) -> None:
         kw["stream"] = torch.cuda.current_stream(kw.get("device", 0)).cuda_stream
 
 
+class Clocks:
+    """cusan_clocks: a1's products for a whole trace (accesses, records, segment clock rows), as a
+    flat image one rank computes and broadcasts so every rank plans its shard without the trace."""
+
+    def __init__(self, h: C.c_void_p):
+        self.h = h
+
+    @classmethod
+    def compute(cls, trace: Trace) -> "Clocks":
+        h = C.c_void_p()
+        _ck(lib.cusan_clocks_compute(trace.h, C.byref(h)))
+        return cls(h)
+
+    def to_bytes(self) -> np.ndarray:
+        n = C.c_uint64()
+        _ck(lib.cusan_clocks_bytes(self.h, C.byref(n)))
+        buf = np.zeros(n.value, np.uint8)
+        _ck(lib.cusan_clocks_export(self.h, _ptr(buf), n.value))
+        return buf
+
+    @classmethod
+    def from_bytes(cls, buf: np.ndarray) -> "Clocks":
+        buf = np.ascontiguousarray(buf, np.uint8)
+        h = C.c_void_p()
+        _ck(lib.cusan_clocks_import(_ptr(buf), len(buf), C.byref(h)))
+        return cls(h)
+
+    def __del__(self, _destroy=lib.cusan_clocks_destroy):
+        if getattr(self, "h", None):
+            _destroy(self.h)
+            self.h = None
+
+
 class Plan:
     """cusan_plan: host preparation (a1, a2) + device tables; run() does a3-a5 on the GPU.
 
     workspace="torch" takes the plan's device memory from PyTorch's caching allocator (a uint8
-    tensor held by the plan) instead of the library's own cudaMalloc."""
+    tensor held by the plan) instead of the library's own cudaMalloc.  `trace` may be a Clocks
+    object (cusan_plan_create_from_clocks)."""
 
-    def __init__(self, trace: Trace, workspace: str | None = None, **kw):
+    def __init__(self, trace, workspace: str | None = None, **kw):
         self.trace = trace            # must outlive the plan
         self.max_runs = kw.get("max_runs", 0)
         self.workspace = None
@@ -220,7 +254,8 @@ class Plan:
         self.device, self.stream = kw.get("device", 0), kw.get("stream")
         o = _opts(**kw)
         h = C.c_void_p()
-        _ck(lib.cusan_plan_create(trace.h, C.byref(o), C.byref(h)))
+        create = lib.cusan_plan_create_from_clocks if isinstance(trace, Clocks) else lib.cusan_plan_create
+        _ck(create(trace.h, C.byref(o), C.byref(h)))
         self.h = h
         if workspace == "torch":
             nbytes = self.workspace_bytes()

@@ -85,6 +85,12 @@ PROTOS = {
     "cusan_plan_destroy": [P],
     "cusan_release_cached_memory": [],
     "cusan_plan_tables": [P, P, u64, P, u64, pu64, pu64],
+    "cusan_clocks_compute": [P, PP],
+    "cusan_clocks_bytes": [P, pu64],
+    "cusan_clocks_export": [P, P, u64],
+    "cusan_clocks_import": [P, u64, PP],
+    "cusan_clocks_destroy": [P],
+    "cusan_plan_create_from_clocks": [P, C.POINTER(cusan_check_opts), PP],
     "cusan_plan_describe": [P, C.POINTER(cusan_check_opts), C.POINTER(cusan_counters)],
     "cusan_session_create": [P, C.POINTER(cusan_check_opts), PP],
     "cusan_session_check": [P, PP],

@@ -563,6 +563,145 @@ int cusan_plan_create(const cusan_trace* t, const cusan_check_opts* o, cusan_pla
     return CUSAN_OK;
 }
 
+// ---- a1 products as a transferable object (multi-GPU: one rank computes, all plan their shard) ----
+namespace {
+constexpr uint32_t CLOCKS_MAGIC = 0x4c435343u;   // "CSCL"
+struct ClocksHdr {
+    uint32_t magic, version, F, pad;
+    uint64_t n_acc, nseg, n_events;
+    cusan_counters ctr;
+};
+}  // namespace
+
+int cusan_clocks_compute(const cusan_trace* t, cusan_clocks** out) {
+    if (!t || !out) return fail(CUSAN_EINVAL, "null argument");
+    *out = nullptr;
+    cusan_clocks* c = new (std::nothrow) cusan_clocks;
+    if (!c) return fail(CUSAN_ENOMEM, "cannot allocate clocks");
+    int st;
+    try {
+        st = compute_clocks(t->t, c->hp);
+    } catch (const std::bad_alloc&) {
+        st = fail(CUSAN_ENOMEM, "host memory exhausted while computing clocks");
+    }
+    if (st) {
+        delete c;
+        return st;
+    }
+    *out = c;
+    return CUSAN_OK;
+}
+
+int cusan_clocks_bytes(const cusan_clocks* c, uint64_t* bytes) {
+    if (!c || !bytes) return fail(CUSAN_EINVAL, "null argument");
+    const HostPlan& hp = c->hp;
+    *bytes = sizeof(ClocksHdr) + hp.acc_g0.size() * (16 + sizeof(AccRec)) + hp.segvc.size() * 4;
+    return CUSAN_OK;
+}
+
+int cusan_clocks_export(const cusan_clocks* c, void* buf, uint64_t bytes) {
+    uint64_t need = 0;
+    if (int st = cusan_clocks_bytes(c, &need)) return st;
+    if (!buf || bytes < need) return fail(CUSAN_EINVAL, "buffer smaller than cusan_clocks_bytes");
+    const HostPlan& hp = c->hp;
+    ClocksHdr h{};
+    h.magic = CLOCKS_MAGIC;
+    h.version = 1;
+    h.F = hp.F;
+    h.n_acc = hp.acc_g0.size();
+    h.nseg = hp.nseg;
+    h.n_events = hp.ctr.n_events;
+    h.ctr = hp.ctr;
+    char* p = (char*)buf;
+    std::memcpy(p, &h, sizeof(h));
+    p += sizeof(h);
+    std::memcpy(p, hp.acc_g0.data(), h.n_acc * 8);
+    p += h.n_acc * 8;
+    std::memcpy(p, hp.acc_g1.data(), h.n_acc * 8);
+    p += h.n_acc * 8;
+    std::memcpy(p, hp.acc_rec.data(), h.n_acc * sizeof(AccRec));
+    p += h.n_acc * sizeof(AccRec);
+    std::memcpy(p, hp.segvc.data(), hp.segvc.size() * 4);
+    return CUSAN_OK;
+}
+
+int cusan_clocks_import(const void* buf, uint64_t bytes, cusan_clocks** out) {
+    if (!buf || !out) return fail(CUSAN_EINVAL, "null argument");
+    *out = nullptr;
+    ClocksHdr h;
+    if (bytes < sizeof(h)) return fail(CUSAN_EINVAL, "clocks image too short");
+    std::memcpy(&h, buf, sizeof(h));
+    if (h.magic != CLOCKS_MAGIC || h.version != 1) return fail(CUSAN_EINVAL, "not a clocks image");
+    if (h.F < 1 || h.F > 256 || h.n_acc > (1ull << 40) || h.nseg > (1ull << 40))
+        return fail(CUSAN_EINVAL, "corrupt clocks image");
+    const uint64_t need = sizeof(h) + h.n_acc * (16 + sizeof(AccRec)) + h.nseg * h.F * 4;
+    if (bytes < need) return fail(CUSAN_EINVAL, "clocks image truncated");
+    cusan_clocks* c = new (std::nothrow) cusan_clocks;
+    if (!c) return fail(CUSAN_ENOMEM, "cannot allocate clocks");
+    try {
+        HostPlan& hp = c->hp;
+        hp.F = h.F;
+        hp.nseg = h.nseg;
+        hp.ctr = h.ctr;
+        const char* p = (const char*)buf + sizeof(h);
+        hp.acc_g0.resize(h.n_acc);
+        hp.acc_g1.resize(h.n_acc);
+        hp.acc_rec.resize(h.n_acc);
+        hp.segvc.resize(h.nseg * h.F);
+        std::memcpy(hp.acc_g0.data(), p, h.n_acc * 8);
+        p += h.n_acc * 8;
+        std::memcpy(hp.acc_g1.data(), p, h.n_acc * 8);
+        p += h.n_acc * 8;
+        std::memcpy(hp.acc_rec.data(), p, h.n_acc * sizeof(AccRec));
+        p += h.n_acc * sizeof(AccRec);
+        std::memcpy(hp.segvc.data(), p, hp.segvc.size() * 4);
+    } catch (const std::bad_alloc&) {
+        delete c;
+        return fail(CUSAN_ENOMEM, "host memory exhausted while importing clocks");
+    }
+    *out = c;
+    return CUSAN_OK;
+}
+
+int cusan_clocks_destroy(cusan_clocks* c) {
+    if (!c) return fail(CUSAN_EINVAL, "clocks is null");
+    delete c;
+    return CUSAN_OK;
+}
+
+int cusan_plan_create_from_clocks(const cusan_clocks* c, const cusan_check_opts* o, cusan_plan** out) {
+    if (!c || !o || !out) return fail(CUSAN_EINVAL, "null argument");
+    *out = nullptr;
+    if (o->nshards < 1 || o->shard < 0 || o->shard >= o->nshards) return fail(CUSAN_EINVAL, "need 0 <= shard < nshards");
+    if (o->window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
+    if (int st = check_flags(*o)) return st;
+    if (o->flags & CUSAN_CHECK_HOST_PLAN) return fail(CUSAN_EINVAL, "plans from clocks build their tables on the device");
+    cusan_plan* p = new (std::nothrow) cusan_plan;
+    if (!p) return fail(CUSAN_ENOMEM, "cannot allocate plan");
+    int st = CUSAN_OK;
+    try {
+        HostPlan& hp = p->hp;
+        hp.opts = *o;
+        hp.F = c->hp.F;
+        hp.nseg = c->hp.nseg;
+        hp.ctr = c->hp.ctr;
+        hp.acc_g0 = c->hp.acc_g0;
+        hp.acc_g1 = c->hp.acc_g1;
+        hp.acc_rec = c->hp.acc_rec;
+        hp.segvc = c->hp.segvc;
+        p->dev_planned = !hp.acc_g0.empty();
+    } catch (const std::bad_alloc&) {
+        st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
+    }
+    if (!st) st = plan_device_setup(p);
+    if (st) {
+        delete p;
+        return st;
+    }
+    *out = p;
+    return CUSAN_OK;
+}
+
 int cusan_plan_describe(const cusan_trace* t, const cusan_check_opts* o, cusan_counters* out) {
     if (!t || !o || !out) return fail(CUSAN_EINVAL, "null argument");
     HostPlan hp;

@@ -169,6 +169,9 @@ struct HostPlan {
 int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uint64_t first_access = 0,
                     uint64_t rec_base = 0, bool a1_only = false);
 
+// a1 of a whole trace for a clocks object (cusan_clocks_compute), with the node's cores
+int compute_clocks(const Trace& t, HostPlan& hp);
+
 // canonical merge of runs (sort by (later, earlier, g_begin), merge abutting) — a4 host part
 void canonicalize_runs(std::vector<cusan_race_run>& runs);
 
@@ -176,6 +179,11 @@ void canonicalize_runs(std::vector<cusan_race_run>& runs);
 
 struct cusan_trace {
     cusan::Trace t;
+};
+
+// a1's products for a whole trace (cusan_clocks_*): accesses, records, segment rows, counters
+struct cusan_clocks {
+    cusan::HostPlan hp;
 };
 
 struct cusan_report {

@@ -259,28 +259,8 @@ std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned thread
     return {CUSAN_OK, ""};
 }
 
-int check_flags(const cusan_check_opts& o) {
-    const int known = CUSAN_CHECK_DEFER_WORKSPACE | CUSAN_CHECK_INTERVAL_SHADOW | CUSAN_CHECK_DENSE_SHADOW |
-                      CUSAN_CHECK_HOST_PLAN;
-    if (o.flags & ~known) return fail(CUSAN_EINVAL, "unknown cusan_check_opts.flags bits");
-    if ((o.flags & CUSAN_CHECK_INTERVAL_SHADOW) && (o.flags & CUSAN_CHECK_DENSE_SHADOW))
-        return fail(CUSAN_EINVAL, "CUSAN_CHECK_INTERVAL_SHADOW and CUSAN_CHECK_DENSE_SHADOW exclude each other");
-    return CUSAN_OK;
-}
-
-int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uint64_t first_access,
-                    uint64_t rec_base, bool a1_only) {
-    if (o.nshards < 1 || o.shard < 0 || o.shard >= o.nshards)
-        return fail(CUSAN_EINVAL, "need 0 <= shard < nshards");
-    if (o.window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
-    if (int st = check_flags(o)) return st;
-    hp.opts = o;
-    const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
-    auto tick = [t0 = std::chrono::steady_clock::now(), dbg](const char* what) {
-        if (dbg)
-            std::fprintf(stderr, "build_host_plan: %-12s %8.3f ms\n", what,
-                         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
-    };
+// The accesses of a trace (granule ranges, event ids) and the clock width; resets the counters.
+static void prepare_accesses(const Trace& t, HostPlan& hp) {
     // clock width = fibers the trace actually uses (≤ max_fibers); the accesses' granule ranges
     uint32_t F = 1;
     uint64_t n_acc = 0;
@@ -309,7 +289,50 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
             k++;
         }
     }
+}
 
+// a1 alone for a clocks object (cusan_clocks_compute): every core of the node — on a multi-GPU
+// node one rank computes the clocks while the others wait for the broadcast.
+int compute_clocks(const Trace& t, HostPlan& hp) {
+    prepare_accesses(t, hp);
+    unsigned hw = std::max(1u, std::thread::hardware_concurrency());
+    cpu_set_t set;
+    if (sched_getaffinity(0, sizeof(set), &set) == 0) hw = std::max(1, CPU_COUNT(&set));
+    if (const char* e = std::getenv("CUSAN_PLAN_THREADS")) {
+        const long v = std::strtol(e, nullptr, 10);
+        if (v > 0) hw = (unsigned)std::min<long>(v, 256) + 1;
+    }
+    const unsigned T = (uint64_t)t.ev.size() * hp.F < (1u << 21) ? 1 : std::max(1u, std::min(hw > 1 ? hw - 1 : 1, 32u));
+    const std::pair<int, std::string> st = run_a1(t, hp, T);
+    return st.first ? fail(st.first, st.second) : CUSAN_OK;
+}
+
+int check_flags(const cusan_check_opts& o) {
+    const int known = CUSAN_CHECK_DEFER_WORKSPACE | CUSAN_CHECK_INTERVAL_SHADOW | CUSAN_CHECK_DENSE_SHADOW |
+                      CUSAN_CHECK_HOST_PLAN;
+    if (o.flags & ~known) return fail(CUSAN_EINVAL, "unknown cusan_check_opts.flags bits");
+    if ((o.flags & CUSAN_CHECK_INTERVAL_SHADOW) && (o.flags & CUSAN_CHECK_DENSE_SHADOW))
+        return fail(CUSAN_EINVAL, "CUSAN_CHECK_INTERVAL_SHADOW and CUSAN_CHECK_DENSE_SHADOW exclude each other");
+    return CUSAN_OK;
+}
+
+int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uint64_t first_access,
+                    uint64_t rec_base, bool a1_only) {
+    if (o.nshards < 1 || o.shard < 0 || o.shard >= o.nshards)
+        return fail(CUSAN_EINVAL, "need 0 <= shard < nshards");
+    if (o.window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
+    if (int st = check_flags(o)) return st;
+    hp.opts = o;
+    const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
+    auto tick = [t0 = std::chrono::steady_clock::now(), dbg](const char* what) {
+        if (dbg)
+            std::fprintf(stderr, "build_host_plan: %-12s %8.3f ms\n", what,
+                         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+    };
+    prepare_accesses(t, hp);
+    const uint32_t F = hp.F;
+    const uint64_t n_acc = hp.acc_g0.size();
+    cusan_counters& c = hp.ctr;
     // ---------------------------------------------------------------- a1: clocks and segments --
     // Runs on its own thread while a2 builds the intervals (a2 needs a1's records only to fill the
     // incidence table at the end).  Errors come back as (status, message).

@@ -24,6 +24,7 @@
 #include <cub/cub.cuh>
 
 #include <algorithm>
+#include <chrono>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -601,6 +602,13 @@ static int grow(char** p, uint64_t* cap, uint64_t need) {
 int device_plan_a2(const HostPlan& hp, const DevPlanArgs& A, DevScratch& S, DevPlanOut& out) {
     cudaStream_t st = S.stream;
     const uint64_t n = hp.acc_g0.size();
+    static const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
+    const auto t0 = std::chrono::steady_clock::now();
+    auto tick = [&](const char* what) {
+        if (dbg)
+            std::fprintf(stderr, "device_plan_a2: %-14s %8.3f ms\n", what,
+                         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+    };
     out = DevPlanOut{};
     const cusan_check_opts& o = hp.opts;
     const bool compressed = compressed_shadow(o);
@@ -695,6 +703,7 @@ int device_plan_a2(const HostPlan& hp, const DevPlanArgs& A, DevScratch& S, DevP
     CK(cudaGetLastError());
     CK(cudaMemcpyAsync(hh, P1.hdr, H_COUNT * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));                             // sync 1: sizes of the pair / span buffers
+    tick("sync 1");
     out.launches += 8;
     const uint64_t niv = hh[H_NIV], npairs = hh[H_NPAIRS], total_dense = hh[H_DENSE];
     out.n_intervals = niv;
@@ -831,6 +840,7 @@ int device_plan_a2(const HostPlan& hp, const DevPlanArgs& A, DevScratch& S, DevP
     CK(cudaGetLastError());
     CK(cudaMemcpyAsync(hh, P1.hdr, H_COUNT * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));                             // sync 2: kept intervals and spans
+    tick("sync 2");
     out.launches += 14;
     const uint64_t nk = hh[H_NKEPT], ns = hh[H_NSPANS];
     out.n_inc = hh[H_NINC];
@@ -878,6 +888,7 @@ int device_plan_a2(const HostPlan& hp, const DevPlanArgs& A, DevScratch& S, DevP
     S.wins_host.resize(nwin_all);
     CK(cudaMemcpyAsync(S.wins_host.data(), PO.wd, nwin_all * sizeof(WinDesc), cudaMemcpyDeviceToHost, st));
     CK(cudaStreamSynchronize(st));                             // sync 3: window descriptors for the launches
+    tick("sync 3");
     out.launches += 20;
     const uint64_t nw = hh[H_NWIN];
     out.wins.assign(S.wins_host.begin(), S.wins_host.begin() + nw);

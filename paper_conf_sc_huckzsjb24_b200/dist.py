@@ -1,11 +1,13 @@
 """Multi-GPU check: the shadow space is sharded by granule range, one shard per rank.
 
-Granules are independent, so every rank builds the same host plan from the same trace (each rank
-holds the trace, or the rank that recorded it broadcasts its events: broadcast_trace), checks only
-its shard on its own GPU
-with no communication inside the check, and the race runs are gathered to rank 0 — the one real
-exchange step — with torch.distributed (NCCL over NVLink on GPUs, gloo in CPU tests).  Rank 0
-stitches runs that abut across shard boundaries and sorts them canonically (cusan_report_merge).
+Granules are independent.  The rank that recorded the trace computes the event clocks once (a1,
+cusan_clocks_compute, on all of the node's cores) and broadcasts them (broadcast_clocks: one flat
+image — access ranges, records, segment clock rows — NCCL over NVLink); every rank then builds the
+tables of its own shard on its own GPU (a2 on the device, cusan_plan_create_from_clocks), checks
+it with no communication inside the check, and the race runs are gathered to rank 0 — the one real
+exchange step — with torch.distributed (NCCL on GPUs, gloo in CPU tests).  Rank 0 stitches runs
+that abut across shard boundaries and sorts them canonically (cusan_report_merge).  Sessions (f1)
+broadcast the raw events instead (broadcast_trace): their planning is incremental per call.
 """
 from __future__ import annotations
 
@@ -13,7 +15,7 @@ import numpy as np
 import torch
 import torch.distributed as dist
 
-from . import RUN_DTYPE, Plan, Report, Session, Trace, report_merge
+from . import RUN_DTYPE, Clocks, Plan, Report, Session, Trace, report_merge
 
 _RUN_U64 = RUN_DTYPE.itemsize // 8          # a run record as three u64 words
 
@@ -72,24 +74,60 @@ def broadcast_trace(trace: Trace | None, src: int = 0, device: torch.device | No
     return out
 
 
+def broadcast_clocks(clocks: Clocks | None, src: int = 0, device: torch.device | None = None,
+                     group=None) -> Clocks:
+    """Rank ``src`` holds the clocks (a1 of the whole trace); every rank returns them: one broadcast
+    of the image size, one of the image (NCCL over NVLink on GPUs)."""
+    dev = device if device is not None else torch.device("cpu")
+    me = dist.get_rank(group)
+    root = dist.get_global_rank(group, src) if group is not None else src
+    img = clocks.to_bytes() if me == src else None
+    meta = torch.tensor([len(img) if me == src else 0], dtype=torch.int64, device=dev)
+    dist.broadcast(meta, root, group=group)
+    n = int(meta[0])
+    buf = torch.from_numpy(img).to(dev) if me == src else torch.empty(n, dtype=torch.uint8, device=dev)
+    dist.broadcast(buf, root, group=group)
+    return clocks if me == src else Clocks.from_bytes(buf.cpu().numpy())
+
+
 class ShardedPlan:
     """One rank's shard of a multi-GPU check.  run() checks the shard on this rank's GPU, gathers
-    the runs and returns the canonical whole-trace Report on rank 0 (None elsewhere)."""
+    the runs and returns the canonical whole-trace Report on rank 0 (None elsewhere).
 
-    def __init__(self, trace: Trace, device: int = 0, group=None, comm_device: torch.device | None = None,
-                 **kw):
+    ``trace``: a Trace every rank holds (each rank computes the clocks itself), or — with
+    ``clocks_src`` set — the recording rank's Trace (None elsewhere): that rank computes the clocks
+    and broadcasts them, the others need no trace.  ``clocks``: clocks every rank already holds."""
+
+    def __init__(self, trace: Trace | None = None, device: int = 0, group=None,
+                 comm_device: torch.device | None = None, clocks: Clocks | None = None,
+                 clocks_src: int | None = None, **kw):
+        import time
         self.group = group
         self.rank = dist.get_rank(group)
         self.world = dist.get_world_size(group)
         self.comm_device = comm_device
         self.max_runs = kw.pop("max_runs", 0)
-        self.plan = Plan(trace, nshards=self.world, shard=self.rank, device=device, **kw)
+        self.timings = {}
+        t0 = time.perf_counter()
+        if clocks is None and clocks_src is not None:
+            mine = Clocks.compute(trace) if self.rank == clocks_src else None
+            t1 = time.perf_counter()
+            clocks = broadcast_clocks(mine, clocks_src, comm_device, group)
+            self.timings["clocks_ms"] = 1e3 * (t1 - t0)
+            self.timings["broadcast_ms"] = 1e3 * (time.perf_counter() - t1)
+        t2 = time.perf_counter()
+        self.plan = Plan(clocks if clocks is not None else trace, nshards=self.world, shard=self.rank,
+                         device=device, **kw)
+        self.timings["plan_ms"] = 1e3 * (time.perf_counter() - t2)
         self.last_shard_report: Report | None = None
 
     def run(self) -> Report | None:
+        import time
         rep = self.plan.run()
         self.last_shard_report = rep
+        t0 = time.perf_counter()
         out = gather_runs(rep.runs, rep.n_race_granules, self.comm_device, self.group)
+        self.timings["gather_ms"] = 1e3 * (time.perf_counter() - t0)
         if out is None:
             return None
         runs, n_race = out

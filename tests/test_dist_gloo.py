@@ -175,3 +175,61 @@ def test_two_rank_trace_broadcast():
         p.join(timeout=60)
         assert p.exitcode == 0
     assert all(r["same"] and r["plan_same"] and r["fibers"] == 255 for r in res), res
+
+
+def _clocks_worker(rank, world, port, q):
+    import sys
+    sys.path.insert(0, ROOT)
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import paper_conf_sc_huckzsjb24_b200 as cs
+        from paper_conf_sc_huckzsjb24_b200.dist import broadcast_clocks
+        from tracegen import configs
+        w = configs.make(5, "small")
+        ops, args = w.arrays(True)
+        mine = cs.Trace(255)                          # what every rank would have lowered itself
+        cs.Lowering(mine).cusan_lower_program(ops, args)
+        want = cs.Clocks.compute(mine).to_bytes()
+        got = broadcast_clocks(cs.Clocks.compute(mine) if rank == 0 else None)   # rank 0 computes
+        q.put(dict(rank=rank, same=bool(np.array_equal(got.to_bytes(), want)), n=len(want)))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_two_rank_clocks_broadcast():
+    """SURVEY §8(e) "event clocks broadcast": rank 0 computes a1 once and broadcasts the clocks
+    image; rank 1's clocks equal the ones it would have computed itself."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_clocks_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=240) for _ in procs]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    assert all(r["same"] and r["n"] > 1000 for r in res), res
+
+
+def test_clocks_image_round_trip_and_validation():
+    """Export → import → export is the identity; the image carries a1's counters; a corrupt or
+    truncated image is rejected (CUSAN_EINVAL), never read past its end."""
+    import paper_conf_sc_huckzsjb24_b200 as cs
+    from tracegen import configs
+    w = configs.make(3, "small")
+    ops, args = w.arrays(True)
+    tr = cs.Trace(255)
+    cs.Lowering(tr).cusan_lower_program(ops, args)
+    img = cs.Clocks.compute(tr).to_bytes()
+    assert np.array_equal(cs.Clocks.from_bytes(img).to_bytes(), img)
+    d = cs.describe(tr)
+    hdr = img[:40].view(np.uint64)                    # magic/version/F/pad, n_acc, nseg, n_events
+    assert int(hdr[2]) == d["n_access"] and int(hdr[3]) == d["n_segments"] and int(hdr[4]) == d["n_events"]
+    bad = img.copy()
+    bad[0] ^= 1
+    with pytest.raises(cs.CusanError):
+        cs.Clocks.from_bytes(bad)
+    with pytest.raises(cs.CusanError):
+        cs.Clocks.from_bytes(img[:-4])

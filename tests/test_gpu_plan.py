@@ -108,3 +108,33 @@ def test_device_plan_edge_cases():
     t.cusan_trace_append_access(1, 0, 0x1000, 64)
     for s in range(6):
         assert_same_plan(t, nshards=6, shard=s, window_events=1)
+
+
+@pytest.mark.parametrize("c", [3, 5])
+def test_plan_from_clocks_equals_plan_from_trace(c):
+    """cusan_plan_create_from_clocks (the multi-GPU path: one rank computes a1, every rank plans its
+    shard from the broadcast image) builds the same tables and report as cusan_plan_create, also
+    from an exported / imported image and per shard; reports equal the oracle's."""
+    w = configs.make(c, "small")
+    ops, args = w.arrays(True)
+    tr = cs.Trace(255)
+    cs.Lowering(tr).cusan_lower_program(ops, args)
+    ref = oracle.check_events(tr.cusan_trace_read(), 256)
+    clocks = cs.Clocks.from_bytes(cs.Clocks.compute(tr).to_bytes())
+    for kw in (dict(window_events=97), dict(window_events=97, flags=cs.CUSAN_CHECK_DENSE_SHADOW),
+               dict(window_events=0)):
+        a_inc, a_sp, a_rep = _tables(tr, **kw)
+        b_inc, b_sp, b_rep = _tables(clocks, **kw)
+        assert a_inc.tobytes() == b_inc.tobytes() and a_sp.tobytes() == b_sp.tobytes()
+        for k in COUNTERS:
+            assert a_rep.counters[k] == b_rep.counters[k], k
+        assert b_rep.n_race_granules == ref["n_race_granules"]
+        assert np.array_equal(b_rep.runs, ref["runs"].astype(b_rep.runs.dtype))
+        parts = [cs.Plan(clocks, nshards=4, shard=s, **kw) for s in range(4)]
+        reps = [p.run() for p in parts]
+        for p in parts:
+            p.close()
+        merged = cs.report_merge(np.concatenate([r.runs for r in reps]), sum(r.n_race_granules for r in reps))
+        assert np.array_equal(merged.runs, ref["runs"].astype(merged.runs.dtype))
+    with pytest.raises(cs.CusanError):
+        cs.Plan(clocks, flags=cs.CUSAN_CHECK_HOST_PLAN)
