@@ -273,3 +273,47 @@ def test_session_read_set_records_are_reclaimed(flags):
         assert rep.counters["heap_live_bytes"] <= rep.counters["heap_bytes"]
     ses.close()
     assert heap[-1] == heap[10] > 0, heap         # bounded: no growth once the layout is stable
+
+
+FULL_GOLDEN = __import__("os").path.join(__import__("os").path.dirname(__import__("os").path.abspath(__file__)),
+                                         "golden", "full")
+
+
+@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_DENSE_SHADOW], ids=["compressed", "dense"])
+@pytest.mark.parametrize("per_call", [4096, 512])
+def test_session_full_size_config5(per_call, flags):
+    """The config-5 racy trace at its full size (64 GiB tracked, 64 fibers) fed to an online
+    session in calls of `per_call` accesses (9 calls of 4096, 71 of 512): every call's report equals
+    the oracle's complete report (tests/golden/full/config5_racy.npz, every granule checked by
+    oracle.c) restricted to the races whose later access is in that call (CuSan
+    checks on the fly); the counts add up to the whole."""
+    import hashlib
+    import os
+
+    import torch
+    torch.cuda.empty_cache()
+    cs.release_cached_memory()
+    g = np.load(os.path.join(FULL_GOLDEN, "config5_racy.npz"))
+    w = configs.make(5, "full")
+    ops, args = w.arrays(True)
+    full = cs.Trace(255)
+    cs.Lowering(full).cusan_lower_program(ops, args)
+    ev = full.cusan_trace_read()
+    assert hashlib.sha256(np.ascontiguousarray(ev).tobytes()).hexdigest() == str(g["events_sha256"])
+    golden = g["runs"]
+    acc_pos = np.flatnonzero(ev["kind"] == EV_ACCESS)
+    cuts = [int(acc_pos[k]) for k in range(per_call, len(acc_pos), per_call)] + [len(ev)]
+    tr = cs.Trace(255)
+    ses = cs.Session(tr, window_events=per_call, flags=flags)
+    start, total, calls = 0, 0, 0
+    for end in cuts:
+        tr.cusan_trace_append_events(ev[start:end])
+        rep = ses.check()
+        want = _by_later(golden, start, end)
+        assert np.array_equal(rep.runs, want.astype(rep.runs.dtype)), (start, end)
+        assert rep.n_race_granules == int(np.sum(want["g_end"] - want["g_begin"]))
+        total += rep.n_race_granules
+        start, calls = end, calls + 1
+    ses.close()
+    assert calls == -(-len(acc_pos) // per_call)
+    assert total == int(g["n_race_granules"]) > 0
