@@ -32,13 +32,15 @@ extern "C" {
 
 #define CUSAN_OK 0
 #define CUSAN_EINVAL (-1)  /* null pointer, fiber >= max_fibers, bad enum, bad option            */
-#define CUSAN_ERANGE (-2)  /* > 2^24-2 events (24-bit event index), addr + nbytes overflows      */
+#define CUSAN_ERANGE (-2)  /* one-shot check of > 2^24-2 events, addr + nbytes overflows, ...    */
 #define CUSAN_ENOMEM (-3)  /* host or device allocation failed / workspace too small             */
 #define CUSAN_ECUDA (-4)   /* CUDA runtime error (includes: no device)                           */
 #define CUSAN_ESTATE (-5)  /* object used in the wrong state                                     */
 
 #define CUSAN_MAX_FIBERS 255u          /* fiber id is 8 bits in a shadow slot; 0xFF tags a spill record */
-#define CUSAN_MAX_EVENTS ((1u << 24) - 2u) /* event index + 1 is 24 bits in a shadow slot   */
+#define CUSAN_MAX_EVENTS ((1u << 24) - 2u) /* one-shot checks: event index + 1 is 24 bits in a shadow slot */
+#define CUSAN_MAX_TRACE_EVENTS 0xFFFFFFFEu /* a trace (event ids are u32 in reports); sessions renumber
+                                               their live epochs to stay inside 24 bits            */
 
 typedef struct cusan_trace cusan_trace;   /* opaque; caller owns (create / destroy)            */
 typedef struct cusan_plan cusan_plan;     /* opaque; caller owns (create / destroy)            */
@@ -245,6 +247,7 @@ typedef struct cusan_counters {
     /* sessions: read-set heap after this call — records some interval still names, and the heap's
        high-water mark (dead records are reused from the next call on, so it tracks the live set) */
     uint64_t heap_live_bytes, heap_bytes;
+    uint64_t renumberings;         /* sessions: epoch renumberings so far (traces past 2^24-2 events) */
 } cusan_counters;
 
 int cusan_report_get(const cusan_report* r, uint64_t* n_race_granules, uint64_t* n_runs,

@@ -416,7 +416,7 @@ int main(int argc, char** argv) {
     events = xmalloc(n_events * sizeof(event_t));
     if (fread(events, sizeof(event_t), n_events, fp) != n_events) die("short trace");
     fclose(fp);
-    if (n_events >= (1u << 24) - 1) die("trace too long");
+    if (n_events >= 0xFFFFFFFFull) die("trace too long (event ids are u32)");
     for (uint64_t i = 0; i < n_events; i++) {
         if (events[i].fiber + 1 > F) F = events[i].fiber + 1;
         if (events[i].kind == EV_FORK && events[i].a + 1 > F) F = (uint32_t)events[i].a + 1;

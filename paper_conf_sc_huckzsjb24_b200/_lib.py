@@ -47,7 +47,8 @@ class cusan_counters(C.Structure):
     _fields_ = ([(n, C.c_uint64) for n in _COUNTER_U64] +
                 [("kernel_ms", C.c_double), ("run_ms", C.c_double), ("kernel_launches", C.c_uint64),
                  ("shadow_cell_bytes", C.c_uint64), ("h2d_bytes", C.c_uint64),
-                 ("d2h_bytes", C.c_uint64), ("heap_live_bytes", C.c_uint64), ("heap_bytes", C.c_uint64)])
+                 ("d2h_bytes", C.c_uint64), ("heap_live_bytes", C.c_uint64), ("heap_bytes", C.c_uint64),
+                 ("renumberings", C.c_uint64)])
 
 
 class cusan_api_call(C.Structure):

@@ -527,9 +527,51 @@ copy_cells(const uint2* src, uint2* dst, const CopySeg* __restrict__ segs, uint3
 }
 
 
+// Session epoch renumbering (session.cpp): read one cell per interval, and write a renumbered cell
+// over every cell of an interval (all cells of an interval are equal).
+__global__ void __launch_bounds__(THREADS)
+gather_cells(const uint2* __restrict__ shadow, const uint64_t* __restrict__ at, uint64_t n, uint2* __restrict__ out) {
+    for (uint64_t i = (uint64_t)blockIdx.x * THREADS + threadIdx.x; i < n; i += (uint64_t)gridDim.x * THREADS)
+        out[i] = shadow[at[i]];
+}
+
+__global__ void __launch_bounds__(THREADS)
+fill_cells(uint2* __restrict__ shadow, const CellFill* __restrict__ f, uint32_t nf, uint64_t total) {
+    const int lane = threadIdx.x & 31;
+    const uint64_t nwarps = (uint64_t)gridDim.x * WARPS;
+    const uint64_t nchunks = (total + COPY_CHUNK - 1) / COPY_CHUNK;
+    for (uint64_t ch = (uint64_t)blockIdx.x * WARPS + (threadIdx.x >> 5); ch < nchunks; ch += nwarps) {
+        const uint64_t c0 = ch * COPY_CHUNK, c1 = min(c0 + COPY_CHUNK, total);
+        uint32_t lo = 0, hi = nf;                         // last fill with prefix <= c0
+        while (hi - lo > 1) {
+            const uint32_t mid = (lo + hi) >> 1;
+            if (f[mid].prefix <= c0) lo = mid; else hi = mid;
+        }
+        for (uint64_t c = c0; c < c1; lo++) {
+            const CellFill x = f[lo];
+            const uint64_t end = min(c1, x.prefix + x.len);
+            const uint2 v = make_uint2(x.w, x.r);
+            for (uint64_t i = c + lane; i < end; i += 32) __stcs(shadow + x.dst + (i - x.prefix), v);
+            c = end;
+        }
+    }
+}
+
 }  // namespace
 
 namespace cusan {
+
+cudaError_t launch_gather_cells(uint32_t grid, cudaStream_t stream, const uint2* shadow, const uint64_t* at, uint64_t n,
+                                uint2* out) {
+    gather_cells<<<grid, THREADS, 0, stream>>>(shadow, at, n, out);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_fill_cells(uint32_t grid, cudaStream_t stream, uint2* shadow, const CellFill* f, uint32_t nf,
+                              uint64_t total) {
+    fill_cells<<<grid, THREADS, 0, stream>>>(shadow, f, nf, total);
+    return cudaGetLastError();
+}
 
 cudaError_t launch_shadow_check(uint32_t grid, cudaStream_t stream, const DSpan* spans, uint32_t nspans,
                                 uint64_t tiles, uint64_t weight, const Ctx& k, unsigned long long* sched) {

@@ -98,6 +98,12 @@ struct CopySeg {
     uint64_t prefix, src, dst, len;       // cells [prefix, prefix + len) of the copy space
 };
 
+// A renumbered cell written over `len` cells from shadow index `dst` (fill space [prefix, prefix+len)).
+struct CellFill {
+    uint64_t prefix, dst, len;
+    uint32_t w, r;
+};
+
 inline int cuda_fail(cudaError_t e, const char* what) {
     return fail(CUSAN_ECUDA, std::string(what) + ": " + cudaGetErrorString(e));
 }
@@ -131,6 +137,11 @@ cudaError_t launch_shadow_check(uint32_t grid, cudaStream_t stream, const DSpan*
 // sessions: copy the cell of a split compressed interval to its new piece
 cudaError_t launch_copy_cells(uint32_t grid, cudaStream_t stream, const uint2* src, uint2* dst,
                               const CopySeg* segs, uint32_t nseg, uint64_t total);
+// sessions: epoch renumbering — one cell per interval out, renumbered cells back in
+cudaError_t launch_gather_cells(uint32_t grid, cudaStream_t stream, const uint2* shadow, const uint64_t* at, uint64_t n,
+                                uint2* out);
+cudaError_t launch_fill_cells(uint32_t grid, cudaStream_t stream, uint2* shadow, const CellFill* f, uint32_t nf,
+                              uint64_t total);
 // resident blocks of K1 per SM (sets K1's dynamic shared memory limit first)
 cudaError_t shadow_check_blocks_per_sm(int* per_sm);        // cached per device
 cudaError_t shadow_check_blocks_per_sm_query(int* per_sm);  // sets the smem attribute, asks the occupancy API

@@ -433,7 +433,7 @@ int cusan_lower_program(cusan_lowering* l, const cusan_api_call* calls, uint64_t
     if (!l || (n && !calls) || (nargs && !args)) return fail(CUSAN_EINVAL, "null argument");
     {   // room for the typical expansion (a launch is ~6 primitives), so the trace grows once
         std::vector<cusan_event>& ev = l->trace->t.ev;
-        const uint64_t want = std::min<uint64_t>(ev.size() + 4 * n + nargs, CUSAN_MAX_EVENTS);
+        const uint64_t want = std::min<uint64_t>(ev.size() + 4 * n + nargs, CUSAN_MAX_TRACE_EVENTS);
         if (want > ev.capacity()) {
             try {
                 ev.reserve(want);

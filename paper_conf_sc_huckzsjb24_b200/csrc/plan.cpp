@@ -294,6 +294,8 @@ static void prepare_accesses(const Trace& t, HostPlan& hp) {
 // a1 alone for a clocks object (cusan_clocks_compute): every core of the node — on a multi-GPU
 // node one rank computes the clocks while the others wait for the broadcast.
 int compute_clocks(const Trace& t, HostPlan& hp) {
+    if (t.ev.size() > CUSAN_MAX_EVENTS)
+        return fail(CUSAN_ERANGE, "a one-shot check takes at most 2^24-2 events (sessions renumber longer traces)");
     prepare_accesses(t, hp);
     unsigned hw = std::max(1u, std::thread::hardware_concurrency());
     cpu_set_t set;
@@ -322,6 +324,8 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
         return fail(CUSAN_EINVAL, "need 0 <= shard < nshards");
     if (o.window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
     if (int st = check_flags(o)) return st;
+    if (t.ev.size() > CUSAN_MAX_EVENTS)
+        return fail(CUSAN_ERANGE, "a one-shot check takes at most 2^24-2 events (sessions renumber longer traces)");
     hp.opts = o;
     const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
     auto tick = [t0 = std::chrono::steady_clock::now(), dbg](const char* what) {

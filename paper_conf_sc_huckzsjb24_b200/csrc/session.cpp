@@ -243,6 +243,13 @@ struct cusan_session {
     std::vector<SIv> ivs;                           // layout of `shadow`
     uint64_t used = 0;                              // cells of `shadow` in use
     uint64_t checked_access = 0, checked_events = 0, n_calls = 0;
+    // epoch renumbering (sessions longer than the 24-bit epoch field, see session_renumber):
+    // trace event i >= the last renumbering point has compact id i - delta; compact values
+    // (id + 1) 1..orig->size()-1 name older events, orig[v] = their trace value (event id + 1)
+    uint64_t delta = 0;
+    std::shared_ptr<const std::vector<uint32_t>> orig = std::make_shared<const std::vector<uint32_t>>(1, 0u);
+    uint64_t limit = CUSAN_MAX_EVENTS;              // compact ids stay below this (CUSAN_SESSION_EVENT_LIMIT)
+    uint64_t renumberings = 0;
     uint32_t blk_log2 = 21;                         // block-cyclic shard map (nshards > 1)
     bool broken = false;                            // a call failed after changing the state
     // ---- device state (every buffer grows in place, see DevBuf) ----
@@ -341,21 +348,24 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
     c.n_fibers = F;
     s->recs.promote();                 // records dead since the previous call's plan are free now
     // ---- a1: clocks and segments for the new events (build_host_plan's pass, resumed) ----------
+    if (tr.ev.size() - s->delta > s->limit)
+        return fail(CUSAN_ERANGE, "one session call holds more events than the 24-bit epoch field can number");
     for (uint64_t i = s->checked_events; i < tr.ev.size(); i++) {
         const cusan_event& e = tr.ev[i];
         const uint32_t f = e.fiber;
         uint32_t* Cf = &s->C[(size_t)f * F];
+        const uint32_t ci = (uint32_t)(i - s->delta);       // compact event id (= i before any renumbering)
         c.n_events++;
         if (e.kind == CUSAN_EV_FORK) {
             const uint32_t src = (uint32_t)e.a;
             uint32_t* Cs = &s->C[(size_t)src * F];
-            Cs[src] = (uint32_t)(i + 1);
+            Cs[src] = ci + 1;
             for (uint32_t g = 0; g < F; g++) Cf[g] = std::max(Cf[g], Cs[g]);
             s->cur_seg[f] = NO_SEG;
             c.n_fork++;
             continue;
         }
-        Cf[f] = (uint32_t)(i + 1);
+        Cf[f] = ci + 1;
         switch (e.kind) {
             case CUSAN_EV_ACCESS: {
                 if (s->cur_seg[f] == NO_SEG) {
@@ -366,7 +376,7 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
                 const uint64_t g0 = e.a >> 3, g1 = e.b ? (e.a + e.b + 7) >> 3 : g0;
                 cp.g0.push_back(g0);
                 cp.g1.push_back(g1);
-                cp.rec.push_back({pack_epoch(f, (uint32_t)i), s->cur_seg[f] | ((uint32_t)e.mode << 31)});
+                cp.rec.push_back({pack_epoch(f, ci), s->cur_seg[f] | ((uint32_t)e.mode << 31)});
                 const uint64_t bytes = 8 * (g1 - g0);
                 c.n_access++;
                 cp.tracked += bytes;
@@ -586,6 +596,8 @@ struct PendingCall {
     uint64_t used_before = 0;                       // shadow cells in use before the call
     pinned_vector<unsigned long long> init, cnt;    // counter initial values / read-back
     uint64_t h2d = 0;
+    uint64_t delta = 0;                             // event numbering the call was planned with
+    std::shared_ptr<const std::vector<uint32_t>> orig;
     std::chrono::steady_clock::time_point t_start;
 };
 
@@ -623,6 +635,8 @@ static int session_plan(cusan_session* s, PendingCall& pc) {
     }
     if (st) return st;
     session_tick(pc, "plan");
+    pc.delta = s->delta;
+    pc.orig = s->orig;
     // the new layout becomes the session's
     pc.used_before = s->used;
     s->ivs.swap(cp.ivs);
@@ -725,6 +739,17 @@ static int session_finish(cusan_session* s, PendingCall& pc, cusan_report** out)
         delete r;
         return mst;
     }
+    if (pc.orig->size() > 1) {          // compact ids -> trace positions (monotone: order is kept)
+        const std::vector<uint32_t>& orig = *pc.orig;
+        auto to_trace = [&](uint32_t id) -> uint32_t {
+            const uint64_t v = (uint64_t)id + 1;
+            return v < orig.size() ? orig[v] - 1 : (uint32_t)(id + pc.delta);
+        };
+        for (cusan_race_run& x : r->runs) {
+            x.earlier = to_trace(x.earlier);
+            x.later = to_trace(x.later);
+        }
+    }
     r->n_runs = r->runs.size();
     r->n_race_granules = cnt[C_RACE];   // exact even when the run list overflowed
     if (runs_ovf) r->truncated = 1;     // the shadow moved on; the call cannot be re-run
@@ -740,10 +765,105 @@ static int session_finish(cusan_session* s, PendingCall& pc, cusan_report** out)
     r->ctr.shadow_bytes = cp.used * sizeof(uint2);
     r->ctr.h2d_bytes = pc.h2d + pc.init.size() * sizeof(unsigned long long);
     r->ctr.d2h_bytes = d2h;
+    r->ctr.renumberings = s->renumberings;
     r->ctr.run_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - pc.t_start).count();
     *out = r;
     // a run list that overflowed is sized for the next call (best effort: this call succeeded)
     if (runs_ovf) grow_runs(s, cnt[C_RUNS] + cnt[C_RUNS] / 8 + 1024);
+    return CUSAN_OK;
+}
+
+// Epoch renumbering.  Shadow cells, read-set records and clocks hold event ids + 1 in 24 bits, so a
+// session whose trace outgrows 2^24-2 events renumbers, between two calls, every id value still in
+// use: the values in live cells and live records, and every entry of the fiber and sync clocks
+// (which are all future clock entries derive from).  Sorted and ranked, each value v becomes
+// rank(v) in 1..n: injective and monotone on that set, so every later happens-before comparison
+// (an earlier epoch's value against a clock entry of its fiber) and every order
+// between ids comes out as before.  Later events continue above n (compact id = trace id - delta)
+// and reports translate ids back to trace positions (orig[] for the renumbered values).  The
+// segment rows of earlier calls are never read again, so segments restart from 0.
+static int session_renumber(cusan_session* s) {
+    CK(cudaStreamSynchronize(s->stream));
+    const size_t niv = s->ivs.size();
+    const bool compressed = compressed_shadow(s->opts);
+    // one cell per interval (all cells of an interval are equal) and the heap's records
+    std::vector<uint2> cells(niv);
+    if (niv) {
+        if (int st = grow_buf(s, s->scratch, 16 * niv + 512, 0, "plan tables")) return st;
+        std::vector<uint64_t> at(niv);
+        for (size_t i = 0; i < niv; i++) at[i] = s->ivs[i].dense;
+        uint64_t* d_at = (uint64_t*)s->scratch.p;
+        uint2* d_out = (uint2*)(s->scratch.p + align_up(8 * niv));
+        CK(cudaMemcpyAsync(d_at, at.data(), 8 * niv, cudaMemcpyHostToDevice, s->stream));
+        CK(launch_gather_cells(std::max(1, std::min(s->max_blocks, (int)((niv + THREADS - 1) / THREADS))), s->stream,
+                               s->shadow.p, d_at, niv, d_out));
+        CK(cudaMemcpyAsync(cells.data(), d_out, 8 * niv, cudaMemcpyDeviceToHost, s->stream));
+    }
+    std::vector<uint32_t> heap(s->recs.hwm * REC_WORDS);
+    if (!heap.empty())
+        CK(cudaMemcpyAsync(heap.data(), s->heap.p, heap.size() * 4, cudaMemcpyDeviceToHost, s->stream));
+    CK(cudaStreamSynchronize(s->stream));
+    // the id values in use
+    auto is_spill = [](uint32_t e) { return (e >> 24) == 0xFFu; };
+    std::vector<uint32_t> vals;
+    vals.reserve(2 * niv + s->C.size() + s->sc.size());
+    auto add_epoch = [&](uint32_t e) { if (e & 0xffffffu) vals.push_back(e & 0xffffffu); };
+    for (const uint2& c : cells) {
+        add_epoch(c.x);
+        if (!is_spill(c.y)) add_epoch(c.y);
+    }
+    for (const auto& rec : s->recs.live) {
+        const uint32_t* r = &heap[(size_t)rec.first * REC_WORDS];
+        for (uint32_t j = 0; j < (r[0] & 0xffffu); j++) add_epoch(r[1 + j]);
+    }
+    for (uint32_t v : s->C) if (v) vals.push_back(v);
+    for (uint32_t v : s->sc) if (v) vals.push_back(v);
+    std::sort(vals.begin(), vals.end());
+    vals.erase(std::unique(vals.begin(), vals.end()), vals.end());
+    if (vals.size() + 1 >= s->limit / 2)
+        return fail(CUSAN_ERANGE, "too many live event ids to renumber into the 24-bit epoch field");
+    auto rank = [&](uint32_t v) -> uint32_t {
+        return v ? 1u + (uint32_t)(std::lower_bound(vals.begin(), vals.end(), v) - vals.begin()) : 0u;
+    };
+    auto remap = [&](uint32_t e) -> uint32_t { return e ? (e & 0xff000000u) | rank(e & 0xffffffu) : 0u; };
+    // rewrite: cells (one fill per interval), live records, clocks
+    std::vector<CellFill> fills(niv);
+    uint64_t total = 0;
+    for (size_t i = 0; i < niv; i++) {
+        const uint2 c = cells[i];
+        fills[i] = CellFill{total, s->ivs[i].dense, compressed ? 1 : s->ivs[i].len, remap(c.x),
+                            is_spill(c.y) ? c.y : remap(c.y)};
+        total += fills[i].len;
+    }
+    for (const auto& rec : s->recs.live) {
+        uint32_t* r = &heap[(size_t)rec.first * REC_WORDS];
+        for (uint32_t j = 0; j < (r[0] & 0xffffu); j++) r[1 + j] = remap(r[1 + j]);
+    }
+    for (uint32_t& v : s->C) v = rank(v);
+    for (uint32_t& v : s->sc) v = rank(v);
+    if (niv) {
+        if (int st = grow_buf(s, s->scratch, sizeof(CellFill) * niv + 256, 0, "plan tables")) return st;
+        CK(cudaMemcpyAsync(s->scratch.p, fills.data(), sizeof(CellFill) * niv, cudaMemcpyHostToDevice, s->stream));
+        CK(launch_fill_cells(s->max_blocks, s->stream, s->shadow.p, (const CellFill*)s->scratch.p, (uint32_t)niv, total));
+    }
+    if (!heap.empty())
+        CK(cudaMemcpyAsync(s->heap.p, heap.data(), heap.size() * 4, cudaMemcpyHostToDevice, s->stream));
+    CK(cudaStreamSynchronize(s->stream));
+    // numbering: renumbered values -> trace values; later events continue above them
+    const std::vector<uint32_t>& old = *s->orig;
+    auto no = std::make_shared<std::vector<uint32_t>>(vals.size() + 1, 0u);
+    for (size_t r = 0; r < vals.size(); r++) {
+        const uint32_t u = vals[r];
+        (*no)[r + 1] = u < old.size() ? old[u] : (uint32_t)(u + s->delta);
+    }
+    s->orig = no;
+    s->delta = s->checked_events - vals.size();
+    // earlier segment rows are never read again
+    s->cur_seg.assign(s->F, NO_SEG);
+    s->nseg = 0;
+    s->seg_uploaded = 0;
+    s->segvc.clear();
+    s->renumberings++;
     return CUSAN_OK;
 }
 
@@ -766,6 +886,10 @@ int cusan_session_create(const cusan_trace* t, const cusan_check_opts* o, cusan_
     s->opts = *o;
     s->opts.persist_shadow = 1;
     s->blk_log2 = o->shard_block ? (uint32_t)__builtin_ctzll(o->shard_block) : 21u;
+    if (const char* e = std::getenv("CUSAN_SESSION_EVENT_LIMIT")) {     // tests: renumber early
+        const unsigned long long v = std::strtoull(e, nullptr, 10);
+        if (v >= 64) s->limit = std::min<uint64_t>(v, CUSAN_MAX_EVENTS);
+    }
     s->F = t->t.max_fibers;
     s->C.assign((size_t)s->F * s->F, 0);
     s->cur_seg.assign(s->F, NO_SEG);
@@ -803,7 +927,23 @@ int cusan_session_submit(cusan_session* s, cusan_report** prev) {
     std::unique_ptr<PendingCall> next(new (std::nothrow) PendingCall);
     if (!next) return fail(CUSAN_ENOMEM, "cannot allocate a call");
     next->t_start = std::chrono::steady_clock::now();
-    int st = session_plan(s, *next);                 // host: overlaps the call in flight
+    int st;
+    if (s->trace->t.ev.size() - s->delta > s->limit) {   // ids would outgrow 24 bits: renumber first
+        if (s->pending) {                                  // (needs the device state of the call in flight)
+            std::unique_ptr<PendingCall> done = std::move(s->pending);
+            st = session_finish(s, *done, prev);
+            if (st) {
+                s->broken = true;
+                return st;
+            }
+        }
+        st = session_renumber(s);
+        if (st) {
+            s->broken = true;
+            return st;
+        }
+    }
+    st = session_plan(s, *next);                     // host: overlaps the call in flight
     if (st) return st;
     if (s->pending) {                                // collect the call in flight
         std::unique_ptr<PendingCall> done = std::move(s->pending);

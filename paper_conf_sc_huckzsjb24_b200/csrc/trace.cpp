@@ -34,7 +34,7 @@ void canonicalize_runs(std::vector<cusan_race_run>& runs) {
 }
 
 static int validate(const Trace& t, const cusan_event& e, uint64_t pos) {
-    if (pos >= CUSAN_MAX_EVENTS) return fail(CUSAN_ERANGE, "trace longer than 2^24-2 events");
+    if (pos >= CUSAN_MAX_TRACE_EVENTS) return fail(CUSAN_ERANGE, "trace longer than 2^32-2 events");
     if (e.fiber >= t.max_fibers) return fail(CUSAN_EINVAL, "fiber >= max_fibers");
     switch (e.kind) {
         case CUSAN_EV_ACCESS:
@@ -72,7 +72,7 @@ int cusan_trace_create(uint32_t max_fibers, uint64_t reserve_events, cusan_trace
     if (!t) return fail(CUSAN_ENOMEM, "cannot allocate trace");
     t->t.max_fibers = max_fibers;
     try {
-        t->t.ev.reserve(std::min<uint64_t>(reserve_events, CUSAN_MAX_EVENTS));
+        t->t.ev.reserve(std::min<uint64_t>(reserve_events, CUSAN_MAX_TRACE_EVENTS));
     } catch (...) {
         delete t;
         return fail(CUSAN_ENOMEM, "cannot reserve trace");

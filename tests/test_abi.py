@@ -111,18 +111,25 @@ def test_fiber_info_and_text_report():
 
 
 def test_event_index_limit():
-    """Maximum trace length: event id + 1 must fit the 24-bit epoch field."""
+    """One-shot checks number events in the 24-bit epoch field: a trace of 2^24 - 2
+    events plans, one more event is CUSAN_ERANGE for the one-shot planner (and the clocks) — the
+    trace itself grows on (u32 event ids; sessions renumber, tests/test_gpu_session.py)."""
     n = (1 << 24) - 2
     ev = np.zeros(n, EVENT_DTYPE)
     ev["kind"] = 1                                       # RELEASE on key 0 by fiber 0
     t = cs.Trace(2)
     t.cusan_trace_append_events(ev)
     assert len(t) == n
-    with pytest.raises(cs.CusanError) as e:
-        t.cusan_trace_append_sync(cs.CUSAN_RELEASE, 0, 1)
-    assert e.value.status == -2
     d = cs.describe(t)                                   # the planner takes the longest trace
     assert d["n_events"] == n and d["n_release"] == n
+    t.cusan_trace_append_sync(cs.CUSAN_RELEASE, 0, 1)
+    assert len(t) == n + 1
+    with pytest.raises(cs.CusanError) as e:
+        cs.describe(t)
+    assert e.value.status == -2
+    with pytest.raises(cs.CusanError) as e:
+        cs.Clocks.compute(t)
+    assert e.value.status == -2
     del ev, t
 
 

@@ -317,3 +317,110 @@ def test_session_full_size_config5(per_call, flags):
     ses.close()
     assert calls == -(-len(acc_pos) // per_call)
     assert total == int(g["n_race_granules"]) > 0
+
+
+@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_DENSE_SHADOW], ids=["compressed", "dense"])
+@pytest.mark.parametrize("window", [0, 3])
+def test_session_epoch_renumbering_fuzz(window, flags, monkeypatch):
+    """Sessions renumber their live event ids when the trace outgrows the epoch field; with the
+    field's limit lowered to a few hundred events (CUSAN_SESSION_EVENT_LIMIT) renumbering happens
+    every few calls, and every call still equals the oracle's report restricted to it (ids are
+    trace positions in the reports), for many readers (records), splits and windows."""
+    monkeypatch.setenv("CUSAN_SESSION_EVENT_LIMIT", "400")
+    rng = np.random.default_rng(4400 + window + flags)
+    renumbered = 0
+    for _ in range(12):
+        nf = int(rng.integers(2, 10))
+        n = int(rng.integers(300, 900))
+        ev = fuzz.random_primitive_trace(rng, n, nf, n_keys=4, n_granules=int(rng.integers(50, 1500)),
+                                         unaligned=bool(rng.integers(2)), p_access=0.5)
+        acc = ev["kind"] == EV_ACCESS
+        ev["mode"][acc & (rng.random(len(ev)) < 0.5)] = 0
+        cuts = list(range(int(rng.integers(20, 60)), n, int(rng.integers(20, 60))))
+        ref = oracle.check_events(ev, nf, threads=2)
+        tr = cs.Trace(nf)
+        ses = cs.Session(tr, window_events=window, flags=flags)
+        start = 0
+        for end in cuts + [n]:
+            tr.cusan_trace_append_events(ev[start:end])
+            rep = ses.check()
+            want = _by_later(ref["runs"], start, end)
+            assert np.array_equal(rep.runs, want.astype(rep.runs.dtype)), (start, end)
+            start = end
+        renumbered += rep.counters["renumberings"]
+        ses.close()
+    assert renumbered > 10
+
+
+def test_session_epoch_renumbering_pipelined_and_sharded(monkeypatch):
+    """Renumbering with a call in flight (submit / finish) and in block-cyclic shard sessions: the
+    merged shard reports of every call equal the oracle's."""
+    monkeypatch.setenv("CUSAN_SESSION_EVENT_LIMIT", "300")
+    rng = np.random.default_rng(4500)
+    for _ in range(6):
+        nf = int(rng.integers(2, 8))
+        n = 900
+        ev = fuzz.random_primitive_trace(rng, n, nf, n_keys=3, n_granules=int(rng.integers(200, 3000)))
+        ref = oracle.check_events(ev, nf, threads=2)
+        cuts = list(range(40, n, 40)) + [n]
+        trs = [cs.Trace(nf) for _ in range(3)]
+        ses = [cs.Session(trs[s], window_events=2, nshards=3, shard=s, shard_block=64) for s in range(3)]
+        got = {s: [] for s in range(3)}
+        start = 0
+        for end in cuts:
+            for t in trs:
+                t.cusan_trace_append_events(ev[start:end])
+            for k, x in enumerate(ses):
+                prev = x.submit()
+                if prev is not None:
+                    got[k].append(prev)
+            start = end
+        for k, x in enumerate(ses):
+            got[k].append(x.finish())
+            x.close()
+        start = 0
+        for c, end in enumerate(cuts):
+            reps = [got[k][c] for k in range(3)]
+            merged = cs.report_merge(np.concatenate([r.runs for r in reps]), sum(r.n_race_granules for r in reps))
+            want = _by_later(ref["runs"], start, end)
+            assert np.array_equal(merged.runs, want.astype(merged.runs.dtype)), (start, end)
+            start = end
+        assert got[0][-1].counters["renumberings"] > 0
+
+
+def test_session_beyond_2_24_events():
+    """A session past 2^24 events (the real epoch field): 2^24 + 2^21 events in 12 calls — writes,
+    reads and syncs among 4 fibers on a few buffers between long runs of releases; every call equals
+    the oracle's report restricted to it, with trace positions past 2^24 in the runs."""
+    from tracegen.program import EVENT_DTYPE, EV_ACQUIRE, EV_RELEASE
+    rng = np.random.default_rng(2424)
+    n = (1 << 24) + (1 << 21)
+    ev = np.zeros(n, EVENT_DTYPE)
+    ev["kind"] = EV_RELEASE
+    ev["fiber"] = 3
+    ev["a"] = 99
+    pos = np.sort(rng.choice(np.arange(10, n), 3000, replace=False))
+    for p in pos:
+        r = rng.random()
+        f = int(rng.integers(0, 4))
+        if r < 0.6:
+            ev[p]["kind"], ev[p]["mode"], ev[p]["fiber"] = EV_ACCESS, int(rng.random() < 0.4), f
+            ev[p]["a"], ev[p]["b"] = (1 << 32) + 4096 * int(rng.integers(0, 6)), 8 * int(rng.integers(1, 700))
+        else:
+            ev[p]["kind"], ev[p]["fiber"], ev[p]["a"] = (EV_RELEASE if r < 0.8 else EV_ACQUIRE), f, int(rng.integers(0, 3))
+    ref = oracle.check_events(ev, 4, threads=8)
+    assert ref["n_race_granules"] > 0 and int(ref["runs"]["later"].max()) > (1 << 24)
+    tr = cs.Trace(4)
+    ses = cs.Session(tr, window_events=64)
+    cuts = [int(x) for x in np.linspace(0, n, 13)[1:]]
+    start, total = 0, 0
+    for end in cuts:
+        tr.cusan_trace_append_events(ev[start:end])
+        rep = ses.check()
+        want = _by_later(ref["runs"], start, end)
+        assert np.array_equal(rep.runs, want.astype(rep.runs.dtype)), (start, end)
+        total += rep.n_race_granules
+        start = end
+    assert rep.counters["renumberings"] >= 1
+    assert total == ref["n_race_granules"]
+    ses.close()

@@ -416,3 +416,40 @@ def test_listings_kill_lowering_mutants(name):
         if got != {(a, b) for a, b, _ in lst.expect}:
             bad.append(lst.name)
     assert bad, f"mutant {name} passes every paper listing"
+
+
+# ------------------------------------------------------------------------------------------------
+# traces longer than 2^24 events (sessions renumber their epochs; the oracle numbers events by
+# trace position in 32 bits): closed forms
+# ------------------------------------------------------------------------------------------------
+def test_oracle_beyond_2_24_events():
+    """Event ids past 2^24 keep their trace positions.  Fiber 0 writes X (event 0); 2^24 + 5
+    releases by fiber 2 follow; fiber 1 writes X unsynchronised (w1), fiber 0 writes Y (wy, an id
+    past 2^24) and releases key 3, fiber 1 reads Y (ry).  Closed form: runs
+    (0 -> w1) over X and (wy -> ry) over Y; when fiber 1 acquires key 3 before reading Y, only
+    (0 -> w1)."""
+    from tracegen.program import EV_ACQUIRE, EV_RELEASE
+    n_fill = (1 << 24) + 5
+    X, Y, nx, ny = 1 << 30, 1 << 31, 64, 40
+    head = [(EV_ACCESS, 1, 0, X, 8 * nx), (EV_RELEASE, 0, 0, 1, 0)]
+    for racy in (True, False):
+        tail = [(EV_ACCESS, 1, 1, X, 8 * nx), (EV_ACCESS, 1, 0, Y, 8 * ny), (EV_RELEASE, 0, 0, 3, 0)]
+        if not racy:
+            tail.append((EV_ACQUIRE, 0, 1, 3, 0))
+        tail.append((EV_ACCESS, 0, 1, Y, 8 * ny))
+        ev = np.zeros(len(head) + n_fill + len(tail), EVENT_DTYPE)
+        ev["kind"][len(head):len(head) + n_fill] = EV_RELEASE
+        ev["fiber"][len(head):len(head) + n_fill] = 2
+        ev["a"][len(head):len(head) + n_fill] = 7
+        for i, (k, m, f, a, b) in enumerate(head):
+            ev[i]["kind"], ev[i]["mode"], ev[i]["fiber"], ev[i]["a"], ev[i]["b"] = k, m, f, a, b
+        base = len(head) + n_fill
+        for i, (k, m, f, a, b) in enumerate(tail):
+            ev[base + i]["kind"], ev[base + i]["mode"], ev[base + i]["fiber"], ev[base + i]["a"], ev[base + i]["b"] = \
+                k, m, f, a, b
+        rep = oracle.check_events(ev, 3, threads=2)
+        w1, wy, ry = base, base + 1, len(ev) - 1
+        want = [(X >> 3, (X >> 3) + nx, 0, w1)] + ([(Y >> 3, (Y >> 3) + ny, wy, ry)] if racy else [])
+        got = [tuple(int(x) for x in r) for r in rep["runs"]]
+        assert got == want, (racy, got, want)
+        assert ry > (1 << 24)
