@@ -114,6 +114,12 @@ typedef struct cusan_check_opts {
     uint64_t workspace_bytes;
     uint64_t shard_block; /* sessions with nshards > 1: granules per block of the block-cyclic shard
                              map, a power of two (0 = 2^21); one-shot checks shard by range instead */
+    int ngpus;            /* cusan_check only: a whole-node check on devices device .. device+ngpus-1
+                             (0 or 1 = one device): the clocks are computed
+                             once, one host thread per device plans and checks one granule-range
+                             shard, the shards' canonical runs are merged (cusan_report_merge).
+                             Needs nshards == 1, no workspace and no stream (each device's legacy
+                             default stream); CUSAN_ECUDA if the node has fewer devices.      */
 } cusan_check_opts;
 
 /* cusan_plan_create computes the plan but neither allocates nor uploads: the caller queries
@@ -140,7 +146,8 @@ typedef struct cusan_check_opts {
 /* Defaults: nshards 1, shard 0, device 0, window_events 0, persist 0, max_runs 0, all NULL. */
 void cusan_check_opts_init(cusan_check_opts* o);
 
-/* Whole check: plan_create + plan_run + plan_destroy.  The trace is not mutated. */
+/* Whole check: plan_create + plan_run + plan_destroy (or, with opts.ngpus > 1, one shard per
+ * device, checked concurrently and merged).  The trace is not mutated. */
 int cusan_check(const cusan_trace* t, const cusan_check_opts* o, cusan_report** out);
 
 /* Host preparation (a1, a2) and upload of the event / clock / interval tables to the device.
@@ -258,6 +265,9 @@ int cusan_report_counters(const cusan_report* r, cusan_counters* out);
 int cusan_report_merge(const cusan_race_run* runs, uint64_t n_runs, uint64_t n_race_granules,
                        uint64_t max_runs, cusan_report** out);
 int cusan_report_free(cusan_report* r);
+
+/* Number of CUDA devices visible to the process (CUSAN_ECUDA if none / no driver). */
+int cusan_device_count(int* n);
 
 const char* cusan_last_error(void);
 const char* cusan_version(void);

@@ -163,13 +163,14 @@ class Report:
 
 
 def _opts(nshards=1, shard=0, device=0, window_events=0, persist_shadow=False, max_runs=0, stream=None,
-          flags=0, shard_block=0):
+          flags=0, shard_block=0, ngpus=0):
     o = cusan_check_opts()
     lib.cusan_check_opts_init(C.byref(o))
     o.nshards, o.shard, o.device, o.flags = nshards, shard, device, flags
     o.window_events, o.persist_shadow, o.max_runs = window_events, int(persist_shadow), max_runs
     o.stream = stream
     o.shard_block = shard_block
+    o.ngpus = ngpus
     return o
 
 
@@ -346,8 +347,9 @@ def describe(trace: Trace, **kw) -> dict:
 
 def check(trace: Trace, workspace: str | None = None, **kw) -> Report:
     """cusan_check: plan + run + destroy.  kw: nshards, shard, device, window_events,
-    persist_shadow, max_runs, stream (a cudaStream_t as int, e.g. torch's current stream), flags;
-    workspace="torch" allocates the device memory through PyTorch."""
+    persist_shadow, max_runs, stream (a cudaStream_t as int, e.g. torch's current stream), flags,
+    ngpus (a whole-node check: one shard per device, merged); workspace="torch" allocates the
+    device memory through PyTorch."""
     if workspace is not None:
         p = Plan(trace, workspace=workspace, **kw)
         try:

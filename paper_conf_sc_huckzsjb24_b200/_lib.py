@@ -33,7 +33,7 @@ class cusan_check_opts(C.Structure):
                 ("window_events", C.c_int), ("persist_shadow", C.c_int), ("flags", C.c_int),
                 ("max_runs", C.c_uint64),
                 ("stream", C.c_void_p), ("workspace", C.c_void_p), ("workspace_bytes", C.c_uint64),
-                ("shard_block", C.c_uint64)]
+                ("shard_block", C.c_uint64), ("ngpus", C.c_int)]
 
 
 _COUNTER_U64 = ["n_events", "n_access", "n_read", "n_write", "n_release", "n_release_store",
@@ -85,6 +85,7 @@ PROTOS = {
     "cusan_plan_run": [P, PP],
     "cusan_plan_destroy": [P],
     "cusan_release_cached_memory": [],
+    "cusan_device_count": [pi32],
     "cusan_plan_tables": [P, P, u64, P, u64, pu64, pu64],
     "cusan_clocks_compute": [P, PP],
     "cusan_clocks_bytes": [P, pu64],

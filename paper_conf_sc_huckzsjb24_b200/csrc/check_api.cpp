@@ -10,6 +10,7 @@
 #include <mutex>
 #include <new>
 #include <string>
+#include <thread>
 
 #include "kernel.cuh"
 #include "plan_dev.h"
@@ -819,6 +820,18 @@ int cusan_plan_tables(const cusan_plan* p, void* inc, uint64_t inc_cap, void* sp
     return CUSAN_OK;
 }
 
+int cusan_device_count(int* n) {
+    if (!n) return fail(CUSAN_EINVAL, "null argument");
+    *n = 0;
+    cudaError_t e = cudaGetDeviceCount(n);
+    if (e != cudaSuccess) {
+        (void)cudaGetLastError();
+        *n = 0;
+        return fail(CUSAN_ECUDA, std::string("no CUDA device available: ") + cudaGetErrorString(e));
+    }
+    return CUSAN_OK;
+}
+
 int cusan_release_cached_memory(void) {
     WsCache& c = ws_cache();
     std::lock_guard<std::mutex> lk(c.m);
@@ -845,7 +858,96 @@ int cusan_plan_destroy(cusan_plan* p) {
     return CUSAN_OK;
 }
 
+// Whole-node check (opts.ngpus > 1): clocks once, one host thread per device planning (a2 on its
+// device) and checking its granule-range shard, runs merged on the host.  The shards' canonical
+// runs come back to host memory with each plan's report anyway, so the gather needs no collective.
+// CUSAN_NODE_SHARE_DEVICES=1 (tests on a one-GPU machine) maps shard d to device (device+d) mod n.
+static int check_node(const cusan_trace* t, const cusan_check_opts* o, cusan_report** out) {
+    if (o->nshards != 1 || o->shard != 0) return fail(CUSAN_EINVAL, "ngpus > 1 shards by itself: nshards must be 1");
+    if (o->workspace || o->stream) return fail(CUSAN_EINVAL, "ngpus > 1 takes no workspace and no stream");
+    if (o->flags & (CUSAN_CHECK_HOST_PLAN | CUSAN_CHECK_DEFER_WORKSPACE))
+        return fail(CUSAN_EINVAL, "ngpus > 1 plans on the devices with library workspaces");
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess || ndev == 0)
+        return fail(CUSAN_ECUDA, std::string("no CUDA device available: ") + cudaGetErrorString(e));
+    const bool share = std::getenv("CUSAN_NODE_SHARE_DEVICES") != nullptr;
+    if (o->device < 0 || (!share && o->device + o->ngpus > ndev))
+        return fail(CUSAN_ECUDA, "ngpus = " + std::to_string(o->ngpus) + " from device " + std::to_string(o->device) +
+                                     " but the node has " + std::to_string(ndev) + " CUDA devices");
+    const auto t0 = std::chrono::steady_clock::now();
+    cusan_clocks* clocks = nullptr;
+    if (int st = cusan_clocks_compute(t, &clocks)) return st;
+    const int n = o->ngpus;
+    std::vector<cusan_report*> parts(n, nullptr);
+    std::vector<int> status(n, CUSAN_OK);
+    std::vector<std::string> errors(n);
+    std::vector<std::thread> th;
+    for (int d = 0; d < n; d++)
+        th.emplace_back([&, d] {
+            cusan_check_opts so = *o;
+            so.ngpus = 0;
+            so.nshards = n;
+            so.shard = d;
+            so.device = (o->device + d) % ndev;
+            cusan_plan* p = nullptr;
+            int st = cusan_plan_create_from_clocks(clocks, &so, &p);
+            if (!st) {
+                st = cusan_plan_run(p, &parts[d]);
+                cusan_plan_destroy(p);
+            }
+            status[d] = st;
+            if (st) errors[d] = cusan_last_error();
+        });
+    for (auto& x : th) x.join();
+    cusan_clocks_destroy(clocks);
+    int st = CUSAN_OK;
+    for (int d = 0; d < n && !st; d++)
+        if (status[d]) st = fail(status[d], "shard " + std::to_string(d) + ": " + errors[d]);
+    cusan_report* r = nullptr;
+    if (!st) {
+        std::vector<cusan_race_run> runs;
+        uint64_t nrace = 0;
+        for (cusan_report* x : parts) {
+            runs.insert(runs.end(), x->runs.begin(), x->runs.end());
+            nrace += x->n_race_granules;
+        }
+        st = cusan_report_merge(runs.data(), runs.size(), nrace, o->max_runs, &r);
+    }
+    if (!st) {                              // counters: the trace's, summed / maxed over shards
+        cusan_counters& c = r->ctr;
+        c = parts[0]->ctr;
+        for (int d = 1; d < n; d++) {
+            const cusan_counters& x = parts[d]->ctr;
+            c.tracked_bytes_shard += x.tracked_bytes_shard;
+            c.shard_granules += x.shard_granules;
+            c.n_incidences += x.n_incidences;
+            c.n_spans += x.n_spans;
+            c.spill_spans += x.spill_spans;
+            c.spill_heap_bytes += x.spill_heap_bytes;
+            c.shadow_bytes += x.shadow_bytes;
+            c.workspace_bytes += x.workspace_bytes;
+            c.raw_runs += x.raw_runs;
+            c.kernel_launches += x.kernel_launches;
+            c.shadow_cell_bytes += x.shadow_cell_bytes;
+            c.h2d_bytes += x.h2d_bytes;
+            c.d2h_bytes += x.d2h_bytes;
+            c.kernel_ms = std::max(c.kernel_ms, x.kernel_ms);
+            c.n_windows = std::max(c.n_windows, x.n_windows);
+        }
+        c.run_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+        *out = r;
+    }
+    for (cusan_report* x : parts)
+        if (x) cusan_report_free(x);
+    return st;
+}
+
 int cusan_check(const cusan_trace* t, const cusan_check_opts* o, cusan_report** out) {
+    if (!t || !o || !out) return fail(CUSAN_EINVAL, "null argument");
+    *out = nullptr;
+    if (o->ngpus < 0) return fail(CUSAN_EINVAL, "ngpus must be >= 0");
+    if (o->ngpus > 1) return check_node(t, o, out);
     cusan_plan* p = nullptr;
     int st = cusan_plan_create(t, o, &p);
     if (st) return st;

@@ -14,6 +14,8 @@ import pytest
 import torch.distributed as dist
 import torch.multiprocessing as mp
 
+import oracle
+
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 pytestmark = pytest.mark.gpu
 
@@ -144,3 +146,62 @@ def test_nccl_collectives_on_one_gpu():
     p.join(timeout=60)
     assert p.exitcode == 0
     assert res == {"plan": True, "pull": True, "session": True}, res
+
+
+def test_whole_node_check_ngpus(monkeypatch):
+    """cusan_check_opts.ngpus: clocks once, one host thread per device checking one
+    granule-range shard, runs merged — equal to the oracle for ngpus = 1, and for 2-5 shards mapped
+    onto this machine's device(s) (CUSAN_NODE_SHARE_DEVICES, the test hook for a one-GPU box);
+    asking for more devices than the node has is CUSAN_ECUDA."""
+    import paper_conf_sc_huckzsjb24_b200 as cs
+    import torch
+    from tracegen import configs
+    for c in (3, 5):
+        w = configs.make(c, "small")
+        ops, args = w.arrays(True)
+        tr = cs.Trace(255)
+        cs.Lowering(tr).cusan_lower_program(ops, args)
+        ref = oracle.check_events(tr.cusan_trace_read(), 256)
+        rep = cs.check(tr, ngpus=1, window_events=97)
+        assert rep.n_race_granules == ref["n_race_granules"] > 0
+        assert np.array_equal(rep.runs, ref["runs"].astype(rep.runs.dtype))
+        ndev = torch.cuda.device_count()
+        with pytest.raises(cs.CusanError) as e:
+            cs.check(tr, ngpus=ndev + 1)
+        assert e.value.status == -4
+        monkeypatch.setenv("CUSAN_NODE_SHARE_DEVICES", "1")
+        for ngpus, flags in ((2, 0), (3, cs.CUSAN_CHECK_DENSE_SHADOW), (5, 0)):
+            rep = cs.check(tr, ngpus=ngpus, window_events=97, flags=flags)
+            assert rep.n_race_granules == ref["n_race_granules"]
+            assert np.array_equal(rep.runs, ref["runs"].astype(rep.runs.dtype))
+            assert rep.counters["tracked_bytes_shard"] == rep.counters["tracked_bytes"]
+        monkeypatch.delenv("CUSAN_NODE_SHARE_DEVICES")
+        with pytest.raises(cs.CusanError):
+            cs.check(tr, ngpus=2, nshards=2)                       # ngpus shards by itself
+
+
+def test_c_example_node_check(tmp_path):
+    """examples/node_check.c: a C program checks a trace file on every device of the node through
+    cusan_check_opts.ngpus; its runs equal the oracle's."""
+    import subprocess
+    import __graft_entry__ as g
+    import paper_conf_sc_huckzsjb24_b200 as cs
+    from tracegen import configs
+    from tracegen.program import save_events
+    exe = [e for e in g.build_examples() if e.endswith("node_check")][0]
+    w = configs.make(5, "small")
+    ops, args = w.arrays(True)
+    tr = cs.Trace(255)
+    cs.Lowering(tr).cusan_lower_program(ops, args)
+    ev = tr.cusan_trace_read()
+    path = str(tmp_path / "c5.trace")
+    save_events(path, ev, 255)
+    ref = oracle.check_events(ev, 256)
+    want = [f"run {int(r['g_begin'])} {int(r['g_end'])} {int(r['earlier'])} {int(r['later'])}" for r in ref["runs"]]
+    for argv, env in (([path], {}), ([path, "3", "64", "dense"], {"CUSAN_NODE_SHARE_DEVICES": "1"})):
+        out = subprocess.run([exe, *argv], capture_output=True, text=True, timeout=300,
+                             env={**__import__("os").environ, **env})
+        assert out.returncode == 0, out.stderr
+        lines = out.stdout.splitlines()
+        assert f"{ref['n_race_granules']} race granules, {ref['n_runs']} runs" in lines[0]
+        assert lines[1:] == want
