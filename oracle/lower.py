@@ -169,6 +169,9 @@ class Lowering:
             bisect.insort(self.alloc_base, a)
             self.alloc[a] = (b, x)
         elif kind == OP_FREE:
+            if a in self.alloc:                          # TypeART's table drops it (★A25,
+                del self.alloc[a]                        # PAPER.md:306-308, 835-855)
+                self.alloc_base.remove(a)
             self.sync_device_host()
         elif kind == OP_STREAM_CREATE:
             f = self.new_fiber()

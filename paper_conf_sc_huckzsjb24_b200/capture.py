@@ -78,6 +78,7 @@ def _install_hooks():
     gt.register_callback_for_event_synchronization(fwd("_on_event_sync"))
     gt.register_callback_for_stream_synchronization(fwd("_on_stream_sync"))
     gt.register_callback_for_device_synchronization(fwd("_on_device_sync"))
+    gt.register_callback_for_memory_deallocation(fwd("_on_memory_deallocation"))
     _HOOKS_INSTALLED = True
 
 
@@ -122,7 +123,14 @@ class Capture:
         self.trace = Trace(max_fibers)
         self.low = Lowering(self.trace)
         self.streams: set[int] = {0}
-        self.allocs: dict[int, int] = {}
+        # Every allocation instance gets its own synthetic address range in the trace: the caching
+        # allocator hands a freed block to the next tensor (after the stream / event ordering it
+        # enforces itself), and that tensor's accesses must start from fresh shadow state, as
+        # PyTorch's stream sanitizer resets a tensor's state at deallocation.  `allocs` maps a live
+        # storage pointer to (synthetic base, size); `real` maps synthetic bases back.
+        self.allocs: dict[int, tuple[int, int]] = {}
+        self.real: dict[int, tuple[int, int]] = {}
+        self._next_base = 1 << 44
         self.ops = 0
         self.op_names: dict[int, str] = {}           # first event id of an op -> op name
         self._req = itertools.count(1)
@@ -169,12 +177,31 @@ class Capture:
         return handle
 
     def _storage(self, t: torch.Tensor) -> int:
+        """The trace address of a tensor's storage: its allocation instance's synthetic base."""
         st = t.untyped_storage()
         ptr, size = st.data_ptr(), st.nbytes()
-        if ptr and self.allocs.get(ptr) != size:
-            self.allocs[ptr] = size
-            self.low.cusan_on_malloc(ptr, size, 0)
-        return ptr
+        if not ptr:
+            return 0
+        cur = self.allocs.get(ptr)
+        if cur is None or cur[1] != size:
+            base = self._next_base
+            self._next_base += (max(size, 1) + 255) // 256 * 256 + 256
+            self.allocs[ptr] = (base, size)
+            self.real[base] = (ptr, size)
+            self.low.cusan_on_malloc(base, size, 0)
+        return self.allocs[ptr][0]
+
+    def real_address(self, addr: int) -> int:
+        """Device address of a trace (synthetic) address, e.g. ``8 * run["g_begin"]``."""
+        import bisect
+        bases = sorted(self.real)
+        i = bisect.bisect_right(bases, addr) - 1
+        if i < 0:
+            raise KeyError(addr)
+        ptr, size = self.real[bases[i]]
+        if addr - bases[i] > size:
+            raise KeyError(addr)
+        return ptr + (addr - bases[i])
 
     # ---- CUDA trace callbacks -----------------------------------------------------------------------
     @_recording
@@ -200,6 +227,12 @@ class Capture:
     @_recording
     def _on_device_sync(self):
         self.low.cusan_on_device_sync()
+
+    @_recording
+    def _on_memory_deallocation(self, ptr: int):
+        # the block goes back to the caching allocator (no cudaFree, no device sync): forget this
+        # instance, so the next tensor at the same address gets a fresh range
+        self.allocs.pop(ptr, None)
 
     # ---- operator dispatch ---------------------------------------------------------------------------
     @_recording

@@ -94,6 +94,13 @@ struct cusan_lowering {
             allocs.insert(it, {base, size, kind});
         by_base[base] = {base, size, kind};
     }
+    // cudaFree(base): TypeART drops the allocation from its lookup table
+    void remove_alloc(uint64_t base) {
+        auto it = std::lower_bound(allocs.begin(), allocs.end(), base,
+                                   [](const Alloc& a, uint64_t x) { return a.base < x; });
+        if (it != allocs.end() && it->base == base) allocs.erase(it);
+        by_base.erase(base);
+    }
     int new_fiber(uint32_t* f) {
         uint32_t mf = 0;
         cusan_trace_size(trace, nullptr, &mf);
@@ -223,8 +230,9 @@ int cusan_on_malloc(cusan_lowering* l, uint64_t ptr, uint64_t size, enum cusan_m
     return CUSAN_OK;
 }
 
-int cusan_on_free(cusan_lowering* l, uint64_t) {
+int cusan_on_free(cusan_lowering* l, uint64_t ptr) {
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
+    l->remove_alloc(ptr);                 // no longer tracked (★A25)
     return l->host_sync_device();
 }
 

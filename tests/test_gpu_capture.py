@@ -198,3 +198,48 @@ def test_host_threads_are_fibers(fixed):
     else:
         assert rep.n_race_granules == n * 4 // 8 and rep.n_runs == 1
     assert threading.Thread.start.__module__ == "threading"   # patches removed on exit
+
+
+def test_caching_allocator_reuse_after_record_stream_is_clean():
+    """A tensor read on a side stream, handed back with record_stream + del: PyTorch's caching
+    allocator reuses its block only after the side stream's work (an event it queries itself, not
+    a traced sync), and the next tensor at the same address must start from fresh state — as in
+    PyTorch's stream sanitizer, which resets a tensor at deallocation.  Without the per-instance
+    ranges the new tensor's default-stream write would race with the old read (a false positive)."""
+    import time
+    torch.cuda.synchronize()
+    s = torch.cuda.Stream()
+    ptrs = []
+    with Capture() as cap:
+        for i in range(6):
+            x = torch.empty(1 << 16, device="cuda")
+            x.fill_(float(i))                                  # default stream writes the block
+            s.wait_stream(torch.cuda.current_stream())
+            with torch.cuda.stream(s):
+                y = x * 2                                      # side stream reads it
+            x.record_stream(s)
+            ptrs.append(x.data_ptr())
+            del x, y
+            time.sleep(0.05)                                   # side stream done (untraced)
+        torch.cuda.synchronize()
+    assert len(set(ptrs)) < len(ptrs)                          # the allocator did reuse a block
+    rep = _parity(cap)
+    assert rep.n_race_granules == 0
+
+
+def test_reused_block_race_is_still_reported_within_an_instance():
+    """Per-instance ranges only separate allocation instances: a race inside one instance (the side
+    stream reads a tensor the default stream writes, unordered) is reported, and its addresses map
+    back to the tensor's device memory (Capture.real_address)."""
+    torch.cuda.synchronize()
+    s = torch.cuda.Stream()
+    with Capture() as cap:
+        x = torch.zeros(1 << 12, device="cuda")
+        with torch.cuda.stream(s):
+            y = x + 1                                          # unordered with zeros' write
+        torch.cuda.synchronize()
+    rep = _parity(cap)
+    assert rep.n_race_granules == (1 << 12) * 4 // 8
+    g0 = int(rep.runs["g_begin"][0])
+    assert cap.real_address(8 * g0) == x.untyped_storage().data_ptr()
+    del y

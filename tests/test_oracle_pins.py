@@ -381,6 +381,8 @@ _LOWER_MUTANTS = {
                                 "if True:                                       # only a successful"),
     # event re-record joins instead of replacing (A4)
     "event_record_joins": ("self.release_store(f, K_event(c))", "self.release(f, K_event(c))"),
+    # cudaFree keeping the freed allocation registered (★A25)
+    "free_keeps_allocation": ("if a in self.alloc:", "if False:"),
     # cudaFree without its device-wide sync (A8)
     "free_no_sync": ("self.sync_device_host()                      # PAPER.md:448-450", "pass  #"),
 }
