@@ -137,11 +137,15 @@ typedef struct cusan_check_opts {
  * Passing both is CUSAN_EINVAL.  (Flag value 1, a removed diagnostic, is rejected too.) */
 #define CUSAN_CHECK_INTERVAL_SHADOW 4
 #define CUSAN_CHECK_DENSE_SHADOW 8
-/* Build the plan's interval, incidence and span tables (step a2) on the host instead of the device.
- * By default cusan_plan_create runs a1 on the host and a2 on the GPU (sm_100a kernels + CUB sorts
- * and scans, plan_dev.cu) and waits for it; the tables are identical either way (the host path is
- * the reference the tests compare the device tables with, and what cusan_plan_describe runs). */
+/* Where cusan_plan_create builds the interval, incidence and span tables (step a2): on the GPU
+ * (sm_100a kernels + CUB sorts and scans, plan_dev.cu; the plan waits for it) or on the host
+ * (build_host_plan).  The tables are byte-identical either way.  Default: the device for traces of
+ * at least 32768 accesses (env CUSAN_DEVICE_PLAN_MIN_ACCESSES), the host below — the device
+ * planner's fixed cost (three host round trips, ~70 launches, ~0.7 ms) only pays off on large
+ * traces (config 5: 2.3 ms vs 7.4 ms per plan; configs 2-4: the host is faster).  These flags force
+ * one side; passing both is CUSAN_EINVAL.  cusan_plan_describe always plans on the host. */
 #define CUSAN_CHECK_HOST_PLAN 16
+#define CUSAN_CHECK_DEVICE_PLAN 32
 
 /* Defaults: nshards 1, shard 0, device 0, window_events 0, persist 0, max_runs 0, all NULL. */
 void cusan_check_opts_init(cusan_check_opts* o);

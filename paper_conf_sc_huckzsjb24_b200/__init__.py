@@ -181,7 +181,8 @@ def _report(h, max_runs):
 CUSAN_CHECK_DEFER_WORKSPACE = 2
 CUSAN_CHECK_INTERVAL_SHADOW = 4    # the default shadow: one cell per elementary interval (f3)
 CUSAN_CHECK_DENSE_SHADOW = 8       # one cell per 8-byte granule (TSan's layout, §8(d) roofline line)
-CUSAN_CHECK_HOST_PLAN = 16         # build the a2 tables on the host (default: on the device)
+CUSAN_CHECK_HOST_PLAN = 16         # build the a2 tables on the host (default: device for >= 32768 accesses)
+CUSAN_CHECK_DEVICE_PLAN = 32       # build them on the device whatever the trace size
 DSPAN_DTYPE = np.dtype([("abs_begin", "<u8"), ("dense_begin", "<u8"), ("len", "<u8"), ("tile0", "<u8"),
                         ("weight0", "<u8"), ("rsize", "<u4"), ("rweight", "<u4"), ("list_off", "<u4"),
                         ("list_cnt", "<u4"), ("flags", "<u4"), ("rec", "<u4"), ("rec_units", "<u4"),

@@ -545,10 +545,15 @@ int cusan_plan_create(const cusan_trace* t, const cusan_check_opts* o, cusan_pla
     cusan_plan* p = new (std::nothrow) cusan_plan;
     if (!p) return fail(CUSAN_ENOMEM, "cannot allocate plan");
     p->trace = t;
-    // a2 on the device unless asked for the host planner (or there are no accesses to plan)
+    // a2 on the device for large traces (or when asked), on the host for small ones
+    static const uint64_t dev_min = [] {
+        const char* e = std::getenv("CUSAN_DEVICE_PLAN_MIN_ACCESSES");
+        return e && *e ? (uint64_t)std::strtoull(e, nullptr, 10) : (uint64_t)32768;
+    }();
     uint64_t n_acc = 0;
     for (const cusan_event& e : t->t.ev) n_acc += e.kind == CUSAN_EV_ACCESS;
-    p->dev_planned = !(o->flags & CUSAN_CHECK_HOST_PLAN) && n_acc > 0;
+    p->dev_planned = n_acc > 0 && !(o->flags & CUSAN_CHECK_HOST_PLAN) &&
+                     ((o->flags & CUSAN_CHECK_DEVICE_PLAN) || n_acc >= dev_min);
     int st;
     try {
         st = build_host_plan(t->t, *o, p->hp, 0, 0, p->dev_planned);

@@ -311,10 +311,12 @@ int compute_clocks(const Trace& t, HostPlan& hp) {
 
 int check_flags(const cusan_check_opts& o) {
     const int known = CUSAN_CHECK_DEFER_WORKSPACE | CUSAN_CHECK_INTERVAL_SHADOW | CUSAN_CHECK_DENSE_SHADOW |
-                      CUSAN_CHECK_HOST_PLAN;
+                      CUSAN_CHECK_HOST_PLAN | CUSAN_CHECK_DEVICE_PLAN;
     if (o.flags & ~known) return fail(CUSAN_EINVAL, "unknown cusan_check_opts.flags bits");
     if ((o.flags & CUSAN_CHECK_INTERVAL_SHADOW) && (o.flags & CUSAN_CHECK_DENSE_SHADOW))
         return fail(CUSAN_EINVAL, "CUSAN_CHECK_INTERVAL_SHADOW and CUSAN_CHECK_DENSE_SHADOW exclude each other");
+    if ((o.flags & CUSAN_CHECK_HOST_PLAN) && (o.flags & CUSAN_CHECK_DEVICE_PLAN))
+        return fail(CUSAN_EINVAL, "CUSAN_CHECK_HOST_PLAN and CUSAN_CHECK_DEVICE_PLAN exclude each other");
     return CUSAN_OK;
 }
 

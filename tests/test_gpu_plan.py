@@ -13,7 +13,7 @@ from tracegen import configs, fuzz
 
 pytestmark = pytest.mark.gpu
 
-HOST = cs.CUSAN_CHECK_HOST_PLAN
+HOST, DEVICE = cs.CUSAN_CHECK_HOST_PLAN, cs.CUSAN_CHECK_DEVICE_PLAN
 COUNTERS = ["n_intervals", "n_incidences", "n_spans", "n_windows", "shard_granules", "tracked_bytes",
             "tracked_bytes_shard", "spill_spans", "spill_heap_bytes", "shadow_bytes", "n_segments", "n_access",
             "shadow_cell_bytes"]
@@ -28,7 +28,7 @@ def _tables(tr, **kw):
 
 
 def assert_same_plan(tr, **kw):
-    di, ds, dr = _tables(tr, **kw)
+    di, ds, dr = _tables(tr, **dict(kw, flags=kw.get("flags", 0) | DEVICE))
     hi, hs, hr = _tables(tr, **dict(kw, flags=kw.get("flags", 0) | HOST))
     assert di.tobytes() == hi.tobytes(), "incidence tables differ"
     assert len(ds) == len(hs) and ds.tobytes() == hs.tobytes(), "span tables differ"
@@ -138,3 +138,5 @@ def test_plan_from_clocks_equals_plan_from_trace(c):
         assert np.array_equal(merged.runs, ref["runs"].astype(merged.runs.dtype))
     with pytest.raises(cs.CusanError):
         cs.Plan(clocks, flags=cs.CUSAN_CHECK_HOST_PLAN)
+    with pytest.raises(cs.CusanError):
+        cs.Plan(tr, flags=cs.CUSAN_CHECK_HOST_PLAN | cs.CUSAN_CHECK_DEVICE_PLAN)
