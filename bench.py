@@ -13,8 +13,8 @@ Two shadow layouts give the identical report; the line carries both:
     fastest exact path; its end-to-end time is host work (lowering, planning), not HBM.
 `e2e` repeats the metric through the public API from host buffers: lowering of the recorded
 CUDA/MPI call program (a0), planning (a1, a2), table upload from pinned host memory, check and
-report download, every step — pipelined (`pipelined_checks`: the host side of step i+1 overlaps
-the GPU side of step i), with the unpipelined per-call number under `e2e.serial` and a per-phase
+report download, every step — pipelined (`pipelined_checks`: lowering, clocks and plan of the next
+steps on host threads overlap the GPU side of step i), with the unpipelined per-call number under `e2e.serial` and a per-phase
 cost breakdown (lower / plan / upload / kernels / merge + download) under `breakdown`.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
@@ -346,16 +346,16 @@ def run_ours(args):
         pkw = dict(window_events=args.window, stream=stream.cuda_stream, flags=flags)
         if world > 1:
             pkw.update(nshards=world, shard=rank)
-        # at least --e2e-steps timed steps and ~2 s of them (short steps are noisy), two warm-up steps
+        # at least --e2e-steps timed steps and ~2 s of them (short steps are noisy), four warm-up steps
         n = max(1, args.e2e_steps, min(800, int(2.0 / max(1e-5, step_s_hint))))
         h2d = d2h = 0
         barrier()
         torch.cuda.synchronize(dev)
         t0 = None
         kms = []
-        for i, (_tr, r2) in enumerate(cs.pipelined_checks(make_trace, n + 2, device=local, **pkw)):
-            if i < 2:                                # warm-up steps: fill the pipeline
-                if i == 1:
+        for i, (_tr, r2) in enumerate(cs.pipelined_checks(make_trace, n + 4, device=local, **pkw)):
+            if i < 4:                                # warm-up steps: fill the pipeline
+                if i == 3:
                     barrier()
                     t0 = time.perf_counter()
                 continue
@@ -540,8 +540,9 @@ def run_ours(args):
         "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "ms_per_step": 1e3 * e2e_step_s, "steps": n_e2e,
                 "kernel_ms_per_step": e2e_kms,
-                "mode": ("pipelined_checks: lowering of step i+2 and planning of step i+1 (host threads) overlap the GPU check of step i; "
-                         "pinned host tables uploaded and the report downloaded every step; 2 warm-up steps") if world == 1 else
+                "mode": ("pipelined_checks: lowering of step i+3, clocks (a1) of step i+2 and the plan (a2) of step i+1 on "
+                         "host threads overlap the GPU check of step i; pinned host tables uploaded and the report "
+                         "downloaded every step; 4 warm-up steps") if world == 1 else
                         ("sharded, serial: rank 0 lowers + computes clocks, broadcast, every rank plans its shard on its GPU, "
                          "checks, runs gathered to rank 0 (median of 3 steps, phases max over ranks)"),
                 "serial": {"value": e2e_serial, "unit": "GB/s", "ms_per_step": dense_breakdown["total_ms"],

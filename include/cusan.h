@@ -196,8 +196,9 @@ int cusan_clocks_bytes(const cusan_clocks* c, uint64_t* bytes);
 int cusan_clocks_export(const cusan_clocks* c, void* buf, uint64_t bytes);
 int cusan_clocks_import(const void* buf, uint64_t bytes, cusan_clocks** out);
 int cusan_clocks_destroy(cusan_clocks* c);
-/* As cusan_plan_create, from clocks (the clocks need not outlive the plan); CUSAN_CHECK_HOST_PLAN
- * is rejected.  Results equal cusan_plan_create's on the trace the clocks came from. */
+/* As cusan_plan_create, from clocks (the clocks need not outlive the plan; a2 on the device or the
+ * host by the same rule).  Tables and results equal cusan_plan_create's on the trace the clocks came
+ * from.  Splitting a0 / a1 / a2 this way lets a pipeline run them on separate host threads. */
 int cusan_plan_create_from_clocks(const cusan_clocks* c, const cusan_check_opts* o, cusan_plan** out);
 /* Host steps a1 and a2 only (no device needed): fills the trace / plan counters the same
  * plan_create would compute (shard clip, intervals, segments, windows, spill records). */

@@ -364,39 +364,51 @@ def check(trace: Trace, workspace: str | None = None, **kw) -> Report:
 
 
 def pipelined_checks(make_trace, steps: int, device: int = 0, **kw):
-    """Check `steps` traces one after another with the host and the GPU overlapped, as a
-    three-stage pipeline: while the GPU checks trace i (a3-a5), one host thread plans trace i+1
-    (a1, a2) and another builds trace i+2 (`make_trace(i+2)`, e.g. lowering the next batch of
-    recorded calls, a0), so a step costs the slowest stage rather than their sum.  This is how an
-    online checker keeps host and GPU busy.  Every plan's tables are uploaded (host -> device) when it is bound, after the
-    previous plan's run completed, and every run downloads its report, so each step still pays
-    its own transfers.  All plans share one workspace from PyTorch's caching allocator (a plan's
-    shadow and records are scratch for its own run).  Yields (trace, report) per step; kw as for
-    Plan (window_events, nshards, shard, stream, flags, ...)."""
+    """Check `steps` traces one after another with the host and the GPU overlapped, as a four-stage
+    pipeline on separate threads: while the GPU checks trace i (a3-a5), one host thread builds the
+    plan of trace i+1 (a2, on the device planner's own stream or on the host), one computes the
+    clocks of trace i+2 (a1, cusan_clocks_compute) and one builds trace i+3 (`make_trace(i+3)`, e.g.
+    lowering the next batch of recorded calls, a0) — a step costs the slowest stage rather than
+    their sum.  This is how an online checker keeps host and GPU busy.  Every plan's tables are
+    uploaded (host -> device) when it is bound, after the previous plan's run completed, and every
+    run downloads its report, so each step still pays its own transfers.  All plans share one
+    workspace from PyTorch's caching allocator (a plan's shadow and records are scratch for its own
+    run).  Yields (trace, report) per step; kw as for Plan (window_events, nshards, shard, stream,
+    flags, ...)."""
     from concurrent.futures import ThreadPoolExecutor
 
-    import torch
     kw = dict(kw)
     kw["flags"] = kw.get("flags", 0) | CUSAN_CHECK_DEFER_WORKSPACE
     kw["device"] = device
     _default_torch_stream(kw)
     kw.pop("device")
+    depth = 3                                   # steps in flight ahead of the GPU
 
     ws = None
-    with ThreadPoolExecutor(1) as lower_ex, ThreadPoolExecutor(1) as plan_ex:
-        traces = {j: lower_ex.submit(make_trace, j) for j in range(min(2, steps))}
+    with ThreadPoolExecutor(1) as lower_ex, ThreadPoolExecutor(1) as clock_ex, ThreadPoolExecutor(1) as plan_ex:
+        futures = {}
 
-        def prepare(j):
-            tr = traces.pop(j).result()
-            return tr, Plan(tr, device=device, **kw)
+        def schedule(j):
+            lf = lower_ex.submit(make_trace, j)
 
-        nxt = plan_ex.submit(prepare, 0) if steps > 0 else None
+            def clocks(f=lf):
+                tr = f.result()
+                return tr, Clocks.compute(tr)
+
+            cf = clock_ex.submit(clocks)
+
+            def plan(f=cf):
+                tr, ck = f.result()
+                return tr, Plan(ck, device=device, **kw)
+
+            futures[j] = plan_ex.submit(plan)
+
+        for j in range(min(depth + 1, steps)):
+            schedule(j)
         for i in range(steps):
-            tr, p = nxt.result()
-            if i + 2 < steps:
-                traces[i + 2] = lower_ex.submit(make_trace, i + 2)
-            if i + 1 < steps:
-                nxt = plan_ex.submit(prepare, i + 1)
+            tr, p = futures.pop(i).result()
+            if i + depth + 1 < steps:
+                schedule(i + depth + 1)
             need = max(p.workspace_bytes(), 256)
             if ws is None or ws.numel() < need:
                 ws = None

@@ -155,6 +155,15 @@ struct cusan_plan {
 
 static int plan_bind(cusan_plan* p, char* ws, uint64_t bytes);
 
+// Traces with at least this many accesses build their a2 tables on the device (cusan.h)
+static uint64_t device_plan_min_accesses() {
+    static const uint64_t v = [] {
+        const char* e = std::getenv("CUSAN_DEVICE_PLAN_MIN_ACCESSES");
+        return e && *e ? (uint64_t)std::strtoull(e, nullptr, 10) : (uint64_t)32768;
+    }();
+    return v;
+}
+
 // ---- pinned host blocks for uploaded tables (common.h) ------------------------------------------
 // Every block carries a 64-byte header {size class, pinned?}.  Freed blocks go back to a cache by
 // size class (powers of two from 64 KiB) up to PINNED_CACHE_MAX bytes; a process without a usable
@@ -546,17 +555,14 @@ int cusan_plan_create(const cusan_trace* t, const cusan_check_opts* o, cusan_pla
     if (!p) return fail(CUSAN_ENOMEM, "cannot allocate plan");
     p->trace = t;
     // a2 on the device for large traces (or when asked), on the host for small ones
-    static const uint64_t dev_min = [] {
-        const char* e = std::getenv("CUSAN_DEVICE_PLAN_MIN_ACCESSES");
-        return e && *e ? (uint64_t)std::strtoull(e, nullptr, 10) : (uint64_t)32768;
-    }();
+    const uint64_t dev_min = device_plan_min_accesses();
     uint64_t n_acc = 0;
     for (const cusan_event& e : t->t.ev) n_acc += e.kind == CUSAN_EV_ACCESS;
     p->dev_planned = n_acc > 0 && !(o->flags & CUSAN_CHECK_HOST_PLAN) &&
                      ((o->flags & CUSAN_CHECK_DEVICE_PLAN) || n_acc >= dev_min);
     int st;
     try {
-        st = build_host_plan(t->t, *o, p->hp, 0, 0, p->dev_planned);
+        st = build_host_plan(&t->t, *o, p->hp, 0, 0, p->dev_planned);
     } catch (const std::bad_alloc&) {
         st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
     }
@@ -681,7 +687,6 @@ int cusan_plan_create_from_clocks(const cusan_clocks* c, const cusan_check_opts*
     if (o->nshards < 1 || o->shard < 0 || o->shard >= o->nshards) return fail(CUSAN_EINVAL, "need 0 <= shard < nshards");
     if (o->window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
     if (int st = check_flags(*o)) return st;
-    if (o->flags & CUSAN_CHECK_HOST_PLAN) return fail(CUSAN_EINVAL, "plans from clocks build their tables on the device");
     cusan_plan* p = new (std::nothrow) cusan_plan;
     if (!p) return fail(CUSAN_ENOMEM, "cannot allocate plan");
     int st = CUSAN_OK;
@@ -695,7 +700,9 @@ int cusan_plan_create_from_clocks(const cusan_clocks* c, const cusan_check_opts*
         hp.acc_g1 = c->hp.acc_g1;
         hp.acc_rec = c->hp.acc_rec;
         hp.segvc = c->hp.segvc;
-        p->dev_planned = !hp.acc_g0.empty();
+        p->dev_planned = !hp.acc_g0.empty() && !(o->flags & CUSAN_CHECK_HOST_PLAN) &&
+                         ((o->flags & CUSAN_CHECK_DEVICE_PLAN) || hp.acc_g0.size() >= device_plan_min_accesses());
+        if (!p->dev_planned) st = build_host_plan(nullptr, *o, hp);   // a2 on the host, from the clocks
     } catch (const std::bad_alloc&) {
         st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
     }
@@ -713,7 +720,7 @@ int cusan_plan_describe(const cusan_trace* t, const cusan_check_opts* o, cusan_c
     HostPlan hp;
     int st;
     try {
-        st = build_host_plan(t->t, *o, hp);
+        st = build_host_plan(&t->t, *o, hp);
     } catch (const std::bad_alloc&) {
         st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
     }

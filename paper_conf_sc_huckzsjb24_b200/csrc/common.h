@@ -165,8 +165,9 @@ struct HostPlan {
 
 // a1 + a2.  Spans (windows) are planned for the accesses from `first_access` on (0 = all);
 // pre-assigned read-set records are numbered from `rec_base`.  a1_only: the accesses and a1 only
-// (a2 runs on the device, plan_dev.cu).
-int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uint64_t first_access = 0,
+// (a2 runs on the device, plan_dev.cu).  t = nullptr: a2 only, hp already holds the accesses and
+// a1's products (a plan from clocks).
+int build_host_plan(const Trace* t, const cusan_check_opts& o, HostPlan& hp, uint64_t first_access = 0,
                     uint64_t rec_base = 0, bool a1_only = false);
 
 // a1 of a whole trace for a clocks object (cusan_clocks_compute), with the node's cores

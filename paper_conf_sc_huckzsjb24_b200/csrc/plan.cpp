@@ -320,13 +320,13 @@ int check_flags(const cusan_check_opts& o) {
     return CUSAN_OK;
 }
 
-int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uint64_t first_access,
+int build_host_plan(const Trace* tp, const cusan_check_opts& o, HostPlan& hp, uint64_t first_access,
                     uint64_t rec_base, bool a1_only) {
     if (o.nshards < 1 || o.shard < 0 || o.shard >= o.nshards)
         return fail(CUSAN_EINVAL, "need 0 <= shard < nshards");
     if (o.window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
     if (int st = check_flags(o)) return st;
-    if (t.ev.size() > CUSAN_MAX_EVENTS)
+    if (tp && tp->ev.size() > CUSAN_MAX_EVENTS)
         return fail(CUSAN_ERANGE, "a one-shot check takes at most 2^24-2 events (sessions renumber longer traces)");
     hp.opts = o;
     const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
@@ -335,17 +335,18 @@ int build_host_plan(const Trace& t, const cusan_check_opts& o, HostPlan& hp, uin
             std::fprintf(stderr, "build_host_plan: %-12s %8.3f ms\n", what,
                          std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
     };
-    prepare_accesses(t, hp);
+    if (tp) prepare_accesses(*tp, hp);        // (no trace: hp holds the accesses and a1's products)
     const uint32_t F = hp.F;
     const uint64_t n_acc = hp.acc_g0.size();
     cusan_counters& c = hp.ctr;
     // ---------------------------------------------------------------- a1: clocks and segments --
     // Runs on its own thread while a2 builds the intervals (a2 needs a1's records only to fill the
     // incidence table at the end).  Errors come back as (status, message).
-    const unsigned a1_threads = plan_threads((uint64_t)t.ev.size() * F / 64);
+    const unsigned a1_threads = plan_threads(hp.ctr.n_events * F / 64);
     auto a1 = [&]() -> std::pair<int, std::string> {
+        if (!tp) return {CUSAN_OK, ""};
         const auto a1_t0 = std::chrono::steady_clock::now();
-        std::pair<int, std::string> st = run_a1(t, hp, a1_threads);
+        std::pair<int, std::string> st = run_a1(*tp, hp, a1_threads);
         tick("a1 (thread)");
         if (dbg)
             std::fprintf(stderr, "build_host_plan: a1 alone     %8.3f ms (%llu segments, %u threads)\n",
