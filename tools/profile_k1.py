@@ -18,12 +18,14 @@ ap.add_argument("--nshards", type=int, default=8)
 ap.add_argument("--shard", type=int, default=0)
 ap.add_argument("--window", type=int, default=4096)
 ap.add_argument("--runs", type=int, default=1)
+ap.add_argument("--compressed", action="store_true", help="the interval-compressed shadow (default: dense)")
 a = ap.parse_args()
 w = configs.make(a.config, "full")
 ops, args = w.arrays(True)
 tr = cs.Trace(255)
 cs.Lowering(tr).cusan_lower_program(ops, args)
-plan = cs.Plan(tr, window_events=a.window, nshards=a.nshards, shard=a.shard)
+plan = cs.Plan(tr, window_events=a.window, nshards=a.nshards, shard=a.shard,
+               flags=0 if a.compressed else cs.CUSAN_CHECK_DENSE_SHADOW)
 for i in range(1 + a.runs):
     r = plan.run()
     c = r.counters
