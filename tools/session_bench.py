@@ -30,12 +30,14 @@ ap.add_argument("--nshards", type=int, default=1)
 ap.add_argument("--shard-block", type=int, default=0)
 ap.add_argument("--summary", action="store_true", help="omit the per-call list")
 ap.add_argument("--max-calls", type=int, default=0, help="stop after this many calls (0 = whole trace)")
+ap.add_argument("--dense", action="store_true", help="per-granule shadow (default: interval-compressed)")
 ap.add_argument("--pipelined", action="store_true",
                 help="submit/finish: plan call i+1 on the host while the GPU checks call i (one shard)")
 a = ap.parse_args()
 if a.pipelined and a.nshards != 1:
     raise SystemExit("--pipelined times one session (on N GPUs every shard pipelines on its own)")
 
+FLAGS = cs.CUSAN_CHECK_DENSE_SHADOW if a.dense else 0
 w = configs.make(a.config, a.size)
 ops, args = w.arrays(True)
 full = cs.Trace(255)
@@ -48,7 +50,7 @@ if a.max_calls:
 
 if a.pipelined:
     tr = cs.Trace(255)
-    ses = cs.Session(tr, window_events=a.window)
+    ses = cs.Session(tr, window_events=a.window, flags=FLAGS)
     reps, start = [], 0
     t0 = time.perf_counter()
     for end in cuts:
@@ -62,13 +64,14 @@ if a.pipelined:
     ses.close()
     tot = sum(r.counters["tracked_bytes"] for r in reps)
     kms = sum(r.counters["kernel_ms"] for r in reps)
-    print(json.dumps(dict(config=a.config, chunk_accesses=a.chunk, pipelined=True, calls=len(reps),
+    print(json.dumps(dict(config=a.config, chunk_accesses=a.chunk, pipelined=True, dense=a.dense, calls=len(reps),
                           tracked_bytes=tot, checked_gbs=tot / secs / 1e9, kernel_checked_gbs=tot / (kms / 1e3) / 1e9,
                           seconds=secs, kernel_ms=kms, race_granules=sum(r.n_race_granules for r in reps))))
     raise SystemExit(0)
 
 trs = [cs.Trace(255) for _ in range(a.nshards)]
-sess = [cs.Session(trs[s], window_events=a.window, nshards=a.nshards, shard=s, shard_block=a.shard_block)
+sess = [cs.Session(trs[s], window_events=a.window, nshards=a.nshards, shard=s, shard_block=a.shard_block,
+                   flags=FLAGS)
         for s in range(a.nshards)]
 start, calls = 0, []
 for end in cuts:
@@ -93,7 +96,7 @@ tot = sum(x["tracked"] for x in calls)
 secs = sum(x["seconds"] for x in calls)
 kms = sum(x["kernel_ms"] for x in calls)
 cell = sum(x["cell_bytes"] for x in calls)
-out = dict(config=a.config, chunk_accesses=a.chunk, nshards=a.nshards, calls=len(calls), tracked_bytes=tot,
+out = dict(config=a.config, chunk_accesses=a.chunk, dense=a.dense, nshards=a.nshards, calls=len(calls), tracked_bytes=tot,
            checked_gbs=tot / secs / 1e9, kernel_checked_gbs=tot / (kms / 1e3) / 1e9,
            kernel_dram_gbs_per_shard=cell / a.nshards / (kms / 1e3) / 1e9, seconds=secs, kernel_ms=kms,
            race_granules=sum(x["races"] for x in calls), per_call=calls)
