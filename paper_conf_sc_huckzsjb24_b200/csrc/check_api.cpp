@@ -402,6 +402,13 @@ static int plan_device_setup(cusan_plan* p) {
         if (!p->dscr) return fail(CUSAN_ENOMEM, "cannot create the device planning scratch");
         DevPlanOut dp;
         int e = device_plan_a2(hp, span_args(p->max_blocks), *p->dscr, dp);
+        if (e == CUSAN_ERANGE) {       // beyond the device planner's 2^31 items: plan a2 on the host
+            plan_dev_release(p->dscr);
+            p->dscr = nullptr;
+            p->dev_planned = false;
+            if ((e = build_host_plan(nullptr, hp.opts, hp))) return e;
+            return plan_device_setup(p);
+        }
         if (e) return e;
         cusan_counters& c = hp.ctr;
         c.n_intervals = dp.n_intervals;

@@ -170,6 +170,7 @@ static void radix_sort_pairs(std::vector<uint64_t>& key, std::vector<uint32_t>& 
 //      tick — so the columns are split among threads, each replaying the whole trace on its columns
 //      and writing them into the segment rows.  Same rows as one pass over whole clocks.
 std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned threads) {
+    const auto t_start = std::chrono::steady_clock::now();
     const uint32_t F = hp.F;
     const uint64_t n = t.ev.size();
     cusan_counters& c = hp.ctr;
@@ -219,6 +220,11 @@ std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned thread
         }
     }
     c.n_segments = hp.nseg;
+    if (std::getenv("CUSAN_DEBUG_TIMING"))
+        std::fprintf(stderr, "run_a1: pre-pass %.3f ms\n",
+                     std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count());
+    static const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
+    const auto t_pre = std::chrono::steady_clock::now();
     hp.segvc.resize(hp.nseg * F);
     const uint32_t nkeys = key_slot.size();
     // columns per thread: multiples of 8, at least 8 (one AVX2 vector of u32)
@@ -256,6 +262,10 @@ std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned thread
                 for (uint32_t g = 0; g < G; g++) Cf[g] = std::max(Cf[g], Sk[g]);
         }
     });
+    if (dbg)
+        std::fprintf(stderr, "run_a1: segvc resize + column pass %.3f ms on %u threads (%u keys)\n",
+                     std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_pre).count(), T,
+                     nkeys);
     return {CUSAN_OK, ""};
 }
 

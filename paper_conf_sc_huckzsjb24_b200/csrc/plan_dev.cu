@@ -707,7 +707,8 @@ int device_plan_a2(const HostPlan& hp, const DevPlanArgs& A, DevScratch& S, DevP
     out.launches += 8;
     const uint64_t niv = hh[H_NIV], npairs = hh[H_NPAIRS], total_dense = hh[H_DENSE];
     out.n_intervals = niv;
-    if (npairs > 0xffffffffull) return fail(CUSAN_ERANGE, "too many interval incidences");
+    if (npairs > 0x7fffffffull)      // CUB's item counts are int; the host planner takes up to 2^32
+        return fail(CUSAN_ERANGE, "more than 2^31 interval incidences: plan on the host (CUSAN_CHECK_HOST_PLAN)");
     if (!niv) return CUSAN_OK;
     // the weights of the shard search must fit 64 bits (the host planner uses 128-bit sums)
     const bool windowed = W < n && !compressed;

@@ -2,11 +2,13 @@
 
 Every case is a seeded random trace (primitive TSan-level events, or a random CUDA-aware MPI call
 program lowered by the product's C lowering and checked against the oracle's own Python lowering)
-checked through every mode — one window and small windows, the range and the lane-parallel paths,
-the interval-compressed shadow (f3), granule-range shards (one-shot) and block-cyclic shard
-sessions, sequential and pipelined sessions — and compared with the oracle bit for bit.
+checked through every mode — one window and small windows, both shadow layouts (interval-compressed,
+the default, and dense), host and device planning, plans from (exported / imported) clocks,
+whole-node checks (ngpus, shards mapped onto this GPU), granule-range shards (one-shot),
+sequential, pipelined and block-cyclic shard sessions, sessions renumbering their event ids every
+few calls — and compared with the oracle bit for bit.
 
-    python tools/fuzz_campaign.py --minutes 20 --seed 1 > profiles/fuzz_campaign_r01.json
+    python tools/fuzz_campaign.py --minutes 20 --seed 1 > profiles/fuzz_campaign_r02.json
 """
 import argparse
 import json
@@ -31,6 +33,8 @@ a = ap.parse_args()
 rng = np.random.default_rng(a.seed)
 stats = {"cases": 0, "checks": 0, "mismatches": 0, "racy_cases": 0, "by_mode": {}, "first_failures": []}
 FL, IV = cs.CUSAN_CHECK_DENSE_SHADOW, cs.CUSAN_CHECK_INTERVAL_SHADOW
+HP, DP = cs.CUSAN_CHECK_HOST_PLAN, cs.CUSAN_CHECK_DEVICE_PLAN
+os.environ["CUSAN_NODE_SHARE_DEVICES"] = "1"          # ngpus > 1 on this one GPU
 
 
 def same(rep_runs, rep_n, ref):
@@ -57,8 +61,18 @@ def one_case(ev, nf, case):
     windows = [0, int(rng.integers(1, 6)), max(1, n_acc // 3)]
     for w in windows:
         for flags in (0, FL, IV):
-            r = cs.check(tr, window_events=w, flags=flags)
-            record(f"oneshot w={'all' if w == 0 else 'small'} flags={flags}", same(r.runs, r.n_race_granules, ref), case)
+            plan = int(rng.choice([HP, DP]))
+            r = cs.check(tr, window_events=w, flags=flags | plan)
+            record(f"oneshot w={'all' if w == 0 else 'small'} flags={flags} {'device' if plan == DP else 'host'} plan",
+                   same(r.runs, r.n_race_granules, ref), case)
+    ck = cs.Clocks.from_bytes(cs.Clocks.compute(tr).to_bytes())
+    flags = int(rng.choice([0, FL])) | int(rng.choice([HP, DP]))
+    p = cs.Plan(ck, window_events=int(rng.integers(0, 5)), flags=flags)
+    r = p.run()
+    p.close()
+    record("plan from clocks", same(r.runs, r.n_race_granules, ref), case)
+    r = cs.check(tr, ngpus=int(rng.integers(2, 5)), window_events=int(rng.integers(0, 5)), flags=int(rng.choice([0, FL])))
+    record("ngpus", same(r.runs, r.n_race_granules, ref), case)
     ns = int(rng.integers(2, 6))
     w = int(rng.integers(0, 5))
     flags = int(rng.choice([0, FL, IV]))          # shards of one check share its options
@@ -67,21 +81,33 @@ def one_case(ev, nf, case):
     record("oneshot shards", same(m.runs, m.n_race_granules, ref), case)
     # sessions: random cut points, sequential / pipelined / block-cyclic shards
     cuts = sorted({0, len(ev), *rng.integers(1, max(2, len(ev)), int(rng.integers(1, 5))).tolist()})
-    for mode in ("session", "pipelined", "session shards"):
+    for mode in ("session", "pipelined", "session shards", "session renumbering"):
         flags = int(rng.choice([0, FL, IV]))
         nsh = int(rng.integers(2, 5)) if mode == "session shards" else 1
         blk = int(2 ** rng.integers(3, 9))
         trs = [cs.Trace(nf) for _ in range(nsh)]
+        if mode == "session renumbering":          # event-id limit low enough to renumber every few calls
+            cuts = sorted({0, len(ev), *range(int(rng.integers(8, 40)), len(ev), int(rng.integers(8, 40)))})
+            os.environ["CUSAN_SESSION_EVENT_LIMIT"] = str(max(64, len(ev) // 2))
         ses = [cs.Session(trs[s], window_events=int(rng.integers(0, 4)), flags=flags, nshards=nsh, shard=s,
                           shard_block=blk) for s in range(nsh)]
+        os.environ.pop("CUSAN_SESSION_EVENT_LIMIT", None)
         runs, n = [], 0
-        for x, y in zip(cuts[:-1], cuts[1:]):
-            for t, se in zip(trs, ses):
-                t.cusan_trace_append_events(ev[x:y])
-                r = se.submit() if mode == "pipelined" else se.check()
-                if r is not None:
-                    runs.append(r.runs)
-                    n += r.n_race_granules
+        try:
+            for x, y in zip(cuts[:-1], cuts[1:]):
+                for t, se in zip(trs, ses):
+                    t.cusan_trace_append_events(ev[x:y])
+                    r = se.submit() if mode == "pipelined" else se.check()
+                    if r is not None:
+                        runs.append(r.runs)
+                        n += r.n_race_granules
+        except cs.CusanError as e:                 # a call or the live ids too large for the lowered limit
+            if mode != "session renumbering" or e.status != -2:
+                raise
+            stats["renumber_limit_too_low"] = stats.get("renumber_limit_too_low", 0) + 1
+            for se in ses:
+                se.close()
+            continue
         for se in ses:
             if mode == "pipelined":
                 r = se.finish()
