@@ -238,7 +238,8 @@ struct cusan_session {
     KeySlots key_slot;
     std::vector<uint32_t> sc;                       // sync clocks, F per key
     std::vector<uint32_t> cur_seg;                  // open segment per fiber
-    pinned_vector<uint32_t> segvc;                  // all segment rows (host copy, uploaded)
+    pinned_vector<uint32_t> segvc;                  // segment rows not uploaded yet: [seg_uploaded, nseg)
+    uint32_t F_used = 1;                            // fibers seen so far: clock columns >= it are all 0
     uint64_t nseg = 0;
     std::vector<SIv> ivs;                           // layout of `shadow`
     uint64_t used = 0;                              // cells of `shadow` in use
@@ -356,11 +357,15 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
         uint32_t* Cf = &s->C[(size_t)f * F];
         const uint32_t ci = (uint32_t)(i - s->delta);       // compact event id (= i before any renumbering)
         c.n_events++;
+        // clock columns of fibers never seen are 0 everywhere: the joins stop at the fibers seen
+        s->F_used = std::max(s->F_used, f + 1);
+        if (e.kind == CUSAN_EV_FORK) s->F_used = std::max(s->F_used, (uint32_t)e.a + 1);
+        const uint32_t FU = s->F_used;
         if (e.kind == CUSAN_EV_FORK) {
             const uint32_t src = (uint32_t)e.a;
             uint32_t* Cs = &s->C[(size_t)src * F];
             Cs[src] = ci + 1;
-            for (uint32_t g = 0; g < F; g++) Cf[g] = std::max(Cf[g], Cs[g]);
+            for (uint32_t g = 0; g < FU; g++) Cf[g] = std::max(Cf[g], Cs[g]);
             s->cur_seg[f] = NO_SEG;
             c.n_fork++;
             continue;
@@ -386,19 +391,19 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
             }
             case CUSAN_EV_RELEASE: {
                 uint32_t* S = s->sync_clock(e.a);
-                for (uint32_t g = 0; g < F; g++) S[g] = std::max(S[g], Cf[g]);
+                for (uint32_t g = 0; g < FU; g++) S[g] = std::max(S[g], Cf[g]);
                 c.n_release++;
                 break;
             }
             case CUSAN_EV_RELEASE_STORE: {
                 uint32_t* S = s->sync_clock(e.a);
-                std::copy(Cf, Cf + F, S);
+                std::copy(Cf, Cf + FU, S);
                 c.n_release_store++;
                 break;
             }
             case CUSAN_EV_ACQUIRE: {
                 uint32_t* S = s->sync_clock(e.a);
-                for (uint32_t g = 0; g < F; g++) Cf[g] = std::max(Cf[g], S[g]);
+                for (uint32_t g = 0; g < FU; g++) Cf[g] = std::max(Cf[g], S[g]);
                 s->cur_seg[f] = NO_SEG;
                 c.n_acquire++;
                 break;
@@ -627,8 +632,9 @@ static int session_plan(cusan_session* s, PendingCall& pc) {
         st = plan_call(s, tr, cp);
         if (!st) {
             build_span_tables(cp.hp, s->max_blocks, pc.tabs);
-            pc.seg_first_word = s->seg_uploaded * s->F;
-            pc.seg_rows.assign(s->segvc.begin() + pc.seg_first_word, s->segvc.begin() + s->nseg * s->F);
+            pc.seg_first_word = s->seg_uploaded * s->F;   // the rows new in this call move to the call
+            pc.seg_rows.swap(s->segvc);
+            s->segvc.clear();
         }
     } catch (const std::bad_alloc&) {
         st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
