@@ -82,6 +82,76 @@ class KeySlots {
     uint32_t n_ = 0;
 };
 
+// A u64 -> V hash map with open addressing (linear probing, backward-shift erase): the lowering
+// looks up stream, request and allocation handles for every recorded call.
+template <class V>
+class FlatMap {
+  public:
+    V* get(uint64_t key) {
+        if (!n_) return nullptr;
+        for (size_t i = slot(key);; i = (i + 1) & (cap_ - 1)) {
+            if (!used_[i]) return nullptr;
+            if (keys_[i] == key) return &vals_[i];
+        }
+    }
+    const V* get(uint64_t key) const { return const_cast<FlatMap*>(this)->get(key); }
+    size_t count(uint64_t key) const { return get(key) ? 1 : 0; }
+    V& operator[](uint64_t key) {
+        if (V* v = get(key)) return *v;
+        if (2 * (n_ + 1) > cap_) grow();
+        size_t i = slot(key);
+        while (used_[i]) i = (i + 1) & (cap_ - 1);
+        used_[i] = 1;
+        keys_[i] = key;
+        vals_[i] = V{};
+        n_++;
+        return vals_[i];
+    }
+    bool erase(uint64_t key) {
+        if (!n_) return false;
+        size_t i = slot(key);
+        for (;; i = (i + 1) & (cap_ - 1)) {
+            if (!used_[i]) return false;
+            if (keys_[i] == key) break;
+        }
+        used_[i] = 0;                                 // backward shift: keep every probe chain intact
+        for (size_t j = (i + 1) & (cap_ - 1); used_[j]; j = (j + 1) & (cap_ - 1)) {
+            const size_t h = slot(keys_[j]);
+            if (((j - h) & (cap_ - 1)) >= ((j - i) & (cap_ - 1))) {
+                keys_[i] = keys_[j];
+                vals_[i] = vals_[j];
+                used_[i] = 1;
+                used_[j] = 0;
+                i = j;
+            }
+        }
+        n_--;
+        return true;
+    }
+
+  private:
+    size_t slot(uint64_t k) const {
+        k ^= k >> 30; k *= 0xBF58476D1CE4E5B9ull; k ^= k >> 27; k *= 0x94D049BB133111EBull; k ^= k >> 31;
+        return (size_t)k & (cap_ - 1);
+    }
+    void grow() {
+        std::vector<uint64_t> k = std::move(keys_);
+        std::vector<V> v = std::move(vals_);
+        std::vector<char> u = std::move(used_);
+        cap_ = cap_ ? 2 * cap_ : 64;
+        keys_.assign(cap_, 0);
+        vals_.assign(cap_, V{});
+        used_.assign(cap_, 0);
+        n_ = 0;
+        for (size_t j = 0; j < u.size(); j++)
+            if (u[j]) (*this)[k[j]] = v[j];
+    }
+    std::vector<uint64_t> keys_;
+    std::vector<V> vals_;
+    std::vector<char> used_;
+    size_t cap_ = 0, n_ = 0;
+};
+
 // Interval-compressed shadow (f3) unless the caller asks for the per-granule dense shadow.
 inline bool compressed_shadow(const cusan_check_opts& o) { return !(o.flags & CUSAN_CHECK_DENSE_SHADOW); }
 // CUSAN_EINVAL for unknown or contradictory flags

@@ -34,21 +34,21 @@ inline uint64_t K_thread(uint64_t t) { return (4ull << 56) | t; }
 
 struct cusan_lowering {
     cusan_trace* trace;
-    std::unordered_map<uint64_t, uint32_t> stream_fiber;   // user stream handle -> fiber
+    FlatMap<uint32_t> stream_fiber;                        // user stream handle -> fiber
     std::vector<uint32_t> streams;                         // S0, then streams (creation order)
     std::vector<uint32_t> blocking;                        // blocking streams (creation order)
     std::vector<char> is_blocking;                         // by fiber
     uint32_t next_fiber = 2;
     std::set<uint32_t> mpi_free;                           // pool of completed request fibers
-    std::unordered_map<uint64_t, uint32_t> req_fiber;
+    FlatMap<uint32_t> req_fiber;                           // MPI request -> its fiber
     struct Alloc {
         uint64_t base, size;
         int kind;
     };
     std::vector<Alloc> allocs;                             // registered allocations, sorted by base
-    std::unordered_map<uint64_t, Alloc> by_base;           // the same, by exact base pointer
-    std::unordered_map<uint64_t, uint32_t> thread_fiber;   // host thread -> fiber (thread 0 -> 0)
-    std::unordered_map<uint64_t, uint32_t> ptds;           // host thread -> per-thread default stream
+    FlatMap<Alloc> by_base;                                // the same, by exact base pointer
+    FlatMap<uint32_t> thread_fiber;                        // host thread -> fiber (thread 0 -> 0)
+    FlatMap<uint32_t> ptds;                                // host thread -> per-thread default stream
     uint64_t thread = 0;                                   // calling host thread
     uint32_t h_fiber = 0;                                  // its fiber (thread_fiber[thread])
     bool per_thread_mode = false;
@@ -76,8 +76,7 @@ struct cusan_lowering {
     const Alloc* find(uint64_t p) const {
         // kernel arguments are nearly always allocation bases: an exact hit is the allocation with
         // the greatest base <= p, so it decides alone
-        const auto hit = by_base.find(p);
-        if (hit != by_base.end()) return hit->second.size ? &hit->second : nullptr;
+        if (const Alloc* hit = by_base.get(p)) return hit->size ? hit : nullptr;
         auto it = std::upper_bound(allocs.begin(), allocs.end(), p,
                                    [](uint64_t x, const Alloc& a) { return x < a.base; });
         if (it == allocs.begin()) return nullptr;
@@ -121,9 +120,8 @@ struct cusan_lowering {
     }
     // the calling thread's per-thread default stream (a blocking stream), created on first use
     int thread_ptds(uint32_t* f) {
-        auto it = ptds.find(thread);
-        if (it != ptds.end()) {
-            *f = it->second;
+        if (const uint32_t* it = ptds.get(thread)) {
+            *f = *it;
             return CUSAN_OK;
         }
         int st = add_stream(f, true);
@@ -144,15 +142,14 @@ struct cusan_lowering {
             return CUSAN_OK;
         }
         if (stream == STREAM_PER_THREAD) return thread_ptds(f);
-        auto it = stream_fiber.find(stream);
-        if (it == stream_fiber.end()) return fail(CUSAN_EINVAL, "unknown stream handle");
-        *f = it->second;
+        const uint32_t* it = stream_fiber.get(stream);
+        if (!it) return fail(CUSAN_EINVAL, "unknown stream handle");
+        *f = *it;
         return CUSAN_OK;
     }
     int thread_fiber_of(uint64_t t, uint32_t* f) {
-        auto it = thread_fiber.find(t);
-        if (it != thread_fiber.end()) {
-            *f = it->second;
+        if (const uint32_t* it = thread_fiber.get(t)) {
+            *f = *it;
             return CUSAN_OK;
         }
         int st = new_fiber(f);
@@ -381,10 +378,9 @@ int cusan_on_mpi_wait(cusan_lowering* l, uint64_t req) {
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
     int st = l->sync(CUSAN_ACQUIRE, l->H(), K_req(req));
     if (st) return st;
-    auto it = l->req_fiber.find(req);
-    if (it != l->req_fiber.end()) {
-        l->mpi_free.insert(it->second);
-        l->req_fiber.erase(it);
+    if (const uint32_t* it = l->req_fiber.get(req)) {
+        l->mpi_free.insert(*it);
+        l->req_fiber.erase(req);
     }
     return CUSAN_OK;
 }
@@ -424,9 +420,9 @@ int cusan_on_thread_create(cusan_lowering* l, uint64_t child) {
 
 int cusan_on_thread_join(cusan_lowering* l, uint64_t child) {
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
-    auto it = l->thread_fiber.find(child);
-    if (it == l->thread_fiber.end()) return CUSAN_OK;
-    int st = l->sync(CUSAN_RELEASE, it->second, K_thread(child));   // the child's end ...
+    const uint32_t* it = l->thread_fiber.get(child);
+    if (!it) return CUSAN_OK;
+    int st = l->sync(CUSAN_RELEASE, *it, K_thread(child));   // the child's end ...
     return st ? st : l->sync(CUSAN_ACQUIRE, l->H(), K_thread(child));   // ... HB the join
 }
 
