@@ -1,5 +1,6 @@
-"""Small workloads for compute-sanitizer runs over the library's kernels (both kernel paths, windows,
-sessions, spill records, the interval-compressed shadow).  Asserts parity with the oracle too."""
+"""Small workloads for compute-sanitizer runs over the library's kernels (both shadow layouts,
+windows, the device planner, plans from clocks, whole-node checks, sessions incl. epoch
+renumbering, spill records).  Asserts parity with the oracle too."""
 import os
 import sys
 
@@ -19,8 +20,12 @@ for c in (1, 3, 5):
     tr = cs.Trace(255)
     cs.Lowering(tr).cusan_lower_program(ops, args)
     ref = oracle.check_events(tr.cusan_trace_read(), 255)
+    DP = cs.CUSAN_CHECK_DEVICE_PLAN
+    os.environ["CUSAN_NODE_SHARE_DEVICES"] = "1"
     for kw in (dict(), dict(window_events=40), dict(window_events=40, flags=cs.CUSAN_CHECK_DENSE_SHADOW),
-               dict(window_events=40, flags=cs.CUSAN_CHECK_INTERVAL_SHADOW), dict(nshards=3, shard=1)):
+               dict(window_events=40, flags=cs.CUSAN_CHECK_INTERVAL_SHADOW), dict(nshards=3, shard=1),
+               dict(flags=DP), dict(window_events=40, flags=DP | cs.CUSAN_CHECK_DENSE_SHADOW),
+               dict(window_events=40, flags=DP, nshards=3, shard=2), dict(window_events=40, ngpus=3)):
         rep = cs.check(tr, **kw)
         if "nshards" not in kw:
             assert rep.n_race_granules == ref["n_race_granules"], (c, kw)
@@ -40,6 +45,20 @@ for _ in range(10):
             n += 1
         ses.close()
         assert total == ref["n_race_granules"], flags
+        os.environ["CUSAN_SESSION_EVENT_LIMIT"] = "80"       # renumber the epochs every call
+        tr = cs.Trace(nf)
+        ses = cs.Session(tr, window_events=7, flags=flags)
+        os.environ.pop("CUSAN_SESSION_EVENT_LIMIT")
+        renum = 0
+        for a, b in ((0, 30), (30, 60), (60, 90), (90, 120)):
+            tr.cusan_trace_append_events(ev[a:b])
+            try:
+                r = ses.check()
+            except cs.CusanError:                           # live ids beyond the lowered limit
+                break
+            renum = r.counters["renumberings"]
+            n += 1
+        ses.close()
         # pipelined calls (submit / finish) and a 2-shard block-cyclic session
         for kw in (dict(), dict(nshards=2, shard=0, shard_block=64), dict(nshards=2, shard=1, shard_block=64)):
             tr = cs.Trace(nf)
