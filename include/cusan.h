@@ -214,8 +214,15 @@ int cusan_plan_describe(const cusan_trace* t, const cusan_check_opts* o, cusan_c
  * processes only its new events) and the shadow layout is stable: cells are updated in place and
  * memory touched for the first time gets cells appended (every device buffer grows inside a
  * reserved virtual range).  Because a call updates the shadow in place it cannot be re-run: a run
- * buffer overflow truncates that call's run list (counts stay exact) and grows the buffer; a
- * read-set heap overflow fails the session (CUSAN_ESTATE afterwards).
+ * buffer overflow truncates that call's run list (counts stay exact) and grows the buffer.
+ * Read-set records are assigned on the host and reclaimed once no interval names them (reused from
+ * the next call on), so the heap holds the live read sets rather than growing per call (counters
+ * heap_live_bytes / heap_bytes).  Traces longer than the 24-bit epoch field: before a call that
+ * would exceed 2^24-2 event ids the session renumbers every id value still in use (live cells, live
+ * records, fiber and sync clocks — ranked, so all later comparisons are unchanged) and reports keep
+ * trace positions (u32); CUSAN_ERANGE only if one call alone, or the live ids, need more than half
+ * the field (counter renumberings).  A call that fails after changing the session's state leaves
+ * it unusable (CUSAN_ESTATE afterwards).
  * Multi-GPU sessions (nshards > 1, one session per rank, each on its own device): the address space
  * is not known in advance, so the granule space is dealt out block-cyclically — granule g belongs
  * to shard (g / shard_block) mod nshards, shard_block a power of two (0 = 2^21 granules = 16 MiB of

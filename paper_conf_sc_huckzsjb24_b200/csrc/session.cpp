@@ -35,8 +35,9 @@ using namespace cusan;
 // interval-compressed shadow (f3) an interval has one cell, so a split piece other than the first
 // gets a new cell copied from it (copy_cells).  In-place updates cannot be re-run: if the run buffer
 // overflows, the call's run list is marked truncated (race-granule counts stay exact) and the buffer
-// grows for later calls; a read-set heap overflow (only possible on the lane-parallel path) fails
-// the session.
+// grows for later calls.  Read-set records are assigned on the host (RecAlloc below: dead ones are
+// reused), and event ids are renumbered when the trace outgrows the 24-bit epoch field
+// (session_renumber).
 // ================================================================================================
 namespace {
 
