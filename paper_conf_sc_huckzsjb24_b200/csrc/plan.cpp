@@ -174,8 +174,17 @@ std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned thread
     const uint32_t F = hp.F;
     const uint64_t n = t.ev.size();
     cusan_counters& c = hp.ctr;
-    constexpr uint32_t NO_SEG = 0xffffffffu, NO_SLOT = 0xffffffffu;
-    std::vector<uint32_t> aux(n);          // per event: key slot (sync) or segment opened (access) or NO_SEG
+    constexpr uint32_t NO_SEG = 0xffffffffu;
+    // The column pass replays only the events that move clock values: forks, syncs and the accesses
+    // that open a segment (their row is the fiber's clock).  A fiber's tick at any other access is
+    // dead: every later read of C_f[f] — a release, a fork from f, a segment row — follows a tick of
+    // its own, so the value is overwritten first.
+    struct Op {
+        uint8_t kind;
+        uint32_t f, aux, tick;             // aux: key slot (sync) / segment (access) / source (fork)
+    };
+    std::vector<Op> ops;
+    ops.reserve(n);
     std::vector<uint32_t> cur_seg(F, NO_SEG);
     KeySlots key_slot;
     hp.nseg = 0;
@@ -186,15 +195,14 @@ std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned thread
         switch (e.kind) {
             case CUSAN_EV_FORK:                    // an event of src's program order; opens a segment on dst
                 cur_seg[f] = NO_SEG;
-                aux[i] = NO_SLOT;
+                ops.push_back({CUSAN_EV_FORK, f, (uint32_t)e.a, (uint32_t)(i + 1)});
                 c.n_fork++;
                 break;
             case CUSAN_EV_ACCESS: {
-                aux[i] = NO_SEG;
                 if (cur_seg[f] == NO_SEG) {
                     if (hp.nseg >= 0x7fffffffu) return {CUSAN_ERANGE, "too many segments"};
                     cur_seg[f] = (uint32_t)hp.nseg++;
-                    aux[i] = cur_seg[f];
+                    ops.push_back({CUSAN_EV_ACCESS, f, cur_seg[f], (uint32_t)(i + 1)});
                 }
                 hp.acc_rec[k] = {pack_epoch(f, (uint32_t)i), cur_seg[f] | ((uint32_t)e.mode << 31)};
                 const uint64_t bytes = 8 * (hp.acc_g1[k] - hp.acc_g0[k]);
@@ -209,7 +217,7 @@ std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned thread
             case CUSAN_EV_RELEASE_STORE:
             case CUSAN_EV_ACQUIRE: {
                 bool fresh;
-                aux[i] = key_slot.get(e.a, &fresh);
+                ops.push_back({e.kind, f, key_slot.get(e.a, &fresh), (uint32_t)(i + 1)});
                 if (e.kind == CUSAN_EV_ACQUIRE) { cur_seg[f] = NO_SEG; c.n_acquire++; }
                 else if (e.kind == CUSAN_EV_RELEASE) c.n_release++;
                 else c.n_release_store++;
@@ -221,14 +229,16 @@ std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned thread
     }
     c.n_segments = hp.nseg;
     if (std::getenv("CUSAN_DEBUG_TIMING"))
-        std::fprintf(stderr, "run_a1: pre-pass %.3f ms\n",
-                     std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count());
+        std::fprintf(stderr, "run_a1: pre-pass %.3f ms (%zu of %llu events replayed)\n",
+                     std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count(),
+                     ops.size(), (unsigned long long)n);
     static const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
     const auto t_pre = std::chrono::steady_clock::now();
     hp.segvc.resize(hp.nseg * F);
     const uint32_t nkeys = key_slot.size();
+    const uint64_t nops = ops.size();
     // columns per thread: multiples of 8, at least 8 (one AVX2 vector of u32)
-    const unsigned T = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>({threads, (F + 7) / 8, n / 4096 + 1}));
+    const unsigned T = (unsigned)std::max<uint64_t>(1, std::min<uint64_t>({threads, (F + 7) / 8, nops / 4096 + 1}));
     parallel_for(T, [&](unsigned th) {
         const uint32_t c0 = (uint32_t)((uint64_t)((F + 7) / 8) * th / T) * 8;
         const uint32_t c1 = std::min<uint32_t>(F, (uint32_t)((uint64_t)((F + 7) / 8) * (th + 1) / T) * 8);
@@ -236,27 +246,27 @@ std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned thread
         const uint32_t G = c1 - c0;
         std::vector<uint32_t> C((size_t)F * G, 0), S((size_t)nkeys * G, 0);
         uint32_t* segvc = hp.segvc.data();
-        for (uint64_t i = 0; i < n; i++) {
-            const cusan_event& e = t.ev[i];
-            const uint32_t f = e.fiber;
+        for (uint64_t q = 0; q < nops; q++) {
+            const Op o = ops[q];
+            const uint32_t f = o.f;
             uint32_t* __restrict__ Cf = &C[(size_t)f * G];
-            if (e.kind == CUSAN_EV_FORK) {         // C_src[src] := i+1; C_dst := C_dst ⊔ C_src
-                const uint32_t src = (uint32_t)e.a;
+            if (o.kind == CUSAN_EV_FORK) {         // C_src[src] := i+1; C_dst := C_dst ⊔ C_src
+                const uint32_t src = o.aux;
                 uint32_t* __restrict__ Cs = &C[(size_t)src * G];
-                if (src >= c0 && src < c1) Cs[src - c0] = (uint32_t)(i + 1);
+                if (src >= c0 && src < c1) Cs[src - c0] = o.tick;
                 if (src != f)
                     for (uint32_t g = 0; g < G; g++) Cf[g] = std::max(Cf[g], Cs[g]);
                 continue;
             }
-            if (f >= c0 && f < c1) Cf[f - c0] = (uint32_t)(i + 1);
-            if (e.kind == CUSAN_EV_ACCESS) {
-                if (aux[i] != NO_SEG) std::copy(Cf, Cf + G, segvc + (size_t)aux[i] * F + c0);
+            if (f >= c0 && f < c1) Cf[f - c0] = o.tick;
+            if (o.kind == CUSAN_EV_ACCESS) {       // a segment opens: its row is C_f
+                std::copy(Cf, Cf + G, segvc + (size_t)o.aux * F + c0);
                 continue;
             }
-            uint32_t* __restrict__ Sk = &S[(size_t)aux[i] * G];
-            if (e.kind == CUSAN_EV_RELEASE)        // SC_k := SC_k ⊔ C_f
+            uint32_t* __restrict__ Sk = &S[(size_t)o.aux * G];
+            if (o.kind == CUSAN_EV_RELEASE)        // SC_k := SC_k ⊔ C_f
                 for (uint32_t g = 0; g < G; g++) Sk[g] = std::max(Sk[g], Cf[g]);
-            else if (e.kind == CUSAN_EV_RELEASE_STORE)   // SC_k := C_f
+            else if (o.kind == CUSAN_EV_RELEASE_STORE)   // SC_k := C_f
                 std::copy(Cf, Cf + G, Sk);
             else                                   // C_f := C_f ⊔ SC_k
                 for (uint32_t g = 0; g < G; g++) Cf[g] = std::max(Cf[g], Sk[g]);

@@ -233,3 +233,71 @@ def test_clocks_image_round_trip_and_validation():
         cs.Clocks.from_bytes(bad)
     with pytest.raises(cs.CusanError):
         cs.Clocks.from_bytes(img[:-4])
+
+
+def _a1_reference(ev, F):
+    """a1 written out per event (DESIGN §2 / SURVEY §8(c) step 2, with PAPER.md:156-173's clock rules):
+    per access its (fiber, id+1) epoch and segment, and one clock row per segment (the accessing
+    fiber's clock at the segment's first access; a segment opens at a fiber's first access after an
+    ACQUIRE or an incoming FORK)."""
+    C = np.zeros((F, F), np.uint32)
+    SC = {}
+    cur = [None] * F
+    rows, recs, g0s, g1s = [], [], [], []
+    for i, e in enumerate(ev):
+        k, f = int(e["kind"]), int(e["fiber"])
+        if k == 4:                                   # FORK(src -> f): an event of src
+            s = int(e["a"])
+            C[s, s] = i + 1
+            C[f] = np.maximum(C[f], C[s])
+            cur[f] = None
+            continue
+        C[f, f] = i + 1
+        if k == 0:
+            if cur[f] is None:
+                cur[f] = len(rows)
+                rows.append(C[f].copy())
+            recs.append(((f << 24) | (i + 1), cur[f] | (int(e["mode"]) << 31)))
+            a, b = int(e["a"]), int(e["b"])
+            g0s.append(a >> 3)
+            g1s.append((a + b + 7) >> 3 if b else a >> 3)
+        elif k == 1:
+            SC[int(e["a"])] = np.maximum(SC.get(int(e["a"]), np.zeros(F, np.uint32)), C[f])
+        elif k == 2:
+            SC[int(e["a"])] = C[f].copy()
+        elif k == 3:
+            C[f] = np.maximum(C[f], SC.get(int(e["a"]), np.zeros(F, np.uint32)))
+            cur[f] = None
+    return rows, recs, g0s, g1s
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_clocks_equal_a1_written_out(seed):
+    """The product's a1 (column-parallel, cusan_clocks_compute) against a1 written out per event:
+    access ranges, epochs, segments and every segment row of the clocks image."""
+    import paper_conf_sc_huckzsjb24_b200 as cs
+    from tracegen import fuzz
+    rng = np.random.default_rng(90 + seed)
+    for t in range(12):
+        nf = int(rng.integers(2, 40))
+        ev = fuzz.random_primitive_trace(rng, int(rng.integers(1, 400)), nf, n_keys=int(rng.integers(1, 6)),
+                                         n_granules=int(rng.integers(1, 300)), unaligned=bool(t % 2))
+        if seed == 3:                                # large enough for the threaded column pass
+            ev = np.concatenate([ev] * 60)
+        tr = cs.Trace(nf)
+        tr.cusan_trace_append_events(ev)
+        img = cs.Clocks.compute(tr).to_bytes()
+        F = int(img[8:12].view(np.uint32)[0])
+        n_acc, nseg = (int(x) for x in img[16:32].view(np.uint64))
+        ctr_bytes = len(img) - (n_acc * 24 + nseg * F * 4) - 40      # the counters struct follows the header
+        p = 40 + ctr_bytes
+        g0 = img[p:p + 8 * n_acc].view(np.uint64); p += 8 * n_acc
+        g1 = img[p:p + 8 * n_acc].view(np.uint64); p += 8 * n_acc
+        rec = img[p:p + 8 * n_acc].view(np.uint32).reshape(-1, 2); p += 8 * n_acc
+        rows = img[p:p + 4 * nseg * F].view(np.uint32).reshape(nseg, F) if nseg else np.zeros((0, F), np.uint32)
+        w_rows, w_recs, w_g0, w_g1 = _a1_reference(ev, F)
+        assert len(w_rows) == nseg and n_acc == len(w_recs)
+        assert [tuple(int(x) for x in r) for r in rec] == w_recs
+        assert list(g0) == w_g0 and list(g1) == w_g1
+        for r, wr in zip(rows, w_rows):
+            assert np.array_equal(r, wr)
