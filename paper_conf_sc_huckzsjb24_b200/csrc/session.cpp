@@ -184,7 +184,9 @@ struct RecAlloc {
     uint64_t hwm = 0;                                       // units ever handed out = heap size needed
     std::vector<std::vector<uint32_t>> free_by_units;       // reusable records by size (units)
     std::vector<std::pair<uint32_t, uint32_t>> pending;     // dead in the current call: (rec, units)
-    std::unordered_map<uint32_t, uint32_t> live;            // allocated: rec -> units
+    std::vector<std::pair<uint32_t, uint32_t>> live;        // allocated: (rec, units)
+    std::vector<uint32_t> stamp;                            // by record unit: last collect naming it
+    uint32_t gen = 0;
     uint64_t live_units = 0;
 
     // a record of `units` units; false if the 24-bit record index is exhausted
@@ -197,7 +199,7 @@ struct RecAlloc {
             *rec = (uint32_t)hwm;
             hwm += units;
         }
-        live.emplace(*rec, units);
+        live.emplace_back(*rec, units);
         live_units += units;
         return true;
     }
@@ -210,16 +212,22 @@ struct RecAlloc {
         pending.clear();
     }
     // after a call's plan: every allocated record the layout no longer names is dead
+    // (mark the named records with this collect's stamp, sweep the live list)
     template <class Layout>
     void collect(const Layout& ivs) {
-        std::unordered_map<uint32_t, char> named;
+        if (stamp.size() < hwm) stamp.resize(hwm, 0);
+        if (++gen == 0) {                                   // stamp wrapped: clear and restart
+            std::fill(stamp.begin(), stamp.end(), 0);
+            gen = 1;
+        }
         for (const auto& v : ivs)
-            if (v.rec != NO_REC) named.emplace(v.rec, 1);
-        for (auto it = live.begin(); it != live.end();) {
-            if (named.count(it->first)) { ++it; continue; }
-            pending.emplace_back(it->first, it->second);
-            live_units -= it->second;
-            it = live.erase(it);
+            if (v.rec != NO_REC) stamp[v.rec] = gen;
+        for (size_t i = 0; i < live.size();) {
+            if (stamp[live[i].first] == gen) { i++; continue; }
+            pending.push_back(live[i]);
+            live_units -= live[i].second;
+            live[i] = live.back();
+            live.pop_back();
         }
     }
 };
@@ -344,6 +352,13 @@ struct CallPlan {
 };
 
 static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
+    static const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
+    const auto t0 = std::chrono::steady_clock::now();
+    auto tick = [&](const char* what) {
+        if (dbg)
+            std::fprintf(stderr, "plan_call: %-10s %8.3f ms\n", what,
+                         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+    };
     const uint32_t F = s->F;
     cusan_counters& c = cp.hp.ctr;
     c = cusan_counters{};
@@ -415,6 +430,7 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
     }
     c.tracked_bytes = cp.tracked;
     c.n_segments = s->nseg;
+    tick("a1");
 
     // ---- a2: refine the layout by the new endpoints -----------------------------------------------
     const uint64_t n_new = cp.g0.size();
@@ -486,6 +502,7 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
         }
     }
     cp.used = used;
+    tick("layout");
     const size_t niv = cp.ivs.size();
     c.n_intervals = niv;
     // new incidences per interval, in trace order
@@ -501,6 +518,7 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
     }
     if (n_inc > 0xffffffffull) return fail(CUSAN_ERANGE, "too many interval incidences");
     c.n_incidences = n_inc;
+    tick("incid cnt");
     cp.inc.resize(n_inc);
     cp.inc_acc.resize(n_inc);
     {
@@ -521,6 +539,7 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
     c.shard_granules = granules;
     c.tracked_bytes_shard = tracked_shard;
 
+    tick("incidences");
     // ---- windows and spans for the new incidences; moves for the untouched intervals ---------------
     const uint64_t W = s->opts.window_events > 0 ? (uint64_t)s->opts.window_events : std::max<uint64_t>(n_new, 1);
     const uint64_t nwin = n_new ? (n_new + W - 1) / W : 0;
@@ -586,7 +605,9 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
     c.n_spans = hp.spans.size();
     c.spill_spans = hp.spill_spans;
     c.spill_heap_bytes = hp.rec_units * REC_WORDS * 4;
+    tick("spans");
     s->recs.collect(cp.ivs);           // records no interval of the new layout names are dead
+    tick("collect");
     c.heap_live_bytes = s->recs.live_units * REC_WORDS * 4;
     c.heap_bytes = s->recs.hwm * REC_WORDS * 4;
     return CUSAN_OK;
