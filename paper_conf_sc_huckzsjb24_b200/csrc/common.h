@@ -29,10 +29,6 @@ struct PinnedAllocator {
     template <class U> PinnedAllocator(const PinnedAllocator<U>&) noexcept {}
     T* allocate(size_t n) { return static_cast<T*>(pinned_alloc(n * sizeof(T))); }
     void deallocate(T* p, size_t) noexcept { pinned_free(p); }
-    // resize() default-initialises (no zero fill: every resized table is written in full before
-    // it is read or uploaded); explicit values construct as usual
-    template <class U> void construct(U* p) noexcept { ::new (static_cast<void*>(p)) U; }
-    template <class U, class... A> void construct(U* p, A&&... a) { ::new (static_cast<void*>(p)) U(std::forward<A>(a)...); }
     template <class U> bool operator==(const PinnedAllocator<U>&) const noexcept { return true; }
     template <class U> bool operator!=(const PinnedAllocator<U>&) const noexcept { return false; }
 };
