@@ -346,16 +346,16 @@ def run_ours(args):
         pkw = dict(window_events=args.window, stream=stream.cuda_stream, flags=flags)
         if world > 1:
             pkw.update(nshards=world, shard=rank)
-        # at least --e2e-steps timed steps and ~2 s of them (short steps are noisy), four warm-up steps
+        # at least --e2e-steps timed steps and ~2 s of them (short steps are noisy), eight warm-up steps
         n = max(1, args.e2e_steps, min(800, int(2.0 / max(1e-5, step_s_hint))))
         h2d = d2h = 0
         barrier()
         torch.cuda.synchronize(dev)
         t0 = None
         kms = []
-        for i, (_tr, r2) in enumerate(cs.pipelined_checks(make_trace, n + 4, device=local, **pkw)):
-            if i < 4:                                # warm-up steps: fill the pipeline
-                if i == 3:
+        for i, (_tr, r2) in enumerate(cs.pipelined_checks(make_trace, n + 8, device=local, **pkw)):
+            if i < 8:                                # warm-up steps: fill the pipeline
+                if i == 7:
                     barrier()
                     t0 = time.perf_counter()
                 continue
@@ -540,9 +540,9 @@ def run_ours(args):
         "e2e": {"value": e2e_value, "unit": "GB/s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "ms_per_step": 1e3 * e2e_step_s, "steps": n_e2e,
                 "kernel_ms_per_step": e2e_kms,
-                "mode": ("pipelined_checks: lowering of step i+3, clocks (a1) of step i+2 and the plan (a2) of step i+1 on "
-                         "host threads overlap the GPU check of step i; pinned host tables uploaded and the report "
-                         "downloaded every step; 4 warm-up steps") if world == 1 else
+                "mode": ("pipelined_checks: lowering (a0), clocks (a1) and plans (a2) of the next steps on host threads "
+                         "(two per stage) overlap the GPU check of step i; pinned host tables uploaded and the report "
+                         "downloaded every step; 8 warm-up steps") if world == 1 else
                         ("sharded, serial: rank 0 lowers + computes clocks, broadcast, every rank plans its shard on its GPU, "
                          "checks, runs gathered to rank 0 (median of 3 steps, phases max over ranks)"),
                 "serial": {"value": e2e_serial, "unit": "GB/s", "ms_per_step": dense_breakdown["total_ms"],

@@ -363,13 +363,15 @@ def check(trace: Trace, workspace: str | None = None, **kw) -> Report:
     return _report(h, kw.get("max_runs", 0))
 
 
-def pipelined_checks(make_trace, steps: int, device: int = 0, **kw):
+def pipelined_checks(make_trace, steps: int, device: int = 0, host_workers: int = 2, **kw):
     """Check `steps` traces one after another with the host and the GPU overlapped, as a four-stage
-    pipeline on separate threads: while the GPU checks trace i (a3-a5), one host thread builds the
-    plan of trace i+1 (a2, on the device planner's own stream or on the host), one computes the
-    clocks of trace i+2 (a1, cusan_clocks_compute) and one builds trace i+3 (`make_trace(i+3)`, e.g.
-    lowering the next batch of recorded calls, a0) — a step costs the slowest stage rather than
-    their sum.  This is how an online checker keeps host and GPU busy.  Every plan's tables are
+    pipeline on separate threads: while the GPU checks trace i (a3-a5), host threads build the plans
+    of the next traces (a2, on the device planner's own stream or on the host), compute their clocks
+    (a1, cusan_clocks_compute) and build the traces after them (`make_trace(j)`, e.g. lowering the
+    next batch of recorded calls, a0) — a step costs the slowest stage rather than their sum.  Each
+    host stage has `host_workers` threads, so consecutive (independent) traces go through a stage at
+    the same time; reports still come back in order, one GPU check after another.  This is how an
+    online checker keeps host and GPU busy.  Every plan's tables are
     uploaded (host -> device) when it is bound, after the previous plan's run completed, and every
     run downloads its report, so each step still pays its own transfers.  All plans share one
     workspace from PyTorch's caching allocator (a plan's shadow and records are scratch for its own
@@ -382,10 +384,11 @@ def pipelined_checks(make_trace, steps: int, device: int = 0, **kw):
     kw["device"] = device
     _default_torch_stream(kw)
     kw.pop("device")
-    depth = 3                                   # steps in flight ahead of the GPU
+    hw = max(1, int(host_workers))
+    depth = 3 * hw                              # steps in flight ahead of the GPU
 
     ws = None
-    with ThreadPoolExecutor(1) as lower_ex, ThreadPoolExecutor(1) as clock_ex, ThreadPoolExecutor(1) as plan_ex:
+    with ThreadPoolExecutor(hw) as lower_ex, ThreadPoolExecutor(hw) as clock_ex, ThreadPoolExecutor(hw) as plan_ex:
         futures = {}
 
         def schedule(j):

@@ -1,0 +1,69 @@
+"""Per-stage times inside pipelined_checks (development aid): lowering (a0), clocks (a1), plan from
+clocks (a2) and the GPU check + report, each measured where it runs (the stages overlap, so the
+step time is bounded by the slowest).
+
+    python tools/pipeline_stages.py --config 5 [--dense]
+"""
+import argparse
+import os
+import statistics
+import sys
+import time
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import paper_conf_sc_huckzsjb24_b200 as cs  # noqa: E402
+from tracegen import configs  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--config", type=int, default=5)
+ap.add_argument("--steps", type=int, default=60)
+ap.add_argument("--dense", action="store_true")
+ap.add_argument("--host-workers", type=int, default=2)
+a = ap.parse_args()
+w = configs.make(a.config, "full")
+ops, args = w.arrays(True)
+T = {"lower": [], "clocks": [], "plan": [], "check": []}
+
+
+def make_trace(_i):
+    t0 = time.perf_counter()
+    t = cs.Trace(255)
+    cs.Lowering(t).cusan_lower_program(ops, args)
+    T["lower"].append(1e3 * (time.perf_counter() - t0))
+    return t
+
+
+orig_compute = cs.Clocks.compute.__func__
+orig_plan = cs.Plan
+
+
+def timed_compute(cls, tr):
+    t0 = time.perf_counter()
+    r = orig_compute(cls, tr)
+    T["clocks"].append(1e3 * (time.perf_counter() - t0))
+    return r
+
+
+class TimedPlan(orig_plan):
+    def __init__(self, *x, **k):
+        t0 = time.perf_counter()
+        super().__init__(*x, **k)
+        T["plan"].append(1e3 * (time.perf_counter() - t0))
+
+
+cs.Clocks.compute = classmethod(timed_compute)
+cs.Plan = TimedPlan
+flags = cs.CUSAN_CHECK_DENSE_SHADOW if a.dense else 0
+t_prev = None
+steps = []
+for i, (_t, rep) in enumerate(cs.pipelined_checks(make_trace, a.steps, window_events=4096, flags=flags,
+                                                          host_workers=a.host_workers)):
+    now = time.perf_counter()
+    if t_prev is not None and i >= 5:
+        steps.append(1e3 * (now - t_prev))
+        T["check"].append(rep.counters["run_ms"])
+    t_prev = now
+med = {k: round(statistics.median(v[5:] if len(v) > 10 else v), 3) for k, v in T.items()}
+print(f"config {a.config} {'dense' if a.dense else 'compressed'} ({a.host_workers} host workers per stage): step "
+      f"{sum(steps) / len(steps):.3f} ms (mean over {len(steps)} steps); stage medians {med}")
