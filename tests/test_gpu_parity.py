@@ -238,9 +238,10 @@ def test_full_size_configs_exact(c, twin):
         assert rep.counters["tracked_bytes"] == int(g["tracked_bytes"])
         assert_equal(rep, ref)
     if c in (4, 5):
-        parts = [cs.check(tr, window_events=4096, nshards=8, shard=k) for k in range(8)]
-        merged = cs.report_merge(np.concatenate([p.runs for p in parts]), sum(p.n_race_granules for p in parts))
-        assert_equal(merged, ref)
+        for flags in (0, cs.CUSAN_CHECK_DENSE_SHADOW):
+            parts = [cs.check(tr, window_events=4096, nshards=8, shard=k, flags=flags) for k in range(8)]
+            merged = cs.report_merge(np.concatenate([p.runs for p in parts]), sum(p.n_race_granules for p in parts))
+            assert_equal(merged, ref)
 
 
 def test_torch_workspace_and_stream():
@@ -391,11 +392,13 @@ def test_pipelined_checks_match_the_oracle_per_step():
         tr.cusan_trace_append_events(traces[i][0])
         return tr
 
-    n = 0
-    for i, (tr, rep) in enumerate(cs.pipelined_checks(make, len(traces), window_events=3)):
-        assert_equal(rep, oracle.check_events(traces[i][0], traces[i][1], threads=2))
-        n += 1
-    assert n == len(traces)
+    for workers in (1, 2, 4):                  # host stages with several threads: reports still in order
+        n = 0
+        for i, (tr, rep) in enumerate(cs.pipelined_checks(make, len(traces), window_events=3,
+                                                          host_workers=workers)):
+            assert_equal(rep, oracle.check_events(traces[i][0], traces[i][1], threads=2))
+            n += 1
+        assert n == len(traces)
 
 
 def test_c_example_fig6a():
