@@ -141,3 +141,37 @@ def test_plan_from_clocks_equals_plan_from_trace(c):
     assert h_inc.tobytes() == d_inc.tobytes() and h_sp.tobytes() == d_sp.tobytes()
     with pytest.raises(cs.CusanError):
         cs.Plan(tr, flags=cs.CUSAN_CHECK_HOST_PLAN | cs.CUSAN_CHECK_DEVICE_PLAN)
+
+
+def test_device_planner_large_random_trace():
+    """A 2.5 M-event trace of ~1.5 M small random accesses (hundreds of thousands of elementary
+    intervals, grid-stride loops and multi-pass sorts in the device planner): device tables =
+    host tables byte for byte, windowed and sharded; the report matches the oracle on sampled
+    granules (every run edge and random interior granules)."""
+    import brute
+    from tracegen.program import EVENT_DTYPE
+    rng = np.random.default_rng(2500)
+    n = 2_500_000
+    ev = np.zeros(n, EVENT_DTYPE)
+    kind = rng.choice([0, 1, 2, 3, 4], size=n, p=[0.6, 0.12, 0.04, 0.16, 0.08])
+    ev["kind"] = kind
+    ev["fiber"] = rng.integers(0, 8, n)
+    acc = kind == 0
+    ev["mode"][acc] = rng.random(int(acc.sum())) < 0.3
+    ev["a"][acc] = (1 << 32) + 8 * rng.integers(0, 1 << 24, int(acc.sum()))          # 128 MiB region
+    ev["b"][acc] = 8 * rng.integers(1, 512, int(acc.sum()))
+    syn = (kind >= 1) & (kind <= 3)
+    ev["a"][syn] = rng.integers(0, 16, int(syn.sum()))
+    fk = kind == 4
+    ev["a"][fk] = rng.integers(0, 8, int(fk.sum()))
+    tr = cs.Trace(8)
+    tr.cusan_trace_append_events(ev)
+    rep = assert_same_plan(tr, window_events=200_000)
+    assert rep.counters["n_intervals"] > 100_000
+    assert_same_plan(tr, window_events=200_000, nshards=3, shard=1, flags=cs.CUSAN_CHECK_DENSE_SHADOW)
+    g = (ev["a"][acc] >> np.uint64(3)).astype(np.uint64)
+    sample = np.unique(np.concatenate([g[rng.integers(0, len(g), 3000)],
+                                       rep.runs["g_begin"][:2000], rep.runs["g_end"][:2000] - np.uint64(1)]))
+    ref = oracle.check_events(ev, 8, sample=sample)
+    sset = set(int(x) for x in sample)
+    assert set(brute.runs_to_triples_in(rep.runs, sset)) == brute.runs_to_triples(ref["runs"])
