@@ -233,7 +233,8 @@ def test_full_size_configs_exact(c, twin):
     assert (ref["n_race_granules"] > 0) == (twin == "racy")
     import torch
     s = torch.cuda.Stream()
-    for flags in (cs.CUSAN_CHECK_DENSE_SHADOW, 0):      # both bench lines: dense, compressed
+    for flags in (cs.CUSAN_CHECK_DENSE_SHADOW, 0,       # both bench lines: dense, compressed
+                  cs.CUSAN_CHECK_DEVICE_PLAN | cs.CUSAN_CHECK_DENSE_SHADOW, cs.CUSAN_CHECK_HOST_PLAN):
         rep = cs.check(tr, window_events=4096, workspace="torch", stream=s.cuda_stream, flags=flags)
         assert rep.counters["tracked_bytes"] == int(g["tracked_bytes"])
         assert_equal(rep, ref)
