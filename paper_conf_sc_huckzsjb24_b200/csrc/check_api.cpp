@@ -154,6 +154,17 @@ struct cusan_plan {
 };
 
 static int plan_bind(cusan_plan* p, char* ws, uint64_t bytes);
+static int plan_device_setup(cusan_plan* p);
+// plan_device_setup with host allocation failures turned into a status (nothing throws through the C ABI)
+static int guarded_setup(cusan_plan* p) {
+    try {
+        return plan_device_setup(p);
+    } catch (const std::bad_alloc&) {
+        return fail(CUSAN_ENOMEM, "host memory exhausted while preparing the plan");
+    } catch (const std::exception& e) {
+        return fail(CUSAN_ESTATE, std::string("internal error while preparing the plan: ") + e.what());
+    }
+}
 
 // Traces with at least this many accesses build their a2 tables on the device (cusan.h)
 static uint64_t device_plan_min_accesses() {
@@ -573,7 +584,7 @@ int cusan_plan_create(const cusan_trace* t, const cusan_check_opts* o, cusan_pla
     } catch (const std::bad_alloc&) {
         st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
     }
-    if (!st) st = plan_device_setup(p);
+    if (!st) st = guarded_setup(p);
     if (st) {
         delete p;
         return st;
@@ -713,7 +724,7 @@ int cusan_plan_create_from_clocks(const cusan_clocks* c, const cusan_check_opts*
     } catch (const std::bad_alloc&) {
         st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
     }
-    if (!st) st = plan_device_setup(p);
+    if (!st) st = guarded_setup(p);
     if (st) {
         delete p;
         return st;
@@ -747,7 +758,7 @@ int cusan_plan_bind_workspace(cusan_plan* p, void* workspace, uint64_t bytes) {
     return plan_bind(p, (char*)workspace, bytes);
 }
 
-int cusan_plan_run(cusan_plan* p, cusan_report** out) {
+static int cusan_plan_run_impl(cusan_plan* p, cusan_report** out) {
     if (!p || !out) return fail(CUSAN_EINVAL, "null argument");
     *out = nullptr;
     if (!p->bound) return fail(CUSAN_ESTATE, "plan has no workspace: call cusan_plan_bind_workspace");
@@ -910,10 +921,15 @@ static int check_node(const cusan_trace* t, const cusan_check_opts* o, cusan_rep
             so.shard = d;
             so.device = (o->device + d) % ndev;
             cusan_plan* p = nullptr;
-            int st = cusan_plan_create_from_clocks(clocks, &so, &p);
-            if (!st) {
-                st = cusan_plan_run(p, &parts[d]);
-                cusan_plan_destroy(p);
+            int st;
+            try {
+                st = cusan_plan_create_from_clocks(clocks, &so, &p);
+                if (!st) {
+                    st = cusan_plan_run(p, &parts[d]);
+                    cusan_plan_destroy(p);
+                }
+            } catch (const std::exception& e) {            // a thread must not end in an exception
+                st = fail(CUSAN_ENOMEM, std::string("shard thread: ") + e.what());
             }
             status[d] = st;
             if (st) errors[d] = cusan_last_error();
@@ -973,6 +989,17 @@ int cusan_check(const cusan_trace* t, const cusan_check_opts* o, cusan_report** 
     st = cusan_plan_run(p, out);
     cusan_plan_destroy(p);
     return st;
+}
+
+
+int cusan_plan_run(cusan_plan* p, cusan_report** out) {
+    try {
+        return cusan_plan_run_impl(p, out);
+    } catch (const std::bad_alloc&) {
+        return fail(CUSAN_ENOMEM, "host memory exhausted in cusan_plan_run");
+    } catch (const std::exception& e) {
+        return fail(CUSAN_ESTATE, std::string("internal error in cusan_plan_run: ") + e.what());
+    }
 }
 
 }  // extern "C"

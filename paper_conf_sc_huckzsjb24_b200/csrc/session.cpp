@@ -947,7 +947,7 @@ int cusan_session_create(const cusan_trace* t, const cusan_check_opts* o, cusan_
     return CUSAN_OK;
 }
 
-int cusan_session_submit(cusan_session* s, cusan_report** prev) {
+static int cusan_session_submit_impl(cusan_session* s, cusan_report** prev) {
     if (!s || !prev) return fail(CUSAN_EINVAL, "null argument");
     *prev = nullptr;
     if (s->broken) return fail(CUSAN_ESTATE, "an earlier call failed after changing the session's state");
@@ -965,7 +965,11 @@ int cusan_session_submit(cusan_session* s, cusan_report** prev) {
                 return st;
             }
         }
-        st = session_renumber(s);
+        try {
+            st = session_renumber(s);
+        } catch (const std::bad_alloc&) {
+            st = fail(CUSAN_ENOMEM, "host memory exhausted while renumbering the session's event ids");
+        }
         if (st) {
             s->broken = true;
             return st;
@@ -988,7 +992,7 @@ int cusan_session_submit(cusan_session* s, cusan_report** prev) {
     return CUSAN_OK;
 }
 
-int cusan_session_finish(cusan_session* s, cusan_report** out) {
+static int cusan_session_finish_impl(cusan_session* s, cusan_report** out) {
     if (!s || !out) return fail(CUSAN_EINVAL, "null argument");
     *out = nullptr;
     if (!s->pending) return CUSAN_OK;
@@ -1012,6 +1016,28 @@ int cusan_session_destroy(cusan_session* s) {
     if (s->stream || s->pending) cudaStreamSynchronize(s->stream);
     delete s;
     return CUSAN_OK;
+}
+
+
+int cusan_session_submit(cusan_session* s, cusan_report** prev) {
+    try {
+        return cusan_session_submit_impl(s, prev);
+    } catch (const std::bad_alloc&) {
+        return fail(CUSAN_ENOMEM, "host memory exhausted in cusan_session_submit");
+    } catch (const std::exception& e) {
+        return fail(CUSAN_ESTATE, std::string("internal error in cusan_session_submit: ") + e.what());
+    }
+}
+
+
+int cusan_session_finish(cusan_session* s, cusan_report** out) {
+    try {
+        return cusan_session_finish_impl(s, out);
+    } catch (const std::bad_alloc&) {
+        return fail(CUSAN_ENOMEM, "host memory exhausted in cusan_session_finish");
+    } catch (const std::exception& e) {
+        return fail(CUSAN_ESTATE, std::string("internal error in cusan_session_finish: ") + e.what());
+    }
 }
 
 }  // extern "C"
