@@ -353,7 +353,8 @@ def run_ours(args):
         torch.cuda.synchronize(dev)
         t0 = None
         kms = []
-        for i, (_tr, r2) in enumerate(cs.pipelined_checks(make_trace, n + 8, device=local, **pkw)):
+        # make_trace lowers a fresh copy of the recorded program per step: safe on two threads
+        for i, (_tr, r2) in enumerate(cs.pipelined_checks(make_trace, n + 8, device=local, lower_workers=2, **pkw)):
             if i < 8:                                # warm-up steps: fill the pipeline
                 if i == 7:
                     barrier()
@@ -541,7 +542,7 @@ def run_ours(args):
                 "ms_per_step": 1e3 * e2e_step_s, "steps": n_e2e,
                 "kernel_ms_per_step": e2e_kms,
                 "mode": ("pipelined_checks: lowering (a0), clocks (a1) and plans (a2) of the next steps on host threads "
-                         "(two per stage) overlap the GPU check of step i; pinned host tables uploaded and the report "
+                         "(two per stage; each step lowers its own copy of the program) overlap the GPU check of step i; pinned host tables uploaded and the report "
                          "downloaded every step; 8 warm-up steps") if world == 1 else
                         ("sharded, serial: rank 0 lowers + computes clocks, broadcast, every rank plans its shard on its GPU, "
                          "checks, runs gathered to rank 0 (median of 3 steps, phases max over ranks)"),

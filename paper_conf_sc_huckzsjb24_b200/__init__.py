@@ -363,7 +363,8 @@ def check(trace: Trace, workspace: str | None = None, **kw) -> Report:
     return _report(h, kw.get("max_runs", 0))
 
 
-def pipelined_checks(make_trace, steps: int, device: int = 0, host_workers: int = 2, **kw):
+def pipelined_checks(make_trace, steps: int, device: int = 0, host_workers: int = 2, lower_workers: int = 1,
+                     **kw):
     """Check `steps` traces one after another with the host and the GPU overlapped, as a four-stage
     pipeline on separate threads: while the GPU checks trace i (a3-a5), host threads build the plans
     of the next traces (a2, on the device planner's own stream or on the host), compute their clocks
@@ -384,11 +385,11 @@ def pipelined_checks(make_trace, steps: int, device: int = 0, host_workers: int 
     kw["device"] = device
     _default_torch_stream(kw)
     kw.pop("device")
-    hw = max(1, int(host_workers))
-    depth = 3 * hw                              # steps in flight ahead of the GPU
+    hw, lw = max(1, int(host_workers)), max(1, int(lower_workers))
+    depth = 3 * max(hw, lw)                     # steps in flight ahead of the GPU
 
     ws = None
-    with ThreadPoolExecutor(hw) as lower_ex, ThreadPoolExecutor(hw) as clock_ex, ThreadPoolExecutor(hw) as plan_ex:
+    with ThreadPoolExecutor(lw) as lower_ex, ThreadPoolExecutor(hw) as clock_ex, ThreadPoolExecutor(hw) as plan_ex:
         futures = {}
 
         def schedule(j):

@@ -169,11 +169,24 @@ static void radix_sort_pairs(std::vector<uint64_t>& key, std::vector<uint32_t>& 
 //      evolves independently of the other columns — each primitive is an element-wise max, copy or
 //      tick — so the columns are split among threads, each replaying the whole trace on its columns
 //      and writing them into the segment rows.  Same rows as one pass over whole clocks.
-std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned threads) {
+std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned threads, bool fill_accesses) {
     const auto t_start = std::chrono::steady_clock::now();
-    const uint32_t F = hp.F;
     const uint64_t n = t.ev.size();
     cusan_counters& c = hp.ctr;
+    if (fill_accesses) {                   // one pass: the accesses, the clock width and the counters too
+        c = cusan_counters{};
+        c.n_events = n;
+        hp.acc_g0.clear();
+        hp.acc_g1.clear();
+        hp.acc_rec.clear();
+        hp.acc_event.clear();
+        hp.acc_g0.reserve(n);
+        hp.acc_g1.reserve(n);
+        hp.acc_rec.reserve(n);
+        hp.F = 1;
+    }
+    uint32_t F = fill_accesses ? CUSAN_MAX_FIBERS + 1 : hp.F;   // (cur_seg size; the width is set below)
+    uint32_t f_max = 1;
     constexpr uint32_t NO_SEG = 0xffffffffu;
     // The column pass replays only the events that move clock values: forks, syncs and the accesses
     // that open a segment (their row is the fiber's clock).  A fiber's tick at any other access is
@@ -192,10 +205,12 @@ std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned thread
     for (uint64_t i = 0; i < n; i++) {
         const cusan_event& e = t.ev[i];
         const uint32_t f = e.fiber;
+        f_max = std::max(f_max, f + 1);
         switch (e.kind) {
             case CUSAN_EV_FORK:                    // an event of src's program order; opens a segment on dst
                 cur_seg[f] = NO_SEG;
                 ops.push_back({CUSAN_EV_FORK, f, (uint32_t)e.a, (uint32_t)(i + 1)});
+                f_max = std::max(f_max, (uint32_t)e.a + 1);
                 c.n_fork++;
                 break;
             case CUSAN_EV_ACCESS: {
@@ -204,7 +219,13 @@ std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned thread
                     cur_seg[f] = (uint32_t)hp.nseg++;
                     ops.push_back({CUSAN_EV_ACCESS, f, cur_seg[f], (uint32_t)(i + 1)});
                 }
-                hp.acc_rec[k] = {pack_epoch(f, (uint32_t)i), cur_seg[f] | ((uint32_t)e.mode << 31)};
+                if (fill_accesses) {
+                    hp.acc_g0.push_back(e.a >> 3);
+                    hp.acc_g1.push_back(e.b ? (e.a + e.b + 7) >> 3 : e.a >> 3);
+                    hp.acc_rec.push_back({pack_epoch(f, (uint32_t)i), cur_seg[f] | ((uint32_t)e.mode << 31)});
+                } else {
+                    hp.acc_rec[k] = {pack_epoch(f, (uint32_t)i), cur_seg[f] | ((uint32_t)e.mode << 31)};
+                }
                 const uint64_t bytes = 8 * (hp.acc_g1[k] - hp.acc_g0[k]);
                 k++;
                 c.n_access++;
@@ -228,6 +249,10 @@ std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned thread
         }
     }
     c.n_segments = hp.nseg;
+    if (fill_accesses) {
+        hp.F = F = f_max;
+        c.n_fibers = F;
+    }
     if (std::getenv("CUSAN_DEBUG_TIMING"))
         std::fprintf(stderr, "run_a1: pre-pass %.3f ms (%zu of %llu events replayed)\n",
                      std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count(),
@@ -316,7 +341,6 @@ static void prepare_accesses(const Trace& t, HostPlan& hp) {
 int compute_clocks(const Trace& t, HostPlan& hp) {
     if (t.ev.size() > CUSAN_MAX_EVENTS)
         return fail(CUSAN_ERANGE, "a one-shot check takes at most 2^24-2 events (sessions renumber longer traces)");
-    prepare_accesses(t, hp);
     unsigned hw = std::max(1u, std::thread::hardware_concurrency());
     cpu_set_t set;
     if (sched_getaffinity(0, sizeof(set), &set) == 0) hw = std::max(1, CPU_COUNT(&set));
@@ -324,8 +348,8 @@ int compute_clocks(const Trace& t, HostPlan& hp) {
         const long v = std::strtol(e, nullptr, 10);
         if (v > 0) hw = (unsigned)std::min<long>(v, 256) + 1;
     }
-    const unsigned T = (uint64_t)t.ev.size() * hp.F < (1u << 21) ? 1 : std::max(1u, std::min(hw > 1 ? hw - 1 : 1, 32u));
-    const std::pair<int, std::string> st = run_a1(t, hp, T);
+    const unsigned T = (uint64_t)t.ev.size() < (1u << 15) ? 1 : std::max(1u, std::min(hw > 1 ? hw - 1 : 1, 32u));
+    const std::pair<int, std::string> st = run_a1(t, hp, T, true);
     return st.first ? fail(st.first, st.second) : CUSAN_OK;
 }
 
@@ -355,18 +379,18 @@ int build_host_plan(const Trace* tp, const cusan_check_opts& o, HostPlan& hp, ui
             std::fprintf(stderr, "build_host_plan: %-12s %8.3f ms\n", what,
                          std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
     };
-    if (tp) prepare_accesses(*tp, hp);        // (no trace: hp holds the accesses and a1's products)
-    const uint32_t F = hp.F;
+    // (no trace: hp holds the accesses and a1's products; a1 only: one fused pass below)
+    if (tp && !a1_only) prepare_accesses(*tp, hp);
     const uint64_t n_acc = hp.acc_g0.size();
     cusan_counters& c = hp.ctr;
     // ---------------------------------------------------------------- a1: clocks and segments --
     // Runs on its own thread while a2 builds the intervals (a2 needs a1's records only to fill the
     // incidence table at the end).  Errors come back as (status, message).
-    const unsigned a1_threads = plan_threads(hp.ctr.n_events * F / 64);
+    const unsigned a1_threads = plan_threads(tp ? (uint64_t)tp->ev.size() : 0);
     auto a1 = [&]() -> std::pair<int, std::string> {
         if (!tp) return {CUSAN_OK, ""};
         const auto a1_t0 = std::chrono::steady_clock::now();
-        std::pair<int, std::string> st = run_a1(*tp, hp, a1_threads);
+        std::pair<int, std::string> st = run_a1(*tp, hp, a1_threads, a1_only);
         tick("a1 (thread)");
         if (dbg)
             std::fprintf(stderr, "build_host_plan: a1 alone     %8.3f ms (%llu segments, %u threads)\n",

@@ -396,7 +396,7 @@ def test_pipelined_checks_match_the_oracle_per_step():
     for workers in (1, 2, 4):                  # host stages with several threads: reports still in order
         n = 0
         for i, (tr, rep) in enumerate(cs.pipelined_checks(make, len(traces), window_events=3,
-                                                          host_workers=workers)):
+                                                          host_workers=workers, lower_workers=workers)):
             assert_equal(rep, oracle.check_events(traces[i][0], traces[i][1], threads=2))
             n += 1
         assert n == len(traces)

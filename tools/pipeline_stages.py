@@ -58,7 +58,7 @@ flags = cs.CUSAN_CHECK_DENSE_SHADOW if a.dense else 0
 t_prev = None
 steps = []
 for i, (_t, rep) in enumerate(cs.pipelined_checks(make_trace, a.steps, window_events=4096, flags=flags,
-                                                          host_workers=a.host_workers)):
+                                                          host_workers=a.host_workers, lower_workers=a.host_workers)):
     now = time.perf_counter()
     if t_prev is not None and i >= 5:
         steps.append(1e3 * (now - t_prev))
