@@ -175,3 +175,22 @@ def test_device_planner_large_random_trace():
     ref = oracle.check_events(ev, 8, sample=sample)
     sset = set(int(x) for x in sample)
     assert set(brute.runs_to_triples_in(rep.runs, sset)) == brute.runs_to_triples(ref["runs"])
+
+
+def test_plans_from_clocks_edge_cases():
+    """Clocks of an empty trace, of a trace without accesses and of one with only empty accesses
+    plan and check to an empty report (host and device planners); a corrupt image is rejected."""
+    for rows in ([], [(cs.CUSAN_RELEASE, 0, 5)], None):
+        t = cs.Trace(4)
+        if rows is None:
+            t.cusan_trace_append_access(0, 1, 0x1000, 0)
+            t.cusan_trace_append_access(1, 1, 0x1000, 0)
+        else:
+            for k, f, key in rows:
+                t.cusan_trace_append_sync(k, f, key)
+        ck = cs.Clocks.from_bytes(cs.Clocks.compute(t).to_bytes())
+        for flags in (0, HOST, DEVICE):
+            p = cs.Plan(ck, window_events=1, flags=flags)
+            r = p.run()
+            p.close()
+            assert r.n_race_granules == 0 and r.n_runs == 0
