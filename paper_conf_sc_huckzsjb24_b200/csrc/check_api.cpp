@@ -6,6 +6,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <functional>
 #include <map>
 #include <mutex>
 #include <new>
@@ -140,6 +141,7 @@ struct cusan_plan {
     RunMerge merge;                         // a4 scratch (device run merge)
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
     bool dev_planned = false;               // a2 ran on the device: tables live in dscr
+    const Trace* a1_trace = nullptr;        // a1 still to run (overlapping the device planner)
     DevScratch* dscr = nullptr;
     uint64_t n_ds = 0;                      // span table records (device-planned)
 
@@ -412,8 +414,17 @@ static int plan_device_setup(cusan_plan* p) {
         p->dscr = plan_dev_acquire(p->device);
         if (!p->dscr) return fail(CUSAN_ENOMEM, "cannot create the device planning scratch");
         DevPlanOut dp;
-        int e = device_plan_a2(hp, span_args(p->max_blocks), *p->dscr, dp);
-        if (e == CUSAN_ERANGE) {       // beyond the device planner's 2^31 items: plan a2 on the host
+        std::function<int()> host_a1;
+        if (p->a1_trace)
+            host_a1 = [p, &hp] {
+                const std::pair<int, std::string> r =
+                    run_a1(*p->a1_trace, hp, a1_threads_for(p->a1_trace->ev.size()), false);
+                if (r.first) return fail(r.first, r.second);
+                p->a1_trace = nullptr;                   // a1 done
+                return CUSAN_OK;
+            };
+        int e = device_plan_a2(hp, span_args(p->max_blocks), *p->dscr, dp, host_a1);
+        if (e == CUSAN_ERANGE && !p->a1_trace) {   // beyond the device planner's 2^31 items: a2 on the host
             plan_dev_release(p->dscr);
             p->dscr = nullptr;
             p->dev_planned = false;
@@ -580,7 +591,12 @@ int cusan_plan_create(const cusan_trace* t, const cusan_check_opts* o, cusan_pla
                      ((o->flags & CUSAN_CHECK_DEVICE_PLAN) || n_acc >= dev_min);
     int st;
     try {
-        st = build_host_plan(&t->t, *o, p->hp, 0, 0, p->dev_planned);
+        if (p->dev_planned) {          // a1 runs inside the device planner, overlapping its first phase
+            st = prepare_plan_accesses(t->t, *o, p->hp);
+            p->a1_trace = &t->t;
+        } else {
+            st = build_host_plan(&t->t, *o, p->hp);
+        }
     } catch (const std::bad_alloc&) {
         st = fail(CUSAN_ENOMEM, "host memory exhausted while planning");
     }

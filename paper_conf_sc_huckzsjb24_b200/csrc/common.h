@@ -243,6 +243,11 @@ int build_host_plan(const Trace* t, const cusan_check_opts& o, HostPlan& hp, uin
 
 // a1 of a whole trace for a clocks object (cusan_clocks_compute), with the node's cores
 int compute_clocks(const Trace& t, HostPlan& hp);
+// a1 itself (plan.cpp): with fill_accesses the accesses' ranges and the counters too (one pass),
+// else hp holds the ranges already (prepare_plan_accesses)
+std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned threads, bool fill_accesses);
+int prepare_plan_accesses(const Trace& t, const cusan_check_opts& o, HostPlan& hp);
+unsigned a1_threads_for(uint64_t n_events);
 
 // canonical merge of runs (sort by (later, earlier, g_begin), merge abutting) — a4 host part
 void canonicalize_runs(std::vector<cusan_race_run>& runs);

@@ -336,6 +336,22 @@ static void prepare_accesses(const Trace& t, HostPlan& hp) {
     }
 }
 
+// The first part of a device-planned plan: options checked, the accesses' granule ranges; a1 follows
+// (run_a1) while the device builds the intervals from the ranges.
+int prepare_plan_accesses(const Trace& t, const cusan_check_opts& o, HostPlan& hp) {
+    if (o.nshards < 1 || o.shard < 0 || o.shard >= o.nshards)
+        return fail(CUSAN_EINVAL, "need 0 <= shard < nshards");
+    if (o.window_events < 0) return fail(CUSAN_EINVAL, "window_events must be >= 0");
+    if (int st = check_flags(o)) return st;
+    if (t.ev.size() > CUSAN_MAX_EVENTS)
+        return fail(CUSAN_ERANGE, "a one-shot check takes at most 2^24-2 events (sessions renumber longer traces)");
+    hp.opts = o;
+    prepare_accesses(t, hp);
+    return CUSAN_OK;
+}
+
+unsigned a1_threads_for(uint64_t n_events) { return plan_threads(n_events); }
+
 // a1 alone for a clocks object (cusan_clocks_compute): every core of the node — on a multi-GPU
 // node one rank computes the clocks while the others wait for the broadcast.
 int compute_clocks(const Trace& t, HostPlan& hp) {

@@ -28,6 +28,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <functional>
 #include <mutex>
 #include <new>
 
@@ -599,7 +600,8 @@ static int grow(char** p, uint64_t* cap, uint64_t need) {
     return CUSAN_OK;
 }
 
-int device_plan_a2(const HostPlan& hp, const DevPlanArgs& A, DevScratch& S, DevPlanOut& out) {
+int device_plan_a2(HostPlan& hp, const DevPlanArgs& A, DevScratch& S, DevPlanOut& out,
+                   const std::function<int()>& host_a1) {
     cudaStream_t st = S.stream;
     const uint64_t n = hp.acc_g0.size();
     static const bool dbg = std::getenv("CUSAN_DEBUG_TIMING") != nullptr;
@@ -622,7 +624,7 @@ int device_plan_a2(const HostPlan& hp, const DevPlanArgs& A, DevScratch& S, DevP
             gmax = std::max(gmax, hp.acc_g1[k]);
             nonempty++;
         }
-    if (!nonempty) return CUSAN_OK;              // nothing covered: no intervals, no windows
+    if (!nonempty) return host_a1 ? host_a1() : CUSAN_OK;   // nothing covered: no intervals, no windows
     const uint64_t sent = gmax - gmin + 1;
     const int kbits = bitlen(sent);
     const uint64_t n2 = 2 * n;
@@ -677,7 +679,6 @@ int device_plan_a2(const HostPlan& hp, const DevPlanArgs& A, DevScratch& S, DevP
 
     CK(cudaMemcpyAsync(P1.g0, hp.acc_g0.data(), n * 8, cudaMemcpyHostToDevice, st));
     CK(cudaMemcpyAsync(P1.g1, hp.acc_g1.data(), n * 8, cudaMemcpyHostToDevice, st));
-    CK(cudaMemcpyAsync(P1.rec, hp.acc_rec.data(), n * sizeof(AccRec), cudaMemcpyHostToDevice, st));
     CK(cudaMemsetAsync(P1.hdr, 0, H_COUNT * sizeof(unsigned long long), st));
     CK(cudaMemsetAsync(P1.diff, 0, (n2 + 1) * sizeof(int), st));
     out.h2d_bytes = n * (16 + sizeof(AccRec));
@@ -702,6 +703,15 @@ int device_plan_a2(const HostPlan& hp, const DevPlanArgs& A, DevScratch& S, DevP
     k_hdr1<<<1, 1, 0, st>>>(n, n2, P1.ilen, P1.idense, P1.icov, P1.ivid, P1.np, P1.poff, P1.hdr);
     CK(cudaGetLastError());
     CK(cudaMemcpyAsync(hh, P1.hdr, H_COUNT * sizeof(unsigned long long), cudaMemcpyDeviceToHost, st));
+    if (host_a1) {                     // a1 on the host while the device builds the intervals (phase 1
+        const int e = host_a1();       // needs only the access ranges; the records go up afterwards)
+        if (e) {
+            cudaStreamSynchronize(st);
+            return e;
+        }
+        tick("host a1");
+    }
+    CK(cudaMemcpyAsync(P1.rec, hp.acc_rec.data(), n * sizeof(AccRec), cudaMemcpyHostToDevice, st));
     CK(cudaStreamSynchronize(st));                             // sync 1: sizes of the pair / span buffers
     tick("sync 1");
     out.launches += 8;

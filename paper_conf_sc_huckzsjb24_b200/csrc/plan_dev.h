@@ -3,6 +3,7 @@
 
 #include <cuda_runtime.h>
 
+#include <functional>
 #include <vector>
 
 #include "kernel.cuh"
@@ -41,8 +42,11 @@ struct DevPlanOut {
     uint64_t h2d_bytes = 0, launches = 0;
 };
 
-// a2 for a plan whose a1 (hp.acc_*, hp.segvc, counters) is done; runs on S.stream and waits for it.
-int device_plan_a2(const HostPlan& hp, const DevPlanArgs& args, DevScratch& S, DevPlanOut& out);
+// a2 on S.stream (waits for it) from the accesses' granule ranges (hp.acc_g0 / acc_g1) and a1's
+// records.  host_a1 (if given) runs a1 on the host while the device's first phase — which needs
+// only the ranges — builds the intervals; otherwise a1 must be done already.
+int device_plan_a2(HostPlan& hp, const DevPlanArgs& args, DevScratch& S, DevPlanOut& out,
+                   const std::function<int()>& host_a1 = nullptr);
 
 DevScratch* plan_dev_acquire(int device);      // nullptr: no memory / stream
 void plan_dev_release(DevScratch* s);          // the caller's work on it is complete
