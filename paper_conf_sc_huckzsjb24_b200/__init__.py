@@ -147,14 +147,22 @@ class Report:
         self.n_runs = nr.value
         self.truncated = bool(tr.value)
         kept = nr.value if not tr.value else min(nr.value, max_runs)
-        ctr = cusan_counters()
-        _ck(lib.cusan_report_counters(h, C.byref(ctr)))
-        self.counters = {n: getattr(ctr, n) for n, _ in cusan_counters._fields_}
+        self._counters = None
         if kept:
             buf = (C.c_char * (kept * RUN_DTYPE.itemsize)).from_address(C.addressof(rp.contents))
             self.runs = np.frombuffer(bytes(buf), RUN_DTYPE).copy()
         else:
             self.runs = np.zeros(0, RUN_DTYPE)
+
+    @property
+    def counters(self) -> dict:
+        """cusan_report_counters as a dict (read on first use: an online checker's per-call report
+        need not pay for it)."""
+        if self._counters is None:
+            ctr = cusan_counters()
+            _ck(lib.cusan_report_counters(self.h, C.byref(ctr)))
+            self._counters = {n: getattr(ctr, n) for n, _ in cusan_counters._fields_}
+        return self._counters
 
     def __del__(self, _free=lib.cusan_report_free):
         if getattr(self, "h", None):

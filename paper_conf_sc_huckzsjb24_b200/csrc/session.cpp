@@ -434,22 +434,39 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
 
     // ---- a2: refine the layout by the new endpoints -----------------------------------------------
     const uint64_t n_new = cp.g0.size();
-    std::vector<uint64_t> P;
-    P.reserve(2 * (n_new + s->ivs.size()));
+    std::vector<uint64_t> E;
+    E.reserve(2 * n_new);
     // with shards, every block edge inside a new access is a boundary too, so each new elementary
     // interval lies in one block and belongs to one shard (old intervals are this shard's already)
     const int nsh = s->opts.nshards;
     const uint32_t L = s->blk_log2;
     for (uint64_t k = 0; k < n_new; k++)
         if (cp.g1[k] > cp.g0[k]) {
-            P.push_back(cp.g0[k]);
-            P.push_back(cp.g1[k]);
+            E.push_back(cp.g0[k]);
+            E.push_back(cp.g1[k]);
             if (nsh > 1)
-                for (uint64_t b = ((cp.g0[k] >> L) + 1) << L; b < cp.g1[k]; b += 1ull << L) P.push_back(b);
+                for (uint64_t b = ((cp.g0[k] >> L) + 1) << L; b < cp.g1[k]; b += 1ull << L) E.push_back(b);
         }
-    for (const SIv& u : s->ivs) { P.push_back(u.abs_begin); P.push_back(u.abs_begin + u.len); }
-    std::sort(P.begin(), P.end());
-    P.erase(std::unique(P.begin(), P.end()), P.end());
+    std::sort(E.begin(), E.end());
+    E.erase(std::unique(E.begin(), E.end()), E.end());
+    // P = the old intervals' endpoints (already in order: the layout is sorted and disjoint) merged
+    // with the new ones — linear in the layout, so a small call does not re-sort the whole layout
+    std::vector<uint64_t> P;
+    P.reserve(E.size() + 2 * s->ivs.size());
+    {
+        size_t e = 0;
+        auto put = [&](uint64_t x) {
+            for (; e < E.size() && E[e] < x; e++)
+                if (P.empty() || P.back() != E[e]) P.push_back(E[e]);
+            if (P.empty() || P.back() != x) P.push_back(x);
+        };
+        for (const SIv& u : s->ivs) {
+            put(u.abs_begin);
+            put(u.abs_begin + u.len);
+        }
+        for (; e < E.size(); e++)
+            if (P.empty() || P.back() != E[e]) P.push_back(E[e]);
+    }
     const uint64_t np = P.size();
     std::vector<int64_t> diff(np + 1, 0);
     std::vector<uint32_t> b0(n_new, 0), b1(n_new, 0);
@@ -463,6 +480,8 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
     const bool compressed = compressed_shadow(s->opts);
     std::vector<uint32_t> iv_of(np ? np - 1 : 0, 0xffffffffu);
     uint64_t used = s->used;
+    cp.ivs.reserve(np);
+    cp.has_state.reserve(np);
     {
         int64_t cov = 0;
         size_t u = 0;
@@ -622,6 +641,7 @@ struct PendingCall {
     uint64_t seg_first_word = 0;                    // where they go in segvc_d
     uint64_t used_before = 0;                       // shadow cells in use before the call
     pinned_vector<unsigned long long> init, cnt;    // counter initial values / read-back
+    pinned_vector<char> stage;                      // the call's tables as uploaded (one copy)
     uint64_t h2d = 0;
     uint64_t delta = 0;                             // event numbering the call was planned with
     std::shared_ptr<const std::vector<uint32_t>> orig;
@@ -705,19 +725,25 @@ static int session_launch(cusan_session* s, PendingCall& pc) {
     DSpan* d_spans = (DSpan*)(s->scratch.p + o_spans);
     CopySeg* d_copy = (CopySeg*)(s->scratch.p + o_copy);
     unsigned long long* d_cnt = (unsigned long long*)(s->scratch.p + o_cnt);
-    CK(cudaMemcpyAsync(d_inc, cp.inc.data(), cp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, s->stream));
-    CK(cudaMemcpyAsync(d_spans, tabs.ds.data(), tabs.ds.size() * sizeof(DSpan), cudaMemcpyHostToDevice, s->stream));
-    CK(cudaMemcpyAsync(d_copy, cp.segs.data(), cp.segs.size() * sizeof(CopySeg), cudaMemcpyHostToDevice, s->stream));
+    // the call's tables and the counters' initial values go up in ONE transfer: staged in a
+    // page-locked buffer laid out as the scratch is (a small call's latency is mostly per-copy cost)
+    pc.init.assign(N_COUNTERS + nwin, 0ull);
+    pc.cnt.assign(N_COUNTERS, 0ull);
+    pc.init[C_HEAP] = s->heap_cap();     // records are host-assigned: no device allocation
+    pc.stage.resize(off);
+    auto put = [&](uint64_t at, const void* src, size_t bytes) {
+        if (bytes) std::memcpy(pc.stage.data() + at, src, bytes);
+    };
+    put(o_inc, cp.inc.data(), cp.inc.size() * sizeof(AccRec));
+    put(o_spans, tabs.ds.data(), tabs.ds.size() * sizeof(DSpan));
+    put(o_copy, cp.segs.data(), cp.segs.size() * sizeof(CopySeg));
+    put(o_cnt, pc.init.data(), pc.init.size() * sizeof(unsigned long long));
+    CK(cudaMemcpyAsync(s->scratch.p, pc.stage.data(), off, cudaMemcpyHostToDevice, s->stream));
     pc.h2d = cp.inc.size() * sizeof(AccRec) + tabs.ds.size() * sizeof(DSpan) + cp.segs.size() * sizeof(CopySeg) +
              pc.seg_rows.size() * sizeof(uint32_t);
     session_tick(pc, "memory");
 
     // ---- a3, in place ------------------------------------------------------------------------------
-    pc.init.assign(N_COUNTERS + nwin, 0ull);
-    pc.cnt.assign(N_COUNTERS, 0ull);
-    pc.init[C_HEAP] = s->heap_cap();     // records are host-assigned: no device allocation
-    CK(cudaMemcpyAsync(d_cnt, pc.init.data(), pc.init.size() * sizeof(unsigned long long), cudaMemcpyHostToDevice,
-                       s->stream));
     CK(cudaEventRecord(s->ev0, s->stream));
     if (cp.copy_cells)
         CK(launch_copy_cells(s->max_blocks, s->stream, s->shadow.p, s->shadow.p, d_copy, (uint32_t)cp.segs.size(),
