@@ -169,8 +169,134 @@ static void radix_sort_pairs(std::vector<uint64_t>& key, std::vector<uint32_t>& 
 //      evolves independently of the other columns — each primitive is an element-wise max, copy or
 //      tick — so the columns are split among threads, each replaying the whole trace on its columns
 //      and writing them into the segment rows.  Same rows as one pass over whole clocks.
+// a1 in ONE pass with whole clock rows, on one thread: the default.  Every primitive is a row
+// operation (max, copy, tick), so rows padded to a multiple of 8 u32 make each one a few 256-bit
+// vector instructions (the function is compiled for AVX2 as well as the baseline ISA, chosen at load
+// time); one pass reads the trace once and leaves the other cores to the stages a pipelined checker
+// runs beside it (lowering, device planning).  Same segment rows, records and counters as the
+// two-pass column form below (CUSAN_A1_COLUMNS=1 selects that one; tests compare the two).
+static inline void row_max(uint32_t* __restrict__ d, const uint32_t* __restrict__ s, uint32_t n) {
+    for (uint32_t g = 0; g < n; g++) d[g] = d[g] > s[g] ? d[g] : s[g];
+}
+
+__attribute__((target_clones("avx2", "default")))
+static std::pair<int, std::string> run_a1_fused(const Trace& t, HostPlan& hp, bool fill_accesses) {
+    constexpr uint32_t NO_SEG = 0xffffffffu;
+    const uint64_t n = t.ev.size();
+    cusan_counters& c = hp.ctr;
+    uint32_t F;
+    if (fill_accesses) {                   // the accesses, the clock width and the counters too
+        c = cusan_counters{};
+        c.n_events = n;
+        F = 1;
+        uint64_t n_acc = 0;
+        for (const cusan_event& e : t.ev) {
+            F = std::max<uint32_t>(F, e.fiber + 1);
+            if (e.kind == CUSAN_EV_FORK) F = std::max<uint32_t>(F, (uint32_t)e.a + 1);
+            n_acc += e.kind == CUSAN_EV_ACCESS;
+        }
+        if (F > CUSAN_MAX_FIBERS + 1) return {CUSAN_EINVAL, "fiber id beyond the trace's fibers"};
+        hp.F = F;
+        c.n_fibers = F;
+        hp.acc_g0.resize(n_acc);
+        hp.acc_g1.resize(n_acc);
+        hp.acc_rec.resize(n_acc);
+        hp.acc_event.clear();
+    } else {
+        F = hp.F;
+    }
+    const uint32_t FP = (F + 7) & ~7u;     // padded row (the padding columns stay 0)
+    std::vector<uint32_t> C((size_t)F * FP, 0), S;
+    S.reserve((size_t)1024 * FP);
+    std::vector<uint32_t> cur_seg(F, NO_SEG);
+    KeySlots key_slot;
+    hp.nseg = 0;
+    hp.segvc.clear();
+    {
+        const uint64_t n_acc = hp.acc_g0.size();
+        if (n_acc * F <= (16ull << 20)) hp.segvc.reserve(n_acc * F);   // ≤ 64 MB: no regrowth
+    }
+    uint64_t k = 0;
+    for (uint64_t i = 0; i < n; i++) {
+        const cusan_event& e = t.ev[i];
+        const uint32_t f = e.fiber;
+        if (f >= F) return {CUSAN_EINVAL, "fiber id beyond the trace's fibers"};
+        uint32_t* Cf = &C[(size_t)f * FP];
+        const uint32_t tick = (uint32_t)(i + 1);
+        switch (e.kind) {
+            case CUSAN_EV_FORK: {                  // an event of src: C_src[src] := i+1; C_dst ⊔= C_src
+                const uint32_t src = (uint32_t)e.a;
+                if (src >= F) return {CUSAN_EINVAL, "fiber id beyond the trace's fibers"};
+                uint32_t* Cs = &C[(size_t)src * FP];
+                Cs[src] = tick;
+                if (src != f) row_max(Cf, Cs, FP);
+                cur_seg[f] = NO_SEG;               // opens a segment on dst
+                c.n_fork++;
+                break;
+            }
+            case CUSAN_EV_ACCESS: {
+                Cf[f] = tick;
+                if (cur_seg[f] == NO_SEG) {        // a segment opens: its row is C_f
+                    if (hp.nseg >= 0x7fffffffu) return {CUSAN_ERANGE, "too many segments"};
+                    cur_seg[f] = (uint32_t)hp.nseg++;
+                    hp.segvc.insert(hp.segvc.end(), Cf, Cf + F);
+                }
+                if (fill_accesses) {
+                    hp.acc_g0[k] = e.a >> 3;
+                    hp.acc_g1[k] = e.b ? (e.a + e.b + 7) >> 3 : e.a >> 3;
+                }
+                hp.acc_rec[k] = {pack_epoch(f, (uint32_t)i), cur_seg[f] | ((uint32_t)e.mode << 31)};
+                const uint64_t bytes = 8 * (hp.acc_g1[k] - hp.acc_g0[k]);
+                k++;
+                c.n_access++;
+                c.tracked_bytes += bytes;
+                if (e.mode) { c.n_write++; c.bytes_written += bytes; }
+                else { c.n_read++; c.bytes_read += bytes; }
+                break;
+            }
+            case CUSAN_EV_RELEASE:
+            case CUSAN_EV_RELEASE_STORE:
+            case CUSAN_EV_ACQUIRE: {
+                Cf[f] = tick;
+                bool fresh;
+                const uint32_t slot = key_slot.get(e.a, &fresh);
+                if (fresh) S.resize(S.size() + FP, 0u);
+                uint32_t* Sk = &S[(size_t)slot * FP];
+                if (e.kind == CUSAN_EV_RELEASE) {              // SC_k := SC_k ⊔ C_f
+                    row_max(Sk, Cf, FP);
+                    c.n_release++;
+                } else if (e.kind == CUSAN_EV_RELEASE_STORE) { // SC_k := C_f
+                    std::copy(Cf, Cf + FP, Sk);
+                    c.n_release_store++;
+                } else {                                       // C_f := C_f ⊔ SC_k
+                    row_max(Cf, Sk, FP);
+                    cur_seg[f] = NO_SEG;
+                    c.n_acquire++;
+                }
+                break;
+            }
+            default:
+                return {CUSAN_EINVAL, "bad event kind in trace"};
+        }
+    }
+    c.n_segments = hp.nseg;
+    return {CUSAN_OK, ""};
+}
+
 std::pair<int, std::string> run_a1(const Trace& t, HostPlan& hp, unsigned threads, bool fill_accesses) {
     const auto t_start = std::chrono::steady_clock::now();
+    static const bool columns = [] {
+        const char* e = std::getenv("CUSAN_A1_COLUMNS");
+        return e && *e && *e != '0';
+    }();
+    if (!columns) {
+        std::pair<int, std::string> st = run_a1_fused(t, hp, fill_accesses);
+        if (std::getenv("CUSAN_DEBUG_TIMING"))
+            std::fprintf(stderr, "run_a1: one pass %.3f ms (%llu events, %llu segments)\n",
+                         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t_start).count(),
+                         (unsigned long long)t.ev.size(), (unsigned long long)hp.nseg);
+        return st;
+    }
     const uint64_t n = t.ev.size();
     cusan_counters& c = hp.ctr;
     if (fill_accesses) {                   // one pass: the accesses, the clock width and the counters too

@@ -301,3 +301,40 @@ def test_clocks_equal_a1_written_out(seed):
         assert list(g0) == w_g0 and list(g1) == w_g1
         for r, wr in zip(rows, w_rows):
             assert np.array_equal(r, wr)
+
+
+def test_clocks_one_pass_equals_column_form(tmp_path):
+    """a1's default one-pass form (whole rows, one thread) and its two-pass column form
+    (CUSAN_A1_COLUMNS=1: serial pre-pass, then column blocks on threads) give the same clocks
+    image byte for byte — ranges, epochs, segment rows and counters."""
+    import subprocess
+    import sys
+
+    import paper_conf_sc_huckzsjb24_b200 as cs
+    from tracegen import fuzz
+    rng = np.random.default_rng(123)
+    traces = []
+    for t in range(10):
+        nf = int(rng.integers(2, 70))
+        ev = fuzz.random_primitive_trace(rng, int(rng.integers(1, 500)), nf, n_keys=int(rng.integers(1, 9)),
+                                         n_granules=int(rng.integers(1, 300)), unaligned=bool(t % 2))
+        if t >= 7:                                   # large enough for the threaded column pass
+            ev = np.concatenate([ev] * 80)
+        traces.append((nf, ev))
+    np.savez(tmp_path / "tr.npz", **{f"ev{i}": ev for i, (_, ev) in enumerate(traces)},
+             nf=np.array([nf for nf, _ in traces]))
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    code = (f"import sys; sys.path.insert(0, {root!r}); import numpy as np; "
+            "import paper_conf_sc_huckzsjb24_b200 as cs; "
+            f"d = np.load({str(tmp_path / 'tr.npz')!r}); out = {{}}\n"
+            "for i, nf in enumerate(d['nf']):\n"
+            "    tr = cs.Trace(int(nf)); tr.cusan_trace_append_events(d[f'ev{i}'])\n"
+            "    out[f'img{i}'] = cs.Clocks.compute(tr).to_bytes()\n"
+            f"np.savez({str(tmp_path / 'img.npz')!r}, **out)\n")
+    env = dict(os.environ, CUSAN_A1_COLUMNS="1", CUSAN_PLAN_THREADS="4")
+    subprocess.run([sys.executable, "-c", code], check=True, env=env)
+    col = np.load(tmp_path / "img.npz")
+    for i, (nf, ev) in enumerate(traces):
+        tr = cs.Trace(nf)
+        tr.cusan_trace_append_events(ev)
+        assert np.array_equal(cs.Clocks.compute(tr).to_bytes(), col[f"img{i}"]), i
