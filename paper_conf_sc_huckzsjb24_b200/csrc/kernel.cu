@@ -211,17 +211,27 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
     rc.nrace = 0;
     // Range assignment: with `sched`, warps grab GRAB consecutive ranges at a time from a per-launch
     // counter (dynamic balance); without, each warp owns one coverage-weighted contiguous slice.
+    // The first grab is static (warp w takes range w: no atomic round trip before the first range of
+    // a launch); later grabs continue after the grid's ranges.  When every span is one range (the
+    // compressed layout, and short dense spans) range t is span t: no search.
     uint64_t tend = 0;
     uint32_t s = 0;
     bool first = true;
+    const bool one_per_span = total_tiles == (uint64_t)nspans;
+    const uint64_t nwarps_all = (uint64_t)gridDim.x * WARPS;
     {
         for (uint64_t t = 0;; t++) {
             if (t >= tend) {
                 uint64_t b, e;
                 if (sched) {
-                    unsigned long long base = 0;
-                    if (lane == 0) base = atomicAdd(sched, (unsigned long long)GRAB);
-                    b = __shfl_sync(FULL, base, 0);
+                    if (first) {
+                        b = (uint64_t)blockIdx.x * WARPS + warp;
+                        first = false;
+                    } else {
+                        unsigned long long base = 0;
+                        if (lane == 0) base = atomicAdd(sched, (unsigned long long)GRAB);
+                        b = nwarps_all + __shfl_sync(FULL, base, 0);
+                    }
                     e = min(b + (uint64_t)GRAB, total_tiles);
                 } else {
                     if (!first) break;
@@ -236,9 +246,10 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                 if (b >= e) break;
                 t = b;
                 tend = e;
-                s = find_span_by_tile(spans, nspans, t);
+                s = one_per_span ? (uint32_t)t : find_span_by_tile(spans, nspans, t);
             }
-            while (t >= spans[s + 1].tile0) s++;   // spans[nspans] is a sentinel
+            if (one_per_span) s = (uint32_t)t;
+            else while (t >= spans[s + 1].tile0) s++;   // spans[nspans] is a sentinel
             const DSpan sp = spans[s];
             // f3: one cell per interval, and a compressed span is always a single range (its cell
             // must have exactly one owner, whatever the interval's length)
