@@ -13,9 +13,8 @@
 // stream").  Stream handle 1 = cudaStreamLegacy, 2 = cudaStreamPerThread,
 // 0 = the default stream of the selected mode.
 #include <algorithm>
-#include <map>
+#include <functional>
 #include <new>
-#include <set>
 #include <unordered_map>
 
 #include "../../include/cusan_lower.h"
@@ -39,7 +38,7 @@ struct cusan_lowering {
     std::vector<uint32_t> blocking;                        // blocking streams (creation order)
     std::vector<char> is_blocking;                         // by fiber
     uint32_t next_fiber = 2;
-    std::set<uint32_t> mpi_free;                           // pool of completed request fibers
+    std::vector<uint32_t> mpi_free;                        // pool of completed request fibers (min-heap)
     FlatMap<uint32_t> req_fiber;                           // MPI request -> its fiber
     struct Alloc {
         uint64_t base, size;
@@ -353,8 +352,9 @@ static int mpi_nonblocking(cusan_lowering* l, uint64_t buf, uint64_t n, uint64_t
     if (!l) return fail(CUSAN_EINVAL, "lowering is null");
     uint32_t m = 0;
     if (!l->mpi_free.empty()) {            // recycled only after completion
-        m = *l->mpi_free.begin();
-        l->mpi_free.erase(l->mpi_free.begin());
+        std::pop_heap(l->mpi_free.begin(), l->mpi_free.end(), std::greater<uint32_t>());   // lowest id
+        m = l->mpi_free.back();
+        l->mpi_free.pop_back();
     } else {
         int st = l->new_fiber(&m);
         if (st) return st;
@@ -379,7 +379,8 @@ int cusan_on_mpi_wait(cusan_lowering* l, uint64_t req) {
     int st = l->sync(CUSAN_ACQUIRE, l->H(), K_req(req));
     if (st) return st;
     if (const uint32_t* it = l->req_fiber.get(req)) {
-        l->mpi_free.insert(*it);
+        l->mpi_free.push_back(*it);
+        std::push_heap(l->mpi_free.begin(), l->mpi_free.end(), std::greater<uint32_t>());
         l->req_fiber.erase(req);
     }
     return CUSAN_OK;
