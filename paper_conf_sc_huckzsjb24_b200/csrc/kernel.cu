@@ -378,11 +378,17 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                     if (rm) {
                         const unsigned cand = isw ? (rm & below & ~(lw < 0 ? 0u : ((2u << lw) - 1u))) : 0u;
                         unsigned hm = 0;
-#pragma unroll 8
-                        for (int p = 0; p < 32; p++) {
-                            const uint32_t ep = __shfl_sync(FULL, r.epoch, p);
-                            const int np = __shfl_sync(FULL, nxt, p);
-                            if (((cand >> p) & 1u) && np > lane && unordered(ep, f, row)) hm |= 1u << p;
+                        // groups of 8 candidate reads (8 independent clock loads in flight); a group
+                        // no write of the batch must check is skipped (short spans: most of them)
+                        const unsigned anyc = __reduce_or_sync(FULL, cand);
+                        for (int p0 = 0; p0 < 32; p0 += 8) {
+                            if (!((anyc >> p0) & 0xffu)) continue;
+#pragma unroll
+                            for (int p = p0; p < p0 + 8; p++) {
+                                const uint32_t ep = __shfl_sync(FULL, r.epoch, p);
+                                const int np = __shfl_sync(FULL, nxt, p);
+                                if (((cand >> p) & 1u) && np > lane && unordered(ep, f, row)) hm |= 1u << p;
+                            }
                         }
                         for (;;) {                                   // one run per (read, write) hit
                             const unsigned any = __ballot_sync(FULL, hm != 0);
