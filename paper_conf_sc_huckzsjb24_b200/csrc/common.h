@@ -214,6 +214,7 @@ struct HostPlan {
     uint32_t F = 1;                       // fibers (row length of segvc)
     pinned_vector<uint32_t> segvc;        // nseg × F (uploaded)
     uint64_t nseg = 0;
+    uint64_t nseg_count = 0;              // segments of the trace, counted ahead of a1 (0 = unknown)
     // accesses in trace order
     std::vector<uint64_t> acc_g0, acc_g1; // granule ranges
     std::vector<uint32_t> acc_event;      // trace position

@@ -189,12 +189,21 @@ static std::pair<int, std::string> run_a1_fused(const Trace& t, HostPlan& hp, bo
         c = cusan_counters{};
         c.n_events = n;
         F = 1;
-        uint64_t n_acc = 0;
+        uint64_t n_acc = 0, nseg = 0;
+        std::vector<char> open(CUSAN_MAX_FIBERS + 1, 0);   // segments, counted for the row allocation
         for (const cusan_event& e : t.ev) {
             F = std::max<uint32_t>(F, e.fiber + 1);
-            if (e.kind == CUSAN_EV_FORK) F = std::max<uint32_t>(F, (uint32_t)e.a + 1);
-            n_acc += e.kind == CUSAN_EV_ACCESS;
+            if (e.fiber > CUSAN_MAX_FIBERS) continue;
+            if (e.kind == CUSAN_EV_ACCESS) {
+                n_acc++;
+                nseg += !open[e.fiber];
+                open[e.fiber] = 1;
+            } else if (e.kind == CUSAN_EV_ACQUIRE || e.kind == CUSAN_EV_FORK) {
+                if (e.kind == CUSAN_EV_FORK) F = std::max<uint32_t>(F, (uint32_t)e.a + 1);
+                open[e.fiber] = 0;
+            }
         }
+        hp.nseg_count = nseg;
         if (F > CUSAN_MAX_FIBERS + 1) return {CUSAN_EINVAL, "fiber id beyond the trace's fibers"};
         hp.F = F;
         c.n_fibers = F;
@@ -212,10 +221,7 @@ static std::pair<int, std::string> run_a1_fused(const Trace& t, HostPlan& hp, bo
     KeySlots key_slot;
     hp.nseg = 0;
     hp.segvc.clear();
-    {
-        const uint64_t n_acc = hp.acc_g0.size();
-        if (n_acc * F <= (16ull << 20)) hp.segvc.reserve(n_acc * F);   // ≤ 64 MB: no regrowth
-    }
+    hp.segvc.reserve(hp.nseg_count * F);     // counted by the access scan (0: rows grow as they come)
     uint64_t k = 0;
     for (uint64_t i = 0; i < n; i++) {
         const cusan_event& e = t.ev[i];
@@ -450,15 +456,22 @@ static void prepare_accesses(const Trace& t, HostPlan& hp) {
     hp.acc_event.resize(n_acc);
     hp.acc_rec.resize(n_acc);
     {
-        uint64_t k = 0;
+        uint64_t k = 0, nseg = 0;
+        std::vector<char> open(F, 0);             // segments, counted for a1's row allocation
         for (uint64_t i = 0; i < t.ev.size(); i++) {
             const cusan_event& e = t.ev[i];
-            if (e.kind != CUSAN_EV_ACCESS) continue;
+            if (e.kind != CUSAN_EV_ACCESS) {
+                if (e.kind == CUSAN_EV_ACQUIRE || e.kind == CUSAN_EV_FORK) open[e.fiber] = 0;
+                continue;
+            }
+            nseg += !open[e.fiber];
+            open[e.fiber] = 1;
             hp.acc_g0[k] = e.a >> 3;
             hp.acc_g1[k] = e.b ? (e.a + e.b + 7) >> 3 : e.a >> 3;
             hp.acc_event[k] = (uint32_t)i;
             k++;
         }
+        hp.nseg_count = nseg;
     }
 }
 
