@@ -568,7 +568,8 @@ static int launch_all(cusan_plan* p) {
     for (size_t i = 0; i < p->wins.size(); i++) {
         const Window& w = p->wins[i];
         unsigned long long* sched = CUSAN_DYNAMIC ? p->d_counters + N_COUNTERS + i : nullptr;
-        CK(launch_shadow_check(w.grid, p->stream, p->d_spans + w.span_off, w.nspans, w.tiles, w.weight, k, sched));
+        CK(launch_shadow_check(w.grid, p->stream, p->d_spans + w.span_off, w.nspans, w.tiles, w.weight, k, sched,
+                               compressed_shadow(p->hp.opts)));
     }
     CK(cudaGetLastError());
     CK(cudaEventRecord(p->ev1, p->stream));

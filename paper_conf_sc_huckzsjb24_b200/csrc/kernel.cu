@@ -27,6 +27,7 @@
 //   default) the range is the whole interval and its one cell is loaded once.  Hits feed a 32-entry
 //   per-warp run cache (one entry per lane) that extends runs across ranges before appending them
 //   to global memory.
+#include <algorithm>
 #include <atomic>
 
 #include "kernel.cuh"
@@ -178,9 +179,14 @@ __device__ __forceinline__ uint64_t tile_at_weight(const DSpan* __restrict__ sp,
     return sp[lo].tile0 + (pos - sp[lo].weight0 + w - 1) / w;
 }
 
-__global__ void __launch_bounds__(THREADS, CUSAN_MIN_BLOCKS)
+// TMA = false: the instantiation for windows whose spans are all interval-compressed (one cell per
+// span, never streamed) — no dynamic shared memory, so more blocks fit on an SM (the compressed
+// check is latency-bound: more warps in flight, fewer spans per warp).
+template <bool TMA>
+__global__ void __launch_bounds__(THREADS, TMA ? CUSAN_MIN_BLOCKS : CUSAN_MIN_BLOCKS_NT)
 shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t total_tiles,
                     uint64_t total_weight, Ctx k, unsigned long long* sched) {
+    constexpr bool kTMA = CUSAN_TMA && TMA;
     __shared__ uint32_t s_list[WARPS][MAXS];
     __shared__ uint8_t s_slot[WARPS][256];
     const int lane = threadIdx.x & 31;
@@ -189,21 +195,21 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
     uint8_t* slot = s_slot[warp];
     for (int i = lane; i < 256; i += 32) slot[i] = 0xFFu;
     __syncwarp();
-#if CUSAN_TMA
-    extern __shared__ __align__(128) unsigned char dsm[];
+    extern __shared__ __align__(128) unsigned char dsm[];     // TMA buffers (none when !kTMA)
     unsigned char* wsm = dsm + (size_t)warp * TMA_WARP_BYTES;
     uint4* s_ld0 = reinterpret_cast<uint4*>(wsm);
     uint4* s_ld1 = reinterpret_cast<uint4*>(wsm + TMA_CHUNK);
     uint4* s_pat = reinterpret_cast<uint4*>(wsm + 2 * TMA_CHUNK);
     uint64_t* s_bar = reinterpret_cast<uint64_t*>(wsm + 2 * TMA_CHUNK + TMA_PAT);
-    if (lane == 0) {
-        mbar_init(&s_bar[0]);
-        mbar_init(&s_bar[1]);
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    if constexpr (kTMA) {
+        if (lane == 0) {
+            mbar_init(&s_bar[0]);
+            mbar_init(&s_bar[1]);
+            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+        }
+        __syncwarp();
     }
-    __syncwarp();
     uint32_t ph0 = 0, ph1 = 0;              // mbarrier phases (warp-uniform)
-#endif
     RunCache rc;
     rc.e = rc.l = 0;
     rc.gb = rc.ge = 0;
@@ -270,8 +276,7 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
             if (sp.flags & SPAN_LOAD) {
                 c = src[0];
                 bool ok = true;
-#if CUSAN_TMA
-                if (n2 * 16 >= TMA_MIN_BYTES) {
+                if (kTMA && n2 * 16 >= TMA_MIN_BYTES) {
                     // bulk copies through a double buffer in shared memory (TMA engine)
                     const uint64_t bytes = n2 * 16;
                     const uint64_t nch = (bytes + TMA_CHUNK - 1) / TMA_CHUNK;
@@ -300,9 +305,7 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                         }
                         __syncwarp();
                     }
-                } else
-#endif
-                {
+                } else {
                     for (uint64_t i = lane; i < n2; i += 32 * UL) {
                         uint4 v[UL];
 #pragma unroll
@@ -480,8 +483,7 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                 const bool dtail = ncell > dhead && ((ncell - dhead) & 1);
                 const uint4 cc = make_uint4(c.x, c.y, c.x, c.y);
                 if (dhead && lane == 0) __stcs(cells, c);
-#if CUSAN_TMA
-                if (m2 * 16 >= TMA_MIN_BYTES) {
+                if (kTMA && m2 * 16 >= TMA_MIN_BYTES) {
                     // a shared-memory tile of the final cell, pushed out by bulk copies
                     if (lane == 0) bulk_wait_read();          // the previous range's stores read the tile
                     __syncwarp();
@@ -496,7 +498,6 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
                         bulk_commit();
                     }
                 } else
-#endif
                 for (uint64_t i = lane; i < m2; i += 32 * UL) {
 #pragma unroll
                     for (int u = 0; u < UL; u++)
@@ -507,10 +508,10 @@ shadow_check_window(const DSpan* __restrict__ spans, uint32_t nspans, uint64_t t
             __syncwarp();
         }
     }
-#if CUSAN_TMA
-    if (lane == 0) bulk_wait_all();                 // bulk stores done before the tile goes away
-    __syncwarp();
-#endif
+    if constexpr (kTMA) {
+        if (lane == 0) bulk_wait_all();             // bulk stores done before the tile goes away
+        __syncwarp();
+    }
     if (rc.ge > rc.gb) flush_entry(rc, k);
     if (lane == 0 && rc.nrace) atomicAdd(&k.counters[C_RACE], rc.nrace);
 }
@@ -590,9 +591,21 @@ cudaError_t launch_fill_cells(uint32_t grid, cudaStream_t stream, uint2* shadow,
     return cudaGetLastError();
 }
 
+// A compressed window runs the !TMA instantiation on a grid of its own occupancy (more blocks per
+// SM); `grid` is the caller's for the TMA one, so only its range count matters there.
 cudaError_t launch_shadow_check(uint32_t grid, cudaStream_t stream, const DSpan* spans, uint32_t nspans,
-                                uint64_t tiles, uint64_t weight, const Ctx& k, unsigned long long* sched) {
-    shadow_check_window<<<grid, THREADS, DYN_SMEM, stream>>>(spans, nspans, tiles, weight, k, sched);
+                                uint64_t tiles, uint64_t weight, const Ctx& k, unsigned long long* sched,
+                                bool compressed) {
+    if (compressed) {
+        int max_blocks = 0;
+        cudaError_t e = shadow_check_max_blocks(true, &max_blocks);
+        if (e != cudaSuccess) return e;
+        const uint64_t want = (tiles + WARPS - 1) / WARPS;
+        const uint32_t g = (uint32_t)std::max<uint64_t>(1, std::min<uint64_t>((uint64_t)max_blocks, want));
+        shadow_check_window<false><<<g, THREADS, 0, stream>>>(spans, nspans, tiles, weight, k, sched);
+    } else {
+        shadow_check_window<true><<<grid, THREADS, DYN_SMEM, stream>>>(spans, nspans, tiles, weight, k, sched);
+    }
     return cudaGetLastError();
 }
 
@@ -601,6 +614,19 @@ cudaError_t launch_copy_cells(uint32_t grid, cudaStream_t stream, const uint2* s
     copy_cells<<<grid, THREADS, 0, stream>>>(src, dst, segs, nseg, total);
     return cudaGetLastError();
 }
+
+template <bool TMA>
+static cudaError_t blocks_per_sm_query(int* per_sm) {
+    const size_t dyn = TMA ? DYN_SMEM : 0;
+    if (dyn) {
+        cudaError_t e = cudaFuncSetAttribute(shadow_check_window<TMA>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             (int)dyn);
+        if (e != cudaSuccess) return e;
+    }
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, shadow_check_window<TMA>, THREADS, dyn);
+}
+
+cudaError_t shadow_check_blocks_per_sm_query(int* per_sm) { return blocks_per_sm_query<true>(per_sm); }
 
 // Once per device: setting a function attribute while that kernel runs waits for it, so a plan
 // prepared on another host thread while a check runs (pipelined checks) would stall here.
@@ -621,13 +647,28 @@ cudaError_t shadow_check_blocks_per_sm(int* per_sm) {
     return e1;
 }
 
-cudaError_t shadow_check_blocks_per_sm_query(int* per_sm) {
-    if (DYN_SMEM) {
-        cudaError_t e = cudaFuncSetAttribute(shadow_check_window, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                             (int)DYN_SMEM);
-        if (e != cudaSuccess) return e;
+// Resident blocks of one K1 instantiation on the whole device (SMs × blocks per SM), cached.
+cudaError_t shadow_check_max_blocks(bool compressed, int* max_blocks) {
+    static std::atomic<int> known[2][256];
+    int dev = 0;
+    cudaError_t e0 = cudaGetDevice(&dev);
+    if (e0 != cudaSuccess) return e0;
+    const int c = compressed ? 1 : 0;
+    if (dev >= 0 && dev < 256) {
+        const int v = known[c][dev].load(std::memory_order_acquire);
+        if (v > 0) {
+            *max_blocks = v;
+            return cudaSuccess;
+        }
     }
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, shadow_check_window, THREADS, DYN_SMEM);
+    int sms = 0, per_sm = 0;
+    cudaError_t e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (e != cudaSuccess) return e;
+    e = compressed ? blocks_per_sm_query<false>(&per_sm) : shadow_check_blocks_per_sm(&per_sm);
+    if (e != cudaSuccess) return e;
+    *max_blocks = std::max(1, sms * per_sm);
+    if (dev >= 0 && dev < 256) known[c][dev].store(*max_blocks, std::memory_order_release);
+    return cudaSuccess;
 }
 
 }  // namespace cusan

@@ -18,6 +18,9 @@ constexpr int CHUNK = 128;              // granule multiple of a warp range (16-
 #ifndef CUSAN_MIN_BLOCKS
 #define CUSAN_MIN_BLOCKS 3
 #endif
+#ifndef CUSAN_MIN_BLOCKS_NT
+#define CUSAN_MIN_BLOCKS_NT 4     // the compressed (no-TMA) instantiation of K1
+#endif
 constexpr int UL = CUSAN_UL;            // 16-B loads / stores in flight per lane when streaming
 #ifndef CUSAN_DYNAMIC
 #define CUSAN_DYNAMIC 1
@@ -132,8 +135,11 @@ struct WinDesc {
 
 // ---- launch wrappers (kernel.cu) ----------------------------------------------------------------
 // K1: one window of the shadow check
+// (compressed: every span of the window is one interval-compressed cell — the instantiation without
+// TMA buffers, on a grid of its own occupancy)
 cudaError_t launch_shadow_check(uint32_t grid, cudaStream_t stream, const DSpan* spans, uint32_t nspans,
-                                uint64_t tiles, uint64_t weight, const Ctx& k, unsigned long long* sched);
+                                uint64_t tiles, uint64_t weight, const Ctx& k, unsigned long long* sched,
+                                bool compressed);
 // sessions: copy the cell of a split compressed interval to its new piece
 cudaError_t launch_copy_cells(uint32_t grid, cudaStream_t stream, const uint2* src, uint2* dst,
                               const CopySeg* segs, uint32_t nseg, uint64_t total);
@@ -145,6 +151,7 @@ cudaError_t launch_fill_cells(uint32_t grid, cudaStream_t stream, uint2* shadow,
 // resident blocks of K1 per SM (sets K1's dynamic shared memory limit first)
 cudaError_t shadow_check_blocks_per_sm(int* per_sm);        // cached per device
 cudaError_t shadow_check_blocks_per_sm_query(int* per_sm);  // sets the smem attribute, asks the occupancy API
+cudaError_t shadow_check_max_blocks(bool compressed, int* max_blocks);   // SMs × blocks per SM, cached
 
 // ---- host helpers shared by check_api.cpp and session.cpp -----------------------------------------
 // Device-side span tables: per window its spans plus a sentinel, with range / weight prefixes.

@@ -761,7 +761,8 @@ static int session_launch(cusan_session* s, PendingCall& pc) {
     for (size_t i = 0; i < nwin; i++) {
         const Window& w = tabs.wins[i];
         unsigned long long* sched = CUSAN_DYNAMIC ? d_cnt + N_COUNTERS + i : nullptr;
-        CK(launch_shadow_check(w.grid, s->stream, d_spans + w.span_off, w.nspans, w.tiles, w.weight, k, sched));
+        CK(launch_shadow_check(w.grid, s->stream, d_spans + w.span_off, w.nspans, w.tiles, w.weight, k, sched,
+                               compressed_shadow(s->opts)));
     }
     CK(cudaEventRecord(s->ev1, s->stream));
     CK(cudaMemcpyAsync(pc.cnt.data(), d_cnt, N_COUNTERS * sizeof(unsigned long long), cudaMemcpyDeviceToHost,
