@@ -1,3 +1,4 @@
+# A/B of a1 forms on one B200: clocks timing and the bench e2e with the one-pass (default) and column (CUSAN_A1_COLUMNS=1) forms
 python -c "import __graft_entry__ as g; g.build()" > /dev/null
 nproc
 echo "== a1 default"; CUSAN_DEBUG_TIMING=1 python tools/a1_timing.py 2>&1 | tail -4
