@@ -61,11 +61,34 @@ struct cusan_lowering {
     uint32_t H() const { return h_fiber; }
 
     // --- primitives ---------------------------------------------------------------------------
+    // Appended straight to the trace: the lowering's fibers, modes and kinds are valid by
+    // construction (fibers come from new_fiber, below max_fibers), so only what a caller's values
+    // decide is checked — the trace length and addr + n overflowing (cusan_trace_append_* check
+    // everything for events a user appends).
+    int push(uint8_t kind, uint8_t mode, uint32_t f, uint64_t a, uint64_t b) {
+        std::vector<cusan_event>& ev = trace->t.ev;
+        if (ev.size() >= CUSAN_MAX_TRACE_EVENTS) return fail(CUSAN_ERANGE, "trace longer than 2^32-2 events");
+        cusan_event e{};
+        e.kind = kind;
+        e.mode = mode;
+        e.fiber = f;
+        e.a = a;
+        e.b = b;
+        try {
+            ev.push_back(e);
+        } catch (...) {
+            return fail(CUSAN_ENOMEM, "trace append failed");
+        }
+        return CUSAN_OK;
+    }
     int access(uint32_t f, int mode, uint64_t addr, uint64_t n) {
-        return cusan_trace_append_access(trace, f, (cusan_mode)mode, addr, n, nullptr);
+        if (addr + n < addr || addr + n + 7 < addr + n) return fail(CUSAN_ERANGE, "addr + nbytes overflows");
+        return push(CUSAN_EV_ACCESS, (uint8_t)(mode ? 1 : 0), f, addr, n);
     }
     int sync(cusan_sync k, uint32_t f, uint64_t key) {
-        return cusan_trace_append_sync(trace, k, f, key, nullptr);
+        static constexpr uint8_t kind_of[4] = {CUSAN_EV_RELEASE, CUSAN_EV_RELEASE_STORE, CUSAN_EV_ACQUIRE,
+                                               CUSAN_EV_FORK};
+        return push(kind_of[k], 0, f, key, 0);
     }
 
     // --- helpers -------------------------------------------------------------------------------
