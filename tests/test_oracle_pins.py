@@ -455,3 +455,110 @@ def test_oracle_beyond_2_24_events():
         got = [tuple(int(x) for x in r) for r in rep["runs"]]
         assert got == want, (racy, got, want)
         assert ry > (1 << 24)
+
+
+# ------------------------------------------------------------------------------------------------
+# checker mutants: each plausible mistake in oracle/oracle.c (vector clocks, the HB test, the
+# per-granule race rule, granule rounding, run canonicalisation) must fail a pin — the brute-force
+# graph-HB race set, the paper listings or a closed form — so the checker is pinned by more than
+# its agreement with the product
+# ------------------------------------------------------------------------------------------------
+# (Two edits that look like mistakes are equivalent for the race set and so cannot be pinned:
+#  `i+1 < VC(b)[g]` for `<=` — every event that hands a fiber's clock on (a release, a fork) ticks
+#  past the accesses before it, so VC(b)[g] never equals an earlier access's i+1 — and a FORK
+#  ticking its destination instead of its source, for the same reason.)
+_CHECKER_MUTANTS = {
+    # HB test reads the later access's own column (a →hb b ⇔ i+1 <= VC(b)[g(a)])
+    "hb_wrong_column": ("return acc_event[a] + 1 <= acc_vc[b * F + g];",
+                        "return acc_event[a] + 1 <= acc_vc[b * F + acc_fiber[b]];"),
+    # FORK hands over only the source's own entry (no transitivity)
+    "fork_not_transitive": ("if (Cs[t] > Cf[t]) Cf[t] = Cs[t];", "if (t == s && Cs[t] > Cf[t]) Cf[t] = Cs[t];"),
+    # FORK joins dst into src
+    "fork_joins_backwards": ("if (Cs[t] > Cf[t]) Cf[t] = Cs[t];", "if (Cf[t] > Cs[t]) Cs[t] = Cf[t];"),
+    # RELEASE overwrites the key clock (AnnotateHappensBefore joins)
+    "release_stores": ("                if (Cf[t] > S[t]) S[t] = Cf[t];", "                S[t] = Cf[t];"),
+    # RELEASE_STORE joins (event re-record, A4)
+    "release_store_joins": ("memcpy(S, Cf, F * sizeof(uint32_t));",
+                            "for (uint32_t t = 0; t < F; t++) if (Cf[t] > S[t]) S[t] = Cf[t];"),
+    # ACQUIRE overwrites the fiber clock instead of joining
+    "acquire_overwrites": ("if (S[t] > Cf[t]) Cf[t] = S[t];", "Cf[t] = S[t];"),
+    # reads are not checked against the last write (every access is)
+    "reads_skip_w_check": ("if (wv && !hb(wv - 1, b))", "if (wv && acc_write[b] && !hb(wv - 1, b))"),
+    # a write is not checked against the reads since the last write
+    "write_skips_reads": ("if (!hb(rv - 1, b)) {", "if (0 && !hb(rv - 1, b)) {"),
+    # the read set is not emptied by a write
+    "reads_survive_write": ("                    Rg[tf] = 0;\n", ""),
+    # a write does not become the last write
+    "w_not_updated": ("w->W[x] = (uint32_t)(b + 1);", "(void)0;"),
+    # a fiber's first read since the write kept instead of its last
+    "first_read_kept": ("Rg[f] = (uint32_t)(b + 1);", "if (!Rg[f]) Rg[f] = (uint32_t)(b + 1);"),
+    # partial last granule dropped ([addr>>3, (addr+n+7)>>3))
+    "granule_end_truncated": ("g1 = (e->a + e->b + 7) >> 3;", "g1 = (e->a + e->b) >> 3;"),
+    # partial first granule dropped
+    "granule_begin_rounded_up": ("uint64_t g0 = e->a >> 3,", "uint64_t g0 = (e->a + 7) >> 3,"),
+    # sync keys share one clock (the key lookup ignores the key)
+    "sync_keys_collide": ("while (sc_tab[h].used && sc_tab[h].key != key)", "while (0)"),
+    # run merge ignores the earlier access
+    "run_merge_ignores_earlier": ("tv->t[j].later == r.later && tv->t[j].earlier == r.earlier &&",
+                                  "tv->t[j].later == r.later &&"),
+    # canonical order (later, earlier, g_begin) swapped to (earlier, later, ...)
+    "run_order_swapped": ("    if (a->later != b->later) return a->later < b->later ? -1 : 1;\n"
+                          "    if (a->earlier != b->earlier) return a->earlier < b->earlier ? -1 : 1;\n"
+                          "    return (a->g_begin",
+                          "    if (a->earlier != b->earlier) return a->earlier < b->earlier ? -1 : 1;\n"
+                          "    if (a->later != b->later) return a->later < b->later ? -1 : 1;\n"
+                          "    return (a->g_begin"),
+    # runs cut at tile boundaries are not stitched
+    "tiles_not_stitched": ("all.r[m - 1].g_end == all.r[i].g_begin)", "all.r[m - 1].g_end == all.r[i].g_begin && 0)"),
+    # runs stitched across a gap
+    "runs_stitched_across_gaps": ("all.r[m - 1].g_end == all.r[i].g_begin)", "1)"),
+}
+
+
+def _pin_battery():
+    """The pins a checker must pass (first failure raised): brute-force graph HB on tiny random
+    traces (aligned and unaligned), canonical runs, every paper listing, and a closed form across
+    tiles (two unordered writes over 150,000 granules: one run)."""
+    for seed in (100, 101):
+        for ev, nf in _fuzz_cases(40, seed, unaligned=bool(seed % 2)):
+            rep = oracle.check_events(ev, nf, threads=1)
+            got = brute.runs_to_triples(rep["runs"])
+            assert got == brute.per_fiber_race_set(ev, brute.hb_closure(ev))
+            assert rep["n_race_granules"] == len(got)
+            keys = [(int(r["later"]), int(r["earlier"]), int(r["g_begin"])) for r in rep["runs"]]
+            assert keys == sorted(keys)
+            for a, b in zip(rep["runs"][:-1], rep["runs"][1:]):
+                if a["later"] == b["later"] and a["earlier"] == b["earlier"]:
+                    assert a["g_end"] < b["g_begin"]
+    for lst in LISTINGS:
+        ops, args = lst.program.arrays()
+        ev, nf, first = oracle_lower_with_offsets(ops, args)
+        rep = oracle.check_events(ev, nf, threads=1)
+        got = set(listing_dsl.observed_pairs(rep["runs"], listing_dsl.label_events(lst, ev, first)))
+        assert got == {(a, b) for a, b, _ in lst.expect}, lst.name
+    n = 150_000                                       # > 2 tiles of 65,536 granules, two workers
+    ev = np.zeros(2, EVENT_DTYPE)
+    ev[0] = (EV_ACCESS, 1, 0, 0, 1 << 30, 8 * n)
+    ev[1] = (EV_ACCESS, 1, 0, 1, 1 << 30, 8 * n)
+    rep = oracle.check_events(ev, 2, threads=2)
+    assert [tuple(int(x) for x in r) for r in rep["runs"]] == [((1 << 30) >> 3, ((1 << 30) >> 3) + n, 0, 1)]
+
+
+def test_pin_battery_passes_on_the_oracle():
+    _pin_battery()
+
+
+@pytest.mark.parametrize("name", sorted(_CHECKER_MUTANTS))
+def test_pins_kill_checker_mutants(name, tmp_path, monkeypatch):
+    """oracle.c with one plausible mistake fails the pin battery (or crashes)."""
+    import subprocess
+    old, new = _CHECKER_MUTANTS[name]
+    src = open(os.path.join(os.path.dirname(oracle.__file__), "oracle.c")).read()
+    assert src.count(old) == 1, (name, "mutation site not found exactly once")
+    (tmp_path / "oracle.c").write_text(src.replace(old, new))
+    binary = str(tmp_path / "oracle_bin")
+    subprocess.check_call(["gcc", "-O2", "-std=c11", "-pthread", "-w", "-o", binary, str(tmp_path / "oracle.c")])
+    monkeypatch.setattr(oracle, "BIN", binary)
+    monkeypatch.setattr(oracle, "build", lambda force=False: binary)
+    with pytest.raises((AssertionError, subprocess.CalledProcessError)):
+        _pin_battery()
