@@ -349,7 +349,7 @@ def run_ours(args):
         if world > 1:
             pkw.update(nshards=world, shard=rank)
         # at least --e2e-steps timed steps and ~2 s of them (short steps are noisy), eight warm-up steps
-        n = max(1, args.e2e_steps, min(800, int(2.0 / max(1e-5, step_s_hint))))
+        n = max(1, args.e2e_steps, min(3000, int(2.0 / max(1e-5, step_s_hint))))
         h2d = d2h = 0
         barrier()
         torch.cuda.synchronize(dev)
@@ -494,7 +494,7 @@ def run_ours(args):
     p4.close()
     del p4
     if world == 1:
-        ic_e2e, ic_e2e_s, ic_n, ic_h2d, ic_d2h, ic_e2e_kms = e2e_pipelined(cs.CUSAN_CHECK_INTERVAL_SHADOW, 0.01, 3)
+        ic_e2e, ic_e2e_s, ic_n, ic_h2d, ic_d2h, ic_e2e_kms = e2e_pipelined(cs.CUSAN_CHECK_INTERVAL_SHADOW, 0.0007, 3)
         ic_serial, ic_breakdown = e2e_serial_and_breakdown(cs.CUSAN_CHECK_INTERVAL_SHADOW, reps=5)
     else:
         ic_e2e, ic_breakdown, ic_h2d, ic_d2h = e2e_sharded(cs.CUSAN_CHECK_INTERVAL_SHADOW, 5)

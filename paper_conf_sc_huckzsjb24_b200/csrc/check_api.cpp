@@ -191,6 +191,13 @@ struct PinCache {
     std::atomic<int> device_ok{-1};   // -1 unknown, 0 no CUDA device, 1 cudaHostAlloc works
 };
 PinCache& pin_cache() { static PinCache* c = new PinCache; return *c; }
+// CUSAN_DEBUG_ALLOC=1: every page-locking allocation / release the cache could not serve, timed
+// (and, in plan_dev.cu, every device planning scratch created or grown)
+// (cudaHostAlloc pins pages, cudaFreeHost waits for the device: both stall a pipeline)
+bool debug_pinned() {
+    static const bool on = std::getenv("CUSAN_DEBUG_ALLOC") != nullptr;
+    return on;
+}
 }  // namespace
 
 void* cusan::pinned_alloc(size_t bytes) {
@@ -210,7 +217,13 @@ void* cusan::pinned_alloc(size_t bytes) {
     void* b = nullptr;
     int pinned = 0;
     if (c.device_ok != 0) {
-        if (cudaHostAlloc(&b, cls, cudaHostAllocPortable) == cudaSuccess) {
+        const auto t0 = std::chrono::steady_clock::now();
+        const cudaError_t he = cudaHostAlloc(&b, cls, cudaHostAllocPortable);
+        if (debug_pinned())
+            std::fprintf(stderr, "cusan pinned: cudaHostAlloc %zu B %.3f ms (cached %zu B)\n", cls,
+                         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count(),
+                         c.cached);
+        if (he == cudaSuccess) {
             pinned = 1;
             c.device_ok = 1;
         } else {
@@ -240,8 +253,15 @@ void cusan::pinned_free(void* p) noexcept {
             return;
         }
     }
-    if (h.pinned) cudaFreeHost(b);
-    else std::free(b);
+    if (h.pinned) {
+        const auto t0 = std::chrono::steady_clock::now();
+        cudaFreeHost(b);
+        if (debug_pinned())
+            std::fprintf(stderr, "cusan pinned: cudaFreeHost %zu B %.3f ms\n", h.cls,
+                         std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count());
+    } else {
+        std::free(b);
+    }
 }
 
 // Work-unit (warp range) sizing, granules.  The compiled defaults (kernel.cuh) can be overridden

@@ -531,6 +531,57 @@ struct ScratchPool {
 };
 ScratchPool& scratch_pool() { static ScratchPool* p = new ScratchPool; return *p; }
 
+// The planning buffers (DevScratch::a per access, ::b per incidence and span: hundreds of MB for a
+// large trace) are needed only while a plan is being built; the plan keeps its output tables in
+// ::o.  So a and b go back to this pool when the planning is done: plans waiting to run (a pipeline
+// keeps several in flight) hold only their tables, and a pipeline needs as many planning buffers
+// as plans are built at once — no cudaMalloc / cudaFree (which waits for the device) per plan.
+struct BufPool {
+    std::mutex m;
+    struct Buf { int device, kind; char* p; uint64_t cap; };
+    std::vector<Buf> free;
+};
+BufPool& buf_pool() { static BufPool* p = new BufPool; return *p; }
+
+void buf_take(int device, int kind, char** p, uint64_t* cap) {
+    if (*p) return;
+    BufPool& P = buf_pool();
+    std::lock_guard<std::mutex> lk(P.m);
+    int best = -1;
+    for (size_t i = 0; i < P.free.size(); i++)
+        if (P.free[i].device == device && P.free[i].kind == kind &&
+            (best < 0 || P.free[i].cap > P.free[(size_t)best].cap))
+            best = (int)i;
+    if (best < 0) return;
+    *p = P.free[(size_t)best].p;
+    *cap = P.free[(size_t)best].cap;
+    P.free.erase(P.free.begin() + best);
+}
+
+// (only once no work on the stream uses the buffer)
+void buf_give(int device, int kind, char** p, uint64_t* cap) {
+    if (!*p) return;
+    BufPool& P = buf_pool();
+    {
+        std::lock_guard<std::mutex> lk(P.m);
+        if (P.free.size() < 32) {
+            P.free.push_back({device, kind, *p, *cap});
+            *p = nullptr;
+            *cap = 0;
+            return;
+        }
+    }
+    cudaFree(*p);
+    *p = nullptr;
+    *cap = 0;
+}
+
+// planning is over (its stream idle): the planning buffers go back to the pool
+void planning_done(DevScratch& S) {
+    buf_give(S.device, 0, &S.a, &S.a_cap);
+    buf_give(S.device, 1, &S.b, &S.b_cap);
+}
+
 struct Carver {
     char* base;
     uint64_t off = 0;
@@ -550,6 +601,7 @@ namespace cusan {
 DevScratch::~DevScratch() {
     if (a) cudaFree(a);
     if (b) cudaFree(b);
+    if (o) cudaFree(o);
     if (hdr_host) cudaFreeHost(hdr_host);
     if (stream) cudaStreamDestroy(stream);
 }
@@ -568,6 +620,7 @@ DevScratch* plan_dev_acquire(int device) {
     }
     DevScratch* s = new (std::nothrow) DevScratch;
     if (!s) return nullptr;
+    if (std::getenv("CUSAN_DEBUG_ALLOC")) std::fprintf(stderr, "cusan plan_dev: new scratch (device %d)\n", device);
     s->device = device;
     if (cudaStreamCreateWithFlags(&s->stream, cudaStreamNonBlocking) != cudaSuccess) {
         (void)cudaGetLastError();
@@ -582,8 +635,11 @@ void plan_dev_release(DevScratch* s) {
     if (!s) return;
     ScratchPool& P = scratch_pool();
     std::lock_guard<std::mutex> lk(P.m);
-    if (P.free.size() < 8) P.free.push_back(s);
-    else delete s;
+    if (P.free.size() < 32) P.free.push_back(s);     // (a plan waiting to run holds only its tables)
+    else {
+        if (std::getenv("CUSAN_DEBUG_ALLOC")) std::fprintf(stderr, "cusan plan_dev: scratch destroyed\n");
+        delete s;
+    }
 }
 
 static int grow(char** p, uint64_t* cap, uint64_t need) {
@@ -592,6 +648,7 @@ static int grow(char** p, uint64_t* cap, uint64_t need) {
     *p = nullptr;
     *cap = 0;
     const uint64_t n = std::max<uint64_t>(need + need / 4, 1 << 20);
+    if (std::getenv("CUSAN_DEBUG_ALLOC")) std::fprintf(stderr, "cusan plan_dev: scratch grows to %llu B\n", (unsigned long long)n);
     if (cudaMalloc((void**)p, n) != cudaSuccess) {
         (void)cudaGetLastError();
         return fail(CUSAN_ENOMEM, "cannot allocate device planning scratch");
@@ -671,6 +728,7 @@ int device_plan_a2(HostPlan& hp, const DevPlanArgs& A, DevScratch& S, DevPlanOut
     };
     Carver m1{nullptr, 0, true};
     carve1(m1);
+    buf_take(S.device, 0, &S.a, &S.a_cap);
     if (int e = grow(&S.a, &S.a_cap, m1.off)) return e;
     Carver c1{S.a, 0, false};
     auto P1 = carve1(c1);
@@ -805,13 +863,15 @@ int device_plan_a2(HostPlan& hp, const DevPlanArgs& A, DevScratch& S, DevPlanOut
         p.wd = c.take<WinDesc>(nwin_all);
         return p;
     };
-    Carver m2{nullptr, 0, true};
+    Carver m2{nullptr, 0, true}, mo{nullptr, 0, true};
     carve2(m2);
-    carve_out(m2);
+    carve_out(mo);
+    buf_take(S.device, 1, &S.b, &S.b_cap);
     if (int e = grow(&S.b, &S.b_cap, m2.off)) return e;
-    Carver c2{S.b, 0, false};
+    if (int e = grow(&S.o, &S.o_cap, mo.off)) return e;
+    Carver c2{S.b, 0, false}, co{S.o, 0, false};
     auto P2 = carve2(c2);
-    auto PO = carve_out(c2);
+    auto PO = carve_out(co);
 
     k_ivs<<<nblk(n2), MT, 0, st>>>(n2, P1.hdr, P1.icov, P1.ivid, P1.B, P1.idense, P1.ilen, P1.cov, P2.iv, P2.cnt);
     tb = tmp2;
@@ -860,7 +920,10 @@ int device_plan_a2(HostPlan& hp, const DevPlanArgs& A, DevScratch& S, DevPlanOut
     out.shard_granules = hh[H_DHI] - hh[H_DLO];
     out.d_lo = hh[H_DLO];
     out.tracked_bytes_shard = hh[H_TRACKED];
-    if (!nk || !ns) return CUSAN_OK;
+    if (!nk || !ns) {
+        planning_done(S);                                      // (the stream is idle: sync 2)
+        return CUSAN_OK;
+    }
     k_span_iota<<<nblk(ns), MT, 0, st>>>(ns, P2.sidx);
     tb = tmp2;
     CK(cub::DeviceRadixSort::SortPairs(P2.tmp, tb, P2.skey, P2.skey2, P2.sidx, P2.sidx2, (int)ns, 0,
@@ -910,6 +973,7 @@ int device_plan_a2(HostPlan& hp, const DevPlanArgs& A, DevScratch& S, DevPlanOut
     out.spill_spans = hh[H_SPILL];
     out.cell_bytes = hh[H_CELLBYTES];
     out.need_shadow = hh[H_NEEDSHADOW] != 0;
+    planning_done(S);                                          // (the stream is idle: sync 3)
     return CUSAN_OK;
 }
 

@@ -23,10 +23,12 @@ struct DevPlanArgs {
 struct DevScratch {
     int device = 0;
     cudaStream_t stream = nullptr;
-    char* a = nullptr;          // per-access buffers
+    char* a = nullptr;          // per-access buffers (pooled: held only while planning)
     uint64_t a_cap = 0;
-    char* b = nullptr;          // per-incidence / per-span buffers and the output tables
+    char* b = nullptr;          // per-incidence / per-span buffers (pooled: held only while planning)
     uint64_t b_cap = 0;
+    char* o = nullptr;          // the output tables the check reads (kept with the plan)
+    uint64_t o_cap = 0;
     unsigned long long* hdr_host = nullptr;   // pinned
     std::vector<WinDesc> wins_host;
     ~DevScratch();

@@ -20,7 +20,11 @@ ap.add_argument("--config", type=int, default=5)
 ap.add_argument("--steps", type=int, default=60)
 ap.add_argument("--dense", action="store_true")
 ap.add_argument("--host-workers", type=int, default=2)
+ap.add_argument("--no-gc", action="store_true", help="Python's cyclic garbage collector off during the run")
 a = ap.parse_args()
+if a.no_gc:
+    import gc
+    gc.disable()
 w = configs.make(a.config, "full")
 ops, args = w.arrays(True)
 T = {"lower": [], "clocks": [], "plan": [], "check": []}
@@ -62,8 +66,15 @@ for i, (_t, rep) in enumerate(cs.pipelined_checks(make_trace, a.steps, window_ev
     now = time.perf_counter()
     if t_prev is not None and i >= 5:
         steps.append(1e3 * (now - t_prev))
+        if steps[-1] > 10:
+            print(f"pipeline_stages: slow step {i}: {steps[-1]:.1f} ms", file=sys.stderr, flush=True)
         T["check"].append(rep.counters["run_ms"])
     t_prev = now
 med = {k: round(statistics.median(v[5:] if len(v) > 10 else v), 3) for k, v in T.items()}
+q = sorted(steps)
+pct = {p: round(q[min(len(q) - 1, int(p / 100 * len(q)))], 3) for p in (50, 90, 99)}
+slow = sorted(((x, i) for i, x in enumerate(steps) if x > 5 * pct[50]), reverse=True)[:8]
 print(f"config {a.config} {'dense' if a.dense else 'compressed'} ({a.host_workers} host workers per stage): step "
-      f"{sum(steps) / len(steps):.3f} ms (mean over {len(steps)} steps); stage medians {med}")
+      f"{sum(steps) / len(steps):.3f} ms (mean over {len(steps)} steps; p50/p90/p99 {pct[50]}/{pct[90]}/{pct[99]}, "
+      f"max {q[-1]:.2f} ms, {sum(1 for x in steps if x > 5 * pct[50])} steps > 5 x p50, slowest (ms, step) "
+      f"{[(round(x, 1), i) for x, i in slow]}); stage medians {med}")
