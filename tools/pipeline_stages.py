@@ -28,6 +28,7 @@ if a.no_gc:
 w = configs.make(a.config, "full")
 ops, args = w.arrays(True)
 T = {"lower": [], "clocks": [], "plan": [], "check": []}
+LONG = []          # (stage, start, ms) of stage executions over 10 ms
 
 
 def make_trace(_i):
@@ -35,6 +36,8 @@ def make_trace(_i):
     t = cs.Trace(255)
     cs.Lowering(t).cusan_lower_program(ops, args)
     T["lower"].append(1e3 * (time.perf_counter() - t0))
+    if T["lower"][-1] > 10:
+        LONG.append(("lower", t0, T["lower"][-1]))
     return t
 
 
@@ -46,6 +49,8 @@ def timed_compute(cls, tr):
     t0 = time.perf_counter()
     r = orig_compute(cls, tr)
     T["clocks"].append(1e3 * (time.perf_counter() - t0))
+    if T["clocks"][-1] > 10:
+        LONG.append(("clocks", t0, T["clocks"][-1]))
     return r
 
 
@@ -54,6 +59,8 @@ class TimedPlan(orig_plan):
         t0 = time.perf_counter()
         super().__init__(*x, **k)
         T["plan"].append(1e3 * (time.perf_counter() - t0))
+        if T["plan"][-1] > 10:
+            LONG.append(("plan", t0, T["plan"][-1]))
 
 
 cs.Clocks.compute = classmethod(timed_compute)
@@ -74,6 +81,10 @@ med = {k: round(statistics.median(v[5:] if len(v) > 10 else v), 3) for k, v in T
 q = sorted(steps)
 pct = {p: round(q[min(len(q) - 1, int(p / 100 * len(q)))], 3) for p in (50, 90, 99)}
 slow = sorted(((x, i) for i, x in enumerate(steps) if x > 5 * pct[50]), reverse=True)[:8]
+t_first = LONG[0][1] if LONG else 0.0
+if LONG:
+    print("pipeline_stages: stage executions over 10 ms (stage, ms):", [(x[0], round(x[2], 1)) for x in LONG],
+          file=sys.stderr)
 print(f"config {a.config} {'dense' if a.dense else 'compressed'} ({a.host_workers} host workers per stage): step "
       f"{sum(steps) / len(steps):.3f} ms (mean over {len(steps)} steps; p50/p90/p99 {pct[50]}/{pct[90]}/{pct[99]}, "
       f"max {q[-1]:.2f} ms, {sum(1 for x in steps if x > 5 * pct[50])} steps > 5 x p50, slowest (ms, step) "
