@@ -119,18 +119,19 @@ class Lowering:
         return first
 
     def __getattr__(self, name):
-        """cusan_on_*(...) → the C call with this lowering as first argument."""
+        """cusan_on_*(...) → the C call with this lowering as first argument (bound once: later
+        lookups find it on the instance)."""
         if name.startswith("cusan_on_"):
             fn = getattr(lib, name)
-
-            def call(*a):
-                if name == "cusan_on_kernel":
-                    stream, ptrs, modes = a
-                    p = (C.c_uint64 * len(ptrs))(*ptrs)
-                    m = (C.c_uint32 * len(modes))(*modes)
-                    _ck(fn(self.h, stream, len(ptrs), p, m))
-                else:
-                    _ck(fn(self.h, *a))
+            h = self.h
+            if name == "cusan_on_kernel":
+                def call(stream, ptrs, modes):
+                    n = len(ptrs)
+                    _ck(fn(h, stream, n, (C.c_uint64 * n)(*ptrs), (C.c_uint32 * n)(*modes)))
+            else:
+                def call(*a):
+                    _ck(fn(h, *a))
+            self.__dict__[name] = call
             return call
         raise AttributeError(name)
 

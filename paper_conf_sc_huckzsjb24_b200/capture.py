@@ -45,7 +45,6 @@ from typing import Any
 
 import torch
 from torch.utils._python_dispatch import TorchDispatchMode
-from torch.utils import _pytree as pytree
 
 from . import Report, Trace, Lowering, check
 
@@ -133,6 +132,7 @@ class Capture:
         self._next_base = 1 << 44
         self.ops = 0
         self.op_names: dict[int, str] = {}           # first event id of an op -> op name
+        self._plans: dict[Any, tuple] = {}           # operator -> its schema's recording plan
         self._req = itertools.count(1)
         self._ev = itertools.count(1 << 40)          # synthetic event handles for NCCL modelling
         self._mode = None
@@ -235,54 +235,72 @@ class Capture:
         self.allocs.pop(ptr, None)
 
     # ---- operator dispatch ---------------------------------------------------------------------------
+    def _op_plan(self, func):
+        """What the operator schema says about each argument, computed once per operator: (name,
+        alloc_only, is the blocking-copy candidate, per argument (name, write, metadata only), per
+        return metadata only)."""
+        plan = self._plans.get(func)
+        if plan is None:
+            schema = func._schema
+            name = schema.name
+            # allocation only (no kernel touches the memory) / tensors passed only for their shape
+            alloc_only = name in ("aten::empty", "aten::empty_like", "aten::empty_strided", "aten::new_empty",
+                                  "aten::new_empty_strided")
+            shape_only_inputs = alloc_only or name.endswith("_like")
+            argv = tuple((a.name, a.alias_info is not None and a.alias_info.is_write,
+                          shape_only_inputs or (a.alias_info is not None and not a.alias_info.is_write))
+                         for a in schema.arguments)
+            rets = tuple(alloc_only or (r.alias_info is not None and not r.alias_info.is_write) for r in schema.returns)
+            plan = (name, name in _COPY_OPS, argv, rets)
+            self._plans[func] = plan
+        return plan
+
     @_recording
     def _on_op(self, func, args, kwargs, out):
-        schema = func._schema
-        name = schema.name
+        name, copy_op, argv, rets = self._op_plan(func)
         if self._in_p2p and name in _P2P_OPS:
             return                                    # recorded by the torch.distributed wrapper
-        # allocation only (no kernel touches the memory) / tensors passed only for their shape
-        alloc_only = name in ("aten::empty", "aten::empty_like", "aten::empty_strided", "aten::new_empty",
-                              "aten::new_empty_strided")
-        shape_only_inputs = alloc_only or name.endswith("_like")
         acc: dict[int, int] = {}                      # storage -> mode (0 R, 1 W)
         host_copy = name == "aten::_local_scalar_dense"   # .item(): blocking device->host read
+        Tensor = torch.Tensor
 
-        def add(v, write, metadata_only):
+        def add(v, write, meta):                      # a tensor, or lists / tuples of them
             nonlocal host_copy
-            if not isinstance(v, torch.Tensor):
-                return
-            if not v.is_cuda:
-                host_copy = True
-                return
-            ptr = self._storage(v)
-            if not ptr:
-                return
-            if write:
-                acc[ptr] = 1
-            elif not metadata_only:
-                acc.setdefault(ptr, 0)
+            if isinstance(v, Tensor):
+                if not v.is_cuda:
+                    host_copy = True
+                    return
+                ptr = self._storage(v)
+                if not ptr:
+                    return
+                if write:
+                    acc[ptr] = 1
+                elif not meta:
+                    acc.setdefault(ptr, 0)
+            elif isinstance(v, (list, tuple)):
+                for x in v:
+                    add(x, write, meta)
 
-        values = list(args) + [kwargs.get(a.name) for a in schema.arguments[len(args):]]
-        for a, v in zip(schema.arguments, values):
-            write = a.alias_info is not None and a.alias_info.is_write
-            meta = shape_only_inputs or (a.alias_info is not None and not a.alias_info.is_write)
-            pytree.tree_map_(lambda x: add(x, write, meta), v)
+        na = len(args)
+        for i, (aname, write, meta) in enumerate(argv):
+            v = args[i] if i < na else kwargs.get(aname)
+            if v is not None:
+                add(v, write, meta)
         outs = out if isinstance(out, (tuple, list)) else (out,)
-        for r, v in zip(schema.returns, outs):
-            meta = alloc_only or (r.alias_info is not None and not r.alias_info.is_write)
-            pytree.tree_map_(lambda x: add(x, not meta, meta), v)
+        for meta, v in zip(rets, outs):
+            add(v, not meta, meta)
         if not acc:
             return
-        stream = self._stream(torch.cuda.current_stream().cuda_stream)
+        stream = self._stream(torch._C._cuda_getCurrentRawStream(torch.cuda.current_device()))
         first = len(self.trace)
         self.low.cusan_on_kernel(stream, list(acc.keys()), list(acc.values()))
-        self.op_names[first] = schema.name
+        self.op_names[first] = name
         self.ops += 1
-        non_blocking = bool(kwargs.get("non_blocking", False)) or (
-            func in (_aten.copy_.default,) and len(args) > 2 and bool(args[2]))
-        if host_copy and not non_blocking and name in _COPY_OPS:
-            self.low.cusan_on_stream_sync(stream)     # blocking host<->device copy
+        if host_copy and copy_op:
+            non_blocking = bool(kwargs.get("non_blocking", False)) or (
+                func is _aten.copy_.default and len(args) > 2 and bool(args[2]))
+            if not non_blocking:
+                self.low.cusan_on_stream_sync(stream)     # blocking host<->device copy
 
     # ---- point-to-point communication ----------------------------------------------------------------
     @_recording
