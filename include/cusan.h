@@ -241,6 +241,18 @@ int cusan_session_check(cusan_session* s, cusan_report** out);
  * CUSAN_ESTATE while a submitted call is in flight.  *prev / *out are freed with cusan_report_free. */
 int cusan_session_submit(cusan_session* s, cusan_report** prev);
 int cusan_session_finish(cusan_session* s, cusan_report** out);
+/* Memory reclamation for long-running sessions: the caller promises that no access appended after
+ * this call touches [addr, addr + nbytes) — the memory was released and a later allocation at that
+ * address is recorded under a new range, as the live capture does (f2; PyTorch's stream sanitizer
+ * resets a block's state at deallocation for the same reason).  At the end of the next call's plan
+ * (after the accesses appended before this call are checked against the old state) the session
+ * drops the elementary intervals lying wholly inside the range from its layout, and read-set
+ * records only they named become reusable; reports are unchanged.  Without it the layout grows with
+ * every allocation a program ever touched, and so does each call's host cost.  An access that
+ * breaks the promise starts from empty state on the dropped part (its races with accesses before
+ * the forget are not reported).  Counter n_intervals = the live layout after the call.  Shadow
+ * cells are not compacted (8 B per dropped interval with the compressed shadow). */
+int cusan_session_forget(cusan_session* s, uint64_t addr, uint64_t nbytes);
 int cusan_session_destroy(cusan_session* s);
 
 /* ---- report (a5) ------------------------------------------------------------------------------ */

@@ -339,6 +339,11 @@ class Session:
         _ck(lib.cusan_session_finish(self.h, C.byref(h)))
         return _report(h, self.max_runs) if h.value else None
 
+    def forget(self, addr: int, nbytes: int) -> None:
+        """cusan_session_forget: no access appended from now on touches [addr, addr + nbytes) (the
+        memory was released); the session drops that range's intervals after the next call."""
+        _ck(lib.cusan_session_forget(self.h, addr, nbytes))
+
     def close(self, _destroy=lib.cusan_session_destroy):
         if getattr(self, "h", None):
             _destroy(self.h)

@@ -98,6 +98,7 @@ PROTOS = {
     "cusan_session_check": [P, PP],
     "cusan_session_submit": [P, PP],
     "cusan_session_finish": [P, PP],
+    "cusan_session_forget": [P, u64, u64],
     "cusan_session_destroy": [P],
     "cusan_report_get": [P, pu64, pu64, C.POINTER(C.POINTER(cusan_race_run)), pi32],
     "cusan_report_counters": [P, C.POINTER(cusan_counters)],

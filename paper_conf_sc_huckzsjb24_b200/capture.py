@@ -41,12 +41,13 @@ from __future__ import annotations
 import functools
 import itertools
 import threading
+import weakref
 from typing import Any
 
 import torch
 from torch.utils._python_dispatch import TorchDispatchMode
 
-from . import Report, Trace, Lowering, check
+from . import Report, Session, Trace, Lowering, check
 
 _aten = torch.ops.aten
 _COPY_OPS = ("aten::copy_", "aten::_to_copy", "aten::_local_scalar_dense", "aten::_copy_from",
@@ -133,6 +134,7 @@ class Capture:
         self.ops = 0
         self.op_names: dict[int, str] = {}           # first event id of an op -> op name
         self._plans: dict[Any, tuple] = {}           # operator -> its schema's recording plan
+        self._sessions: list = []                    # weak references to sessions from session()
         self._req = itertools.count(1)
         self._ev = itertools.count(1 << 40)          # synthetic event handles for NCCL modelling
         self._mode = None
@@ -168,6 +170,16 @@ class Capture:
     def check(self, **kw) -> Report:
         """Run the race check on the captured trace (kw: cusan_check options)."""
         return check(self.trace, **kw)
+
+    def session(self, **kw) -> Session:
+        """An online check of the captured trace (f1): `session().check()` checks what the program
+        did since the previous call.  Allocation instances the caching allocator releases are
+        forgotten by the session (cusan_session_forget: their ranges are never touched again — the
+        next tensor at that address gets a new range), so its layout and per-call cost stay
+        bounded however long the program runs.  kw: Session options."""
+        ses = Session(self.trace, **kw)
+        self._sessions.append(weakref.ref(ses))
+        return ses
 
     # ---- helpers ----------------------------------------------------------------------------------
     def _stream(self, handle: int) -> int:
@@ -232,7 +244,15 @@ class Capture:
     def _on_memory_deallocation(self, ptr: int):
         # the block goes back to the caching allocator (no cudaFree, no device sync): forget this
         # instance, so the next tensor at the same address gets a fresh range
-        self.allocs.pop(ptr, None)
+        inst = self.allocs.pop(ptr, None)
+        if inst is not None and self._sessions:
+            live = []
+            for ref in self._sessions:
+                ses = ref()
+                if ses is not None and getattr(ses, "h", None):
+                    ses.forget(inst[0], inst[1])
+                    live.append(ref)
+            self._sessions = live
 
     # ---- operator dispatch ---------------------------------------------------------------------------
     def _op_plan(self, func):

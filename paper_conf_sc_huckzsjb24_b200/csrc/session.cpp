@@ -251,6 +251,7 @@ struct cusan_session {
     uint32_t F_used = 1;                            // fibers seen so far: clock columns >= it are all 0
     uint64_t nseg = 0;
     std::vector<SIv> ivs;                           // layout of `shadow`
+    std::vector<std::pair<uint64_t, uint64_t>> forget;   // granule ranges to drop after the next plan
     uint64_t used = 0;                              // cells of `shadow` in use
     uint64_t checked_access = 0, checked_events = 0, n_calls = 0;
     // epoch renumbering (sessions longer than the 24-bit epoch field, see session_renumber):
@@ -625,6 +626,22 @@ static int plan_call(cusan_session* s, const Trace& tr, CallPlan& cp) {
     c.spill_spans = hp.spill_spans;
     c.spill_heap_bytes = hp.rec_units * REC_WORDS * 4;
     tick("spans");
+    if (!s->forget.empty()) {          // cusan_session_forget: released memory leaves the layout
+        std::vector<std::pair<uint64_t, uint64_t>>& fg = s->forget;
+        std::sort(fg.begin(), fg.end());
+        size_t keep = 0, r = 0;
+        uint64_t reach = 0;            // furthest end of the ranges starting at or before the interval
+        for (size_t i = 0; i < cp.ivs.size(); i++) {
+            const SIv& v = cp.ivs[i];
+            while (r < fg.size() && fg[r].first <= v.abs_begin) reach = std::max(reach, fg[r++].second);
+            if (reach >= v.abs_begin + v.len) continue;          // wholly inside a released range
+            if (keep != i) cp.ivs[keep] = cp.ivs[i];
+            keep++;
+        }
+        cp.ivs.resize(keep);
+        fg.clear();
+        c.n_intervals = keep;
+    }
     s->recs.collect(cp.ivs);           // records no interval of the new layout names are dead
     tick("collect");
     c.heap_live_bytes = s->recs.live_units * REC_WORDS * 4;
@@ -1036,6 +1053,19 @@ int cusan_session_check(cusan_session* s, cusan_report** out) {
     int st = cusan_session_submit(s, &none);
     if (st) return st;
     return cusan_session_finish(s, out);
+}
+
+int cusan_session_forget(cusan_session* s, uint64_t addr, uint64_t nbytes) {
+    if (!s) return fail(CUSAN_EINVAL, "session is null");
+    if (addr + nbytes < addr) return fail(CUSAN_ERANGE, "addr + nbytes overflows");
+    if (!nbytes) return CUSAN_OK;
+    try {
+        const uint64_t g0 = (addr + 7) >> 3, g1 = (addr + nbytes) >> 3;   // granules wholly inside
+        if (g1 > g0) s->forget.push_back({g0, g1});
+    } catch (const std::bad_alloc&) {
+        return fail(CUSAN_ENOMEM, "host memory exhausted in cusan_session_forget");
+    }
+    return CUSAN_OK;
 }
 
 int cusan_session_destroy(cusan_session* s) {

@@ -243,3 +243,40 @@ def test_reused_block_race_is_still_reported_within_an_instance():
     g0 = int(rep.runs["g_begin"][0])
     assert cap.real_address(8 * g0) == x.untyped_storage().data_ptr()
     del y
+
+
+@pytest.mark.parametrize("racy", [False, True], ids=["clean", "racy"])
+def test_capture_online_session_forgets_released_temporaries(racy):
+    """Capture.session(): checked every iteration while the program runs, the calls' reports add up
+    to the post-mortem check of the same trace (which equals the oracle's), and the session forgets
+    each temporary the caching allocator releases, so its layout stays at the live tensors."""
+    torch.cuda.synchronize()
+    comp, halo = torch.cuda.Stream(), torch.cuda.Stream()
+    n = 256
+    with Capture() as cap:
+        a = torch.rand(n, n, device="cuda")
+        b = torch.zeros(n, n, device="cuda")
+        send = torch.zeros(n, device="cuda")
+        torch.cuda.synchronize()                     # (the side streams do not wait for stream 0)
+        ses = cap.session()
+        total, ivs = 0, []
+        for it in range(40):
+            with torch.cuda.stream(halo):
+                if not racy:
+                    halo.wait_stream(comp)
+                send.copy_(a[1, :] * 1.0)            # a temporary per iteration
+            with torch.cuda.stream(comp):
+                b[1:-1, 1:-1] = 0.25 * (a[:-2, 1:-1] + a[2:, 1:-1] + a[1:-1, :-2] + a[1:-1, 2:])
+                comp.wait_stream(halo)
+                b[0, :].copy_(send)
+            a, b = b, a
+            rep = ses.check()
+            total += rep.n_race_granules
+            ivs.append(rep.counters["n_intervals"])
+        torch.cuda.synchronize()
+        ses.close()
+    post = _parity(cap)
+    assert total == post.n_race_granules
+    assert (post.n_race_granules > 0) == racy
+    assert len(cap.real) > 100                       # allocation instances the program went through
+    assert ivs[-1] < len(cap.real) // 4, ivs         # the layout holds about the live ones

@@ -424,3 +424,69 @@ def test_session_beyond_2_24_events():
     assert rep.counters["renumberings"] >= 1
     assert total == ref["n_race_granules"]
     ses.close()
+
+
+def _instances_trace(rng, n, nf, n_keys=3):
+    """Events over short-lived allocation instances (disjoint 64-granule ranges, a sliding set of
+    three live ones), as the live capture records a program's temporaries; returns the events and
+    each instance's (range, last access position)."""
+    from tracegen.program import EVENT_DTYPE, EV_ACQUIRE, EV_FORK, EV_RELEASE
+    base = 1 << 36
+    ev = np.zeros(n, EVENT_DTYPE)
+    last = {}
+    for i in range(n):
+        f = int(rng.integers(nf))
+        if rng.random() < 0.6:
+            inst = i // 12 + int(rng.integers(3))
+            g0 = int(rng.integers(64))
+            g1 = int(rng.integers(g0 + 1, 65))
+            ev[i] = (EV_ACCESS, int(rng.random() < 0.45), 0, f, base + 512 * inst + 8 * g0, 8 * (g1 - g0))
+            last[inst] = i
+        else:
+            u = rng.random()
+            if u < 0.4:
+                ev[i] = (EV_RELEASE, 0, 0, f, 1000 + int(rng.integers(n_keys)), 0)
+            elif u < 0.8:
+                ev[i] = (EV_ACQUIRE, 0, 0, f, 1000 + int(rng.integers(n_keys)), 0)
+            else:
+                src = (f + 1 + int(rng.integers(nf - 1))) % nf
+                ev[i] = (EV_FORK, 0, 0, f, src, 0)
+    return ev, {k: ((base + 512 * k, 512), p) for k, p in last.items()}
+
+
+@pytest.mark.parametrize("flags", [0, cs.CUSAN_CHECK_DENSE_SHADOW], ids=["compressed", "dense"])
+def test_session_forget_released_ranges(flags):
+    """cusan_session_forget of ranges no later access touches leaves every call's report equal to
+    the oracle's, and keeps the layout to the live ranges (it grows without)."""
+    rng = np.random.default_rng(4242)
+    for _ in range(12):
+        nf = int(rng.integers(2, 7))
+        n = int(rng.integers(200, 600))
+        ev, inst = _instances_trace(rng, n, nf)
+        ref = oracle.check_events(ev, nf, threads=2)
+        cuts = sorted(set(int(x) for x in rng.integers(1, n, size=12))) + [n]
+        tr, tr2 = cs.Trace(nf), cs.Trace(nf)
+        ses, ses2 = cs.Session(tr, flags=flags), cs.Session(tr2, flags=flags)
+        start, forgotten = 0, set()
+        ivs, ivs2 = [], []
+        for end in cuts:
+            if end <= start:
+                continue
+            for t in (tr, tr2):
+                t.cusan_trace_append_events(ev[start:end])
+            rep, rep2 = ses.check(), ses2.check()
+            want = _by_later(ref["runs"], start, end)
+            for r in (rep, rep2):
+                assert np.array_equal(r.runs, want.astype(r.runs.dtype)), (start, end)
+                assert r.n_race_granules == int(np.sum(want["g_end"] - want["g_begin"]))
+            ivs.append(rep.counters["n_intervals"])
+            ivs2.append(rep2.counters["n_intervals"])
+            # instances whose last access is already appended are released: never touched again
+            for k, ((addr, size), p) in inst.items():
+                if p < end and k not in forgotten:
+                    ses.forget(addr, size)
+                    forgotten.add(k)
+            start = end
+        ses.close()
+        ses2.close()
+        assert ivs[-1] < ivs2[-1], (ivs, ivs2)

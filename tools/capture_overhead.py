@@ -93,7 +93,7 @@ def run(mode: str):
     ses = None
     if cap is not None:
         cap.__enter__()
-        ses = cs.Session(cap.trace) if mode == "online" else None
+        ses = cap.session() if mode == "online" else None   # forgets released temporaries
     n_race = [0]
 
     def iterate(k, start):
