@@ -180,7 +180,8 @@ int cusan_plan_destroy(cusan_plan* p);
  * host-built ones (CUSAN_CHECK_HOST_PLAN).  Waits for the plan's stream. */
 int cusan_plan_tables(const cusan_plan* p, void* inc, uint64_t inc_cap, void* spans, uint64_t spans_cap,
                       uint64_t* n_inc, uint64_t* n_spans);
-/* Frees the parked workspaces (all devices).  Set CUSAN_NO_WORKSPACE_CACHE=1 to never park. */
+/* Frees the parked check workspaces and the pooled device-planning scratch (all devices).  Set
+ * CUSAN_NO_WORKSPACE_CACHE=1 to never park a check workspace. */
 int cusan_release_cached_memory(void);
 /* ---- a1's products as a transferable object ("event clocks broadcast") ----------
  * cusan_clocks_compute runs a1 over the whole trace (on all of the node's cores): per access its

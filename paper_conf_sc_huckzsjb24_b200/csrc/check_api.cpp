@@ -912,6 +912,7 @@ int cusan_release_cached_memory(void) {
             c.bytes[d] = 0;
         }
     cudaSetDevice(cur);
+    plan_dev_release_all();
     return CUSAN_OK;
 }
 

@@ -642,6 +642,33 @@ void plan_dev_release(DevScratch* s) {
     }
 }
 
+// cusan_release_cached_memory: the pooled planning scratches and buffers (all devices)
+void plan_dev_release_all() {
+    std::vector<DevScratch*> scr;
+    {
+        ScratchPool& P = scratch_pool();
+        std::lock_guard<std::mutex> lk(P.m);
+        scr.swap(P.free);
+    }
+    int cur = 0;
+    cudaGetDevice(&cur);
+    for (DevScratch* s : scr) {
+        cudaSetDevice(s->device);
+        delete s;
+    }
+    std::vector<BufPool::Buf> bufs;
+    {
+        BufPool& P = buf_pool();
+        std::lock_guard<std::mutex> lk(P.m);
+        bufs.swap(P.free);
+    }
+    for (const BufPool::Buf& b : bufs) {
+        cudaSetDevice(b.device);
+        cudaFree(b.p);
+    }
+    cudaSetDevice(cur);
+}
+
 static int grow(char** p, uint64_t* cap, uint64_t need) {
     if (*cap >= need && *p) return CUSAN_OK;
     if (*p) cudaFree(*p);

@@ -52,5 +52,6 @@ int device_plan_a2(HostPlan& hp, const DevPlanArgs& args, DevScratch& S, DevPlan
 
 DevScratch* plan_dev_acquire(int device);      // nullptr: no memory / stream
 void plan_dev_release(DevScratch* s);          // the caller's work on it is complete
+void plan_dev_release_all();                   // frees every pooled scratch and planning buffer
 
 }  // namespace cusan
