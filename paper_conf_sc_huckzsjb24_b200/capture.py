@@ -100,8 +100,8 @@ class _Dispatch(TorchDispatchMode):
     def __torch_dispatch__(self, func, types, args=(), kwargs=None):
         kwargs = kwargs or {}
         out = func(*args, **kwargs)
-        if func is not _aten.record_stream.default and _ACTIVE is self.cap:   # (threads may outlive it)
-            self.cap._on_op(func, args, kwargs, out)
+        if func not in self.cap._silent and func is not _aten.record_stream.default and _ACTIVE is self.cap:
+            self.cap._on_op(func, args, kwargs, out)          # (threads may outlive the capture)
         return out
 
 
@@ -134,6 +134,7 @@ class Capture:
         self.ops = 0
         self.op_names: dict[int, str] = {}           # first event id of an op -> op name
         self._plans: dict[Any, tuple] = {}           # operator -> its schema's recording plan
+        self._silent: set = set()                    # operators that never touch tensor memory (views)
         self._sessions: list = []                    # weak references to sessions from session()
         self._req = itertools.count(1)
         self._ev = itertools.count(1 << 40)          # synthetic event handles for NCCL modelling
@@ -273,6 +274,9 @@ class Capture:
             rets = tuple(alloc_only or (r.alias_info is not None and not r.alias_info.is_write) for r in schema.returns)
             plan = (name, name in _COPY_OPS, argv, rets)
             self._plans[func] = plan
+            if all(meta and not write for _, write, meta in argv) and all(rets) and name not in _P2P_OPS \
+                    and name != "aten::_local_scalar_dense":
+                self._silent.add(func)                # views: no tensor is read or written
         return plan
 
     @_recording
