@@ -192,6 +192,10 @@ class ShardedSession:
         rep = self.session.finish()
         return self._gather(rep) if rep is not None else None
 
+    def forget(self, addr: int, nbytes: int) -> None:
+        """cusan_session_forget on this rank's shard (call it on every rank, like check())."""
+        self.session.forget(addr, nbytes)
+
     def close(self):
         self.session.close()
 

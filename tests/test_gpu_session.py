@@ -490,3 +490,17 @@ def test_session_forget_released_ranges(flags):
         ses.close()
         ses2.close()
         assert ivs[-1] < ivs2[-1], (ivs, ivs2)
+
+
+def test_c_example_online_jacobi():
+    """examples/online_jacobi.c: a session through the C ABI checks a two-stream Jacobi after every
+    iteration and forgets each released temporary; the calls add up to one cusan_check of the whole
+    trace, the racy variant (no halo-stream wait) races and the clean one does not, and the layout
+    stays bounded."""
+    import subprocess
+    import __graft_entry__ as g
+    exe = [e for e in g.build_examples() if e.endswith("online_jacobi")][0]
+    for racy in (False, True):
+        r = subprocess.run([exe] + (["--racy"] if racy else []), capture_output=True, text=True, timeout=300)
+        assert r.returncode == 0, (r.stdout, r.stderr)
+        assert ("racy:" if racy else "clean:") in r.stdout
