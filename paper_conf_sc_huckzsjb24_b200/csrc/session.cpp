@@ -42,6 +42,7 @@ using namespace cusan;
 namespace {
 
 constexpr uint32_t NO_SEG = 0xffffffffu;
+constexpr uint64_t STAGE_MAX = 256 << 10;            // calls with more table bytes upload them directly
 
 // ---- growable shadow in a reserved virtual range (CUDA virtual memory management) --------------
 // The session reserves a virtual range as large as the device's memory once and maps physical
@@ -252,6 +253,7 @@ struct cusan_session {
     uint64_t nseg = 0;
     std::vector<SIv> ivs;                           // layout of `shadow`
     std::vector<std::pair<uint64_t, uint64_t>> forget;   // granule ranges to drop after the next plan
+    pinned_vector<char> stage;                      // a small call's tables, staged for one upload
     uint64_t used = 0;                              // cells of `shadow` in use
     uint64_t checked_access = 0, checked_events = 0, n_calls = 0;
     // epoch renumbering (sessions longer than the 24-bit epoch field, see session_renumber):
@@ -658,7 +660,7 @@ struct PendingCall {
     uint64_t seg_first_word = 0;                    // where they go in segvc_d
     uint64_t used_before = 0;                       // shadow cells in use before the call
     pinned_vector<unsigned long long> init, cnt;    // counter initial values / read-back
-    pinned_vector<char> stage;                      // the call's tables as uploaded (one copy)
+    pinned_vector<CopySeg> segs_pinned;             // cell copies, page-locked (large calls)
     uint64_t h2d = 0;
     uint64_t delta = 0;                             // event numbering the call was planned with
     std::shared_ptr<const std::vector<uint32_t>> orig;
@@ -742,20 +744,32 @@ static int session_launch(cusan_session* s, PendingCall& pc) {
     DSpan* d_spans = (DSpan*)(s->scratch.p + o_spans);
     CopySeg* d_copy = (CopySeg*)(s->scratch.p + o_copy);
     unsigned long long* d_cnt = (unsigned long long*)(s->scratch.p + o_cnt);
-    // the call's tables and the counters' initial values go up in ONE transfer: staged in a
-    // page-locked buffer laid out as the scratch is (a small call's latency is mostly per-copy cost)
     pc.init.assign(N_COUNTERS + nwin, 0ull);
     pc.cnt.assign(N_COUNTERS, 0ull);
     pc.init[C_HEAP] = s->heap_cap();     // records are host-assigned: no device allocation
-    pc.stage.resize(off);
-    auto put = [&](uint64_t at, const void* src, size_t bytes) {
-        if (bytes) std::memcpy(pc.stage.data() + at, src, bytes);
-    };
-    put(o_inc, cp.inc.data(), cp.inc.size() * sizeof(AccRec));
-    put(o_spans, tabs.ds.data(), tabs.ds.size() * sizeof(DSpan));
-    put(o_copy, cp.segs.data(), cp.segs.size() * sizeof(CopySeg));
-    put(o_cnt, pc.init.data(), pc.init.size() * sizeof(unsigned long long));
-    CK(cudaMemcpyAsync(s->scratch.p, pc.stage.data(), off, cudaMemcpyHostToDevice, s->stream));
+    if (off <= STAGE_MAX) {
+        // a small call's tables and the counters' initial values go up in ONE transfer, staged in
+        // the session's page-locked buffer laid out as the scratch is (its latency is mostly
+        // per-copy cost).  The buffer is free again: the previous call finished before this launch.
+        if (s->stage.size() < off) s->stage.resize(STAGE_MAX);
+        auto put = [&](uint64_t at, const void* src, size_t bytes) {
+            if (bytes) std::memcpy(s->stage.data() + at, src, bytes);
+        };
+        put(o_inc, cp.inc.data(), cp.inc.size() * sizeof(AccRec));
+        put(o_spans, tabs.ds.data(), tabs.ds.size() * sizeof(DSpan));
+        put(o_copy, cp.segs.data(), cp.segs.size() * sizeof(CopySeg));
+        put(o_cnt, pc.init.data(), pc.init.size() * sizeof(unsigned long long));
+        CK(cudaMemcpyAsync(s->scratch.p, s->stage.data(), off, cudaMemcpyHostToDevice, s->stream));
+    } else {                             // large tables: straight from their page-locked vectors
+        pc.segs_pinned.assign(cp.segs.begin(), cp.segs.end());
+        CK(cudaMemcpyAsync(d_inc, cp.inc.data(), cp.inc.size() * sizeof(AccRec), cudaMemcpyHostToDevice, s->stream));
+        CK(cudaMemcpyAsync(d_spans, tabs.ds.data(), tabs.ds.size() * sizeof(DSpan), cudaMemcpyHostToDevice,
+                           s->stream));
+        CK(cudaMemcpyAsync(d_copy, pc.segs_pinned.data(), pc.segs_pinned.size() * sizeof(CopySeg),
+                           cudaMemcpyHostToDevice, s->stream));
+        CK(cudaMemcpyAsync(d_cnt, pc.init.data(), pc.init.size() * sizeof(unsigned long long), cudaMemcpyHostToDevice,
+                           s->stream));
+    }
     pc.h2d = cp.inc.size() * sizeof(AccRec) + tabs.ds.size() * sizeof(DSpan) + cp.segs.size() * sizeof(CopySeg) +
              pc.seg_rows.size() * sizeof(uint32_t);
     session_tick(pc, "memory");
