@@ -265,6 +265,13 @@ def run_ours(args):
     stream = torch.cuda.current_stream(dev)
 
     w, ops, args_, wname = workload(args)
+    # The interpreter's objects so far (torch and its imports: ~10^6) move to the permanent
+    # generation, so Python's cyclic collector does not rescan them during the timed steps (a full
+    # collection of them is a ~35 ms pause every ~0.5 s of a pipelined run, all host stages held).
+    # Objects created from here on are collected as usual.
+    import gc
+    gc.collect()
+    gc.freeze()
     tr = vc = None
     if world == 1 or rank == 0:
         tr = cs.Trace(255)

@@ -391,7 +391,10 @@ def pipelined_checks(make_trace, steps: int, device: int = 0, host_workers: int 
     run downloads its report, so each step still pays its own transfers.  All plans share one
     workspace from PyTorch's caching allocator (a plan's shadow and records are scratch for its own
     run).  Yields (trace, report) per step; kw as for Plan (window_events, nshards, shard, stream,
-    flags, ...)."""
+    flags, ...).  Steps take well under a millisecond, so a full pass of Python's cyclic garbage
+    collector over a large process (tens of ms with torch imported) shows up as a stall of every
+    stage; a caller that wants flat latency can `gc.freeze()` its long-lived objects first (bench.py
+    does)."""
     from concurrent.futures import ThreadPoolExecutor
 
     kw = dict(kw)
