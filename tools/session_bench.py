@@ -47,6 +47,11 @@ acc_pos = np.flatnonzero(ev["kind"] == 0)
 cuts = [int(acc_pos[i]) for i in range(a.chunk, len(acc_pos), a.chunk)] + [len(ev)]
 if a.max_calls:
     cuts = cuts[:a.max_calls]
+# import-time objects out of the cyclic collector's way (a full pass is a ~35 ms pause with torch
+# imported: it would dominate runs of a few hundred sub-millisecond calls)
+import gc  # noqa: E402
+gc.collect()
+gc.freeze()
 
 if a.pipelined:
     tr = cs.Trace(255)

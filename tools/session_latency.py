@@ -40,6 +40,11 @@ ev = full.cusan_trace_read()
 acc_pos = np.flatnonzero(ev["kind"] == 0)
 cuts = [int(acc_pos[i]) for i in range(a.chunk, len(acc_pos), a.chunk)] + [len(ev)]
 cuts = cuts[: a.calls]
+# import-time objects out of the cyclic collector's way (a full pass is a ~35 ms pause with torch
+# imported: it would dominate runs of a few hundred sub-millisecond calls)
+import gc  # noqa: E402
+gc.collect()
+gc.freeze()
 
 tr = cs.Trace(255)
 ses = cs.Session(tr, flags=cs.CUSAN_CHECK_DENSE_SHADOW if a.dense else 0)
