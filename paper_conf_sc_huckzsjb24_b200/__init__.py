@@ -123,14 +123,13 @@ class Lowering:
         lookups find it on the instance)."""
         if name.startswith("cusan_on_"):
             fn = getattr(lib, name)
-            h = self.h
             if name == "cusan_on_kernel":
                 def call(stream, ptrs, modes):
                     n = len(ptrs)
-                    _ck(fn(h, stream, n, (C.c_uint64 * n)(*ptrs), (C.c_uint32 * n)(*modes)))
+                    _ck(fn(self.h, stream, n, (C.c_uint64 * n)(*ptrs), (C.c_uint32 * n)(*modes)))
             else:
                 def call(*a):
-                    _ck(fn(h, *a))
+                    _ck(fn(self.h, *a))           # (self.h read per call: None once destroyed)
             self.__dict__[name] = call
             return call
         raise AttributeError(name)
