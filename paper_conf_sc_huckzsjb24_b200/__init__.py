@@ -122,14 +122,16 @@ class Lowering:
         """cusan_on_*(...) → the C call with this lowering as first argument (bound once: later
         lookups find it on the instance)."""
         if name.startswith("cusan_on_"):
+            import weakref
             fn = getattr(lib, name)
+            me = weakref.ref(self)                # (no reference cycle through the cached call)
             if name == "cusan_on_kernel":
                 def call(stream, ptrs, modes):
                     n = len(ptrs)
-                    _ck(fn(self.h, stream, n, (C.c_uint64 * n)(*ptrs), (C.c_uint32 * n)(*modes)))
+                    _ck(fn(me().h, stream, n, (C.c_uint64 * n)(*ptrs), (C.c_uint32 * n)(*modes)))
             else:
                 def call(*a):
-                    _ck(fn(self.h, *a))           # (self.h read per call: None once destroyed)
+                    _ck(fn(me().h, *a))           # (the handle read per call: None once destroyed)
             self.__dict__[name] = call
             return call
         raise AttributeError(name)
