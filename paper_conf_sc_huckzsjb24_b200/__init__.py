@@ -81,6 +81,9 @@ class Trace:
         return self.cusan_trace_size()[0]
 
 
+_LOWERING_FNS: dict = {}                     # cusan_on_* name -> its ctypes function
+
+
 class Lowering:
     """cusan_lowering: CUDA / MPI call -> primitive lowering (CuSan's per-device context)."""
 
@@ -119,20 +122,18 @@ class Lowering:
         return first
 
     def __getattr__(self, name):
-        """cusan_on_*(...) → the C call with this lowering as first argument (bound once: later
-        lookups find it on the instance)."""
+        """cusan_on_*(...) → the C call with this lowering as first argument."""
         if name.startswith("cusan_on_"):
-            import weakref
-            fn = getattr(lib, name)
-            me = weakref.ref(self)                # (no reference cycle through the cached call)
+            fn = _LOWERING_FNS.get(name)
+            if fn is None:
+                fn = _LOWERING_FNS[name] = getattr(lib, name)
             if name == "cusan_on_kernel":
                 def call(stream, ptrs, modes):
                     n = len(ptrs)
-                    _ck(fn(me().h, stream, n, (C.c_uint64 * n)(*ptrs), (C.c_uint32 * n)(*modes)))
+                    _ck(fn(self.h, stream, n, (C.c_uint64 * n)(*ptrs), (C.c_uint32 * n)(*modes)))
             else:
                 def call(*a):
-                    _ck(fn(me().h, *a))           # (the handle read per call: None once destroyed)
-            self.__dict__[name] = call
+                    _ck(fn(self.h, *a))
             return call
         raise AttributeError(name)
 
