@@ -6,7 +6,7 @@ checked through every mode — one window and small windows, both shadow layouts
 the default, and dense), host and device planning, plans from (exported / imported) clocks,
 whole-node checks (ngpus, shards mapped onto this GPU), granule-range shards (one-shot),
 sequential, pipelined and block-cyclic shard sessions, sessions renumbering their event ids every
-few calls — and compared with the oracle bit for bit.
+few calls, sessions forgetting the memory no later access touches — and compared with the oracle bit for bit.
 
     python tools/fuzz_campaign.py --minutes 20 --seed 1 > profiles/fuzz_campaign_r02.json
 """
@@ -81,7 +81,15 @@ def one_case(ev, nf, case):
     record("oneshot shards", same(m.runs, m.n_race_granules, ref), case)
     # sessions: random cut points, sequential / pipelined / block-cyclic shards
     cuts = sorted({0, len(ev), *rng.integers(1, max(2, len(ev)), int(rng.integers(1, 5))).tolist()})
-    for mode in ("session", "pipelined", "session shards", "session renumbering"):
+    # granules no access after position y touches: what "session forget" may release after a call
+    acc_i = np.flatnonzero(ev["kind"] == 0)
+    g0s = (ev["a"][acc_i] >> 3).astype(np.int64)
+    g1s = np.where(ev["b"][acc_i] > 0, (ev["a"][acc_i] + ev["b"][acc_i] + 7) >> 3, ev["a"][acc_i] >> 3).astype(np.int64)
+    gbase = int(g0s.min()) if len(acc_i) else 0
+    last = np.full(int(g1s.max()) - gbase if len(acc_i) else 0, -1, np.int64)
+    for i, a0, a1 in zip(acc_i, g0s, g1s):
+        last[a0 - gbase:a1 - gbase] = i
+    for mode in ("session", "pipelined", "session shards", "session renumbering", "session forget"):
         flags = int(rng.choice([0, FL, IV]))
         nsh = int(rng.integers(2, 5)) if mode == "session shards" else 1
         blk = int(2 ** rng.integers(3, 9))
@@ -101,6 +109,13 @@ def one_case(ev, nf, case):
                     if r is not None:
                         runs.append(r.runs)
                         n += r.n_race_granules
+                    if mode == "session forget":      # released: granules no later access touches
+                        dead = (last >= 0) & (last < y)
+                        if x > 0:
+                            dead &= last >= x          # (earlier ones were forgotten already)
+                        edges = np.flatnonzero(np.diff(np.concatenate([[0], dead.astype(np.int8), [0]])))
+                        for b, e in zip(edges[::2], edges[1::2]):
+                            se.forget(8 * (gbase + int(b)), 8 * int(e - b))
         except cs.CusanError as e:                 # a call or the live ids too large for the lowered limit
             if mode != "session renumbering" or e.status != -2:
                 raise
