@@ -385,6 +385,39 @@ _LOWER_MUTANTS = {
     "free_keeps_allocation": ("if a in self.alloc:", "if False:"),
     # cudaFree without its device-wide sync (A8)
     "free_no_sync": ("self.sync_device_host()                      # PAPER.md:448-450", "pass  #"),
+    # cudaStreamSynchronize(S0) not covering the blocking streams (A5)
+    "s0_sync_skips_blocking": ("""        self.acquire(self.H, K_stream(f))
+        if f == S0:
+            for u in self.blocking_user:
+                self.acquire(self.H, K_stream(u))""", """        self.acquire(self.H, K_stream(f))"""),
+    # an operation on S0 not waiting for the blocking streams (Fig. 3, PAPER.md:356-364, A5)
+    "s0_op_skips_blocking": ("""        if f == S0:
+            for u in self.blocking_user:
+                self.acquire(S0, K_stream(u))""", ""),
+    # an operation on a blocking stream not waiting for S0 (Fig. 3, PAPER.md:356-364, A5)
+    "blocking_op_skips_s0": ("""        if f in self.blocking_user:
+            self.acquire(f, K_stream(S0))""", ""),
+    # cudaDeviceSynchronize covering only the default stream (PAPER.md:405-407)
+    "device_sync_only_s0": ("        for f in self.all_streams:\n            self.acquire(self.H, K_stream(f))",
+                            "        for f in [S0]:\n            self.acquire(self.H, K_stream(f))"),
+    # a kernel without its release on the stream (AnnotateHappensBefore, PAPER.md:653-654)
+    "kernel_no_release": ("""                self.access(f, mode, al[0], al[1])         # whole allocation (PAPER.md:652-654)
+            self.epilogue(f)""", """                self.access(f, mode, al[0], al[1])         # whole allocation (PAPER.md:652-654)"""),
+    # a read-write kernel argument annotated as a read (A10)
+    "rw_arg_as_read": ("mode = READ if int(args[j][\"mode\"]) == MODE_R else WRITE",
+                       "mode = WRITE if int(args[j][\"mode\"]) == 1 else READ"),
+    # cudaMemcpy's destination annotated as read
+    "memcpy_dst_read": ("                self.access(f, WRITE, a, c)\n            if self.tracked_range(b, c):",
+                        "                self.access(f, READ, a, c)\n            if self.tracked_range(b, c):"),
+    # MPI_Isend's buffer annotated as written (MPI_Isend reads it)
+    "isend_writes": ("READ if kind == OP_MPI_ISEND else WRITE", "WRITE"),
+    # a non-blocking MPI call without its issue edge from the host (A3)
+    "mpi_no_issue_edge": ("self.fork(self.H, m)                            # PAPER.md:211-218,615-619", "pass"),
+    # a joined thread's work not ordered before the join's return
+    "join_no_acquire": ("self.acquire(self.H, K_thread(a))                  # ... HB the join's return", "pass"),
+    # the per-thread default stream treated as non-blocking
+    "ptds_nonblocking": ("            self.all_streams.append(f)\n            self.blocking_user.append(f)\n        return self.ptds[t]",
+                         "            self.all_streams.append(f)\n        return self.ptds[t]"),
 }
 
 
